@@ -1,0 +1,358 @@
+"""Counter-based, seeded generator of XML-shaped sparse datasets.
+
+Recipe:
+
+* RNG: splitmix64 finaliser chained over integer keys (seed, stream, idx...),
+  so every draw is a pure function of its indices -- rows are independent of
+  chunking, thread count and machine.  Uniforms take the top 53 bits.
+  Streams: 0 nnz counts, 1 feature ids, 2 values, 3 label counts, 4 label ids,
+  5 label signatures, 6 per-pass permutations, 7 init weights, 8 block nnz
+  multipliers, 9 label-rank scramble, 10 feature-rank scramble.
+* nnz per row: lognormal with mean s_bar (sigma per config), rounded
+  half-to-even, clipped to [1, F].  Wiki10-shaped rows come in blocks of 64
+  sharing a lognormal(sigma_b = 1, mean 1) multiplier ("heavy nnz skew across
+  batches").
+* labels per row: 1 + Poisson(y_bar - 1) by inversion; label ids Zipf(1) over
+  L ranks, ranks scrambled by a fixed permutation; distinct, sorted.
+* features: a planted structure so P@1 is learnable -- every label owns a
+  fixed 16-feature signature (uniform over F); a row's candidate stream is
+  floor(s/2) draws from its labels' signatures followed by Zipf(1) noise
+  draws (scrambled ranks); the row keeps the first s distinct ids (fewer if
+  the candidate stream runs out), sorted ascending.
+* values: U(0.5, 1.5), then L2-normalised per row (fp64), stored fp32.
+* per-pass permutation: stable argsort of per-(pass, row) random keys.
+* init (reading Q5): W1 ~ N(0, 1/H), W2 ~ N(0, 1/L),
+  biases 0, fp32.
+
+Nothing here implements the method; the oracle and the CUDA path both take
+these arrays as given.
+"""
+from __future__ import annotations
+
+import dataclasses
+import math
+from typing import Dict, Optional
+
+import numpy as np
+
+# ----------------------------------------------------------------------------
+# configurations (BASELINE.json configs)
+# ----------------------------------------------------------------------------
+
+
+@dataclasses.dataclass(frozen=True)
+class XmlConfig:
+    name: str
+    index: int              # position in BASELINE.json "configs"
+    F: int                  # features
+    L: int                  # labels
+    H: int                  # hidden width
+    n_train: int
+    n_test: int
+    s_bar: float            # mean nnz per row
+    s_sigma: float          # lognormal sigma of nnz per row
+    y_bar: float            # mean labels per row
+    b_max: int
+    block_skew: bool = False  # Wiki10: blocks of 64 rows share a multiplier
+    lr_max: float = 1.0       # Q25: powers-of-10 grid at b_max
+    n_sim: int = 1            # simulated replicas (tiny: 2)
+
+    @property
+    def b_min(self) -> int:          # b_min = b_max / 8
+        return self.b_max // 8
+
+    @property
+    def beta(self) -> int:           # beta = b_min / 2
+        return self.b_min // 2
+
+    @property
+    def mega_batch(self) -> int:     # Q8: M = 100 * b_max (tiny: 10 * 32)
+        return (10 if self.name == "tiny" else 100) * self.b_max
+
+    @property
+    def seed(self) -> int:
+        return 20220000 + self.index
+
+    @property
+    def n_params(self) -> int:
+        return self.F * self.H + self.H + self.L * self.H + self.L
+
+
+CONFIGS: Dict[str, XmlConfig] = {
+    c.name: c for c in [
+        XmlConfig("tiny", 0, F=2000, L=100, H=64, n_train=4096, n_test=1024,
+                  s_bar=20.0, s_sigma=0.5, y_bar=3.0, b_max=32, n_sim=2),
+        XmlConfig("eurlex4k", 1, F=5000, L=3993, H=256, n_train=15539,
+                  n_test=3809, s_bar=236.8, s_sigma=0.8, y_bar=5.31, b_max=256),
+        XmlConfig("amazoncat13k", 2, F=203882, L=13330, H=256,
+                  n_train=1186239, n_test=306782, s_bar=71.2, s_sigma=0.8,
+                  y_bar=5.04, b_max=1024),
+        XmlConfig("wiki10_31k", 3, F=101938, L=30938, H=256, n_train=14146,
+                  n_test=6616, s_bar=673.4, s_sigma=1.0, y_bar=18.64,
+                  b_max=256, block_skew=True),
+        XmlConfig("amazon670k", 4, F=135909, L=670091, H=256, n_train=490449,
+                  n_test=153025, s_bar=76.0, s_sigma=0.8, y_bar=5.0,
+                  b_max=1024),
+    ]
+}
+
+
+def config(name: str, **overrides) -> XmlConfig:
+    c = CONFIGS[name]
+    return dataclasses.replace(c, **overrides) if overrides else c
+
+
+def param_layout(F: int, H: int, L: int):
+    """Offsets of the flat parameter vector: W1 (F x H), b1 (H), W2 (L x H), b2 (L)."""
+    o_w1 = 0
+    o_b1 = o_w1 + F * H
+    o_w2 = o_b1 + H
+    o_b2 = o_w2 + L * H
+    return {"W1": (o_w1, (F, H)), "b1": (o_b1, (H,)),
+            "W2": (o_w2, (L, H)), "b2": (o_b2, (L,)), "P": o_b2 + L}
+
+
+# ----------------------------------------------------------------------------
+# counter-based RNG
+# ----------------------------------------------------------------------------
+_M1 = np.uint64(0xBF58476D1CE4E5B9)
+_M2 = np.uint64(0x94D049BB133111EB)
+_G = np.uint64(0x9E3779B97F4A7C15)
+_S30, _S27, _S31, _S11 = (np.uint64(s) for s in (30, 27, 31, 11))
+
+
+def _mix64(x):
+    x = x ^ (x >> _S30)
+    x = x * _M1
+    x = x ^ (x >> _S27)
+    x = x * _M2
+    return x ^ (x >> _S31)
+
+
+def _hash(seed: int, stream: int, *idx):
+    with np.errstate(over="ignore"):
+        h = _mix64(np.uint64(seed) * _G + np.uint64(stream))
+        for i in idx:
+            h = _mix64(h + np.asarray(i).astype(np.uint64) * _G)
+    return h
+
+
+def _u01(h):
+    """[0, 1) with 53 random bits."""
+    return (h >> _S11).astype(np.float64) * (1.0 / 9007199254740992.0)
+
+
+def _normal(seed, stream, *idx):
+    """Box-Muller; the two uniforms come from idx + (0,) and idx + (1,)."""
+    u1 = 1.0 - _u01(_hash(seed, stream, *idx, 0))      # (0, 1]
+    u2 = _u01(_hash(seed, stream, *idx, 1))
+    return np.sqrt(-2.0 * np.log(u1)) * np.cos(2.0 * math.pi * u2)
+
+
+def _zipf_cdf(n: int) -> np.ndarray:
+    w = 1.0 / np.arange(1, n + 1, dtype=np.float64)
+    c = np.cumsum(w)
+    return c / c[-1]
+
+
+def _zipf_rank(cdf: np.ndarray, u: np.ndarray) -> np.ndarray:
+    r = np.searchsorted(cdf, u, side="right")
+    return np.minimum(r, len(cdf) - 1)
+
+
+def _scramble(seed: int, stream: int, n: int) -> np.ndarray:
+    keys = _hash(seed, stream, np.arange(n, dtype=np.int64))
+    return np.argsort(keys, kind="stable").astype(np.int64)
+
+
+def _poisson_inv(lam: float, u: np.ndarray, kmax: int) -> np.ndarray:
+    k = np.arange(kmax + 1)
+    logp = -lam + k * math.log(lam) - np.array([math.lgamma(i + 1) for i in k]) if lam > 0 \
+        else np.where(k == 0, 0.0, -np.inf)
+    cdf = np.cumsum(np.exp(logp))
+    cdf[-1] = 1.0
+    return np.searchsorted(cdf, u, side="right")
+
+
+def _first_k_distinct(row, pos, ident, k_row, n_ids):
+    """Per row keep the first k_row[row] distinct ids in `pos` order.
+
+    Returns (row, ident, rank) of the kept entries sorted by (row, rank)."""
+    key = row * np.int64(n_ids) + ident
+    order = np.lexsort((pos, key))
+    ks = key[order]
+    first = np.ones(len(ks), dtype=bool)
+    first[1:] = ks[1:] != ks[:-1]
+    keep = order[first]
+    keep = keep[np.lexsort((pos[keep], row[keep]))]
+    r = row[keep]
+    # rank within row
+    starts = np.searchsorted(r, r, side="left")
+    rank = np.arange(len(r)) - starts
+    sel = rank < k_row[r]
+    return r[sel], ident[keep][sel], rank[sel]
+
+
+# ----------------------------------------------------------------------------
+# dataset
+# ----------------------------------------------------------------------------
+
+
+@dataclasses.dataclass
+class Dataset:
+    """One split in CSR: features (row_ptr, col, val) and labels (lab_ptr, lab)."""
+    row_ptr: np.ndarray   # int64 [n+1]
+    col: np.ndarray       # int32 [nnz], sorted & unique within a row
+    val: np.ndarray       # float32 [nnz]
+    lab_ptr: np.ndarray   # int64 [n+1]
+    lab: np.ndarray       # int32 [n_lab], sorted & unique within a row
+    n_features: int
+    n_labels: int
+
+    @property
+    def n_rows(self) -> int:
+        return len(self.row_ptr) - 1
+
+    @property
+    def nnz(self) -> int:
+        return int(self.row_ptr[-1])
+
+    def row_slice(self, rows: np.ndarray) -> "Dataset":
+        """CSR of the given rows, in that order (data movement only)."""
+        rows = np.asarray(rows, dtype=np.int64)
+        lens = self.row_ptr[rows + 1] - self.row_ptr[rows]
+        rp = np.zeros(len(rows) + 1, dtype=np.int64)
+        np.cumsum(lens, out=rp[1:])
+        idx = np.repeat(self.row_ptr[rows] - rp[:-1], lens) + np.arange(rp[-1])
+        llens = self.lab_ptr[rows + 1] - self.lab_ptr[rows]
+        lp = np.zeros(len(rows) + 1, dtype=np.int64)
+        np.cumsum(llens, out=lp[1:])
+        lidx = np.repeat(self.lab_ptr[rows] - lp[:-1], llens) + np.arange(lp[-1])
+        return Dataset(rp, self.col[idx], self.val[idx], lp, self.lab[lidx],
+                       self.n_features, self.n_labels)
+
+
+def _gen_split(cfg: XmlConfig, split: int, n: int, chunk: int = 32768) -> Dataset:
+    seed, F, L = cfg.seed, cfg.F, cfg.L
+    cdf_F, cdf_L = _zipf_cdf(F), _zipf_cdf(L)
+    scr_F = _scramble(seed, 10, F)
+    scr_L = _scramble(seed, 9, L)
+    # label signatures: 16 uniform features per label (stream 5)
+    sig = np.floor(_u01(_hash(seed, 5, np.arange(L, dtype=np.int64)[:, None],
+                              np.arange(16, dtype=np.int64)[None, :])) * F).astype(np.int64)
+    mu = math.log(cfg.s_bar) - 0.5 * cfg.s_sigma ** 2
+    rp_parts, col_parts, val_parts, lp_parts, lab_parts = [], [], [], [], []
+    for r0 in range(0, n, chunk):
+        rows = np.arange(r0, min(n, r0 + chunk), dtype=np.int64)
+        nr = len(rows)
+        # --- nnz per row (streams 0, 8)
+        z = _normal(seed, 0, split, rows)
+        s = np.exp(mu + cfg.s_sigma * z)
+        if cfg.block_skew:
+            blk = rows // 64
+            zb = _normal(seed, 8, split, blk)
+            s = s * np.exp(-0.5 + 1.0 * zb)
+        s_n = np.clip(np.rint(s), 1, F).astype(np.int64)
+        # --- labels (streams 3, 4)
+        kmax = int(cfg.y_bar * 6 + 20)
+        c_n = 1 + _poisson_inv(cfg.y_bar - 1.0, _u01(_hash(seed, 3, split, rows)), kmax)
+        c_n = np.minimum(c_n, L).astype(np.int64)
+        nl_cand = 2 * c_n + 4
+        lrow = np.repeat(np.arange(nr), nl_cand)
+        lpos = np.arange(len(lrow)) - np.repeat(np.cumsum(nl_cand) - nl_cand, nl_cand)
+        u = _u01(_hash(seed, 4, split, rows[lrow], lpos))
+        lid = scr_L[_zipf_rank(cdf_L, u)]
+        lr_, lid_, _ = _first_k_distinct(lrow, lpos, lid, c_n, L)
+        order = np.lexsort((lid_, lr_))
+        lr_, lid_ = lr_[order], lid_[order]
+        lcnt = np.bincount(lr_, minlength=nr)
+        lptr = np.zeros(nr + 1, dtype=np.int64)
+        np.cumsum(lcnt, out=lptr[1:])
+        # --- features (stream 1): signature draws then Zipf noise draws
+        n_sig = s_n // 2
+        n_noise = 2 * s_n + 8
+        n_cand = n_sig + n_noise
+        frow = np.repeat(np.arange(nr), n_cand)
+        fpos = np.arange(len(frow)) - np.repeat(np.cumsum(n_cand) - n_cand, n_cand)
+        h1 = _hash(seed, 1, split, rows[frow], fpos, 0)
+        h2 = _hash(seed, 1, split, rows[frow], fpos, 1)
+        is_sig = fpos < n_sig[frow]
+        # signature draw: a random label of the row, a random one of its 16 ids
+        nlab_row = lcnt[frow]
+        pick = np.minimum((_u01(h1) * nlab_row).astype(np.int64), nlab_row - 1)
+        lab_of = lid_[lptr[frow] + pick]
+        k16 = np.minimum((_u01(h2) * 16).astype(np.int64), 15)
+        fid_sig = sig[lab_of, k16]
+        fid_noise = scr_F[_zipf_rank(cdf_F, _u01(h1))]
+        fid = np.where(is_sig, fid_sig, fid_noise)
+        fr_, fid_, frank = _first_k_distinct(frow, fpos, fid, s_n, F)
+        # --- values (stream 2): U(0.5, 1.5), L2-normalised per row
+        v = 0.5 + _u01(_hash(seed, 2, split, rows[fr_], frank))
+        sq = np.bincount(fr_, weights=v * v, minlength=nr)
+        v = v / np.sqrt(sq)[fr_]
+        order = np.lexsort((fid_, fr_))
+        fr_, fid_, v = fr_[order], fid_[order], v[order]
+        fcnt = np.bincount(fr_, minlength=nr)
+        rp_parts.append(fcnt)
+        col_parts.append(fid_.astype(np.int32))
+        val_parts.append(v.astype(np.float32))
+        lp_parts.append(lcnt)
+        lab_parts.append(lid_.astype(np.int32))
+    fc = np.concatenate(rp_parts)
+    lc = np.concatenate(lp_parts)
+    row_ptr = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(fc, out=row_ptr[1:])
+    lab_ptr = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(lc, out=lab_ptr[1:])
+    return Dataset(row_ptr, np.concatenate(col_parts), np.concatenate(val_parts),
+                   lab_ptr, np.concatenate(lab_parts), F, L)
+
+
+def generate(cfg: XmlConfig, split: str = "train", n_rows: Optional[int] = None) -> Dataset:
+    """Generate the train (split 0) or test (split 1) set; optionally only the
+    first n_rows rows (identical to the prefix of the full split)."""
+    sid = {"train": 0, "test": 1}[split]
+    n = cfg.n_train if sid == 0 else cfg.n_test
+    if n_rows is not None:
+        n = min(n, n_rows)
+    return _gen_split(cfg, sid, n)
+
+
+def pass_permutation(cfg: XmlConfig, p: int, n_train: Optional[int] = None) -> np.ndarray:
+    """Sample order of pass p (stream 6): int32 permutation of [0, n_train)."""
+    n = cfg.n_train if n_train is None else n_train
+    keys = _hash(cfg.seed, 6, p, np.arange(n, dtype=np.int64))
+    return np.argsort(keys, kind="stable").astype(np.int32)
+
+
+def sample_stream(cfg: XmlConfig, start: int, length: int,
+                  n_train: Optional[int] = None) -> np.ndarray:
+    """Stream positions [start, start+length) of the concatenation of the
+    per-pass permutations pi_0, pi_1, ... (reading Q31)."""
+    n = cfg.n_train if n_train is None else n_train
+    out = np.empty(length, dtype=np.int32)
+    pos, i = start, 0
+    while i < length:
+        p, off = divmod(pos, n)
+        take = min(n - off, length - i)
+        out[i:i + take] = pass_permutation(cfg, p, n)[off:off + take]
+        i += take
+        pos += take
+    return out
+
+
+def init_params(cfg: XmlConfig) -> np.ndarray:
+    """Flat fp32 parameters W1, b1, W2, b2 (stream 7), reading Q5."""
+    lay = param_layout(cfg.F, cfg.H, cfg.L)
+    w = np.zeros(lay["P"], dtype=np.float32)
+    o, (F, H) = lay["W1"]
+    n1 = F * H
+    for c0 in range(0, n1, 1 << 24):
+        i = np.arange(c0, min(n1, c0 + (1 << 24)), dtype=np.int64)
+        w[o + c0:o + c0 + len(i)] = (_normal(cfg.seed, 7, 0, i) / math.sqrt(cfg.H)).astype(np.float32)
+    o, (L, H) = lay["W2"]
+    n2 = L * H
+    for c0 in range(0, n2, 1 << 24):
+        i = np.arange(c0, min(n2, c0 + (1 << 24)), dtype=np.int64)
+        w[o + c0:o + c0 + len(i)] = (_normal(cfg.seed, 7, 2, i) / math.sqrt(cfg.L)).astype(np.float32)
+    return w
