@@ -1,0 +1,267 @@
+/*
+ * asgd.h -- C ABI of libasgd.so, the B200 (sm_100a) hot path of Adaptive SGD
+ * (Ma, Rusu, Wu, Sim, "Adaptive Optimization for Sparse Data on Heterogeneous
+ * GPUs", IPDPSW 2022).  "P:a-b" cites lines a..b of the paper's text
+ * (/root/reference/PAPER.md); "Qn" cites a reading listed in DESIGN.md.
+ *
+ * Conventions (all entry points):
+ *  - Every call returns int status: ASGD_OK (0) or one of ASGD_E_*.  The
+ *    message of the last failure on the calling thread is asgd_last_error().
+ *    No C++ exception crosses this boundary and the library never aborts.
+ *  - Device pointers ("_dev" / documented as device) must be CUDA device
+ *    memory of the ctx's device; host pointers ("_host") are host memory.
+ *    Float/int arrays must be aligned to 16 bytes.
+ *  - The CALLER owns all device memory (dataset, params, w, d, outputs and
+ *    the workspace sized by asgd_workspace_bytes).  The library allocates only
+ *    the host-side ctx / scheduler structs.
+ *  - All device work is enqueued on the ctx's cudaStream_t (passed as void*);
+ *    calls are asynchronous unless documented "synchronous".  Asynchronous
+ *    CUDA / device-side errors are sticky: the next call on the ctx (or
+ *    asgd_sync) reports them as ASGD_E_CUDA.
+ *  - One ctx per GPU (per replica), driven by one thread at a time.  The
+ *    host-pure functions (asgd_merge_weights, asgd_scale_batches,
+ *    asgd_route_*, asgd_precision_at_k) are reentrant.
+ *  - There is no CPU fallback: without an sm_100 device every device call
+ *    fails with ASGD_E_CUDA / ASGD_E_UNSUPPORTED.
+ *
+ * Model (§V-A; D3): a 3-layer MLP  X (B x F, CSR) -> ReLU hidden
+ * (H) -> softmax over L labels, cross-entropy loss with the uniform target
+ * T_nj = 1/|Y_n| on the true labels (Q3), batch-mean reduction (Q4).  The
+ * parameters are ONE flat fp32 vector of P = F*H + H + L*H + L entries, in
+ * order W1 (F x H row-major, feature-major), b1 (H), W2 (L x H row-major,
+ * label-major), b2 (L), so that one all-reduce covers the whole replica.
+ */
+#ifndef ASGD_H_
+#define ASGD_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define ASGD_OK 0
+#define ASGD_E_ARG 1          /* null / misaligned pointer, bad scalar        */
+#define ASGD_E_SHAPE 2        /* sizes inconsistent with the model / data     */
+#define ASGD_E_CUDA 3         /* CUDA runtime / device-side error (sticky)    */
+#define ASGD_E_STATE 4        /* call out of order (e.g. no data registered)  */
+#define ASGD_E_UNSUPPORTED 5  /* configuration not supported by this build    */
+
+/* Arithmetic of the dense output-layer contractions (Q28).
+ * ASGD_PREC_FP32: fp32 CUDA-core FFMA contractions (tolerance 1e-4 vs fp64).
+ * ASGD_PREC_BF16: tcgen05 tensor-core GEMMs, bf16 operands, fp32 accumulate
+ *                 (tolerance 2e-2).  Master weights are fp32 in both. */
+#define ASGD_PREC_FP32 0
+#define ASGD_PREC_BF16 1
+
+typedef struct asgd_ctx asgd_ctx;
+typedef struct asgd_sched asgd_sched;
+
+typedef struct {
+  int64_t F;              /* input features                                 */
+  int64_t L;              /* labels (output units)                          */
+  int64_t H;              /* hidden units; one of 64, 128, 256, 512         */
+  int32_t precision;      /* ASGD_PREC_*                                    */
+  int32_t b_max;          /* max rows of one local step (<= 2048)           */
+  int64_t max_step_nnz;   /* max feature nnz of one step's rows             */
+  int64_t max_step_labels;/* max label entries of one step's rows           */
+} asgd_model_desc;
+
+/* A CSR split: features (row_ptr, col, val) and labels (lab_ptr, lab).
+ * row_ptr/lab_ptr: int64[n_rows+1], monotone, row_ptr[0] = lab_ptr[0] = 0;
+ * col: int32[nnz] in [0, F), strictly increasing within a row; val: fp32[nnz];
+ * lab: int32[n_lab] in [0, L), strictly increasing within a row, >= 1 label
+ * per row (Table I; D1, D2). */
+typedef struct {
+  const int64_t* row_ptr;
+  const int32_t* col;
+  const float* val;
+  const int64_t* lab_ptr;
+  const int32_t* lab;
+  int64_t n_rows;
+  int64_t nnz;
+  int64_t n_lab;
+} asgd_csr;
+
+/* ---------------------------------------------------------------- replica */
+
+/* Bytes of device workspace one ctx needs for this model (>= 0; 0 = bad desc). */
+size_t asgd_workspace_bytes(const asgd_model_desc* desc);
+
+/* Create the replica context of one GPU (S2: the "GPU manager").
+ * params: fp32[P] device, the replica w_i; w: fp32[P] device, the global
+ * model; d: fp32[P] device, w - w_p (Q19: caller zero-fills before the first
+ * merge).  ws: device workspace of ws_bytes >= asgd_workspace_bytes(desc).
+ * stream: cudaStream_t (NULL = legacy default stream).  Synchronous.
+ * Sets u = 0.  Errors: ASGD_E_ARG, ASGD_E_SHAPE, ASGD_E_UNSUPPORTED
+ * (H not supported, device is not sm_100), ASGD_E_CUDA. */
+int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device,
+                      void* stream, float* params, float* w, float* d, void* ws,
+                      size_t ws_bytes);
+
+/* Free the host-side ctx (device memory belongs to the caller). */
+int asgd_replica_destroy(asgd_ctx* ctx);
+
+/* Switch the stream later calls enqueue on. */
+int asgd_set_stream(asgd_ctx* ctx, void* stream);
+
+/* The caller changed params outside the library (e.g. copied w into it at a
+ * mega-batch start): refresh derived copies (bf16 shadow of W2).
+ * Asynchronous. */
+int asgd_params_changed(asgd_ctx* ctx);
+
+/* Register the (device-resident, read-only) training split the local steps
+ * index into.  Validates the CSR invariants once on the device (monotone
+ * pointers, ids in range, strictly increasing within rows, >= 1 label per
+ * row).  Synchronous.  ASGD_E_SHAPE if an invariant fails. */
+int asgd_data_register(asgd_ctx* ctx, const asgd_csr* dev_csr);
+
+/* Copy a HOST split (pinned memory for asynchronous copies) into caller-owned
+ * device arrays dev_dst (same sizes) on the ctx stream and register it without
+ * re-validation (the e2e path: host buffers -> device -> local steps).
+ * Asynchronous. */
+int asgd_data_upload(asgd_ctx* ctx, const asgd_csr* host_src, const asgd_csr* dev_dst);
+
+/* One local minibatch SGD step on the replica (A1; rows a2-a8 of
+ * DESIGN.md §Path): rows_dev: int32[n_rows] device, sample ids of the batch
+ * (a slice of the pass permutation, Q31), 1 <= n_rows <= b_max; lr: this
+ * replica's learning rate lr_i.  Computes, all on the device:
+ *   K-0 batch CSR view + touched-feature set (sorted unique cols, segments);
+ *   K-1 A1 = X W1 + b1, H1 = ReLU(A1);   G1 Z = H1 W2^T + b2;
+ *   softmax-CE: per-row lse, loss, dZ = (softmax(Z) - T)/B;
+ *   G2 dH1 = dZ W2 (pre-step W2), dA1 = dH1 * [A1 > 0], b1 -= lr 1^T dA1;
+ *   G3 W2 -= lr dZ^T H1, b2 -= lr 1^T dZ;
+ *   K-5 W1[f,:] -= lr sum_{n: X_nf != 0} X_nf dA1[n,:] on touched f only.
+ * loss_dev: nullable fp32 device scalar, receives the step's mean loss (Q33).
+ * u += 1 (a truncated batch counts, Q9).  Asynchronous. */
+int asgd_local_step(asgd_ctx* ctx, const int32_t* rows_dev, int32_t n_rows,
+                    float lr, float* loss_dev);
+
+/* Number of local steps since the last asgd_merge_finish (u_i). */
+int asgd_updates(const asgd_ctx* ctx, int64_t* u_out);
+
+/* Debug/parity: when grad_dev (fp32[P] device) is non-null, the next local
+ * steps also write their full gradient there (zero outside touched W1 rows).
+ * The fused kernels never materialise it otherwise.  NULL turns it off. */
+int asgd_set_debug_grads(asgd_ctx* ctx, float* grad_dev);
+
+/* Debug/parity: the sorted unique feature ids of the last local step
+ * (touched W1 rows).  out_dev: int32[cap] device; *n_out_host = count.
+ * Synchronous. ASGD_E_SHAPE if cap is too small. */
+int asgd_last_touched(asgd_ctx* ctx, int32_t* out_dev, int64_t cap, int64_t* n_out_host);
+
+/* ------------------------------------------------------------------ merge */
+
+/* sum_k params[k]^2 in fp64 (deterministic order) for Alg. 2 line 4's
+ * ||w_i||_2 / |w| (Q16).  out_dev: fp64 device scalar.  Asynchronous. */
+int asgd_replica_sqnorm(asgd_ctx* ctx, double* out_dev);
+
+/* Alg. 2 lines 1-7, host, pure.  u, b: int64[n]; nu: fp64[n]
+ * norms per parameter ||w_i||_2 / P.  Ties: key (u_i, b_i), lowest index,
+ * perturbation skipped when key(r) == key(s) (Q17); no renormalisation unless
+ * pert_renorm != 0 (Q18, Q34).  alpha_out: fp64[n]; r_out, s_out,
+ * perturbed_out: nullable. */
+int asgd_merge_weights(int32_t n, const int64_t* u, const int64_t* b,
+                       const double* nu, double pert_thr, double delta,
+                       int32_t pert_renorm, double* alpha_out, int32_t* r_out,
+                       int32_t* s_out, int32_t* perturbed_out);
+
+/* params <- alpha * params (Alg. 2 line 8's alpha_i w_i, K-6).  Asynchronous.
+ * After it the caller sums the prescaled replicas (one NCCL all-reduce SUM
+ * over NVLink, or asgd_replicas_weighted_sum on one device). */
+int asgd_merge_prescale(asgd_ctx* ctx, double alpha);
+
+/* Alg. 2 lines 8-9 epilogue (K-7), params holding S = sum_i alpha_i w_i:
+ * w' = S + gamma d;  d <- w' - w;  w <- w';  params <- w' (Q20, Q21);
+ * refreshes derived copies; u <- 0.  Asynchronous. */
+int asgd_merge_finish(asgd_ctx* ctx, float gamma);
+
+/* Single-device stand-in for the all-reduce (simulated replicas):
+ * out[k] = sum_i alpha_i * replicas[i][k] for k < P, alpha in fp64, summed in
+ * replica order.  replicas_dev: device array of n device pointers.
+ * Enqueued on ctx's stream. */
+int asgd_replicas_weighted_sum(asgd_ctx* ctx, const float* const* replicas_dev,
+                               const double* alpha_dev, int32_t n, float* out_dev);
+
+/* ---------------------------------------------------------------- scaling */
+
+/* Alg. 1, host, pure, exact integers: increments
+ * beta (u_i - mu~) = beta (N u_i - sum u)/N truncated toward zero (Q12); a
+ * violated bound leaves b_i unchanged (Q13); lr_i = lr_max * b_i / b_max (Q14).
+ * b_inout: int64[n]; lr_out: fp64[n] (nullable). */
+int asgd_scale_batches(int32_t n, const int64_t* u, int64_t* b_inout,
+                       double* lr_out, int64_t b_min, int64_t b_max,
+                       int64_t beta, double lr_max);
+
+/* -------------------------------------------------------------- routing */
+
+/* Dynamic scheduler (S3): a ticket counter in POSIX
+ * shared memory `shm_name` shared by the n_ranks processes of one node.
+ * Rank 0 creates (create != 0), the others attach.  Each mega-batch holds M
+ * samples (Q8). */
+int asgd_sched_open(const char* shm_name, int32_t n_ranks, int64_t M,
+                    int32_t create, asgd_sched** out);
+/* Next batch for `rank` with batch size b_i: on success *start, *len are the
+ * range [c, min(c + b_i, M)) of the mega-batch and the return is 1; 0 when
+ * the mega-batch is exhausted (c >= M); < 0 on error (negated ASGD_E_*).
+ * Lock-free (atomic fetch-add); appends (ticket, rank, start, len) to the log. */
+int asgd_sched_next(asgd_sched* s, int32_t rank, int64_t b_i, int64_t* start,
+                    int64_t* len);
+/* Copy the log of the current mega-batch: out: int64[4*cap] rows of
+ * (ticket, rank, start, len) in ticket order; *n_out = entries. */
+int asgd_sched_log(asgd_sched* s, int64_t* out, int64_t cap, int64_t* n_out);
+/* Start mega-batch `mb` (rank 0 only, after every rank is done with mb - 1):
+ * cursor <- 0, then publishes mb (release). */
+int asgd_sched_reset(asgd_sched* s, int64_t mb);
+/* Block until mega-batch `mb` (or a later one) is published by
+ * asgd_sched_reset, at most timeout_ms; ASGD_E_STATE on timeout. */
+int asgd_sched_wait(asgd_sched* s, int64_t mb, int64_t timeout_ms);
+int asgd_sched_close(asgd_sched* s, int32_t unlink_shm);
+
+/* Replay (parity): ranks in ticket order -> routes (rank, start, len) with the
+ * batch sizes b[rank], stopping at M.  out: int64[3*cap]. */
+int asgd_route_replay(int32_t n_tickets, const int32_t* order, const int64_t* b,
+                      int64_t M, int64_t* out, int64_t cap, int64_t* n_out);
+/* Simulated clock (Q10): every rank free at t = 0; the rank free first (ties:
+ * lowest id) takes the next batch; it stays busy
+ * cost_factor[r] * (nnz(batch) + per_row * len).  row_nnz: int64[M] nnz of the
+ * mega-batch's samples in stream order.  out: int64[3*cap]. */
+int asgd_route_simulate(int32_t n, const int64_t* b, int64_t M,
+                        const double* cost_factor, double per_row,
+                        const int64_t* row_nnz, int64_t* out, int64_t cap,
+                        int64_t* n_out);
+
+/* ------------------------------------------------------------- evaluate */
+
+/* Top-k labels of the replica's model for test rows (a13):
+ * rows_dev: int32[n] ids into test_dev (device CSR, validated on first use);
+ * topk_dev: int32[n*k] device, per row the k highest-scoring labels, ties to
+ * the lower id (Q23); 1 <= k <= 8.  Asynchronous.  Untimed. */
+int asgd_eval_topk(asgd_ctx* ctx, const asgd_csr* test_dev, const int32_t* rows_dev,
+                   int32_t n, int32_t k, int32_t* topk_dev);
+
+/* Host, pure: hits = sum_n |topk_n[:k] cap Y_n| for P@k = hits / (k n). */
+int asgd_precision_at_k(const int32_t* topk_host, const int64_t* lab_ptr,
+                        const int32_t* lab, int32_t n, int32_t k, int64_t* hits_out);
+
+/* --------------------------------------------------------------- misc */
+
+/* Wait for the ctx's stream; report sticky asynchronous errors. */
+int asgd_sync(asgd_ctx* ctx);
+
+/* Number of kernels this ctx launched so far (for the bench's gpu_launches). */
+int asgd_kernel_launches(const asgd_ctx* ctx, int64_t* out);
+
+/* Async copy device -> host (pinned) on the ctx stream (e2e result read). */
+int asgd_copy_to_host(asgd_ctx* ctx, void* dst_host, const void* src_dev, size_t bytes);
+
+const char* asgd_last_error(void);
+
+/* Build identification, e.g. "asgd sm_100a <git-ish>". */
+const char* asgd_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ASGD_H_ */

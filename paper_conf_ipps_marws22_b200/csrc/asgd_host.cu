@@ -1,0 +1,672 @@
+// libasgd host side: the C ABI of include/asgd.h.
+//  - replica ctx (the paper's GPU manager, PAPER.md P:1184-1198 / Fig. 3):
+//    workspace carve-up, per-step kernel sequence, merge entry points;
+//  - host-pure algorithms: Alg. 1, Alg. 2 lines 1-7,
+//    routing replay / simulated clock, P@k counting;
+//  - the dynamic scheduler as a lock-free ticket counter in
+//    POSIX shared memory, shared by the one-process-per-GPU ranks.
+#include <fcntl.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "asgd_internal.h"
+
+using namespace asgd;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+int cuda_fail(cudaError_t e, const char* where) {
+  return fail(ASGD_E_CUDA, "%s: %s (%s)", where, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+#define CU(call)                                              \
+  do {                                                        \
+    cudaError_t _e = (call);                                  \
+    if (_e != cudaSuccess) return cuda_fail(_e, #call);       \
+  } while (0)
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+size_t up256(size_t x) { return (x + 255) & ~size_t(255); }
+
+constexpr int kSqnormParts = 1024;
+
+int splitk_for(const asgd_model_desc& d) {
+  // G2 (dH1 = dZ W2, M = b_max, N = H, K = L): split K so ~2 waves of CTAs run.
+  int64_t tiles;
+  if (d.precision == ASGD_PREC_BF16) tiles = ((d.b_max + 127) / 128) * ((d.H + 255) / 256);
+  else tiles = ((d.b_max + 63) / 64) * ((d.H + 63) / 64);
+  int64_t s = (2 * 148 + tiles - 1) / tiles;
+  s = std::min<int64_t>(s, std::max<int64_t>(1, d.L / 256));
+  return (int)std::max<int64_t>(1, std::min<int64_t>(s, 64));
+}
+
+}  // namespace
+
+namespace asgd {
+
+WsLayout ws_layout(const asgd_model_desc& d) {
+  WsLayout L{};
+  const int64_t F = d.F, H = d.H, Lb = d.L, B = d.b_max;
+  L.nz_cap = d.max_step_nnz;
+  L.nl_cap = d.max_step_labels;
+  L.u_cap = std::min<int64_t>(F, L.nz_cap);
+  L.n_pieces = (L.nz_cap + kPiece - 1) / kPiece;
+  L.n_tiles_f = (F + kScanTile - 1) / kScanTile;
+  L.splitk = splitk_for(d);
+  L.n_rowblk = (B + 15) / 16;
+  L.n_red = kSqnormParts;
+  L.part_stride = B * H;
+  const bool bf = d.precision == ASGD_PREC_BF16;
+  size_t o = 0;
+  auto take = [&](size_t bytes) { size_t r = o; o = up256(o + std::max<size_t>(bytes, 1)); return r; };
+  L.meta = take(64 * 4);
+  L.boff = take((B + 1) * 4);
+  L.loff = take((B + 1) * 4);
+  L.cnt = take(F * 4);
+  L.fseg = take(F * 4);
+  L.fuid = take(F * 4);
+  L.uniq = take((L.u_cap + 1) * 4);
+  L.useg = take((L.u_cap + 1) * 4);
+  L.tsum = take(L.n_tiles_f * 8);
+  L.tpre = take(L.n_tiles_f * 8);
+  L.e_n = take(L.nz_cap * 4);
+  L.e_v = take(L.nz_cap * 4);
+  L.e_u = take(L.nz_cap * 4);
+  L.part1 = take((size_t)2 * L.n_pieces * H * 4);
+  L.rowcnt = take(B * 4);
+  L.part5 = take((size_t)2 * L.n_pieces * H * 4);
+  L.ucnt = take((L.u_cap + 1) * 4);
+  L.h1 = take(B * H * 4);
+  L.h1b = take(bf ? B * H * 2 : 0);
+  L.z = take((size_t)B * Lb * 4);
+  L.dzb = take(bf ? (size_t)B * Lb * 2 : 0);
+  L.rowloss = take(B * 4);
+  L.dhpart = take((size_t)L.splitk * B * H * 4);
+  L.da1 = take(B * H * 4);
+  L.db1part = take(L.n_rowblk * H * 4);
+  L.w2b = take(bf ? (size_t)Lb * H * 2 : 0);
+  L.red = take((L.n_red + 8) * 8);
+  L.eval_top = take(B * 8 * 4);
+  L.total = o;
+  return L;
+}
+
+Ptrs ws_ptrs(char* b, const WsLayout& L) {
+  Ptrs p;
+  p.meta = (int32_t*)(b + L.meta); p.boff = (int32_t*)(b + L.boff); p.loff = (int32_t*)(b + L.loff);
+  p.cnt = (int32_t*)(b + L.cnt); p.fseg = (int32_t*)(b + L.fseg); p.fuid = (int32_t*)(b + L.fuid);
+  p.uniq = (int32_t*)(b + L.uniq); p.useg = (int32_t*)(b + L.useg); p.tsum = (int32_t*)(b + L.tsum);
+  p.tpre = (int32_t*)(b + L.tpre); p.e_n = (int32_t*)(b + L.e_n); p.e_v = (float*)(b + L.e_v);
+  p.e_u = (int32_t*)(b + L.e_u); p.part1 = (float*)(b + L.part1); p.rowcnt = (int32_t*)(b + L.rowcnt);
+  p.part5 = (float*)(b + L.part5); p.ucnt = (int32_t*)(b + L.ucnt); p.h1 = (float*)(b + L.h1);
+  p.h1b = (bf16*)(b + L.h1b); p.z = (float*)(b + L.z); p.dzb = (bf16*)(b + L.dzb);
+  p.rowloss = (float*)(b + L.rowloss); p.dhpart = (float*)(b + L.dhpart); p.da1 = (float*)(b + L.da1);
+  p.db1part = (float*)(b + L.db1part); p.w2b = (bf16*)(b + L.w2b); p.red = (double*)(b + L.red);
+  p.eval_top = (int32_t*)(b + L.eval_top);
+  return p;
+}
+
+}  // namespace asgd
+
+struct asgd_ctx {
+  asgd_model_desc d;
+  int device;
+  int sms;
+  cudaStream_t s;
+  float* params;
+  float* w;
+  float* dd;
+  char* ws;
+  size_t ws_bytes;
+  WsLayout L;
+  Ptrs P;
+  asgd_csr data;
+  bool has_data;
+  const void* eval_validated;
+  float* dbg;
+  int64_t u;
+  int64_t launches;
+  int64_t Pn;
+  int64_t o_w1, o_b1, o_w2, o_b2;
+  Launch lc() { return Launch{s, &launches, sms}; }
+};
+
+extern "C" {
+
+const char* asgd_last_error(void) { return g_err.c_str(); }
+
+const char* asgd_version(void) { return "libasgd sm_100a (tcgen05/TMA bf16 + fp32 SIMT) r1"; }
+
+size_t asgd_workspace_bytes(const asgd_model_desc* d) {
+  if (!d || d->F <= 0 || d->L <= 0 || d->b_max <= 0 || d->max_step_nnz <= 0) return 0;
+  return ws_layout(*d).total;
+}
+
+int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device, void* stream,
+                      float* params, float* w, float* d, void* ws, size_t ws_bytes) {
+  if (!out || !desc || !params || !w || !d || !ws) return fail(ASGD_E_ARG, "null argument");
+  if (!aligned16(params) || !aligned16(w) || !aligned16(d) || !aligned16(ws))
+    return fail(ASGD_E_ARG, "device buffers must be 16-byte aligned");
+  const asgd_model_desc& m = *desc;
+  if (m.H != 64 && m.H != 128 && m.H != 256 && m.H != 512)
+    return fail(ASGD_E_UNSUPPORTED, "H=%lld not in {64,128,256,512}", (long long)m.H);
+  if (m.F <= 0 || m.L <= 0 || m.b_max <= 0 || m.b_max > 2048 || m.max_step_nnz <= 0 ||
+      m.max_step_nnz >= (1ll << 31) || m.max_step_labels <= 0 || (int64_t)m.b_max * m.L >= (1ll << 40))
+    return fail(ASGD_E_SHAPE, "bad model desc (F=%lld L=%lld b_max=%d nnz=%lld)", (long long)m.F,
+                (long long)m.L, m.b_max, (long long)m.max_step_nnz);
+  if (m.precision != ASGD_PREC_FP32 && m.precision != ASGD_PREC_BF16)
+    return fail(ASGD_E_ARG, "precision %d", m.precision);
+  const size_t need = ws_layout(m).total;
+  if (ws_bytes < need) return fail(ASGD_E_SHAPE, "workspace %zu < %zu bytes", ws_bytes, need);
+  CU(cudaSetDevice(device));
+  cudaDeviceProp prop;
+  CU(cudaGetDeviceProperties(&prop, device));
+  if (prop.major != 10 || prop.minor != 0)
+    return fail(ASGD_E_UNSUPPORTED, "device %d is sm_%d%d; libasgd is built for sm_100a only", device,
+                prop.major, prop.minor);
+  if (m.precision == ASGD_PREC_BF16 && !tc_available())
+    return fail(ASGD_E_UNSUPPORTED, "bf16 tcgen05 path not built");
+  asgd_ctx* c = new (std::nothrow) asgd_ctx();
+  if (!c) return fail(ASGD_E_ARG, "out of host memory");
+  c->d = m;
+  c->device = device;
+  c->sms = prop.multiProcessorCount;
+  c->s = static_cast<cudaStream_t>(stream);
+  c->params = params;
+  c->w = w;
+  c->dd = d;
+  c->ws = static_cast<char*>(ws);
+  c->ws_bytes = ws_bytes;
+  c->L = ws_layout(m);
+  c->P = ws_ptrs(c->ws, c->L);
+  c->has_data = false;
+  c->eval_validated = nullptr;
+  c->dbg = nullptr;
+  c->u = 0;
+  c->launches = 0;
+  c->o_w1 = 0;
+  c->o_b1 = m.F * m.H;
+  c->o_w2 = c->o_b1 + m.H;
+  c->o_b2 = c->o_w2 + m.L * m.H;
+  c->Pn = c->o_b2 + m.L;
+  cudaError_t e = cudaMemsetAsync(c->ws, 0, c->L.total, c->s);
+  if (e == cudaSuccess && m.precision == ASGD_PREC_BF16)
+    e = launch_to_bf16(c->lc(), c->params + c->o_w2, c->P.w2b, m.L * m.H);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(c->s);
+  if (e != cudaSuccess) { delete c; return cuda_fail(e, "replica_init"); }
+  *out = c;
+  return ASGD_OK;
+}
+
+int asgd_replica_destroy(asgd_ctx* c) {
+  delete c;
+  return ASGD_OK;
+}
+
+int asgd_set_stream(asgd_ctx* c, void* stream) {
+  if (!c) return fail(ASGD_E_ARG, "null ctx");
+  c->s = static_cast<cudaStream_t>(stream);
+  return ASGD_OK;
+}
+
+int asgd_params_changed(asgd_ctx* c) {
+  if (!c) return fail(ASGD_E_ARG, "null ctx");
+  if (c->d.precision == ASGD_PREC_BF16)
+    CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->P.w2b, c->d.L * c->d.H));
+  return ASGD_OK;
+}
+
+static int validate(asgd_ctx* c, const asgd_csr* x) {
+  int32_t* err = c->P.meta + 16;
+  CU(cudaMemsetAsync(err, 0, 4, c->s));
+  CU(launch_validate_csr(c->lc(), x, c->d.F, c->d.L, err));
+  int32_t h = 0;
+  CU(cudaMemcpyAsync(&h, err, 4, cudaMemcpyDeviceToHost, c->s));
+  CU(cudaStreamSynchronize(c->s));
+  if (h) return fail(ASGD_E_SHAPE, "CSR invariant violated (bits 0x%x)", h);
+  return ASGD_OK;
+}
+
+int asgd_data_register(asgd_ctx* c, const asgd_csr* x) {
+  if (!c || !x || !x->row_ptr || !x->col || !x->val || !x->lab_ptr || !x->lab)
+    return fail(ASGD_E_ARG, "null argument");
+  if (x->n_rows <= 0 || x->nnz < 0 || x->n_lab <= 0) return fail(ASGD_E_SHAPE, "empty split");
+  int rc = validate(c, x);
+  if (rc) return rc;
+  c->data = *x;
+  c->has_data = true;
+  return ASGD_OK;
+}
+
+int asgd_data_upload(asgd_ctx* c, const asgd_csr* h, const asgd_csr* dv) {
+  if (!c || !h || !dv) return fail(ASGD_E_ARG, "null argument");
+  if (h->n_rows != dv->n_rows || h->nnz > dv->nnz || h->n_lab > dv->n_lab)
+    return fail(ASGD_E_SHAPE, "destination too small");
+  CU(cudaMemcpyAsync((void*)dv->row_ptr, h->row_ptr, (h->n_rows + 1) * 8, cudaMemcpyHostToDevice, c->s));
+  CU(cudaMemcpyAsync((void*)dv->col, h->col, h->nnz * 4, cudaMemcpyHostToDevice, c->s));
+  CU(cudaMemcpyAsync((void*)dv->val, h->val, h->nnz * 4, cudaMemcpyHostToDevice, c->s));
+  CU(cudaMemcpyAsync((void*)dv->lab_ptr, h->lab_ptr, (h->n_rows + 1) * 8, cudaMemcpyHostToDevice, c->s));
+  CU(cudaMemcpyAsync((void*)dv->lab, h->lab, h->n_lab * 4, cudaMemcpyHostToDevice, c->s));
+  c->data = *dv;
+  c->data.nnz = h->nnz;
+  c->data.n_lab = h->n_lab;
+  c->has_data = true;
+  return ASGD_OK;
+}
+
+int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float* loss_dev) {
+  if (!c || !rows) return fail(ASGD_E_ARG, "null argument");
+  if (!c->has_data) return fail(ASGD_E_STATE, "no data registered");
+  const asgd_model_desc& m = c->d;
+  if (n < 1 || n > m.b_max) return fail(ASGD_E_SHAPE, "n_rows=%d not in [1, %d]", n, m.b_max);
+  Launch lc = c->lc();
+  const Ptrs& P = c->P;
+  const asgd_csr& x = c->data;
+  const bool bf = m.precision == ASGD_PREC_BF16;
+  const int H = (int)m.H;
+  const int64_t Lb = m.L;
+  float* W1 = c->params + c->o_w1;
+  float* b1 = c->params + c->o_b1;
+  float* W2 = c->params + c->o_w2;
+  float* b2 = c->params + c->o_b2;
+  float* g = c->dbg;
+  if (g) CU(cudaMemsetAsync(g, 0, c->Pn * sizeof(float), c->s));
+  // K-0: batch view + touched-feature set
+  CU(launch_batch_scan(lc, rows, n, x.row_ptr, x.lab_ptr, x.n_rows, P, c->L.nz_cap, c->L.nl_cap));
+  CU(launch_touched(lc, rows, n, x.row_ptr, x.col, x.val, m.F, P, c->L, m.b_max));
+  // K-1
+  CU(launch_spmm_fwd(lc, rows, n, x.row_ptr, x.col, x.val, W1, b1, H, P, c->L, bf));
+  if (!bf) {
+    GemmArgs a{};
+    // G1: Z[n x L] = H1 W2^T + b2
+    a = GemmArgs{};
+    a.M = n; a.N = (int)Lb; a.K = H;
+    a.A = P.h1; a.as0 = H; a.as1 = 1;
+    a.B = W2; a.bs0 = 1; a.bs1 = H;
+    a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = Lb; a.bias = b2; a.splitk = 1;
+    CU(launch_gemm_f32(lc, a));
+    CU(launch_softmax_ce(lc, n, Lb, rows, x.lab_ptr, x.lab, P, false));
+    // G2: dH1 partials = dZ W2 (pre-step W2)
+    a = GemmArgs{};
+    a.M = n; a.N = H; a.K = (int)Lb;
+    a.A = P.z; a.as0 = Lb; a.as1 = 1;
+    a.B = W2; a.bs0 = H; a.bs1 = 1;
+    a.epi = EPI_SPLITK; a.C = P.dhpart; a.ldc = H; a.splitk = (int)c->L.splitk;
+    a.part_stride = c->L.part_stride;
+    CU(launch_gemm_f32(lc, a));
+  } else {
+    CU(launch_gemm_tc(lc, 1, n, Lb, H, lr, P, c->L, W2, b2, nullptr));
+    CU(launch_softmax_ce(lc, n, Lb, rows, x.lab_ptr, x.lab, P, true));
+    CU(launch_gemm_tc(lc, 2, n, Lb, H, lr, P, c->L, W2, b2, nullptr));
+  }
+  CU(launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L));
+  CU(launch_b1_update(lc, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev));
+  CU(launch_b2_update(lc, n, Lb, b2, lr, P, bf, g ? g + c->o_b2 : nullptr));
+  if (!bf) {
+    // G3: W2 -= lr dZ^T H1
+    GemmArgs a{};
+    a.M = (int)Lb; a.N = H; a.K = n;
+    a.A = P.z; a.as0 = 1; a.as1 = Lb;
+    a.B = P.h1; a.bs0 = H; a.bs1 = 1;
+    a.epi = EPI_SGD; a.C = W2; a.ldc = H; a.lr = lr; a.grad = g ? g + c->o_w2 : nullptr;
+    a.splitk = 1;
+    CU(launch_gemm_f32(lc, a));
+  } else {
+    CU(launch_gemm_tc(lc, 3, n, Lb, H, lr, P, c->L, W2, b2, g ? g + c->o_w2 : nullptr));
+  }
+  // K-5
+  CU(launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr));
+  ++c->u;
+  return ASGD_OK;
+}
+
+int asgd_updates(const asgd_ctx* c, int64_t* u) {
+  if (!c || !u) return fail(ASGD_E_ARG, "null argument");
+  *u = c->u;
+  return ASGD_OK;
+}
+
+int asgd_set_debug_grads(asgd_ctx* c, float* g) {
+  if (!c) return fail(ASGD_E_ARG, "null ctx");
+  if (g && !aligned16(g)) return fail(ASGD_E_ARG, "grad buffer must be 16-byte aligned");
+  c->dbg = g;
+  return ASGD_OK;
+}
+
+int asgd_last_touched(asgd_ctx* c, int32_t* out, int64_t cap, int64_t* n_out) {
+  if (!c || !out || !n_out) return fail(ASGD_E_ARG, "null argument");
+  int32_t U = 0;
+  CU(cudaMemcpyAsync(&U, c->P.meta + M_U, 4, cudaMemcpyDeviceToHost, c->s));
+  CU(cudaStreamSynchronize(c->s));
+  *n_out = U;
+  if (U > cap) return fail(ASGD_E_SHAPE, "cap %lld < %d touched", (long long)cap, U);
+  CU(cudaMemcpyAsync(out, c->P.uniq, (size_t)U * 4, cudaMemcpyDeviceToDevice, c->s));
+  CU(cudaStreamSynchronize(c->s));
+  return ASGD_OK;
+}
+
+int asgd_replica_sqnorm(asgd_ctx* c, double* out_dev) {
+  if (!c || !out_dev) return fail(ASGD_E_ARG, "null argument");
+  CU(launch_sqnorm(c->lc(), c->params, c->Pn, c->P.red, (int)c->L.n_red, out_dev));
+  return ASGD_OK;
+}
+
+int asgd_merge_prescale(asgd_ctx* c, double alpha) {
+  if (!c) return fail(ASGD_E_ARG, "null ctx");
+  CU(launch_scale(c->lc(), c->params, c->Pn, alpha));
+  return ASGD_OK;
+}
+
+int asgd_merge_finish(asgd_ctx* c, float gamma) {
+  if (!c) return fail(ASGD_E_ARG, "null ctx");
+  CU(launch_finish(c->lc(), c->params, c->w, c->dd, c->Pn, gamma));
+  if (c->d.precision == ASGD_PREC_BF16)
+    CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->P.w2b, c->d.L * c->d.H));
+  c->u = 0;
+  return ASGD_OK;
+}
+
+int asgd_replicas_weighted_sum(asgd_ctx* c, const float* const* reps, const double* alpha, int32_t n,
+                               float* out) {
+  if (!c || !reps || !alpha || !out || n < 1) return fail(ASGD_E_ARG, "bad argument");
+  CU(launch_wsum(c->lc(), reps, alpha, n, c->Pn, out));
+  return ASGD_OK;
+}
+
+int asgd_eval_topk(asgd_ctx* c, const asgd_csr* t, const int32_t* rows, int32_t n, int32_t k,
+                   int32_t* topk) {
+  if (!c || !t || !rows || !topk) return fail(ASGD_E_ARG, "null argument");
+  if (k < 1 || k > 8) return fail(ASGD_E_ARG, "k=%d not in [1, 8]", k);
+  if (c->eval_validated != (const void*)t->row_ptr) {
+    int rc = validate(c, t);
+    if (rc) return rc;
+    c->eval_validated = t->row_ptr;
+  }
+  const asgd_model_desc& m = c->d;
+  Launch lc = c->lc();
+  const Ptrs& P = c->P;
+  const int H = (int)m.H;
+  const bool bf = m.precision == ASGD_PREC_BF16;
+  float* W1 = c->params + c->o_w1;
+  float* b1 = c->params + c->o_b1;
+  float* W2 = c->params + c->o_w2;
+  float* b2 = c->params + c->o_b2;
+  for (int32_t r0 = 0; r0 < n; r0 += m.b_max) {
+    const int nb = std::min<int32_t>(m.b_max, n - r0);
+    CU(launch_batch_scan(lc, rows + r0, nb, t->row_ptr, t->lab_ptr, t->n_rows, P, c->L.nz_cap,
+                         c->L.nl_cap));
+    CU(launch_spmm_fwd(lc, rows + r0, nb, t->row_ptr, t->col, t->val, W1, b1, H, P, c->L, bf));
+    if (!bf) {
+      GemmArgs a{};
+      a.M = nb; a.N = (int)m.L; a.K = H;
+      a.A = P.h1; a.as0 = H; a.as1 = 1;
+      a.B = W2; a.bs0 = 1; a.bs1 = H;
+      a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = m.L; a.bias = b2; a.splitk = 1;
+      CU(launch_gemm_f32(lc, a));
+    } else {
+      CU(launch_gemm_tc(lc, 1, nb, m.L, H, 0.f, P, c->L, W2, b2, nullptr));
+    }
+    CU(launch_topk(lc, nb, m.L, k, P.z, topk + (int64_t)r0 * k));
+  }
+  return ASGD_OK;
+}
+
+int asgd_sync(asgd_ctx* c) {
+  if (!c) return fail(ASGD_E_ARG, "null ctx");
+  CU(cudaStreamSynchronize(c->s));
+  CU(cudaGetLastError());
+  int32_t err = 0;
+  CU(cudaMemcpy(&err, c->P.meta + M_ERR, 4, cudaMemcpyDeviceToHost));
+  if (err) {
+    CU(cudaMemset(c->P.meta + M_ERR, 0, 4));
+    return fail(ASGD_E_SHAPE, "device-side error 0x%x (1: step nnz > max_step_nnz, 2: labels > "
+                "max_step_labels, 4: row id out of range)", err);
+  }
+  return ASGD_OK;
+}
+
+int asgd_kernel_launches(const asgd_ctx* c, int64_t* out) {
+  if (!c || !out) return fail(ASGD_E_ARG, "null argument");
+  *out = c->launches;
+  return ASGD_OK;
+}
+
+int asgd_copy_to_host(asgd_ctx* c, void* dst, const void* src, size_t bytes) {
+  if (!c || !dst || !src) return fail(ASGD_E_ARG, "null argument");
+  CU(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, c->s));
+  return ASGD_OK;
+}
+
+// =================================================================== host-pure
+
+int asgd_merge_weights(int32_t n, const int64_t* u, const int64_t* b, const double* nu,
+                       double pert_thr, double delta, int32_t pert_renorm, double* alpha,
+                       int32_t* r_out, int32_t* s_out, int32_t* perturbed_out) {
+  if (n < 1 || !u || !b || !nu || !alpha) return fail(ASGD_E_ARG, "bad argument");
+  bool equal = true;                                   // Alg. 2 line 2
+  for (int i = 1; i < n; ++i) equal = equal && (u[i] == u[0]);
+  if (equal) {
+    int64_t sb = 0;
+    for (int i = 0; i < n; ++i) sb += b[i];
+    const double d = (double)sb;
+    for (int i = 0; i < n; ++i) alpha[i] = (double)b[i] / d;
+  } else {                                             // line 3
+    int64_t su = 0;
+    for (int i = 0; i < n; ++i) su += u[i];
+    const double d = (double)su;
+    for (int i = 0; i < n; ++i) alpha[i] = (double)u[i] / d;
+  }
+  bool gate = true;                                    // line 4 (Q16: strict <)
+  for (int i = 0; i < n; ++i) gate = gate && (nu[i] < pert_thr);
+  int r = 0, s = 0, pert = 0;
+  if (gate) {                                          // line 5 (Q17: key (u, b), lowest index)
+    for (int i = 1; i < n; ++i) {
+      if (u[i] > u[r] || (u[i] == u[r] && b[i] > b[r])) r = i;
+      if (u[i] < u[s] || (u[i] == u[s] && b[i] < b[s])) s = i;
+    }
+    if (u[r] != u[s] || b[r] != b[s]) {                // line 6
+      alpha[r] = (1.0 + delta) * alpha[r];
+      alpha[s] = (1.0 - delta) * alpha[s];
+      pert = 1;
+    }
+  }
+  if (pert_renorm) {                                   // Q34 option
+    double tot = 0.0;
+    for (int i = 0; i < n; ++i) tot += alpha[i];
+    for (int i = 0; i < n; ++i) alpha[i] = alpha[i] / tot;
+  }
+  if (r_out) *r_out = r;
+  if (s_out) *s_out = s;
+  if (perturbed_out) *perturbed_out = pert;
+  return ASGD_OK;
+}
+
+int asgd_scale_batches(int32_t n, const int64_t* u, int64_t* b, double* lr_out, int64_t b_min,
+                       int64_t b_max, int64_t beta, double lr_max) {
+  if (n < 1 || !u || !b || b_min < 1 || b_max < b_min) return fail(ASGD_E_ARG, "bad argument");
+  int64_t su = 0;                                      // Alg. 1 line 1
+  for (int i = 0; i < n; ++i) su += u[i];
+  for (int i = 0; i < n; ++i) {                        // line 2
+    const int64_t num = beta * ((int64_t)n * u[i] - su);
+    const int64_t delta = num >= 0 ? num / n : -((-num) / n);   // Q12: truncate toward 0
+    if ((int64_t)n * u[i] > su && b[i] + delta <= b_max) b[i] += delta;        // lines 3-5
+    else if ((int64_t)n * u[i] < su && b[i] + delta >= b_min) b[i] += delta;   // lines 6-8
+  }
+  if (lr_out)
+    for (int i = 0; i < n; ++i) lr_out[i] = lr_max * (double)b[i] / (double)b_max;  // Q14
+  return ASGD_OK;
+}
+
+int asgd_route_replay(int32_t nt, const int32_t* order, const int64_t* b, int64_t M, int64_t* out,
+                      int64_t cap, int64_t* n_out) {
+  if (nt < 0 || (nt && !order) || !b || !out || !n_out) return fail(ASGD_E_ARG, "bad argument");
+  int64_t c = 0, k = 0;
+  for (int32_t t = 0; t < nt && c < M; ++t) {
+    const int32_t r = order[t];
+    const int64_t len = std::min<int64_t>(b[r], M - c);
+    if (k >= cap) return fail(ASGD_E_SHAPE, "route cap %lld too small", (long long)cap);
+    out[3 * k] = r; out[3 * k + 1] = c; out[3 * k + 2] = len;
+    ++k;
+    c += len;
+  }
+  *n_out = k;
+  return ASGD_OK;
+}
+
+int asgd_route_simulate(int32_t n, const int64_t* b, int64_t M, const double* cf, double per_row,
+                        const int64_t* row_nnz, int64_t* out, int64_t cap, int64_t* n_out) {
+  if (n < 1 || !b || !cf || !row_nnz || !out || !n_out) return fail(ASGD_E_ARG, "bad argument");
+  std::vector<double> fr(n, 0.0);
+  int64_t c = 0, k = 0;
+  while (c < M) {
+    int r = 0;
+    for (int i = 1; i < n; ++i) if (fr[i] < fr[r]) r = i;   // ties: lowest id
+    const int64_t len = std::min<int64_t>(b[r], M - c);
+    if (len < 1) return fail(ASGD_E_ARG, "batch size < 1");
+    int64_t nnz = 0;
+    for (int64_t j = c; j < c + len; ++j) nnz += row_nnz[j];
+    if (k >= cap) return fail(ASGD_E_SHAPE, "route cap %lld too small", (long long)cap);
+    out[3 * k] = r; out[3 * k + 1] = c; out[3 * k + 2] = len;
+    ++k;
+    fr[r] += cf[r] * ((double)nnz + per_row * (double)len);
+    c += len;
+  }
+  *n_out = k;
+  return ASGD_OK;
+}
+
+int asgd_precision_at_k(const int32_t* top, const int64_t* lab_ptr, const int32_t* lab, int32_t n,
+                        int32_t k, int64_t* hits_out) {
+  if (!top || !lab_ptr || !lab || !hits_out || k < 1) return fail(ASGD_E_ARG, "bad argument");
+  int64_t hits = 0;
+  for (int32_t r = 0; r < n; ++r) {
+    const int32_t* y = lab + lab_ptr[r];
+    const int64_t ny = lab_ptr[r + 1] - lab_ptr[r];
+    for (int32_t j = 0; j < k; ++j) {
+      const int32_t p = top[(int64_t)r * k + j];
+      if (std::binary_search(y, y + ny, p)) ++hits;   // labels sorted within a row
+    }
+  }
+  *hits_out = hits;
+  return ASGD_OK;
+}
+
+// ------------------------------------------------------------------- scheduler
+struct ShmSched {
+  std::atomic<uint64_t> packed;   // ticket << 40 | cursor
+  int64_t M;
+  int64_t mb;
+  int64_t n_ranks;
+  int64_t cap;
+  int64_t log[1][4];
+};
+
+struct asgd_sched {
+  ShmSched* h;
+  size_t bytes;
+  std::string name;
+};
+
+static constexpr uint64_t kCurMask = (1ull << 40) - 1;
+
+int asgd_sched_open(const char* name, int32_t n_ranks, int64_t M, int32_t create, asgd_sched** out) {
+  if (!name || !out || n_ranks < 1 || M < 1 || M >= (1ll << 38)) return fail(ASGD_E_ARG, "bad argument");
+  const int64_t cap = M + 16;
+  const size_t bytes = sizeof(ShmSched) + (size_t)cap * 4 * sizeof(int64_t);
+  int fd = shm_open(name, create ? (O_CREAT | O_RDWR) : O_RDWR, 0600);
+  if (fd < 0) return fail(ASGD_E_ARG, "shm_open(%s) failed", name);
+  if (create && ftruncate(fd, (off_t)bytes) != 0) { close(fd); return fail(ASGD_E_ARG, "ftruncate failed"); }
+  void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  close(fd);
+  if (p == MAP_FAILED) return fail(ASGD_E_ARG, "mmap failed");
+  ShmSched* h = static_cast<ShmSched*>(p);
+  if (create) {
+    new (&h->packed) std::atomic<uint64_t>(0);
+    h->M = M; h->mb = 0; h->n_ranks = n_ranks; h->cap = cap;
+  }
+  asgd_sched* s = new (std::nothrow) asgd_sched{h, bytes, name};
+  if (!s) { munmap(p, bytes); return fail(ASGD_E_ARG, "out of host memory"); }
+  *out = s;
+  return ASGD_OK;
+}
+
+int asgd_sched_next(asgd_sched* s, int32_t rank, int64_t b, int64_t* start, int64_t* len) {
+  if (!s || !start || !len || b < 1) return -ASGD_E_ARG;
+  ShmSched* h = s->h;
+  const uint64_t v = h->packed.fetch_add((1ull << 40) | (uint64_t)b, std::memory_order_acq_rel);
+  const int64_t ticket = (int64_t)(v >> 40), c = (int64_t)(v & kCurMask);
+  if (c >= h->M) return 0;
+  const int64_t l = std::min<int64_t>(b, h->M - c);
+  if (ticket < h->cap) {
+    h->log[ticket][0] = ticket; h->log[ticket][1] = rank; h->log[ticket][2] = c; h->log[ticket][3] = l;
+  }
+  *start = c;
+  *len = l;
+  return 1;
+}
+
+int asgd_sched_log(asgd_sched* s, int64_t* out, int64_t cap, int64_t* n_out) {
+  if (!s || !out || !n_out) return fail(ASGD_E_ARG, "null argument");
+  ShmSched* h = s->h;
+  const int64_t T = (int64_t)(h->packed.load(std::memory_order_acquire) >> 40);
+  int64_t c = 0, k = 0;
+  while (k < T && k < h->cap && c < h->M) {
+    if (h->log[k][2] != c) return fail(ASGD_E_STATE, "log entry %lld not yet written", (long long)k);
+    if (k >= cap) return fail(ASGD_E_SHAPE, "cap too small");
+    for (int j = 0; j < 4; ++j) out[4 * k + j] = h->log[k][j];
+    c += h->log[k][3];
+    ++k;
+  }
+  *n_out = k;
+  return ASGD_OK;
+}
+
+int asgd_sched_reset(asgd_sched* s, int64_t mb) {
+  if (!s) return fail(ASGD_E_ARG, "null argument");
+  s->h->packed.store(0, std::memory_order_release);
+  reinterpret_cast<std::atomic<int64_t>*>(&s->h->mb)->store(mb, std::memory_order_release);
+  return ASGD_OK;
+}
+
+int asgd_sched_wait(asgd_sched* s, int64_t mb, int64_t timeout_ms) {
+  if (!s) return fail(ASGD_E_ARG, "null argument");
+  auto* p = reinterpret_cast<std::atomic<int64_t>*>(&s->h->mb);
+  for (int64_t spins = 0;; ++spins) {
+    if (p->load(std::memory_order_acquire) >= mb) return ASGD_OK;
+    if (spins / 20 > timeout_ms) return fail(ASGD_E_STATE, "timeout waiting for mega-batch %lld", (long long)mb);
+    usleep(50);
+  }
+}
+
+int asgd_sched_close(asgd_sched* s, int32_t unlink_shm) {
+  if (!s) return fail(ASGD_E_ARG, "null argument");
+  munmap(s->h, s->bytes);
+  if (unlink_shm) shm_unlink(s->name.c_str());
+  delete s;
+  return ASGD_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,102 @@
+// Internal declarations shared by the libasgd translation units (not ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+
+#include "../../include/asgd.h"
+
+namespace asgd {
+
+// Entries per work piece of the nnz-balanced sparse kernels (K-1, K-5).
+constexpr int kPiece = 32;
+// Max labels per row the softmax kernel stages in shared memory.
+constexpr int kMaxRowLabels = 1024;
+// Features per tile of the touched-feature scan.
+constexpr int kScanTile = 4096;
+// meta[] slots (int32, device)
+enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_COUNT = 8 };
+// error bits in meta[M_ERR]
+enum { ERR_NNZ_CAP = 1, ERR_LAB_CAP = 2, ERR_ROW_ID = 4 };
+
+typedef __nv_bfloat16 bf16;
+
+// Device workspace carve-up (byte offsets from ws base; all 256-B aligned).
+struct WsLayout {
+  size_t meta, boff, loff, cnt, fseg, fuid, uniq, useg, tsum, tpre;
+  size_t e_n, e_v, e_u, part1, rowcnt, part5, ucnt;
+  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, red, eval_top;
+  size_t total;
+  int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride;
+};
+
+WsLayout ws_layout(const asgd_model_desc& d);
+
+struct Ptrs {  // typed views of the workspace
+  int32_t* meta; int32_t* boff; int32_t* loff; int32_t* cnt; int32_t* fseg; int32_t* fuid;
+  int32_t* uniq; int32_t* useg; int32_t* tsum; int32_t* tpre;
+  int32_t* e_n; float* e_v; int32_t* e_u; float* part1; int32_t* rowcnt; float* part5;
+  int32_t* ucnt; float* h1; bf16* h1b; float* z; bf16* dzb; float* rowloss; float* dhpart;
+  float* da1; float* db1part; bf16* w2b; double* red; int32_t* eval_top;
+};
+Ptrs ws_ptrs(char* base, const WsLayout& L);
+
+struct Launch {       // launch bookkeeping of one ctx
+  cudaStream_t s;
+  int64_t* counter;
+  int sms;
+};
+
+// ---------------------------------------------------------------- K-0
+cudaError_t launch_batch_scan(const Launch&, const int32_t* rows, int n, const int64_t* row_ptr,
+                              const int64_t* lab_ptr, int64_t n_data_rows, const Ptrs&,
+                              int64_t nz_cap, int64_t nl_cap);
+cudaError_t launch_touched(const Launch&, const int32_t* rows, int n, const int64_t* row_ptr,
+                           const int32_t* col, const float* val, int64_t F, const Ptrs&,
+                           const WsLayout&, int b_max);
+// ---------------------------------------------------------------- K-1
+cudaError_t launch_spmm_fwd(const Launch&, const int32_t* rows, int n, const int64_t* row_ptr,
+                            const int32_t* col, const float* val, const float* W1, const float* b1,
+                            int H, const Ptrs&, const WsLayout&, bool want_bf16);
+// ---------------------------------------------------------------- K-5
+cudaError_t launch_scatter_sgd(const Launch&, float* W1, int H, float lr, const Ptrs&,
+                               const WsLayout&, float* grad_w1);
+// ---------------------------------------------------------------- dense (fp32 SIMT)
+// C(m,n) = sum_k A(m,k) B(k,n), A(m,k) = A[m*as0 + k*as1], B(k,n) = B[k*bs0 + n*bs1]
+enum GemmEpi { EPI_STORE_BIAS = 0, EPI_SPLITK = 1, EPI_SGD = 2 };
+struct GemmArgs {
+  int M, N, K;
+  const float* A; int64_t as0, as1;
+  const float* B; int64_t bs0, bs1;
+  int epi;
+  float* C; int64_t ldc;          // STORE_BIAS: C[m*ldc+n] = acc + bias[n]
+  const float* bias;
+  int splitk; int64_t part_stride; // SPLITK: C[z*part_stride + m*ldc + n]
+  float lr; float* grad;           // SGD: C[m*ldc+n] -= lr*acc; grad[m*ldc+n] = acc
+  bf16* shadow;                    // SGD: shadow[m*ldc+n] = bf16(new C)
+};
+cudaError_t launch_gemm_f32(const Launch&, const GemmArgs&);
+cudaError_t launch_softmax_ce(const Launch&, int n, int64_t L, const int32_t* rows,
+                              const int64_t* lab_ptr, const int32_t* lab, const Ptrs&,
+                              bool bf16_out);
+cudaError_t launch_dh_reduce(const Launch&, int n, int H, int splitk, const Ptrs&, const WsLayout&);
+cudaError_t launch_b1_update(const Launch&, int n, int H, float* b1, float lr, const Ptrs&,
+                             const WsLayout&, float* grad_b1, float* loss_dev);
+cudaError_t launch_b2_update(const Launch&, int n, int64_t L, float* b2, float lr, const Ptrs&,
+                             bool from_bf16, float* grad_b2);
+cudaError_t launch_to_bf16(const Launch&, const float* src, bf16* dst, int64_t count);
+// ---------------------------------------------------------------- tcgen05 (bf16)
+bool tc_available();
+cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int H, float lr,
+                           const Ptrs&, const WsLayout&, float* W2, const float* b2, float* grad_w2);
+// ---------------------------------------------------------------- merge / eval
+cudaError_t launch_sqnorm(const Launch&, const float* x, int64_t P, double* partials, int nparts,
+                          double* out);
+cudaError_t launch_scale(const Launch&, float* x, int64_t P, double alpha);
+cudaError_t launch_finish(const Launch&, float* params, float* w, float* d, int64_t P, float gamma);
+cudaError_t launch_wsum(const Launch&, const float* const* reps, const double* alpha, int n,
+                        int64_t P, float* out);
+cudaError_t launch_topk(const Launch&, int n, int64_t L, int k, const float* z, int32_t* out);
+cudaError_t launch_validate_csr(const Launch&, const asgd_csr* c, int64_t F, int64_t L, int32_t* err);
+
+}  // namespace asgd

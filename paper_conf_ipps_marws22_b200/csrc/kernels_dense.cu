@@ -1,0 +1,282 @@
+// Dense kernels of the local step (sm_100a), fp32 path and shared epilogues:
+//   G1  Z = H1 W2^T + b2                     (row a4)
+//   softmax-CE: lse, loss, dZ = (softmax(Z) - T)/B   (row a5)
+//   G2  dH1 = dZ W2 (split-K partials), dA1 = dH1 * [A1 > 0], b1 update (rows a6, a7)
+//   G3  W2 -= lr dZ^T H1 (SGD fused into the GEMM epilogue), b2 -= lr 1^T dZ (row a6)
+// Model: PAPER.md P:1525-1531 (§V-A); SGD: P:437-455 (§II); fused element-wise
+// work follows the paper's kernel fusion (§IV).
+// The fp32 contractions here run on CUDA cores (FFMA) so that the fp32 path
+// keeps fp32 products (tolerance 1e-4 vs the fp64 oracle); the bf16 path runs
+// G1-G3 on tcgen05 tensor cores (kernels_tc.cu).
+#include <algorithm>
+
+#include "asgd_internal.h"
+
+namespace asgd {
+namespace {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+// ----------------------------------------------------------------- SIMT GEMM
+constexpr int BM = 64, BN = 64, BK = 16;
+
+__global__ void __launch_bounds__(256) k_gemm_f32(GemmArgs g) {
+  __shared__ float As[BK][BM + 4];
+  __shared__ float Bs[BK][BN + 4];
+  const int t = threadIdx.x, tx = t & 15, ty = t >> 4;
+  const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
+  // split-K range
+  int kc = (g.K + g.splitk - 1) / g.splitk;
+  kc = (kc + BK - 1) / BK * BK;
+  const int kb = blockIdx.z * kc, ke = min(g.K, kb + kc);
+  float acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) acc[i][j] = 0.f;
+  const bool a_kcontig = (g.as1 == 1);
+  const bool b_ncontig = (g.bs1 == 1);
+  for (int k0 = kb; k0 < ke; k0 += BK) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int i = t + 256 * q;
+      int m, k;
+      if (a_kcontig) { k = i & 15; m = i >> 4; } else { m = i & 63; k = i >> 6; }
+      const int gm = m0 + m, gk = k0 + k;
+      As[k][m] = (gm < g.M && gk < ke) ? g.A[(int64_t)gm * g.as0 + (int64_t)gk * g.as1] : 0.f;
+      int n, kk;
+      if (b_ncontig) { n = i & 63; kk = i >> 6; } else { kk = i & 15; n = i >> 4; }
+      const int gn = n0 + n, gk2 = k0 + kk;
+      Bs[kk][n] = (gn < g.N && gk2 < ke) ? g.B[(int64_t)gk2 * g.bs0 + (int64_t)gn * g.bs1] : 0.f;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < BK; ++k) {
+      float a[4], b[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) a[i] = As[k][ty + 16 * i];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) b[j] = Bs[k][tx + 16 * j];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int m = m0 + ty + 16 * i;
+    if (m >= g.M) continue;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int n = n0 + tx + 16 * j;
+      if (n >= g.N) continue;
+      const int64_t o = (int64_t)m * g.ldc + n;
+      if (g.epi == EPI_STORE_BIAS) {
+        g.C[o] = acc[i][j] + (g.bias ? g.bias[n] : 0.f);
+      } else if (g.epi == EPI_SPLITK) {
+        g.C[(int64_t)blockIdx.z * g.part_stride + o] = acc[i][j];
+      } else {  // EPI_SGD
+        const float nw = g.C[o] - g.lr * acc[i][j];
+        g.C[o] = nw;
+        if (g.grad) g.grad[o] = acc[i][j];
+        if (g.shadow) g.shadow[o] = __float2bfloat16_rn(nw);
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------ softmax + CE
+// One CTA per batch row n: lse = log sum_j exp(Z_nj); loss_n = lse - mean_{y in Y_n} Z_ny;
+// dZ_nj = (exp(Z_nj - lse) - T_nj) / B with T_nj = 1/|Y_n| on Y_n (Q3, Q4).
+__global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, const int32_t* __restrict__ rows,
+                                                    const int64_t* __restrict__ lab_ptr,
+                                                    const int32_t* __restrict__ lab, float* Z,
+                                                    bf16* dZb, float* rowloss) {
+  __shared__ int s_lab[kMaxRowLabels];
+  __shared__ float s_lz[kMaxRowLabels];
+  __shared__ float s_m[16], s_s[16];
+  __shared__ float s_lse, s_lsum;
+  const int n = blockIdx.x;
+  const int64_t id = rows[n];
+  const int64_t l0 = lab_ptr[id];
+  const int64_t nl64 = lab_ptr[id + 1] - l0;
+  const int nl = (int)(nl64 < kMaxRowLabels ? nl64 : kMaxRowLabels);
+  float* z = Z + (int64_t)n * L;
+  for (int i = threadIdx.x; i < nl; i += blockDim.x) {
+    int y = lab[l0 + i];
+    s_lab[i] = y;
+    s_lz[i] = z[y];
+  }
+  // pass 1: online max / sum-exp
+  float m = -INFINITY, s = 0.f;
+  for (int64_t j = threadIdx.x; j < L; j += blockDim.x) {
+    const float v = z[j];
+    if (v > m) { s = s * __expf(m - v) + 1.f; m = v; }
+    else s += __expf(v - m);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const float om = __shfl_xor_sync(kFull, m, o), os = __shfl_xor_sync(kFull, s, o);
+    const float nm = fmaxf(m, om);
+    s = (m == -INFINITY ? 0.f : s * __expf(m - nm)) + (om == -INFINITY ? 0.f : os * __expf(om - nm));
+    m = nm;
+  }
+  const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) { s_m[wid] = m; s_s[wid] = s; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float M = -INFINITY, S = 0.f;
+    const int nw = blockDim.x >> 5;
+    for (int w = 0; w < nw; ++w) M = fmaxf(M, s_m[w]);
+    for (int w = 0; w < nw; ++w) S += (s_m[w] == -INFINITY) ? 0.f : s_s[w] * __expf(s_m[w] - M);
+    const float lse = M + logf(S);
+    float ls = 0.f;
+    for (int i = 0; i < nl; ++i) ls += s_lz[i];
+    s_lse = lse;
+    s_lsum = ls;
+    rowloss[n] = lse - ls / (float)nl;
+  }
+  __syncthreads();
+  const float lse = s_lse, invB = 1.f / (float)B;
+  if (dZb) {
+    bf16* d = dZb + (int64_t)n * L;
+    for (int64_t j = threadIdx.x; j < L; j += blockDim.x) d[j] = __float2bfloat16_rn(__expf(z[j] - lse) * invB);
+    __syncthreads();
+    for (int i = threadIdx.x; i < nl; i += blockDim.x)
+      d[s_lab[i]] = __float2bfloat16_rn((__expf(s_lz[i] - lse) - 1.f / (float)nl) * invB);
+  } else {
+    for (int64_t j = threadIdx.x; j < L; j += blockDim.x) z[j] = __expf(z[j] - lse) * invB;
+    __syncthreads();
+    for (int i = threadIdx.x; i < nl; i += blockDim.x)
+      z[s_lab[i]] = (__expf(s_lz[i] - lse) - 1.f / (float)nl) * invB;
+  }
+}
+
+// ------------------------------------------------------ dH1 reduce + ReLU'
+// dA1[r][c] = [H1[r][c] > 0] * sum_z part[z][r][c];  db1 partial per row block.
+constexpr int kRowBlk = 16;
+__global__ void __launch_bounds__(256) k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
+                                                   const float* __restrict__ part,
+                                                   const float* __restrict__ H1, float* dA1,
+                                                   float* db1part) {
+  __shared__ float sp[256];
+  const int cw = min(H, 256);           // columns per pass
+  const int tpc = 256 / cw;             // row groups
+  const int c0 = threadIdx.x % cw, g = threadIdx.x / cw;
+  const int r0 = blockIdx.x * kRowBlk;
+  for (int cb = 0; cb < H; cb += cw) {
+    const int c = cb + c0;
+    float colsum = 0.f;
+    for (int rr = g; rr < kRowBlk; rr += tpc) {
+      const int r = r0 + rr;
+      if (r >= n) break;
+      const int64_t o = (int64_t)r * H + c;
+      float s = 0.f;
+      for (int z = 0; z < splitk; ++z) s += part[z * part_stride + o];
+      const float v = H1[o] > 0.f ? s : 0.f;
+      dA1[o] = v;
+      colsum += v;
+    }
+    sp[threadIdx.x] = colsum;
+    __syncthreads();
+    if (threadIdx.x < cw) {
+      float t = 0.f;
+      for (int q = 0; q < tpc; ++q) t += sp[q * cw + threadIdx.x];
+      db1part[(int64_t)blockIdx.x * H + c] = t;
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void k_b1_update(int n, int H, int nblk, const float* __restrict__ db1part, float* b1,
+                            float lr, float* grad_b1, const float* __restrict__ rowloss,
+                            float* loss_dev) {
+  for (int c = threadIdx.x; c < H; c += blockDim.x) {
+    float s = 0.f;
+    for (int b = 0; b < nblk; ++b) s += db1part[(int64_t)b * H + c];
+    b1[c] -= lr * s;
+    if (grad_b1) grad_b1[c] = s;
+  }
+  if (threadIdx.x == 0 && loss_dev) {
+    float s = 0.f;
+    for (int r = 0; r < n; ++r) s += rowloss[r];
+    *loss_dev = s / (float)n;
+  }
+}
+
+// db2[j] = sum_n dZ[n][j];  b2 -= lr db2
+__global__ void k_b2_update(int n, int64_t L, const float* __restrict__ dz,
+                            const bf16* __restrict__ dzb, float* b2, float lr, float* grad_b2) {
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < L;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    float s = 0.f;
+    if (dzb) for (int r = 0; r < n; ++r) s += __bfloat162float(dzb[(int64_t)r * L + j]);
+    else for (int r = 0; r < n; ++r) s += dz[(int64_t)r * L + j];
+    b2[j] -= lr * s;
+    if (grad_b2) grad_b2[j] = s;
+  }
+}
+
+__global__ void k_to_bf16(const float* __restrict__ src, bf16* dst, int64_t count) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count;
+       i += (int64_t)gridDim.x * blockDim.x)
+    dst[i] = __float2bfloat16_rn(src[i]);
+}
+
+}  // namespace
+
+cudaError_t launch_gemm_f32(const Launch& lc, const GemmArgs& g) {
+  if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaSuccess;
+  dim3 grid((g.N + BN - 1) / BN, (g.M + BM - 1) / BM, g.splitk);
+  k_gemm_f32<<<grid, 256, 0, lc.s>>>(g);
+  ++*lc.counter;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_softmax_ce(const Launch& lc, int n, int64_t L, const int32_t* rows,
+                              const int64_t* lab_ptr, const int32_t* lab, const Ptrs& P,
+                              bool bf16_out) {
+  k_softmax_ce<<<n, 512, 0, lc.s>>>(n, L, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
+                                    P.rowloss);
+  ++*lc.counter;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_dh_reduce(const Launch& lc, int n, int H, int splitk, const Ptrs& P,
+                             const WsLayout& L) {
+  const int nblk = (n + kRowBlk - 1) / kRowBlk;
+  // split-K partial z of dH1 lives at dhpart + z * (b_max * H)
+  k_dh_reduce<<<nblk, 256, 0, lc.s>>>(n, H, splitk, L.part_stride, P.dhpart, P.h1, P.da1,
+                                      P.db1part);
+  ++*lc.counter;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_b1_update(const Launch& lc, int n, int H, float* b1, float lr, const Ptrs& P,
+                             const WsLayout& L, float* grad_b1, float* loss_dev) {
+  const int nblk = (n + kRowBlk - 1) / kRowBlk;
+  k_b1_update<<<1, 512, 0, lc.s>>>(n, H, nblk, P.db1part, b1, lr, grad_b1, P.rowloss, loss_dev);
+  ++*lc.counter;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_b2_update(const Launch& lc, int n, int64_t L, float* b2, float lr, const Ptrs& P,
+                             bool from_bf16, float* grad_b2) {
+  const int64_t blocks = std::min<int64_t>((L + 255) / 256, (int64_t)lc.sms * 16);
+  k_b2_update<<<(int)blocks, 256, 0, lc.s>>>(n, L, P.z, from_bf16 ? P.dzb : nullptr, b2, lr, grad_b2);
+  ++*lc.counter;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_to_bf16(const Launch& lc, const float* src, bf16* dst, int64_t count) {
+  const int64_t blocks = std::min<int64_t>((count + 255) / 256, (int64_t)lc.sms * 16);
+  k_to_bf16<<<(int)std::max<int64_t>(blocks, 1), 256, 0, lc.s>>>(src, dst, count);
+  ++*lc.counter;
+  return cudaGetLastError();
+}
+
+int row_block() { return kRowBlk; }
+
+}  // namespace asgd

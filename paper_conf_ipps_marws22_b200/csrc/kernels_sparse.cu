@@ -1,0 +1,659 @@
+// Sparse kernels of the local step (sm_100a):
+//   K-0  batch CSR view + touched-feature set (rows a2 of DESIGN.md),
+//   K-1  CSR SpMM forward A1 = X W1 + b1, H1 = ReLU(A1)   (row a3),
+//   K-5  scatter-SGD  W1[f,:] -= lr sum_n X_nf dA1[n,:]     (row a8).
+// The first layer is X (B x F, CSR) times W1 (F x H)
+// (§V-A) with the sparse algebra the paper ran through cuSPARSE
+// (P:1503-1506); its cost tracks the batch's nnz, so both K-1 and
+// K-5 split the batch's nnz into fixed pieces of kPiece entries (one warp
+// each) instead of one warp per row / per feature: a skewed row (Wiki10-shaped
+// rows reach 10^4 nnz) spans many warps.  Segments spanning pieces are
+// combined by the last-arriving warp in piece order, so every sum has a
+// fixed order: results are bitwise deterministic.
+#include "asgd_internal.h"
+
+namespace asgd {
+
+namespace {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+__device__ __forceinline__ int entry_row(const int32_t* sboff, int n, int e) {
+  // largest r in [0, n) with sboff[r] <= e (rows may be empty)
+  int lo = 0, hi = n;          // invariant: answer in [lo, hi)
+  while (hi - lo > 1) {
+    int mid = (lo + hi) >> 1;
+    if (sboff[mid] <= e) lo = mid; else hi = mid;
+  }
+  // skip empty rows that share the offset
+  while (lo + 1 < n && sboff[lo + 1] <= e) ++lo;
+  return lo;
+}
+
+// lane <-> column map of a row of H = 32 * VPL floats
+template <int VPL>
+struct RowIO {
+  __device__ __forceinline__ static int col(int lane, int i) {
+    if constexpr (VPL == 2) return 2 * lane + i;
+    else return (i >> 2) * 128 + 4 * lane + (i & 3);
+  }
+  __device__ __forceinline__ static void load_ldg(const float* row, int lane, float (&v)[VPL]) {
+    if constexpr (VPL == 2) {
+      float2 t = __ldg(reinterpret_cast<const float2*>(row) + lane);
+      v[0] = t.x; v[1] = t.y;
+    } else {
+#pragma unroll
+      for (int j = 0; j < VPL / 4; ++j) {
+        float4 t = __ldg(reinterpret_cast<const float4*>(row + j * 128) + lane);
+        v[4 * j] = t.x; v[4 * j + 1] = t.y; v[4 * j + 2] = t.z; v[4 * j + 3] = t.w;
+      }
+    }
+  }
+  __device__ __forceinline__ static void load_cg(const float* row, int lane, float (&v)[VPL]) {
+    if constexpr (VPL == 2) {
+      float2 t = __ldcg(reinterpret_cast<const float2*>(row) + lane);
+      v[0] = t.x; v[1] = t.y;
+    } else {
+#pragma unroll
+      for (int j = 0; j < VPL / 4; ++j) {
+        float4 t = __ldcg(reinterpret_cast<const float4*>(row + j * 128) + lane);
+        v[4 * j] = t.x; v[4 * j + 1] = t.y; v[4 * j + 2] = t.z; v[4 * j + 3] = t.w;
+      }
+    }
+  }
+  __device__ __forceinline__ static void load(const float* row, int lane, float (&v)[VPL]) {
+    if constexpr (VPL == 2) {
+      float2 t = reinterpret_cast<const float2*>(row)[lane];
+      v[0] = t.x; v[1] = t.y;
+    } else {
+#pragma unroll
+      for (int j = 0; j < VPL / 4; ++j) {
+        float4 t = reinterpret_cast<const float4*>(row + j * 128)[lane];
+        v[4 * j] = t.x; v[4 * j + 1] = t.y; v[4 * j + 2] = t.z; v[4 * j + 3] = t.w;
+      }
+    }
+  }
+  __device__ __forceinline__ static void store(float* row, int lane, const float (&v)[VPL]) {
+    if constexpr (VPL == 2) {
+      reinterpret_cast<float2*>(row)[lane] = make_float2(v[0], v[1]);
+    } else {
+#pragma unroll
+      for (int j = 0; j < VPL / 4; ++j)
+        reinterpret_cast<float4*>(row + j * 128)[lane] =
+            make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
+    }
+  }
+  __device__ __forceinline__ static void store_cg(float* row, int lane, const float (&v)[VPL]) {
+    if constexpr (VPL == 2) {
+      __stcg(reinterpret_cast<float2*>(row) + lane, make_float2(v[0], v[1]));
+    } else {
+#pragma unroll
+      for (int j = 0; j < VPL / 4; ++j)
+        __stcg(reinterpret_cast<float4*>(row + j * 128) + lane,
+               make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]));
+    }
+  }
+  __device__ __forceinline__ static void store_bf16(bf16* row, int lane, const float (&v)[VPL]) {
+    if constexpr (VPL == 2) {
+      reinterpret_cast<__nv_bfloat162*>(row)[lane] = __floats2bfloat162_rn(v[0], v[1]);
+    } else {
+#pragma unroll
+      for (int j = 0; j < VPL / 4; ++j) {
+        __nv_bfloat162 a = __floats2bfloat162_rn(v[4 * j], v[4 * j + 1]);
+        __nv_bfloat162 b = __floats2bfloat162_rn(v[4 * j + 2], v[4 * j + 3]);
+        uint2 pk;
+        pk.x = *reinterpret_cast<uint32_t*>(&a);
+        pk.y = *reinterpret_cast<uint32_t*>(&b);
+        reinterpret_cast<uint2*>(row + j * 128)[lane] = pk;
+      }
+    }
+  }
+};
+
+// -------------------------------------------------------------------------
+// K-0 (a): per-row entry / label offsets of the batch (one CTA, exclusive scan)
+// -------------------------------------------------------------------------
+__global__ void __launch_bounds__(1024) k_batch_scan(const int32_t* __restrict__ rows, int n,
+                                                     const int64_t* __restrict__ row_ptr,
+                                                     const int64_t* __restrict__ lab_ptr,
+                                                     int64_t n_data_rows, int32_t* boff,
+                                                     int32_t* loff, int32_t* meta, int64_t nz_cap,
+                                                     int64_t nl_cap) {
+  __shared__ long long wf[32], wl[32];
+  const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
+  const int per = (n + blockDim.x - 1) / blockDim.x;
+  const int r0 = min(n, t * per), r1 = min(n, r0 + per);
+  long long sf = 0, sl = 0;
+  int bad = 0;
+  for (int r = r0; r < r1; ++r) {
+    int64_t id = rows[r];
+    if (id < 0 || id >= n_data_rows) { bad = 1; continue; }
+    sf += row_ptr[id + 1] - row_ptr[id];
+    sl += lab_ptr[id + 1] - lab_ptr[id];
+  }
+  // inclusive warp scan
+  long long xf = sf, xl = sl;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    long long yf = __shfl_up_sync(kFull, xf, o), yl = __shfl_up_sync(kFull, xl, o);
+    if (lane >= o) { xf += yf; xl += yl; }
+  }
+  if (lane == 31) { wf[wid] = xf; wl[wid] = xl; }
+  __syncthreads();
+  if (wid == 0) {
+    long long a = lane < (int)(blockDim.x >> 5) ? wf[lane] : 0;
+    long long b = lane < (int)(blockDim.x >> 5) ? wl[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      long long ya = __shfl_up_sync(kFull, a, o), yb = __shfl_up_sync(kFull, b, o);
+      if (lane >= o) { a += ya; b += yb; }
+    }
+    wf[lane] = a; wl[lane] = b;
+  }
+  __syncthreads();
+  long long pf = xf - sf + (wid ? wf[wid - 1] : 0);
+  long long pl = xl - sl + (wid ? wl[wid - 1] : 0);
+  for (int r = r0; r < r1; ++r) {
+    boff[r] = (int32_t)min(pf, (long long)nz_cap);
+    loff[r] = (int32_t)min(pl, (long long)nl_cap);
+    int64_t id = rows[r];
+    if (id < 0 || id >= n_data_rows) continue;
+    pf += row_ptr[id + 1] - row_ptr[id];
+    pl += lab_ptr[id + 1] - lab_ptr[id];
+  }
+  if (bad) atomicOr(&meta[M_ERR], ERR_ROW_ID);
+  if (t == blockDim.x - 1) {
+    long long tf = wf[(blockDim.x >> 5) - 1], tl = wl[(blockDim.x >> 5) - 1];
+    int err = 0;
+    if (tf > nz_cap) { err |= ERR_NNZ_CAP; tf = nz_cap; }
+    if (tl > nl_cap) { err |= ERR_LAB_CAP; tl = nl_cap; }
+    boff[n] = (int32_t)tf;
+    loff[n] = (int32_t)tl;
+    meta[M_NNZ] = (int32_t)tf;
+    meta[M_NLAB] = (int32_t)tl;
+    meta[M_NROWS] = n;
+    if (err) atomicOr(&meta[M_ERR], err);
+  }
+}
+
+// map a flat batch entry e to its dataset index; returns row in *r
+__device__ __forceinline__ int64_t entry_index(const int32_t* sboff, int n,
+                                               const int32_t* __restrict__ rows,
+                                               const int64_t* __restrict__ row_ptr, int e, int* r) {
+  int rr = entry_row(sboff, n, e);
+  *r = rr;
+  return row_ptr[rows[rr]] + (e - sboff[rr]);
+}
+
+__device__ __forceinline__ void load_boff(int32_t* sboff, const int32_t* boff, int n) {
+  for (int i = threadIdx.x; i <= n; i += blockDim.x) sboff[i] = boff[i];
+  __syncthreads();
+}
+
+// K-0 (b): cnt[f] += 1 for every batch entry
+__global__ void k_count(const int32_t* __restrict__ rows, int n, const int64_t* __restrict__ row_ptr,
+                        const int32_t* __restrict__ col, const int32_t* __restrict__ boff,
+                        const int32_t* __restrict__ meta, int32_t* cnt) {
+  extern __shared__ int32_t sboff[];
+  load_boff(sboff, boff, n);
+  const int nnz = meta[M_NNZ];
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x) {
+    int r;
+    int64_t k = entry_index(sboff, n, rows, row_ptr, e, &r);
+    atomicAdd(&cnt[col[k]], 1);
+  }
+}
+
+// K-0 (c): touched-feature scan over F in tiles: tsum[2t] = sum cnt, tsum[2t+1] = #touched
+__global__ void __launch_bounds__(256) k_fscan_tile(const int32_t* __restrict__ cnt, int64_t F,
+                                                    int32_t* tsum) {
+  __shared__ int s0[8], s1[8];
+  const int64_t base = (int64_t)blockIdx.x * kScanTile;
+  int a = 0, b = 0;
+  for (int i = threadIdx.x; i < kScanTile; i += 256) {
+    int64_t f = base + i;
+    if (f < F) { int c = cnt[f]; a += c; b += (c > 0); }
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) { a += __shfl_xor_sync(kFull, a, o); b += __shfl_xor_sync(kFull, b, o); }
+  if ((threadIdx.x & 31) == 0) { s0[threadIdx.x >> 5] = a; s1[threadIdx.x >> 5] = b; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int x = 0, y = 0;
+    for (int w = 0; w < 8; ++w) { x += s0[w]; y += s1[w]; }
+    tsum[2 * blockIdx.x] = x;
+    tsum[2 * blockIdx.x + 1] = y;
+  }
+}
+
+// exclusive scan of the tile sums (one CTA, sequential over <= a few thousand tiles)
+__global__ void k_fscan_top(const int32_t* __restrict__ tsum, int ntiles, int32_t* tpre,
+                            int32_t* meta) {
+  __shared__ int sa[1024], sb[1024];
+  // each thread owns a contiguous chunk of tiles
+  const int t = threadIdx.x, per = (ntiles + blockDim.x - 1) / blockDim.x;
+  const int i0 = min(ntiles, t * per), i1 = min(ntiles, i0 + per);
+  int a = 0, b = 0;
+  for (int i = i0; i < i1; ++i) { a += tsum[2 * i]; b += tsum[2 * i + 1]; }
+  sa[t] = a; sb[t] = b;
+  __syncthreads();
+  if (t == 0) {
+    int x = 0, y = 0;
+    for (int j = 0; j < (int)blockDim.x; ++j) {
+      int ta = sa[j], tb = sb[j];
+      sa[j] = x; sb[j] = y;
+      x += ta; y += tb;
+    }
+    meta[M_U] = y;
+  }
+  __syncthreads();
+  a = sa[t]; b = sb[t];
+  for (int i = i0; i < i1; ++i) {
+    tpre[2 * i] = a; tpre[2 * i + 1] = b;
+    a += tsum[2 * i]; b += tsum[2 * i + 1];
+  }
+}
+
+// K-0 (d): write segment starts / unique ids
+__global__ void __launch_bounds__(256) k_fscan_write(const int32_t* __restrict__ cnt, int64_t F,
+                                                     const int32_t* __restrict__ tpre,
+                                                     const int32_t* __restrict__ meta,
+                                                     int32_t* fseg, int32_t* fuid, int32_t* uniq,
+                                                     int32_t* useg) {
+  // each thread scans 16 consecutive features; block scan of the thread sums
+  constexpr int PER = kScanTile / 256;
+  __shared__ int sa[256], sb[256];
+  const int64_t f0 = (int64_t)blockIdx.x * kScanTile + threadIdx.x * PER;
+  int c[PER];
+  int a = 0, b = 0;
+#pragma unroll
+  for (int i = 0; i < PER; ++i) {
+    c[i] = (f0 + i < F) ? cnt[f0 + i] : 0;
+    a += c[i]; b += (c[i] > 0);
+  }
+  sa[threadIdx.x] = a; sb[threadIdx.x] = b;
+  __syncthreads();
+  // Hillis-Steele inclusive scan over 256 entries
+  for (int o = 1; o < 256; o <<= 1) {
+    int xa = threadIdx.x >= o ? sa[threadIdx.x - o] : 0;
+    int xb = threadIdx.x >= o ? sb[threadIdx.x - o] : 0;
+    __syncthreads();
+    sa[threadIdx.x] += xa; sb[threadIdx.x] += xb;
+    __syncthreads();
+  }
+  int pa = tpre[2 * blockIdx.x] + sa[threadIdx.x] - a;
+  int pb = tpre[2 * blockIdx.x + 1] + sb[threadIdx.x] - b;
+#pragma unroll
+  for (int i = 0; i < PER; ++i) {
+    if (c[i] > 0) {
+      fseg[f0 + i] = pa;
+      fuid[f0 + i] = pb;
+      uniq[pb] = (int32_t)(f0 + i);
+      useg[pb] = pa;
+      ++pb;
+    }
+    pa += c[i];
+  }
+  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) useg[meta[M_U]] = meta[M_NNZ];
+}
+
+// K-0 (e): scatter entries into their feature segment (cnt returns to zero)
+__global__ void k_place(const int32_t* __restrict__ rows, int n, const int64_t* __restrict__ row_ptr,
+                        const int32_t* __restrict__ col, const float* __restrict__ val,
+                        const int32_t* __restrict__ boff, const int32_t* __restrict__ meta,
+                        int32_t* cnt, const int32_t* __restrict__ fseg,
+                        const int32_t* __restrict__ fuid, int32_t* e_n, float* e_v, int32_t* e_u) {
+  extern __shared__ int32_t sboff[];
+  load_boff(sboff, boff, n);
+  const int nnz = meta[M_NNZ];
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x) {
+    int r;
+    int64_t k = entry_index(sboff, n, rows, row_ptr, e, &r);
+    int f = col[k];
+    int pos = fseg[f] + atomicSub(&cnt[f], 1) - 1;
+    e_n[pos] = r;
+    e_v[pos] = val[k];
+    e_u[pos] = fuid[f];
+  }
+}
+
+// K-0 (f): order every segment by batch row (deterministic summation order).
+// Row ids inside a segment are distinct (cols are unique within a row).
+__global__ void k_segsort(const int32_t* __restrict__ useg, const int32_t* __restrict__ meta,
+                          int32_t* e_n, float* e_v, int words) {
+  extern __shared__ uint32_t sm[];
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  uint32_t* bm = sm + (size_t)wib * words * 33;
+  float* vb = reinterpret_cast<float*>(bm + words);
+  const int U = meta[M_U];
+  const int nw = gridDim.x * (blockDim.x >> 5);
+  for (int w = lane; w < words; w += 32) bm[w] = 0;
+  __syncwarp();
+  for (int u = blockIdx.x * (blockDim.x >> 5) + wib; u < U; u += nw) {
+    const int s = useg[u], m = useg[u + 1] - s;
+    if (m <= 1) continue;
+    if (m <= 32) {
+      int myn = lane < m ? e_n[s + lane] : 0x7fffffff;
+      float myv = lane < m ? e_v[s + lane] : 0.f;
+      int rank = 0;
+#pragma unroll
+      for (int j = 0; j < 32; ++j) rank += (__shfl_sync(kFull, myn, j) < myn);
+      __syncwarp();
+      if (lane < m) { e_n[s + rank] = myn; e_v[s + rank] = myv; }
+      __syncwarp();
+    } else {
+      for (int i = lane; i < m; i += 32) {
+        int r = e_n[s + i];
+        vb[r] = e_v[s + i];
+        atomicOr(&bm[r >> 5], 1u << (r & 31));
+      }
+      __syncwarp();
+      // words per lane
+      const int wpl = (words + 31) / 32;
+      const int w0 = lane * wpl;
+      int cntl = 0;
+      for (int j = 0; j < wpl; ++j) if (w0 + j < words) cntl += __popc(bm[w0 + j]);
+      int incl = cntl;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        int y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+      }
+      int pos = s + incl - cntl;
+      for (int j = 0; j < wpl; ++j) {
+        if (w0 + j >= words) break;
+        uint32_t bits = bm[w0 + j];
+        while (bits) {
+          int b = __ffs(bits) - 1;
+          bits &= bits - 1;
+          int r = (w0 + j) * 32 + b;
+          e_n[pos] = r;
+          e_v[pos] = vb[r];
+          ++pos;
+        }
+        bm[w0 + j] = 0;
+      }
+      __syncwarp();
+    }
+  }
+}
+
+// -------------------------------------------------------------------------
+// K-1: A1 = X W1 + b1, H1 = ReLU(A1)
+// -------------------------------------------------------------------------
+template <int VPL>
+__global__ void __launch_bounds__(256) k_spmm_fwd(const int32_t* __restrict__ rows, int n,
+                                                  const int64_t* __restrict__ row_ptr,
+                                                  const int32_t* __restrict__ col,
+                                                  const float* __restrict__ val,
+                                                  const float* __restrict__ W1,
+                                                  const float* __restrict__ b1,
+                                                  const int32_t* __restrict__ boff,
+                                                  const int32_t* __restrict__ meta, float* H1,
+                                                  bf16* H1b, float* part, int32_t* rowcnt) {
+  using IO = RowIO<VPL>;
+  constexpr int H = 32 * VPL;
+  extern __shared__ int32_t sboff[];
+  load_boff(sboff, boff, n);
+  const int lane = threadIdx.x & 31;
+  const int nnz = meta[M_NNZ];
+  const int npieces = (nnz + kPiece - 1) / kPiece;
+  const int nwarps = gridDim.x * (blockDim.x >> 5);
+  float bias[VPL];
+  IO::load_ldg(b1, lane, bias);
+
+  for (int p = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); p < npieces; p += nwarps) {
+    const int e0 = p * kPiece, e1 = min(e0 + kPiece, nnz);
+    int r = entry_row(sboff, n, e0);
+    int e = e0;
+    while (e < e1) {
+      const int rs = sboff[r], re = sboff[r + 1];
+      const int se = min(re, e1);
+      float acc[VPL];
+#pragma unroll
+      for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+      const int64_t base = row_ptr[rows[r]] - rs;   // dataset index of flat entry e: base + e
+      const int cnt = se - e;                        // <= kPiece = 32
+      int mycol = 0;
+      float myval = 0.f;
+      if (lane < cnt) { mycol = __ldg(col + base + e + lane); myval = __ldg(val + base + e + lane); }
+      int j = 0;
+      for (; j + 4 <= cnt; j += 4) {
+        float w[4][VPL];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          int c = __shfl_sync(kFull, mycol, j + q);
+          IO::load_ldg(W1 + (int64_t)c * H, lane, w[q]);
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          float v = __shfl_sync(kFull, myval, j + q);
+#pragma unroll
+          for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, w[q][i], acc[i]);
+        }
+      }
+      for (; j < cnt; ++j) {
+        int c = __shfl_sync(kFull, mycol, j);
+        float v = __shfl_sync(kFull, myval, j);
+        float w[VPL];
+        IO::load_ldg(W1 + (int64_t)c * H, lane, w);
+#pragma unroll
+        for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, w[i], acc[i]);
+      }
+      const bool before = rs < e0, after = re > e1;
+      bool finish = !before && !after;
+      if (!finish) {
+        const int slot = before ? 2 * p : 2 * p + 1;
+        IO::store_cg(part + (int64_t)slot * H, lane, acc);
+        __threadfence();
+        int old = 0;
+        if (lane == 0) old = atomicAdd(&rowcnt[r], 1);
+        old = __shfl_sync(kFull, old, 0);
+        const int q0 = rs / kPiece, q1 = (re - 1) / kPiece;
+        if (old == q1 - q0) {
+          __threadfence();
+#pragma unroll
+          for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+          for (int q = q0; q <= q1; ++q) {
+            float t[VPL];
+            IO::load_cg(part + (int64_t)(q == q0 ? 2 * q + 1 : 2 * q) * H, lane, t);
+#pragma unroll
+            for (int i = 0; i < VPL; ++i) acc[i] += t[i];
+          }
+          if (lane == 0) rowcnt[r] = 0;
+          finish = true;
+        }
+      }
+      if (finish) {
+#pragma unroll
+        for (int i = 0; i < VPL; ++i) acc[i] = fmaxf(acc[i] + bias[i], 0.f);
+        IO::store(H1 + (int64_t)r * H, lane, acc);
+        if (H1b) IO::store_bf16(H1b + (int64_t)r * H, lane, acc);
+      }
+      e = se;
+      ++r;
+    }
+  }
+  // rows without entries: H1 = ReLU(b1)
+  const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  for (int r = gw; r < n; r += nwarps) {
+    if (sboff[r + 1] == sboff[r]) {
+      float acc[VPL];
+#pragma unroll
+      for (int i = 0; i < VPL; ++i) acc[i] = fmaxf(bias[i], 0.f);
+      IO::store(H1 + (int64_t)r * H, lane, acc);
+      if (H1b) IO::store_bf16(H1b + (int64_t)r * H, lane, acc);
+    }
+  }
+}
+
+// -------------------------------------------------------------------------
+// K-5: W1[f,:] -= lr * sum_{entries of f, ascending row} v * dA1[row,:]
+// -------------------------------------------------------------------------
+template <int VPL>
+__global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__ e_n,
+                                                     const float* __restrict__ e_v,
+                                                     const int32_t* __restrict__ e_u,
+                                                     const int32_t* __restrict__ useg,
+                                                     const int32_t* __restrict__ uniq,
+                                                     const int32_t* __restrict__ meta,
+                                                     const float* __restrict__ dA1, float* W1,
+                                                     float lr, float* part, int32_t* ucnt,
+                                                     float* grad_w1) {
+  using IO = RowIO<VPL>;
+  constexpr int H = 32 * VPL;
+  const int lane = threadIdx.x & 31;
+  const int nnz = meta[M_NNZ];
+  const int npieces = (nnz + kPiece - 1) / kPiece;
+  const int nwarps = gridDim.x * (blockDim.x >> 5);
+  for (int p = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); p < npieces; p += nwarps) {
+    const int e0 = p * kPiece, e1 = min(e0 + kPiece, nnz);
+    int myn = 0;
+    float myv = 0.f;
+    if (e0 + lane < e1) { myn = e_n[e0 + lane]; myv = e_v[e0 + lane]; }
+    int u = e_u[e0];
+    int e = e0;
+    while (e < e1) {
+      const int ss = useg[u], se_ = useg[u + 1];
+      const int se = min(se_, e1);
+      float acc[VPL];
+#pragma unroll
+      for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+      int j = e - e0;
+      const int jend = se - e0;
+      for (; j + 4 <= jend; j += 4) {
+        float g[4][VPL];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          int r = __shfl_sync(kFull, myn, j + q);
+          IO::load_ldg(dA1 + (int64_t)r * H, lane, g[q]);
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          float v = __shfl_sync(kFull, myv, j + q);
+#pragma unroll
+          for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, g[q][i], acc[i]);
+        }
+      }
+      for (; j < jend; ++j) {
+        int r = __shfl_sync(kFull, myn, j);
+        float v = __shfl_sync(kFull, myv, j);
+        float g[VPL];
+        IO::load_ldg(dA1 + (int64_t)r * H, lane, g);
+#pragma unroll
+        for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, g[i], acc[i]);
+      }
+      const bool before = ss < e0, after = se_ > e1;
+      bool finish = !before && !after;
+      if (!finish) {
+        const int slot = before ? 2 * p : 2 * p + 1;
+        IO::store_cg(part + (int64_t)slot * H, lane, acc);
+        __threadfence();
+        int old = 0;
+        if (lane == 0) old = atomicAdd(&ucnt[u], 1);
+        old = __shfl_sync(kFull, old, 0);
+        const int q0 = ss / kPiece, q1 = (se_ - 1) / kPiece;
+        if (old == q1 - q0) {
+          __threadfence();
+#pragma unroll
+          for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+          for (int q = q0; q <= q1; ++q) {
+            float t[VPL];
+            IO::load_cg(part + (int64_t)(q == q0 ? 2 * q + 1 : 2 * q) * H, lane, t);
+#pragma unroll
+            for (int i = 0; i < VPL; ++i) acc[i] += t[i];
+          }
+          if (lane == 0) ucnt[u] = 0;
+          finish = true;
+        }
+      }
+      if (finish) {
+        const int64_t f = uniq[u];
+        float w[VPL];
+        IO::load(W1 + f * H, lane, w);
+#pragma unroll
+        for (int i = 0; i < VPL; ++i) w[i] = w[i] - lr * acc[i];
+        IO::store(W1 + f * H, lane, w);
+        if (grad_w1) IO::store(grad_w1 + f * H, lane, acc);
+      }
+      e = se;
+      ++u;
+    }
+  }
+}
+
+template <int VPL>
+cudaError_t spmm_fwd_t(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
+                       const int32_t* col, const float* val, const float* W1, const float* b1,
+                       const Ptrs& P, const WsLayout& L, bool want_bf16) {
+  int grid = lc.sms * 8;
+  size_t smem = (size_t)(n + 1) * sizeof(int32_t);
+  k_spmm_fwd<VPL><<<grid, 256, smem, lc.s>>>(rows, n, row_ptr, col, val, W1, b1, P.boff, P.meta,
+                                             P.h1, want_bf16 ? P.h1b : nullptr, P.part1, P.rowcnt);
+  ++*lc.counter;
+  return cudaGetLastError();
+}
+
+template <int VPL>
+cudaError_t scatter_t(const Launch& lc, float* W1, float lr, const Ptrs& P, float* grad_w1) {
+  int grid = lc.sms * 8;
+  k_scatter_sgd<VPL><<<grid, 256, 0, lc.s>>>(P.e_n, P.e_v, P.e_u, P.useg, P.uniq, P.meta, P.da1,
+                                             W1, lr, P.part5, P.ucnt, grad_w1);
+  ++*lc.counter;
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_batch_scan(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
+                              const int64_t* lab_ptr, int64_t n_data_rows, const Ptrs& P,
+                              int64_t nz_cap, int64_t nl_cap) {
+  k_batch_scan<<<1, 1024, 0, lc.s>>>(rows, n, row_ptr, lab_ptr, n_data_rows, P.boff, P.loff, P.meta,
+                                     nz_cap, nl_cap);
+  ++*lc.counter;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_touched(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
+                           const int32_t* col, const float* val, int64_t F, const Ptrs& P,
+                           const WsLayout& L, int b_max) {
+  const size_t smem = (size_t)(n + 1) * sizeof(int32_t);
+  const int grid = lc.sms * 4;
+  k_count<<<grid, 256, smem, lc.s>>>(rows, n, row_ptr, col, P.boff, P.meta, P.cnt);
+  const int nt = (int)L.n_tiles_f;
+  k_fscan_tile<<<nt, 256, 0, lc.s>>>(P.cnt, F, P.tsum);
+  k_fscan_top<<<1, 1024, 0, lc.s>>>(P.tsum, nt, P.tpre, P.meta);
+  k_fscan_write<<<nt, 256, 0, lc.s>>>(P.cnt, F, P.tpre, P.meta, P.fseg, P.fuid, P.uniq, P.useg);
+  k_place<<<grid, 256, smem, lc.s>>>(rows, n, row_ptr, col, val, P.boff, P.meta, P.cnt, P.fseg,
+                                     P.fuid, P.e_n, P.e_v, P.e_u);
+  const int words = (b_max + 31) / 32;
+  const size_t ssmem = (size_t)8 * words * 33 * sizeof(uint32_t);
+  k_segsort<<<lc.sms * 2, 256, ssmem, lc.s>>>(P.useg, P.meta, P.e_n, P.e_v, words);
+  *lc.counter += 6;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_spmm_fwd(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
+                            const int32_t* col, const float* val, const float* W1, const float* b1,
+                            int H, const Ptrs& P, const WsLayout& L, bool want_bf16) {
+  switch (H) {
+    case 64: return spmm_fwd_t<2>(lc, rows, n, row_ptr, col, val, W1, b1, P, L, want_bf16);
+    case 128: return spmm_fwd_t<4>(lc, rows, n, row_ptr, col, val, W1, b1, P, L, want_bf16);
+    case 256: return spmm_fwd_t<8>(lc, rows, n, row_ptr, col, val, W1, b1, P, L, want_bf16);
+    case 512: return spmm_fwd_t<16>(lc, rows, n, row_ptr, col, val, W1, b1, P, L, want_bf16);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+cudaError_t launch_scatter_sgd(const Launch& lc, float* W1, int H, float lr, const Ptrs& P,
+                               const WsLayout& L, float* grad_w1) {
+  switch (H) {
+    case 64: return scatter_t<2>(lc, W1, lr, P, grad_w1);
+    case 128: return scatter_t<4>(lc, W1, lr, P, grad_w1);
+    case 256: return scatter_t<8>(lc, W1, lr, P, grad_w1);
+    case 512: return scatter_t<16>(lc, W1, lr, P, grad_w1);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace asgd

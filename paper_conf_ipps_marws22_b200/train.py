@@ -1,0 +1,207 @@
+"""Adaptive SGD driver: mega-batches of dynamically routed local steps, then
+the normalized merge and batch size scaling (§III, P:619-1160;
+§IV).
+
+Two drivers over the same libasgd calls:
+  * DistributedAdaptiveSGD -- one process per GPU (torch.distributed); batches
+    come from the cross-process shm ticket scheduler; the merge is prescale
+    (K-6) -> one all-reduce SUM (NCCL over NVLink) -> momentum epilogue (K-7).
+  * SimulatedAdaptiveSGD -- N replicas on one GPU, routed by the simulated
+    clock (or replayed); the all-reduce is replaced by the in-device weighted
+    sum (the parity configuration of BASELINE.json configs[0]).
+The host logic that sits between the kernels (ticket loop, statistics
+exchange + Alg. 2 weights, Alg. 1) is written device-agnostic so the gloo CPU
+tests exercise it unchanged.
+"""
+from __future__ import annotations
+
+import dataclasses
+import math
+from typing import Callable, List, Optional, Sequence
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+from . import api
+
+
+@dataclasses.dataclass
+class Hyper:
+    b_max: int
+    b_min: int
+    beta: int
+    lr_max: float
+    M: int                      # mega-batch samples (Q8)
+    gamma: float = 0.9
+    delta: float = 0.1
+    pert_thr: float = 0.1
+    pert_renorm: bool = False   # Q34 option (literal Alg. 2 by default)
+
+    @classmethod
+    def from_config(cls, cfg, **kw):
+        h = dict(b_max=cfg.b_max, b_min=cfg.b_min, beta=cfg.beta, lr_max=cfg.lr_max, M=cfg.mega_batch)
+        h.update(kw)
+        return cls(**h)
+
+
+@dataclasses.dataclass
+class MegaBatchStats:
+    mb: int
+    u: List[int]
+    b: List[int]
+    lr: List[float]
+    nu: List[float]
+    alpha: List[float]
+    r: int
+    s: int
+    perturbed: bool
+    routes: list
+    n_steps: int
+
+
+# --------------------------------------------------------------- host logic
+def run_tickets(sched: api.Scheduler, rank: int, b_i: int,
+                step: Callable[[int, int, int], None], inflight: int = 2,
+                wait: Optional[Callable[[int], None]] = None) -> int:
+    """Take tickets until the mega-batch is exhausted.
+
+    step(k, start, len) enqueues local step k; wait(k) blocks until step k
+    finished.  With inflight = 1 a rank asks for its next batch only after
+    its previous step completed (paper-faithful); inflight = 2 lets the host
+    take the next ticket while one step is still running (reading Q32)."""
+    k = 0
+    while True:
+        if wait is not None and k >= inflight:
+            wait(k - inflight)
+        t = sched.next(rank, b_i)
+        if t is None:
+            return k
+        step(k, t[0], t[1])
+        k += 1
+
+
+def exchange_stats(u: int, b: int, sqnorm: torch.Tensor, P: int, world: int,
+                   group=None):
+    """All-gather (u_i, b_i, ||w_i||^2) and return host lists + nu = ||w||_2 / P.
+
+    sqnorm: fp64 scalar tensor on the collective's device."""
+    dev = sqnorm.device
+    mine = torch.stack([torch.tensor(float(u), dtype=torch.float64, device=dev),
+                        torch.tensor(float(b), dtype=torch.float64, device=dev),
+                        sqnorm.reshape(())])
+    if world > 1:
+        allv = [torch.empty_like(mine) for _ in range(world)]
+        dist.all_gather(allv, mine, group=group)
+        allv = torch.stack(allv).cpu().numpy()
+    else:
+        allv = mine.reshape(1, 3).cpu().numpy()
+    us = [int(round(x)) for x in allv[:, 0]]
+    bs = [int(round(x)) for x in allv[:, 1]]
+    nu = [math.sqrt(float(x)) / P for x in allv[:, 2]]
+    return us, bs, nu
+
+
+# --------------------------------------------------------------- drivers
+class DistributedAdaptiveSGD:
+    """Rank `rank` of `world` (one GPU each)."""
+
+    def __init__(self, replica: api.Replica, hyper: Hyper, rank: int, world: int,
+                 sched: api.Scheduler, group=None, inflight: int = 2):
+        self.rep, self.h, self.rank, self.world = replica, hyper, rank, world
+        self.sched, self.group, self.inflight = sched, group, inflight
+        self.b = [hyper.b_max] * world            # initial b = b_max
+        self.lr = [hyper.lr_max] * world
+        dev = replica.device
+        cap = hyper.M // max(1, hyper.b_min) + 2
+        self.losses = torch.zeros(cap, dtype=torch.float32, device=dev)
+        self.sq = torch.zeros(1, dtype=torch.float64, device=dev)
+        self.events = [torch.cuda.Event() for _ in range(cap)]
+        self.mb = 0
+
+    def megabatch(self, stream_rows: torch.Tensor, keep_log: bool = False) -> MegaBatchStats:
+        """One mega-batch over the M sample ids stream_rows (device int32)."""
+        rep, h, r = self.rep, self.h, self.rank
+        self.sched.wait(self.mb)
+        b_i, lr_i = self.b[r], self.lr[r]
+
+        def step(k, start, n):
+            rep.step(stream_rows[start:start + n], lr_i, self.losses[k:k + 1])
+            self.events[k].record(rep.stream)
+
+        n_steps = run_tickets(self.sched, r, b_i, step, self.inflight,
+                              wait=lambda k: self.events[k].synchronize())
+        # ---- merge (Alg. 2) -------------------------------------------------
+        rep.sqnorm(self.sq)
+        us, bs, nu = exchange_stats(n_steps, b_i, self.sq, rep.P, self.world, self.group)
+        routes = self.sched.log() if keep_log and r == 0 else []
+        if r == 0:
+            self.sched.reset(self.mb + 1)        # every rank is past its tickets
+        alpha, rr, ss, pert = api.merge_weights(us, bs, nu, h.pert_thr, h.delta, h.pert_renorm)
+        rep.prescale(alpha[r])
+        if self.world > 1:
+            dist.all_reduce(rep.params, op=dist.ReduceOp.SUM, group=self.group)
+        rep.finish(h.gamma)
+        # ---- Alg. 1 ----------------------------------------------------------
+        lr_used = list(self.lr)
+        self.b, self.lr = api.scale_batches(us, bs, h.b_min, h.b_max, h.beta, h.lr_max)
+        st = MegaBatchStats(self.mb, us, bs, lr_used, nu, alpha, rr, ss, pert, routes, n_steps)
+        self.mb += 1
+        return st
+
+
+class SimulatedAdaptiveSGD:
+    """N replicas on one GPU; routing by the simulated clock (Q10) or replay."""
+
+    def __init__(self, replicas: Sequence[api.Replica], hyper: Hyper, row_nnz: np.ndarray,
+                 cost_factors: Sequence[float], per_row: float = 5.0):
+        self.reps, self.h = list(replicas), hyper
+        self.n = len(self.reps)
+        self.row_nnz = np.asarray(row_nnz, dtype=np.int64)
+        self.cf = list(cost_factors)
+        self.per_row = per_row
+        self.b = [hyper.b_max] * self.n
+        self.lr = [hyper.lr_max] * self.n
+        dev = self.reps[0].device
+        self.sq = torch.zeros(self.n, dtype=torch.float64, device=dev)
+        cap = hyper.M // max(1, hyper.b_min) + 2
+        self.losses = torch.zeros(cap, dtype=torch.float32, device=dev)
+        self.mb = 0
+
+    def megabatch(self, stream_rows: torch.Tensor, stream_ids: np.ndarray,
+                  route_order: Optional[Sequence[int]] = None) -> MegaBatchStats:
+        h = self.h
+        if route_order is not None:
+            routes = api.route_replay(route_order, self.b, h.M)
+        else:
+            routes = api.route_simulate(self.b, h.M, self.cf, self.per_row, self.row_nnz[stream_ids])
+        for k, (r, start, n) in enumerate(routes):
+            self.reps[r].step(stream_rows[start:start + n], self.lr[r], self.losses[k:k + 1])
+        u = [0] * self.n
+        for r, _, _ in routes:
+            u[r] += 1
+        for i, rep in enumerate(self.reps):
+            rep.sqnorm(self.sq[i:i + 1])
+        P = self.reps[0].P
+        nu = [math.sqrt(float(x)) / P for x in self.sq.cpu().numpy()]
+        alpha, rr, ss, pert = api.merge_weights(u, self.b, nu, h.pert_thr, h.delta, h.pert_renorm)
+        r0 = self.reps[0]
+        r0.weighted_sum(self.reps, alpha, r0.params)
+        r0.finish(h.gamma)
+        for rep in self.reps[1:]:
+            rep.params.copy_(r0.params)
+            rep.params_changed()
+        lr_used, b_used = list(self.lr), list(self.b)
+        self.b, self.lr = api.scale_batches(u, self.b, h.b_min, h.b_max, h.beta, h.lr_max)
+        st = MegaBatchStats(self.mb, u, b_used, lr_used, nu, alpha, rr, ss, pert, routes, len(routes))
+        self.mb += 1
+        return st
+
+
+def precision_at_k(replica: api.Replica, test: api.DeviceCsr, test_host, rows: np.ndarray, k: int = 1) -> float:
+    """P@k of the replica's model on test rows (a13; untimed)."""
+    rows_d = torch.as_tensor(np.asarray(rows, dtype=np.int32), device=replica.device)
+    top = replica.eval_topk(test, rows_d, k).cpu().numpy()
+    sub = test_host.row_slice(rows)
+    hits = api.precision_at_k_hits(top, sub.lab_ptr, sub.lab, k)
+    return hits / (k * len(rows))

@@ -1,0 +1,155 @@
+"""C-ABI checks that need no GPU: the library loads, exports every symbol the
+header declares, its host-pure functions agree bit-exactly with the oracle,
+and device entry points fail cleanly (no crash) without a usable GPU."""
+import ctypes as C
+import json
+import os
+import random
+import uuid
+
+import numpy as np
+import pytest
+
+from paper_conf_ipps_marws22_b200 import _lib, api
+from paper_conf_ipps_marws22_b200.build import build
+from oracle import merge, metrics, routing, scaling
+from tests.conftest import GOLDEN
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _built():
+    build()
+
+
+def test_exports_every_header_symbol():
+    syms = _lib.header_symbols()
+    assert len(syms) >= 30
+    L = _lib.lib()
+    missing = [s for s in syms if not hasattr(L, s)]
+    assert not missing, missing
+    assert set(syms) == set(_lib._SIGS), set(syms) ^ set(_lib._SIGS)
+    assert "sm_100a" in api.version()
+
+
+def test_device_entry_points_fail_cleanly_without_gpu():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    desc = _lib.ModelDesc(100, 10, 64, 0, 8, 100, 10)
+    assert _lib.lib().asgd_workspace_bytes(C.byref(desc)) > 0
+    h = C.c_void_p()
+    buf = (C.c_float * 64)()
+    p = C.addressof(buf) + (-C.addressof(buf)) % 16
+    rc = _lib.lib().asgd_replica_init(C.byref(h), C.byref(desc), 0, None, p, p, p, p, 1 << 40)
+    assert rc in (_lib.E_CUDA, _lib.E_UNSUPPORTED)
+    assert _lib.lib().asgd_last_error()
+    # argument validation before any device work
+    rc = _lib.lib().asgd_replica_init(C.byref(h), C.byref(desc), 0, None, p + 4, p, p, p, 1 << 40)
+    assert rc == _lib.E_ARG
+    bad = _lib.ModelDesc(100, 10, 96, 0, 8, 100, 10)
+    rc = _lib.lib().asgd_replica_init(C.byref(h), C.byref(bad), 0, None, p, p, p, p, 1 << 40)
+    assert rc == _lib.E_UNSUPPORTED
+
+
+def _load(name):
+    with open(os.path.join(GOLDEN, name)) as f:
+        return json.load(f)
+
+
+@pytest.mark.parametrize("case", _load("alg2_vectors.json")["cases"])
+def test_merge_weights_golden_bitexact(case):
+    a, r, s, p = api.merge_weights(case["u"], case["b"], case["nu"], 0.1, 0.1)
+    ao, ro, so, po = merge.merge_weights(case["u"], case["b"], case["nu"], 0.1, 0.1)
+    assert a == ao and p == po == case["perturbed"]
+    if p:
+        assert (r, s) == (ro, so)
+
+
+def test_merge_weights_random_bitexact():
+    rng = random.Random(5)
+    for _ in range(3000):
+        n = rng.randint(1, 8)
+        u = [rng.randint(0, 6) for _ in range(n)]
+        if sum(u) == 0:
+            u[0] = 1
+        b = [rng.choice([32, 64, 100, 128]) for _ in range(n)]
+        nu = [rng.choice([0.01, 0.05, 0.2]) for _ in range(n)]
+        renorm = rng.random() < 0.3
+        got = api.merge_weights(u, b, nu, 0.1, 0.1, renorm)
+        want = merge.merge_weights(u, b, nu, 0.1, 0.1, renorm)
+        assert got[0] == want[0] and got[3] == want[3], (u, b, nu)
+        if want[3]:
+            assert got[1:3] == want[1:3]
+
+
+@pytest.mark.parametrize("case", _load("alg1_vectors.json")["cases"])
+def test_scale_batches_golden(case):
+    b, lr = api.scale_batches(case["u"], case["b"], case["b_min"], case["b_max"], case["beta"], 1.0)
+    assert b == case["b_out"]
+    bo, lro = scaling.scale_batches(case["u"], case["b"], case["b_min"], case["b_max"], case["beta"], 1.0)
+    assert lr == lro
+
+
+def test_scale_batches_random_bitexact():
+    rng = random.Random(6)
+    for _ in range(3000):
+        n = rng.randint(1, 8)
+        u = [rng.randint(0, 30) for _ in range(n)]
+        b_max = rng.choice([32, 256, 1024])
+        b_min = b_max // 8
+        beta = rng.choice([b_min // 2, 3, 7])
+        b = [rng.randint(b_min, b_max) for _ in range(n)]
+        lr_max = rng.choice([1.0, 0.1, 0.3])
+        assert api.scale_batches(u, b, b_min, b_max, beta, lr_max) == \
+            tuple(scaling.scale_batches(u, b, b_min, b_max, beta, lr_max))
+
+
+def test_routing_bitexact():
+    g = _load("fig2_routing.json")
+    rng = random.Random(7)
+    for _ in range(300):
+        n = rng.randint(1, 6)
+        b = [rng.randint(1, 40) for _ in range(n)]
+        M = rng.randint(1, 400)
+        row_nnz = np.array([rng.randint(0, 50) for _ in range(M)], dtype=np.int64)
+        cf = [rng.choice([1.0, 1.1, 1.2, 1.32]) for _ in range(n)]
+        got = api.route_simulate(b, M, cf, 5.0, row_nnz)
+        want = routing.simulate(b, M, lambda r, s, l: cf[r] * (float(row_nnz[s:s + l].sum()) + 5.0 * l))
+        assert got == want
+        order = [rr for rr, _, _ in want]
+        assert api.route_replay(order, b, M) == routing.replay(order, b, M)
+    # Fig. 2: per-batch costs via one nnz-free row per batch
+    b = [1, 1]
+    got = api.route_simulate(b, 5, [1.0, 1.5], 1.0, np.zeros(5, dtype=np.int64))
+    assert [r for r, _, _ in got] == g["expected_order"]
+
+
+def test_precision_at_k_matches_oracle():
+    rng = np.random.default_rng(8)
+    Z = rng.integers(0, 4, size=(40, 9)).astype(np.float64)
+    for k in (1, 3, 5):
+        top = metrics.topk(Z, k)
+        lab_ptr = np.arange(0, 81, 2, dtype=np.int64)
+        lab = np.concatenate([np.sort(rng.choice(9, 2, replace=False)) for _ in range(40)]).astype(np.int32)
+        hits = api.precision_at_k_hits(top, lab_ptr, lab, k)
+        assert hits / (k * 40) == metrics.precision_at_k(top, lab_ptr, lab, k)
+
+
+def test_scheduler_single_process():
+    name = "/asgd_t_" + uuid.uuid4().hex[:8]
+    s = api.Scheduler(name, 1, 100, create=True)
+    try:
+        got = []
+        while True:
+            t = s.next(0, 32)
+            if t is None:
+                break
+            got.append(t)
+        assert got == [(0, 32), (32, 32), (64, 32), (96, 4)]
+        assert [(r, st, n) for _, r, st, n in s.log()] == [(0, 0, 32), (0, 32, 32), (0, 64, 32), (0, 96, 4)]
+        s.reset(1)
+        s.wait(1, 10)
+        assert s.next(0, 100) == (0, 100)
+        assert s.next(0, 1) is None
+    finally:
+        s.close()
