@@ -16,6 +16,7 @@ HEADER = os.path.join(_HERE, "..", "include", "asgd.h")
 
 OK, E_ARG, E_SHAPE, E_CUDA, E_STATE, E_UNSUPPORTED = 0, 1, 2, 3, 4, 5
 PREC_FP32, PREC_BF16 = 0, 1
+PROF_NAMES = ["touched", "spmm", "g1", "softmax", "g2", "dh_b1", "b2", "g3", "scatter", "merge"]
 
 
 class ModelDesc(C.Structure):
@@ -68,6 +69,8 @@ _SIGS = {
     "asgd_precision_at_k": (C.c_int, [_P, _P, _P, _i32, _i32, C.POINTER(_i64)]),
     "asgd_sync": (C.c_int, [_P]),
     "asgd_kernel_launches": (C.c_int, [_P, C.POINTER(_i64)]),
+    "asgd_profile": (C.c_int, [_P, _i32]),
+    "asgd_profile_read": (C.c_int, [_P, _P, _P]),
     "asgd_copy_to_host": (C.c_int, [_P, _P, _P, C.c_size_t]),
     "asgd_last_error": (C.c_char_p, []),
     "asgd_version": (C.c_char_p, []),

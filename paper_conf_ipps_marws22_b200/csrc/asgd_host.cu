@@ -151,8 +151,45 @@ struct asgd_ctx {
   int64_t launches;
   int64_t Pn;
   int64_t o_w1, o_b1, o_w2, o_b2;
+  bool prof_on = false;
+  std::vector<cudaEvent_t> pev[ASGD_PROF_N];   // (start, end) pairs
+  size_t pused[ASGD_PROF_N] = {};
   Launch lc() { return Launch{s, &launches, sms}; }
 };
+
+namespace {
+constexpr size_t kMaxProfPairs = 8192;
+
+// Record an event on the ctx stream at the start / end of a kernel-class section.
+void prof_mark(asgd_ctx* c, int cls, bool begin) {
+  if (!c->prof_on) return;
+  auto& v = c->pev[cls];
+  size_t& u = c->pused[cls];
+  if (begin) {
+    if (u >= kMaxProfPairs) return;
+    if (v.size() < 2 * (u + 1)) {
+      cudaEvent_t a, b;
+      if (cudaEventCreate(&a) != cudaSuccess) return;
+      if (cudaEventCreate(&b) != cudaSuccess) { cudaEventDestroy(a); return; }
+      v.push_back(a);
+      v.push_back(b);
+    }
+    cudaEventRecord(v[2 * u], c->s);
+  } else {
+    if (u >= kMaxProfPairs || v.size() < 2 * (u + 1)) return;
+    cudaEventRecord(v[2 * u + 1], c->s);
+    ++u;
+  }
+}
+}  // namespace
+
+#define PCU(cls, call)                                      \
+  do {                                                      \
+    prof_mark(c, cls, true);                                \
+    cudaError_t _e = (call);                                \
+    prof_mark(c, cls, false);                               \
+    if (_e != cudaSuccess) return cuda_fail(_e, #call);     \
+  } while (0)
 
 extern "C" {
 
@@ -222,6 +259,9 @@ int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device, v
 }
 
 int asgd_replica_destroy(asgd_ctx* c) {
+  if (c)
+    for (auto& v : c->pev)
+      for (cudaEvent_t e : v) cudaEventDestroy(e);
   delete c;
   return ASGD_OK;
 }
@@ -295,20 +335,22 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
   float* g = c->dbg;
   if (g) CU(cudaMemsetAsync(g, 0, c->Pn * sizeof(float), c->s));
   // K-0: batch view + touched-feature set
-  CU(launch_batch_scan(lc, rows, n, x.row_ptr, x.lab_ptr, x.n_rows, P, c->L.nz_cap, c->L.nl_cap));
-  CU(launch_touched(lc, rows, n, x.row_ptr, x.col, x.val, m.F, P, c->L, m.b_max));
+  PCU(ASGD_K_TOUCHED, ([&]() -> cudaError_t {
+        cudaError_t e = launch_batch_scan(lc, rows, n, x.row_ptr, x.lab_ptr, x.n_rows, P, c->L.nz_cap,
+                                          c->L.nl_cap);
+        return e != cudaSuccess ? e : launch_touched(lc, rows, n, x.row_ptr, x.col, x.val, m.F, P, c->L, m.b_max);
+      })());
   // K-1
-  CU(launch_spmm_fwd(lc, rows, n, x.row_ptr, x.col, x.val, W1, b1, H, P, c->L, bf));
+  PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, rows, n, x.row_ptr, x.col, x.val, W1, b1, H, P, c->L, bf));
   if (!bf) {
     GemmArgs a{};
     // G1: Z[n x L] = H1 W2^T + b2
-    a = GemmArgs{};
     a.M = n; a.N = (int)Lb; a.K = H;
     a.A = P.h1; a.as0 = H; a.as1 = 1;
     a.B = W2; a.bs0 = 1; a.bs1 = H;
     a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = Lb; a.bias = b2; a.splitk = 1;
-    CU(launch_gemm_f32(lc, a));
-    CU(launch_softmax_ce(lc, n, Lb, rows, x.lab_ptr, x.lab, P, false));
+    PCU(ASGD_K_G1, launch_gemm_f32(lc, a));
+    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, rows, x.lab_ptr, x.lab, P, false));
     // G2: dH1 partials = dZ W2 (pre-step W2)
     a = GemmArgs{};
     a.M = n; a.N = H; a.K = (int)Lb;
@@ -316,15 +358,17 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     a.B = W2; a.bs0 = H; a.bs1 = 1;
     a.epi = EPI_SPLITK; a.C = P.dhpart; a.ldc = H; a.splitk = (int)c->L.splitk;
     a.part_stride = c->L.part_stride;
-    CU(launch_gemm_f32(lc, a));
+    PCU(ASGD_K_G2, launch_gemm_f32(lc, a));
   } else {
-    CU(launch_gemm_tc(lc, 1, n, Lb, H, lr, P, c->L, W2, b2, nullptr));
-    CU(launch_softmax_ce(lc, n, Lb, rows, x.lab_ptr, x.lab, P, true));
-    CU(launch_gemm_tc(lc, 2, n, Lb, H, lr, P, c->L, W2, b2, nullptr));
+    PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, P, c->L, W2, b2, nullptr));
+    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, rows, x.lab_ptr, x.lab, P, true));
+    PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, lr, P, c->L, W2, b2, nullptr));
   }
-  CU(launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L));
-  CU(launch_b1_update(lc, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev));
-  CU(launch_b2_update(lc, n, Lb, b2, lr, P, bf, g ? g + c->o_b2 : nullptr));
+  PCU(ASGD_K_DH, ([&]() -> cudaError_t {
+        cudaError_t e = launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L);
+        return e != cudaSuccess ? e : launch_b1_update(lc, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev);
+      })());
+  PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, b2, lr, P, bf, g ? g + c->o_b2 : nullptr));
   if (!bf) {
     // G3: W2 -= lr dZ^T H1
     GemmArgs a{};
@@ -333,12 +377,12 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     a.B = P.h1; a.bs0 = H; a.bs1 = 1;
     a.epi = EPI_SGD; a.C = W2; a.ldc = H; a.lr = lr; a.grad = g ? g + c->o_w2 : nullptr;
     a.splitk = 1;
-    CU(launch_gemm_f32(lc, a));
+    PCU(ASGD_K_G3, launch_gemm_f32(lc, a));
   } else {
-    CU(launch_gemm_tc(lc, 3, n, Lb, H, lr, P, c->L, W2, b2, g ? g + c->o_w2 : nullptr));
+    PCU(ASGD_K_G3, launch_gemm_tc(lc, 3, n, Lb, H, lr, P, c->L, W2, b2, g ? g + c->o_w2 : nullptr));
   }
   // K-5
-  CU(launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr));
+  PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr));
   ++c->u;
   return ASGD_OK;
 }
@@ -370,19 +414,19 @@ int asgd_last_touched(asgd_ctx* c, int32_t* out, int64_t cap, int64_t* n_out) {
 
 int asgd_replica_sqnorm(asgd_ctx* c, double* out_dev) {
   if (!c || !out_dev) return fail(ASGD_E_ARG, "null argument");
-  CU(launch_sqnorm(c->lc(), c->params, c->Pn, c->P.red, (int)c->L.n_red, out_dev));
+  PCU(ASGD_K_MERGE, launch_sqnorm(c->lc(), c->params, c->Pn, c->P.red, (int)c->L.n_red, out_dev));
   return ASGD_OK;
 }
 
 int asgd_merge_prescale(asgd_ctx* c, double alpha) {
   if (!c) return fail(ASGD_E_ARG, "null ctx");
-  CU(launch_scale(c->lc(), c->params, c->Pn, alpha));
+  PCU(ASGD_K_MERGE, launch_scale(c->lc(), c->params, c->Pn, alpha));
   return ASGD_OK;
 }
 
 int asgd_merge_finish(asgd_ctx* c, float gamma) {
   if (!c) return fail(ASGD_E_ARG, "null ctx");
-  CU(launch_finish(c->lc(), c->params, c->w, c->dd, c->Pn, gamma));
+  PCU(ASGD_K_MERGE, launch_finish(c->lc(), c->params, c->w, c->dd, c->Pn, gamma));
   if (c->d.precision == ASGD_PREC_BF16)
     CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->P.w2b, c->d.L * c->d.H));
   c->u = 0;
@@ -451,6 +495,29 @@ int asgd_sync(asgd_ctx* c) {
 int asgd_kernel_launches(const asgd_ctx* c, int64_t* out) {
   if (!c || !out) return fail(ASGD_E_ARG, "null argument");
   *out = c->launches;
+  return ASGD_OK;
+}
+
+int asgd_profile(asgd_ctx* c, int32_t enable) {
+  if (!c) return fail(ASGD_E_ARG, "null ctx");
+  c->prof_on = enable != 0;
+  for (int k = 0; k < ASGD_PROF_N; ++k) c->pused[k] = 0;
+  return ASGD_OK;
+}
+
+int asgd_profile_read(asgd_ctx* c, double* ms, int64_t* cnt) {
+  if (!c || !ms || !cnt) return fail(ASGD_E_ARG, "null argument");
+  CU(cudaStreamSynchronize(c->s));
+  for (int k = 0; k < ASGD_PROF_N; ++k) {
+    double t = 0.0;
+    for (size_t i = 0; i < c->pused[k]; ++i) {
+      float e = 0.f;
+      CU(cudaEventElapsedTime(&e, c->pev[k][2 * i], c->pev[k][2 * i + 1]));
+      t += e;
+    }
+    ms[k] = t;
+    cnt[k] = (int64_t)c->pused[k];
+  }
   return ASGD_OK;
 }
 

@@ -1,0 +1,94 @@
+"""Parity of the merge kernels and of the whole method on simulated replicas
+(CUDA path vs oracle), plus top-k evaluation."""
+import numpy as np
+import pytest
+import torch
+
+from oracle import adaptive, merge as omerge, metrics, model as omodel
+from synth import config, init_params, sample_stream
+from tests.gpu_helpers import dataset, make_replica, normwise
+
+pytestmark = pytest.mark.gpu
+
+
+def test_sqnorm_prescale_finish():
+    cfg = config("tiny")
+    data = dataset("tiny")
+    rng = np.random.default_rng(0)
+    w0 = init_params(cfg)
+    rep = make_replica(cfg, data, "fp32", w0=w0)
+    x = (w0 + rng.normal(0, 0.01, w0.shape)).astype(np.float32)
+    d0 = rng.normal(0, 0.01, w0.shape).astype(np.float32)
+    rep.params.copy_(torch.from_numpy(x))
+    rep.d.copy_(torch.from_numpy(d0))
+    sq = torch.zeros(1, dtype=torch.float64, device="cuda")
+    rep.sqnorm(sq)
+    rep.sync()
+    ref = float(np.dot(x.astype(np.float64), x.astype(np.float64)))
+    assert abs(sq.item() - ref) <= 1e-12 * ref
+    rep.prescale(0.37)
+    rep.finish(0.9)
+    rep.sync()
+    wn, dn = omerge.merge_models([x], [0.37], w0, d0, 0.9)
+    assert normwise(rep.params.cpu().numpy(), wn) <= 1e-6
+    assert normwise(rep.w.cpu().numpy(), wn) <= 1e-6
+    assert normwise(rep.d.cpu().numpy(), dn) <= 1e-5
+    assert rep.updates() == 0
+
+
+def test_simulated_two_replicas_tiny_trajectory():
+    """BASELINE.json configs[0]: 2 simulated replicas, ~50 steps, free-running."""
+    from paper_conf_ipps_marws22_b200 import api, train
+    cfg = config("tiny")
+    data = dataset("tiny")
+    w0 = init_params(cfg)
+    h = train.Hyper.from_config(cfg)
+    r0 = make_replica(cfg, data, "fp32", w0=w0)
+    r1 = api.Replica(cfg.F, cfg.L, cfg.H, cfg.b_max, r0.desc.max_step_nnz, r0.desc.max_step_labels,
+                     "fp32", w0=w0, share_global=r0)
+    r1.register(r0._keep_data)
+    lens = np.diff(data.row_ptr)
+    cf = [1.0, 1.32]
+    sim = train.SimulatedAdaptiveSGD([r0, r1], h, lens, cf)
+    n_mb = 5
+    stats = []
+    for mb in range(n_mb):
+        ids = sample_stream(cfg, mb * h.M, h.M)
+        stats.append(sim.megabatch(torch.as_tensor(ids, device="cuda"), ids))
+    recs = adaptive.run(cfg.F, cfg.H, cfg.L, data, w0, lambda mb: sample_stream(cfg, mb * h.M, h.M),
+                        n_rep=2, n_mb=n_mb, M=h.M, b_max=h.b_max, b_min=h.b_min, beta=h.beta,
+                        lr_max=h.lr_max, cost_factors=cf)
+    for st, rec in zip(stats, recs):
+        assert [tuple(x) for x in st.routes] == [tuple(x) for x in rec.routes]   # bit-exact
+        assert st.u == rec.u and st.b == rec.b and st.lr == rec.lr
+        assert st.perturbed == rec.perturbed
+        np.testing.assert_allclose(st.alpha, rec.alpha, rtol=1e-12)
+    assert normwise(r0.w.cpu().numpy(), recs[-1].w) <= 1e-4
+    assert sum(s.n_steps for s in stats) >= 45
+
+
+def test_eval_topk_matches_oracle():
+    cfg = config("tiny")
+    data = dataset("tiny")
+    test = dataset("tiny", None, "test")
+    from paper_conf_ipps_marws22_b200 import api
+    rep = make_replica(cfg, data, "fp32", extra=(test,))
+    td = api.DeviceCsr(test)
+    rows = np.arange(300, dtype=np.int32)
+    top = rep.eval_topk(td, torch.as_tensor(rows, device="cuda"), 5).cpu().numpy()
+    _, _, Z = omodel.forward(init_params(cfg).astype(np.float64), test.row_slice(rows), cfg.F, cfg.H, cfg.L)
+    ref = metrics.topk(Z, 5)
+    # exact where the ranking is not within fp32 rounding of a tie
+    srt = -np.sort(-Z, axis=1)
+    clear = (srt[:, :5] - srt[:, 1:6]).min(axis=1) > 1e-5
+    assert clear.sum() > 250
+    np.testing.assert_array_equal(top[clear], ref[clear])
+    sub = test.row_slice(rows)
+    assert api.precision_at_k_hits(top[clear], *_lab(sub, clear), 5) == \
+        round(metrics.precision_at_k(ref[clear], *_lab(sub, clear), 5) * 5 * clear.sum())
+
+
+def _lab(sub, mask):
+    idx = np.nonzero(mask)[0]
+    s2 = sub.row_slice(idx)
+    return s2.lab_ptr, s2.lab
