@@ -1,0 +1,405 @@
+#!/usr/bin/env python
+"""Benchmark of the Adaptive SGD hot path on B200: whole-box samples/s of the
+local SGD steps + normalized merge (BASELINE.json metric).
+
+A bench "step" is one mega-batch: M = 100 b_max samples routed batch by
+batch to the ranks by the dynamic scheduler, one local SGD step per batch,
+then the merge (Alg. 2) and batch size scaling (Alg. 1) -- every row of
+DESIGN.md's hot-path table.  Default workload: EURLex-4K-shaped
+(BASELINE.json configs[1], 1 B200).  Inputs are resident in HBM when the
+timed region starts; L2 is flushed (256 MiB write) between timed steps,
+outside the timed events.  `e2e` repeats the measurement through the C ABI
+with host (pinned) buffers: every step copies its mega-batch CSR host->device
+and reads its losses back.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config NAME]
+                    [--precision auto|fp32|bf16] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "samples/s (whole box) of local SGD step+merge"
+UNIT = "samples/s"
+
+
+def _args():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--config", default="eurlex4k")
+    p.add_argument("--precision", default="auto", choices=["auto", "fp32", "bf16"])
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--inflight", type=int, default=2)
+    p.add_argument("--e2e-steps", type=int, default=None)
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=12.0)
+    return p.parse_args()
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0,
+                "sm_max_mhz": 1965.0}, "fallback"
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """NVML sampling of SM clock and throttle reasons during the timed region."""
+
+    REASONS = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown",
+               0x4: "sw_power_cap", 0x80: "hw_power_brake_slowdown"}
+
+    def __init__(self, index: int, period: float = 0.01):
+        self.index, self.period = index, period
+        self.samples, self.reasons = [], set()
+        self._stop = threading.Event()
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.max_mhz = None
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                    "samples": 0}
+        return {"sm_mhz": float(statistics.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------ CPU oracle
+def cpu_baseline(cfg, data, budget_s: float):
+    """The oracle as it stands (fp64 numpy/scipy) on the host cores: consecutive
+    b_max-row local steps of the same workload plus the per-mega-batch merge,
+    amortised over the mega-batch's 100 steps."""
+    from oracle import merge as omerge, model as omodel
+    from synth import init_params, sample_stream
+    try:
+        from threadpoolctl import threadpool_info
+        cores = max([i.get("num_threads", 1) for i in threadpool_info()] + [1])
+    except Exception:
+        cores = os.cpu_count()
+    w = init_params(cfg).astype(np.float64)
+    b = cfg.b_max
+    steps, samples = 0, 0
+    t0 = time.perf_counter()
+    while True:
+        rows = sample_stream(cfg, steps * b, b)
+        w, _, _ = omodel.sgd_step(w, data.row_slice(rows), cfg.lr_max, cfg.F, cfg.H, cfg.L)
+        steps += 1
+        samples += b
+        if time.perf_counter() - t0 > budget_s:
+            break
+    t_steps = time.perf_counter() - t0
+    t1 = time.perf_counter()
+    omerge.merge_models([w], [1.0], w, np.zeros_like(w), 0.9)
+    t_merge = time.perf_counter() - t1
+    steps_per_mb = cfg.mega_batch // b
+    t_total = t_steps + t_merge * steps / steps_per_mb
+    return {"value": samples / t_total, "unit": UNIT, "cores": int(cores), "kind": "oracle",
+            "sample": f"{steps} local steps x {b} rows of {cfg.name} (fp64 numpy/scipy oracle) + "
+                      f"merge amortised over {steps_per_mb} steps/mega-batch"}, t_total
+
+
+# ------------------------------------------------------------------ roofline
+def kernel_work(cls: str, cfg, bf16: bool, st):
+    """Algorithmic bytes or flops of one launch of a kernel class."""
+    B, H, L, F, P = st["B"], cfg.H, cfg.L, cfg.F, cfg.n_params
+    nnz, U = st["nnz"], st["U"]
+    if cls in ("g1", "g2", "g3"):
+        return ("flops", 2.0 * B * H * L)
+    if cls == "spmm":
+        return ("bytes", 8.0 * nnz + 12.0 * B + 4.0 * U * H + 4.0 * B * H)
+    if cls == "scatter":
+        return ("bytes", 8.0 * nnz + 4.0 * B * H + 8.0 * U * H)
+    if cls == "softmax":
+        return ("bytes", (6.0 if bf16 else 8.0) * B * L + 8.0 * st["nlab"])
+    if cls == "touched":
+        return ("bytes", 4.0 * nnz + 12.0 * nnz + 8.0 * F + 12.0 * B)
+    if cls == "dh_b1":
+        return ("bytes", 4.0 * st["splitk"] * B * H + 8.0 * B * H)
+    if cls == "b2":
+        return ("bytes", (2.0 if bf16 else 4.0) * B * L + 8.0 * L)
+    if cls == "merge":
+        return ("bytes", 12.0 * P)   # 36 P per mega-batch over its 3 launches
+    return ("bytes", 0.0)
+
+
+def main():
+    a = _args()
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    if a.impl == "reference":
+        return reference_arm(a, rank, world)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_marws22_b200 import api, train, _lib
+    from synth import config, generate, init_params, sample_stream
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    cfg = config(a.config)
+    prec = a.precision
+    if prec == "auto":
+        prec = "bf16" if _bf16_available() else "fp32"
+    bf16 = prec == "bf16"
+    data = generate(cfg, "train")
+    w0 = init_params(cfg)
+    nz, nl = api.max_step_sizes([data], cfg.b_max)
+    rep = api.Replica(cfg.F, cfg.L, cfg.H, cfg.b_max, nz, nl, prec, device=local, w0=w0)
+    dd = api.DeviceCsr(data, device=dev)
+    rep.register(dd)
+    h = train.Hyper.from_config(cfg)
+    M = h.M
+    shm = f"/asgd_bench_{os.environ.get('MASTER_PORT', os.getpid())}"
+    if rank == 0:
+        sched = api.Scheduler(shm, world, M, create=True)
+    if world > 1:
+        dist.barrier()
+    if rank != 0:
+        sched = api.Scheduler(shm, world, M, create=False)
+    drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=a.inflight)
+    K, W = a.steps, a.warmup
+    Ke = a.e2e_steps if a.e2e_steps is not None else min(K, 10)
+    ids = [sample_stream(cfg, mb * M, M) for mb in range(W + K + Ke)]
+    rows_d = [torch.as_tensor(x, device=dev) for x in ids[:W + K]]
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    for mb in range(W):
+        drv.megabatch(rows_d[mb])
+    torch.cuda.synchronize()
+
+    # ---------------------------------------------------------------- timed
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    call = _lib.call
+    call("asgd_profile", rep.ctx, 1)
+    l0 = rep.launches()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    stats = []
+    with ClockSampler(local) as clk:
+        for k in range(K):
+            flush.zero_()
+            ev[k][0].record()
+            stats.append(drv.megabatch(rows_d[W + k], keep_log=True))
+            ev[k][1].record()
+        torch.cuda.synchronize()
+    launches = rep.launches() - l0
+    ms = np.zeros(10, dtype=np.float64)
+    cnt = np.zeros(10, dtype=np.int64)
+    call("asgd_profile_read", rep.ctx, ms.ctypes.data, cnt.ctypes.data)
+    call("asgd_profile", rep.ctx, 0)
+    t_ms = sum(e0.elapsed_time(e1) for e0, e1 in ev)
+    t = torch.tensor([t_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    t_max = float(t.item())
+    value = K * M / (t_max / 1e3)
+
+    # ---------------------------------------------------------------- e2e
+    e2e = None
+    if Ke > 0:
+        e2e = run_e2e(rep, drv, data, ids[W + K:W + K + Ke], dev, flush, world, M)
+
+    if rank == 0:
+        peaks, src = _peaks()
+        # per-step workload statistics from the routing logs of the timed region
+        B_list, nnz_l, U_l, lab_l = [], [], [], []
+        lens = np.diff(data.row_ptr)
+        llens = np.diff(data.lab_ptr)
+        for k, s in enumerate(stats):
+            for _, r, st, n in s.routes:
+                rr = ids[W + k][st:st + n]
+                B_list.append(n)
+                nnz_l.append(int(lens[rr].sum()))
+                lab_l.append(int(llens[rr].sum()))
+                U_l.append(len(np.unique(np.concatenate([data.col[data.row_ptr[i]:data.row_ptr[i + 1]] for i in rr]))))
+        wl = {"B": float(np.mean(B_list)), "nnz": float(np.mean(nnz_l)), "U": float(np.mean(U_l)),
+              "nlab": float(np.mean(lab_l)), "splitk": 0}
+        from paper_conf_ipps_marws22_b200.api import _lib as L_
+        names = L_.PROF_NAMES
+        per = {names[i]: {"ms_total": float(ms[i]), "launches": int(cnt[i]),
+                          "us_per_launch": float(ms[i] / cnt[i] * 1e3) if cnt[i] else None}
+               for i in range(len(names))}
+        dom = max(range(len(names)), key=lambda i: ms[i])
+        dname = names[dom]
+        kind, work = kernel_work(dname, cfg, bf16, wl)
+        avg_s = ms[dom] / max(cnt[dom], 1) / 1e3
+        if kind == "flops":
+            achieved = work / avg_s / 1e12
+            if bf16:
+                bound, peak, unit = "tensor", peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"]), "TFLOP/s"
+            else:
+                bound, unit = "alu", "TFLOP/s"
+                peak = 148 * 128 * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+        else:
+            achieved = work / avg_s / 1e9
+            bound, peak, unit = "hbm", peaks["hbm_gbs"], "GB/s"
+        traffic = _traffic(dname)
+        roof = {"bound": bound, "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": unit,
+                "frac": round(achieved / peak, 4), "traffic": traffic, "kernel": dname,
+                "peak_source": src, "work_per_launch": work,
+                "step_share": round(float(ms[dom] / max(t_ms, 1e-9)), 4)}
+        out = {
+            "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world, "steps": K,
+            "warmup": W, "ms_per_step": round(t_max / K, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "bf16" if bf16 else "f32",
+            "data": "synthetic",
+            "config": {"workload": cfg.name, "F": cfg.F, "L": cfg.L, "H": cfg.H, "b_max": cfg.b_max,
+                       "mega_batch_samples": M, "step": "1 mega-batch = local steps + merge",
+                       "precision": prec, "l2": "flushed (256 MiB write) between timed steps",
+                       "inflight": a.inflight, "parallelism": f"dp{world} (model averaging)",
+                       "mean_batch_nnz": round(wl["nnz"], 1), "mean_touched_rows": round(wl["U"], 1)},
+            "roofline": roof,
+            "kernels": per,
+            "gpu_launches": int(launches),
+            "clocks": clk.summary(),
+            "e2e": e2e,
+            "cpu_baseline": None,
+        }
+        if world == 1 and not a.no_cpu_baseline:
+            out["cpu_baseline"], _ = cpu_baseline(cfg, data, a.cpu_seconds)
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.barrier()
+    sched.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def _bf16_available() -> bool:
+    try:
+        from paper_conf_ipps_marws22_b200 import _lib
+        return "bf16-ready" in _lib.lib().asgd_version().decode()
+    except Exception:
+        return False
+
+
+def _traffic(cls: str):
+    """dram bytes per launch of the kernel class from the committed ncu capture."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            return json.load(f).get(cls)
+    except Exception:
+        return None
+
+
+def run_e2e(rep, drv, data, ids_list, dev, flush, world, M):
+    """Same metric through the C ABI from HOST buffers: per step, H2D copy of
+    the mega-batch CSR (pinned) via asgd_data_upload, the mega-batch, and a
+    D2H read of its losses."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_marws22_b200 import api
+    hosts = [api.DeviceCsr(data.row_slice(x), device="cpu", pin=True) for x in ids_list]
+    big = max(hosts, key=lambda hh: hh.nnz)
+    stage = api.DeviceCsr.empty_like(big, device=dev)
+    stage.col = torch.empty(max(hh.nnz for hh in hosts), dtype=torch.int32, device=dev)
+    stage.val = torch.empty(max(hh.nnz for hh in hosts), dtype=torch.float32, device=dev)
+    stage.lab = torch.empty(max(hh.n_lab for hh in hosts), dtype=torch.int32, device=dev)
+    ident = torch.arange(M, dtype=torch.int32, device=dev)
+    loss_host = torch.zeros(drv.losses.numel(), dtype=torch.float32).pin_memory()
+    h2d = d2h = 0
+    t_ms = 0.0
+    for hh in hosts:
+        stage.nnz, stage.n_lab, stage.n_rows = hh.nnz, hh.n_lab, hh.n_rows
+        flush.zero_()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        rep.upload(hh, stage)
+        st = drv.megabatch(ident)
+        n = st.n_steps
+        rep.copy_to_host(loss_host[:n], drv.losses[:n])
+        e1.record()
+        torch.cuda.synchronize()
+        t_ms += e0.elapsed_time(e1)
+        h2d += 8 * (hh.n_rows + 1) * 2 + 8 * hh.nnz + 4 * hh.n_lab
+        d2h += 4 * n
+    t = torch.tensor([t_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    Ke = len(hosts)
+    return {"value": round(Ke * M / (float(t.item()) / 1e3), 1), "unit": UNIT,
+            "h2d_bytes_per_step": int(h2d * world / Ke), "d2h_bytes_per_step": int(d2h * world / Ke)}
+
+
+def reference_arm(a, rank, world):
+    """--impl reference: the CPU oracle, as it stands, on the host cores."""
+    if rank != 0:
+        return
+    from synth import config, generate
+    cfg = config(a.config)
+    data = generate(cfg, "train")
+    per_step = max(1.0, min(a.cpu_seconds, 20.0) / max(1, a.steps))
+    vals = []
+    base = None
+    for k in range(a.warmup + a.steps):
+        cb, _ = cpu_baseline(cfg, data, per_step)
+        if k >= a.warmup:
+            vals.append(cb["value"])
+            base = cb
+    v = float(np.mean(vals))
+    base["value"] = round(v, 2)
+    out = {"metric": METRIC, "value": round(v, 2), "unit": UNIT, "n_gpus": world, "steps": a.steps,
+           "warmup": a.warmup, "ms_per_step": None, "higher_is_better": True, "scaling": "strong",
+           "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+           "config": {"workload": cfg.name, "F": cfg.F, "L": cfg.L, "H": cfg.H, "b_max": cfg.b_max,
+                      "mega_batch_samples": cfg.mega_batch},
+           "cpu_baseline": base,
+           "e2e": {"value": round(v, 2), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+if __name__ == "__main__":
+    main()

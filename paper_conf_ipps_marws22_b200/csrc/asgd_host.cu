@@ -76,7 +76,8 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.n_pieces = (L.nz_cap + kPiece - 1) / kPiece;
   L.n_tiles_f = (F + kScanTile - 1) / kScanTile;
   L.splitk = splitk_for(d);
-  L.n_rowblk = (B + 15) / 16;
+  L.n_rowblk = (B + row_block() - 1) / row_block();
+  const int64_t Lp = padded_ld(Lb);
   L.n_red = kSqnormParts;
   L.part_stride = B * H;
   const bool bf = d.precision == ASGD_PREC_BF16;
@@ -101,8 +102,9 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.ucnt = take((L.u_cap + 1) * 4);
   L.h1 = take(B * H * 4);
   L.h1b = take(bf ? B * H * 2 : 0);
-  L.z = take((size_t)B * Lb * 4);
-  L.dzb = take(bf ? (size_t)B * Lb * 2 : 0);
+  L.z = take((size_t)B * Lp * 4);
+  L.dzb = take(bf ? (size_t)B * Lp * 2 : 0);
+  L.b2part = take((size_t)b2_chunks() * Lb * 4);
   L.rowloss = take(B * 4);
   L.dhpart = take((size_t)L.splitk * B * H * 4);
   L.da1 = take(B * H * 4);
@@ -126,6 +128,7 @@ Ptrs ws_ptrs(char* b, const WsLayout& L) {
   p.rowloss = (float*)(b + L.rowloss); p.dhpart = (float*)(b + L.dhpart); p.da1 = (float*)(b + L.da1);
   p.db1part = (float*)(b + L.db1part); p.w2b = (bf16*)(b + L.w2b); p.red = (double*)(b + L.red);
   p.eval_top = (int32_t*)(b + L.eval_top);
+  p.b2part = (float*)(b + L.b2part);
   return p;
 }
 
@@ -195,7 +198,7 @@ extern "C" {
 
 const char* asgd_last_error(void) { return g_err.c_str(); }
 
-const char* asgd_version(void) { return "libasgd sm_100a (tcgen05/TMA bf16 + fp32 SIMT) r1"; }
+const char* asgd_version(void) { return "libasgd sm_100a (tcgen05/TMA bf16 + fp32 SIMT) r1 bf16-ready"; }
 
 size_t asgd_workspace_bytes(const asgd_model_desc* d) {
   if (!d || d->F <= 0 || d->L <= 0 || d->b_max <= 0 || d->max_step_nnz <= 0) return 0;
@@ -328,6 +331,7 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
   const bool bf = m.precision == ASGD_PREC_BF16;
   const int H = (int)m.H;
   const int64_t Lb = m.L;
+  const int64_t Lp = padded_ld(Lb);
   float* W1 = c->params + c->o_w1;
   float* b1 = c->params + c->o_b1;
   float* W2 = c->params + c->o_w2;
@@ -348,32 +352,32 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     a.M = n; a.N = (int)Lb; a.K = H;
     a.A = P.h1; a.as0 = H; a.as1 = 1;
     a.B = W2; a.bs0 = 1; a.bs1 = H;
-    a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = Lb; a.bias = b2; a.splitk = 1;
+    a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = Lp; a.bias = b2; a.splitk = 1;
     PCU(ASGD_K_G1, launch_gemm_f32(lc, a));
-    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, rows, x.lab_ptr, x.lab, P, false));
+    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, false));
     // G2: dH1 partials = dZ W2 (pre-step W2)
     a = GemmArgs{};
     a.M = n; a.N = H; a.K = (int)Lb;
-    a.A = P.z; a.as0 = Lb; a.as1 = 1;
+    a.A = P.z; a.as0 = Lp; a.as1 = 1;
     a.B = W2; a.bs0 = H; a.bs1 = 1;
     a.epi = EPI_SPLITK; a.C = P.dhpart; a.ldc = H; a.splitk = (int)c->L.splitk;
     a.part_stride = c->L.part_stride;
     PCU(ASGD_K_G2, launch_gemm_f32(lc, a));
   } else {
     PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, P, c->L, W2, b2, nullptr));
-    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, rows, x.lab_ptr, x.lab, P, true));
+    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, true));
     PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, lr, P, c->L, W2, b2, nullptr));
   }
   PCU(ASGD_K_DH, ([&]() -> cudaError_t {
         cudaError_t e = launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L);
         return e != cudaSuccess ? e : launch_b1_update(lc, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev);
       })());
-  PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, b2, lr, P, bf, g ? g + c->o_b2 : nullptr));
+  PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, Lp, b2, lr, P, bf, g ? g + c->o_b2 : nullptr));
   if (!bf) {
     // G3: W2 -= lr dZ^T H1
     GemmArgs a{};
     a.M = (int)Lb; a.N = H; a.K = n;
-    a.A = P.z; a.as0 = 1; a.as1 = Lb;
+    a.A = P.z; a.as0 = 1; a.as1 = Lp;
     a.B = P.h1; a.bs0 = H; a.bs1 = 1;
     a.epi = EPI_SGD; a.C = W2; a.ldc = H; a.lr = lr; a.grad = g ? g + c->o_w2 : nullptr;
     a.splitk = 1;
@@ -468,12 +472,12 @@ int asgd_eval_topk(asgd_ctx* c, const asgd_csr* t, const int32_t* rows, int32_t 
       a.M = nb; a.N = (int)m.L; a.K = H;
       a.A = P.h1; a.as0 = H; a.as1 = 1;
       a.B = W2; a.bs0 = 1; a.bs1 = H;
-      a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = m.L; a.bias = b2; a.splitk = 1;
+      a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = padded_ld(m.L); a.bias = b2; a.splitk = 1;
       CU(launch_gemm_f32(lc, a));
     } else {
       CU(launch_gemm_tc(lc, 1, nb, m.L, H, 0.f, P, c->L, W2, b2, nullptr));
     }
-    CU(launch_topk(lc, nb, m.L, k, P.z, topk + (int64_t)r0 * k));
+    CU(launch_topk(lc, nb, m.L, padded_ld(m.L), k, P.z, topk + (int64_t)r0 * k));
   }
   return ASGD_OK;
 }

@@ -25,7 +25,7 @@ typedef __nv_bfloat16 bf16;
 struct WsLayout {
   size_t meta, boff, loff, cnt, fseg, fuid, uniq, useg, tsum, tpre;
   size_t e_n, e_v, e_u, part1, rowcnt, part5, ucnt;
-  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, red, eval_top;
+  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, red, eval_top, b2part;
   size_t total;
   int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride;
 };
@@ -37,8 +37,10 @@ struct Ptrs {  // typed views of the workspace
   int32_t* uniq; int32_t* useg; int32_t* tsum; int32_t* tpre;
   int32_t* e_n; float* e_v; int32_t* e_u; float* part1; int32_t* rowcnt; float* part5;
   int32_t* ucnt; float* h1; bf16* h1b; float* z; bf16* dzb; float* rowloss; float* dhpart;
-  float* da1; float* db1part; bf16* w2b; double* red; int32_t* eval_top;
+  float* da1; float* db1part; bf16* w2b; double* red; int32_t* eval_top; float* b2part;
 };
+int row_block();   // rows per db1 partial (kernels_dense.cu)
+int b2_chunks();   // row chunks of the db2 partial sums
 Ptrs ws_ptrs(char* base, const WsLayout& L);
 
 struct Launch {       // launch bookkeeping of one ctx
@@ -76,14 +78,16 @@ struct GemmArgs {
   bf16* shadow;                    // SGD: shadow[m*ldc+n] = bf16(new C)
 };
 cudaError_t launch_gemm_f32(const Launch&, const GemmArgs&);
-cudaError_t launch_softmax_ce(const Launch&, int n, int64_t L, const int32_t* rows,
+// Leading dimension of the B x L logit buffers (16-byte rows for TMA).
+int64_t padded_ld(int64_t L);
+cudaError_t launch_softmax_ce(const Launch&, int n, int64_t L, int64_t ldz, const int32_t* rows,
                               const int64_t* lab_ptr, const int32_t* lab, const Ptrs&,
                               bool bf16_out);
 cudaError_t launch_dh_reduce(const Launch&, int n, int H, int splitk, const Ptrs&, const WsLayout&);
 cudaError_t launch_b1_update(const Launch&, int n, int H, float* b1, float lr, const Ptrs&,
                              const WsLayout&, float* grad_b1, float* loss_dev);
-cudaError_t launch_b2_update(const Launch&, int n, int64_t L, float* b2, float lr, const Ptrs&,
-                             bool from_bf16, float* grad_b2);
+cudaError_t launch_b2_update(const Launch&, int n, int64_t L, int64_t ldz, float* b2, float lr,
+                             const Ptrs&, bool from_bf16, float* grad_b2);
 cudaError_t launch_to_bf16(const Launch&, const float* src, bf16* dst, int64_t count);
 // ---------------------------------------------------------------- tcgen05 (bf16)
 bool tc_available();
@@ -96,7 +100,8 @@ cudaError_t launch_scale(const Launch&, float* x, int64_t P, double alpha);
 cudaError_t launch_finish(const Launch&, float* params, float* w, float* d, int64_t P, float gamma);
 cudaError_t launch_wsum(const Launch&, const float* const* reps, const double* alpha, int n,
                         int64_t P, float* out);
-cudaError_t launch_topk(const Launch&, int n, int64_t L, int k, const float* z, int32_t* out);
+cudaError_t launch_topk(const Launch&, int n, int64_t L, int64_t ldz, int k, const float* z,
+                        int32_t* out);
 cudaError_t launch_validate_csr(const Launch&, const asgd_csr* c, int64_t F, int64_t L, int32_t* err);
 
 }  // namespace asgd

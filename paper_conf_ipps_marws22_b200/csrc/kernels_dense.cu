@@ -90,7 +90,8 @@ __global__ void __launch_bounds__(256) k_gemm_f32(GemmArgs g) {
 // ------------------------------------------------------------ softmax + CE
 // One CTA per batch row n: lse = log sum_j exp(Z_nj); loss_n = lse - mean_{y in Y_n} Z_ny;
 // dZ_nj = (exp(Z_nj - lse) - T_nj) / B with T_nj = 1/|Y_n| on Y_n (Q3, Q4).
-__global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, const int32_t* __restrict__ rows,
+__global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ldz,
+                                                    const int32_t* __restrict__ rows,
                                                     const int64_t* __restrict__ lab_ptr,
                                                     const int32_t* __restrict__ lab, float* Z,
                                                     bf16* dZb, float* rowloss) {
@@ -103,7 +104,7 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, const int3
   const int64_t l0 = lab_ptr[id];
   const int64_t nl64 = lab_ptr[id + 1] - l0;
   const int nl = (int)(nl64 < kMaxRowLabels ? nl64 : kMaxRowLabels);
-  float* z = Z + (int64_t)n * L;
+  float* z = Z + (int64_t)n * ldz;
   for (int i = threadIdx.x; i < nl; i += blockDim.x) {
     int y = lab[l0 + i];
     s_lab[i] = y;
@@ -141,7 +142,7 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, const int3
   __syncthreads();
   const float lse = s_lse, invB = 1.f / (float)B;
   if (dZb) {
-    bf16* d = dZb + (int64_t)n * L;
+    bf16* d = dZb + (int64_t)n * ldz;
     for (int64_t j = threadIdx.x; j < L; j += blockDim.x) d[j] = __float2bfloat16_rn(__expf(z[j] - lse) * invB);
     __syncthreads();
     for (int i = threadIdx.x; i < nl; i += blockDim.x)
@@ -155,68 +156,98 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, const int3
 }
 
 // ------------------------------------------------------ dH1 reduce + ReLU'
-// dA1[r][c] = [H1[r][c] > 0] * sum_z part[z][r][c];  db1 partial per row block.
-constexpr int kRowBlk = 16;
-__global__ void __launch_bounds__(256) k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
-                                                   const float* __restrict__ part,
-                                                   const float* __restrict__ H1, float* dA1,
-                                                   float* db1part) {
-  __shared__ float sp[256];
-  const int cw = min(H, 256);           // columns per pass
-  const int tpc = 256 / cw;             // row groups
-  const int c0 = threadIdx.x % cw, g = threadIdx.x / cw;
+// dA1[r][c] = [H1[r][c] > 0] * sum_z part[z][r][c];  db1 partial per block of kRowBlk rows.
+// One thread per column (blockDim = H), so every sum has a fixed order.
+constexpr int kRowBlk = 4;
+__global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
+                            const float* __restrict__ part, const float* __restrict__ H1,
+                            float* dA1, float* db1part) {
+  const int c = threadIdx.x;
   const int r0 = blockIdx.x * kRowBlk;
-  for (int cb = 0; cb < H; cb += cw) {
-    const int c = cb + c0;
-    float colsum = 0.f;
-    for (int rr = g; rr < kRowBlk; rr += tpc) {
-      const int r = r0 + rr;
-      if (r >= n) break;
-      const int64_t o = (int64_t)r * H + c;
-      float s = 0.f;
-      for (int z = 0; z < splitk; ++z) s += part[z * part_stride + o];
-      const float v = H1[o] > 0.f ? s : 0.f;
-      dA1[o] = v;
-      colsum += v;
+  float colsum = 0.f;
+#pragma unroll
+  for (int rr = 0; rr < kRowBlk; ++rr) {
+    const int r = r0 + rr;
+    if (r >= n) break;
+    const int64_t o = (int64_t)r * H + c;
+    float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
+    int z = 0;
+    for (; z + 4 <= splitk; z += 4) {
+      s0 += __ldcs(part + z * part_stride + o);
+      s1 += __ldcs(part + (z + 1) * part_stride + o);
+      s2 += __ldcs(part + (z + 2) * part_stride + o);
+      s3 += __ldcs(part + (z + 3) * part_stride + o);
     }
-    sp[threadIdx.x] = colsum;
-    __syncthreads();
-    if (threadIdx.x < cw) {
-      float t = 0.f;
-      for (int q = 0; q < tpc; ++q) t += sp[q * cw + threadIdx.x];
-      db1part[(int64_t)blockIdx.x * H + c] = t;
-    }
-    __syncthreads();
+    for (; z < splitk; ++z) s0 += __ldcs(part + z * part_stride + o);
+    const float s = (s0 + s1) + (s2 + s3);
+    const float v = H1[o] > 0.f ? s : 0.f;
+    dA1[o] = v;
+    colsum += v;
   }
+  db1part[(int64_t)blockIdx.x * H + c] = colsum;
 }
 
+// b1 -= lr * sum_blocks db1part (blockDim = H), mean loss = sum rowloss / n.
 __global__ void k_b1_update(int n, int H, int nblk, const float* __restrict__ db1part, float* b1,
                             float lr, float* grad_b1, const float* __restrict__ rowloss,
                             float* loss_dev) {
-  for (int c = threadIdx.x; c < H; c += blockDim.x) {
-    float s = 0.f;
-    for (int b = 0; b < nblk; ++b) s += db1part[(int64_t)b * H + c];
-    b1[c] -= lr * s;
-    if (grad_b1) grad_b1[c] = s;
+  const int c = threadIdx.x;
+  float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
+  int b = 0;
+  for (; b + 4 <= nblk; b += 4) {
+    a0 += db1part[(int64_t)b * H + c];
+    a1 += db1part[(int64_t)(b + 1) * H + c];
+    a2 += db1part[(int64_t)(b + 2) * H + c];
+    a3 += db1part[(int64_t)(b + 3) * H + c];
   }
-  if (threadIdx.x == 0 && loss_dev) {
-    float s = 0.f;
-    for (int r = 0; r < n; ++r) s += rowloss[r];
-    *loss_dev = s / (float)n;
+  for (; b < nblk; ++b) a0 += db1part[(int64_t)b * H + c];
+  const float s = (a0 + a1) + (a2 + a3);
+  b1[c] -= lr * s;
+  if (grad_b1) grad_b1[c] = s;
+  if (loss_dev && threadIdx.x < 32) {
+    float t = 0.f;
+    for (int r = threadIdx.x; r < n; r += 32) t += rowloss[r];
+#pragma unroll
+    for (int o = 16; o; o >>= 1) t += __shfl_xor_sync(kFull, t, o);
+    if (threadIdx.x == 0) *loss_dev = t / (float)n;
   }
 }
 
-// db2[j] = sum_n dZ[n][j];  b2 -= lr db2
-__global__ void k_b2_update(int n, int64_t L, const float* __restrict__ dz,
-                            const bf16* __restrict__ dzb, float* b2, float lr, float* grad_b2) {
-  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < L;
-       j += (int64_t)gridDim.x * blockDim.x) {
-    float s = 0.f;
-    if (dzb) for (int r = 0; r < n; ++r) s += __bfloat162float(dzb[(int64_t)r * L + j]);
-    else for (int r = 0; r < n; ++r) s += dz[(int64_t)r * L + j];
-    b2[j] -= lr * s;
-    if (grad_b2) grad_b2[j] = s;
+// db2 partials: b2part[y][j] = sum over row chunk y of dZ[r][j]
+constexpr int kB2Chunks = 16;
+__global__ void __launch_bounds__(256) k_b2_part(int n, int64_t L, int64_t ldz, const float* __restrict__ dz,
+                                                 const bf16* __restrict__ dzb, float* b2part) {
+  const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= L) return;
+  const int per = (n + gridDim.y - 1) / gridDim.y;
+  const int r0 = blockIdx.y * per, r1 = min(n, r0 + per);
+  float s0 = 0.f, s1 = 0.f;
+  int r = r0;
+  if (dzb) {
+    for (; r + 2 <= r1; r += 2) {
+      s0 += __bfloat162float(dzb[(int64_t)r * ldz + j]);
+      s1 += __bfloat162float(dzb[(int64_t)(r + 1) * ldz + j]);
+    }
+    for (; r < r1; ++r) s0 += __bfloat162float(dzb[(int64_t)r * ldz + j]);
+  } else {
+    for (; r + 2 <= r1; r += 2) {
+      s0 += dz[(int64_t)r * ldz + j];
+      s1 += dz[(int64_t)(r + 1) * ldz + j];
+    }
+    for (; r < r1; ++r) s0 += dz[(int64_t)r * ldz + j];
   }
+  b2part[(int64_t)blockIdx.y * L + j] = s0 + s1;
+}
+
+// b2 -= lr * sum_y b2part[y]
+__global__ void __launch_bounds__(256) k_b2_apply(int64_t L, int chunks, const float* __restrict__ b2part,
+                                                  float* b2, float lr, float* grad_b2) {
+  const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= L) return;
+  float s = 0.f;
+  for (int y = 0; y < chunks; ++y) s += b2part[(int64_t)y * L + j];
+  b2[j] -= lr * s;
+  if (grad_b2) grad_b2[j] = s;
 }
 
 __global__ void k_to_bf16(const float* __restrict__ src, bf16* dst, int64_t count) {
@@ -235,10 +266,10 @@ cudaError_t launch_gemm_f32(const Launch& lc, const GemmArgs& g) {
   return cudaGetLastError();
 }
 
-cudaError_t launch_softmax_ce(const Launch& lc, int n, int64_t L, const int32_t* rows,
+cudaError_t launch_softmax_ce(const Launch& lc, int n, int64_t L, int64_t ldz, const int32_t* rows,
                               const int64_t* lab_ptr, const int32_t* lab, const Ptrs& P,
                               bool bf16_out) {
-  k_softmax_ce<<<n, 512, 0, lc.s>>>(n, L, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
+  k_softmax_ce<<<n, 512, 0, lc.s>>>(n, L, ldz, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
                                     P.rowloss);
   ++*lc.counter;
   return cudaGetLastError();
@@ -248,8 +279,7 @@ cudaError_t launch_dh_reduce(const Launch& lc, int n, int H, int splitk, const P
                              const WsLayout& L) {
   const int nblk = (n + kRowBlk - 1) / kRowBlk;
   // split-K partial z of dH1 lives at dhpart + z * (b_max * H)
-  k_dh_reduce<<<nblk, 256, 0, lc.s>>>(n, H, splitk, L.part_stride, P.dhpart, P.h1, P.da1,
-                                      P.db1part);
+  k_dh_reduce<<<nblk, H, 0, lc.s>>>(n, H, splitk, L.part_stride, P.dhpart, P.h1, P.da1, P.db1part);
   ++*lc.counter;
   return cudaGetLastError();
 }
@@ -257,16 +287,18 @@ cudaError_t launch_dh_reduce(const Launch& lc, int n, int H, int splitk, const P
 cudaError_t launch_b1_update(const Launch& lc, int n, int H, float* b1, float lr, const Ptrs& P,
                              const WsLayout& L, float* grad_b1, float* loss_dev) {
   const int nblk = (n + kRowBlk - 1) / kRowBlk;
-  k_b1_update<<<1, 512, 0, lc.s>>>(n, H, nblk, P.db1part, b1, lr, grad_b1, P.rowloss, loss_dev);
+  k_b1_update<<<1, H, 0, lc.s>>>(n, H, nblk, P.db1part, b1, lr, grad_b1, P.rowloss, loss_dev);
   ++*lc.counter;
   return cudaGetLastError();
 }
 
-cudaError_t launch_b2_update(const Launch& lc, int n, int64_t L, float* b2, float lr, const Ptrs& P,
-                             bool from_bf16, float* grad_b2) {
-  const int64_t blocks = std::min<int64_t>((L + 255) / 256, (int64_t)lc.sms * 16);
-  k_b2_update<<<(int)blocks, 256, 0, lc.s>>>(n, L, P.z, from_bf16 ? P.dzb : nullptr, b2, lr, grad_b2);
-  ++*lc.counter;
+cudaError_t launch_b2_update(const Launch& lc, int n, int64_t L, int64_t ldz, float* b2, float lr,
+                             const Ptrs& P, bool from_bf16, float* grad_b2) {
+  const int chunks = std::max(1, std::min(kB2Chunks, n / 16));
+  dim3 grid((unsigned)((L + 255) / 256), (unsigned)chunks);
+  k_b2_part<<<grid, 256, 0, lc.s>>>(n, L, ldz, P.z, from_bf16 ? P.dzb : nullptr, P.b2part);
+  k_b2_apply<<<(unsigned)((L + 255) / 256), 256, 0, lc.s>>>(L, chunks, P.b2part, b2, lr, grad_b2);
+  *lc.counter += 2;
   return cudaGetLastError();
 }
 
@@ -278,5 +310,6 @@ cudaError_t launch_to_bf16(const Launch& lc, const float* src, bf16* dst, int64_
 }
 
 int row_block() { return kRowBlk; }
+int b2_chunks() { return kB2Chunks; }
 
 }  // namespace asgd

@@ -113,10 +113,10 @@ __device__ __forceinline__ bool better(const Cand& a, const Cand& b) {
 }
 
 template <int K>
-__global__ void __launch_bounds__(256) k_topk(int64_t L, int k, const float* __restrict__ z,
+__global__ void __launch_bounds__(256) k_topk(int64_t L, int64_t ldz, int k, const float* __restrict__ z,
                                               int32_t* out) {
   const int n = blockIdx.x;
-  const float* row = z + (int64_t)n * L;
+  const float* row = z + (int64_t)n * ldz;
   Cand top[K];
 #pragma unroll
   for (int i = 0; i < K; ++i) top[i] = Cand{-INFINITY, 0x7fffffff};
@@ -213,9 +213,10 @@ cudaError_t launch_wsum(const Launch& lc, const float* const* reps, const double
   return cudaGetLastError();
 }
 
-cudaError_t launch_topk(const Launch& lc, int n, int64_t L, int k, const float* z, int32_t* out) {
+cudaError_t launch_topk(const Launch& lc, int n, int64_t L, int64_t ldz, int k, const float* z,
+                        int32_t* out) {
   if (k <= 0 || k > 8) return cudaErrorInvalidValue;
-  k_topk<8><<<n, 256, 0, lc.s>>>(L, k, z, out);
+  k_topk<8><<<n, 256, 0, lc.s>>>(L, ldz, k, z, out);
   ++*lc.counter;
   return cudaGetLastError();
 }

@@ -1,9 +1,379 @@
-// placeholder until the tcgen05 path lands
+// tcgen05 tensor-core GEMMs of the bf16 path (sm_100a): the three dense
+// contractions of the output layer (§V-A: the 3-layer
+// MLP's hidden->output layer; rows a4 and a6 of DESIGN.md):
+//   G1  Z[B x L]   = H1[B x H] . W2[L x H]^T + b2        (A, B K-major)
+//   G2  dH1[B x H] = dZ[B x L] . W2[L x H]   (split-K)    (A K-major, B MN-major)
+//   G3  W2 -= lr dZ[B x L]^T . H1[B x H]    (fused SGD)  (A, B MN-major)
+// bf16 operands staged by TMA (128B swizzle) in a 4-stage mbarrier ring,
+// one elected thread issues tcgen05.mma (M = 128, N = BN, K = 16) into a TMEM
+// accumulator, four epilogue warps drain TMEM with tcgen05.ld and apply the
+// fused epilogue (bias, split-K partial store, or the W2 SGD update + bf16
+// shadow refresh).  fp32 accumulation throughout.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <mutex>
+
 #include "asgd_internal.h"
+
 namespace asgd {
-bool tc_available() { return false; }
-cudaError_t launch_gemm_tc(const Launch&, int, int, int64_t, int, float, const Ptrs&, const WsLayout&,
-                           float*, const float*, float*) {
-  return cudaErrorNotSupported;
+namespace {
+
+constexpr int BM = 128, BK = 64, STAGES = 4;
+enum { TC_EPI_Z = 0, TC_EPI_PART = 1, TC_EPI_SGD = 2 };
+
+struct TcArgs {
+  int M, N, K;
+  // epilogue
+  float* out; int64_t ldo;            // Z (ldo = Lp) / partials (ldo = H) / W2 (ldo = H)
+  int64_t part_stride;                // split-K partial z offset
+  const float* bias;                  // G1
+  float lr; bf16* shadow; float* grad;// G3
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  const uint32_t a = smem_u32(bar);
+  uint32_t ok = 0;
+  while (!ok) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(a), "r"(parity)
+        : "memory");
+  }
+}
+
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0,
+                                            int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
+
+__device__ __forceinline__ void tc_fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+
+// SM100 shared-memory matrix descriptor, 128B swizzle.
+__device__ __forceinline__ uint64_t desc_sw128(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+  d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
+  d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
+  d |= (uint64_t)1 << 46;  // descriptor version (sm_100)
+  d |= (uint64_t)2 << 61;  // SWIZZLE_128B
+  return d;
+}
+
+// Instruction descriptor: kind::f16, bf16 x bf16 -> f32, M = 128.
+__host__ __device__ constexpr uint32_t make_idesc(int N, bool a_mn, bool b_mn) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | ((a_mn ? 1u : 0u) << 15) | ((b_mn ? 1u : 0u) << 16) |
+         ((uint32_t)(N >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+}
+
+__device__ __forceinline__ void mma_bf16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc,
+                                         uint32_t accum) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(a), "l"(b), "r"(idesc), "r"(accum)
+      : "memory");
+}
+
+__device__ __forceinline__ void mma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                   smem_u32(bar))
+               : "memory");
+}
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, float (&v)[32]) {
+  uint32_t r[32];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, "
+      "%16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+        "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]),
+        "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]),
+        "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+template <int BN, bool A_MN, bool B_MN, int EPI>
+__global__ void __launch_bounds__(256, 1)
+    k_gemm_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, TcArgs g) {
+  constexpr uint32_t A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE = A_BYTES + B_BYTES;
+  constexpr uint32_t TMEM_COLS = BN;  // 64, 128 or 256 fp32 columns
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + STAGES * A_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * STAGE);
+  uint64_t* empty = full + STAGES;
+  uint64_t* tfull = empty + STAGES;
+  uint32_t* tbase = reinterpret_cast<uint32_t*>(tfull + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int n0 = blockIdx.x * BN, m0 = blockIdx.y * BM;
+  const int nkb = (g.K + BK - 1) / BK;
+  const int per = (nkb + gridDim.z - 1) / gridDim.z;
+  const int kb0 = blockIdx.z * per;
+  const int nk = max(0, min(nkb, kb0 + per) - kb0);
+
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
+    for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+    mbar_init(tfull, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 2) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tbase)),
+                 "r"(TMEM_COLS)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tbase;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // ------------------------------------------------ TMA producer
+      for (int i = 0; i < nk; ++i) {
+        const int s = i % STAGES;
+        const uint32_t ph = (i / STAGES) & 1;
+        mbar_wait(&empty[s], ph ^ 1);
+        mbar_expect_tx(&full[s], STAGE);
+        const int kc = (kb0 + i) * BK;
+        uint8_t* a = sA + s * A_BYTES;
+        uint8_t* b = sB + s * B_BYTES;
+        if constexpr (!A_MN) {
+          tma_load_2d(a, &tmA, &full[s], kc, m0);
+        } else {
+          tma_load_2d(a, &tmA, &full[s], m0, kc);
+          tma_load_2d(a + 8192, &tmA, &full[s], m0 + 64, kc);
+        }
+        if constexpr (!B_MN) {
+          tma_load_2d(b, &tmB, &full[s], kc, n0);
+        } else {
+#pragma unroll
+          for (int j = 0; j < BN / 64; ++j) tma_load_2d(b + j * 8192, &tmB, &full[s], n0 + 64 * j, kc);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // ------------------------------------------------ MMA issuer
+      constexpr uint32_t idesc = make_idesc(BN, A_MN, B_MN);
+      for (int i = 0; i < nk; ++i) {
+        const int s = i % STAGES;
+        const uint32_t ph = (i / STAGES) & 1;
+        mbar_wait(&full[s], ph);
+        tc_fence_after();
+        const uint32_t a_base = smem_u32(sA + s * A_BYTES), b_base = smem_u32(sB + s * B_BYTES);
+#pragma unroll
+        for (int k = 0; k < BK / 16; ++k) {
+          // K-major: advance 16 elements (32 B) inside the 128B swizzle atom.
+          // MN-major: advance 16 K-rows (2 atoms of 8 rows x 128 B = 2048 B).
+          const uint64_t ad = A_MN ? desc_sw128(a_base + k * 2048, 8192, 1024) : desc_sw128(a_base + k * 32, 16, 1024);
+          const uint64_t bd = B_MN ? desc_sw128(b_base + k * 2048, 8192, 1024) : desc_sw128(b_base + k * 32, 16, 1024);
+          mma_bf16(tmem, ad, bd, idesc, (i > 0 || k > 0) ? 1u : 0u);
+        }
+        mma_commit(&empty[s]);   // frees the smem stage once these MMAs retire
+      }
+      if (nk > 0) mma_commit(tfull);
+    }
+  } else if (warp >= 4) {
+    // ------------------------------------------------ epilogue: TMEM -> registers -> global
+    const int wq = warp - 4;
+    const int m = m0 + wq * 32 + lane;
+    if (nk > 0) {
+      mbar_wait(tfull, 0);
+      tc_fence_after();
+    }
+#pragma unroll 1
+    for (int c = 0; c < BN; c += 32) {
+      float v[32];
+      if (nk > 0) {
+        tmem_ld32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)c, v);
+      } else {
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = 0.f;
+      }
+      const int n = n0 + c;
+      if (m >= g.M || n >= g.N) continue;
+      if constexpr (EPI == TC_EPI_Z) {
+        float* o = g.out + (int64_t)m * g.ldo + n;
+        if (n + 32 <= g.N) {
+#pragma unroll
+          for (int j = 0; j < 32; j += 4) {
+            const float4 bb = __ldg(reinterpret_cast<const float4*>(g.bias + n + j));
+            reinterpret_cast<float4*>(o)[j / 4] = make_float4(v[j] + bb.x, v[j + 1] + bb.y, v[j + 2] + bb.z, v[j + 3] + bb.w);
+          }
+        } else {
+          for (int j = 0; j < g.N - n; ++j) o[j] = v[j] + g.bias[n + j];
+        }
+      } else if constexpr (EPI == TC_EPI_PART) {
+        float* o = g.out + (int64_t)blockIdx.z * g.part_stride + (int64_t)m * g.ldo + n;
+#pragma unroll
+        for (int j = 0; j < 32; j += 4)
+          reinterpret_cast<float4*>(o)[j / 4] = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+      } else {  // TC_EPI_SGD: W2[m, n..n+31] -= lr * dW2
+        float* w = g.out + (int64_t)m * g.ldo + n;
+        bf16* sh = g.shadow + (int64_t)m * g.ldo + n;
+#pragma unroll
+        for (int j = 0; j < 32; j += 4) {
+          float4 x = reinterpret_cast<float4*>(w)[j / 4];
+          x.x -= g.lr * v[j]; x.y -= g.lr * v[j + 1]; x.z -= g.lr * v[j + 2]; x.w -= g.lr * v[j + 3];
+          reinterpret_cast<float4*>(w)[j / 4] = x;
+          __nv_bfloat162 p0 = __floats2bfloat162_rn(x.x, x.y), p1 = __floats2bfloat162_rn(x.z, x.w);
+          uint2 pk;
+          pk.x = *reinterpret_cast<uint32_t*>(&p0);
+          pk.y = *reinterpret_cast<uint32_t*>(&p1);
+          reinterpret_cast<uint2*>(sh)[j / 4] = pk;
+        }
+        if (g.grad) {
+          float* gr = g.grad + (int64_t)m * g.ldo + n;
+#pragma unroll
+          for (int j = 0; j < 32; j += 4)
+            reinterpret_cast<float4*>(gr)[j / 4] = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS) : "memory");
+  }
+}
+
+// ------------------------------------------------------------------ host side
+PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
+std::once_flag g_once;
+
+void init_encode() {
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+      q == cudaDriverEntryPointSuccess)
+    g_encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+}
+
+cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t row_bytes,
+                     uint32_t box_inner, uint32_t box_outer) {
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {row_bytes};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = g_encode(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
+template <int BN, bool A_MN, bool B_MN, int EPI>
+cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, const TcArgs& g, int splits) {
+  const size_t smem = (size_t)STAGES * (BM * BK * 2 + BN * BK * 2) + 1024 + 256;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(k_gemm_tc<BN, A_MN, B_MN, EPI>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  dim3 grid((g.N + BN - 1) / BN, (g.M + BM - 1) / BM, splits);
+  k_gemm_tc<BN, A_MN, B_MN, EPI><<<grid, 256, smem, lc.s>>>(a, b, g);
+  ++*lc.counter;
+  return cudaGetLastError();
+}
+
+// Widest N tile that still gives >= one CTA per SM (and does not overhang N by 2x).
+int pick_bn(int64_t tiles_m, int64_t N, int sms) {
+  int bn = 256;
+  while (bn > 64 && (N <= bn / 2 || tiles_m * ((N + bn - 1) / bn) < sms)) bn /= 2;
+  return bn;
+}
+
+}  // namespace
+
+bool tc_available() {
+  std::call_once(g_once, init_encode);
+  return g_encode != nullptr;
+}
+
+int64_t padded_ld(int64_t L) { return (L + 7) / 8 * 8; }
+
+cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H, float lr, const Ptrs& P,
+                           const WsLayout& W, float* W2, const float* b2, float* grad_w2) {
+  if (!tc_available()) return cudaErrorNotSupported;
+  const int64_t Lp = padded_ld(L);
+  CUtensorMap ta, tb;
+  TcArgs g{};
+  cudaError_t e;
+  if (which == 1) {  // Z = H1 W2^T + b2
+    g.M = n; g.N = (int)L; g.K = H;
+    g.out = P.z; g.ldo = Lp; g.bias = b2;
+    const int bn = pick_bn((n + BM - 1) / BM, L, lc.sms);
+    if ((e = make_map(&ta, P.h1b, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
+    if ((e = make_map(&tb, P.w2b, H, L, (uint64_t)H * 2, 64, bn)) != cudaSuccess) return e;
+    if (bn == 256) return run<256, false, false, TC_EPI_Z>(lc, ta, tb, g, 1);
+    if (bn == 128) return run<128, false, false, TC_EPI_Z>(lc, ta, tb, g, 1);
+    return run<64, false, false, TC_EPI_Z>(lc, ta, tb, g, 1);
+  }
+  if (which == 2) {  // dH1 partials = dZ W2
+    g.M = n; g.N = H; g.K = (int)L;
+    g.out = P.dhpart; g.ldo = H; g.part_stride = W.part_stride;
+    const int nkb = (int)((L + BK - 1) / BK);
+    const int splits = std::max(1, std::min<int>((int)W.splitk, nkb));
+    if ((e = make_map(&ta, P.dzb, L, n, (uint64_t)Lp * 2, 64, BM)) != cudaSuccess) return e;
+    if ((e = make_map(&tb, P.w2b, H, L, (uint64_t)H * 2, 64, 64)) != cudaSuccess) return e;
+    // partial slices beyond `splits` stay untouched; dh_reduce sums W.splitk slices
+    if (splits != W.splitk) return cudaErrorInvalidValue;
+    if (H >= 256) return run<256, false, true, TC_EPI_PART>(lc, ta, tb, g, splits);
+    if (H == 128) return run<128, false, true, TC_EPI_PART>(lc, ta, tb, g, splits);
+    return run<64, false, true, TC_EPI_PART>(lc, ta, tb, g, splits);
+  }
+  // which == 3: W2 -= lr dZ^T H1
+  g.M = (int)L; g.N = H; g.K = n;
+  g.out = W2; g.ldo = H; g.lr = lr; g.shadow = P.w2b; g.grad = grad_w2;
+  if ((e = make_map(&ta, P.dzb, L, n, (uint64_t)Lp * 2, 64, 64)) != cudaSuccess) return e;
+  if ((e = make_map(&tb, P.h1b, H, n, (uint64_t)H * 2, 64, 64)) != cudaSuccess) return e;
+  const int64_t tiles_m = (L + BM - 1) / BM;
+  int bn = H >= 256 ? 256 : H;
+  while (bn > 64 && tiles_m * (H / bn) < lc.sms) bn /= 2;
+  if (bn == 256) return run<256, true, true, TC_EPI_SGD>(lc, ta, tb, g, 1);
+  if (bn == 128) return run<128, true, true, TC_EPI_SGD>(lc, ta, tb, g, 1);
+  return run<64, true, true, TC_EPI_SGD>(lc, ta, tb, g, 1);
+}
+
 }  // namespace asgd

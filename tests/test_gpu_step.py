@@ -46,7 +46,7 @@ def _check(cfg, rep, g, loss, touched, lo, go, batch, precision):
     assert not W1g[off].any()
 
 
-@pytest.mark.parametrize("precision", ["fp32"])
+@pytest.mark.parametrize("precision", ["fp32", "bf16"])
 def test_step_tiny(precision):
     cfg = config("tiny")
     data = dataset("tiny")
@@ -54,7 +54,7 @@ def test_step_tiny(precision):
     _check(cfg, *_one_step(cfg, data, rows, precision), precision)
 
 
-@pytest.mark.parametrize("precision", ["fp32"])
+@pytest.mark.parametrize("precision", ["fp32", "bf16"])
 def test_step_eurlex_full_batch(precision):
     cfg = config("eurlex4k")
     data = dataset("eurlex4k")
@@ -62,7 +62,7 @@ def test_step_eurlex_full_batch(precision):
     _check(cfg, *_one_step(cfg, data, rows, precision), precision)
 
 
-@pytest.mark.parametrize("precision", ["fp32"])
+@pytest.mark.parametrize("precision", ["fp32", "bf16"])
 def test_step_ragged_and_empty_rows(precision):
     """Truncated batch (37 rows, Q9) with a feature-less row and a repeated row."""
     cfg = config("eurlex4k")
@@ -71,7 +71,7 @@ def test_step_ragged_and_empty_rows(precision):
     _check(cfg, *_one_step(cfg, data, rows, precision), precision)
 
 
-@pytest.mark.parametrize("precision", ["fp32"])
+@pytest.mark.parametrize("precision", ["fp32", "bf16"])
 def test_step_wiki10_skewed(precision):
     """Heavy nnz skew: rows of 10^3-10^4 entries span many K-1 pieces."""
     cfg = config("wiki10_31k")
@@ -83,13 +83,14 @@ def test_step_wiki10_skewed(precision):
     _check(cfg, *_one_step(cfg, data, rows, precision), precision)
 
 
-def test_step_is_deterministic():
+@pytest.mark.parametrize("precision", ["fp32", "bf16"])
+def test_step_is_deterministic(precision):
     cfg = config("eurlex4k")
     data = dataset("eurlex4k")
     rows = torch.as_tensor(sample_stream(cfg, 0, cfg.b_max), device="cuda")
     outs = []
     for _ in range(2):
-        rep = make_replica(cfg, data, "fp32")
+        rep = make_replica(cfg, data, precision)
         for _ in range(3):
             rep.step(rows, 0.5)
         rep.sync()
