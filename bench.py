@@ -215,16 +215,24 @@ def main():
     rows_d = [torch.as_tensor(x, device=dev) for x in ids[:W + K]]
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
+    # warm-up with every kernel class timed: picks the dominant kernel, whose
+    # launches alone are then timed live in the timed region (2 events/step).
+    call = _lib.call
+    NCLS = len(_lib.PROF_NAMES)
+    call("asgd_profile", rep.ctx, (1 << NCLS) - 1)
     for mb in range(W):
         drv.megabatch(rows_d[mb])
     torch.cuda.synchronize()
+    wms = np.zeros(NCLS, dtype=np.float64)
+    wcnt = np.zeros(NCLS, dtype=np.int64)
+    call("asgd_profile_read", rep.ctx, wms.ctypes.data, wcnt.ctypes.data)
+    dom = int(np.argmax(wms))
 
     # ---------------------------------------------------------------- timed
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    call = _lib.call
-    call("asgd_profile", rep.ctx, 1)
+    call("asgd_profile", rep.ctx, 1 << dom)
     l0 = rep.launches()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
     stats = []
@@ -236,8 +244,8 @@ def main():
             ev[k][1].record()
         torch.cuda.synchronize()
     launches = rep.launches() - l0
-    ms = np.zeros(10, dtype=np.float64)
-    cnt = np.zeros(10, dtype=np.int64)
+    ms = np.zeros(NCLS, dtype=np.float64)
+    cnt = np.zeros(NCLS, dtype=np.int64)
     call("asgd_profile_read", rep.ctx, ms.ctypes.data, cnt.ctypes.data)
     call("asgd_profile", rep.ctx, 0)
     t_ms = sum(e0.elapsed_time(e1) for e0, e1 in ev)
@@ -269,10 +277,9 @@ def main():
               "nlab": float(np.mean(lab_l)), "splitk": 0}
         from paper_conf_ipps_marws22_b200.api import _lib as L_
         names = L_.PROF_NAMES
-        per = {names[i]: {"ms_total": float(ms[i]), "launches": int(cnt[i]),
-                          "us_per_launch": float(ms[i] / cnt[i] * 1e3) if cnt[i] else None}
+        per = {names[i]: {"us_per_launch": round(float(wms[i] / wcnt[i] * 1e3), 3) if wcnt[i] else None,
+                          "launches": int(wcnt[i])}
                for i in range(len(names))}
-        dom = max(range(len(names)), key=lambda i: ms[i])
         dname = names[dom]
         kind, work = kernel_work(dname, cfg, bf16, wl)
         avg_s = ms[dom] / max(cnt[dom], 1) / 1e3
@@ -302,7 +309,7 @@ def main():
                        "inflight": a.inflight, "parallelism": f"dp{world} (model averaging)",
                        "mean_batch_nnz": round(wl["nnz"], 1), "mean_touched_rows": round(wl["U"], 1)},
             "roofline": roof,
-            "kernels": per,
+            "kernels_warmup_profile": per,
             "gpu_launches": int(launches),
             "clocks": clk.summary(),
             "e2e": e2e,

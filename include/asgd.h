@@ -253,10 +253,14 @@ int asgd_sync(asgd_ctx* ctx);
 /* Number of kernels this ctx launched so far (for the bench's gpu_launches). */
 int asgd_kernel_launches(const asgd_ctx* ctx, int64_t* out);
 
-/* Live per-kernel timing with CUDA events recorded on the ctx stream around
- * every launch of a kernel class (for the bench's roofline).  enable != 0
- * starts (and resets) recording; asgd_profile_read is synchronous and returns
- * per class the summed milliseconds and the number of timed launches. */
+/* Live per-kernel timing with CUDA events recorded on the launching stream
+ * around every launch of the kernel classes in class_mask (bit k = class k,
+ * ASGD_PROF_ALL = all; 0 = off) -- for the bench's roofline.  Starting resets
+ * the counters; asgd_profile_read is synchronous and returns per class the
+ * summed milliseconds and the number of timed launches.  K-0 (class
+ * ASGD_K_TOUCHED) runs on the ctx's internal side stream, overlapped with
+ * K-1..G3, and is joined back before K-5. */
+#define ASGD_PROF_ALL 0x3ff
 #define ASGD_K_TOUCHED 0   /* K-0: batch scan, count, scan, place, segment sort */
 #define ASGD_K_SPMM 1      /* K-1: X W1 + b1, ReLU                              */
 #define ASGD_K_G1 2        /* Z = H1 W2^T + b2                                  */
@@ -268,7 +272,7 @@ int asgd_kernel_launches(const asgd_ctx* ctx, int64_t* out);
 #define ASGD_K_SCATTER 8   /* K-5 scatter-SGD on touched W1 rows                */
 #define ASGD_K_MERGE 9     /* K-6 / K-7: sqnorm, prescale, momentum epilogue    */
 #define ASGD_PROF_N 10
-int asgd_profile(asgd_ctx* ctx, int32_t enable);
+int asgd_profile(asgd_ctx* ctx, int32_t class_mask);
 int asgd_profile_read(asgd_ctx* ctx, double* ms_out, int64_t* count_out);
 
 /* Async copy device -> host (pinned) on the ctx stream (e2e result read). */

@@ -105,6 +105,7 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.z = take((size_t)B * Lp * 4);
   L.dzb = take(bf ? (size_t)B * Lp * 2 : 0);
   L.b2part = take((size_t)b2_chunks() * Lb * 4);
+  L.rbase = take((size_t)(B + 1) * 8);
   L.rowloss = take(B * 4);
   L.dhpart = take((size_t)L.splitk * B * H * 4);
   L.da1 = take(B * H * 4);
@@ -129,6 +130,7 @@ Ptrs ws_ptrs(char* b, const WsLayout& L) {
   p.db1part = (float*)(b + L.db1part); p.w2b = (bf16*)(b + L.w2b); p.red = (double*)(b + L.red);
   p.eval_top = (int32_t*)(b + L.eval_top);
   p.b2part = (float*)(b + L.b2part);
+  p.rbase = (int64_t*)(b + L.rbase);
   return p;
 }
 
@@ -154,18 +156,21 @@ struct asgd_ctx {
   int64_t launches;
   int64_t Pn;
   int64_t o_w1, o_b1, o_w2, o_b2;
-  bool prof_on = false;
+  uint32_t prof_mask = 0;                        // kernel classes timed with events
   std::vector<cudaEvent_t> pev[ASGD_PROF_N];   // (start, end) pairs
   size_t pused[ASGD_PROF_N] = {};
+  cudaStream_t s2 = nullptr;                     // side stream: K-0 overlaps the dense chain
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   Launch lc() { return Launch{s, &launches, sms}; }
+  Launch lc2() { return Launch{s2, &launches, sms}; }
 };
 
 namespace {
 constexpr size_t kMaxProfPairs = 8192;
 
-// Record an event on the ctx stream at the start / end of a kernel-class section.
-void prof_mark(asgd_ctx* c, int cls, bool begin) {
-  if (!c->prof_on) return;
+// Record an event on stream st at the start / end of a kernel-class section.
+void prof_mark(asgd_ctx* c, int cls, bool begin, cudaStream_t st) {
+  if (!(c->prof_mask & (1u << cls))) return;
   auto& v = c->pev[cls];
   size_t& u = c->pused[cls];
   if (begin) {
@@ -177,22 +182,23 @@ void prof_mark(asgd_ctx* c, int cls, bool begin) {
       v.push_back(a);
       v.push_back(b);
     }
-    cudaEventRecord(v[2 * u], c->s);
+    cudaEventRecord(v[2 * u], st);
   } else {
     if (u >= kMaxProfPairs || v.size() < 2 * (u + 1)) return;
-    cudaEventRecord(v[2 * u + 1], c->s);
+    cudaEventRecord(v[2 * u + 1], st);
     ++u;
   }
 }
 }  // namespace
 
-#define PCU(cls, call)                                      \
+#define PCU_ON(st, cls, call)                               \
   do {                                                      \
-    prof_mark(c, cls, true);                                \
+    prof_mark(c, cls, true, st);                            \
     cudaError_t _e = (call);                                \
-    prof_mark(c, cls, false);                               \
+    prof_mark(c, cls, false, st);                           \
     if (_e != cudaSuccess) return cuda_fail(_e, #call);     \
   } while (0)
+#define PCU(cls, call) PCU_ON(c->s, cls, call)
 
 extern "C" {
 
@@ -252,19 +258,26 @@ int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device, v
   c->o_w2 = c->o_b1 + m.H;
   c->o_b2 = c->o_w2 + m.L * m.H;
   c->Pn = c->o_b2 + m.L;
-  cudaError_t e = cudaMemsetAsync(c->ws, 0, c->L.total, c->s);
+  cudaError_t e = cudaStreamCreateWithFlags(&c->s2, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->ws, 0, c->L.total, c->s);
   if (e == cudaSuccess && m.precision == ASGD_PREC_BF16)
     e = launch_to_bf16(c->lc(), c->params + c->o_w2, c->P.w2b, m.L * m.H);
   if (e == cudaSuccess) e = cudaStreamSynchronize(c->s);
-  if (e != cudaSuccess) { delete c; return cuda_fail(e, "replica_init"); }
+  if (e != cudaSuccess) { asgd_replica_destroy(c); return cuda_fail(e, "replica_init"); }
   *out = c;
   return ASGD_OK;
 }
 
 int asgd_replica_destroy(asgd_ctx* c) {
-  if (c)
+  if (c) {
     for (auto& v : c->pev)
       for (cudaEvent_t e : v) cudaEventDestroy(e);
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
+    if (c->s2) cudaStreamDestroy(c->s2);
+  }
   delete c;
   return ASGD_OK;
 }
@@ -338,12 +351,12 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
   float* b2 = c->params + c->o_b2;
   float* g = c->dbg;
   if (g) CU(cudaMemsetAsync(g, 0, c->Pn * sizeof(float), c->s));
-  // K-0: batch view + touched-feature set
-  PCU(ASGD_K_TOUCHED, ([&]() -> cudaError_t {
-        cudaError_t e = launch_batch_scan(lc, rows, n, x.row_ptr, x.lab_ptr, x.n_rows, P, c->L.nz_cap,
-                                          c->L.nl_cap);
-        return e != cudaSuccess ? e : launch_touched(lc, rows, n, x.row_ptr, x.col, x.val, m.F, P, c->L, m.b_max);
-      })());
+  // K-0 (a): batch view; (b-f): touched-feature set on the side stream, joined before K-5
+  CU(launch_batch_scan(lc, rows, n, x.row_ptr, x.lab_ptr, x.n_rows, P, c->L.nz_cap, c->L.nl_cap));
+  CU(cudaEventRecord(c->ev_fork, c->s));
+  CU(cudaStreamWaitEvent(c->s2, c->ev_fork, 0));
+  PCU_ON(c->s2, ASGD_K_TOUCHED, launch_touched(c->lc2(), rows, n, x.row_ptr, x.col, x.val, m.F, P, c->L, m.b_max));
+  CU(cudaEventRecord(c->ev_join, c->s2));
   // K-1
   PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, rows, n, x.row_ptr, x.col, x.val, W1, b1, H, P, c->L, bf));
   if (!bf) {
@@ -364,15 +377,15 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     a.part_stride = c->L.part_stride;
     PCU(ASGD_K_G2, launch_gemm_f32(lc, a));
   } else {
-    PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, P, c->L, W2, b2, nullptr));
+    PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, P, c->L, W2, b2, nullptr, nullptr));
     PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, true));
-    PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, lr, P, c->L, W2, b2, nullptr));
+    PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, lr, P, c->L, W2, b2, nullptr, nullptr));
   }
   PCU(ASGD_K_DH, ([&]() -> cudaError_t {
         cudaError_t e = launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L);
         return e != cudaSuccess ? e : launch_b1_update(lc, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev);
       })());
-  PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, Lp, b2, lr, P, bf, g ? g + c->o_b2 : nullptr));
+  if (!bf) PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, Lp, b2, lr, P, false, g ? g + c->o_b2 : nullptr));
   if (!bf) {
     // G3: W2 -= lr dZ^T H1
     GemmArgs a{};
@@ -383,9 +396,11 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     a.splitk = 1;
     PCU(ASGD_K_G3, launch_gemm_f32(lc, a));
   } else {
-    PCU(ASGD_K_G3, launch_gemm_tc(lc, 3, n, Lb, H, lr, P, c->L, W2, b2, g ? g + c->o_w2 : nullptr));
+    PCU(ASGD_K_G3, launch_gemm_tc(lc, 3, n, Lb, H, lr, P, c->L, W2, b2, g ? g + c->o_w2 : nullptr,
+                                  g ? g + c->o_b2 : nullptr));
   }
-  // K-5
+  // K-5 (needs K-0's segments)
+  CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
   PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr));
   ++c->u;
   return ASGD_OK;
@@ -475,7 +490,7 @@ int asgd_eval_topk(asgd_ctx* c, const asgd_csr* t, const int32_t* rows, int32_t 
       a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = padded_ld(m.L); a.bias = b2; a.splitk = 1;
       CU(launch_gemm_f32(lc, a));
     } else {
-      CU(launch_gemm_tc(lc, 1, nb, m.L, H, 0.f, P, c->L, W2, b2, nullptr));
+      CU(launch_gemm_tc(lc, 1, nb, m.L, H, 0.f, P, c->L, W2, b2, nullptr, nullptr));
     }
     CU(launch_topk(lc, nb, m.L, padded_ld(m.L), k, P.z, topk + (int64_t)r0 * k));
   }
@@ -502,9 +517,9 @@ int asgd_kernel_launches(const asgd_ctx* c, int64_t* out) {
   return ASGD_OK;
 }
 
-int asgd_profile(asgd_ctx* c, int32_t enable) {
+int asgd_profile(asgd_ctx* c, int32_t class_mask) {
   if (!c) return fail(ASGD_E_ARG, "null ctx");
-  c->prof_on = enable != 0;
+  c->prof_mask = (uint32_t)class_mask & ((1u << ASGD_PROF_N) - 1);
   for (int k = 0; k < ASGD_PROF_N; ++k) c->pused[k] = 0;
   return ASGD_OK;
 }
@@ -512,6 +527,7 @@ int asgd_profile(asgd_ctx* c, int32_t enable) {
 int asgd_profile_read(asgd_ctx* c, double* ms, int64_t* cnt) {
   if (!c || !ms || !cnt) return fail(ASGD_E_ARG, "null argument");
   CU(cudaStreamSynchronize(c->s));
+  CU(cudaStreamSynchronize(c->s2));
   for (int k = 0; k < ASGD_PROF_N; ++k) {
     double t = 0.0;
     for (size_t i = 0; i < c->pused[k]; ++i) {

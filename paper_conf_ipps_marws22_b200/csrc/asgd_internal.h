@@ -13,9 +13,9 @@ constexpr int kPiece = 32;
 // Max labels per row the softmax kernel stages in shared memory.
 constexpr int kMaxRowLabels = 1024;
 // Features per tile of the touched-feature scan.
-constexpr int kScanTile = 4096;
+constexpr int kScanTile = 1024;
 // meta[] slots (int32, device)
-enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_COUNT = 8 };
+enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_COUNT = 8 };
 // error bits in meta[M_ERR]
 enum { ERR_NNZ_CAP = 1, ERR_LAB_CAP = 2, ERR_ROW_ID = 4 };
 
@@ -25,7 +25,7 @@ typedef __nv_bfloat16 bf16;
 struct WsLayout {
   size_t meta, boff, loff, cnt, fseg, fuid, uniq, useg, tsum, tpre;
   size_t e_n, e_v, e_u, part1, rowcnt, part5, ucnt;
-  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, red, eval_top, b2part;
+  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, red, eval_top, b2part, rbase;
   size_t total;
   int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride;
 };
@@ -38,6 +38,7 @@ struct Ptrs {  // typed views of the workspace
   int32_t* e_n; float* e_v; int32_t* e_u; float* part1; int32_t* rowcnt; float* part5;
   int32_t* ucnt; float* h1; bf16* h1b; float* z; bf16* dzb; float* rowloss; float* dhpart;
   float* da1; float* db1part; bf16* w2b; double* red; int32_t* eval_top; float* b2part;
+  int64_t* rbase;   // row_ptr[rows[r]] of the current batch (written by K-0 (a))
 };
 int row_block();   // rows per db1 partial (kernels_dense.cu)
 int b2_chunks();   // row chunks of the db2 partial sums
@@ -91,8 +92,11 @@ cudaError_t launch_b2_update(const Launch&, int n, int64_t L, int64_t ldz, float
 cudaError_t launch_to_bf16(const Launch&, const float* src, bf16* dst, int64_t count);
 // ---------------------------------------------------------------- tcgen05 (bf16)
 bool tc_available();
+// which: 1 = G1 (Z = H1 W2^T + b2), 2 = G2 (dH1 split-K partials), 3 = G3 (W2 -= lr dZ^T H1 and
+// b2 -= lr 1^T dZ, both fused in the epilogue)
 cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int H, float lr,
-                           const Ptrs&, const WsLayout&, float* W2, const float* b2, float* grad_w2);
+                           const Ptrs&, const WsLayout&, float* W2, float* b2, float* grad_w2,
+                           float* grad_b2);
 // ---------------------------------------------------------------- merge / eval
 cudaError_t launch_sqnorm(const Launch&, const float* x, int64_t P, double* partials, int nparts,
                           double* out);

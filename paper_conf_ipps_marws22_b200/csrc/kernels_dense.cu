@@ -156,60 +156,52 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
 }
 
 // ------------------------------------------------------ dH1 reduce + ReLU'
-// dA1[r][c] = [H1[r][c] > 0] * sum_z part[z][r][c];  db1 partial per block of kRowBlk rows.
-// One thread per column (blockDim = H), so every sum has a fixed order.
-constexpr int kRowBlk = 4;
+// dA1[r][c] = [H1[r][c] > 0] * sum_z part[z][r][c]: one thread per element, its
+// split-K loads all in flight; fixed summation order (deterministic).
 __global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
-                            const float* __restrict__ part, const float* __restrict__ H1,
-                            float* dA1, float* db1part) {
-  const int c = threadIdx.x;
-  const int r0 = blockIdx.x * kRowBlk;
-  float colsum = 0.f;
+                            const float* __restrict__ part, const float* __restrict__ H1, float* dA1) {
+  const int r = blockIdx.x, c = threadIdx.x;
+  const int64_t o = (int64_t)r * H + c;
+  float a[8];
 #pragma unroll
-  for (int rr = 0; rr < kRowBlk; ++rr) {
-    const int r = r0 + rr;
-    if (r >= n) break;
-    const int64_t o = (int64_t)r * H + c;
-    float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
-    int z = 0;
-    for (; z + 4 <= splitk; z += 4) {
-      s0 += __ldcs(part + z * part_stride + o);
-      s1 += __ldcs(part + (z + 1) * part_stride + o);
-      s2 += __ldcs(part + (z + 2) * part_stride + o);
-      s3 += __ldcs(part + (z + 3) * part_stride + o);
-    }
-    for (; z < splitk; ++z) s0 += __ldcs(part + z * part_stride + o);
-    const float s = (s0 + s1) + (s2 + s3);
-    const float v = H1[o] > 0.f ? s : 0.f;
-    dA1[o] = v;
-    colsum += v;
+  for (int q = 0; q < 8; ++q) a[q] = 0.f;
+  for (int z = 0; z < splitk; z += 8) {
+#pragma unroll
+    for (int q = 0; q < 8; ++q)
+      if (z + q < splitk) a[q] += __ldcs(part + (int64_t)(z + q) * part_stride + o);
   }
-  db1part[(int64_t)blockIdx.x * H + c] = colsum;
+  const float s = ((a[0] + a[1]) + (a[2] + a[3])) + ((a[4] + a[5]) + (a[6] + a[7]));
+  dA1[o] = H1[o] > 0.f ? s : 0.f;
 }
 
-// b1 -= lr * sum_blocks db1part (blockDim = H), mean loss = sum rowloss / n.
-__global__ void k_b1_update(int n, int H, int nblk, const float* __restrict__ db1part, float* b1,
-                            float lr, float* grad_b1, const float* __restrict__ rowloss,
-                            float* loss_dev) {
-  const int c = threadIdx.x;
-  float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
-  int b = 0;
-  for (; b + 4 <= nblk; b += 4) {
-    a0 += db1part[(int64_t)b * H + c];
-    a1 += db1part[(int64_t)(b + 1) * H + c];
-    a2 += db1part[(int64_t)(b + 2) * H + c];
-    a3 += db1part[(int64_t)(b + 3) * H + c];
-  }
-  for (; b < nblk; ++b) a0 += db1part[(int64_t)b * H + c];
-  const float s = (a0 + a1) + (a2 + a3);
-  b1[c] -= lr * s;
-  if (grad_b1) grad_b1[c] = s;
-  if (loss_dev && threadIdx.x < 32) {
+// db1[c] = sum_r dA1[r][c] (one warp per column, lanes over rows, fixed shuffle
+// tree); b1 -= lr db1.  The extra last warp computes the mean loss.
+__global__ void __launch_bounds__(256) k_b1_update(int n, int H, const float* __restrict__ dA1, float* b1,
+                                                   float lr, float* grad_b1,
+                                                   const float* __restrict__ rowloss, float* loss_dev) {
+  const int lane = threadIdx.x & 31;
+  const int c = blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (c < H) {
+    float t[4] = {0.f, 0.f, 0.f, 0.f};
+    int r = lane;
+    for (; r + 96 < n; r += 128) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) t[q] += dA1[(int64_t)(r + 32 * q) * H + c];
+    }
+    for (; r < n; r += 32) t[0] += dA1[(int64_t)r * H + c];
+    float v = (t[0] + t[1]) + (t[2] + t[3]);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+    if (lane == 0) {
+      b1[c] -= lr * v;
+      if (grad_b1) grad_b1[c] = v;
+    }
+  } else if (c == H && loss_dev) {
     float t = 0.f;
-    for (int r = threadIdx.x; r < n; r += 32) t += rowloss[r];
+    for (int r = lane; r < n; r += 32) t += rowloss[r];
 #pragma unroll
     for (int o = 16; o; o >>= 1) t += __shfl_xor_sync(kFull, t, o);
-    if (threadIdx.x == 0) *loss_dev = t / (float)n;
+    if (lane == 0) *loss_dev = t / (float)n;
   }
 }
 
@@ -277,17 +269,15 @@ cudaError_t launch_softmax_ce(const Launch& lc, int n, int64_t L, int64_t ldz, c
 
 cudaError_t launch_dh_reduce(const Launch& lc, int n, int H, int splitk, const Ptrs& P,
                              const WsLayout& L) {
-  const int nblk = (n + kRowBlk - 1) / kRowBlk;
   // split-K partial z of dH1 lives at dhpart + z * (b_max * H)
-  k_dh_reduce<<<nblk, H, 0, lc.s>>>(n, H, splitk, L.part_stride, P.dhpart, P.h1, P.da1, P.db1part);
+  k_dh_reduce<<<n, H, 0, lc.s>>>(n, H, splitk, L.part_stride, P.dhpart, P.h1, P.da1);
   ++*lc.counter;
   return cudaGetLastError();
 }
 
 cudaError_t launch_b1_update(const Launch& lc, int n, int H, float* b1, float lr, const Ptrs& P,
                              const WsLayout& L, float* grad_b1, float* loss_dev) {
-  const int nblk = (n + kRowBlk - 1) / kRowBlk;
-  k_b1_update<<<1, H, 0, lc.s>>>(n, H, nblk, P.db1part, b1, lr, grad_b1, P.rowloss, loss_dev);
+  k_b1_update<<<H / 8 + 1, 256, 0, lc.s>>>(n, H, P.da1, b1, lr, grad_b1, P.rowloss, loss_dev);
   ++*lc.counter;
   return cudaGetLastError();
 }
@@ -309,7 +299,7 @@ cudaError_t launch_to_bf16(const Launch& lc, const float* src, bf16* dst, int64_
   return cudaGetLastError();
 }
 
-int row_block() { return kRowBlk; }
+int row_block() { return 1; }
 int b2_chunks() { return kB2Chunks; }
 
 }  // namespace asgd

@@ -10,6 +10,8 @@
 // rows reach 10^4 nnz) spans many warps.  Segments spanning pieces are
 // combined by the last-arriving warp in piece order, so every sum has a
 // fixed order: results are bitwise deterministic.
+#include <algorithm>
+
 #include "asgd_internal.h"
 
 namespace asgd {
@@ -118,7 +120,7 @@ __global__ void __launch_bounds__(1024) k_batch_scan(const int32_t* __restrict__
                                                      const int64_t* __restrict__ lab_ptr,
                                                      int64_t n_data_rows, int32_t* boff,
                                                      int32_t* loff, int32_t* meta, int64_t nz_cap,
-                                                     int64_t nl_cap) {
+                                                     int64_t nl_cap, int64_t* rbase) {
   __shared__ long long wf[32], wl[32];
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
   const int per = (n + blockDim.x - 1) / blockDim.x;
@@ -157,6 +159,7 @@ __global__ void __launch_bounds__(1024) k_batch_scan(const int32_t* __restrict__
     boff[r] = (int32_t)min(pf, (long long)nz_cap);
     loff[r] = (int32_t)min(pl, (long long)nl_cap);
     int64_t id = rows[r];
+    rbase[r] = (id < 0 || id >= n_data_rows) ? 0 : row_ptr[id];
     if (id < 0 || id >= n_data_rows) continue;
     pf += row_ptr[id + 1] - row_ptr[id];
     pl += lab_ptr[id + 1] - lab_ptr[id];
@@ -176,113 +179,122 @@ __global__ void __launch_bounds__(1024) k_batch_scan(const int32_t* __restrict__
   }
 }
 
-// map a flat batch entry e to its dataset index; returns row in *r
-__device__ __forceinline__ int64_t entry_index(const int32_t* sboff, int n,
-                                               const int32_t* __restrict__ rows,
-                                               const int64_t* __restrict__ row_ptr, int e, int* r) {
-  int rr = entry_row(sboff, n, e);
-  *r = rr;
-  return row_ptr[rows[rr]] + (e - sboff[rr]);
+// Batch view in shared memory: sboff[n + 1] entry offsets, then srbase[n] (8-byte
+// aligned) = row_ptr[rows[r]], both written by K-0 (a).
+__host__ __device__ __forceinline__ size_t view_smem(int n) {
+  return (((size_t)(n + 1) * 4 + 7) & ~size_t(7)) + (size_t)n * 8;
+}
+__device__ __forceinline__ const int64_t* view_rbase(const int32_t* sboff, int n) {
+  return reinterpret_cast<const int64_t*>(reinterpret_cast<const char*>(sboff) + (((size_t)(n + 1) * 4 + 7) & ~size_t(7)));
 }
 
-__device__ __forceinline__ void load_boff(int32_t* sboff, const int32_t* boff, int n) {
+// map a flat batch entry e to its dataset index; returns row in *r
+__device__ __forceinline__ int64_t entry_index(const int32_t* sboff, int n, int e, int* r) {
+  int rr = entry_row(sboff, n, e);
+  *r = rr;
+  return view_rbase(sboff, n)[rr] + (e - sboff[rr]);
+}
+
+__device__ __forceinline__ void load_view(int32_t* sboff, const int32_t* boff, const int64_t* rbase, int n) {
+  int64_t* srb = const_cast<int64_t*>(view_rbase(sboff, n));
   for (int i = threadIdx.x; i <= n; i += blockDim.x) sboff[i] = boff[i];
+  for (int i = threadIdx.x; i < n; i += blockDim.x) srb[i] = rbase[i];
   __syncthreads();
 }
 
-// K-0 (b): cnt[f] += 1 for every batch entry
-__global__ void k_count(const int32_t* __restrict__ rows, int n, const int64_t* __restrict__ row_ptr,
+// K-0 (b): cnt[f] += 1 for every batch entry; CTA 0 also resets the scan's
+// tile-status words and tile ticket for k_fscan.
+__global__ void k_count(int n, const int64_t* __restrict__ rbase,
                         const int32_t* __restrict__ col, const int32_t* __restrict__ boff,
-                        const int32_t* __restrict__ meta, int32_t* cnt) {
+                        int32_t* meta, int32_t* cnt, unsigned long long* status, int ntiles) {
   extern __shared__ int32_t sboff[];
-  load_boff(sboff, boff, n);
+  if (blockIdx.x == 0) {
+    for (int i = threadIdx.x; i < ntiles; i += blockDim.x) status[i] = 0ull;
+    if (threadIdx.x == 0) meta[M_TILE] = 0;
+  }
+  load_view(sboff, boff, rbase, n);
   const int nnz = meta[M_NNZ];
   for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x) {
     int r;
-    int64_t k = entry_index(sboff, n, rows, row_ptr, e, &r);
+    int64_t k = entry_index(sboff, n, e, &r);
     atomicAdd(&cnt[col[k]], 1);
   }
 }
 
-// K-0 (c): touched-feature scan over F in tiles: tsum[2t] = sum cnt, tsum[2t+1] = #touched
-__global__ void __launch_bounds__(256) k_fscan_tile(const int32_t* __restrict__ cnt, int64_t F,
-                                                    int32_t* tsum) {
-  __shared__ int s0[8], s1[8];
-  const int64_t base = (int64_t)blockIdx.x * kScanTile;
-  int a = 0, b = 0;
-  for (int i = threadIdx.x; i < kScanTile; i += 256) {
-    int64_t f = base + i;
-    if (f < F) { int c = cnt[f]; a += c; b += (c > 0); }
-  }
-#pragma unroll
-  for (int o = 16; o; o >>= 1) { a += __shfl_xor_sync(kFull, a, o); b += __shfl_xor_sync(kFull, b, o); }
-  if ((threadIdx.x & 31) == 0) { s0[threadIdx.x >> 5] = a; s1[threadIdx.x >> 5] = b; }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    int x = 0, y = 0;
-    for (int w = 0; w < 8; ++w) { x += s0[w]; y += s1[w]; }
-    tsum[2 * blockIdx.x] = x;
-    tsum[2 * blockIdx.x + 1] = y;
-  }
+// K-0 (c): single-pass scan over F (decoupled look-back, tiles of kScanTile
+// features in ticket order).  Per touched feature f: fseg[f] = segment start,
+// fuid[f] = its rank u; uniq[u] = f and useg[u] = segment start (sorted by f).
+// Status word: flag (2 bits: 1 aggregate, 2 inclusive prefix) | count (31) | touched (31).
+constexpr unsigned long long kFlagAgg = 1ull << 62, kFlagPre = 2ull << 62;
+__device__ __forceinline__ unsigned long long pack_st(unsigned long long flag, int a, int b) {
+  return flag | ((unsigned long long)(unsigned)a << 31) | (unsigned long long)(unsigned)b;
 }
 
-// exclusive scan of the tile sums (one CTA, sequential over <= a few thousand tiles)
-__global__ void k_fscan_top(const int32_t* __restrict__ tsum, int ntiles, int32_t* tpre,
-                            int32_t* meta) {
-  __shared__ int sa[1024], sb[1024];
-  // each thread owns a contiguous chunk of tiles
-  const int t = threadIdx.x, per = (ntiles + blockDim.x - 1) / blockDim.x;
-  const int i0 = min(ntiles, t * per), i1 = min(ntiles, i0 + per);
-  int a = 0, b = 0;
-  for (int i = i0; i < i1; ++i) { a += tsum[2 * i]; b += tsum[2 * i + 1]; }
-  sa[t] = a; sb[t] = b;
-  __syncthreads();
-  if (t == 0) {
-    int x = 0, y = 0;
-    for (int j = 0; j < (int)blockDim.x; ++j) {
-      int ta = sa[j], tb = sb[j];
-      sa[j] = x; sb[j] = y;
-      x += ta; y += tb;
-    }
-    meta[M_U] = y;
-  }
-  __syncthreads();
-  a = sa[t]; b = sb[t];
-  for (int i = i0; i < i1; ++i) {
-    tpre[2 * i] = a; tpre[2 * i + 1] = b;
-    a += tsum[2 * i]; b += tsum[2 * i + 1];
-  }
-}
-
-// K-0 (d): write segment starts / unique ids
-__global__ void __launch_bounds__(256) k_fscan_write(const int32_t* __restrict__ cnt, int64_t F,
-                                                     const int32_t* __restrict__ tpre,
-                                                     const int32_t* __restrict__ meta,
-                                                     int32_t* fseg, int32_t* fuid, int32_t* uniq,
-                                                     int32_t* useg) {
-  // each thread scans 16 consecutive features; block scan of the thread sums
+__global__ void __launch_bounds__(256) k_fscan(const int32_t* __restrict__ cnt, int64_t F,
+                                               unsigned long long* status, int ntiles, int32_t* meta,
+                                               int32_t* fseg, int32_t* fuid, int32_t* uniq,
+                                               int32_t* useg) {
   constexpr int PER = kScanTile / 256;
-  __shared__ int sa[256], sb[256];
-  const int64_t f0 = (int64_t)blockIdx.x * kScanTile + threadIdx.x * PER;
+  __shared__ int s_tile, s_pa, s_pb;
+  __shared__ int wa[8], wb[8];
+  if (threadIdx.x == 0) s_tile = atomicAdd(&meta[M_TILE], 1);
+  __syncthreads();
+  const int t = s_tile;
+  const int64_t f0 = (int64_t)t * kScanTile + threadIdx.x * PER;
   int c[PER];
   int a = 0, b = 0;
 #pragma unroll
   for (int i = 0; i < PER; ++i) {
     c[i] = (f0 + i < F) ? cnt[f0 + i] : 0;
-    a += c[i]; b += (c[i] > 0);
+    a += c[i];
+    b += (c[i] > 0);
   }
-  sa[threadIdx.x] = a; sb[threadIdx.x] = b;
+  // block exclusive scan of (a, b)
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  int xa = a, xb = b;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int ya = __shfl_up_sync(kFull, xa, o), yb = __shfl_up_sync(kFull, xb, o);
+    if (lane >= o) { xa += ya; xb += yb; }
+  }
+  if (lane == 31) { wa[wid] = xa; wb[wid] = xb; }
   __syncthreads();
-  // Hillis-Steele inclusive scan over 256 entries
-  for (int o = 1; o < 256; o <<= 1) {
-    int xa = threadIdx.x >= o ? sa[threadIdx.x - o] : 0;
-    int xb = threadIdx.x >= o ? sb[threadIdx.x - o] : 0;
-    __syncthreads();
-    sa[threadIdx.x] += xa; sb[threadIdx.x] += xb;
-    __syncthreads();
+  int oa = 0, ob = 0, ta = 0, tb = 0;
+#pragma unroll
+  for (int w = 0; w < 8; ++w) {
+    if (w < wid) { oa += wa[w]; ob += wb[w]; }
+    ta += wa[w]; tb += wb[w];
   }
-  int pa = tpre[2 * blockIdx.x] + sa[threadIdx.x] - a;
-  int pb = tpre[2 * blockIdx.x + 1] + sb[threadIdx.x] - b;
+  if (threadIdx.x == 0) {
+    volatile unsigned long long* st = status;
+    if (t == 0) {
+      st[0] = pack_st(kFlagPre, ta, tb);
+      s_pa = 0; s_pb = 0;
+    } else {
+      st[t] = pack_st(kFlagAgg, ta, tb);
+      __threadfence();
+      int pa = 0, pb = 0;
+      for (int j = t - 1; j >= 0;) {
+        const unsigned long long v = st[j];
+        const unsigned long long flag = v & (3ull << 62);
+        if (!flag) continue;   // predecessor not published yet
+        pa += (int)((v >> 31) & 0x7fffffffull);
+        pb += (int)(v & 0x7fffffffull);
+        if (flag == kFlagPre) break;
+        --j;
+      }
+      __threadfence();
+      st[t] = pack_st(kFlagPre, pa + ta, pb + tb);
+      s_pa = pa; s_pb = pb;
+    }
+    if (t == ntiles - 1) {
+      meta[M_U] = s_pb + tb;
+      useg[s_pb + tb] = s_pa + ta;   // == batch nnz
+    }
+  }
+  __syncthreads();
+  int pa = s_pa + oa + (xa - a);   // exclusive prefix of this thread
+  int pb = s_pb + ob + (xb - b);
 #pragma unroll
   for (int i = 0; i < PER; ++i) {
     if (c[i] > 0) {
@@ -294,21 +306,20 @@ __global__ void __launch_bounds__(256) k_fscan_write(const int32_t* __restrict__
     }
     pa += c[i];
   }
-  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) useg[meta[M_U]] = meta[M_NNZ];
 }
 
 // K-0 (e): scatter entries into their feature segment (cnt returns to zero)
-__global__ void k_place(const int32_t* __restrict__ rows, int n, const int64_t* __restrict__ row_ptr,
+__global__ void k_place(int n, const int64_t* __restrict__ rbase,
                         const int32_t* __restrict__ col, const float* __restrict__ val,
                         const int32_t* __restrict__ boff, const int32_t* __restrict__ meta,
                         int32_t* cnt, const int32_t* __restrict__ fseg,
                         const int32_t* __restrict__ fuid, int32_t* e_n, float* e_v, int32_t* e_u) {
   extern __shared__ int32_t sboff[];
-  load_boff(sboff, boff, n);
+  load_view(sboff, boff, rbase, n);
   const int nnz = meta[M_NNZ];
   for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x) {
     int r;
-    int64_t k = entry_index(sboff, n, rows, row_ptr, e, &r);
+    int64_t k = entry_index(sboff, n, e, &r);
     int f = col[k];
     int pos = fseg[f] + atomicSub(&cnt[f], 1) - 1;
     e_n[pos] = r;
@@ -382,8 +393,7 @@ __global__ void k_segsort(const int32_t* __restrict__ useg, const int32_t* __res
 // K-1: A1 = X W1 + b1, H1 = ReLU(A1)
 // -------------------------------------------------------------------------
 template <int VPL>
-__global__ void __launch_bounds__(256) k_spmm_fwd(const int32_t* __restrict__ rows, int n,
-                                                  const int64_t* __restrict__ row_ptr,
+__global__ void __launch_bounds__(256) k_spmm_fwd(int n, const int64_t* __restrict__ rbase,
                                                   const int32_t* __restrict__ col,
                                                   const float* __restrict__ val,
                                                   const float* __restrict__ W1,
@@ -393,8 +403,10 @@ __global__ void __launch_bounds__(256) k_spmm_fwd(const int32_t* __restrict__ ro
                                                   bf16* H1b, float* part, int32_t* rowcnt) {
   using IO = RowIO<VPL>;
   constexpr int H = 32 * VPL;
+  constexpr int kU = VPL >= 16 ? 4 : 8;   // W1 rows in flight per warp
   extern __shared__ int32_t sboff[];
-  load_boff(sboff, boff, n);
+  load_view(sboff, boff, rbase, n);
+  const int64_t* srb = view_rbase(sboff, n);
   const int lane = threadIdx.x & 31;
   const int nnz = meta[M_NNZ];
   const int npieces = (nnz + kPiece - 1) / kPiece;
@@ -412,21 +424,21 @@ __global__ void __launch_bounds__(256) k_spmm_fwd(const int32_t* __restrict__ ro
       float acc[VPL];
 #pragma unroll
       for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
-      const int64_t base = row_ptr[rows[r]] - rs;   // dataset index of flat entry e: base + e
+      const int64_t base = srb[r] - rs;   // dataset index of flat entry e: base + e
       const int cnt = se - e;                        // <= kPiece = 32
       int mycol = 0;
       float myval = 0.f;
       if (lane < cnt) { mycol = __ldg(col + base + e + lane); myval = __ldg(val + base + e + lane); }
       int j = 0;
-      for (; j + 4 <= cnt; j += 4) {
-        float w[4][VPL];
+      for (; j + kU <= cnt; j += kU) {
+        float w[kU][VPL];
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
+        for (int q = 0; q < kU; ++q) {
           int c = __shfl_sync(kFull, mycol, j + q);
           IO::load_ldg(W1 + (int64_t)c * H, lane, w[q]);
         }
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
+        for (int q = 0; q < kU; ++q) {
           float v = __shfl_sync(kFull, myval, j + q);
 #pragma unroll
           for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, w[q][i], acc[i]);
@@ -502,6 +514,7 @@ __global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__
                                                      float* grad_w1) {
   using IO = RowIO<VPL>;
   constexpr int H = 32 * VPL;
+  constexpr int kU = VPL >= 16 ? 4 : 8;   // dA1 rows in flight per warp
   const int lane = threadIdx.x & 31;
   const int nnz = meta[M_NNZ];
   const int npieces = (nnz + kPiece - 1) / kPiece;
@@ -521,15 +534,15 @@ __global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__
       for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
       int j = e - e0;
       const int jend = se - e0;
-      for (; j + 4 <= jend; j += 4) {
-        float g[4][VPL];
+      for (; j + kU <= jend; j += kU) {
+        float g[kU][VPL];
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
+        for (int q = 0; q < kU; ++q) {
           int r = __shfl_sync(kFull, myn, j + q);
           IO::load_ldg(dA1 + (int64_t)r * H, lane, g[q]);
         }
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
+        for (int q = 0; q < kU; ++q) {
           float v = __shfl_sync(kFull, myv, j + q);
 #pragma unroll
           for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, g[q][i], acc[i]);
@@ -582,21 +595,34 @@ __global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__
   }
 }
 
+// One resident wave of 256-thread CTAs (occupancy from the compiled kernel), no
+// more CTAs than there are 8-piece groups for the largest step.
+template <typename K>
+int wave_grid(const Launch& lc, K kernel, size_t smem, int64_t pieces, int& occ) {
+  if (!occ && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, 256, smem) != cudaSuccess || occ < 1))
+    occ = 1;
+  const int64_t need = (pieces + 7) / 8;
+  return (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)lc.sms * occ));
+}
+
 template <int VPL>
 cudaError_t spmm_fwd_t(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
                        const int32_t* col, const float* val, const float* W1, const float* b1,
                        const Ptrs& P, const WsLayout& L, bool want_bf16) {
-  int grid = lc.sms * 8;
-  size_t smem = (size_t)(n + 1) * sizeof(int32_t);
-  k_spmm_fwd<VPL><<<grid, 256, smem, lc.s>>>(rows, n, row_ptr, col, val, W1, b1, P.boff, P.meta,
+  const size_t smem = view_smem(n);
+  static int occ = 0;
+  const int grid = wave_grid(lc, k_spmm_fwd<VPL>, view_smem(2048), L.n_pieces, occ);
+  k_spmm_fwd<VPL><<<grid, 256, smem, lc.s>>>(n, P.rbase, col, val, W1, b1, P.boff, P.meta,
                                              P.h1, want_bf16 ? P.h1b : nullptr, P.part1, P.rowcnt);
   ++*lc.counter;
   return cudaGetLastError();
 }
 
 template <int VPL>
-cudaError_t scatter_t(const Launch& lc, float* W1, float lr, const Ptrs& P, float* grad_w1) {
-  int grid = lc.sms * 8;
+cudaError_t scatter_t(const Launch& lc, float* W1, float lr, const Ptrs& P, const WsLayout& L,
+                      float* grad_w1) {
+  static int occ = 0;
+  const int grid = wave_grid(lc, k_scatter_sgd<VPL>, 0, L.n_pieces, occ);
   k_scatter_sgd<VPL><<<grid, 256, 0, lc.s>>>(P.e_n, P.e_v, P.e_u, P.useg, P.uniq, P.meta, P.da1,
                                              W1, lr, P.part5, P.ucnt, grad_w1);
   ++*lc.counter;
@@ -609,7 +635,7 @@ cudaError_t launch_batch_scan(const Launch& lc, const int32_t* rows, int n, cons
                               const int64_t* lab_ptr, int64_t n_data_rows, const Ptrs& P,
                               int64_t nz_cap, int64_t nl_cap) {
   k_batch_scan<<<1, 1024, 0, lc.s>>>(rows, n, row_ptr, lab_ptr, n_data_rows, P.boff, P.loff, P.meta,
-                                     nz_cap, nl_cap);
+                                     nz_cap, nl_cap, P.rbase);
   ++*lc.counter;
   return cudaGetLastError();
 }
@@ -617,19 +643,18 @@ cudaError_t launch_batch_scan(const Launch& lc, const int32_t* rows, int n, cons
 cudaError_t launch_touched(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
                            const int32_t* col, const float* val, int64_t F, const Ptrs& P,
                            const WsLayout& L, int b_max) {
-  const size_t smem = (size_t)(n + 1) * sizeof(int32_t);
+  const size_t smem = view_smem(n);
   const int grid = lc.sms * 4;
-  k_count<<<grid, 256, smem, lc.s>>>(rows, n, row_ptr, col, P.boff, P.meta, P.cnt);
   const int nt = (int)L.n_tiles_f;
-  k_fscan_tile<<<nt, 256, 0, lc.s>>>(P.cnt, F, P.tsum);
-  k_fscan_top<<<1, 1024, 0, lc.s>>>(P.tsum, nt, P.tpre, P.meta);
-  k_fscan_write<<<nt, 256, 0, lc.s>>>(P.cnt, F, P.tpre, P.meta, P.fseg, P.fuid, P.uniq, P.useg);
-  k_place<<<grid, 256, smem, lc.s>>>(rows, n, row_ptr, col, val, P.boff, P.meta, P.cnt, P.fseg,
+  unsigned long long* status = reinterpret_cast<unsigned long long*>(P.tsum);
+  k_count<<<grid, 256, smem, lc.s>>>(n, P.rbase, col, P.boff, P.meta, P.cnt, status, nt);
+  k_fscan<<<nt, 256, 0, lc.s>>>(P.cnt, F, status, nt, P.meta, P.fseg, P.fuid, P.uniq, P.useg);
+  k_place<<<grid, 256, smem, lc.s>>>(n, P.rbase, col, val, P.boff, P.meta, P.cnt, P.fseg,
                                      P.fuid, P.e_n, P.e_v, P.e_u);
   const int words = (b_max + 31) / 32;
   const size_t ssmem = (size_t)8 * words * 33 * sizeof(uint32_t);
   k_segsort<<<lc.sms * 2, 256, ssmem, lc.s>>>(P.useg, P.meta, P.e_n, P.e_v, words);
-  *lc.counter += 6;
+  *lc.counter += 4;
   return cudaGetLastError();
 }
 
@@ -648,10 +673,10 @@ cudaError_t launch_spmm_fwd(const Launch& lc, const int32_t* rows, int n, const 
 cudaError_t launch_scatter_sgd(const Launch& lc, float* W1, int H, float lr, const Ptrs& P,
                                const WsLayout& L, float* grad_w1) {
   switch (H) {
-    case 64: return scatter_t<2>(lc, W1, lr, P, grad_w1);
-    case 128: return scatter_t<4>(lc, W1, lr, P, grad_w1);
-    case 256: return scatter_t<8>(lc, W1, lr, P, grad_w1);
-    case 512: return scatter_t<16>(lc, W1, lr, P, grad_w1);
+    case 64: return scatter_t<2>(lc, W1, lr, P, L, grad_w1);
+    case 128: return scatter_t<4>(lc, W1, lr, P, L, grad_w1);
+    case 256: return scatter_t<8>(lc, W1, lr, P, L, grad_w1);
+    case 512: return scatter_t<16>(lc, W1, lr, P, L, grad_w1);
     default: return cudaErrorInvalidValue;
   }
 }

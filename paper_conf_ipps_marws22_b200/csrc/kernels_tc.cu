@@ -30,6 +30,7 @@ struct TcArgs {
   int64_t part_stride;                // split-K partial z offset
   const float* bias;                  // G1
   float lr; bf16* shadow; float* grad;// G3
+  float* b2; float* grad_b2;          // G3: db2 = dZ^T 1 via an extra N = 16 MMA on N-tile 0
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -129,12 +130,15 @@ template <int BN, bool A_MN, bool B_MN, int EPI>
 __global__ void __launch_bounds__(256, 1)
     k_gemm_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, TcArgs g) {
   constexpr uint32_t A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE = A_BYTES + B_BYTES;
-  constexpr uint32_t TMEM_COLS = BN;  // 64, 128 or 256 fp32 columns
+  constexpr bool ONES = (EPI == TC_EPI_SGD);           // db2 column
+  constexpr uint32_t TMEM_COLS = ONES ? 2 * BN : BN;   // power of two >= BN (+16)
+  constexpr uint32_t ONES_BYTES = ONES ? 16 * 128 : 0; // K-major 16 x 64 bf16 tile, row 0 = 1
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * A_BYTES;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * STAGE);
+  uint8_t* sOnes = smem + STAGES * STAGE;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * STAGE + ONES_BYTES);
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
   uint32_t* tbase = reinterpret_cast<uint32_t*>(tfull + 1);
@@ -158,6 +162,13 @@ __global__ void __launch_bounds__(256, 1)
                  "r"(TMEM_COLS)
                  : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  if constexpr (ONES) {
+    if (warp == 3) {   // row 0 = 64 x bf16(1.0) (unswizzled: row 0 of the atom), rows 1..15 = 0
+      uint32_t* p = reinterpret_cast<uint32_t*>(sOnes);
+      for (int i = lane; i < (int)(ONES_BYTES / 4); i += 32) p[i] = (i < 32) ? 0x3F803F80u : 0u;
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
   }
   tc_fence_before();
   __syncthreads();
@@ -193,6 +204,9 @@ __global__ void __launch_bounds__(256, 1)
     if (lane == 0) {
       // ------------------------------------------------ MMA issuer
       constexpr uint32_t idesc = make_idesc(BN, A_MN, B_MN);
+      constexpr uint32_t idesc1 = make_idesc(16, A_MN, false);
+      const bool ones = ONES && blockIdx.x == 0;
+      const uint32_t ones_base = smem_u32(sOnes);
       for (int i = 0; i < nk; ++i) {
         const int s = i % STAGES;
         const uint32_t ph = (i / STAGES) & 1;
@@ -206,6 +220,8 @@ __global__ void __launch_bounds__(256, 1)
           const uint64_t ad = A_MN ? desc_sw128(a_base + k * 2048, 8192, 1024) : desc_sw128(a_base + k * 32, 16, 1024);
           const uint64_t bd = B_MN ? desc_sw128(b_base + k * 2048, 8192, 1024) : desc_sw128(b_base + k * 32, 16, 1024);
           mma_bf16(tmem, ad, bd, idesc, (i > 0 || k > 0) ? 1u : 0u);
+          if (ONES && ones)   // TMEM column BN += dZ^T tile . e_0  (db2)
+            mma_bf16(tmem + BN, ad, desc_sw128(ones_base + k * 32, 16, 1024), idesc1, (i > 0 || k > 0) ? 1u : 0u);
         }
         mma_commit(&empty[s]);   // frees the smem stage once these MMAs retire
       }
@@ -268,6 +284,20 @@ __global__ void __launch_bounds__(256, 1)
         }
       }
     }
+    if constexpr (ONES) {
+      if (blockIdx.x == 0) {   // db2[m] = sum_n dZ[n, m]; b2 -= lr db2
+        float v[32];
+        if (nk > 0) {
+          tmem_ld32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)BN, v);
+        } else {
+          v[0] = 0.f;
+        }
+        if (m < g.M) {
+          g.b2[m] -= g.lr * v[0];
+          if (g.grad_b2) g.grad_b2[m] = v[0];
+        }
+      }
+    }
   }
   tc_fence_before();
   __syncthreads();
@@ -303,7 +333,7 @@ cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t 
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
 cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, const TcArgs& g, int splits) {
-  const size_t smem = (size_t)STAGES * (BM * BK * 2 + BN * BK * 2) + 1024 + 256;
+  const size_t smem = (size_t)STAGES * (BM * BK * 2 + BN * BK * 2) + (EPI == TC_EPI_SGD ? 2048 : 0) + 1024 + 256;
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(k_gemm_tc<BN, A_MN, B_MN, EPI>,
@@ -334,7 +364,7 @@ bool tc_available() {
 int64_t padded_ld(int64_t L) { return (L + 7) / 8 * 8; }
 
 cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H, float lr, const Ptrs& P,
-                           const WsLayout& W, float* W2, const float* b2, float* grad_w2) {
+                           const WsLayout& W, float* W2, float* b2, float* grad_w2, float* grad_b2) {
   if (!tc_available()) return cudaErrorNotSupported;
   const int64_t Lp = padded_ld(L);
   CUtensorMap ta, tb;
@@ -366,6 +396,7 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
   // which == 3: W2 -= lr dZ^T H1
   g.M = (int)L; g.N = H; g.K = n;
   g.out = W2; g.ldo = H; g.lr = lr; g.shadow = P.w2b; g.grad = grad_w2;
+  g.b2 = b2; g.grad_b2 = grad_b2;
   if ((e = make_map(&ta, P.dzb, L, n, (uint64_t)Lp * 2, 64, 64)) != cudaSuccess) return e;
   if ((e = make_map(&tb, P.h1b, H, n, (uint64_t)H * 2, 64, 64)) != cudaSuccess) return e;
   const int64_t tiles_m = (L + BM - 1) / BM;
