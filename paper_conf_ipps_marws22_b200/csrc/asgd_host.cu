@@ -111,6 +111,7 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.da1 = take(B * H * 4);
   L.db1part = take(L.n_rowblk * H * 4);
   L.w2b = take(bf ? (size_t)Lb * H * 2 : 0);
+  L.w2b2 = take(bf ? (size_t)Lb * H * 2 : 0);
   L.red = take((L.n_red + 8) * 8);
   L.eval_top = take(B * 8 * 4);
   L.total = o;
@@ -160,9 +161,13 @@ struct asgd_ctx {
   std::vector<cudaEvent_t> pev[ASGD_PROF_N];   // (start, end) pairs
   size_t pused[ASGD_PROF_N] = {};
   cudaStream_t s2 = nullptr;                     // side stream: K-0 overlaps the dense chain
-  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  cudaStream_t s3 = nullptr;                     // side stream: G3 + b1 (bf16 path)
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_sm = nullptr, ev_dh = nullptr, ev_a = nullptr;
+  bf16* w2b_buf[2] = {nullptr, nullptr};         // double-buffered bf16 W2 shadow
+  int w2b_cur = 0;
   Launch lc() { return Launch{s, &launches, sms}; }
   Launch lc2() { return Launch{s2, &launches, sms}; }
+  Launch lc3() { return Launch{s3, &launches, sms}; }
 };
 
 namespace {
@@ -258,12 +263,15 @@ int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device, v
   c->o_w2 = c->o_b1 + m.H;
   c->o_b2 = c->o_w2 + m.L * m.H;
   c->Pn = c->o_b2 + m.L;
+  c->w2b_buf[0] = c->P.w2b;
+  c->w2b_buf[1] = reinterpret_cast<bf16*>(c->ws + c->L.w2b2);
   cudaError_t e = cudaStreamCreateWithFlags(&c->s2, cudaStreamNonBlocking);
-  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
-  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->s3, cudaStreamNonBlocking);
+  for (cudaEvent_t* ev : {&c->ev_fork, &c->ev_join, &c->ev_sm, &c->ev_dh, &c->ev_a})
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(ev, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->ws, 0, c->L.total, c->s);
   if (e == cudaSuccess && m.precision == ASGD_PREC_BF16)
-    e = launch_to_bf16(c->lc(), c->params + c->o_w2, c->P.w2b, m.L * m.H);
+    e = launch_to_bf16(c->lc(), c->params + c->o_w2, c->w2b_buf[c->w2b_cur], m.L * m.H);
   if (e == cudaSuccess) e = cudaStreamSynchronize(c->s);
   if (e != cudaSuccess) { asgd_replica_destroy(c); return cuda_fail(e, "replica_init"); }
   *out = c;
@@ -274,9 +282,10 @@ int asgd_replica_destroy(asgd_ctx* c) {
   if (c) {
     for (auto& v : c->pev)
       for (cudaEvent_t e : v) cudaEventDestroy(e);
-    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
-    if (c->ev_join) cudaEventDestroy(c->ev_join);
+    for (cudaEvent_t ev : {c->ev_fork, c->ev_join, c->ev_sm, c->ev_dh, c->ev_a})
+      if (ev) cudaEventDestroy(ev);
     if (c->s2) cudaStreamDestroy(c->s2);
+    if (c->s3) cudaStreamDestroy(c->s3);
   }
   delete c;
   return ASGD_OK;
@@ -291,7 +300,7 @@ int asgd_set_stream(asgd_ctx* c, void* stream) {
 int asgd_params_changed(asgd_ctx* c) {
   if (!c) return fail(ASGD_E_ARG, "null ctx");
   if (c->d.precision == ASGD_PREC_BF16)
-    CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->P.w2b, c->d.L * c->d.H));
+    CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->w2b_buf[c->w2b_cur], c->d.L * c->d.H));
   return ASGD_OK;
 }
 
@@ -360,6 +369,7 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
   // K-1
   PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, rows, n, x.row_ptr, x.col, x.val, W1, b1, H, P, c->L, bf));
   if (!bf) {
+    // fp32 path: one stream, G2 reads W2 before G3 updates it in place
     GemmArgs a{};
     // G1: Z[n x L] = H1 W2^T + b2
     a.M = n; a.N = (int)Lb; a.K = H;
@@ -376,32 +386,49 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     a.epi = EPI_SPLITK; a.C = P.dhpart; a.ldc = H; a.splitk = (int)c->L.splitk;
     a.part_stride = c->L.part_stride;
     PCU(ASGD_K_G2, launch_gemm_f32(lc, a));
-  } else {
-    PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, P, c->L, W2, b2, nullptr, nullptr));
-    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, true));
-    PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, lr, P, c->L, W2, b2, nullptr, nullptr));
-  }
-  PCU(ASGD_K_DH, ([&]() -> cudaError_t {
-        cudaError_t e = launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L);
-        return e != cudaSuccess ? e : launch_b1_update(lc, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev);
-      })());
-  if (!bf) PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, Lp, b2, lr, P, false, g ? g + c->o_b2 : nullptr));
-  if (!bf) {
+    PCU(ASGD_K_DH, ([&]() -> cudaError_t {
+          cudaError_t e = launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L);
+          return e != cudaSuccess ? e : launch_b1_update(lc, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev);
+        })());
+    PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, Lp, b2, lr, P, false, g ? g + c->o_b2 : nullptr));
     // G3: W2 -= lr dZ^T H1
-    GemmArgs a{};
+    a = GemmArgs{};
     a.M = (int)Lb; a.N = H; a.K = n;
     a.A = P.z; a.as0 = 1; a.as1 = Lp;
     a.B = P.h1; a.bs0 = H; a.bs1 = 1;
     a.epi = EPI_SGD; a.C = W2; a.ldc = H; a.lr = lr; a.grad = g ? g + c->o_w2 : nullptr;
     a.splitk = 1;
     PCU(ASGD_K_G3, launch_gemm_f32(lc, a));
+    // K-5 (needs K-0's segments)
+    CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
+    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr));
   } else {
-    PCU(ASGD_K_G3, launch_gemm_tc(lc, 3, n, Lb, H, lr, P, c->L, W2, b2, g ? g + c->o_w2 : nullptr,
-                                  g ? g + c->o_b2 : nullptr));
+    // bf16 path, a DAG over three streams:
+    //   s : G1 -> softmax -> G2 -> dH reduce -> [K-0 joined] K-5
+    //   s3: [after softmax] G3 (W2, b2 and the next step's bf16 W2 shadow) -> [after dH] b1
+    // G1/G2 read the bf16 shadow w2b[cur]; G3 writes w2b[cur ^ 1], so G2 and G3 never race.
+    Ptrs Pr = P, Pw = P;
+    Pr.w2b = c->w2b_buf[c->w2b_cur];
+    Pw.w2b = c->w2b_buf[c->w2b_cur ^ 1];
+    Launch lc3 = c->lc3();
+    PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr));
+    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, true));
+    CU(cudaEventRecord(c->ev_sm, c->s));
+    CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
+    PCU_ON(c->s3, ASGD_K_G3, launch_gemm_tc(lc3, 3, n, Lb, H, lr, Pw, c->L, W2, b2, g ? g + c->o_w2 : nullptr,
+                                            g ? g + c->o_b2 : nullptr));
+    PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr));
+    PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L));
+    CU(cudaEventRecord(c->ev_dh, c->s));
+    CU(cudaStreamWaitEvent(c->s3, c->ev_dh, 0));
+    PCU_ON(c->s3, ASGD_K_DH, launch_b1_update(lc3, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev));
+    CU(cudaEventRecord(c->ev_a, c->s3));
+    // K-5 (needs K-0's segments)
+    CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
+    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr));
+    CU(cudaStreamWaitEvent(c->s, c->ev_a, 0));
+    c->w2b_cur ^= 1;
   }
-  // K-5 (needs K-0's segments)
-  CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
-  PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr));
   ++c->u;
   return ASGD_OK;
 }
@@ -447,7 +474,7 @@ int asgd_merge_finish(asgd_ctx* c, float gamma) {
   if (!c) return fail(ASGD_E_ARG, "null ctx");
   PCU(ASGD_K_MERGE, launch_finish(c->lc(), c->params, c->w, c->dd, c->Pn, gamma));
   if (c->d.precision == ASGD_PREC_BF16)
-    CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->P.w2b, c->d.L * c->d.H));
+    CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->w2b_buf[c->w2b_cur], c->d.L * c->d.H));
   c->u = 0;
   return ASGD_OK;
 }
@@ -490,7 +517,9 @@ int asgd_eval_topk(asgd_ctx* c, const asgd_csr* t, const int32_t* rows, int32_t 
       a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = padded_ld(m.L); a.bias = b2; a.splitk = 1;
       CU(launch_gemm_f32(lc, a));
     } else {
-      CU(launch_gemm_tc(lc, 1, nb, m.L, H, 0.f, P, c->L, W2, b2, nullptr, nullptr));
+      Ptrs Pr = P;
+      Pr.w2b = c->w2b_buf[c->w2b_cur];
+      CU(launch_gemm_tc(lc, 1, nb, m.L, H, 0.f, Pr, c->L, W2, b2, nullptr, nullptr));
     }
     CU(launch_topk(lc, nb, m.L, padded_ld(m.L), k, P.z, topk + (int64_t)r0 * k));
   }
@@ -528,6 +557,7 @@ int asgd_profile_read(asgd_ctx* c, double* ms, int64_t* cnt) {
   if (!c || !ms || !cnt) return fail(ASGD_E_ARG, "null argument");
   CU(cudaStreamSynchronize(c->s));
   CU(cudaStreamSynchronize(c->s2));
+  CU(cudaStreamSynchronize(c->s3));
   for (int k = 0; k < ASGD_PROF_N; ++k) {
     double t = 0.0;
     for (size_t i = 0; i < c->pused[k]; ++i) {

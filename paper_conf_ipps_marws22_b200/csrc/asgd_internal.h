@@ -25,7 +25,7 @@ typedef __nv_bfloat16 bf16;
 struct WsLayout {
   size_t meta, boff, loff, cnt, fseg, fuid, uniq, useg, tsum, tpre;
   size_t e_n, e_v, e_u, part1, rowcnt, part5, ucnt;
-  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, red, eval_top, b2part, rbase;
+  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, b2part, rbase;
   size_t total;
   int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride;
 };
@@ -49,6 +49,31 @@ struct Launch {       // launch bookkeeping of one ctx
   int64_t* counter;
   int sms;
 };
+
+// Programmatic dependent launch: every kernel of the step lets its successor be
+// scheduled as soon as all of its own CTAs run (pdl_trigger at entry) and waits
+// for its predecessor's completion + memory flush (pdl_wait) before touching
+// the predecessor's outputs, so prologues (smem carve-up, mbarrier init, TMEM
+// alloc, tensormap prefetch) overlap the previous kernel's tail.
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k(const Launch& lc, void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                     Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = lc.s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  ++*lc.counter;
+  return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
 
 // ---------------------------------------------------------------- K-0
 cudaError_t launch_batch_scan(const Launch&, const int32_t* rows, int n, const int64_t* row_ptr,

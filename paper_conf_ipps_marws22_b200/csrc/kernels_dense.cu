@@ -21,6 +21,8 @@ constexpr unsigned kFull = 0xffffffffu;
 constexpr int BM = 64, BN = 64, BK = 16;
 
 __global__ void __launch_bounds__(256) k_gemm_f32(GemmArgs g) {
+  pdl_trigger();
+  pdl_wait();
   __shared__ float As[BK][BM + 4];
   __shared__ float Bs[BK][BN + 4];
   const int t = threadIdx.x, tx = t & 15, ty = t >> 4;
@@ -95,6 +97,8 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
                                                     const int64_t* __restrict__ lab_ptr,
                                                     const int32_t* __restrict__ lab, float* Z,
                                                     bf16* dZb, float* rowloss) {
+  pdl_trigger();
+  pdl_wait();
   __shared__ int s_lab[kMaxRowLabels];
   __shared__ float s_lz[kMaxRowLabels];
   __shared__ float s_m[16], s_s[16];
@@ -160,6 +164,8 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
 // split-K loads all in flight; fixed summation order (deterministic).
 __global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
                             const float* __restrict__ part, const float* __restrict__ H1, float* dA1) {
+  pdl_trigger();
+  pdl_wait();
   const int r = blockIdx.x, c = threadIdx.x;
   const int64_t o = (int64_t)r * H + c;
   float a[8];
@@ -179,6 +185,8 @@ __global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
 __global__ void __launch_bounds__(256) k_b1_update(int n, int H, const float* __restrict__ dA1, float* b1,
                                                    float lr, float* grad_b1,
                                                    const float* __restrict__ rowloss, float* loss_dev) {
+  pdl_trigger();
+  pdl_wait();
   const int lane = threadIdx.x & 31;
   const int c = blockIdx.x * 8 + (threadIdx.x >> 5);
   if (c < H) {
@@ -209,6 +217,8 @@ __global__ void __launch_bounds__(256) k_b1_update(int n, int H, const float* __
 constexpr int kB2Chunks = 16;
 __global__ void __launch_bounds__(256) k_b2_part(int n, int64_t L, int64_t ldz, const float* __restrict__ dz,
                                                  const bf16* __restrict__ dzb, float* b2part) {
+  pdl_trigger();
+  pdl_wait();
   const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= L) return;
   const int per = (n + gridDim.y - 1) / gridDim.y;
@@ -234,6 +244,8 @@ __global__ void __launch_bounds__(256) k_b2_part(int n, int64_t L, int64_t ldz, 
 // b2 -= lr * sum_y b2part[y]
 __global__ void __launch_bounds__(256) k_b2_apply(int64_t L, int chunks, const float* __restrict__ b2part,
                                                   float* b2, float lr, float* grad_b2) {
+  pdl_trigger();
+  pdl_wait();
   const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= L) return;
   float s = 0.f;
@@ -243,6 +255,8 @@ __global__ void __launch_bounds__(256) k_b2_apply(int64_t L, int chunks, const f
 }
 
 __global__ void k_to_bf16(const float* __restrict__ src, bf16* dst, int64_t count) {
+  pdl_trigger();
+  pdl_wait();
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count;
        i += (int64_t)gridDim.x * blockDim.x)
     dst[i] = __float2bfloat16_rn(src[i]);
@@ -253,32 +267,28 @@ __global__ void k_to_bf16(const float* __restrict__ src, bf16* dst, int64_t coun
 cudaError_t launch_gemm_f32(const Launch& lc, const GemmArgs& g) {
   if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaSuccess;
   dim3 grid((g.N + BN - 1) / BN, (g.M + BM - 1) / BM, g.splitk);
-  k_gemm_f32<<<grid, 256, 0, lc.s>>>(g);
-  ++*lc.counter;
+  launch_k(lc, k_gemm_f32, dim3(grid), dim3(256), 0, g);
   return cudaGetLastError();
 }
 
 cudaError_t launch_softmax_ce(const Launch& lc, int n, int64_t L, int64_t ldz, const int32_t* rows,
                               const int64_t* lab_ptr, const int32_t* lab, const Ptrs& P,
                               bool bf16_out) {
-  k_softmax_ce<<<n, 512, 0, lc.s>>>(n, L, ldz, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
+  launch_k(lc, k_softmax_ce, dim3(n), dim3(512), 0, n, L, ldz, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
                                     P.rowloss);
-  ++*lc.counter;
   return cudaGetLastError();
 }
 
 cudaError_t launch_dh_reduce(const Launch& lc, int n, int H, int splitk, const Ptrs& P,
                              const WsLayout& L) {
   // split-K partial z of dH1 lives at dhpart + z * (b_max * H)
-  k_dh_reduce<<<n, H, 0, lc.s>>>(n, H, splitk, L.part_stride, P.dhpart, P.h1, P.da1);
-  ++*lc.counter;
+  launch_k(lc, k_dh_reduce, dim3(n), dim3(H), 0, n, H, splitk, L.part_stride, P.dhpart, P.h1, P.da1);
   return cudaGetLastError();
 }
 
 cudaError_t launch_b1_update(const Launch& lc, int n, int H, float* b1, float lr, const Ptrs& P,
                              const WsLayout& L, float* grad_b1, float* loss_dev) {
-  k_b1_update<<<H / 8 + 1, 256, 0, lc.s>>>(n, H, P.da1, b1, lr, grad_b1, P.rowloss, loss_dev);
-  ++*lc.counter;
+  launch_k(lc, k_b1_update, dim3(H / 8 + 1), dim3(256), 0, n, H, P.da1, b1, lr, grad_b1, P.rowloss, loss_dev);
   return cudaGetLastError();
 }
 
@@ -286,16 +296,14 @@ cudaError_t launch_b2_update(const Launch& lc, int n, int64_t L, int64_t ldz, fl
                              const Ptrs& P, bool from_bf16, float* grad_b2) {
   const int chunks = std::max(1, std::min(kB2Chunks, n / 16));
   dim3 grid((unsigned)((L + 255) / 256), (unsigned)chunks);
-  k_b2_part<<<grid, 256, 0, lc.s>>>(n, L, ldz, P.z, from_bf16 ? P.dzb : nullptr, P.b2part);
-  k_b2_apply<<<(unsigned)((L + 255) / 256), 256, 0, lc.s>>>(L, chunks, P.b2part, b2, lr, grad_b2);
-  *lc.counter += 2;
+  launch_k(lc, k_b2_part, dim3(grid), dim3(256), 0, n, L, ldz, P.z, from_bf16 ? P.dzb : nullptr, P.b2part);
+  launch_k(lc, k_b2_apply, dim3((unsigned)((L + 255) / 256)), dim3(256), 0, L, chunks, P.b2part, b2, lr, grad_b2);
   return cudaGetLastError();
 }
 
 cudaError_t launch_to_bf16(const Launch& lc, const float* src, bf16* dst, int64_t count) {
   const int64_t blocks = std::min<int64_t>((count + 255) / 256, (int64_t)lc.sms * 16);
-  k_to_bf16<<<(int)std::max<int64_t>(blocks, 1), 256, 0, lc.s>>>(src, dst, count);
-  ++*lc.counter;
+  launch_k(lc, k_to_bf16, dim3((int)std::max<int64_t>(blocks, 1)), dim3(256), 0, src, dst, count);
   return cudaGetLastError();
 }
 

@@ -18,6 +18,8 @@ constexpr unsigned kFull = 0xffffffffu;
 
 __global__ void __launch_bounds__(256) k_sqnorm_part(const float* __restrict__ x, int64_t P,
                                                      double* partials) {
+  pdl_trigger();
+  pdl_wait();
   double s = 0.0;
   const int64_t P4 = P / 4;
   const float4* x4 = reinterpret_cast<const float4*>(x);
@@ -41,6 +43,8 @@ __global__ void __launch_bounds__(256) k_sqnorm_part(const float* __restrict__ x
 }
 
 __global__ void k_sqnorm_final(const double* __restrict__ partials, int n, double* out) {
+  pdl_trigger();
+  pdl_wait();
   __shared__ double sh[32];
   double s = 0.0;
   // fixed assignment: thread t sums partials t, t+blockDim, ... in order
@@ -58,6 +62,8 @@ __global__ void k_sqnorm_final(const double* __restrict__ partials, int n, doubl
 }
 
 __global__ void __launch_bounds__(256) k_scale(float* x, int64_t P, double alpha) {
+  pdl_trigger();
+  pdl_wait();
   const int64_t P4 = P / 4;
   float4* x4 = reinterpret_cast<float4*>(x);
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P4;
@@ -80,6 +86,8 @@ __device__ __forceinline__ void finish1(float& p, float& w, float& d, float gamm
 
 __global__ void __launch_bounds__(256) k_finish(float* params, float* w, float* d, int64_t P,
                                                 float gamma) {
+  pdl_trigger();
+  pdl_wait();
   const int64_t P4 = P / 4;
   float4* p4 = reinterpret_cast<float4*>(params);
   float4* w4 = reinterpret_cast<float4*>(w);
@@ -98,6 +106,8 @@ __global__ void __launch_bounds__(256) k_finish(float* params, float* w, float* 
 __global__ void __launch_bounds__(256) k_wsum(const float* const* __restrict__ reps,
                                               const double* __restrict__ alpha, int n, int64_t P,
                                               float* out) {
+  pdl_trigger();
+  pdl_wait();
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P;
        i += (int64_t)gridDim.x * blockDim.x) {
     double s = 0.0;
@@ -115,6 +125,8 @@ __device__ __forceinline__ bool better(const Cand& a, const Cand& b) {
 template <int K>
 __global__ void __launch_bounds__(256) k_topk(int64_t L, int64_t ldz, int k, const float* __restrict__ z,
                                               int32_t* out) {
+  pdl_trigger();
+  pdl_wait();
   const int n = blockIdx.x;
   const float* row = z + (int64_t)n * ldz;
   Cand top[K];
@@ -151,6 +163,8 @@ __global__ void __launch_bounds__(256) k_topk(int64_t L, int64_t ldz, int k, con
 
 // -------------------------------------------------------------- validation
 __global__ void k_validate(asgd_csr c, int64_t F, int64_t L, int32_t* err) {
+  pdl_trigger();
+  pdl_wait();
   for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < c.n_rows;
        r += (int64_t)gridDim.x * blockDim.x) {
     int e = 0;
@@ -187,44 +201,38 @@ inline int grid_for(const Launch& lc, int64_t work) {
 
 cudaError_t launch_sqnorm(const Launch& lc, const float* x, int64_t P, double* partials,
                           int nparts, double* out) {
-  k_sqnorm_part<<<nparts, 256, 0, lc.s>>>(x, P, partials);
-  k_sqnorm_final<<<1, 1024, 0, lc.s>>>(partials, nparts, out);
-  *lc.counter += 2;
+  launch_k(lc, k_sqnorm_part, dim3(nparts), dim3(256), 0, x, P, partials);
+  launch_k(lc, k_sqnorm_final, dim3(1), dim3(1024), 0, partials, nparts, out);
   return cudaGetLastError();
 }
 
 cudaError_t launch_scale(const Launch& lc, float* x, int64_t P, double alpha) {
-  k_scale<<<grid_for(lc, P / 4), 256, 0, lc.s>>>(x, P, alpha);
-  ++*lc.counter;
+  launch_k(lc, k_scale, dim3(grid_for(lc, P / 4)), dim3(256), 0, x, P, alpha);
   return cudaGetLastError();
 }
 
 cudaError_t launch_finish(const Launch& lc, float* params, float* w, float* d, int64_t P,
                           float gamma) {
-  k_finish<<<grid_for(lc, P / 4), 256, 0, lc.s>>>(params, w, d, P, gamma);
-  ++*lc.counter;
+  launch_k(lc, k_finish, dim3(grid_for(lc, P / 4)), dim3(256), 0, params, w, d, P, gamma);
   return cudaGetLastError();
 }
 
 cudaError_t launch_wsum(const Launch& lc, const float* const* reps, const double* alpha, int n,
                         int64_t P, float* out) {
-  k_wsum<<<grid_for(lc, P), 256, 0, lc.s>>>(reps, alpha, n, P, out);
-  ++*lc.counter;
+  launch_k(lc, k_wsum, dim3(grid_for(lc, P)), dim3(256), 0, reps, alpha, n, P, out);
   return cudaGetLastError();
 }
 
 cudaError_t launch_topk(const Launch& lc, int n, int64_t L, int64_t ldz, int k, const float* z,
                         int32_t* out) {
   if (k <= 0 || k > 8) return cudaErrorInvalidValue;
-  k_topk<8><<<n, 256, 0, lc.s>>>(L, ldz, k, z, out);
-  ++*lc.counter;
+  launch_k(lc, k_topk<8>, dim3(n), dim3(256), 0, L, ldz, k, z, out);
   return cudaGetLastError();
 }
 
 cudaError_t launch_validate_csr(const Launch& lc, const asgd_csr* c, int64_t F, int64_t L,
                                 int32_t* err) {
-  k_validate<<<grid_for(lc, c->n_rows), 256, 0, lc.s>>>(*c, F, L, err);
-  ++*lc.counter;
+  launch_k(lc, k_validate, dim3(grid_for(lc, c->n_rows)), dim3(256), 0, *c, F, L, err);
   return cudaGetLastError();
 }
 

@@ -121,6 +121,8 @@ __global__ void __launch_bounds__(1024) k_batch_scan(const int32_t* __restrict__
                                                      int64_t n_data_rows, int32_t* boff,
                                                      int32_t* loff, int32_t* meta, int64_t nz_cap,
                                                      int64_t nl_cap, int64_t* rbase) {
+  pdl_trigger();
+  pdl_wait();
   __shared__ long long wf[32], wl[32];
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
   const int per = (n + blockDim.x - 1) / blockDim.x;
@@ -207,6 +209,8 @@ __device__ __forceinline__ void load_view(int32_t* sboff, const int32_t* boff, c
 __global__ void k_count(int n, const int64_t* __restrict__ rbase,
                         const int32_t* __restrict__ col, const int32_t* __restrict__ boff,
                         int32_t* meta, int32_t* cnt, unsigned long long* status, int ntiles) {
+  pdl_trigger();
+  pdl_wait();
   extern __shared__ int32_t sboff[];
   if (blockIdx.x == 0) {
     for (int i = threadIdx.x; i < ntiles; i += blockDim.x) status[i] = 0ull;
@@ -234,6 +238,8 @@ __global__ void __launch_bounds__(256) k_fscan(const int32_t* __restrict__ cnt, 
                                                unsigned long long* status, int ntiles, int32_t* meta,
                                                int32_t* fseg, int32_t* fuid, int32_t* uniq,
                                                int32_t* useg) {
+  pdl_trigger();
+  pdl_wait();
   constexpr int PER = kScanTile / 256;
   __shared__ int s_tile, s_pa, s_pb;
   __shared__ int wa[8], wb[8];
@@ -314,6 +320,8 @@ __global__ void k_place(int n, const int64_t* __restrict__ rbase,
                         const int32_t* __restrict__ boff, const int32_t* __restrict__ meta,
                         int32_t* cnt, const int32_t* __restrict__ fseg,
                         const int32_t* __restrict__ fuid, int32_t* e_n, float* e_v, int32_t* e_u) {
+  pdl_trigger();
+  pdl_wait();
   extern __shared__ int32_t sboff[];
   load_view(sboff, boff, rbase, n);
   const int nnz = meta[M_NNZ];
@@ -332,6 +340,8 @@ __global__ void k_place(int n, const int64_t* __restrict__ rbase,
 // Row ids inside a segment are distinct (cols are unique within a row).
 __global__ void k_segsort(const int32_t* __restrict__ useg, const int32_t* __restrict__ meta,
                           int32_t* e_n, float* e_v, int words) {
+  pdl_trigger();
+  pdl_wait();
   extern __shared__ uint32_t sm[];
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   uint32_t* bm = sm + (size_t)wib * words * 33;
@@ -401,6 +411,8 @@ __global__ void __launch_bounds__(256) k_spmm_fwd(int n, const int64_t* __restri
                                                   const int32_t* __restrict__ boff,
                                                   const int32_t* __restrict__ meta, float* H1,
                                                   bf16* H1b, float* part, int32_t* rowcnt) {
+  pdl_trigger();
+  pdl_wait();
   using IO = RowIO<VPL>;
   constexpr int H = 32 * VPL;
   constexpr int kU = VPL >= 16 ? 4 : 8;   // W1 rows in flight per warp
@@ -512,6 +524,8 @@ __global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__
                                                      const float* __restrict__ dA1, float* W1,
                                                      float lr, float* part, int32_t* ucnt,
                                                      float* grad_w1) {
+  pdl_trigger();
+  pdl_wait();
   using IO = RowIO<VPL>;
   constexpr int H = 32 * VPL;
   constexpr int kU = VPL >= 16 ? 4 : 8;   // dA1 rows in flight per warp
@@ -612,9 +626,8 @@ cudaError_t spmm_fwd_t(const Launch& lc, const int32_t* rows, int n, const int64
   const size_t smem = view_smem(n);
   static int occ = 0;
   const int grid = wave_grid(lc, k_spmm_fwd<VPL>, view_smem(2048), L.n_pieces, occ);
-  k_spmm_fwd<VPL><<<grid, 256, smem, lc.s>>>(n, P.rbase, col, val, W1, b1, P.boff, P.meta,
+  launch_k(lc, k_spmm_fwd<VPL>, dim3(grid), dim3(256), smem, n, P.rbase, col, val, W1, b1, P.boff, P.meta,
                                              P.h1, want_bf16 ? P.h1b : nullptr, P.part1, P.rowcnt);
-  ++*lc.counter;
   return cudaGetLastError();
 }
 
@@ -623,9 +636,8 @@ cudaError_t scatter_t(const Launch& lc, float* W1, float lr, const Ptrs& P, cons
                       float* grad_w1) {
   static int occ = 0;
   const int grid = wave_grid(lc, k_scatter_sgd<VPL>, 0, L.n_pieces, occ);
-  k_scatter_sgd<VPL><<<grid, 256, 0, lc.s>>>(P.e_n, P.e_v, P.e_u, P.useg, P.uniq, P.meta, P.da1,
+  launch_k(lc, k_scatter_sgd<VPL>, dim3(grid), dim3(256), 0, P.e_n, P.e_v, P.e_u, P.useg, P.uniq, P.meta, P.da1,
                                              W1, lr, P.part5, P.ucnt, grad_w1);
-  ++*lc.counter;
   return cudaGetLastError();
 }
 
@@ -634,9 +646,8 @@ cudaError_t scatter_t(const Launch& lc, float* W1, float lr, const Ptrs& P, cons
 cudaError_t launch_batch_scan(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
                               const int64_t* lab_ptr, int64_t n_data_rows, const Ptrs& P,
                               int64_t nz_cap, int64_t nl_cap) {
-  k_batch_scan<<<1, 1024, 0, lc.s>>>(rows, n, row_ptr, lab_ptr, n_data_rows, P.boff, P.loff, P.meta,
+  launch_k(lc, k_batch_scan, dim3(1), dim3(1024), 0, rows, n, row_ptr, lab_ptr, n_data_rows, P.boff, P.loff, P.meta,
                                      nz_cap, nl_cap, P.rbase);
-  ++*lc.counter;
   return cudaGetLastError();
 }
 
@@ -647,14 +658,13 @@ cudaError_t launch_touched(const Launch& lc, const int32_t* rows, int n, const i
   const int grid = lc.sms * 4;
   const int nt = (int)L.n_tiles_f;
   unsigned long long* status = reinterpret_cast<unsigned long long*>(P.tsum);
-  k_count<<<grid, 256, smem, lc.s>>>(n, P.rbase, col, P.boff, P.meta, P.cnt, status, nt);
-  k_fscan<<<nt, 256, 0, lc.s>>>(P.cnt, F, status, nt, P.meta, P.fseg, P.fuid, P.uniq, P.useg);
-  k_place<<<grid, 256, smem, lc.s>>>(n, P.rbase, col, val, P.boff, P.meta, P.cnt, P.fseg,
+  launch_k(lc, k_count, dim3(grid), dim3(256), smem, n, P.rbase, col, P.boff, P.meta, P.cnt, status, nt);
+  launch_k(lc, k_fscan, dim3(nt), dim3(256), 0, P.cnt, F, status, nt, P.meta, P.fseg, P.fuid, P.uniq, P.useg);
+  launch_k(lc, k_place, dim3(grid), dim3(256), smem, n, P.rbase, col, val, P.boff, P.meta, P.cnt, P.fseg,
                                      P.fuid, P.e_n, P.e_v, P.e_u);
   const int words = (b_max + 31) / 32;
   const size_t ssmem = (size_t)8 * words * 33 * sizeof(uint32_t);
-  k_segsort<<<lc.sms * 2, 256, ssmem, lc.s>>>(P.useg, P.meta, P.e_n, P.e_v, words);
-  *lc.counter += 4;
+  launch_k(lc, k_segsort, dim3(lc.sms * 2), dim3(256), ssmem, P.useg, P.meta, P.e_n, P.e_v, words);
   return cudaGetLastError();
 }
 

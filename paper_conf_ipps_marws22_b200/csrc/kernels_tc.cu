@@ -143,6 +143,7 @@ __global__ void __launch_bounds__(256, 1)
   uint64_t* tfull = empty + STAGES;
   uint32_t* tbase = reinterpret_cast<uint32_t*>(tfull + 1);
 
+  pdl_trigger();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n0 = blockIdx.x * BN, m0 = blockIdx.y * BM;
   const int nkb = (g.K + BK - 1) / BK;
@@ -174,6 +175,7 @@ __global__ void __launch_bounds__(256, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tbase;
+  pdl_wait();   // operands / outputs of the previous kernel are visible from here on
 
   if (warp == 0) {
     if (lane == 0) {
@@ -342,9 +344,7 @@ cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, co
     attr = true;
   }
   dim3 grid((g.N + BN - 1) / BN, (g.M + BM - 1) / BM, splits);
-  k_gemm_tc<BN, A_MN, B_MN, EPI><<<grid, 256, smem, lc.s>>>(a, b, g);
-  ++*lc.counter;
-  return cudaGetLastError();
+  return launch_k(lc, k_gemm_tc<BN, A_MN, B_MN, EPI>, grid, dim3(256), smem, a, b, g);
 }
 
 // Widest N tile that still gives >= one CTA per SM (and does not overhang N by 2x).
