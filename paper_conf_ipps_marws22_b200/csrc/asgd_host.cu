@@ -14,6 +14,7 @@
 #include <atomic>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -96,16 +97,19 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.e_n = take(L.nz_cap * 4);
   L.e_v = take(L.nz_cap * 4);
   L.e_u = take(L.nz_cap * 4);
+  L.e_f = take(L.nz_cap * 4);
   L.part1 = take((size_t)2 * L.n_pieces * H * 4);
   L.rowcnt = take(B * 4);
   L.part5 = take((size_t)2 * L.n_pieces * H * 4);
-  L.ucnt = take((L.u_cap + 1) * 4);
+  L.ucnt = take((L.u_cap + 1) * 4 * 8);   // per (segment, column slice)
+  L.bits = take((size_t)L.u_cap * ((B + 31) / 32) * 4);   // K-0 row bitmaps per touched feature
   L.h1 = take(B * H * 4);
   L.h1b = take(bf ? B * H * 2 : 0);
   L.z = take((size_t)B * Lp * 4);
   L.dzb = take(bf ? (size_t)B * Lp * 2 : 0);
   L.b2part = take((size_t)b2_chunks() * Lb * 4);
   L.rbase = take((size_t)(B + 1) * 8);
+  L.da1b = take(bf ? (size_t)B * H * 2 : 0);
   L.rowloss = take(B * 4);
   L.dhpart = take((size_t)L.splitk * B * H * 4);
   L.da1 = take(B * H * 4);
@@ -124,7 +128,8 @@ Ptrs ws_ptrs(char* b, const WsLayout& L) {
   p.cnt = (int32_t*)(b + L.cnt); p.fseg = (int32_t*)(b + L.fseg); p.fuid = (int32_t*)(b + L.fuid);
   p.uniq = (int32_t*)(b + L.uniq); p.useg = (int32_t*)(b + L.useg); p.tsum = (int32_t*)(b + L.tsum);
   p.tpre = (int32_t*)(b + L.tpre); p.e_n = (int32_t*)(b + L.e_n); p.e_v = (float*)(b + L.e_v);
-  p.e_u = (int32_t*)(b + L.e_u); p.part1 = (float*)(b + L.part1); p.rowcnt = (int32_t*)(b + L.rowcnt);
+  p.e_u = (int32_t*)(b + L.e_u); p.e_f = (int32_t*)(b + L.e_f);
+  p.bits = (uint32_t*)(b + L.bits); p.part1 = (float*)(b + L.part1); p.rowcnt = (int32_t*)(b + L.rowcnt);
   p.part5 = (float*)(b + L.part5); p.ucnt = (int32_t*)(b + L.ucnt); p.h1 = (float*)(b + L.h1);
   p.h1b = (bf16*)(b + L.h1b); p.z = (float*)(b + L.z); p.dzb = (bf16*)(b + L.dzb);
   p.rowloss = (float*)(b + L.rowloss); p.dhpart = (float*)(b + L.dhpart); p.da1 = (float*)(b + L.da1);
@@ -132,6 +137,7 @@ Ptrs ws_ptrs(char* b, const WsLayout& L) {
   p.eval_top = (int32_t*)(b + L.eval_top);
   p.b2part = (float*)(b + L.b2part);
   p.rbase = (int64_t*)(b + L.rbase);
+  p.da1b = (bf16*)(b + L.da1b);
   return p;
 }
 
@@ -387,7 +393,7 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     a.part_stride = c->L.part_stride;
     PCU(ASGD_K_G2, launch_gemm_f32(lc, a));
     PCU(ASGD_K_DH, ([&]() -> cudaError_t {
-          cudaError_t e = launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L);
+          cudaError_t e = launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, false);
           return e != cudaSuccess ? e : launch_b1_update(lc, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev);
         })());
     PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, Lp, b2, lr, P, false, g ? g + c->o_b2 : nullptr));
@@ -401,7 +407,7 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     PCU(ASGD_K_G3, launch_gemm_f32(lc, a));
     // K-5 (needs K-0's segments)
     CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
-    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr));
+    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
   } else {
     // bf16 path, a DAG over three streams:
     //   s : G1 -> softmax -> G2 -> dH reduce -> [K-0 joined] K-5
@@ -418,14 +424,14 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     PCU_ON(c->s3, ASGD_K_G3, launch_gemm_tc(lc3, 3, n, Lb, H, lr, Pw, c->L, W2, b2, g ? g + c->o_w2 : nullptr,
                                             g ? g + c->o_b2 : nullptr));
     PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr));
-    PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L));
+    PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, true));
     CU(cudaEventRecord(c->ev_dh, c->s));
     CU(cudaStreamWaitEvent(c->s3, c->ev_dh, 0));
     PCU_ON(c->s3, ASGD_K_DH, launch_b1_update(lc3, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev));
     CU(cudaEventRecord(c->ev_a, c->s3));
     // K-5 (needs K-0's segments)
     CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
-    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr));
+    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
     CU(cudaStreamWaitEvent(c->s, c->ev_a, 0));
     c->w2b_cur ^= 1;
   }
@@ -787,3 +793,13 @@ int asgd_sched_close(asgd_sched* s, int32_t unlink_shm) {
 }
 
 }  // extern "C"
+
+namespace asgd {
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* v = getenv("ASGD_PDL");   // measured slower on the EURLex step: off by default
+    return v && v[0] == '1';
+  }();
+  return on;
+}
+}  // namespace asgd

@@ -15,7 +15,7 @@ constexpr int kMaxRowLabels = 1024;
 // Features per tile of the touched-feature scan.
 constexpr int kScanTile = 1024;
 // meta[] slots (int32, device)
-enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_COUNT = 8 };
+enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_COUNT = 8, M_BAR = 32 };  // M_BAR: 64-bit grid-barrier counter (slots 32-33)
 // error bits in meta[M_ERR]
 enum { ERR_NNZ_CAP = 1, ERR_LAB_CAP = 2, ERR_ROW_ID = 4 };
 
@@ -24,8 +24,8 @@ typedef __nv_bfloat16 bf16;
 // Device workspace carve-up (byte offsets from ws base; all 256-B aligned).
 struct WsLayout {
   size_t meta, boff, loff, cnt, fseg, fuid, uniq, useg, tsum, tpre;
-  size_t e_n, e_v, e_u, part1, rowcnt, part5, ucnt;
-  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, b2part, rbase;
+  size_t e_n, e_v, e_u, e_f, part1, rowcnt, part5, ucnt, bits;
+  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, b2part, rbase, da1b;
   size_t total;
   int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride;
 };
@@ -35,10 +35,11 @@ WsLayout ws_layout(const asgd_model_desc& d);
 struct Ptrs {  // typed views of the workspace
   int32_t* meta; int32_t* boff; int32_t* loff; int32_t* cnt; int32_t* fseg; int32_t* fuid;
   int32_t* uniq; int32_t* useg; int32_t* tsum; int32_t* tpre;
-  int32_t* e_n; float* e_v; int32_t* e_u; float* part1; int32_t* rowcnt; float* part5;
+  int32_t* e_n; float* e_v; int32_t* e_u; int32_t* e_f; uint32_t* bits; float* part1; int32_t* rowcnt; float* part5;
   int32_t* ucnt; float* h1; bf16* h1b; float* z; bf16* dzb; float* rowloss; float* dhpart;
   float* da1; float* db1part; bf16* w2b; double* red; int32_t* eval_top; float* b2part;
   int64_t* rbase;   // row_ptr[rows[r]] of the current batch (written by K-0 (a))
+  bf16* da1b;       // bf16 copy of dA1 (bf16 path; staged by K-5)
 };
 int row_block();   // rows per db1 partial (kernels_dense.cu)
 int b2_chunks();   // row chunks of the db2 partial sums
@@ -58,6 +59,8 @@ struct Launch {       // launch bookkeeping of one ctx
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 
+bool pdl_enabled();   // ASGD_PDL=0 disables programmatic dependent launch (default on)
+
 template <typename... KArgs, typename... Args>
 cudaError_t launch_k(const Launch& lc, void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
                      Args&&... args) {
@@ -70,7 +73,7 @@ cudaError_t launch_k(const Launch& lc, void (*kernel)(KArgs...), dim3 grid, dim3
   at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
   ++*lc.counter;
   return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
 }
@@ -87,8 +90,9 @@ cudaError_t launch_spmm_fwd(const Launch&, const int32_t* rows, int n, const int
                             const int32_t* col, const float* val, const float* W1, const float* b1,
                             int H, const Ptrs&, const WsLayout&, bool want_bf16);
 // ---------------------------------------------------------------- K-5
+// dA1b: bf16 copy of dA1 (bf16 path) or null (fp32 path stages fp32 dA1).
 cudaError_t launch_scatter_sgd(const Launch&, float* W1, int H, float lr, const Ptrs&,
-                               const WsLayout&, float* grad_w1);
+                               const WsLayout&, float* grad_w1, const bf16* dA1b, int b_max);
 // ---------------------------------------------------------------- dense (fp32 SIMT)
 // C(m,n) = sum_k A(m,k) B(k,n), A(m,k) = A[m*as0 + k*as1], B(k,n) = B[k*bs0 + n*bs1]
 enum GemmEpi { EPI_STORE_BIAS = 0, EPI_SPLITK = 1, EPI_SGD = 2 };
@@ -109,7 +113,8 @@ int64_t padded_ld(int64_t L);
 cudaError_t launch_softmax_ce(const Launch&, int n, int64_t L, int64_t ldz, const int32_t* rows,
                               const int64_t* lab_ptr, const int32_t* lab, const Ptrs&,
                               bool bf16_out);
-cudaError_t launch_dh_reduce(const Launch&, int n, int H, int splitk, const Ptrs&, const WsLayout&);
+cudaError_t launch_dh_reduce(const Launch&, int n, int H, int splitk, const Ptrs&, const WsLayout&,
+                             bool want_bf16);
 cudaError_t launch_b1_update(const Launch&, int n, int H, float* b1, float lr, const Ptrs&,
                              const WsLayout&, float* grad_b1, float* loss_dev);
 cudaError_t launch_b2_update(const Launch&, int n, int64_t L, int64_t ldz, float* b2, float lr,

@@ -114,12 +114,22 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
     s_lab[i] = y;
     s_lz[i] = z[y];
   }
-  // pass 1: online max / sum-exp
+  // pass 1: online max / sum-exp, kSU loads in flight per thread
+  constexpr int kSU = 8;
   float m = -INFINITY, s = 0.f;
-  for (int64_t j = threadIdx.x; j < L; j += blockDim.x) {
-    const float v = z[j];
-    if (v > m) { s = s * __expf(m - v) + 1.f; m = v; }
-    else s += __expf(v - m);
+  for (int64_t j0 = threadIdx.x; j0 < L; j0 += (int64_t)kSU * blockDim.x) {
+    float v[kSU];
+#pragma unroll
+    for (int k = 0; k < kSU; ++k) {
+      const int64_t j = j0 + (int64_t)k * blockDim.x;
+      v[k] = j < L ? z[j] : -INFINITY;
+    }
+    float bm = v[0];
+#pragma unroll
+    for (int k = 1; k < kSU; ++k) bm = fmaxf(bm, v[k]);
+    if (bm > m) { s = (m == -INFINITY) ? 0.f : s * __expf(m - bm); m = bm; }
+#pragma unroll
+    for (int k = 0; k < kSU; ++k) s += __expf(v[k] - m);   // exp(-inf) = 0 for the tail
   }
 #pragma unroll
   for (int o = 16; o; o >>= 1) {
@@ -147,12 +157,36 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
   const float lse = s_lse, invB = 1.f / (float)B;
   if (dZb) {
     bf16* d = dZb + (int64_t)n * ldz;
-    for (int64_t j = threadIdx.x; j < L; j += blockDim.x) d[j] = __float2bfloat16_rn(__expf(z[j] - lse) * invB);
+    for (int64_t j0 = threadIdx.x; j0 < L; j0 += (int64_t)kSU * blockDim.x) {
+      float v[kSU];
+#pragma unroll
+      for (int k = 0; k < kSU; ++k) {
+        const int64_t j = j0 + (int64_t)k * blockDim.x;
+        v[k] = j < L ? z[j] : 0.f;
+      }
+#pragma unroll
+      for (int k = 0; k < kSU; ++k) {
+        const int64_t j = j0 + (int64_t)k * blockDim.x;
+        if (j < L) d[j] = __float2bfloat16_rn(__expf(v[k] - lse) * invB);
+      }
+    }
     __syncthreads();
     for (int i = threadIdx.x; i < nl; i += blockDim.x)
       d[s_lab[i]] = __float2bfloat16_rn((__expf(s_lz[i] - lse) - 1.f / (float)nl) * invB);
   } else {
-    for (int64_t j = threadIdx.x; j < L; j += blockDim.x) z[j] = __expf(z[j] - lse) * invB;
+    for (int64_t j0 = threadIdx.x; j0 < L; j0 += (int64_t)kSU * blockDim.x) {
+      float v[kSU];
+#pragma unroll
+      for (int k = 0; k < kSU; ++k) {
+        const int64_t j = j0 + (int64_t)k * blockDim.x;
+        v[k] = j < L ? z[j] : 0.f;
+      }
+#pragma unroll
+      for (int k = 0; k < kSU; ++k) {
+        const int64_t j = j0 + (int64_t)k * blockDim.x;
+        if (j < L) z[j] = __expf(v[k] - lse) * invB;
+      }
+    }
     __syncthreads();
     for (int i = threadIdx.x; i < nl; i += blockDim.x)
       z[s_lab[i]] = (__expf(s_lz[i] - lse) - 1.f / (float)nl) * invB;
@@ -163,7 +197,8 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
 // dA1[r][c] = [H1[r][c] > 0] * sum_z part[z][r][c]: one thread per element, its
 // split-K loads all in flight; fixed summation order (deterministic).
 __global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
-                            const float* __restrict__ part, const float* __restrict__ H1, float* dA1) {
+                            const float* __restrict__ part, const float* __restrict__ H1, float* dA1,
+                            bf16* dA1b) {
   pdl_trigger();
   pdl_wait();
   const int r = blockIdx.x, c = threadIdx.x;
@@ -177,7 +212,9 @@ __global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
       if (z + q < splitk) a[q] += __ldcs(part + (int64_t)(z + q) * part_stride + o);
   }
   const float s = ((a[0] + a[1]) + (a[2] + a[3])) + ((a[4] + a[5]) + (a[6] + a[7]));
-  dA1[o] = H1[o] > 0.f ? s : 0.f;
+  const float v = H1[o] > 0.f ? s : 0.f;
+  dA1[o] = v;
+  if (dA1b) dA1b[o] = __float2bfloat16_rn(v);
 }
 
 // db1[c] = sum_r dA1[r][c] (one warp per column, lanes over rows, fixed shuffle
@@ -280,9 +317,10 @@ cudaError_t launch_softmax_ce(const Launch& lc, int n, int64_t L, int64_t ldz, c
 }
 
 cudaError_t launch_dh_reduce(const Launch& lc, int n, int H, int splitk, const Ptrs& P,
-                             const WsLayout& L) {
+                             const WsLayout& L, bool want_bf16) {
   // split-K partial z of dH1 lives at dhpart + z * (b_max * H)
-  launch_k(lc, k_dh_reduce, dim3(n), dim3(H), 0, n, H, splitk, L.part_stride, P.dhpart, P.h1, P.da1);
+  launch_k(lc, k_dh_reduce, dim3(n), dim3(H), 0, n, H, splitk, L.part_stride, P.dhpart, P.h1, P.da1,
+                  want_bf16 ? P.da1b : nullptr);
   return cudaGetLastError();
 }
 

@@ -314,12 +314,173 @@ __global__ void __launch_bounds__(256) k_fscan(const int32_t* __restrict__ cnt, 
   }
 }
 
+// -------------------------------------------------------------------------
+// K-0 (b-e) fused: one persistent kernel of kTouchCtas co-operating CTAs with
+// software grid barriers (the only other work on the GPU is the dense chain on
+// other streams, which never waits for this kernel, so every CTA eventually
+// runs).  Phases:
+//   A  cnt[f] += 1 per batch entry
+//   B  tile sums of (cnt, [cnt > 0]) over F;  C  prefix + segment starts fseg,
+//      ranks fuid, sorted unique ids uniq, segment offsets useg
+//   D  row bitmap of every touched feature: bits[u][r / 32] |= 1 << r % 32
+//   E  deterministic placement: the entry of row r in feature f's segment goes
+//      to fseg[f] + #{rows r' < r of the batch containing f} (popcounts), so
+//      every segment is sorted by row without a sort
+//   F  cnt and bitmaps back to zero for the next step
+// -------------------------------------------------------------------------
+constexpr int kTouchCtas = 64;
+
+__device__ __forceinline__ void grid_barrier(unsigned long long* ctr) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const unsigned long long arrive = atomicAdd(ctr, 1ull) + 1ull;
+    const unsigned long long goal = (arrive + gridDim.x - 1) / gridDim.x * gridDim.x;
+    volatile unsigned long long* vc = ctr;
+    while (*vc < goal) __nanosleep(64);
+    __threadfence();
+  }
+  __syncthreads();
+}
+
+__global__ void __launch_bounds__(512) k_touched(int n, const int64_t* __restrict__ rbase,
+                                                 const int32_t* __restrict__ col,
+                                                 const float* __restrict__ val,
+                                                 const int32_t* __restrict__ boff, int32_t* meta,
+                                                 int32_t* cnt, int32_t* tsum, int64_t F, int ntiles,
+                                                 int32_t* fseg, int32_t* fuid, int32_t* uniq,
+                                                 int32_t* useg, uint32_t* bits, int W, int32_t* e_n,
+                                                 float* e_v, int32_t* e_u, int32_t* e_f) {
+  pdl_trigger();
+  pdl_wait();
+  extern __shared__ int32_t sboff[];
+  __shared__ int s_red[2][16];
+  __shared__ int s_pre[2];
+  unsigned long long* bar = reinterpret_cast<unsigned long long*>(meta + M_BAR);
+  load_view(sboff, boff, rbase, n);
+  const int nnz = meta[M_NNZ];
+  const int gt = blockIdx.x * blockDim.x + threadIdx.x, gs = gridDim.x * blockDim.x;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  // ---- A
+  for (int e = gt; e < nnz; e += gs) {
+    int r;
+    atomicAdd(&cnt[col[entry_index(sboff, n, e, &r)]], 1);
+  }
+  grid_barrier(bar);
+  // ---- B: tile sums (kScanTile features per tile, 2 per thread at 512 threads)
+  constexpr int PER = kScanTile / 512;
+  for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    const int64_t f0 = (int64_t)t * kScanTile + threadIdx.x * PER;
+    int a = 0, b = 0;
+#pragma unroll
+    for (int i = 0; i < PER; ++i) {
+      const int c = (f0 + i < F) ? cnt[f0 + i] : 0;
+      a += c; b += (c > 0);
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) { a += __shfl_xor_sync(kFull, a, o); b += __shfl_xor_sync(kFull, b, o); }
+    if (lane == 0) { s_red[0][wid] = a; s_red[1][wid] = b; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      int x = 0, y = 0;
+      for (int w = 0; w < nw; ++w) { x += s_red[0][w]; y += s_red[1][w]; }
+      tsum[2 * t] = x; tsum[2 * t + 1] = y;
+    }
+    __syncthreads();
+  }
+  grid_barrier(bar);
+  // ---- C: prefix of the earlier tiles + in-tile scan
+  for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    int a = 0, b = 0;
+    for (int j = threadIdx.x; j < t; j += blockDim.x) { a += tsum[2 * j]; b += tsum[2 * j + 1]; }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) { a += __shfl_xor_sync(kFull, a, o); b += __shfl_xor_sync(kFull, b, o); }
+    if (lane == 0) { s_red[0][wid] = a; s_red[1][wid] = b; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      int x = 0, y = 0;
+      for (int w = 0; w < nw; ++w) { x += s_red[0][w]; y += s_red[1][w]; }
+      s_pre[0] = x; s_pre[1] = y;
+      if (t == ntiles - 1) {
+        meta[M_U] = y + tsum[2 * t + 1];
+        useg[y + tsum[2 * t + 1]] = x + tsum[2 * t];
+      }
+    }
+    __syncthreads();
+    const int64_t f0 = (int64_t)t * kScanTile + threadIdx.x * PER;
+    int c[PER];
+    int ta = 0, tb = 0;
+#pragma unroll
+    for (int i = 0; i < PER; ++i) {
+      c[i] = (f0 + i < F) ? cnt[f0 + i] : 0;
+      ta += c[i]; tb += (c[i] > 0);
+    }
+    // block exclusive scan of (ta, tb)
+    int xa = ta, xb = tb;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int ya = __shfl_up_sync(kFull, xa, o), yb = __shfl_up_sync(kFull, xb, o);
+      if (lane >= o) { xa += ya; xb += yb; }
+    }
+    __syncthreads();
+    if (lane == 31) { s_red[0][wid] = xa; s_red[1][wid] = xb; }
+    __syncthreads();
+    int oa = 0, ob = 0;
+    for (int w = 0; w < wid; ++w) { oa += s_red[0][w]; ob += s_red[1][w]; }
+    int pa = s_pre[0] + oa + xa - ta, pb = s_pre[1] + ob + xb - tb;
+#pragma unroll
+    for (int i = 0; i < PER; ++i) {
+      if (c[i] > 0) {
+        fseg[f0 + i] = pa;
+        fuid[f0 + i] = pb;
+        uniq[pb] = (int32_t)(f0 + i);
+        useg[pb] = pa;
+        ++pb;
+      }
+      pa += c[i];
+    }
+    __syncthreads();
+  }
+  grid_barrier(bar);
+  // ---- D: row bitmaps
+  for (int e = gt; e < nnz; e += gs) {
+    int r;
+    const int f = col[entry_index(sboff, n, e, &r)];
+    atomicOr(&bits[(int64_t)fuid[f] * W + (r >> 5)], 1u << (r & 31));
+  }
+  grid_barrier(bar);
+  // ---- E: placement
+  for (int e = gt; e < nnz; e += gs) {
+    int r;
+    const int64_t k = entry_index(sboff, n, e, &r);
+    const int f = col[k];
+    const int u = fuid[f];
+    const uint32_t* bw = bits + (int64_t)u * W;
+    int rank = __popc(bw[r >> 5] & ((1u << (r & 31)) - 1u));
+    for (int w = 0; w < (r >> 5); ++w) rank += __popc(bw[w]);
+    const int pos = fseg[f] + rank;
+    e_n[pos] = r;
+    e_v[pos] = val[k];
+    e_u[pos] = u;
+    e_f[pos] = f;
+  }
+  grid_barrier(bar);
+  // ---- F: reset for the next step
+  for (int e = gt; e < nnz; e += gs) {
+    int r;
+    const int f = col[entry_index(sboff, n, e, &r)];
+    cnt[f] = 0;
+    bits[(int64_t)fuid[f] * W + (r >> 5)] = 0u;
+  }
+}
+
 // K-0 (e): scatter entries into their feature segment (cnt returns to zero)
 __global__ void k_place(int n, const int64_t* __restrict__ rbase,
                         const int32_t* __restrict__ col, const float* __restrict__ val,
                         const int32_t* __restrict__ boff, const int32_t* __restrict__ meta,
                         int32_t* cnt, const int32_t* __restrict__ fseg,
-                        const int32_t* __restrict__ fuid, int32_t* e_n, float* e_v, int32_t* e_u) {
+                        const int32_t* __restrict__ fuid, int32_t* e_n, float* e_v, int32_t* e_u,
+                        int32_t* e_f) {
   pdl_trigger();
   pdl_wait();
   extern __shared__ int32_t sboff[];
@@ -333,6 +494,7 @@ __global__ void k_place(int n, const int64_t* __restrict__ rbase,
     e_n[pos] = r;
     e_v[pos] = val[k];
     e_u[pos] = fuid[f];
+    e_f[pos] = f;
   }
 }
 
@@ -609,6 +771,192 @@ __global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__
   }
 }
 
+// K-5 with the batch's dA1 column slice staged in shared memory (one CTA per SM,
+// grid.y = column slice).  Gathers become shared-memory reads; per piece only the
+// entry list, the segment bounds and the touched W1 row go to L2/HBM.  Same
+// pieces, combine order and results as k_scatter_sgd (bitwise, for T = float).
+template <typename T, int CPL>
+struct SliceIO {
+  // lane's CPL contiguous columns of a staged row -> fp32
+  __device__ __forceinline__ static void load(const T* row, int lane, float (&v)[CPL]) {
+    if constexpr (sizeof(T) == 2) {
+      if constexpr (CPL == 8) {
+        uint4 q = reinterpret_cast<const uint4*>(row)[lane];
+        const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&q);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) { float2 f = __bfloat1622float2(h[i]); v[2 * i] = f.x; v[2 * i + 1] = f.y; }
+      } else if constexpr (CPL == 4) {
+        uint2 q = reinterpret_cast<const uint2*>(row)[lane];
+        const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&q);
+#pragma unroll
+        for (int i = 0; i < 2; ++i) { float2 f = __bfloat1622float2(h[i]); v[2 * i] = f.x; v[2 * i + 1] = f.y; }
+      } else {
+        float2 f = __bfloat1622float2(reinterpret_cast<const __nv_bfloat162*>(row)[lane]);
+        v[0] = f.x; v[1] = f.y;
+      }
+    } else {
+      if constexpr (CPL >= 4) {
+#pragma unroll
+        for (int i = 0; i < CPL / 4; ++i) {
+          float4 f = reinterpret_cast<const float4*>(row)[lane * (CPL / 4) + i];
+          v[4 * i] = f.x; v[4 * i + 1] = f.y; v[4 * i + 2] = f.z; v[4 * i + 3] = f.w;
+        }
+      } else {
+        float2 f = reinterpret_cast<const float2*>(row)[lane];
+        v[0] = f.x; v[1] = f.y;
+      }
+    }
+  }
+};
+
+template <int CPL>
+__device__ __forceinline__ void ld_cols(const float* p, float (&v)[CPL], bool cg) {
+#pragma unroll
+  for (int i = 0; i < CPL; i += (CPL >= 4 ? 4 : 2)) {
+    if constexpr (CPL >= 4) {
+      float4 f = cg ? __ldcg(reinterpret_cast<const float4*>(p + i)) : *reinterpret_cast<const float4*>(p + i);
+      v[i] = f.x; v[i + 1] = f.y; v[i + 2] = f.z; v[i + 3] = f.w;
+    } else {
+      float2 f = cg ? __ldcg(reinterpret_cast<const float2*>(p + i)) : *reinterpret_cast<const float2*>(p + i);
+      v[i] = f.x; v[i + 1] = f.y;
+    }
+  }
+}
+template <int CPL>
+__device__ __forceinline__ void st_cols(float* p, const float (&v)[CPL], bool cg) {
+#pragma unroll
+  for (int i = 0; i < CPL; i += (CPL >= 4 ? 4 : 2)) {
+    if constexpr (CPL >= 4) {
+      const float4 f = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+      if (cg) __stcg(reinterpret_cast<float4*>(p + i), f); else *reinterpret_cast<float4*>(p + i) = f;
+    } else {
+      const float2 f = make_float2(v[i], v[i + 1]);
+      if (cg) __stcg(reinterpret_cast<float2*>(p + i), f); else *reinterpret_cast<float2*>(p + i) = f;
+    }
+  }
+}
+
+template <typename T, int CPL>
+__global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restrict__ e_n,
+                                                          const float* __restrict__ e_v,
+                                                          const int32_t* __restrict__ e_u,
+                                                          const int32_t* __restrict__ e_f,
+                                                          const int32_t* __restrict__ useg,
+                                                          const int32_t* __restrict__ meta,
+                                                          const T* __restrict__ dA1, int H, float* W1,
+                                                          float lr, float* part, int32_t* ucnt,
+                                                          float* grad_w1) {
+  pdl_trigger();
+  pdl_wait();
+  constexpr int CS = 32 * CPL;               // columns of this CTA's slice
+  constexpr int kU = 8;
+  extern __shared__ __align__(16) uint8_t sm_raw[];
+  T* sd = reinterpret_cast<T*>(sm_raw);      // [n][CS]
+  const int nsl = gridDim.y, slice = blockIdx.y, c0 = slice * CS;
+  const int n = meta[M_NROWS];
+  {  // stage dA1[:, c0 : c0 + CS] (16-byte chunks, 8 loads in flight per thread)
+    constexpr int CH = CS * (int)sizeof(T) / 16;
+    const uint4* src = reinterpret_cast<const uint4*>(dA1);
+    uint4* dst = reinterpret_cast<uint4*>(sd);
+    const int rowchunks = H * (int)sizeof(T) / 16;
+    const int total = n * CH;
+    for (int i0 = threadIdx.x; i0 < total; i0 += 8 * blockDim.x) {
+      uint4 v[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const int i = i0 + k * blockDim.x;
+        if (i < total) v[k] = __ldg(src + (int64_t)(i / CH) * rowchunks + slice * CH + (i % CH));
+      }
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const int i = i0 + k * blockDim.x;
+        if (i < total) dst[i] = v[k];
+      }
+    }
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int nnz = meta[M_NNZ];
+  const int npieces = (nnz + kPiece - 1) / kPiece;
+  const int nwarps = gridDim.x * (blockDim.x >> 5);
+  using IO = SliceIO<T, CPL>;
+  for (int p = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); p < npieces; p += nwarps) {
+    const int e0 = p * kPiece, e1 = min(e0 + kPiece, nnz), cnt = e1 - e0;
+    // one round trip for the whole piece: entries + the neighbours' features
+    int myn = 0, myf = -1, myu = 0;
+    float myv = 0.f;
+    if (lane < cnt) { myn = e_n[e0 + lane]; myv = e_v[e0 + lane]; myf = e_f[e0 + lane]; myu = e_u[e0 + lane]; }
+    int nb = -1;
+    if (lane == 0 && e0 > 0) nb = e_f[e0 - 1];
+    if (lane == 1 && e1 < nnz) nb = e_f[e1];
+    const int fprev = __shfl_sync(kFull, nb, 0), fnext = __shfl_sync(kFull, nb, 1);
+    const int fup = __shfl_up_sync(kFull, myf, 1);
+    uint32_t smask = __ballot_sync(kFull, lane < cnt && (lane == 0 || myf != fup));
+    while (smask) {
+      const int j0 = __ffs(smask) - 1;
+      smask &= smask - 1;
+      const int j1 = smask ? __ffs(smask) - 1 : cnt;
+      const int f = __shfl_sync(kFull, myf, j0), u = __shfl_sync(kFull, myu, j0);
+      const bool before = (j0 == 0 && fprev == f), after = (j1 == cnt && fnext == f);
+      float* wrow = W1 + (int64_t)f * H + c0 + lane * CPL;
+      float w[CPL];
+      if (!before && !after) ld_cols<CPL>(wrow, w, false);     // in flight during the gathers
+      float acc[CPL];
+#pragma unroll
+      for (int i = 0; i < CPL; ++i) acc[i] = 0.f;
+      int j = j0;
+      for (; j + kU <= j1; j += kU) {
+        float g[kU][CPL];
+#pragma unroll
+        for (int q = 0; q < kU; ++q) IO::load(sd + (int64_t)__shfl_sync(kFull, myn, j + q) * CS, lane, g[q]);
+#pragma unroll
+        for (int q = 0; q < kU; ++q) {
+          const float v = __shfl_sync(kFull, myv, j + q);
+#pragma unroll
+          for (int i = 0; i < CPL; ++i) acc[i] = fmaf(v, g[q][i], acc[i]);
+        }
+      }
+      for (; j < j1; ++j) {
+        float g[CPL];
+        IO::load(sd + (int64_t)__shfl_sync(kFull, myn, j) * CS, lane, g);
+        const float v = __shfl_sync(kFull, myv, j);
+#pragma unroll
+        for (int i = 0; i < CPL; ++i) acc[i] = fmaf(v, g[i], acc[i]);
+      }
+      bool finish = !before && !after;
+      if (!finish) {
+        const int slot = before ? 2 * p : 2 * p + 1;
+        st_cols<CPL>(part + (int64_t)slot * H + c0 + lane * CPL, acc, true);
+        __threadfence();
+        int old = 0;
+        if (lane == 0) old = atomicAdd(&ucnt[(int64_t)u * nsl + slice], 1);
+        old = __shfl_sync(kFull, old, 0);
+        const int q0 = useg[u] / kPiece, q1 = (useg[u + 1] - 1) / kPiece;
+        if (old == q1 - q0) {
+          __threadfence();
+          ld_cols<CPL>(wrow, w, false);
+#pragma unroll
+          for (int i = 0; i < CPL; ++i) acc[i] = 0.f;
+          for (int q = q0; q <= q1; ++q) {
+            float t[CPL];
+            ld_cols<CPL>(part + (int64_t)(q == q0 ? 2 * q + 1 : 2 * q) * H + c0 + lane * CPL, t, true);
+#pragma unroll
+            for (int i = 0; i < CPL; ++i) acc[i] += t[i];
+          }
+          if (lane == 0) ucnt[(int64_t)u * nsl + slice] = 0;
+          finish = true;
+        }
+      }
+      if (finish) {
+#pragma unroll
+        for (int i = 0; i < CPL; ++i) w[i] = w[i] - lr * acc[i];
+        st_cols<CPL>(wrow, w, false);
+        if (grad_w1) st_cols<CPL>(grad_w1 + (int64_t)f * H + c0 + lane * CPL, acc, false);
+      }
+    }
+  }
+}
+
 // One resident wave of 256-thread CTAs (occupancy from the compiled kernel), no
 // more CTAs than there are 8-piece groups for the largest step.
 template <typename K>
@@ -655,17 +1003,11 @@ cudaError_t launch_touched(const Launch& lc, const int32_t* rows, int n, const i
                            const int32_t* col, const float* val, int64_t F, const Ptrs& P,
                            const WsLayout& L, int b_max) {
   const size_t smem = view_smem(n);
-  const int grid = lc.sms * 4;
   const int nt = (int)L.n_tiles_f;
-  unsigned long long* status = reinterpret_cast<unsigned long long*>(P.tsum);
-  launch_k(lc, k_count, dim3(grid), dim3(256), smem, n, P.rbase, col, P.boff, P.meta, P.cnt, status, nt);
-  launch_k(lc, k_fscan, dim3(nt), dim3(256), 0, P.cnt, F, status, nt, P.meta, P.fseg, P.fuid, P.uniq, P.useg);
-  launch_k(lc, k_place, dim3(grid), dim3(256), smem, n, P.rbase, col, val, P.boff, P.meta, P.cnt, P.fseg,
-                                     P.fuid, P.e_n, P.e_v, P.e_u);
-  const int words = (b_max + 31) / 32;
-  const size_t ssmem = (size_t)8 * words * 33 * sizeof(uint32_t);
-  launch_k(lc, k_segsort, dim3(lc.sms * 2), dim3(256), ssmem, P.useg, P.meta, P.e_n, P.e_v, words);
-  return cudaGetLastError();
+  const int W = (b_max + 31) / 32;
+  return launch_k(lc, k_touched, dim3(std::min(kTouchCtas, lc.sms)), dim3(512), smem, n, P.rbase, col, val,
+                  P.boff, P.meta, P.cnt, P.tsum, F, nt, P.fseg, P.fuid, P.uniq, P.useg, P.bits, W, P.e_n,
+                  P.e_v, P.e_u, P.e_f);
 }
 
 cudaError_t launch_spmm_fwd(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
@@ -680,8 +1022,45 @@ cudaError_t launch_spmm_fwd(const Launch& lc, const int32_t* rows, int n, const 
   }
 }
 
+template <typename T, int CPL>
+cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float* W1, float lr,
+                        const Ptrs& P, float* grad_w1) {
+  constexpr int CS = 32 * CPL;
+  const int nsl = H / CS;
+  const size_t smem = (size_t)b_max * CS * sizeof(T);
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(k_scatter_sgd_s<T, CPL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         200 * 1024);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  const int gx = std::max(1, lc.sms / nsl);
+  return launch_k(lc, k_scatter_sgd_s<T, CPL>, dim3(gx, nsl), dim3(512), smem, P.e_n, P.e_v, P.e_u,
+                  P.e_f, P.useg, P.meta, dA1, H, W1, lr, P.part5, P.ucnt, grad_w1);
+}
+
+// Widest column slice whose staged dA1 fits 160 KB of shared memory (0 = none).
+int scatter_slice(int H, int b_max, size_t elem) {
+  for (int cs = std::min(H, 256); cs >= 64; cs /= 2)
+    if (H % cs == 0 && (size_t)b_max * cs * elem <= 160 * 1024) return cs;
+  return 0;
+}
+
 cudaError_t launch_scatter_sgd(const Launch& lc, float* W1, int H, float lr, const Ptrs& P,
-                               const WsLayout& L, float* grad_w1) {
+                               const WsLayout& L, float* grad_w1, const bf16* dA1b, int b_max) {
+  const size_t elem = dA1b ? 2 : 4;
+  const int cs = scatter_slice(H, b_max, elem);
+  if (cs) {
+    if (dA1b) {
+      if (cs == 256) return scatter_s_t<bf16, 8>(lc, dA1b, H, b_max, W1, lr, P, grad_w1);
+      if (cs == 128) return scatter_s_t<bf16, 4>(lc, dA1b, H, b_max, W1, lr, P, grad_w1);
+      return scatter_s_t<bf16, 2>(lc, dA1b, H, b_max, W1, lr, P, grad_w1);
+    }
+    if (cs == 256) return scatter_s_t<float, 8>(lc, P.da1, H, b_max, W1, lr, P, grad_w1);
+    if (cs == 128) return scatter_s_t<float, 4>(lc, P.da1, H, b_max, W1, lr, P, grad_w1);
+    return scatter_s_t<float, 2>(lc, P.da1, H, b_max, W1, lr, P, grad_w1);
+  }
   switch (H) {
     case 64: return scatter_t<2>(lc, W1, lr, P, L, grad_w1);
     case 128: return scatter_t<4>(lc, W1, lr, P, L, grad_w1);

@@ -233,12 +233,30 @@ __global__ void __launch_bounds__(256, 1)
     // ------------------------------------------------ epilogue: TMEM -> registers -> global
     const int wq = warp - 4;
     const int m = m0 + wq * 32 + lane;
+    // G3: the W2 row chunk this thread updates is loaded before the MMAs finish,
+    // and chunk c + 32 while chunk c is processed.
+    float4 wcur[8], wnxt[8];
+    const bool wrow_ok = (EPI == TC_EPI_SGD) && m < g.M;
+    if constexpr (EPI == TC_EPI_SGD) {
+      if (wrow_ok) {
+        const float4* w4 = reinterpret_cast<const float4*>(g.out + (int64_t)m * g.ldo + n0);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) wcur[j] = w4[j];
+      }
+    }
     if (nk > 0) {
       mbar_wait(tfull, 0);
       tc_fence_after();
     }
 #pragma unroll 1
     for (int c = 0; c < BN; c += 32) {
+      if constexpr (EPI == TC_EPI_SGD) {
+        if (wrow_ok && c + 32 < BN) {
+          const float4* w4 = reinterpret_cast<const float4*>(g.out + (int64_t)m * g.ldo + n0 + c + 32);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) wnxt[j] = w4[j];
+        }
+      }
       float v[32];
       if (nk > 0) {
         tmem_ld32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)c, v);
@@ -269,7 +287,7 @@ __global__ void __launch_bounds__(256, 1)
         bf16* sh = g.shadow + (int64_t)m * g.ldo + n;
 #pragma unroll
         for (int j = 0; j < 32; j += 4) {
-          float4 x = reinterpret_cast<float4*>(w)[j / 4];
+          float4 x = wcur[j / 4];
           x.x -= g.lr * v[j]; x.y -= g.lr * v[j + 1]; x.z -= g.lr * v[j + 2]; x.w -= g.lr * v[j + 3];
           reinterpret_cast<float4*>(w)[j / 4] = x;
           __nv_bfloat162 p0 = __floats2bfloat162_rn(x.x, x.y), p1 = __floats2bfloat162_rn(x.z, x.w);
@@ -284,6 +302,8 @@ __global__ void __launch_bounds__(256, 1)
           for (int j = 0; j < 32; j += 4)
             reinterpret_cast<float4*>(gr)[j / 4] = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
         }
+#pragma unroll
+        for (int j = 0; j < 8; ++j) wcur[j] = wnxt[j];
       }
     }
     if constexpr (ONES) {
