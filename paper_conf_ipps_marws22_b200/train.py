@@ -91,6 +91,8 @@ def exchange_stats(u: int, b: int, sqnorm: torch.Tensor, P: int, world: int,
                         torch.tensor(float(b), dtype=torch.float64, device=dev),
                         sqnorm.reshape(())])
     if world > 1:
+        if dist.get_backend(group) == "gloo":
+            mine = mine.cpu()
         allv = [torch.empty_like(mine) for _ in range(world)]
         dist.all_gather(allv, mine, group=group)
         allv = torch.stack(allv).cpu().numpy()
