@@ -49,6 +49,7 @@ def _args():
     p.add_argument("--cpu-seconds", type=float, default=12.0)
     p.add_argument("--ttp-megabatches", type=int, default=40, help="time-to-P@1 budget (0 = skip)")
     p.add_argument("--lr-max", type=float, default=None)
+    p.add_argument("--train-rows", type=int, default=None, help="generate only the first N train rows")
     return p.parse_args()
 
 
@@ -195,7 +196,9 @@ def main():
     if prec == "auto":
         prec = "bf16" if _bf16_available() else "fp32"
     bf16 = prec == "bf16"
-    data = generate(cfg, "train")
+    data = generate(cfg, "train", a.train_rows)
+    if a.train_rows:
+        cfg = config(a.config, n_train=data.n_rows)
     w0 = init_params(cfg)
     nz, nl = api.max_step_sizes([data], cfg.b_max)
     rep = api.Replica(cfg.F, cfg.L, cfg.H, cfg.b_max, nz, nl, prec, device=local, w0=w0)
@@ -305,7 +308,7 @@ def main():
             "warmup": W, "ms_per_step": round(t_max / K, 4), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "bf16" if bf16 else "f32",
             "data": "synthetic",
-            "config": {"workload": cfg.name, "F": cfg.F, "L": cfg.L, "H": cfg.H, "b_max": cfg.b_max,
+            "config": {"workload": cfg.name, "train_rows": int(data.n_rows), "F": cfg.F, "L": cfg.L, "H": cfg.H, "b_max": cfg.b_max,
                        "mega_batch_samples": M, "step": "1 mega-batch = local steps + merge",
                        "precision": prec, "l2": "flushed (256 MiB write) between timed steps",
                        "inflight": a.inflight, "parallelism": f"dp{world} (model averaging)",

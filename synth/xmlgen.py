@@ -31,6 +31,7 @@ from __future__ import annotations
 
 import dataclasses
 import math
+import os
 from typing import Dict, Optional
 
 import numpy as np
@@ -177,14 +178,16 @@ def _poisson_inv(lam: float, u: np.ndarray, kmax: int) -> np.ndarray:
 def _first_k_distinct(row, pos, ident, k_row, n_ids):
     """Per row keep the first k_row[row] distinct ids in `pos` order.
 
-    Returns (row, ident, rank) of the kept entries sorted by (row, rank)."""
-    key = row * np.int64(n_ids) + ident
-    order = np.lexsort((pos, key))
-    ks = key[order]
+    Returns (row, ident, rank) of the kept entries sorted by (row, rank).
+    (row, id, pos) are packed into one int64 sort key (rows < 2^20 per chunk,
+    ids < 2^23, positions < 2^20)."""
+    key = ((row.astype(np.int64) * np.int64(n_ids) + ident) << np.int64(20)) | pos.astype(np.int64)
+    order = np.argsort(key, kind="stable")
+    ks = key[order] >> np.int64(20)
     first = np.ones(len(ks), dtype=bool)
     first[1:] = ks[1:] != ks[:-1]
     keep = order[first]
-    keep = keep[np.lexsort((pos[keep], row[keep]))]
+    keep = keep[np.argsort((row[keep].astype(np.int64) << np.int64(20)) | pos[keep], kind="stable")]
     r = row[keep]
     # rank within row
     starts = np.searchsorted(r, r, side="left")
@@ -233,79 +236,95 @@ class Dataset:
 
 
 def _gen_split(cfg: XmlConfig, split: int, n: int, chunk: int = 32768) -> Dataset:
-    seed, F, L = cfg.seed, cfg.F, cfg.L
-    cdf_F, cdf_L = _zipf_cdf(F), _zipf_cdf(L)
-    scr_F = _scramble(seed, 10, F)
-    scr_L = _scramble(seed, 9, L)
-    # label signatures: 16 uniform features per label (stream 5)
-    sig = np.floor(_u01(_hash(seed, 5, np.arange(L, dtype=np.int64)[:, None],
-                              np.arange(16, dtype=np.int64)[None, :])) * F).astype(np.int64)
-    mu = math.log(cfg.s_bar) - 0.5 * cfg.s_sigma ** 2
-    rp_parts, col_parts, val_parts, lp_parts, lab_parts = [], [], [], [], []
-    for r0 in range(0, n, chunk):
-        rows = np.arange(r0, min(n, r0 + chunk), dtype=np.int64)
-        nr = len(rows)
-        # --- nnz per row (streams 0, 8)
-        z = _normal(seed, 0, split, rows)
-        s = np.exp(mu + cfg.s_sigma * z)
-        if cfg.block_skew:
-            blk = rows // 64
-            zb = _normal(seed, 8, split, blk)
-            s = s * np.exp(-0.5 + 1.0 * zb)
-        s_n = np.clip(np.rint(s), 1, F).astype(np.int64)
-        # --- labels (streams 3, 4)
-        kmax = int(cfg.y_bar * 6 + 20)
-        c_n = 1 + _poisson_inv(cfg.y_bar - 1.0, _u01(_hash(seed, 3, split, rows)), kmax)
-        c_n = np.minimum(c_n, L).astype(np.int64)
-        nl_cand = 2 * c_n + 4
-        lrow = np.repeat(np.arange(nr), nl_cand)
-        lpos = np.arange(len(lrow)) - np.repeat(np.cumsum(nl_cand) - nl_cand, nl_cand)
-        u = _u01(_hash(seed, 4, split, rows[lrow], lpos))
-        lid = scr_L[_zipf_rank(cdf_L, u)]
-        lr_, lid_, _ = _first_k_distinct(lrow, lpos, lid, c_n, L)
-        order = np.lexsort((lid_, lr_))
-        lr_, lid_ = lr_[order], lid_[order]
-        lcnt = np.bincount(lr_, minlength=nr)
-        lptr = np.zeros(nr + 1, dtype=np.int64)
-        np.cumsum(lcnt, out=lptr[1:])
-        # --- features (stream 1): signature draws then Zipf noise draws
-        n_sig = s_n // 2
-        n_noise = 2 * s_n + 8
-        n_cand = n_sig + n_noise
-        frow = np.repeat(np.arange(nr), n_cand)
-        fpos = np.arange(len(frow)) - np.repeat(np.cumsum(n_cand) - n_cand, n_cand)
-        h1 = _hash(seed, 1, split, rows[frow], fpos, 0)
-        h2 = _hash(seed, 1, split, rows[frow], fpos, 1)
-        is_sig = fpos < n_sig[frow]
-        # signature draw: a random label of the row, a random one of its 16 ids
-        nlab_row = lcnt[frow]
-        pick = np.minimum((_u01(h1) * nlab_row).astype(np.int64), nlab_row - 1)
-        lab_of = lid_[lptr[frow] + pick]
-        k16 = np.minimum((_u01(h2) * 16).astype(np.int64), 15)
-        fid_sig = sig[lab_of, k16]
-        fid_noise = scr_F[_zipf_rank(cdf_F, _u01(h1))]
-        fid = np.where(is_sig, fid_sig, fid_noise)
-        fr_, fid_, frank = _first_k_distinct(frow, fpos, fid, s_n, F)
-        # --- values (stream 2): U(0.5, 1.5), L2-normalised per row
-        v = 0.5 + _u01(_hash(seed, 2, split, rows[fr_], frank))
-        sq = np.bincount(fr_, weights=v * v, minlength=nr)
-        v = v / np.sqrt(sq)[fr_]
-        order = np.lexsort((fid_, fr_))
-        fr_, fid_, v = fr_[order], fid_[order], v[order]
-        fcnt = np.bincount(fr_, minlength=nr)
-        rp_parts.append(fcnt)
-        col_parts.append(fid_.astype(np.int32))
-        val_parts.append(v.astype(np.float32))
-        lp_parts.append(lcnt)
-        lab_parts.append(lid_.astype(np.int32))
-    fc = np.concatenate(rp_parts)
-    lc = np.concatenate(lp_parts)
+    """Rows are generated in independent chunks (in parallel worker processes
+    for large splits); the result does not depend on the chunking."""
+    starts = list(range(0, n, chunk))
+    workers = min(len(starts), os.cpu_count() or 1, 16)
+    if workers > 1 and n >= 4 * chunk:
+        import multiprocessing as mp
+        with mp.get_context("fork").Pool(workers) as pool:
+            parts = pool.starmap(_gen_rows, [(cfg, split, r0, min(n, r0 + chunk)) for r0 in starts])
+    else:
+        parts = [_gen_rows(cfg, split, r0, min(n, r0 + chunk)) for r0 in starts]
+    fc = np.concatenate([p[0] for p in parts])
+    lc = np.concatenate([p[3] for p in parts])
     row_ptr = np.zeros(n + 1, dtype=np.int64)
     np.cumsum(fc, out=row_ptr[1:])
     lab_ptr = np.zeros(n + 1, dtype=np.int64)
     np.cumsum(lc, out=lab_ptr[1:])
-    return Dataset(row_ptr, np.concatenate(col_parts), np.concatenate(val_parts),
-                   lab_ptr, np.concatenate(lab_parts), F, L)
+    return Dataset(row_ptr, np.concatenate([p[1] for p in parts]), np.concatenate([p[2] for p in parts]),
+                   lab_ptr, np.concatenate([p[4] for p in parts]), cfg.F, cfg.L)
+
+
+_TABLES = {}
+
+
+def _tables(cfg: XmlConfig):
+    key = (cfg.seed, cfg.F, cfg.L)
+    if key not in _TABLES:
+        seed, F, L = cfg.seed, cfg.F, cfg.L
+        sig = np.floor(_u01(_hash(seed, 5, np.arange(L, dtype=np.int64)[:, None],
+                                  np.arange(16, dtype=np.int64)[None, :])) * F).astype(np.int64)
+        _TABLES[key] = (_zipf_cdf(F), _zipf_cdf(L), _scramble(seed, 10, F), _scramble(seed, 9, L), sig)
+    return _TABLES[key]
+
+
+def _gen_rows(cfg: XmlConfig, split: int, r0: int, r1: int):
+    """Rows [r0, r1) of a split: (feature counts, cols, vals, label counts, labels)."""
+    seed, F, L = cfg.seed, cfg.F, cfg.L
+    cdf_F, cdf_L, scr_F, scr_L, sig = _tables(cfg)
+    mu = math.log(cfg.s_bar) - 0.5 * cfg.s_sigma ** 2
+    rows = np.arange(r0, r1, dtype=np.int64)
+    nr = len(rows)
+    # --- nnz per row (streams 0, 8)
+    z = _normal(seed, 0, split, rows)
+    s = np.exp(mu + cfg.s_sigma * z)
+    if cfg.block_skew:
+        blk = rows // 64
+        zb = _normal(seed, 8, split, blk)
+        s = s * np.exp(-0.5 + 1.0 * zb)
+    s_n = np.clip(np.rint(s), 1, F).astype(np.int64)
+    # --- labels (streams 3, 4)
+    kmax = int(cfg.y_bar * 6 + 20)
+    c_n = 1 + _poisson_inv(cfg.y_bar - 1.0, _u01(_hash(seed, 3, split, rows)), kmax)
+    c_n = np.minimum(c_n, L).astype(np.int64)
+    nl_cand = 2 * c_n + 4
+    lrow = np.repeat(np.arange(nr), nl_cand)
+    lpos = np.arange(len(lrow)) - np.repeat(np.cumsum(nl_cand) - nl_cand, nl_cand)
+    u = _u01(_hash(seed, 4, split, rows[lrow], lpos))
+    lid = scr_L[_zipf_rank(cdf_L, u)]
+    lr_, lid_, _ = _first_k_distinct(lrow, lpos, lid, c_n, L)
+    order = np.lexsort((lid_, lr_))
+    lr_, lid_ = lr_[order], lid_[order]
+    lcnt = np.bincount(lr_, minlength=nr)
+    lptr = np.zeros(nr + 1, dtype=np.int64)
+    np.cumsum(lcnt, out=lptr[1:])
+    # --- features (stream 1): signature draws then Zipf noise draws
+    n_sig = s_n // 2
+    n_noise = 2 * s_n + 8
+    n_cand = n_sig + n_noise
+    frow = np.repeat(np.arange(nr), n_cand)
+    fpos = np.arange(len(frow)) - np.repeat(np.cumsum(n_cand) - n_cand, n_cand)
+    h1 = _hash(seed, 1, split, rows[frow], fpos, 0)
+    h2 = _hash(seed, 1, split, rows[frow], fpos, 1)
+    is_sig = fpos < n_sig[frow]
+    # signature draw: a random label of the row, a random one of its 16 ids
+    nlab_row = lcnt[frow]
+    pick = np.minimum((_u01(h1) * nlab_row).astype(np.int64), nlab_row - 1)
+    lab_of = lid_[lptr[frow] + pick]
+    k16 = np.minimum((_u01(h2) * 16).astype(np.int64), 15)
+    fid_sig = sig[lab_of, k16]
+    fid_noise = scr_F[_zipf_rank(cdf_F, _u01(h1))]
+    fid = np.where(is_sig, fid_sig, fid_noise)
+    fr_, fid_, frank = _first_k_distinct(frow, fpos, fid, s_n, F)
+    # --- values (stream 2): U(0.5, 1.5), L2-normalised per row
+    v = 0.5 + _u01(_hash(seed, 2, split, rows[fr_], frank))
+    sq = np.bincount(fr_, weights=v * v, minlength=nr)
+    v = v / np.sqrt(sq)[fr_]
+    order = np.lexsort((fid_, fr_))
+    fr_, fid_, v = fr_[order], fid_[order], v[order]
+    fcnt = np.bincount(fr_, minlength=nr)
+    return fcnt, fid_.astype(np.int32), v.astype(np.float32), lcnt, lid_.astype(np.int32)
 
 
 def generate(cfg: XmlConfig, split: str = "train", n_rows: Optional[int] = None) -> Dataset:
