@@ -110,6 +110,8 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.b2part = take((size_t)b2_chunks() * Lb * 4);
   L.rbase = take((size_t)(B + 1) * 8);
   L.da1b = take(bf ? (size_t)B * H * 2 : 0);
+  L.stats_ld = B;
+  L.zstat = take(bf ? (size_t)((Lb + 31) / 32 + 2) * B * 8 : 0);   // G1 softmax partials (2 per N tile)
   L.rowloss = take(B * 4);
   L.dhpart = take((size_t)L.splitk * B * H * 4);
   L.da1 = take(B * H * 4);
@@ -417,8 +419,11 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     Pr.w2b = c->w2b_buf[c->w2b_cur];
     Pw.w2b = c->w2b_buf[c->w2b_cur ^ 1];
     Launch lc3 = c->lc3();
-    PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr));
-    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, true));
+    float2* zstat = reinterpret_cast<float2*>(c->ws + c->L.zstat);
+    int ntiles = 0;
+    PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
+    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, true, zstat, ntiles,
+                                          c->L.stats_ld));
     CU(cudaEventRecord(c->ev_sm, c->s));
     CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
     PCU_ON(c->s3, ASGD_K_G3, launch_gemm_tc(lc3, 3, n, Lb, H, lr, Pw, c->L, W2, b2, g ? g + c->o_w2 : nullptr,

@@ -25,9 +25,9 @@ typedef __nv_bfloat16 bf16;
 struct WsLayout {
   size_t meta, boff, loff, cnt, fseg, fuid, uniq, useg, tsum, tpre;
   size_t e_n, e_v, e_u, e_f, part1, rowcnt, part5, ucnt, bits;
-  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, b2part, rbase, da1b;
+  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, b2part, rbase, da1b, zstat;
   size_t total;
-  int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride;
+  int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride, stats_ld;
 };
 
 WsLayout ws_layout(const asgd_model_desc& d);
@@ -110,9 +110,11 @@ struct GemmArgs {
 cudaError_t launch_gemm_f32(const Launch&, const GemmArgs&);
 // Leading dimension of the B x L logit buffers (16-byte rows for TMA).
 int64_t padded_ld(int64_t L);
+// stats (nullable): G1's per (N tile, row) (max, sum exp) partials -> one pass over Z.
 cudaError_t launch_softmax_ce(const Launch&, int n, int64_t L, int64_t ldz, const int32_t* rows,
                               const int64_t* lab_ptr, const int32_t* lab, const Ptrs&,
-                              bool bf16_out);
+                              bool bf16_out, const float2* stats = nullptr, int ntiles = 0,
+                              int64_t stats_ld = 0);
 cudaError_t launch_dh_reduce(const Launch&, int n, int H, int splitk, const Ptrs&, const WsLayout&,
                              bool want_bf16);
 cudaError_t launch_b1_update(const Launch&, int n, int H, float* b1, float lr, const Ptrs&,
@@ -124,9 +126,10 @@ cudaError_t launch_to_bf16(const Launch&, const float* src, bf16* dst, int64_t c
 bool tc_available();
 // which: 1 = G1 (Z = H1 W2^T + b2), 2 = G2 (dH1 split-K partials), 3 = G3 (W2 -= lr dZ^T H1 and
 // b2 -= lr 1^T dZ, both fused in the epilogue)
+// stats (G1 only, nullable): per (N tile, row) softmax partials; *stats_ntiles = N tiles.
 cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int H, float lr,
                            const Ptrs&, const WsLayout&, float* W2, float* b2, float* grad_w2,
-                           float* grad_b2);
+                           float* grad_b2, float2* stats = nullptr, int* stats_ntiles = nullptr);
 // ---------------------------------------------------------------- merge / eval
 cudaError_t launch_sqnorm(const Launch&, const float* x, int64_t P, double* partials, int nparts,
                           double* out);

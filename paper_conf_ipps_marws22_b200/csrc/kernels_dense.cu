@@ -96,7 +96,9 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
                                                     const int32_t* __restrict__ rows,
                                                     const int64_t* __restrict__ lab_ptr,
                                                     const int32_t* __restrict__ lab, float* Z,
-                                                    bf16* dZb, float* rowloss) {
+                                                    bf16* dZb, float* rowloss,
+                                                    const float2* __restrict__ stats, int ntiles,
+                                                    int64_t stats_ld) {
   pdl_trigger();
   pdl_wait();
   __shared__ int s_lab[kMaxRowLabels];
@@ -114,10 +116,19 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
     s_lab[i] = y;
     s_lz[i] = z[y];
   }
-  // pass 1: online max / sum-exp, kSU loads in flight per thread
+  // pass 1: online max / sum-exp, kSU loads in flight per thread -- or, when G1
+  // left per-tile partials, combine those instead of re-reading the row.
   constexpr int kSU = 8;
   float m = -INFINITY, s = 0.f;
-  for (int64_t j0 = threadIdx.x; j0 < L; j0 += (int64_t)kSU * blockDim.x) {
+  if (stats) {
+    for (int t = threadIdx.x; t < ntiles; t += blockDim.x) {
+      const float2 p = stats[(int64_t)t * stats_ld + n];
+      if (p.x == -INFINITY) continue;
+      if (p.x > m) { s = (m == -INFINITY ? 0.f : s * __expf(m - p.x)) + p.y; m = p.x; }
+      else s += p.y * __expf(p.x - m);
+    }
+  }
+  for (int64_t j0 = stats ? L : threadIdx.x; j0 < L; j0 += (int64_t)kSU * blockDim.x) {
     float v[kSU];
 #pragma unroll
     for (int k = 0; k < kSU; ++k) {
@@ -310,9 +321,9 @@ cudaError_t launch_gemm_f32(const Launch& lc, const GemmArgs& g) {
 
 cudaError_t launch_softmax_ce(const Launch& lc, int n, int64_t L, int64_t ldz, const int32_t* rows,
                               const int64_t* lab_ptr, const int32_t* lab, const Ptrs& P,
-                              bool bf16_out) {
+                              bool bf16_out, const float2* stats, int ntiles, int64_t stats_ld) {
   launch_k(lc, k_softmax_ce, dim3(n), dim3(512), 0, n, L, ldz, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
-                                    P.rowloss);
+                                    P.rowloss, stats, ntiles, stats_ld);
   return cudaGetLastError();
 }
 

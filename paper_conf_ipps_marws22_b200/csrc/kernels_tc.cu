@@ -20,7 +20,8 @@
 namespace asgd {
 namespace {
 
-constexpr int BM = 128, BK = 64, STAGES = 4;
+constexpr int BM = 128, BK = 64;
+
 enum { TC_EPI_Z = 0, TC_EPI_PART = 1, TC_EPI_SGD = 2 };
 
 struct TcArgs {
@@ -31,6 +32,9 @@ struct TcArgs {
   const float* bias;                  // G1
   float lr; bf16* shadow; float* grad;// G3
   float* b2; float* grad_b2;          // G3: db2 = dZ^T 1 via an extra N = 16 MMA on N-tile 0
+  float2* stats; int64_t stats_ld;    // G1: per (N-tile half, row) softmax partials (max, sum exp)
+  int splits;                         // split-K factor (tiles = M tiles x N tiles x splits)
+  int n_fast;                         // tile order: N tiles vary fastest (else M tiles)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -126,36 +130,76 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float (&v)[32]) {
   for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
 }
 
+__device__ __forceinline__ float ex2_approx(float x) {   // 2^x on the MUFU (ex2.approx, -inf -> 0)
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+constexpr uint32_t pow2ceil(uint32_t x) {
+  uint32_t p = 32;
+  while (p < x) p <<= 1;
+  return p;
+}
+
+// Persistent tcgen05 GEMM.  CTA = 12 warps: warp 0 TMA producer, warp 1 MMA
+// issuer, warp 2 TMEM allocator, warps 4-11 epilogue (warp w drains TMEM lanes
+// 32 (w % 4) .. + 31, column half (w - 4) / 4).  Tiles (M fastest, or N fastest
+// when g.n_fast) are strided over the grid; the smem ring (full/empty mbarriers)
+// and the TMEM accumulators (tfull/tempty, double-buffered when 2 fit in 512
+// columns) carry across tiles, so a tile's epilogue overlaps the next tile's
+// loads and MMAs.
+template <int EPI>
+constexpr int stages_of() { return EPI == 2 ? 4 : (EPI == 0 ? 2 : 3); }
+template <int EPI>
+constexpr uint32_t staging_bytes() { return EPI == 2 ? 0u : 8u * 2u * 4096u; }   // 2 x 4 KB per epilogue warp
+
 template <int BN, bool A_MN, bool B_MN, int EPI>
-__global__ void __launch_bounds__(256, 1)
-    k_gemm_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, TcArgs g) {
+__global__ void __launch_bounds__(384, 1)
+    k_gemm_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+              const __grid_constant__ CUtensorMap tmC, TcArgs g) {
+  constexpr int STAGES = stages_of<EPI>();
   constexpr uint32_t A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE = A_BYTES + B_BYTES;
-  constexpr bool ONES = (EPI == TC_EPI_SGD);           // db2 column
-  constexpr uint32_t TMEM_COLS = ONES ? 2 * BN : BN;   // power of two >= BN (+16)
+  constexpr bool ONES = (EPI == TC_EPI_SGD);           // db2 column block after the accumulator
+  constexpr int ACC_COLS = BN + (ONES ? 32 : 0);
+  constexpr int NACC = (2 * ACC_COLS <= 512) ? 2 : 1;
+  constexpr uint32_t TMEM_COLS = pow2ceil(NACC * ACC_COLS);
   constexpr uint32_t ONES_BYTES = ONES ? 16 * 128 : 0; // K-major 16 x 64 bf16 tile, row 0 = 1
+  constexpr int EPI_WARPS = 8;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * A_BYTES;
   uint8_t* sOnes = smem + STAGES * STAGE;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * STAGE + ONES_BYTES);
+  uint8_t* sStg = smem + STAGES * STAGE + ONES_BYTES;   // TMA-store staging (1024-aligned)
+  uint64_t* full = reinterpret_cast<uint64_t*>(sStg + staging_bytes<EPI>());
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
-  uint32_t* tbase = reinterpret_cast<uint32_t*>(tfull + 1);
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tbase = reinterpret_cast<uint32_t*>(tempty + 2);
 
   pdl_trigger();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int n0 = blockIdx.x * BN, m0 = blockIdx.y * BM;
+  const int MT = (g.M + BM - 1) / BM, NT = (g.N + BN - 1) / BN, Z = g.splits;
+  const int T = MT * NT * Z;
   const int nkb = (g.K + BK - 1) / BK;
-  const int per = (nkb + gridDim.z - 1) / gridDim.z;
-  const int kb0 = blockIdx.z * per;
-  const int nk = max(0, min(nkb, kb0 + per) - kb0);
+  const int per = (nkb + Z - 1) / Z;
+  auto decode = [&](int t, int& mt, int& nt, int& z, int& kb0, int& nk) {
+    if (g.n_fast) { nt = t % NT; mt = (t / NT) % MT; } else { mt = t % MT; nt = (t / MT) % NT; }
+    z = t / (MT * NT);
+    kb0 = z * per;
+    nk = max(0, min(nkb, kb0 + per) - kb0);
+  };
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
     for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-    mbar_init(tfull, 1);
+    for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], EPI_WARPS); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
@@ -180,25 +224,31 @@ __global__ void __launch_bounds__(256, 1)
   if (warp == 0) {
     if (lane == 0) {
       // ------------------------------------------------ TMA producer
-      for (int i = 0; i < nk; ++i) {
-        const int s = i % STAGES;
-        const uint32_t ph = (i / STAGES) & 1;
-        mbar_wait(&empty[s], ph ^ 1);
-        mbar_expect_tx(&full[s], STAGE);
-        const int kc = (kb0 + i) * BK;
-        uint8_t* a = sA + s * A_BYTES;
-        uint8_t* b = sB + s * B_BYTES;
-        if constexpr (!A_MN) {
-          tma_load_2d(a, &tmA, &full[s], kc, m0);
-        } else {
-          tma_load_2d(a, &tmA, &full[s], m0, kc);
-          tma_load_2d(a + 8192, &tmA, &full[s], m0 + 64, kc);
-        }
-        if constexpr (!B_MN) {
-          tma_load_2d(b, &tmB, &full[s], kc, n0);
-        } else {
+      int it = 0;
+      for (int t = blockIdx.x; t < T; t += gridDim.x) {
+        int mt, nt, z, kb0, nk;
+        decode(t, mt, nt, z, kb0, nk);
+        const int m0 = mt * BM, n0 = nt * BN;
+        for (int i = 0; i < nk; ++i, ++it) {
+          const int s = it % STAGES;
+          const uint32_t ph = (it / STAGES) & 1;
+          mbar_wait(&empty[s], ph ^ 1);
+          mbar_expect_tx(&full[s], STAGE);
+          const int kc = (kb0 + i) * BK;
+          uint8_t* a = sA + s * A_BYTES;
+          uint8_t* b = sB + s * B_BYTES;
+          if constexpr (!A_MN) {
+            tma_load_2d(a, &tmA, &full[s], kc, m0);
+          } else {
+            tma_load_2d(a, &tmA, &full[s], m0, kc);
+            tma_load_2d(a + 8192, &tmA, &full[s], m0 + 64, kc);
+          }
+          if constexpr (!B_MN) {
+            tma_load_2d(b, &tmB, &full[s], kc, n0);
+          } else {
 #pragma unroll
-          for (int j = 0; j < BN / 64; ++j) tma_load_2d(b + j * 8192, &tmB, &full[s], n0 + 64 * j, kc);
+            for (int j = 0; j < BN / 64; ++j) tma_load_2d(b + j * 8192, &tmB, &full[s], n0 + 64 * j, kc);
+          }
         }
       }
     }
@@ -207,118 +257,164 @@ __global__ void __launch_bounds__(256, 1)
       // ------------------------------------------------ MMA issuer
       constexpr uint32_t idesc = make_idesc(BN, A_MN, B_MN);
       constexpr uint32_t idesc1 = make_idesc(16, A_MN, false);
-      const bool ones = ONES && blockIdx.x == 0;
       const uint32_t ones_base = smem_u32(sOnes);
-      for (int i = 0; i < nk; ++i) {
-        const int s = i % STAGES;
-        const uint32_t ph = (i / STAGES) & 1;
-        mbar_wait(&full[s], ph);
+      int it = 0, tl = 0;
+      for (int t = blockIdx.x; t < T; t += gridDim.x, ++tl) {
+        int mt, nt, z, kb0, nk;
+        decode(t, mt, nt, z, kb0, nk);
+        const int acc = tl % NACC;
+        const uint32_t aph = (tl / NACC) & 1;
+        mbar_wait(&tempty[acc], aph ^ 1);     // epilogue drained this accumulator
         tc_fence_after();
-        const uint32_t a_base = smem_u32(sA + s * A_BYTES), b_base = smem_u32(sB + s * B_BYTES);
+        const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS);
+        const bool ones = ONES && nt == 0;
+        for (int i = 0; i < nk; ++i, ++it) {
+          const int s = it % STAGES;
+          const uint32_t ph = (it / STAGES) & 1;
+          mbar_wait(&full[s], ph);
+          tc_fence_after();
+          const uint32_t a_base = smem_u32(sA + s * A_BYTES), b_base = smem_u32(sB + s * B_BYTES);
 #pragma unroll
-        for (int k = 0; k < BK / 16; ++k) {
-          // K-major: advance 16 elements (32 B) inside the 128B swizzle atom.
-          // MN-major: advance 16 K-rows (2 atoms of 8 rows x 128 B = 2048 B).
-          const uint64_t ad = A_MN ? desc_sw128(a_base + k * 2048, 8192, 1024) : desc_sw128(a_base + k * 32, 16, 1024);
-          const uint64_t bd = B_MN ? desc_sw128(b_base + k * 2048, 8192, 1024) : desc_sw128(b_base + k * 32, 16, 1024);
-          mma_bf16(tmem, ad, bd, idesc, (i > 0 || k > 0) ? 1u : 0u);
-          if (ONES && ones)   // TMEM column BN += dZ^T tile . e_0  (db2)
-            mma_bf16(tmem + BN, ad, desc_sw128(ones_base + k * 32, 16, 1024), idesc1, (i > 0 || k > 0) ? 1u : 0u);
+          for (int k = 0; k < BK / 16; ++k) {
+            // K-major: advance 16 elements (32 B) inside the 128B swizzle atom.
+            // MN-major: advance 16 K-rows (2 atoms of 8 rows x 128 B = 2048 B).
+            const uint64_t ad = A_MN ? desc_sw128(a_base + k * 2048, 8192, 1024) : desc_sw128(a_base + k * 32, 16, 1024);
+            const uint64_t bd = B_MN ? desc_sw128(b_base + k * 2048, 8192, 1024) : desc_sw128(b_base + k * 32, 16, 1024);
+            mma_bf16(d, ad, bd, idesc, (i > 0 || k > 0) ? 1u : 0u);
+            if (ONES && ones)   // TMEM column BN += dZ^T tile . e_0  (db2)
+              mma_bf16(d + BN, ad, desc_sw128(ones_base + k * 32, 16, 1024), idesc1, (i > 0 || k > 0) ? 1u : 0u);
+          }
+          mma_commit(&empty[s]);   // frees the smem stage once these MMAs retire
         }
-        mma_commit(&empty[s]);   // frees the smem stage once these MMAs retire
+        mma_commit(&tfull[acc]);   // accumulator ready (immediately if nk == 0)
       }
-      if (nk > 0) mma_commit(tfull);
     }
   } else if (warp >= 4) {
-    // ------------------------------------------------ epilogue: TMEM -> registers -> global
-    const int wq = warp - 4;
-    const int m = m0 + wq * 32 + lane;
-    // G3: the W2 row chunk this thread updates is loaded before the MMAs finish,
-    // and chunk c + 32 while chunk c is processed.
-    float4 wcur[8], wnxt[8];
-    const bool wrow_ok = (EPI == TC_EPI_SGD) && m < g.M;
-    if constexpr (EPI == TC_EPI_SGD) {
-      if (wrow_ok) {
-        const float4* w4 = reinterpret_cast<const float4*>(g.out + (int64_t)m * g.ldo + n0);
-#pragma unroll
-        for (int j = 0; j < 8; ++j) wcur[j] = w4[j];
-      }
-    }
-    if (nk > 0) {
-      mbar_wait(tfull, 0);
+    // ------------------------------------------------ epilogue (8 warps)
+    const int wq = (warp - 4) & 3, wh = (warp - 4) >> 2;
+    int tl = 0, sbuf = 0;
+    for (int t = blockIdx.x; t < T; t += gridDim.x, ++tl) {
+      int mt, nt, z, kb0, nk;
+      decode(t, mt, nt, z, kb0, nk);
+      const int m0 = mt * BM, n0 = nt * BN;
+      const int acc = tl % NACC;
+      const uint32_t aph = (tl / NACC) & 1;
+      mbar_wait(&tfull[acc], aph);
       tc_fence_after();
-    }
+      const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS) + ((uint32_t)(wq * 32) << 16);
+      const int m = m0 + wq * 32 + lane;
+      float st_m = -INFINITY, st_s = 0.f;   // G1 softmax partials of row m over this column half
 #pragma unroll 1
-    for (int c = 0; c < BN; c += 32) {
-      if constexpr (EPI == TC_EPI_SGD) {
-        if (wrow_ok && c + 32 < BN) {
-          const float4* w4 = reinterpret_cast<const float4*>(g.out + (int64_t)m * g.ldo + n0 + c + 32);
-#pragma unroll
-          for (int j = 0; j < 8; ++j) wnxt[j] = w4[j];
-        }
-      }
-      float v[32];
-      if (nk > 0) {
-        tmem_ld32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)c, v);
-      } else {
-#pragma unroll
-        for (int i = 0; i < 32; ++i) v[i] = 0.f;
-      }
-      const int n = n0 + c;
-      if (m >= g.M || n >= g.N) continue;
-      if constexpr (EPI == TC_EPI_Z) {
-        float* o = g.out + (int64_t)m * g.ldo + n;
-        if (n + 32 <= g.N) {
-#pragma unroll
-          for (int j = 0; j < 32; j += 4) {
-            const float4 bb = __ldg(reinterpret_cast<const float4*>(g.bias + n + j));
-            reinterpret_cast<float4*>(o)[j / 4] = make_float4(v[j] + bb.x, v[j + 1] + bb.y, v[j + 2] + bb.z, v[j + 3] + bb.w);
-          }
-        } else {
-          for (int j = 0; j < g.N - n; ++j) o[j] = v[j] + g.bias[n + j];
-        }
-      } else if constexpr (EPI == TC_EPI_PART) {
-        float* o = g.out + (int64_t)blockIdx.z * g.part_stride + (int64_t)m * g.ldo + n;
-#pragma unroll
-        for (int j = 0; j < 32; j += 4)
-          reinterpret_cast<float4*>(o)[j / 4] = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-      } else {  // TC_EPI_SGD: W2[m, n..n+31] -= lr * dW2
-        float* w = g.out + (int64_t)m * g.ldo + n;
-        bf16* sh = g.shadow + (int64_t)m * g.ldo + n;
-#pragma unroll
-        for (int j = 0; j < 32; j += 4) {
-          float4 x = wcur[j / 4];
-          x.x -= g.lr * v[j]; x.y -= g.lr * v[j + 1]; x.z -= g.lr * v[j + 2]; x.w -= g.lr * v[j + 3];
-          reinterpret_cast<float4*>(w)[j / 4] = x;
-          __nv_bfloat162 p0 = __floats2bfloat162_rn(x.x, x.y), p1 = __floats2bfloat162_rn(x.z, x.w);
-          uint2 pk;
-          pk.x = *reinterpret_cast<uint32_t*>(&p0);
-          pk.y = *reinterpret_cast<uint32_t*>(&p1);
-          reinterpret_cast<uint2*>(sh)[j / 4] = pk;
-        }
-        if (g.grad) {
-          float* gr = g.grad + (int64_t)m * g.ldo + n;
-#pragma unroll
-          for (int j = 0; j < 32; j += 4)
-            reinterpret_cast<float4*>(gr)[j / 4] = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-        }
-#pragma unroll
-        for (int j = 0; j < 8; ++j) wcur[j] = wnxt[j];
-      }
-    }
-    if constexpr (ONES) {
-      if (blockIdx.x == 0) {   // db2[m] = sum_n dZ[n, m]; b2 -= lr db2
+      for (int c = wh * (BN / 2); c < (wh + 1) * (BN / 2); c += 32) {
         float v[32];
         if (nk > 0) {
-          tmem_ld32(tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)BN, v);
+          tmem_ld32(d + (uint32_t)c, v);
         } else {
-          v[0] = 0.f;
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = 0.f;
         }
-        if (m < g.M) {
-          g.b2[m] -= g.lr * v[0];
-          if (g.grad_b2) g.grad_b2[m] = v[0];
+        const int n = n0 + c;
+        if (n >= g.N) continue;   // warp-uniform
+        if constexpr (EPI == TC_EPI_Z) {
+          const float bl = n + lane < g.N ? __ldg(g.bias + n + lane) : 0.f;
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            v[j] += __shfl_sync(0xffffffffu, bl, j);
+            if (n + j >= g.N) v[j] = -INFINITY;
+          }
+          if (g.stats) {   // online (max, sum exp) of row m over the columns seen so far
+            float cm = v[0];
+#pragma unroll
+            for (int j = 1; j < 32; ++j) cm = fmaxf(cm, v[j]);
+            constexpr float kL2E = 1.4426950408889634f;
+            if (cm > st_m) { st_s = (st_m == -INFINITY) ? 0.f : st_s * ex2_approx((st_m - cm) * kL2E); st_m = cm; }
+            const float ms = st_m * kL2E;
+            float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;   // 4 independent MUFU -> FADD chains
+#pragma unroll
+            for (int j = 0; j < 32; j += 4) {
+              a0 += ex2_approx(fmaf(v[j], kL2E, -ms));
+              a1 += ex2_approx(fmaf(v[j + 1], kL2E, -ms));
+              a2 += ex2_approx(fmaf(v[j + 2], kL2E, -ms));
+              a3 += ex2_approx(fmaf(v[j + 3], kL2E, -ms));
+            }
+            st_s += (a0 + a1) + (a2 + a3);
+          }
+        }
+        if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_PART) {
+          // stage the warp's 32 x 32 fp32 box (128B swizzle: conflict-free) and TMA-store it;
+          // rows >= M / columns >= N are clipped by the tensor map
+          uint8_t* buf = sStg + ((warp - 4) * 2 + sbuf) * 4096;
+          if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+          __syncwarp();
+#pragma unroll
+          for (int q = 0; q < 8; ++q)
+            *reinterpret_cast<float4*>(buf + lane * 128 + ((q ^ (lane & 7)) * 16)) =
+                make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          __syncwarp();
+          if (lane == 0) {
+            if constexpr (EPI == TC_EPI_Z)
+              asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                               reinterpret_cast<uint64_t>(&tmC)),
+                           "r"(smem_u32(buf)), "r"(n), "r"(m0 + wq * 32)
+                           : "memory");
+            else
+              asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];" ::"l"(
+                               reinterpret_cast<uint64_t>(&tmC)),
+                           "r"(smem_u32(buf)), "r"(n), "r"(m0 + wq * 32), "r"(z)
+                           : "memory");
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+          }
+          sbuf ^= 1;
+        } else {  // TC_EPI_SGD: W2[m, n..n+31] -= lr * dW2, bf16 shadow, debug grad
+          if (m >= g.M) continue;   // rows past L would run into b2 (flat parameter layout)
+          float* w = g.out + (int64_t)m * g.ldo + n;
+          bf16* sh = g.shadow + (int64_t)m * g.ldo + n;
+          float4 x4[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) x4[j] = reinterpret_cast<const float4*>(w)[j];
+#pragma unroll
+          for (int j = 0; j < 32; j += 4) {
+            float4 x = x4[j / 4];
+            x.x -= g.lr * v[j]; x.y -= g.lr * v[j + 1]; x.z -= g.lr * v[j + 2]; x.w -= g.lr * v[j + 3];
+            reinterpret_cast<float4*>(w)[j / 4] = x;
+            __nv_bfloat162 p0 = __floats2bfloat162_rn(x.x, x.y), p1 = __floats2bfloat162_rn(x.z, x.w);
+            uint2 pk;
+            pk.x = *reinterpret_cast<uint32_t*>(&p0);
+            pk.y = *reinterpret_cast<uint32_t*>(&p1);
+            reinterpret_cast<uint2*>(sh)[j / 4] = pk;
+          }
+          if (g.grad) {
+            float* gr = g.grad + (int64_t)m * g.ldo + n;
+#pragma unroll
+            for (int j = 0; j < 32; j += 4)
+              reinterpret_cast<float4*>(gr)[j / 4] = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+          }
         }
       }
+      if constexpr (EPI == TC_EPI_Z) {
+        if (g.stats && m < g.M) g.stats[(int64_t)(nt * 2 + wh) * g.stats_ld + m] = make_float2(st_m, st_s);
+      }
+      if constexpr (ONES) {
+        if (nt == 0 && wh == 0) {   // db2[m] = sum_n dZ[n, m]; b2 -= lr db2
+          float v[32];
+          if (nk > 0) {
+            tmem_ld32(d + (uint32_t)BN, v);
+          } else {
+            v[0] = 0.f;
+          }
+          if (m < g.M) {
+            g.b2[m] -= g.lr * v[0];
+            if (g.grad_b2) g.grad_b2[m] = v[0];
+          }
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[acc]);   // accumulator may be overwritten
+    }
+    if constexpr (EPI != TC_EPI_SGD) {
+      if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // stores complete
     }
   }
   tc_fence_before();
@@ -341,6 +437,22 @@ void init_encode() {
     g_encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
 }
 
+// fp32 store maps (128B swizzle, 32 x 32 boxes): Z [rows][ldz] and the split-K partials
+// [splits][b_max][H] (3D, so rows >= b_max of a slice never spill into the next slice).
+cudaError_t make_store_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer,
+                           uint64_t row_bytes, uint64_t depth, uint64_t slice_bytes, int rank) {
+  cuuint64_t dims[3] = {inner, outer, depth};
+  cuuint64_t strides[2] = {row_bytes, slice_bytes};
+  cuuint32_t box[3] = {32, 32, 1};
+  cuuint32_t es[3] = {1, 1, 1};
+  if (rank == 3 && slice_bytes == 0) slice_bytes = row_bytes * outer;
+  strides[1] = slice_bytes;
+  CUresult r = g_encode(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, rank, const_cast<void*>(base), dims,
+                        strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
 cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t row_bytes,
                      uint32_t box_inner, uint32_t box_outer) {
   cuuint64_t dims[2] = {inner, outer};
@@ -354,8 +466,10 @@ cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t 
 }
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
-cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, const TcArgs& g, int splits) {
-  const size_t smem = (size_t)STAGES * (BM * BK * 2 + BN * BK * 2) + (EPI == TC_EPI_SGD ? 2048 : 0) + 1024 + 256;
+cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c, TcArgs g,
+               int splits) {
+  const size_t smem = (size_t)stages_of<EPI>() * (BM * BK * 2 + BN * BK * 2) + (EPI == TC_EPI_SGD ? 2048 : 0) +
+                      staging_bytes<EPI>() + 1024 + 256;
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(k_gemm_tc<BN, A_MN, B_MN, EPI>,
@@ -363,8 +477,10 @@ cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, co
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  dim3 grid((g.N + BN - 1) / BN, (g.M + BM - 1) / BM, splits);
-  return launch_k(lc, k_gemm_tc<BN, A_MN, B_MN, EPI>, grid, dim3(256), smem, a, b, g);
+  g.splits = splits;
+  const int64_t tiles = (int64_t)((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN) * splits;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, lc.sms));
+  return launch_k(lc, k_gemm_tc<BN, A_MN, B_MN, EPI>, dim3(grid), dim3(384), smem, a, b, c, g);
 }
 
 // Widest N tile that still gives >= one CTA per SM (and does not overhang N by 2x).
@@ -384,21 +500,25 @@ bool tc_available() {
 int64_t padded_ld(int64_t L) { return (L + 7) / 8 * 8; }
 
 cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H, float lr, const Ptrs& P,
-                           const WsLayout& W, float* W2, float* b2, float* grad_w2, float* grad_b2) {
+                           const WsLayout& W, float* W2, float* b2, float* grad_w2, float* grad_b2,
+                           float2* stats, int* stats_ntiles) {
   if (!tc_available()) return cudaErrorNotSupported;
   const int64_t Lp = padded_ld(L);
-  CUtensorMap ta, tb;
+  CUtensorMap ta, tb, tc;
   TcArgs g{};
   cudaError_t e;
   if (which == 1) {  // Z = H1 W2^T + b2
     g.M = n; g.N = (int)L; g.K = H;
     g.out = P.z; g.ldo = Lp; g.bias = b2;
     const int bn = pick_bn((n + BM - 1) / BM, L, lc.sms);
+    g.stats = stats; g.stats_ld = W.stats_ld;
+    if (stats_ntiles) *stats_ntiles = (int)(2 * ((L + bn - 1) / bn));   // two column halves per tile
     if ((e = make_map(&ta, P.h1b, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
     if ((e = make_map(&tb, P.w2b, H, L, (uint64_t)H * 2, 64, bn)) != cudaSuccess) return e;
-    if (bn == 256) return run<256, false, false, TC_EPI_Z>(lc, ta, tb, g, 1);
-    if (bn == 128) return run<128, false, false, TC_EPI_Z>(lc, ta, tb, g, 1);
-    return run<64, false, false, TC_EPI_Z>(lc, ta, tb, g, 1);
+    if ((e = make_store_map(&tc, P.z, L, n, (uint64_t)Lp * 4, 1, 0, 2)) != cudaSuccess) return e;
+    if (bn == 256) return run<256, false, false, TC_EPI_Z>(lc, ta, tb, tc, g, 1);
+    if (bn == 128) return run<128, false, false, TC_EPI_Z>(lc, ta, tb, tc, g, 1);
+    return run<64, false, false, TC_EPI_Z>(lc, ta, tb, tc, g, 1);
   }
   if (which == 2) {  // dH1 partials = dZ W2
     g.M = n; g.N = H; g.K = (int)L;
@@ -409,9 +529,12 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
     if ((e = make_map(&tb, P.w2b, H, L, (uint64_t)H * 2, 64, 64)) != cudaSuccess) return e;
     // partial slices beyond `splits` stay untouched; dh_reduce sums W.splitk slices
     if (splits != W.splitk) return cudaErrorInvalidValue;
-    if (H >= 256) return run<256, false, true, TC_EPI_PART>(lc, ta, tb, g, splits);
-    if (H == 128) return run<128, false, true, TC_EPI_PART>(lc, ta, tb, g, splits);
-    return run<64, false, true, TC_EPI_PART>(lc, ta, tb, g, splits);
+    const int64_t bmax = W.part_stride / H;
+    if ((e = make_store_map(&tc, P.dhpart, H, bmax, (uint64_t)H * 4, splits,
+                            (uint64_t)W.part_stride * 4, 3)) != cudaSuccess) return e;
+    if (H >= 256) return run<256, false, true, TC_EPI_PART>(lc, ta, tb, tc, g, splits);
+    if (H == 128) return run<128, false, true, TC_EPI_PART>(lc, ta, tb, tc, g, splits);
+    return run<64, false, true, TC_EPI_PART>(lc, ta, tb, tc, g, splits);
   }
   // which == 3: W2 -= lr dZ^T H1
   g.M = (int)L; g.N = H; g.K = n;
@@ -419,12 +542,16 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
   g.b2 = b2; g.grad_b2 = grad_b2;
   if ((e = make_map(&ta, P.dzb, L, n, (uint64_t)Lp * 2, 64, 64)) != cudaSuccess) return e;
   if ((e = make_map(&tb, P.h1b, H, n, (uint64_t)H * 2, 64, 64)) != cudaSuccess) return e;
+  // N tiles of one M tile run back to back (n_fast), so the dZ^T tile is read
+  // once from HBM; BN <= 128 keeps two accumulators (+ db2 column) in TMEM.
   const int64_t tiles_m = (L + BM - 1) / BM;
-  int bn = H >= 256 ? 256 : H;
+  int bn = std::min(H, 128);
   while (bn > 64 && tiles_m * (H / bn) < lc.sms) bn /= 2;
-  if (bn == 256) return run<256, true, true, TC_EPI_SGD>(lc, ta, tb, g, 1);
-  if (bn == 128) return run<128, true, true, TC_EPI_SGD>(lc, ta, tb, g, 1);
-  return run<64, true, true, TC_EPI_SGD>(lc, ta, tb, g, 1);
+  g.n_fast = 1;
+  tc = ta;   // unused by the SGD epilogue
+  if (bn == 256) return run<256, true, true, TC_EPI_SGD>(lc, ta, tb, tc, g, 1);
+  if (bn == 128) return run<128, true, true, TC_EPI_SGD>(lc, ta, tb, tc, g, 1);
+  return run<64, true, true, TC_EPI_SGD>(lc, ta, tb, tc, g, 1);
 }
 
 }  // namespace asgd

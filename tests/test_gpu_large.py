@@ -1,0 +1,66 @@
+"""Parity at the big BASELINE.json shapes, in the launch configuration bench.py
+times (full F, L, H and b_max; the dataset is a generated prefix of the
+split).  The oracle's batch-mean gradient is evaluated in row chunks:
+grad(B rows) = sum_chunks (|chunk| / B) grad(chunk), which is the definition
+of the mean and keeps the fp64 working set bounded."""
+import numpy as np
+import pytest
+import torch
+
+from oracle import model as omodel
+from synth import config, init_params, sample_stream
+from tests.gpu_helpers import dataset, make_replica, normwise, split_grad
+
+pytestmark = pytest.mark.gpu
+
+TOL = {"fp32": 1e-4, "bf16": 2e-2}
+
+
+def _chunked_oracle(w, batch, F, H, L, chunk):
+    B = batch.n_rows
+    loss, g = 0.0, None
+    for r0 in range(0, B, chunk):
+        sub = batch.row_slice(np.arange(r0, min(B, r0 + chunk)))
+        lo, go = omodel.loss_and_grad(w, sub, F, H, L)
+        f = sub.n_rows / B
+        loss += f * lo
+        g = f * go if g is None else g + f * go
+    return loss, g
+
+
+def _check_big(name, n_rows, precision, chunk, seed_pos=0):
+    cfg = config(name)
+    data = dataset(name, n_rows)
+    cfg_sub = config(name, n_train=data.n_rows)
+    rows = sample_stream(cfg_sub, seed_pos, cfg.b_max)
+    w0 = init_params(cfg)
+    rep = make_replica(cfg, data, precision, w0=w0)
+    g = torch.zeros(rep.P, dtype=torch.float32, device="cuda")
+    loss = torch.zeros(1, dtype=torch.float32, device="cuda")
+    rep.set_debug_grads(g)
+    rep.step(torch.as_tensor(rows, device="cuda"), 0.5, loss)
+    rep.sync()
+    touched = rep.last_touched().cpu().numpy()
+    batch = data.row_slice(rows)
+    lo, go = _chunked_oracle(w0.astype(np.float64), batch, cfg.F, cfg.H, cfg.L, chunk)
+    tol = TOL[precision]
+    assert abs(loss.item() - lo) <= tol * abs(lo)
+    np.testing.assert_array_equal(touched, omodel.touched_features(batch))
+    gg, og = split_grad(g.cpu().numpy(), cfg.F, cfg.H, cfg.L), split_grad(go, cfg.F, cfg.H, cfg.L)
+    for k in ("W1", "b1", "W2", "b2"):
+        e = normwise(gg[k], og[k])
+        assert e <= tol, (name, precision, k, e)
+
+
+@pytest.mark.parametrize("precision", ["bf16", "fp32"])
+def test_amazoncat_bench_launch(precision):
+    _check_big("amazoncat13k", 32768, precision, chunk=1024)
+
+
+def test_amazon670k_bench_launch():
+    """L = 670,091: G1 stores 2.7 GB of logits, G2 splits K over 37 slices."""
+    _check_big("amazon670k", 16384, "bf16", chunk=128)
+
+
+def test_wiki10_full_split_bench_launch():
+    _check_big("wiki10_31k", None, "bf16", chunk=256)
