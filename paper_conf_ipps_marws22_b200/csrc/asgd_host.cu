@@ -53,6 +53,9 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) ==
 size_t up256(size_t x) { return (x + 255) & ~size_t(255); }
 
 constexpr int kSqnormParts = 1024;
+// Above this many bytes of fp32 logits per step the bf16 path fuses softmax-CE
+// into the GEMMs (Z never written); below, Z stays L2-resident and is stored.
+constexpr int64_t kFusedCeBytes = 64ll << 20;
 
 int splitk_for(const asgd_model_desc& d) {
   // G2 (dH1 = dZ W2, M = b_max, N = H, K = L): split K so ~2 waves of CTAs run.
@@ -111,6 +114,7 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.rbase = take((size_t)(B + 1) * 8);
   L.da1b = take(bf ? (size_t)B * H * 2 : 0);
   L.stats_ld = B;
+  L.lse = take(B * 4);
   L.zstat = take(bf ? (size_t)((Lb + 31) / 32 + 2) * B * 8 : 0);   // G1 softmax partials (2 per N tile)
   L.rowloss = take(B * 4);
   L.dhpart = take((size_t)L.splitk * B * H * 4);
@@ -140,6 +144,7 @@ Ptrs ws_ptrs(char* b, const WsLayout& L) {
   p.b2part = (float*)(b + L.b2part);
   p.rbase = (int64_t*)(b + L.rbase);
   p.da1b = (bf16*)(b + L.da1b);
+  p.lse = (float*)(b + L.lse);
   return p;
 }
 
@@ -421,9 +426,23 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     Launch lc3 = c->lc3();
     float2* zstat = reinterpret_cast<float2*>(c->ws + c->L.zstat);
     int ntiles = 0;
-    PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
-    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, true, zstat, ntiles,
-                                          c->L.stats_ld));
+    if ((int64_t)m.b_max * Lb * 4 <= kFusedCeBytes) {
+      // logits fit in L2: G1 stores Z (+ per-tile softmax partials), one pass of softmax-CE
+      PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
+      PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, true, zstat, ntiles,
+                                            c->L.stats_ld));
+    } else {
+      // fused softmax-CE: G1 keeps only per-tile (max, sum exp); k_lse -> lse, row loss;
+      // G1b recomputes Z tile by tile and writes dZ = (softmax - T)/B (bf16) -- Z never hits HBM
+      PCU(ASGD_K_G1, launch_gemm_tc(lc, 5, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
+    PCU(ASGD_K_SOFTMAX, ([&]() -> cudaError_t {
+          cudaError_t e = launch_lse(lc, n, H, ntiles, c->L.stats_ld, zstat, rows, x.lab_ptr, x.lab, P.h1b,
+                                     Pr.w2b, b2, P);
+          return e != cudaSuccess ? e
+                                  : launch_gemm_tc(lc, 4, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr,
+                                                   nullptr, nullptr, rows, x.lab_ptr, x.lab);
+        })());
+    }
     CU(cudaEventRecord(c->ev_sm, c->s));
     CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
     PCU_ON(c->s3, ASGD_K_G3, launch_gemm_tc(lc3, 3, n, Lb, H, lr, Pw, c->L, W2, b2, g ? g + c->o_w2 : nullptr,

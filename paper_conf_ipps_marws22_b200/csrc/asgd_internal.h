@@ -25,7 +25,7 @@ typedef __nv_bfloat16 bf16;
 struct WsLayout {
   size_t meta, boff, loff, cnt, fseg, fuid, uniq, useg, tsum, tpre;
   size_t e_n, e_v, e_u, e_f, part1, rowcnt, part5, ucnt, bits;
-  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, b2part, rbase, da1b, zstat;
+  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, b2part, rbase, da1b, zstat, lse;
   size_t total;
   int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride, stats_ld;
 };
@@ -40,6 +40,7 @@ struct Ptrs {  // typed views of the workspace
   float* da1; float* db1part; bf16* w2b; double* red; int32_t* eval_top; float* b2part;
   int64_t* rbase;   // row_ptr[rows[r]] of the current batch (written by K-0 (a))
   bf16* da1b;       // bf16 copy of dA1 (bf16 path; staged by K-5)
+  float* lse;       // per-row log-sum-exp of Z (bf16 path)
 };
 int row_block();   // rows per db1 partial (kernels_dense.cu)
 int b2_chunks();   // row chunks of the db2 partial sums
@@ -129,7 +130,14 @@ bool tc_available();
 // stats (G1 only, nullable): per (N tile, row) softmax partials; *stats_ntiles = N tiles.
 cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int H, float lr,
                            const Ptrs&, const WsLayout&, float* W2, float* b2, float* grad_w2,
-                           float* grad_b2, float2* stats = nullptr, int* stats_ntiles = nullptr);
+                           float* grad_b2, float2* stats = nullptr, int* stats_ntiles = nullptr,
+                           const int32_t* dz_rows = nullptr, const int64_t* dz_lab_ptr = nullptr,
+                           const int32_t* dz_lab = nullptr);
+// which = 4 (G1b): dZ = (softmax - T)/B from a recomputed Z tile; needs P.lse from k_lse.
+// which = 5: G1 without storing Z (only the softmax partials), for the fused path.
+cudaError_t launch_lse(const Launch&, int n, int H, int ntiles, int64_t stats_ld, const float2* stats,
+                       const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab, const bf16* h1b,
+                       const bf16* w2b, const float* b2, const Ptrs&);
 // ---------------------------------------------------------------- merge / eval
 cudaError_t launch_sqnorm(const Launch&, const float* x, int64_t P, double* partials, int nparts,
                           double* out);

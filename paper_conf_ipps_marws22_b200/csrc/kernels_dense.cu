@@ -204,6 +204,64 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
   }
 }
 
+// ------------------------------------------------------------ fused CE: lse
+// lse_n from G1's per-tile (max, sum exp) partials; the label logits
+// Z_ny = H1_n . W2_y + b2_y (bf16 operands, fp32 sum, as on the tensor cores);
+// row loss = lse_n - mean_y Z_ny (Q3, Q4).  One CTA per row.
+__global__ void __launch_bounds__(256) k_lse(int H, int ntiles, int64_t stats_ld, const float2* __restrict__ stats,
+                                             const int32_t* __restrict__ rows, const int64_t* __restrict__ lab_ptr,
+                                             const int32_t* __restrict__ lab, const bf16* __restrict__ h1b,
+                                             const bf16* __restrict__ w2b, const float* __restrict__ b2,
+                                             float* lse, float* rowloss) {
+  pdl_trigger();
+  pdl_wait();
+  __shared__ float s_m[8], s_s[8], s_z[8];
+  const int n = blockIdx.x, lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  float m = -INFINITY, s = 0.f;
+  for (int t = threadIdx.x; t < ntiles; t += blockDim.x) {
+    const float2 p = stats[(int64_t)t * stats_ld + n];
+    if (p.x == -INFINITY) continue;
+    if (p.x > m) { s = (m == -INFINITY ? 0.f : s * __expf(m - p.x)) + p.y; m = p.x; }
+    else s += p.y * __expf(p.x - m);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const float om = __shfl_xor_sync(kFull, m, o), os = __shfl_xor_sync(kFull, s, o);
+    const float nm = fmaxf(m, om);
+    s = (m == -INFINITY ? 0.f : s * __expf(m - nm)) + (om == -INFINITY ? 0.f : os * __expf(om - nm));
+    m = nm;
+  }
+  // label logits: warp w takes labels w, w + 8, ...
+  const int64_t id = rows[n];
+  const int64_t l0 = lab_ptr[id], l1 = lab_ptr[id + 1];
+  float zs = 0.f;
+  for (int64_t i = l0 + wid; i < l1; i += 8) {
+    const int y = lab[i];
+    float d = 0.f;
+    for (int k = lane * 2; k < H; k += 64) {
+      const float2 a = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(h1b + (int64_t)n * H + k));
+      const float2 b = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(w2b + (int64_t)y * H + k));
+      d = fmaf(a.x, b.x, fmaf(a.y, b.y, d));
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) d += __shfl_xor_sync(kFull, d, o);
+    zs += d + b2[y];
+  }
+  if (lane == 0) { s_m[wid] = m; s_s[wid] = s; s_z[wid] = zs; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float M = -INFINITY, S = 0.f, Zs = 0.f;
+    for (int w = 0; w < 8; ++w) M = fmaxf(M, s_m[w]);
+    for (int w = 0; w < 8; ++w) {
+      S += (s_m[w] == -INFINITY) ? 0.f : s_s[w] * __expf(s_m[w] - M);
+      Zs += s_z[w];
+    }
+    const float l = M + logf(S);
+    lse[n] = l;
+    rowloss[n] = l - Zs / (float)(l1 - l0);
+  }
+}
+
 // ------------------------------------------------------ dH1 reduce + ReLU'
 // dA1[r][c] = [H1[r][c] > 0] * sum_z part[z][r][c]: one thread per element, its
 // split-K loads all in flight; fixed summation order (deterministic).
@@ -325,6 +383,13 @@ cudaError_t launch_softmax_ce(const Launch& lc, int n, int64_t L, int64_t ldz, c
   launch_k(lc, k_softmax_ce, dim3(n), dim3(512), 0, n, L, ldz, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
                                     P.rowloss, stats, ntiles, stats_ld);
   return cudaGetLastError();
+}
+
+cudaError_t launch_lse(const Launch& lc, int n, int H, int ntiles, int64_t stats_ld, const float2* stats,
+                       const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab, const bf16* h1b,
+                       const bf16* w2b, const float* b2, const Ptrs& P) {
+  return launch_k(lc, k_lse, dim3(n), dim3(256), 0, H, ntiles, stats_ld, stats, rows, lab_ptr, lab, h1b, w2b, b2,
+                  P.lse, P.rowloss);
 }
 
 cudaError_t launch_dh_reduce(const Launch& lc, int n, int H, int splitk, const Ptrs& P,

@@ -22,7 +22,7 @@ namespace {
 
 constexpr int BM = 128, BK = 64;
 
-enum { TC_EPI_Z = 0, TC_EPI_PART = 1, TC_EPI_SGD = 2 };
+enum { TC_EPI_Z = 0, TC_EPI_PART = 1, TC_EPI_SGD = 2, TC_EPI_DZ = 3 };
 
 struct TcArgs {
   int M, N, K;
@@ -35,6 +35,9 @@ struct TcArgs {
   float2* stats; int64_t stats_ld;    // G1: per (N-tile half, row) softmax partials (max, sum exp)
   int splits;                         // split-K factor (tiles = M tiles x N tiles x splits)
   int n_fast;                         // tile order: N tiles vary fastest (else M tiles)
+  int write_z;                        // G1: store Z (eval) or only the softmax partials (step)
+  // G1b (TC_EPI_DZ): dZ = (exp(Z - lse) - T) / B recomputed from the MMA, stored bf16
+  const float* lse; const int32_t* rows; const int64_t* lab_ptr; const int32_t* lab; float invB;
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -154,14 +157,16 @@ constexpr uint32_t pow2ceil(uint32_t x) {
 // columns) carry across tiles, so a tile's epilogue overlaps the next tile's
 // loads and MMAs.
 template <int EPI>
-constexpr int stages_of() { return EPI == 2 ? 4 : (EPI == 0 ? 2 : 3); }
+constexpr int stages_of() { return EPI == 2 ? 3 : ((EPI == 0 || EPI == 3) ? 2 : 3); }
 template <int EPI>
-constexpr uint32_t staging_bytes() { return EPI == 2 ? 0u : 8u * 2u * 4096u; }   // 2 x 4 KB per epilogue warp
+constexpr uint32_t staging_bytes() {   // per epilogue warp: 2 x 4 KB fp32 boxes (+ 2 x 2 KB bf16 for G3)
+  return EPI == 2 ? 8u * 12288u : 8u * 2u * 4096u;
+}
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
 __global__ void __launch_bounds__(384, 1)
     k_gemm_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-              const __grid_constant__ CUtensorMap tmC, TcArgs g) {
+              const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmD, TcArgs g) {
   constexpr int STAGES = stages_of<EPI>();
   constexpr uint32_t A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE = A_BYTES + B_BYTES;
   constexpr bool ONES = (EPI == TC_EPI_SGD);           // db2 column block after the accumulator
@@ -180,7 +185,8 @@ __global__ void __launch_bounds__(384, 1)
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
   uint64_t* tempty = tfull + 2;
-  uint32_t* tbase = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* wbar = tempty + 2;   // G3: per epilogue warp, 2 W2-box load barriers
+  uint32_t* tbase = reinterpret_cast<uint32_t*>(wbar + 16);
 
   pdl_trigger();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -200,6 +206,8 @@ __global__ void __launch_bounds__(384, 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
     for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
     for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], EPI_WARPS); }
+    if constexpr (EPI == TC_EPI_SGD)
+      for (int a = 0; a < 16; ++a) mbar_init(&wbar[a], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
@@ -292,7 +300,7 @@ __global__ void __launch_bounds__(384, 1)
   } else if (warp >= 4) {
     // ------------------------------------------------ epilogue (8 warps)
     const int wq = (warp - 4) & 3, wh = (warp - 4) >> 2;
-    int tl = 0, sbuf = 0;
+    int tl = 0, sbuf = 0, kc = 0;
     for (int t = blockIdx.x; t < T; t += gridDim.x, ++tl) {
       int mt, nt, z, kb0, nk;
       decode(t, mt, nt, z, kb0, nk);
@@ -304,6 +312,20 @@ __global__ void __launch_bounds__(384, 1)
       const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS) + ((uint32_t)(wq * 32) << 16);
       const int m = m0 + wq * 32 + lane;
       float st_m = -INFINITY, st_s = 0.f;   // G1 softmax partials of row m over this column half
+      float lse_m = 0.f, tinv = 0.f;        // G1b: row m's lse and 1 / (|Y_m| B)
+      int64_t lab_cur = 0, lab_end = 0;
+      if constexpr (EPI == TC_EPI_DZ) {
+        if (m < g.M) {
+          lse_m = g.lse[m];
+          const int64_t id = g.rows[m];
+          lab_cur = g.lab_ptr[id];
+          lab_end = g.lab_ptr[id + 1];
+          tinv = g.invB / (float)(lab_end - lab_cur);
+          // skip labels left of this warp's first column
+          const int cfirst = n0 + wh * (BN / 2);
+          while (lab_cur < lab_end && g.lab[lab_cur] < cfirst) ++lab_cur;
+        }
+      }
 #pragma unroll 1
       for (int c = wh * (BN / 2); c < (wh + 1) * (BN / 2); c += 32) {
         float v[32];
@@ -315,13 +337,57 @@ __global__ void __launch_bounds__(384, 1)
         }
         const int n = n0 + c;
         if (n >= g.N) continue;   // warp-uniform
-        if constexpr (EPI == TC_EPI_Z) {
+        if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_DZ) {
           const float bl = n + lane < g.N ? __ldg(g.bias + n + lane) : 0.f;
 #pragma unroll
           for (int j = 0; j < 32; ++j) {
             v[j] += __shfl_sync(0xffffffffu, bl, j);
             if (n + j >= g.N) v[j] = -INFINITY;
           }
+        }
+        if constexpr (EPI == TC_EPI_DZ) {
+          // softmax - uniform target over the row's labels (Q3), / B (Q4); labels are sorted,
+          // lab_cur walks forward as this warp's columns increase
+          constexpr float kL2E = 1.4426950408889634f;
+          const float ls = lse_m * kL2E;
+#pragma unroll
+          for (int j = 0; j < 32; ++j) v[j] = ex2_approx(fmaf(v[j], kL2E, -ls)) * g.invB;
+          while (lab_cur < lab_end) {
+            const int y = g.lab[lab_cur];
+            if (y >= n + 32) break;
+            if (y >= n) {
+              const int jy = y - n;
+#pragma unroll
+              for (int j = 0; j < 32; ++j)
+                if (j == jy) v[j] -= tinv;
+            }
+            ++lab_cur;
+          }
+          // stage a 32 x 32 bf16 box (64B swizzle) and TMA-store it into dZ
+          uint8_t* buf = sStg + ((warp - 4) * 2 + sbuf) * 4096;
+          if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+          __syncwarp();
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            __nv_bfloat162 p0 = __floats2bfloat162_rn(v[4 * q], v[4 * q + 1]);
+            __nv_bfloat162 p1 = __floats2bfloat162_rn(v[4 * q + 2], v[4 * q + 3]);
+            uint2 pk;
+            pk.x = *reinterpret_cast<uint32_t*>(&p0);
+            pk.y = *reinterpret_cast<uint32_t*>(&p1);
+            *reinterpret_cast<uint2*>(buf + lane * 64 + ((((q >> 1) ^ ((lane >> 1) & 3))) * 16) + (q & 1) * 8) = pk;
+          }
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          __syncwarp();
+          if (lane == 0) {
+            asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                             reinterpret_cast<uint64_t>(&tmC)), "r"(smem_u32(buf)), "r"(n), "r"(m0 + wq * 32)
+                         : "memory");
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+          }
+          sbuf ^= 1;
+          continue;
+        }
+        if constexpr (EPI == TC_EPI_Z) {
           if (g.stats) {   // online (max, sum exp) of row m over the columns seen so far
             float cm = v[0];
 #pragma unroll
@@ -339,6 +405,9 @@ __global__ void __launch_bounds__(384, 1)
             }
             st_s += (a0 + a1) + (a2 + a3);
           }
+        }
+        if constexpr (EPI == TC_EPI_Z) {
+          if (!g.write_z) continue;   // step: only the softmax partials are needed
         }
         if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_PART) {
           // stage the warp's 32 x 32 fp32 box (128B swizzle: conflict-free) and TMA-store it;
@@ -366,29 +435,46 @@ __global__ void __launch_bounds__(384, 1)
             asm volatile("cp.async.bulk.commit_group;" ::: "memory");
           }
           sbuf ^= 1;
-        } else {  // TC_EPI_SGD: W2[m, n..n+31] -= lr * dW2, bf16 shadow, debug grad
-          if (m >= g.M) continue;   // rows past L would run into b2 (flat parameter layout)
-          float* w = g.out + (int64_t)m * g.ldo + n;
-          bf16* sh = g.shadow + (int64_t)m * g.ldo + n;
-          float4 x4[8];
+        } else {  // TC_EPI_SGD: W2 box += -lr dW2 through smem; TMA load, TMA stores (W2 fp32, bf16 shadow)
+          const int b = kc & 1;
+          const uint32_t ph = (kc >> 1) & 1;
+          ++kc;
+          uint8_t* wb = sStg + (warp - 4) * 12288 + b * 4096;          // 32 x 32 fp32, 128B swizzle
+          uint8_t* hb = sStg + (warp - 4) * 12288 + 8192 + b * 2048;   // 32 x 32 bf16, 64B swizzle
+          uint64_t* wl = &wbar[(warp - 4) * 2 + b];
+          const int row0 = m0 + wq * 32;
+          if (lane == 0) {
+            asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");   // buffer b read out
+            mbar_expect_tx(wl, 4096);
+            tma_load_2d(wb, &tmC, wl, n, row0);   // rows >= L are zero-filled
+          }
+          mbar_wait(wl, ph);
 #pragma unroll
-          for (int j = 0; j < 8; ++j) x4[j] = reinterpret_cast<const float4*>(w)[j];
-#pragma unroll
-          for (int j = 0; j < 32; j += 4) {
-            float4 x = x4[j / 4];
-            x.x -= g.lr * v[j]; x.y -= g.lr * v[j + 1]; x.z -= g.lr * v[j + 2]; x.w -= g.lr * v[j + 3];
-            reinterpret_cast<float4*>(w)[j / 4] = x;
+          for (int q = 0; q < 8; ++q) {
+            float4* p = reinterpret_cast<float4*>(wb + lane * 128 + ((q ^ (lane & 7)) * 16));
+            float4 x = *p;
+            x.x -= g.lr * v[4 * q]; x.y -= g.lr * v[4 * q + 1]; x.z -= g.lr * v[4 * q + 2]; x.w -= g.lr * v[4 * q + 3];
+            *p = x;
             __nv_bfloat162 p0 = __floats2bfloat162_rn(x.x, x.y), p1 = __floats2bfloat162_rn(x.z, x.w);
             uint2 pk;
             pk.x = *reinterpret_cast<uint32_t*>(&p0);
             pk.y = *reinterpret_cast<uint32_t*>(&p1);
-            reinterpret_cast<uint2*>(sh)[j / 4] = pk;
+            *reinterpret_cast<uint2*>(hb + lane * 64 + ((((q >> 1) ^ ((lane >> 1) & 3))) * 16) + (q & 1) * 8) = pk;
           }
-          if (g.grad) {
+          if (g.grad && m < g.M) {
             float* gr = g.grad + (int64_t)m * g.ldo + n;
 #pragma unroll
             for (int j = 0; j < 32; j += 4)
               reinterpret_cast<float4*>(gr)[j / 4] = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+          }
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          __syncwarp();
+          if (lane == 0) {   // rows >= L are clipped (never touch b2)
+            asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                             reinterpret_cast<uint64_t>(&tmC)), "r"(smem_u32(wb)), "r"(n), "r"(row0) : "memory");
+            asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                             reinterpret_cast<uint64_t>(&tmD)), "r"(smem_u32(hb)), "r"(n), "r"(row0) : "memory");
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
           }
         }
       }
@@ -413,9 +499,7 @@ __global__ void __launch_bounds__(384, 1)
       __syncwarp();
       if (lane == 0) mbar_arrive(&tempty[acc]);   // accumulator may be overwritten
     }
-    if constexpr (EPI != TC_EPI_SGD) {
-      if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // stores complete
-    }
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // stores complete
   }
   tc_fence_before();
   __syncthreads();
@@ -453,6 +537,19 @@ cudaError_t make_store_map(CUtensorMap* m, const void* base, uint64_t inner, uin
   return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }
 
+// bf16 [outer][inner] store map, 32 x 32 boxes (64 B rows, 64B swizzle)
+cudaError_t make_bf16_store_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer,
+                                uint64_t row_bytes = 0) {
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {row_bytes ? row_bytes : inner * 2};
+  cuuint32_t box[2] = {32, 32};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = g_encode(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
 cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t row_bytes,
                      uint32_t box_inner, uint32_t box_outer) {
   cuuint64_t dims[2] = {inner, outer};
@@ -466,10 +563,10 @@ cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t 
 }
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
-cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c, TcArgs g,
-               int splits) {
+cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c,
+               const CUtensorMap& d, TcArgs g, int splits) {
   const size_t smem = (size_t)stages_of<EPI>() * (BM * BK * 2 + BN * BK * 2) + (EPI == TC_EPI_SGD ? 2048 : 0) +
-                      staging_bytes<EPI>() + 1024 + 256;
+                      staging_bytes<EPI>() + 1024 + 512;
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(k_gemm_tc<BN, A_MN, B_MN, EPI>,
@@ -480,7 +577,7 @@ cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, co
   g.splits = splits;
   const int64_t tiles = (int64_t)((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN) * splits;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, lc.sms));
-  return launch_k(lc, k_gemm_tc<BN, A_MN, B_MN, EPI>, dim3(grid), dim3(384), smem, a, b, c, g);
+  return launch_k(lc, k_gemm_tc<BN, A_MN, B_MN, EPI>, dim3(grid), dim3(384), smem, a, b, c, d, g);
 }
 
 // Widest N tile that still gives >= one CTA per SM (and does not overhang N by 2x).
@@ -501,24 +598,37 @@ int64_t padded_ld(int64_t L) { return (L + 7) / 8 * 8; }
 
 cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H, float lr, const Ptrs& P,
                            const WsLayout& W, float* W2, float* b2, float* grad_w2, float* grad_b2,
-                           float2* stats, int* stats_ntiles) {
+                           float2* stats, int* stats_ntiles, const int32_t* dz_rows,
+                           const int64_t* dz_lab_ptr, const int32_t* dz_lab) {
   if (!tc_available()) return cudaErrorNotSupported;
   const int64_t Lp = padded_ld(L);
   CUtensorMap ta, tb, tc;
   TcArgs g{};
   cudaError_t e;
-  if (which == 1) {  // Z = H1 W2^T + b2
+  if (which == 1 || which == 5) {  // Z = H1 W2^T + b2 (5: only the per-tile softmax partials)
     g.M = n; g.N = (int)L; g.K = H;
     g.out = P.z; g.ldo = Lp; g.bias = b2;
     const int bn = pick_bn((n + BM - 1) / BM, L, lc.sms);
     g.stats = stats; g.stats_ld = W.stats_ld;
+    g.write_z = which == 1;
     if (stats_ntiles) *stats_ntiles = (int)(2 * ((L + bn - 1) / bn));   // two column halves per tile
     if ((e = make_map(&ta, P.h1b, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
     if ((e = make_map(&tb, P.w2b, H, L, (uint64_t)H * 2, 64, bn)) != cudaSuccess) return e;
     if ((e = make_store_map(&tc, P.z, L, n, (uint64_t)Lp * 4, 1, 0, 2)) != cudaSuccess) return e;
-    if (bn == 256) return run<256, false, false, TC_EPI_Z>(lc, ta, tb, tc, g, 1);
-    if (bn == 128) return run<128, false, false, TC_EPI_Z>(lc, ta, tb, tc, g, 1);
-    return run<64, false, false, TC_EPI_Z>(lc, ta, tb, tc, g, 1);
+    if (bn == 256) return run<256, false, false, TC_EPI_Z>(lc, ta, tb, tc, tc, g, 1);
+    if (bn == 128) return run<128, false, false, TC_EPI_Z>(lc, ta, tb, tc, tc, g, 1);
+    return run<64, false, false, TC_EPI_Z>(lc, ta, tb, tc, tc, g, 1);
+  }
+  if (which == 4) {  // G1b: dZ (bf16) = (softmax(H1 W2^T + b2) - T) / B, recomputed tile by tile
+    g.M = n; g.N = (int)L; g.K = H;
+    g.bias = b2; g.lse = P.lse; g.rows = dz_rows; g.lab_ptr = dz_lab_ptr; g.lab = dz_lab; g.invB = 1.f / (float)n;
+    const int bn = pick_bn((n + BM - 1) / BM, L, lc.sms);
+    if ((e = make_map(&ta, P.h1b, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
+    if ((e = make_map(&tb, P.w2b, H, L, (uint64_t)H * 2, 64, bn)) != cudaSuccess) return e;
+    if ((e = make_bf16_store_map(&tc, P.dzb, L, n, (uint64_t)Lp * 2)) != cudaSuccess) return e;
+    if (bn == 256) return run<256, false, false, TC_EPI_DZ>(lc, ta, tb, tc, tc, g, 1);
+    if (bn == 128) return run<128, false, false, TC_EPI_DZ>(lc, ta, tb, tc, tc, g, 1);
+    return run<64, false, false, TC_EPI_DZ>(lc, ta, tb, tc, tc, g, 1);
   }
   if (which == 2) {  // dH1 partials = dZ W2
     g.M = n; g.N = H; g.K = (int)L;
@@ -532,9 +642,9 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
     const int64_t bmax = W.part_stride / H;
     if ((e = make_store_map(&tc, P.dhpart, H, bmax, (uint64_t)H * 4, splits,
                             (uint64_t)W.part_stride * 4, 3)) != cudaSuccess) return e;
-    if (H >= 256) return run<256, false, true, TC_EPI_PART>(lc, ta, tb, tc, g, splits);
-    if (H == 128) return run<128, false, true, TC_EPI_PART>(lc, ta, tb, tc, g, splits);
-    return run<64, false, true, TC_EPI_PART>(lc, ta, tb, tc, g, splits);
+    if (H >= 256) return run<256, false, true, TC_EPI_PART>(lc, ta, tb, tc, tc, g, splits);
+    if (H == 128) return run<128, false, true, TC_EPI_PART>(lc, ta, tb, tc, tc, g, splits);
+    return run<64, false, true, TC_EPI_PART>(lc, ta, tb, tc, tc, g, splits);
   }
   // which == 3: W2 -= lr dZ^T H1
   g.M = (int)L; g.N = H; g.K = n;
@@ -548,10 +658,12 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
   int bn = std::min(H, 128);
   while (bn > 64 && tiles_m * (H / bn) < lc.sms) bn /= 2;
   g.n_fast = 1;
-  tc = ta;   // unused by the SGD epilogue
-  if (bn == 256) return run<256, true, true, TC_EPI_SGD>(lc, ta, tb, tc, g, 1);
-  if (bn == 128) return run<128, true, true, TC_EPI_SGD>(lc, ta, tb, tc, g, 1);
-  return run<64, true, true, TC_EPI_SGD>(lc, ta, tb, tc, g, 1);
+  CUtensorMap td;   // W2 fp32 boxes (load + store) and the bf16 shadow boxes (store)
+  if ((e = make_store_map(&tc, W2, H, L, (uint64_t)H * 4, 1, 0, 2)) != cudaSuccess) return e;
+  if ((e = make_bf16_store_map(&td, P.w2b, H, L)) != cudaSuccess) return e;
+  if (bn == 256) return run<256, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
+  if (bn == 128) return run<128, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
+  return run<64, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
 }
 
 }  // namespace asgd
