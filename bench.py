@@ -174,6 +174,17 @@ def kernel_work(cls: str, cfg, bf16: bool, st):
     return ("bytes", 0.0)
 
 
+def step_ideal_s(cfg, B, nnz, U, nlab, hbm_gbs, tc_tflops):
+    """SURVEY.md §8(d) ideal time of one local step: max(algorithmic HBM bytes /
+    HBM peak, algorithmic flops / tensor peak).  Bytes: 8 nnz + 12 B + 4 labels
+    + 8 U H (touched W1 rows read+written) + 8 (H L + L) (W2/b2 read+written)
+    + 8 H (b1); flops: 6 B H L (G1-G3) + 4 nnz H (K-1, K-5)."""
+    H, L = cfg.H, cfg.L
+    by = 8.0 * nnz + 12.0 * B + 4.0 * nlab + 8.0 * U * H + 8.0 * (H * L + L) + 8.0 * H
+    fl = 6.0 * B * H * L + 4.0 * nnz * H
+    return max(by / (hbm_gbs * 1e9), fl / (tc_tflops * 1e12))
+
+
 def main():
     a = _args()
     rank = int(os.environ.get("RANK", 0))
@@ -298,11 +309,19 @@ def main():
         else:
             achieved = work / avg_s / 1e9
             bound, peak, unit = "hbm", peaks["hbm_gbs"], "GB/s"
-        traffic = _traffic(dname)
+        traffic = _traffic(cfg.name, prec, dname)
         roof = {"bound": bound, "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": unit,
                 "frac": round(achieved / peak, 4), "traffic": traffic, "kernel": dname,
                 "peak_source": src, "work_per_launch": work,
                 "step_share": round(float(ms[dom] / max(t_ms, 1e-9)), 4)}
+        # whole-job roofline: sum of per-step ideal times with
+        # each step's measured B, nnz, U, + merge 36 P bytes / HBM peak, over the timed time
+        tc_peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"]) if bf16 else \
+            148 * 128 * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+        t_ideal = sum(step_ideal_s(cfg, b_, z_, u_, l_, peaks["hbm_gbs"], tc_peak)
+                      for b_, z_, u_, l_ in zip(B_list, nnz_l, U_l, lab_l))
+        t_ideal += K * 36.0 * cfg.n_params / (peaks["hbm_gbs"] * 1e9)
+        roof["whole_step_frac"] = round(t_ideal / world / (t_max / 1e3), 4)
         out = {
             "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world, "steps": K,
             "warmup": W, "ms_per_step": round(t_max / K, 4), "higher_is_better": True,
@@ -340,11 +359,12 @@ def _bf16_available() -> bool:
         return False
 
 
-def _traffic(cls: str):
-    """dram bytes per launch of the kernel class from the committed ncu capture."""
+def _traffic(workload: str, prec: str, cls: str):
+    """dram read+write bytes per launch of the kernel class, from the committed
+    `ncu --set full` capture (profiles/traffic.json, tools/ncu_traffic.py)."""
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            return json.load(f).get(cls)
+            return json.load(f)[f"{workload}/{prec}"]["per_launch_bytes"].get(cls)
     except Exception:
         return None
 

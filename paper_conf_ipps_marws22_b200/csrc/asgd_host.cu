@@ -435,13 +435,13 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
       // fused softmax-CE: G1 keeps only per-tile (max, sum exp); k_lse -> lse, row loss;
       // G1b recomputes Z tile by tile and writes dZ = (softmax - T)/B (bf16) -- Z never hits HBM
       PCU(ASGD_K_G1, launch_gemm_tc(lc, 5, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
-    PCU(ASGD_K_SOFTMAX, ([&]() -> cudaError_t {
-          cudaError_t e = launch_lse(lc, n, H, ntiles, c->L.stats_ld, zstat, rows, x.lab_ptr, x.lab, P.h1b,
-                                     Pr.w2b, b2, P);
-          return e != cudaSuccess ? e
-                                  : launch_gemm_tc(lc, 4, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr,
-                                                   nullptr, nullptr, rows, x.lab_ptr, x.lab);
-        })());
+      PCU(ASGD_K_SOFTMAX, ([&]() -> cudaError_t {
+            cudaError_t e = launch_lse(lc, n, H, ntiles, c->L.stats_ld, zstat, rows, x.lab_ptr, x.lab, P.h1b,
+                                       Pr.w2b, b2, P);
+            return e != cudaSuccess ? e
+                                    : launch_gemm_tc(lc, 4, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr,
+                                                     nullptr, nullptr, rows, x.lab_ptr, x.lab);
+          })());
     }
     CU(cudaEventRecord(c->ev_sm, c->s));
     CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));

@@ -10,7 +10,7 @@ import sys
 
 def kname(s: str) -> str:
     s = s.replace("void ", "")
-    s = s.replace("asgd::<unnamed>::", "").replace("asgd::", "")
+    s = re.sub(r"^.*?(unnamed>|anonymous namespace\))::", "", s).replace("asgd::", "")
     s = s.split("(")[0]
     m = re.match(r"([A-Za-z0-9_:]+)(<.*>)?", s)
     base = m.group(1) if m else s
