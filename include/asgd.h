@@ -219,6 +219,21 @@ int asgd_sched_reset(asgd_sched* s, int64_t mb);
 int asgd_sched_wait(asgd_sched* s, int64_t mb, int64_t timeout_ms);
 int asgd_sched_close(asgd_sched* s, int32_t unlink_shm);
 
+/* Rank `rank`'s share of the current mega-batch (the dynamic routing loop,
+ * P:631-636, Fig. 2), run natively: until the scheduler is exhausted, take a
+ * ticket [start, start + len) of b_i samples and enqueue
+ * asgd_local_step(ctx, stream_rows_dev + start, len, lr, losses_dev + k) on the
+ * ctx stream for the k-th ticket.  At most `inflight` (1..8) of the rank's
+ * steps are outstanding when a ticket is taken: 1 = ask only when the previous
+ * step finished (paper-faithful), 2 = ask while one step still runs (Q32).
+ * stream_rows_dev: int32[M] device sample ids of the mega-batch (owned by the
+ * caller); losses_dev: nullable fp32 device[losses_cap] (a step k >= losses_cap
+ * gets no loss).  *n_steps = tickets taken (u_i of this mega-batch).  Returns
+ * when the last step is enqueued (asynchronous); errors as asgd_local_step. */
+int asgd_run_tickets(asgd_ctx* ctx, asgd_sched* s, int32_t rank, int64_t b_i,
+                     const int32_t* stream_rows_dev, float lr, float* losses_dev,
+                     int64_t losses_cap, int32_t inflight, int64_t* n_steps);
+
 /* Replay (parity): ranks in ticket order -> routes (rank, start, len) with the
  * batch sizes b[rank], stopping at M.  out: int64[3*cap]. */
 int asgd_route_replay(int32_t n_tickets, const int32_t* order, const int64_t* b,

@@ -126,6 +126,17 @@ class Replica:
         call("asgd_local_step", self.ctx, _ptr(rows), int(rows.numel()), float(lr),
              _ptr(loss_out) if loss_out is not None else None)
 
+    def run_tickets(self, sched: "Scheduler", rank: int, b: int, stream_rows: torch.Tensor, lr: float,
+                    losses: Optional[torch.Tensor] = None, inflight: int = 2) -> int:
+        """This rank's share of the mega-batch (asgd_run_tickets): the ticket loop
+        in native code; returns the number of local steps enqueued."""
+        assert stream_rows.dtype == torch.int32 and stream_rows.is_cuda and stream_rows.is_contiguous()
+        n = C.c_int64()
+        call("asgd_run_tickets", self.ctx, sched.h, int(rank), int(b), _ptr(stream_rows), float(lr),
+             _ptr(losses) if losses is not None else None, int(losses.numel()) if losses is not None else 0,
+             int(inflight), C.byref(n))
+        return n.value
+
     def updates(self) -> int:
         u = C.c_int64()
         call("asgd_updates", self.ctx, C.byref(u))

@@ -53,6 +53,7 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) ==
 size_t up256(size_t x) { return (x + 255) & ~size_t(255); }
 
 constexpr int kSqnormParts = 1024;
+constexpr int kMaxInflight = 8;
 // Above this many bytes of fp32 logits per step the bf16 path fuses softmax-CE
 // into the GEMMs (Z never written); below, Z stays L2-resident and is stored.
 constexpr int64_t kFusedCeBytes = 64ll << 20;
@@ -124,6 +125,7 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.w2b2 = take(bf ? (size_t)Lb * H * 2 : 0);
   L.red = take((L.n_red + 8) * 8);
   L.eval_top = take(B * 8 * 4);
+  L.rowsc = take(B * 4);
   L.total = o;
   return L;
 }
@@ -145,10 +147,26 @@ Ptrs ws_ptrs(char* b, const WsLayout& L) {
   p.rbase = (int64_t*)(b + L.rbase);
   p.da1b = (bf16*)(b + L.da1b);
   p.lse = (float*)(b + L.lse);
+  p.rowsc = (int32_t*)(b + L.rowsc);
   return p;
 }
 
 }  // namespace asgd
+
+// One captured local step (everything after K-0 (a), which is launched eagerly
+// with the step's row ids, lr and loss pointer and publishes them to the rest).
+struct StepGraph {
+  int n = 0, cur = 0;
+  uint32_t mask = 0;
+  int seen = 0;                       // captured on the 2nd step with this key
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t exec = nullptr;
+  int64_t kernels = 0;                // kernel nodes (asgd_kernel_launches per replay)
+  struct Prof { cudaGraphNode_t node; int cls; bool begin; };
+  std::vector<Prof> prof;             // profiling event-record nodes, capture order
+  std::vector<cudaEvent_t> placeholders;
+  uint64_t last_use = 0;
+};
 
 struct asgd_ctx {
   asgd_model_desc d;
@@ -175,9 +193,16 @@ struct asgd_ctx {
   size_t pused[ASGD_PROF_N] = {};
   cudaStream_t s2 = nullptr;                     // side stream: K-0 overlaps the dense chain
   cudaStream_t s3 = nullptr;                     // side stream: G3 + b1 (bf16 path)
+  cudaStream_t sc = nullptr;                     // private stream the step graphs are captured on
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_sm = nullptr, ev_dh = nullptr, ev_a = nullptr;
   bf16* w2b_buf[2] = {nullptr, nullptr};         // double-buffered bf16 W2 shadow
   int w2b_cur = 0;
+  std::vector<StepGraph> graphs;                 // CUDA-graph cache of the step, LRU
+  uint64_t graph_clock = 0;
+  bool capturing = false;
+  std::vector<std::pair<cudaEvent_t, int>> cap_ph;   // (placeholder, cls * 2 + begin) during capture
+  cudaEvent_t prof_sink = nullptr;                // target of profiling nodes past kMaxProfPairs
+  cudaEvent_t ev_ring[8] = {};                    // asgd_run_tickets: completion of the last steps
   Launch lc() { return Launch{s, &launches, sms}; }
   Launch lc2() { return Launch{s2, &launches, sms}; }
   Launch lc3() { return Launch{s3, &launches, sms}; }
@@ -189,6 +214,13 @@ constexpr size_t kMaxProfPairs = 8192;
 // Record an event on stream st at the start / end of a kernel-class section.
 void prof_mark(asgd_ctx* c, int cls, bool begin, cudaStream_t st) {
   if (!(c->prof_mask & (1u << cls))) return;
+  if (c->capturing) {   // an event-record node; its event is set per replay (bind_prof_events)
+    cudaEvent_t ph;
+    if (cudaEventCreate(&ph) != cudaSuccess) return;
+    cudaEventRecordWithFlags(ph, st, cudaEventRecordExternal);
+    c->cap_ph.push_back({ph, cls * 2 + (begin ? 1 : 0)});
+    return;
+  }
   auto& v = c->pev[cls];
   size_t& u = c->pused[cls];
   if (begin) {
@@ -205,6 +237,48 @@ void prof_mark(asgd_ctx* c, int cls, bool begin, cudaStream_t st) {
     if (u >= kMaxProfPairs || v.size() < 2 * (u + 1)) return;
     cudaEventRecord(v[2 * u + 1], st);
     ++u;
+  }
+}
+
+void destroy_graph(StepGraph& g) {
+  if (g.exec) cudaGraphExecDestroy(g.exec);
+  if (g.graph) cudaGraphDestroy(g.graph);
+  for (cudaEvent_t e : g.placeholders) cudaEventDestroy(e);
+  g = StepGraph{};
+}
+
+void clear_graphs(asgd_ctx* c) {
+  for (auto& g : c->graphs) destroy_graph(g);
+  c->graphs.clear();
+}
+
+bool graphs_enabled() {
+  static const int on = [] {
+    const char* e = getenv("ASGD_GRAPH");
+    return (e && e[0] == '0') ? 0 : 1;
+  }();
+  return on != 0;
+}
+
+// Point the graph's profiling nodes at fresh pool events, in the order prof_mark
+// would have used them for an eager step.
+void bind_prof_events(asgd_ctx* c, StepGraph& g) {
+  for (const auto& pn : g.prof) {
+    auto& v = c->pev[pn.cls];
+    size_t& u = c->pused[pn.cls];
+    cudaEvent_t ev = c->prof_sink;
+    if (u < kMaxProfPairs) {
+      if (v.size() < 2 * (u + 1)) {
+        cudaEvent_t a, b;
+        if (cudaEventCreate(&a) == cudaSuccess) {
+          if (cudaEventCreate(&b) == cudaSuccess) { v.push_back(a); v.push_back(b); }
+          else cudaEventDestroy(a);
+        }
+      }
+      if (v.size() >= 2 * (u + 1)) ev = v[2 * u + (pn.begin ? 0 : 1)];
+      if (!pn.begin) ++u;
+    }
+    if (ev) cudaGraphExecEventRecordNodeSetEvent(g.exec, pn.node, ev);
   }
 }
 }  // namespace
@@ -293,12 +367,17 @@ int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device, v
 
 int asgd_replica_destroy(asgd_ctx* c) {
   if (c) {
+    clear_graphs(c);
+    if (c->prof_sink) cudaEventDestroy(c->prof_sink);
+    for (cudaEvent_t ev : c->ev_ring)
+      if (ev) cudaEventDestroy(ev);
     for (auto& v : c->pev)
       for (cudaEvent_t e : v) cudaEventDestroy(e);
     for (cudaEvent_t ev : {c->ev_fork, c->ev_join, c->ev_sm, c->ev_dh, c->ev_a})
       if (ev) cudaEventDestroy(ev);
     if (c->s2) cudaStreamDestroy(c->s2);
     if (c->s3) cudaStreamDestroy(c->s3);
+    if (c->sc) cudaStreamDestroy(c->sc);
   }
   delete c;
   return ASGD_OK;
@@ -334,6 +413,7 @@ int asgd_data_register(asgd_ctx* c, const asgd_csr* x) {
   if (x->n_rows <= 0 || x->nnz < 0 || x->n_lab <= 0) return fail(ASGD_E_SHAPE, "empty split");
   int rc = validate(c, x);
   if (rc) return rc;
+  if (!c->has_data || memcmp(&c->data, x, sizeof(*x)) != 0) clear_graphs(c);   // graphs hold the pointers
   c->data = *x;
   c->has_data = true;
   return ASGD_OK;
@@ -348,6 +428,9 @@ int asgd_data_upload(asgd_ctx* c, const asgd_csr* h, const asgd_csr* dv) {
   CU(cudaMemcpyAsync((void*)dv->val, h->val, h->nnz * 4, cudaMemcpyHostToDevice, c->s));
   CU(cudaMemcpyAsync((void*)dv->lab_ptr, h->lab_ptr, (h->n_rows + 1) * 8, cudaMemcpyHostToDevice, c->s));
   CU(cudaMemcpyAsync((void*)dv->lab, h->lab, h->n_lab * 4, cudaMemcpyHostToDevice, c->s));
+  if (!c->has_data || c->data.row_ptr != dv->row_ptr || c->data.col != dv->col || c->data.val != dv->val ||
+      c->data.lab_ptr != dv->lab_ptr || c->data.lab != dv->lab || c->data.n_rows != dv->n_rows)
+    clear_graphs(c);   // graphs hold the dataset pointers and row count
   c->data = *dv;
   c->data.nnz = h->nnz;
   c->data.n_lab = h->n_lab;
@@ -355,14 +438,18 @@ int asgd_data_upload(asgd_ctx* c, const asgd_csr* h, const asgd_csr* dv) {
   return ASGD_OK;
 }
 
-int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float* loss_dev) {
-  if (!c || !rows) return fail(ASGD_E_ARG, "null argument");
-  if (!c->has_data) return fail(ASGD_E_STATE, "no data registered");
-  const asgd_model_desc& m = c->d;
-  if (n < 1 || n > m.b_max) return fail(ASGD_E_SHAPE, "n_rows=%d not in [1, %d]", n, m.b_max);
+}  // extern "C"
+
+namespace {
+// Everything of a local step after K-0 (a): reads the step's rows / lr / loss
+// pointer from the workspace (P.rowsc, meta), so it can be captured once per
+// (n, shadow buffer, profile mask) and replayed.
+// (b-f): touched-feature set on side stream s2, joined before K-5.
+int enqueue_step(asgd_ctx* c, int n) {
   Launch lc = c->lc();
   const Ptrs& P = c->P;
   const asgd_csr& x = c->data;
+  const asgd_model_desc& m = c->d;
   const bool bf = m.precision == ASGD_PREC_BF16;
   const int H = (int)m.H;
   const int64_t Lb = m.L;
@@ -372,15 +459,18 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
   float* W2 = c->params + c->o_w2;
   float* b2 = c->params + c->o_b2;
   float* g = c->dbg;
-  if (g) CU(cudaMemsetAsync(g, 0, c->Pn * sizeof(float), c->s));
-  // K-0 (a): batch view; (b-f): touched-feature set on the side stream, joined before K-5
-  CU(launch_batch_scan(lc, rows, n, x.row_ptr, x.lab_ptr, x.n_rows, P, c->L.nz_cap, c->L.nl_cap));
-  CU(cudaEventRecord(c->ev_fork, c->s));
-  CU(cudaStreamWaitEvent(c->s2, c->ev_fork, 0));
-  PCU_ON(c->s2, ASGD_K_TOUCHED, launch_touched(c->lc2(), rows, n, x.row_ptr, x.col, x.val, m.F, P, c->L, m.b_max));
-  CU(cudaEventRecord(c->ev_join, c->s2));
+  static const bool k0_late = [] { const char* e = getenv("ASGD_K0_LATE"); return e && e[0] == '1'; }();
+  auto fork_k0 = [&]() -> int {
+    CU(cudaEventRecord(c->ev_fork, c->s));
+    CU(cudaStreamWaitEvent(c->s2, c->ev_fork, 0));
+    PCU_ON(c->s2, ASGD_K_TOUCHED, launch_touched(c->lc2(), P.rowsc, n, x.row_ptr, x.col, x.val, m.F, P, c->L, m.b_max));
+    CU(cudaEventRecord(c->ev_join, c->s2));
+    return ASGD_OK;
+  };
+  if (!k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   // K-1
-  PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, rows, n, x.row_ptr, x.col, x.val, W1, b1, H, P, c->L, bf));
+  PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, P.rowsc, n, x.row_ptr, x.col, x.val, W1, b1, H, P, c->L, bf));
+  if (k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   if (!bf) {
     // fp32 path: one stream, G2 reads W2 before G3 updates it in place
     GemmArgs a{};
@@ -390,7 +480,7 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     a.B = W2; a.bs0 = 1; a.bs1 = H;
     a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = Lp; a.bias = b2; a.splitk = 1;
     PCU(ASGD_K_G1, launch_gemm_f32(lc, a));
-    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, false));
+    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, false));
     // G2: dH1 partials = dZ W2 (pre-step W2)
     a = GemmArgs{};
     a.M = n; a.N = H; a.K = (int)Lb;
@@ -401,20 +491,20 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     PCU(ASGD_K_G2, launch_gemm_f32(lc, a));
     PCU(ASGD_K_DH, ([&]() -> cudaError_t {
           cudaError_t e = launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, false);
-          return e != cudaSuccess ? e : launch_b1_update(lc, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev);
+          return e != cudaSuccess ? e : launch_b1_update(lc, n, H, b1, P, c->L, g ? g + c->o_b1 : nullptr);
         })());
-    PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, Lp, b2, lr, P, false, g ? g + c->o_b2 : nullptr));
+    PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, Lp, b2, P, false, g ? g + c->o_b2 : nullptr));
     // G3: W2 -= lr dZ^T H1
     a = GemmArgs{};
     a.M = (int)Lb; a.N = H; a.K = n;
     a.A = P.z; a.as0 = 1; a.as1 = Lp;
     a.B = P.h1; a.bs0 = H; a.bs1 = 1;
-    a.epi = EPI_SGD; a.C = W2; a.ldc = H; a.lr = lr; a.grad = g ? g + c->o_w2 : nullptr;
+    a.epi = EPI_SGD; a.C = W2; a.ldc = H; a.meta = P.meta; a.grad = g ? g + c->o_w2 : nullptr;
     a.splitk = 1;
     PCU(ASGD_K_G3, launch_gemm_f32(lc, a));
     // K-5 (needs K-0's segments)
     CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
-    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
+    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
   } else {
     // bf16 path, a DAG over three streams:
     //   s : G1 -> softmax -> G2 -> dH reduce -> [K-0 joined] K-5
@@ -428,37 +518,131 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     int ntiles = 0;
     if ((int64_t)m.b_max * Lb * 4 <= kFusedCeBytes) {
       // logits fit in L2: G1 stores Z (+ per-tile softmax partials), one pass of softmax-CE
-      PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
-      PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, rows, x.lab_ptr, x.lab, P, true, zstat, ntiles,
+      PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
+      PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, true, zstat, ntiles,
                                             c->L.stats_ld));
     } else {
       // fused softmax-CE: G1 keeps only per-tile (max, sum exp); k_lse -> lse, row loss;
       // G1b recomputes Z tile by tile and writes dZ = (softmax - T)/B (bf16) -- Z never hits HBM
-      PCU(ASGD_K_G1, launch_gemm_tc(lc, 5, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
+      PCU(ASGD_K_G1, launch_gemm_tc(lc, 5, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
       PCU(ASGD_K_SOFTMAX, ([&]() -> cudaError_t {
-            cudaError_t e = launch_lse(lc, n, H, ntiles, c->L.stats_ld, zstat, rows, x.lab_ptr, x.lab, P.h1b,
+            cudaError_t e = launch_lse(lc, n, H, ntiles, c->L.stats_ld, zstat, P.rowsc, x.lab_ptr, x.lab, P.h1b,
                                        Pr.w2b, b2, P);
             return e != cudaSuccess ? e
-                                    : launch_gemm_tc(lc, 4, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr,
-                                                     nullptr, nullptr, rows, x.lab_ptr, x.lab);
+                                    : launch_gemm_tc(lc, 4, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr,
+                                                     nullptr, nullptr, P.rowsc, x.lab_ptr, x.lab);
           })());
     }
     CU(cudaEventRecord(c->ev_sm, c->s));
     CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
-    PCU_ON(c->s3, ASGD_K_G3, launch_gemm_tc(lc3, 3, n, Lb, H, lr, Pw, c->L, W2, b2, g ? g + c->o_w2 : nullptr,
+    PCU_ON(c->s3, ASGD_K_G3, launch_gemm_tc(lc3, 3, n, Lb, H, Pw, c->L, W2, b2, g ? g + c->o_w2 : nullptr,
                                             g ? g + c->o_b2 : nullptr));
-    PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, lr, Pr, c->L, W2, b2, nullptr, nullptr));
+    PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr));
     PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, true));
     CU(cudaEventRecord(c->ev_dh, c->s));
     CU(cudaStreamWaitEvent(c->s3, c->ev_dh, 0));
-    PCU_ON(c->s3, ASGD_K_DH, launch_b1_update(lc3, n, H, b1, lr, P, c->L, g ? g + c->o_b1 : nullptr, loss_dev));
+    PCU_ON(c->s3, ASGD_K_DH, launch_b1_update(lc3, n, H, b1, P, c->L, g ? g + c->o_b1 : nullptr));
     CU(cudaEventRecord(c->ev_a, c->s3));
     // K-5 (needs K-0's segments)
     CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
-    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, lr, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
+    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
     CU(cudaStreamWaitEvent(c->s, c->ev_a, 0));
-    c->w2b_cur ^= 1;
   }
+  return ASGD_OK;
+}
+
+
+constexpr size_t kMaxGraphs = 16;
+
+// Replay (capturing on the 2nd use of a key) the rest of the step as a CUDA graph.
+int step_graph(asgd_ctx* c, int n) {
+  StepGraph* hit = nullptr;
+  for (auto& gr : c->graphs)
+    if (gr.n == n && gr.cur == c->w2b_cur && gr.mask == c->prof_mask) { hit = &gr; break; }
+  if (!hit) {
+    if (c->graphs.size() >= kMaxGraphs) {
+      auto lru = std::min_element(c->graphs.begin(), c->graphs.end(),
+                                  [](const StepGraph& a, const StepGraph& b) { return a.last_use < b.last_use; });
+      destroy_graph(*lru);
+      c->graphs.erase(lru);
+    }
+    c->graphs.emplace_back();
+    hit = &c->graphs.back();
+    hit->n = n; hit->cur = c->w2b_cur; hit->mask = c->prof_mask;
+  }
+  StepGraph& G = *hit;
+  G.last_use = ++c->graph_clock;
+  if (!G.exec && G.seen++ == 0) return enqueue_step(c, n);   // first use: eager (warms attributes)
+  if (!G.exec) {
+    // capture on the private stream sc (the ctx stream may be the legacy default
+    // stream, which cannot capture); the graph itself is launched on c->s
+    if (!c->sc) CU(cudaStreamCreateWithFlags(&c->sc, cudaStreamNonBlocking));
+    const int64_t l0 = c->launches;
+    c->cap_ph.clear();
+    cudaStream_t user = c->s;
+    c->s = c->sc;
+    cudaError_t eb = cudaStreamBeginCapture(c->s, cudaStreamCaptureModeThreadLocal);
+    if (eb != cudaSuccess) { c->s = user; return cuda_fail(eb, "cudaStreamBeginCapture"); }
+    c->capturing = true;
+    const int rc = enqueue_step(c, n);
+    c->capturing = false;
+    cudaGraph_t graph = nullptr;
+    const cudaError_t ec = cudaStreamEndCapture(c->s, &graph);
+    c->s = user;
+    for (auto& ph : c->cap_ph) G.placeholders.push_back(ph.first);
+    G.kernels = c->launches - l0;
+    c->launches = l0;
+    if (rc != ASGD_OK || ec != cudaSuccess) {
+      if (graph) cudaGraphDestroy(graph);
+      return rc != ASGD_OK ? rc : cuda_fail(ec, "cudaStreamEndCapture");
+    }
+    G.graph = graph;
+    CU(cudaGraphInstantiate(&G.exec, graph, 0));
+    if (!c->cap_ph.empty()) {
+      size_t nn = 0;
+      CU(cudaGraphGetNodes(graph, nullptr, &nn));
+      std::vector<cudaGraphNode_t> nodes(nn);
+      CU(cudaGraphGetNodes(graph, nodes.data(), &nn));
+      std::vector<cudaGraphNode_t> by_ph(c->cap_ph.size(), nullptr);
+      for (cudaGraphNode_t nd : nodes) {
+        cudaGraphNodeType t;
+        if (cudaGraphNodeGetType(nd, &t) != cudaSuccess || t != cudaGraphNodeTypeEventRecord) continue;
+        cudaEvent_t ev;
+        if (cudaGraphEventRecordNodeGetEvent(nd, &ev) != cudaSuccess) continue;
+        for (size_t i = 0; i < c->cap_ph.size(); ++i)
+          if (c->cap_ph[i].first == ev) by_ph[i] = nd;
+      }
+      for (size_t i = 0; i < c->cap_ph.size(); ++i)
+        if (by_ph[i]) G.prof.push_back({by_ph[i], c->cap_ph[i].second / 2, (c->cap_ph[i].second & 1) != 0});
+      if (!c->prof_sink) CU(cudaEventCreate(&c->prof_sink));
+    }
+    c->cap_ph.clear();
+  }
+  if (!G.prof.empty()) bind_prof_events(c, G);
+  CU(cudaGraphLaunch(G.exec, c->s));
+  c->launches += G.kernels;
+  return ASGD_OK;
+}
+}  // namespace
+
+extern "C" {
+
+int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float* loss_dev) {
+  if (!c || !rows) return fail(ASGD_E_ARG, "null argument");
+  if (!c->has_data) return fail(ASGD_E_STATE, "no data registered");
+  const asgd_model_desc& m = c->d;
+  if (n < 1 || n > m.b_max) return fail(ASGD_E_SHAPE, "n_rows=%d not in [1, %d]", n, m.b_max);
+  Launch lc = c->lc();
+  const Ptrs& P = c->P;
+  const asgd_csr& x = c->data;
+  float* g = c->dbg;
+  if (g) CU(cudaMemsetAsync(g, 0, c->Pn * sizeof(float), c->s));
+  // K-0 (a): batch view + the step's row ids, lr and loss pointer, launched eagerly;
+  // the rest of the step replays a cached CUDA graph when possible
+  CU(launch_batch_scan(lc, rows, n, x.row_ptr, x.lab_ptr, x.n_rows, P, c->L.nz_cap, c->L.nl_cap, lr, loss_dev));
+  const int rc = (graphs_enabled() && !g) ? step_graph(c, n) : enqueue_step(c, n);
+  if (rc != ASGD_OK) return rc;
+  if (m.precision == ASGD_PREC_BF16) c->w2b_cur ^= 1;
   ++c->u;
   return ASGD_OK;
 }
@@ -549,7 +733,7 @@ int asgd_eval_topk(asgd_ctx* c, const asgd_csr* t, const int32_t* rows, int32_t 
     } else {
       Ptrs Pr = P;
       Pr.w2b = c->w2b_buf[c->w2b_cur];
-      CU(launch_gemm_tc(lc, 1, nb, m.L, H, 0.f, Pr, c->L, W2, b2, nullptr, nullptr));
+      CU(launch_gemm_tc(lc, 1, nb, m.L, H, Pr, c->L, W2, b2, nullptr, nullptr));
     }
     CU(launch_topk(lc, nb, m.L, padded_ld(m.L), k, P.z, topk + (int64_t)r0 * k));
   }
@@ -773,6 +957,29 @@ int asgd_sched_next(asgd_sched* s, int32_t rank, int64_t b, int64_t* start, int6
   *start = c;
   *len = l;
   return 1;
+}
+
+int asgd_run_tickets(asgd_ctx* c, asgd_sched* s, int32_t rank, int64_t b_i, const int32_t* stream_rows,
+                     float lr, float* losses, int64_t losses_cap, int32_t inflight, int64_t* n_steps) {
+  if (!c || !s || !stream_rows || !n_steps || b_i < 1) return fail(ASGD_E_ARG, "bad argument");
+  if (inflight < 1 || inflight > kMaxInflight) return fail(ASGD_E_ARG, "inflight=%d not in [1, %d]", inflight, kMaxInflight);
+  for (auto& ev : c->ev_ring)
+    if (!ev) CU(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+  int64_t k = 0;
+  for (;;) {
+    if (k >= inflight) CU(cudaEventSynchronize(c->ev_ring[(k - inflight) % kMaxInflight]));
+    int64_t start = 0, len = 0;
+    const int r = asgd_sched_next(s, rank, b_i, &start, &len);
+    if (r < 0) return fail(-r, "asgd_sched_next failed");
+    if (r == 0) break;
+    const int rc = asgd_local_step(c, stream_rows + start, (int32_t)len, lr,
+                                   (losses && k < losses_cap) ? losses + k : nullptr);
+    if (rc != ASGD_OK) return rc;
+    CU(cudaEventRecord(c->ev_ring[k % kMaxInflight], c->s));
+    ++k;
+  }
+  *n_steps = k;
+  return ASGD_OK;
 }
 
 int asgd_sched_log(asgd_sched* s, int64_t* out, int64_t cap, int64_t* n_out) {

@@ -15,7 +15,12 @@ constexpr int kMaxRowLabels = 1024;
 // Features per tile of the touched-feature scan.
 constexpr int kScanTile = 1024;
 // meta[] slots (int32, device)
-enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_COUNT = 8, M_BAR = 32 };  // M_BAR: 64-bit grid-barrier counter (slots 32-33)
+// M_LR: the step's learning rate (float bits), M_LOSS: 64-bit device pointer the
+// step's mean loss goes to (slots 10-11), both written by K-0 (a) so that the
+// rest of the step (and its CUDA graph) takes no per-step scalar arguments;
+// M_BAR: 64-bit grid-barrier counter (slots 32-33).
+enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_LR = 6, M_COUNT = 8, M_LOSS = 10,
+       M_BAR = 32 };
 // error bits in meta[M_ERR]
 enum { ERR_NNZ_CAP = 1, ERR_LAB_CAP = 2, ERR_ROW_ID = 4 };
 
@@ -26,6 +31,7 @@ struct WsLayout {
   size_t meta, boff, loff, cnt, fseg, fuid, uniq, useg, tsum, tpre;
   size_t e_n, e_v, e_u, e_f, part1, rowcnt, part5, ucnt, bits;
   size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, b2part, rbase, da1b, zstat, lse;
+  size_t rowsc;
   size_t total;
   int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride, stats_ld;
 };
@@ -41,7 +47,12 @@ struct Ptrs {  // typed views of the workspace
   int64_t* rbase;   // row_ptr[rows[r]] of the current batch (written by K-0 (a))
   bf16* da1b;       // bf16 copy of dA1 (bf16 path; staged by K-5)
   float* lse;       // per-row log-sum-exp of Z (bf16 path)
+  int32_t* rowsc;   // copy of the step's dataset row ids (written by K-0 (a))
 };
+__device__ __forceinline__ float step_lr(const int32_t* meta) { return __int_as_float(meta[M_LR]); }
+__device__ __forceinline__ float* step_loss(const int32_t* meta) {
+  return *reinterpret_cast<float* const*>(meta + M_LOSS);
+}
 int row_block();   // rows per db1 partial (kernels_dense.cu)
 int b2_chunks();   // row chunks of the db2 partial sums
 Ptrs ws_ptrs(char* base, const WsLayout& L);
@@ -80,9 +91,10 @@ cudaError_t launch_k(const Launch& lc, void (*kernel)(KArgs...), dim3 grid, dim3
 }
 
 // ---------------------------------------------------------------- K-0
+// Also copies rows to P.rowsc and stores lr / loss_dev in meta (M_LR, M_LOSS).
 cudaError_t launch_batch_scan(const Launch&, const int32_t* rows, int n, const int64_t* row_ptr,
                               const int64_t* lab_ptr, int64_t n_data_rows, const Ptrs&,
-                              int64_t nz_cap, int64_t nl_cap);
+                              int64_t nz_cap, int64_t nl_cap, float lr = 0.f, float* loss_dev = nullptr);
 cudaError_t launch_touched(const Launch&, const int32_t* rows, int n, const int64_t* row_ptr,
                            const int32_t* col, const float* val, int64_t F, const Ptrs&,
                            const WsLayout&, int b_max);
@@ -92,7 +104,8 @@ cudaError_t launch_spmm_fwd(const Launch&, const int32_t* rows, int n, const int
                             int H, const Ptrs&, const WsLayout&, bool want_bf16);
 // ---------------------------------------------------------------- K-5
 // dA1b: bf16 copy of dA1 (bf16 path) or null (fp32 path stages fp32 dA1).
-cudaError_t launch_scatter_sgd(const Launch&, float* W1, int H, float lr, const Ptrs&,
+// The learning rate of every SGD update is the step's meta[M_LR].
+cudaError_t launch_scatter_sgd(const Launch&, float* W1, int H, const Ptrs&,
                                const WsLayout&, float* grad_w1, const bf16* dA1b, int b_max);
 // ---------------------------------------------------------------- dense (fp32 SIMT)
 // C(m,n) = sum_k A(m,k) B(k,n), A(m,k) = A[m*as0 + k*as1], B(k,n) = B[k*bs0 + n*bs1]
@@ -105,7 +118,7 @@ struct GemmArgs {
   float* C; int64_t ldc;          // STORE_BIAS: C[m*ldc+n] = acc + bias[n]
   const float* bias;
   int splitk; int64_t part_stride; // SPLITK: C[z*part_stride + m*ldc + n]
-  float lr; float* grad;           // SGD: C[m*ldc+n] -= lr*acc; grad[m*ldc+n] = acc
+  const int32_t* meta; float* grad; // SGD: C[m*ldc+n] -= lr*acc (lr = meta[M_LR]); grad[m*ldc+n] = acc
   bf16* shadow;                    // SGD: shadow[m*ldc+n] = bf16(new C)
 };
 cudaError_t launch_gemm_f32(const Launch&, const GemmArgs&);
@@ -118,9 +131,9 @@ cudaError_t launch_softmax_ce(const Launch&, int n, int64_t L, int64_t ldz, cons
                               int64_t stats_ld = 0);
 cudaError_t launch_dh_reduce(const Launch&, int n, int H, int splitk, const Ptrs&, const WsLayout&,
                              bool want_bf16);
-cudaError_t launch_b1_update(const Launch&, int n, int H, float* b1, float lr, const Ptrs&,
-                             const WsLayout&, float* grad_b1, float* loss_dev);
-cudaError_t launch_b2_update(const Launch&, int n, int64_t L, int64_t ldz, float* b2, float lr,
+cudaError_t launch_b1_update(const Launch&, int n, int H, float* b1, const Ptrs&,
+                             const WsLayout&, float* grad_b1);
+cudaError_t launch_b2_update(const Launch&, int n, int64_t L, int64_t ldz, float* b2,
                              const Ptrs&, bool from_bf16, float* grad_b2);
 cudaError_t launch_to_bf16(const Launch&, const float* src, bf16* dst, int64_t count);
 // ---------------------------------------------------------------- tcgen05 (bf16)
@@ -128,7 +141,7 @@ bool tc_available();
 // which: 1 = G1 (Z = H1 W2^T + b2), 2 = G2 (dH1 split-K partials), 3 = G3 (W2 -= lr dZ^T H1 and
 // b2 -= lr 1^T dZ, both fused in the epilogue)
 // stats (G1 only, nullable): per (N tile, row) softmax partials; *stats_ntiles = N tiles.
-cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int H, float lr,
+cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int H,
                            const Ptrs&, const WsLayout&, float* W2, float* b2, float* grad_w2,
                            float* grad_b2, float2* stats = nullptr, int* stats_ntiles = nullptr,
                            const int32_t* dz_rows = nullptr, const int64_t* dz_lab_ptr = nullptr,

@@ -80,7 +80,7 @@ __global__ void __launch_bounds__(256) k_gemm_f32(GemmArgs g) {
       } else if (g.epi == EPI_SPLITK) {
         g.C[(int64_t)blockIdx.z * g.part_stride + o] = acc[i][j];
       } else {  // EPI_SGD
-        const float nw = g.C[o] - g.lr * acc[i][j];
+        const float nw = g.C[o] - step_lr(g.meta) * acc[i][j];
         g.C[o] = nw;
         if (g.grad) g.grad[o] = acc[i][j];
         if (g.shadow) g.shadow[o] = __float2bfloat16_rn(nw);
@@ -289,10 +289,12 @@ __global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
 // db1[c] = sum_r dA1[r][c] (one warp per column, lanes over rows, fixed shuffle
 // tree); b1 -= lr db1.  The extra last warp computes the mean loss.
 __global__ void __launch_bounds__(256) k_b1_update(int n, int H, const float* __restrict__ dA1, float* b1,
-                                                   float lr, float* grad_b1,
-                                                   const float* __restrict__ rowloss, float* loss_dev) {
+                                                   const int32_t* __restrict__ meta, float* grad_b1,
+                                                   const float* __restrict__ rowloss) {
   pdl_trigger();
   pdl_wait();
+  const float lr = step_lr(meta);
+  float* loss_dev = step_loss(meta);
   const int lane = threadIdx.x & 31;
   const int c = blockIdx.x * 8 + (threadIdx.x >> 5);
   if (c < H) {
@@ -349,9 +351,10 @@ __global__ void __launch_bounds__(256) k_b2_part(int n, int64_t L, int64_t ldz, 
 
 // b2 -= lr * sum_y b2part[y]
 __global__ void __launch_bounds__(256) k_b2_apply(int64_t L, int chunks, const float* __restrict__ b2part,
-                                                  float* b2, float lr, float* grad_b2) {
+                                                  float* b2, const int32_t* __restrict__ meta, float* grad_b2) {
   pdl_trigger();
   pdl_wait();
+  const float lr = step_lr(meta);
   const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= L) return;
   float s = 0.f;
@@ -400,18 +403,18 @@ cudaError_t launch_dh_reduce(const Launch& lc, int n, int H, int splitk, const P
   return cudaGetLastError();
 }
 
-cudaError_t launch_b1_update(const Launch& lc, int n, int H, float* b1, float lr, const Ptrs& P,
-                             const WsLayout& L, float* grad_b1, float* loss_dev) {
-  launch_k(lc, k_b1_update, dim3(H / 8 + 1), dim3(256), 0, n, H, P.da1, b1, lr, grad_b1, P.rowloss, loss_dev);
+cudaError_t launch_b1_update(const Launch& lc, int n, int H, float* b1, const Ptrs& P,
+                             const WsLayout& L, float* grad_b1) {
+  launch_k(lc, k_b1_update, dim3(H / 8 + 1), dim3(256), 0, n, H, P.da1, b1, P.meta, grad_b1, P.rowloss);
   return cudaGetLastError();
 }
 
-cudaError_t launch_b2_update(const Launch& lc, int n, int64_t L, int64_t ldz, float* b2, float lr,
+cudaError_t launch_b2_update(const Launch& lc, int n, int64_t L, int64_t ldz, float* b2,
                              const Ptrs& P, bool from_bf16, float* grad_b2) {
   const int chunks = std::max(1, std::min(kB2Chunks, n / 16));
   dim3 grid((unsigned)((L + 255) / 256), (unsigned)chunks);
   launch_k(lc, k_b2_part, dim3(grid), dim3(256), 0, n, L, ldz, P.z, from_bf16 ? P.dzb : nullptr, P.b2part);
-  launch_k(lc, k_b2_apply, dim3((unsigned)((L + 255) / 256)), dim3(256), 0, L, chunks, P.b2part, b2, lr, grad_b2);
+  launch_k(lc, k_b2_apply, dim3((unsigned)((L + 255) / 256)), dim3(256), 0, L, chunks, P.b2part, b2, P.meta, grad_b2);
   return cudaGetLastError();
 }
 

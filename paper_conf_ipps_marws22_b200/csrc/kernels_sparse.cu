@@ -120,9 +120,14 @@ __global__ void __launch_bounds__(1024) k_batch_scan(const int32_t* __restrict__
                                                      const int64_t* __restrict__ lab_ptr,
                                                      int64_t n_data_rows, int32_t* boff,
                                                      int32_t* loff, int32_t* meta, int64_t nz_cap,
-                                                     int64_t nl_cap, int64_t* rbase) {
+                                                     int64_t nl_cap, int64_t* rbase, int32_t* rowsc,
+                                                     float lr, float* loss_dev) {
   pdl_trigger();
   pdl_wait();
+  if (threadIdx.x == 0) {
+    meta[M_LR] = __float_as_int(lr);
+    *reinterpret_cast<float**>(meta + M_LOSS) = loss_dev;
+  }
   __shared__ long long wf[32], wl[32];
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
   const int per = (n + blockDim.x - 1) / blockDim.x;
@@ -161,6 +166,7 @@ __global__ void __launch_bounds__(1024) k_batch_scan(const int32_t* __restrict__
     boff[r] = (int32_t)min(pf, (long long)nz_cap);
     loff[r] = (int32_t)min(pl, (long long)nl_cap);
     int64_t id = rows[r];
+    rowsc[r] = (int32_t)id;
     rbase[r] = (id < 0 || id >= n_data_rows) ? 0 : row_ptr[id];
     if (id < 0 || id >= n_data_rows) continue;
     pf += row_ptr[id + 1] - row_ptr[id];
@@ -202,116 +208,6 @@ __device__ __forceinline__ void load_view(int32_t* sboff, const int32_t* boff, c
   for (int i = threadIdx.x; i <= n; i += blockDim.x) sboff[i] = boff[i];
   for (int i = threadIdx.x; i < n; i += blockDim.x) srb[i] = rbase[i];
   __syncthreads();
-}
-
-// K-0 (b): cnt[f] += 1 for every batch entry; CTA 0 also resets the scan's
-// tile-status words and tile ticket for k_fscan.
-__global__ void k_count(int n, const int64_t* __restrict__ rbase,
-                        const int32_t* __restrict__ col, const int32_t* __restrict__ boff,
-                        int32_t* meta, int32_t* cnt, unsigned long long* status, int ntiles) {
-  pdl_trigger();
-  pdl_wait();
-  extern __shared__ int32_t sboff[];
-  if (blockIdx.x == 0) {
-    for (int i = threadIdx.x; i < ntiles; i += blockDim.x) status[i] = 0ull;
-    if (threadIdx.x == 0) meta[M_TILE] = 0;
-  }
-  load_view(sboff, boff, rbase, n);
-  const int nnz = meta[M_NNZ];
-  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x) {
-    int r;
-    int64_t k = entry_index(sboff, n, e, &r);
-    atomicAdd(&cnt[col[k]], 1);
-  }
-}
-
-// K-0 (c): single-pass scan over F (decoupled look-back, tiles of kScanTile
-// features in ticket order).  Per touched feature f: fseg[f] = segment start,
-// fuid[f] = its rank u; uniq[u] = f and useg[u] = segment start (sorted by f).
-// Status word: flag (2 bits: 1 aggregate, 2 inclusive prefix) | count (31) | touched (31).
-constexpr unsigned long long kFlagAgg = 1ull << 62, kFlagPre = 2ull << 62;
-__device__ __forceinline__ unsigned long long pack_st(unsigned long long flag, int a, int b) {
-  return flag | ((unsigned long long)(unsigned)a << 31) | (unsigned long long)(unsigned)b;
-}
-
-__global__ void __launch_bounds__(256) k_fscan(const int32_t* __restrict__ cnt, int64_t F,
-                                               unsigned long long* status, int ntiles, int32_t* meta,
-                                               int32_t* fseg, int32_t* fuid, int32_t* uniq,
-                                               int32_t* useg) {
-  pdl_trigger();
-  pdl_wait();
-  constexpr int PER = kScanTile / 256;
-  __shared__ int s_tile, s_pa, s_pb;
-  __shared__ int wa[8], wb[8];
-  if (threadIdx.x == 0) s_tile = atomicAdd(&meta[M_TILE], 1);
-  __syncthreads();
-  const int t = s_tile;
-  const int64_t f0 = (int64_t)t * kScanTile + threadIdx.x * PER;
-  int c[PER];
-  int a = 0, b = 0;
-#pragma unroll
-  for (int i = 0; i < PER; ++i) {
-    c[i] = (f0 + i < F) ? cnt[f0 + i] : 0;
-    a += c[i];
-    b += (c[i] > 0);
-  }
-  // block exclusive scan of (a, b)
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  int xa = a, xb = b;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const int ya = __shfl_up_sync(kFull, xa, o), yb = __shfl_up_sync(kFull, xb, o);
-    if (lane >= o) { xa += ya; xb += yb; }
-  }
-  if (lane == 31) { wa[wid] = xa; wb[wid] = xb; }
-  __syncthreads();
-  int oa = 0, ob = 0, ta = 0, tb = 0;
-#pragma unroll
-  for (int w = 0; w < 8; ++w) {
-    if (w < wid) { oa += wa[w]; ob += wb[w]; }
-    ta += wa[w]; tb += wb[w];
-  }
-  if (threadIdx.x == 0) {
-    volatile unsigned long long* st = status;
-    if (t == 0) {
-      st[0] = pack_st(kFlagPre, ta, tb);
-      s_pa = 0; s_pb = 0;
-    } else {
-      st[t] = pack_st(kFlagAgg, ta, tb);
-      __threadfence();
-      int pa = 0, pb = 0;
-      for (int j = t - 1; j >= 0;) {
-        const unsigned long long v = st[j];
-        const unsigned long long flag = v & (3ull << 62);
-        if (!flag) continue;   // predecessor not published yet
-        pa += (int)((v >> 31) & 0x7fffffffull);
-        pb += (int)(v & 0x7fffffffull);
-        if (flag == kFlagPre) break;
-        --j;
-      }
-      __threadfence();
-      st[t] = pack_st(kFlagPre, pa + ta, pb + tb);
-      s_pa = pa; s_pb = pb;
-    }
-    if (t == ntiles - 1) {
-      meta[M_U] = s_pb + tb;
-      useg[s_pb + tb] = s_pa + ta;   // == batch nnz
-    }
-  }
-  __syncthreads();
-  int pa = s_pa + oa + (xa - a);   // exclusive prefix of this thread
-  int pb = s_pb + ob + (xb - b);
-#pragma unroll
-  for (int i = 0; i < PER; ++i) {
-    if (c[i] > 0) {
-      fseg[f0 + i] = pa;
-      fuid[f0 + i] = pb;
-      uniq[pb] = (int32_t)(f0 + i);
-      useg[pb] = pa;
-      ++pb;
-    }
-    pa += c[i];
-  }
 }
 
 // -------------------------------------------------------------------------
@@ -474,98 +370,12 @@ __global__ void __launch_bounds__(512) k_touched(int n, const int64_t* __restric
   }
 }
 
-// K-0 (e): scatter entries into their feature segment (cnt returns to zero)
-__global__ void k_place(int n, const int64_t* __restrict__ rbase,
-                        const int32_t* __restrict__ col, const float* __restrict__ val,
-                        const int32_t* __restrict__ boff, const int32_t* __restrict__ meta,
-                        int32_t* cnt, const int32_t* __restrict__ fseg,
-                        const int32_t* __restrict__ fuid, int32_t* e_n, float* e_v, int32_t* e_u,
-                        int32_t* e_f) {
-  pdl_trigger();
-  pdl_wait();
-  extern __shared__ int32_t sboff[];
-  load_view(sboff, boff, rbase, n);
-  const int nnz = meta[M_NNZ];
-  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x) {
-    int r;
-    int64_t k = entry_index(sboff, n, e, &r);
-    int f = col[k];
-    int pos = fseg[f] + atomicSub(&cnt[f], 1) - 1;
-    e_n[pos] = r;
-    e_v[pos] = val[k];
-    e_u[pos] = fuid[f];
-    e_f[pos] = f;
-  }
-}
-
-// K-0 (f): order every segment by batch row (deterministic summation order).
-// Row ids inside a segment are distinct (cols are unique within a row).
-__global__ void k_segsort(const int32_t* __restrict__ useg, const int32_t* __restrict__ meta,
-                          int32_t* e_n, float* e_v, int words) {
-  pdl_trigger();
-  pdl_wait();
-  extern __shared__ uint32_t sm[];
-  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  uint32_t* bm = sm + (size_t)wib * words * 33;
-  float* vb = reinterpret_cast<float*>(bm + words);
-  const int U = meta[M_U];
-  const int nw = gridDim.x * (blockDim.x >> 5);
-  for (int w = lane; w < words; w += 32) bm[w] = 0;
-  __syncwarp();
-  for (int u = blockIdx.x * (blockDim.x >> 5) + wib; u < U; u += nw) {
-    const int s = useg[u], m = useg[u + 1] - s;
-    if (m <= 1) continue;
-    if (m <= 32) {
-      int myn = lane < m ? e_n[s + lane] : 0x7fffffff;
-      float myv = lane < m ? e_v[s + lane] : 0.f;
-      int rank = 0;
-#pragma unroll
-      for (int j = 0; j < 32; ++j) rank += (__shfl_sync(kFull, myn, j) < myn);
-      __syncwarp();
-      if (lane < m) { e_n[s + rank] = myn; e_v[s + rank] = myv; }
-      __syncwarp();
-    } else {
-      for (int i = lane; i < m; i += 32) {
-        int r = e_n[s + i];
-        vb[r] = e_v[s + i];
-        atomicOr(&bm[r >> 5], 1u << (r & 31));
-      }
-      __syncwarp();
-      // words per lane
-      const int wpl = (words + 31) / 32;
-      const int w0 = lane * wpl;
-      int cntl = 0;
-      for (int j = 0; j < wpl; ++j) if (w0 + j < words) cntl += __popc(bm[w0 + j]);
-      int incl = cntl;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        int y = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl += y;
-      }
-      int pos = s + incl - cntl;
-      for (int j = 0; j < wpl; ++j) {
-        if (w0 + j >= words) break;
-        uint32_t bits = bm[w0 + j];
-        while (bits) {
-          int b = __ffs(bits) - 1;
-          bits &= bits - 1;
-          int r = (w0 + j) * 32 + b;
-          e_n[pos] = r;
-          e_v[pos] = vb[r];
-          ++pos;
-        }
-        bm[w0 + j] = 0;
-      }
-      __syncwarp();
-    }
-  }
-}
-
 // -------------------------------------------------------------------------
 // K-1: A1 = X W1 + b1, H1 = ReLU(A1)
 // -------------------------------------------------------------------------
 template <int VPL>
-__global__ void __launch_bounds__(256) k_spmm_fwd(int n, const int64_t* __restrict__ rbase,
+// (256, 2): two CTAs per SM, all kU gathers of a group in flight (<= 128 regs)
+__global__ void __launch_bounds__(256, 2) k_spmm_fwd(int n, const int64_t* __restrict__ rbase,
                                                   const int32_t* __restrict__ col,
                                                   const float* __restrict__ val,
                                                   const float* __restrict__ W1,
@@ -588,77 +398,94 @@ __global__ void __launch_bounds__(256) k_spmm_fwd(int n, const int64_t* __restri
   float bias[VPL];
   IO::load_ldg(b1, lane, bias);
 
-  for (int p = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); p < npieces; p += nwarps) {
-    const int e0 = p * kPiece, e1 = min(e0 + kPiece, nnz);
-    int r = entry_row(sboff, n, e0);
-    int e = e0;
-    while (e < e1) {
-      const int rs = sboff[r], re = sboff[r + 1];
-      const int se = min(re, e1);
-      float acc[VPL];
+  // Row segment [.., ..) of row r ends inside this piece: finish it (ReLU(acc + b1))
+  // when the piece holds the whole row, else publish a partial; the last of the
+  // row's pieces to arrive sums the partials in piece order and finishes.
+  auto flush = [&](int p, int e0, int e1, int r, float (&acc)[VPL]) {
+    const int rs = sboff[r], re = sboff[r + 1];
+    const bool before = rs < e0, after = re > e1;
+    if (before || after) {
+      IO::store_cg(part + (int64_t)(before ? 2 * p : 2 * p + 1) * H, lane, acc);
+      __threadfence();
+      int old = 0;
+      if (lane == 0) old = atomicAdd(&rowcnt[r], 1);
+      old = __shfl_sync(kFull, old, 0);
+      const int q0 = rs / kPiece, q1 = (re - 1) / kPiece;
+      if (old != q1 - q0) return;
+      __threadfence();
 #pragma unroll
       for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
-      const int64_t base = srb[r] - rs;   // dataset index of flat entry e: base + e
-      const int cnt = se - e;                        // <= kPiece = 32
-      int mycol = 0;
-      float myval = 0.f;
-      if (lane < cnt) { mycol = __ldg(col + base + e + lane); myval = __ldg(val + base + e + lane); }
-      int j = 0;
-      for (; j + kU <= cnt; j += kU) {
-        float w[kU][VPL];
+      for (int q = q0; q <= q1; q += 4) {   // 4 partials in flight, summed in piece order
+        float t[4][VPL];
 #pragma unroll
-        for (int q = 0; q < kU; ++q) {
-          int c = __shfl_sync(kFull, mycol, j + q);
-          IO::load_ldg(W1 + (int64_t)c * H, lane, w[q]);
+        for (int u = 0; u < 4; ++u) {
+          if (q + u <= q1) IO::load_cg(part + (int64_t)(q + u == q0 ? 2 * q0 + 1 : 2 * (q + u)) * H, lane, t[u]);
+          else {
+#pragma unroll
+            for (int i = 0; i < VPL; ++i) t[u][i] = 0.f;
+          }
         }
 #pragma unroll
-        for (int q = 0; q < kU; ++q) {
-          float v = __shfl_sync(kFull, myval, j + q);
+        for (int u = 0; u < 4; ++u) {
+          if (q + u <= q1) {
+#pragma unroll
+            for (int i = 0; i < VPL; ++i) acc[i] += t[u][i];
+          }
+        }
+      }
+      if (lane == 0) rowcnt[r] = 0;
+    }
+#pragma unroll
+    for (int i = 0; i < VPL; ++i) acc[i] = fmaxf(acc[i] + bias[i], 0.f);
+    IO::store(H1 + (int64_t)r * H, lane, acc);
+    if (H1b) IO::store_bf16(H1b + (int64_t)r * H, lane, acc);
+  };
+
+  for (int p = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); p < npieces; p += nwarps) {
+    const int e0 = p * kPiece, e1 = min(e0 + kPiece, nnz), cnt = e1 - e0;
+    // lane j holds entry e0 + j: its row, column and value (one round trip)
+    int myr = 0, mycol = 0;
+    float myval = 0.f;
+    if (lane < cnt) {
+      myr = entry_row(sboff, n, e0 + lane);
+      const int64_t k = srb[myr] + (e0 + lane - sboff[myr]);
+      mycol = __ldg(col + k);
+      myval = __ldg(val + k);
+    }
+    int rcur = __shfl_sync(kFull, myr, 0);
+    float acc[VPL];
+#pragma unroll
+    for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+    // groups of kU W1 rows in flight, row changes handled between FMAs
+    for (int j0 = 0; j0 < cnt; j0 += kU) {
+      float w[kU][VPL];
+#pragma unroll
+      for (int q = 0; q < kU; ++q) {
+        const int c = __shfl_sync(kFull, mycol, j0 + q);
+        if (j0 + q < cnt) IO::load_ldg(W1 + (int64_t)c * H, lane, w[q]);
+        else {
+#pragma unroll
+          for (int i = 0; i < VPL; ++i) w[q][i] = 0.f;
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < kU; ++q) {
+        const int j = j0 + q;
+        const int rq = __shfl_sync(kFull, myr, j);
+        const float v = __shfl_sync(kFull, myval, j);
+        if (j < cnt) {
+          if (rq != rcur) {
+            flush(p, e0, e1, rcur, acc);
+#pragma unroll
+            for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+            rcur = rq;
+          }
 #pragma unroll
           for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, w[q][i], acc[i]);
         }
       }
-      for (; j < cnt; ++j) {
-        int c = __shfl_sync(kFull, mycol, j);
-        float v = __shfl_sync(kFull, myval, j);
-        float w[VPL];
-        IO::load_ldg(W1 + (int64_t)c * H, lane, w);
-#pragma unroll
-        for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, w[i], acc[i]);
-      }
-      const bool before = rs < e0, after = re > e1;
-      bool finish = !before && !after;
-      if (!finish) {
-        const int slot = before ? 2 * p : 2 * p + 1;
-        IO::store_cg(part + (int64_t)slot * H, lane, acc);
-        __threadfence();
-        int old = 0;
-        if (lane == 0) old = atomicAdd(&rowcnt[r], 1);
-        old = __shfl_sync(kFull, old, 0);
-        const int q0 = rs / kPiece, q1 = (re - 1) / kPiece;
-        if (old == q1 - q0) {
-          __threadfence();
-#pragma unroll
-          for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
-          for (int q = q0; q <= q1; ++q) {
-            float t[VPL];
-            IO::load_cg(part + (int64_t)(q == q0 ? 2 * q + 1 : 2 * q) * H, lane, t);
-#pragma unroll
-            for (int i = 0; i < VPL; ++i) acc[i] += t[i];
-          }
-          if (lane == 0) rowcnt[r] = 0;
-          finish = true;
-        }
-      }
-      if (finish) {
-#pragma unroll
-        for (int i = 0; i < VPL; ++i) acc[i] = fmaxf(acc[i] + bias[i], 0.f);
-        IO::store(H1 + (int64_t)r * H, lane, acc);
-        if (H1b) IO::store_bf16(H1b + (int64_t)r * H, lane, acc);
-      }
-      e = se;
-      ++r;
     }
+    if (cnt > 0) flush(p, e0, e1, rcur, acc);
   }
   // rows without entries: H1 = ReLU(b1)
   const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
@@ -684,10 +511,11 @@ __global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__
                                                      const int32_t* __restrict__ uniq,
                                                      const int32_t* __restrict__ meta,
                                                      const float* __restrict__ dA1, float* W1,
-                                                     float lr, float* part, int32_t* ucnt,
+                                                     float* part, int32_t* ucnt,
                                                      float* grad_w1) {
   pdl_trigger();
   pdl_wait();
+  const float lr = step_lr(meta);
   using IO = RowIO<VPL>;
   constexpr int H = 32 * VPL;
   constexpr int kU = VPL >= 16 ? 4 : 8;   // dA1 rows in flight per warp
@@ -844,10 +672,11 @@ __global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restr
                                                           const int32_t* __restrict__ useg,
                                                           const int32_t* __restrict__ meta,
                                                           const T* __restrict__ dA1, int H, float* W1,
-                                                          float lr, float* part, int32_t* ucnt,
+                                                          float* part, int32_t* ucnt,
                                                           float* grad_w1) {
   pdl_trigger();
   pdl_wait();
+  const float lr = step_lr(meta);
   constexpr int CS = 32 * CPL;               // columns of this CTA's slice
   constexpr int kU = 8;
   extern __shared__ __align__(16) uint8_t sm_raw[];
@@ -937,11 +766,24 @@ __global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restr
           ld_cols<CPL>(wrow, w, false);
 #pragma unroll
           for (int i = 0; i < CPL; ++i) acc[i] = 0.f;
-          for (int q = q0; q <= q1; ++q) {
-            float t[CPL];
-            ld_cols<CPL>(part + (int64_t)(q == q0 ? 2 * q + 1 : 2 * q) * H + c0 + lane * CPL, t, true);
+          for (int q = q0; q <= q1; q += 4) {   // 4 partials in flight, summed in piece order
+            float t[4][CPL];
 #pragma unroll
-            for (int i = 0; i < CPL; ++i) acc[i] += t[i];
+            for (int u = 0; u < 4; ++u) {
+              if (q + u <= q1)
+                ld_cols<CPL>(part + (int64_t)(q + u == q0 ? 2 * q0 + 1 : 2 * (q + u)) * H + c0 + lane * CPL, t[u], true);
+              else {
+#pragma unroll
+                for (int i = 0; i < CPL; ++i) t[u][i] = 0.f;
+              }
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+              if (q + u <= q1) {
+#pragma unroll
+                for (int i = 0; i < CPL; ++i) acc[i] += t[u][i];
+              }
+            }
           }
           if (lane == 0) ucnt[(int64_t)u * nsl + slice] = 0;
           finish = true;
@@ -980,12 +822,12 @@ cudaError_t spmm_fwd_t(const Launch& lc, const int32_t* rows, int n, const int64
 }
 
 template <int VPL>
-cudaError_t scatter_t(const Launch& lc, float* W1, float lr, const Ptrs& P, const WsLayout& L,
+cudaError_t scatter_t(const Launch& lc, float* W1, const Ptrs& P, const WsLayout& L,
                       float* grad_w1) {
   static int occ = 0;
   const int grid = wave_grid(lc, k_scatter_sgd<VPL>, 0, L.n_pieces, occ);
   launch_k(lc, k_scatter_sgd<VPL>, dim3(grid), dim3(256), 0, P.e_n, P.e_v, P.e_u, P.useg, P.uniq, P.meta, P.da1,
-                                             W1, lr, P.part5, P.ucnt, grad_w1);
+                                             W1, P.part5, P.ucnt, grad_w1);
   return cudaGetLastError();
 }
 
@@ -993,9 +835,9 @@ cudaError_t scatter_t(const Launch& lc, float* W1, float lr, const Ptrs& P, cons
 
 cudaError_t launch_batch_scan(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
                               const int64_t* lab_ptr, int64_t n_data_rows, const Ptrs& P,
-                              int64_t nz_cap, int64_t nl_cap) {
+                              int64_t nz_cap, int64_t nl_cap, float lr, float* loss_dev) {
   launch_k(lc, k_batch_scan, dim3(1), dim3(1024), 0, rows, n, row_ptr, lab_ptr, n_data_rows, P.boff, P.loff, P.meta,
-                                     nz_cap, nl_cap, P.rbase);
+                                     nz_cap, nl_cap, P.rbase, P.rowsc, lr, loss_dev);
   return cudaGetLastError();
 }
 
@@ -1023,7 +865,7 @@ cudaError_t launch_spmm_fwd(const Launch& lc, const int32_t* rows, int n, const 
 }
 
 template <typename T, int CPL>
-cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float* W1, float lr,
+cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float* W1,
                         const Ptrs& P, float* grad_w1) {
   constexpr int CS = 32 * CPL;
   const int nsl = H / CS;
@@ -1037,7 +879,7 @@ cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float*
   }
   const int gx = std::max(1, lc.sms / nsl);
   return launch_k(lc, k_scatter_sgd_s<T, CPL>, dim3(gx, nsl), dim3(512), smem, P.e_n, P.e_v, P.e_u,
-                  P.e_f, P.useg, P.meta, dA1, H, W1, lr, P.part5, P.ucnt, grad_w1);
+                  P.e_f, P.useg, P.meta, dA1, H, W1, P.part5, P.ucnt, grad_w1);
 }
 
 // Widest column slice whose staged dA1 fits 160 KB of shared memory (0 = none).
@@ -1047,25 +889,25 @@ int scatter_slice(int H, int b_max, size_t elem) {
   return 0;
 }
 
-cudaError_t launch_scatter_sgd(const Launch& lc, float* W1, int H, float lr, const Ptrs& P,
+cudaError_t launch_scatter_sgd(const Launch& lc, float* W1, int H, const Ptrs& P,
                                const WsLayout& L, float* grad_w1, const bf16* dA1b, int b_max) {
   const size_t elem = dA1b ? 2 : 4;
   const int cs = scatter_slice(H, b_max, elem);
   if (cs) {
     if (dA1b) {
-      if (cs == 256) return scatter_s_t<bf16, 8>(lc, dA1b, H, b_max, W1, lr, P, grad_w1);
-      if (cs == 128) return scatter_s_t<bf16, 4>(lc, dA1b, H, b_max, W1, lr, P, grad_w1);
-      return scatter_s_t<bf16, 2>(lc, dA1b, H, b_max, W1, lr, P, grad_w1);
+      if (cs == 256) return scatter_s_t<bf16, 8>(lc, dA1b, H, b_max, W1, P, grad_w1);
+      if (cs == 128) return scatter_s_t<bf16, 4>(lc, dA1b, H, b_max, W1, P, grad_w1);
+      return scatter_s_t<bf16, 2>(lc, dA1b, H, b_max, W1, P, grad_w1);
     }
-    if (cs == 256) return scatter_s_t<float, 8>(lc, P.da1, H, b_max, W1, lr, P, grad_w1);
-    if (cs == 128) return scatter_s_t<float, 4>(lc, P.da1, H, b_max, W1, lr, P, grad_w1);
-    return scatter_s_t<float, 2>(lc, P.da1, H, b_max, W1, lr, P, grad_w1);
+    if (cs == 256) return scatter_s_t<float, 8>(lc, P.da1, H, b_max, W1, P, grad_w1);
+    if (cs == 128) return scatter_s_t<float, 4>(lc, P.da1, H, b_max, W1, P, grad_w1);
+    return scatter_s_t<float, 2>(lc, P.da1, H, b_max, W1, P, grad_w1);
   }
   switch (H) {
-    case 64: return scatter_t<2>(lc, W1, lr, P, L, grad_w1);
-    case 128: return scatter_t<4>(lc, W1, lr, P, L, grad_w1);
-    case 256: return scatter_t<8>(lc, W1, lr, P, L, grad_w1);
-    case 512: return scatter_t<16>(lc, W1, lr, P, L, grad_w1);
+    case 64: return scatter_t<2>(lc, W1, P, L, grad_w1);
+    case 128: return scatter_t<4>(lc, W1, P, L, grad_w1);
+    case 256: return scatter_t<8>(lc, W1, P, L, grad_w1);
+    case 512: return scatter_t<16>(lc, W1, P, L, grad_w1);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -30,7 +30,7 @@ struct TcArgs {
   float* out; int64_t ldo;            // Z (ldo = Lp) / partials (ldo = H) / W2 (ldo = H)
   int64_t part_stride;                // split-K partial z offset
   const float* bias;                  // G1
-  float lr; bf16* shadow; float* grad;// G3
+  const int32_t* meta; bf16* shadow; float* grad;// G3 (lr = meta[M_LR])
   float* b2; float* grad_b2;          // G3: db2 = dZ^T 1 via an extra N = 16 MMA on N-tile 0
   float2* stats; int64_t stats_ld;    // G1: per (N-tile half, row) softmax partials (max, sum exp)
   int splits;                         // split-K factor (tiles = M tiles x N tiles x splits)
@@ -300,6 +300,7 @@ __global__ void __launch_bounds__(384, 1)
   } else if (warp >= 4) {
     // ------------------------------------------------ epilogue (8 warps)
     const int wq = (warp - 4) & 3, wh = (warp - 4) >> 2;
+    const float lr = EPI == TC_EPI_SGD ? step_lr(g.meta) : 0.f;
     int tl = 0, sbuf = 0, kc = 0;
     for (int t = blockIdx.x; t < T; t += gridDim.x, ++tl) {
       int mt, nt, z, kb0, nk;
@@ -453,7 +454,7 @@ __global__ void __launch_bounds__(384, 1)
           for (int q = 0; q < 8; ++q) {
             float4* p = reinterpret_cast<float4*>(wb + lane * 128 + ((q ^ (lane & 7)) * 16));
             float4 x = *p;
-            x.x -= g.lr * v[4 * q]; x.y -= g.lr * v[4 * q + 1]; x.z -= g.lr * v[4 * q + 2]; x.w -= g.lr * v[4 * q + 3];
+            x.x -= lr * v[4 * q]; x.y -= lr * v[4 * q + 1]; x.z -= lr * v[4 * q + 2]; x.w -= lr * v[4 * q + 3];
             *p = x;
             __nv_bfloat162 p0 = __floats2bfloat162_rn(x.x, x.y), p1 = __floats2bfloat162_rn(x.z, x.w);
             uint2 pk;
@@ -490,7 +491,7 @@ __global__ void __launch_bounds__(384, 1)
             v[0] = 0.f;
           }
           if (m < g.M) {
-            g.b2[m] -= g.lr * v[0];
+            g.b2[m] -= lr * v[0];
             if (g.grad_b2) g.grad_b2[m] = v[0];
           }
         }
@@ -596,7 +597,7 @@ bool tc_available() {
 
 int64_t padded_ld(int64_t L) { return (L + 7) / 8 * 8; }
 
-cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H, float lr, const Ptrs& P,
+cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H, const Ptrs& P,
                            const WsLayout& W, float* W2, float* b2, float* grad_w2, float* grad_b2,
                            float2* stats, int* stats_ntiles, const int32_t* dz_rows,
                            const int64_t* dz_lab_ptr, const int32_t* dz_lab) {
@@ -648,7 +649,7 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
   }
   // which == 3: W2 -= lr dZ^T H1
   g.M = (int)L; g.N = H; g.K = n;
-  g.out = W2; g.ldo = H; g.lr = lr; g.shadow = P.w2b; g.grad = grad_w2;
+  g.out = W2; g.ldo = H; g.meta = P.meta; g.shadow = P.w2b; g.grad = grad_w2;
   g.b2 = b2; g.grad_b2 = grad_b2;
   if ((e = make_map(&ta, P.dzb, L, n, (uint64_t)Lp * 2, 64, 64)) != cudaSuccess) return e;
   if ((e = make_map(&tb, P.h1b, H, n, (uint64_t)H * 2, 64, 64)) != cudaSuccess) return e;

@@ -109,8 +109,11 @@ class DistributedAdaptiveSGD:
     """Rank `rank` of `world` (one GPU each)."""
 
     def __init__(self, replica: api.Replica, hyper: Hyper, rank: int, world: int,
-                 sched: api.Scheduler, group=None, inflight: int = 2):
+                 sched: api.Scheduler, group=None, inflight: int = 2, native: bool = True):
+        """native: run the ticket loop in libasgd (asgd_run_tickets); False keeps
+        the Python loop of run_tickets (same routing semantics)."""
         self.rep, self.h, self.rank, self.world = replica, hyper, rank, world
+        self.native = native
         self.sched, self.group, self.inflight = sched, group, inflight
         self.b = [hyper.b_max] * world            # P:1565-1566: initial b = b_max
         self.lr = [hyper.lr_max] * world
@@ -127,12 +130,15 @@ class DistributedAdaptiveSGD:
         self.sched.wait(self.mb)
         b_i, lr_i = self.b[r], self.lr[r]
 
-        def step(k, start, n):
-            rep.step(stream_rows[start:start + n], lr_i, self.losses[k:k + 1])
-            self.events[k].record(rep.stream)
+        if self.native:
+            n_steps = rep.run_tickets(self.sched, r, b_i, stream_rows, lr_i, self.losses, self.inflight)
+        else:
+            def step(k, start, n):
+                rep.step(stream_rows[start:start + n], lr_i, self.losses[k:k + 1])
+                self.events[k].record(rep.stream)
 
-        n_steps = run_tickets(self.sched, r, b_i, step, self.inflight,
-                              wait=lambda k: self.events[k].synchronize())
+            n_steps = run_tickets(self.sched, r, b_i, step, self.inflight,
+                                  wait=lambda k: self.events[k].synchronize())
         # ---- merge (Alg. 2) -------------------------------------------------
         rep.sqnorm(self.sq)
         us, bs, nu = exchange_stats(n_steps, b_i, self.sq, rep.P, self.world, self.group)

@@ -1,0 +1,9 @@
+timeout 900 python -m pytest tests/test_gpu_step.py tests/test_gpu_merge.py tests/test_gpu_large.py -x -q 2>&1 | grep -E "^E |FAILED|passed|failed" | head -10
+timeout 300 python bench.py --steps 20 --warmup 3 --no-cpu-baseline --ttp-megabatches 0 --e2e-steps 0 2>/dev/null | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); print('eurlex', d['value'], d['ms_per_step'], d['roofline']['whole_step_frac'], {k:v['us_per_launch'] for k,v in d['kernels_warmup_profile'].items()})"
+timeout 600 python bench.py --config wiki10_31k --steps 5 --warmup 3 --no-cpu-baseline --ttp-megabatches 0 --e2e-steps 0 2>/dev/null | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); print('wiki10', d['value'], d['ms_per_step'], {k:v['us_per_launch'] for k,v in d['kernels_warmup_profile'].items()})"
+mkdir -p gpurun_out
+A="--steps 1 --warmup 3 --no-cpu-baseline --ttp-megabatches 0 --e2e-steps 0"
+timeout 900 ncu --metrics gpu__time_duration.sum --cache-control none --clock-control none -k regex:"k_" -s 600 -c 300 --csv \
+  --log-file gpurun_out/launches_eurlex_warm.csv python bench.py $A > /dev/null 2>&1; echo l1 $?
