@@ -96,7 +96,7 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.fuid = take(F * 4);
   L.uniq = take((L.u_cap + 1) * 4);
   L.useg = take((L.u_cap + 1) * 4);
-  L.tsum = take(L.n_tiles_f * 8);
+  L.tsum = take(L.n_tiles_f * 16);   // K-0 tile (count, touched) sums, double-buffered
   L.tpre = take(L.n_tiles_f * 8);
   L.e_n = take(L.nz_cap * 4);
   L.e_v = take(L.nz_cap * 4);
@@ -106,7 +106,7 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.rowcnt = take(B * 4);
   L.part5 = take((size_t)2 * L.n_pieces * H * 4);
   L.ucnt = take((L.u_cap + 1) * 4 * 8);   // per (segment, column slice)
-  L.bits = take((size_t)L.u_cap * ((B + 31) / 32) * 4);   // K-0 row bitmaps per touched feature
+  L.bits = take((size_t)F * ((B + 31) / 32) * 4);   // K-0 row bitmap per feature (zero between steps)
   L.h1 = take(B * H * 4);
   L.h1b = take(bf ? B * H * 2 : 0);
   L.z = take((size_t)B * Lp * 4);
@@ -513,7 +513,11 @@ int enqueue_step(asgd_ctx* c, int n) {
     Ptrs Pr = P, Pw = P;
     Pr.w2b = c->w2b_buf[c->w2b_cur];
     Pw.w2b = c->w2b_buf[c->w2b_cur ^ 1];
+    // G3 (s3) runs beside G2 (s): both need ~200 KB of smem per CTA, so G3's
+    // persistent grid leaves G2's CTAs their own SMs when G2 is small
     Launch lc3 = c->lc3();
+    const int g2c = gemm_tc_g2_ctas(n, H, c->L, c->sms);
+    if (2 * g2c <= c->sms) lc3.sms = c->sms - g2c;
     float2* zstat = reinterpret_cast<float2*>(c->ws + c->L.zstat);
     int ntiles = 0;
     if ((int64_t)m.b_max * Lb * 4 <= kFusedCeBytes) {

@@ -19,8 +19,9 @@ constexpr int kScanTile = 1024;
 // step's mean loss goes to (slots 10-11), both written by K-0 (a) so that the
 // rest of the step (and its CUDA graph) takes no per-step scalar arguments;
 // M_BAR: 64-bit grid-barrier counter (slots 32-33).
-enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_LR = 6, M_COUNT = 8, M_LOSS = 10,
-       M_BAR = 32 };
+// M_K0PAR: parity of K-0's double-buffered tile sums.
+enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_LR = 6, M_K0PAR = 7, M_COUNT = 8,
+       M_LOSS = 10, M_BAR = 32 };
 // error bits in meta[M_ERR]
 enum { ERR_NNZ_CAP = 1, ERR_LAB_CAP = 2, ERR_ROW_ID = 4 };
 
@@ -146,6 +147,8 @@ cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int 
                            float* grad_b2, float2* stats = nullptr, int* stats_ntiles = nullptr,
                            const int32_t* dz_rows = nullptr, const int64_t* dz_lab_ptr = nullptr,
                            const int32_t* dz_lab = nullptr);
+// CTAs G2 runs with (the concurrent G3 leaves those SMs to it).
+int gemm_tc_g2_ctas(int n, int H, const WsLayout&, int sms);
 // which = 4 (G1b): dZ = (softmax - T)/B from a recomputed Z tile; needs P.lse from k_lse.
 // which = 5: G1 without storing Z (only the softmax partials), for the fused path.
 cudaError_t launch_lse(const Launch&, int n, int H, int ntiles, int64_t stats_ld, const float2* stats,

@@ -11,6 +11,7 @@
 // combined by the last-arriving warp in piece order, so every sum has a
 // fixed order: results are bitwise deterministic.
 #include <algorithm>
+#include <cstdlib>
 
 #include "asgd_internal.h"
 
@@ -211,19 +212,22 @@ __device__ __forceinline__ void load_view(int32_t* sboff, const int32_t* boff, c
 }
 
 // -------------------------------------------------------------------------
-// K-0 (b-e) fused: one persistent kernel of kTouchCtas co-operating CTAs with
-// software grid barriers (the only other work on the GPU is the dense chain on
-// other streams, which never waits for this kernel, so every CTA eventually
-// runs).  Phases:
-//   A  cnt[f] += 1 per batch entry
-//   B  tile sums of (cnt, [cnt > 0]) over F;  C  prefix + segment starts fseg,
-//      ranks fuid, sorted unique ids uniq, segment offsets useg
-//   D  row bitmap of every touched feature: bits[u][r / 32] |= 1 << r % 32
+// K-0 (b-e) fused: one persistent kernel of co-operating CTAs (one per SM at
+// most) with two software grid barriers (the only other work on the GPU is the
+// dense chain on other streams, which never waits for this kernel, so every CTA
+// eventually runs).  Phases:
+//   A  per batch entry (row r, feature f): cnt[f] += 1 and the row bitmap
+//      bits[f][r / 32] |= 1 << r % 32; per-tile (count, touched) histograms in
+//      shared memory, flushed to tsum[par] once per CTA
+//   C  tile prefix + in-tile scan: segment starts fseg, ranks fuid, sorted
+//      unique ids uniq, segment offsets useg; tsum[par ^ 1] zeroed for the next step
 //   E  deterministic placement: the entry of row r in feature f's segment goes
-//      to fseg[f] + #{rows r' < r of the batch containing f} (popcounts), so
-//      every segment is sorted by row without a sort
-//   F  cnt and bitmaps back to zero for the next step
+//      to fseg[f] + #{rows r' < r of the batch containing f} (popcounts of
+//      bits[f]), so every segment is sorted by row without a sort
+// cnt[f] and bits[f][*] go back to zero in K-5, which finishes each segment.
 // -------------------------------------------------------------------------
+// 64 CTAs: enough entries in flight, while leaving the register file of most
+// SMs to K-1, which runs beside K-0 (measured: 148 CTAs slow K-1 by ~3 us).
 constexpr int kTouchCtas = 64;
 
 __device__ __forceinline__ void grid_barrier(unsigned long long* ctr) {
@@ -233,7 +237,7 @@ __device__ __forceinline__ void grid_barrier(unsigned long long* ctr) {
     const unsigned long long arrive = atomicAdd(ctr, 1ull) + 1ull;
     const unsigned long long goal = (arrive + gridDim.x - 1) / gridDim.x * gridDim.x;
     volatile unsigned long long* vc = ctr;
-    while (*vc < goal) __nanosleep(64);
+    while (*vc < goal) __nanosleep(32);
     __threadfence();
   }
   __syncthreads();
@@ -253,6 +257,11 @@ __global__ void __launch_bounds__(512) k_touched(int n, const int64_t* __restric
   __shared__ int s_red[2][16];
   __shared__ int s_pre[2];
   unsigned long long* bar = reinterpret_cast<unsigned long long*>(meta + M_BAR);
+  const int par = meta[M_K0PAR] & 1;
+  int32_t* ts = tsum + (size_t)par * 2 * ntiles;          // this step's tile (count, touched) sums
+  int32_t* ts_next = tsum + (size_t)(par ^ 1) * 2 * ntiles;
+  int32_t* hist = sboff + ((view_smem(n) + 3) / 4);       // [ntiles][2] after the batch view
+  for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x) hist[i] = 0;
   load_view(sboff, boff, rbase, n);
   const int nnz = meta[M_NNZ];
   const int gt = blockIdx.x * blockDim.x + threadIdx.x, gs = gridDim.x * blockDim.x;
@@ -260,35 +269,22 @@ __global__ void __launch_bounds__(512) k_touched(int n, const int64_t* __restric
   // ---- A
   for (int e = gt; e < nnz; e += gs) {
     int r;
-    atomicAdd(&cnt[col[entry_index(sboff, n, e, &r)]], 1);
+    const int f = col[entry_index(sboff, n, e, &r)];
+    const int old = atomicAdd(&cnt[f], 1);
+    atomicOr(&bits[(int64_t)f * W + (r >> 5)], 1u << (r & 31));
+    const int t = f / kScanTile;
+    atomicAdd(&hist[2 * t], 1);
+    if (old == 0) atomicAdd(&hist[2 * t + 1], 1);
   }
-  grid_barrier(bar);
-  // ---- B: tile sums (kScanTile features per tile, 2 per thread at 512 threads)
-  constexpr int PER = kScanTile / 512;
-  for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
-    const int64_t f0 = (int64_t)t * kScanTile + threadIdx.x * PER;
-    int a = 0, b = 0;
-#pragma unroll
-    for (int i = 0; i < PER; ++i) {
-      const int c = (f0 + i < F) ? cnt[f0 + i] : 0;
-      a += c; b += (c > 0);
-    }
-#pragma unroll
-    for (int o = 16; o; o >>= 1) { a += __shfl_xor_sync(kFull, a, o); b += __shfl_xor_sync(kFull, b, o); }
-    if (lane == 0) { s_red[0][wid] = a; s_red[1][wid] = b; }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      int x = 0, y = 0;
-      for (int w = 0; w < nw; ++w) { x += s_red[0][w]; y += s_red[1][w]; }
-      tsum[2 * t] = x; tsum[2 * t + 1] = y;
-    }
-    __syncthreads();
-  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x)
+    if (hist[i]) atomicAdd(&ts[i], hist[i]);
   grid_barrier(bar);
   // ---- C: prefix of the earlier tiles + in-tile scan
+  constexpr int PER = kScanTile / 512;
   for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
     int a = 0, b = 0;
-    for (int j = threadIdx.x; j < t; j += blockDim.x) { a += tsum[2 * j]; b += tsum[2 * j + 1]; }
+    for (int j = threadIdx.x; j < t; j += blockDim.x) { a += ts[2 * j]; b += ts[2 * j + 1]; }
 #pragma unroll
     for (int o = 16; o; o >>= 1) { a += __shfl_xor_sync(kFull, a, o); b += __shfl_xor_sync(kFull, b, o); }
     if (lane == 0) { s_red[0][wid] = a; s_red[1][wid] = b; }
@@ -298,9 +294,11 @@ __global__ void __launch_bounds__(512) k_touched(int n, const int64_t* __restric
       for (int w = 0; w < nw; ++w) { x += s_red[0][w]; y += s_red[1][w]; }
       s_pre[0] = x; s_pre[1] = y;
       if (t == ntiles - 1) {
-        meta[M_U] = y + tsum[2 * t + 1];
-        useg[y + tsum[2 * t + 1]] = x + tsum[2 * t];
+        meta[M_U] = y + ts[2 * t + 1];
+        useg[y + ts[2 * t + 1]] = x + ts[2 * t];
       }
+      ts_next[2 * t] = 0;
+      ts_next[2 * t + 1] = 0;
     }
     __syncthreads();
     const int64_t f0 = (int64_t)t * kScanTile + threadIdx.x * PER;
@@ -338,36 +336,21 @@ __global__ void __launch_bounds__(512) k_touched(int n, const int64_t* __restric
     __syncthreads();
   }
   grid_barrier(bar);
-  // ---- D: row bitmaps
-  for (int e = gt; e < nnz; e += gs) {
-    int r;
-    const int f = col[entry_index(sboff, n, e, &r)];
-    atomicOr(&bits[(int64_t)fuid[f] * W + (r >> 5)], 1u << (r & 31));
-  }
-  grid_barrier(bar);
   // ---- E: placement
   for (int e = gt; e < nnz; e += gs) {
     int r;
     const int64_t k = entry_index(sboff, n, e, &r);
     const int f = col[k];
-    const int u = fuid[f];
-    const uint32_t* bw = bits + (int64_t)u * W;
+    const uint32_t* bw = bits + (int64_t)f * W;
     int rank = __popc(bw[r >> 5] & ((1u << (r & 31)) - 1u));
     for (int w = 0; w < (r >> 5); ++w) rank += __popc(bw[w]);
     const int pos = fseg[f] + rank;
     e_n[pos] = r;
     e_v[pos] = val[k];
-    e_u[pos] = u;
+    e_u[pos] = fuid[f];
     e_f[pos] = f;
   }
-  grid_barrier(bar);
-  // ---- F: reset for the next step
-  for (int e = gt; e < nnz; e += gs) {
-    int r;
-    const int f = col[entry_index(sboff, n, e, &r)];
-    cnt[f] = 0;
-    bits[(int64_t)fuid[f] * W + (r >> 5)] = 0u;
-  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) meta[M_K0PAR] = par ^ 1;   // every CTA read par before barrier 1
 }
 
 // -------------------------------------------------------------------------
@@ -500,6 +483,13 @@ __global__ void __launch_bounds__(256, 2) k_spmm_fwd(int n, const int64_t* __res
   }
 }
 
+// K-0's per-feature count and row bitmap back to zero (the warp that finishes
+// feature f's segment; K-0 of the next step starts from zeros).
+__device__ __forceinline__ void reset_feature(int32_t* cnt, uint32_t* bits, int W, int f, int lane) {
+  if (lane == 0) cnt[f] = 0;
+  for (int w = lane; w < W; w += 32) bits[(int64_t)f * W + w] = 0u;
+}
+
 // -------------------------------------------------------------------------
 // K-5: W1[f,:] -= lr * sum_{entries of f, ascending row} v * dA1[row,:]
 // -------------------------------------------------------------------------
@@ -512,7 +502,7 @@ __global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__
                                                      const int32_t* __restrict__ meta,
                                                      const float* __restrict__ dA1, float* W1,
                                                      float* part, int32_t* ucnt,
-                                                     float* grad_w1) {
+                                                     float* grad_w1, int32_t* cnt, uint32_t* bits, int W) {
   pdl_trigger();
   pdl_wait();
   const float lr = step_lr(meta);
@@ -592,6 +582,7 @@ __global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__
         for (int i = 0; i < VPL; ++i) w[i] = w[i] - lr * acc[i];
         IO::store(W1 + f * H, lane, w);
         if (grad_w1) IO::store(grad_w1 + f * H, lane, acc);
+        reset_feature(cnt, bits, W, (int)f, lane);
       }
       e = se;
       ++u;
@@ -673,7 +664,8 @@ __global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restr
                                                           const int32_t* __restrict__ meta,
                                                           const T* __restrict__ dA1, int H, float* W1,
                                                           float* part, int32_t* ucnt,
-                                                          float* grad_w1) {
+                                                          float* grad_w1, int32_t* fcnt, uint32_t* bits,
+                                                          int W) {
   pdl_trigger();
   pdl_wait();
   const float lr = step_lr(meta);
@@ -794,6 +786,7 @@ __global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restr
         for (int i = 0; i < CPL; ++i) w[i] = w[i] - lr * acc[i];
         st_cols<CPL>(wrow, w, false);
         if (grad_w1) st_cols<CPL>(grad_w1 + (int64_t)f * H + c0 + lane * CPL, acc, false);
+        if (slice == 0) reset_feature(fcnt, bits, W, f, lane);
       }
     }
   }
@@ -823,11 +816,12 @@ cudaError_t spmm_fwd_t(const Launch& lc, const int32_t* rows, int n, const int64
 
 template <int VPL>
 cudaError_t scatter_t(const Launch& lc, float* W1, const Ptrs& P, const WsLayout& L,
-                      float* grad_w1) {
+                      float* grad_w1, int b_max) {
+  const int W = (b_max + 31) / 32;
   static int occ = 0;
   const int grid = wave_grid(lc, k_scatter_sgd<VPL>, 0, L.n_pieces, occ);
   launch_k(lc, k_scatter_sgd<VPL>, dim3(grid), dim3(256), 0, P.e_n, P.e_v, P.e_u, P.useg, P.uniq, P.meta, P.da1,
-                                             W1, P.part5, P.ucnt, grad_w1);
+                                             W1, P.part5, P.ucnt, grad_w1, P.cnt, P.bits, W);
   return cudaGetLastError();
 }
 
@@ -847,7 +841,17 @@ cudaError_t launch_touched(const Launch& lc, const int32_t* rows, int n, const i
   const size_t smem = view_smem(n);
   const int nt = (int)L.n_tiles_f;
   const int W = (b_max + 31) / 32;
-  return launch_k(lc, k_touched, dim3(std::min(kTouchCtas, lc.sms)), dim3(512), smem, n, P.rbase, col, val,
+  const size_t smem_all = ((smem + 3) / 4) * 4 + (size_t)nt * 8;
+  static const int max_ctas = [] { const char* e = getenv("ASGD_K0_CTAS"); return e ? atoi(e) : 0; }();
+  int64_t cap = max_ctas > 0 ? max_ctas : kTouchCtas;
+  const int ctas = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)lc.sms, cap, (L.nz_cap + 1023) / 1024}));
+  static size_t attr = 48 * 1024;
+  if (smem_all > attr) {
+    cudaError_t e = cudaFuncSetAttribute(k_touched, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_all);
+    if (e != cudaSuccess) return e;
+    attr = smem_all;
+  }
+  return launch_k(lc, k_touched, dim3(ctas), dim3(512), smem_all, n, P.rbase, col, val,
                   P.boff, P.meta, P.cnt, P.tsum, F, nt, P.fseg, P.fuid, P.uniq, P.useg, P.bits, W, P.e_n,
                   P.e_v, P.e_u, P.e_f);
 }
@@ -879,7 +883,8 @@ cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float*
   }
   const int gx = std::max(1, lc.sms / nsl);
   return launch_k(lc, k_scatter_sgd_s<T, CPL>, dim3(gx, nsl), dim3(512), smem, P.e_n, P.e_v, P.e_u,
-                  P.e_f, P.useg, P.meta, dA1, H, W1, P.part5, P.ucnt, grad_w1);
+                  P.e_f, P.useg, P.meta, dA1, H, W1, P.part5, P.ucnt, grad_w1, P.cnt, P.bits,
+                  (b_max + 31) / 32);
 }
 
 // Widest column slice whose staged dA1 fits 160 KB of shared memory (0 = none).
@@ -904,10 +909,10 @@ cudaError_t launch_scatter_sgd(const Launch& lc, float* W1, int H, const Ptrs& P
     return scatter_s_t<float, 2>(lc, P.da1, H, b_max, W1, P, grad_w1);
   }
   switch (H) {
-    case 64: return scatter_t<2>(lc, W1, P, L, grad_w1);
-    case 128: return scatter_t<4>(lc, W1, P, L, grad_w1);
-    case 256: return scatter_t<8>(lc, W1, P, L, grad_w1);
-    case 512: return scatter_t<16>(lc, W1, P, L, grad_w1);
+    case 64: return scatter_t<2>(lc, W1, P, L, grad_w1, b_max);
+    case 128: return scatter_t<4>(lc, W1, P, L, grad_w1, b_max);
+    case 256: return scatter_t<8>(lc, W1, P, L, grad_w1, b_max);
+    case 512: return scatter_t<16>(lc, W1, P, L, grad_w1, b_max);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -590,6 +590,12 @@ int pick_bn(int64_t tiles_m, int64_t N, int sms) {
 
 }  // namespace
 
+int gemm_tc_g2_ctas(int n, int H, const WsLayout& W, int sms) {
+  const int bn = H >= 256 ? 256 : H;
+  const int64_t tiles = (int64_t)((n + BM - 1) / BM) * ((H + bn - 1) / bn) * W.splitk;
+  return (int)std::min<int64_t>(tiles, sms);
+}
+
 bool tc_available() {
   std::call_once(g_once, init_encode);
   return g_encode != nullptr;
