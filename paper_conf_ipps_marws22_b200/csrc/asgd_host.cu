@@ -16,6 +16,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <list>
 #include <new>
 #include <string>
 #include <vector>
@@ -164,6 +165,9 @@ struct StepGraph {
   int64_t kernels = 0;                // kernel nodes (asgd_kernel_launches per replay)
   struct Prof { cudaGraphNode_t node; int cls; bool begin; };
   std::vector<Prof> prof;             // profiling event-record nodes, capture order
+  struct ArgNode { cudaGraphNode_t node; cudaKernelNodeParams p; std::vector<void*> args; };
+  std::vector<ArgNode> arg_nodes;     // K-0 and K-1: parameter 0 (StepArgs) is updated per replay
+  StepArgs sa{};                      // storage parameter 0 of arg_nodes points at
   std::vector<cudaEvent_t> placeholders;
   uint64_t last_use = 0;
 };
@@ -197,12 +201,14 @@ struct asgd_ctx {
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_sm = nullptr, ev_dh = nullptr, ev_a = nullptr;
   bf16* w2b_buf[2] = {nullptr, nullptr};         // double-buffered bf16 W2 shadow
   int w2b_cur = 0;
-  std::vector<StepGraph> graphs;                 // CUDA-graph cache of the step, LRU
+  std::list<StepGraph> graphs;                   // CUDA-graph cache of the step, LRU (stable addresses:
+                                                 // the graphs point at their own StepArgs)
   uint64_t graph_clock = 0;
   bool capturing = false;
   std::vector<std::pair<cudaEvent_t, int>> cap_ph;   // (placeholder, cls * 2 + begin) during capture
   cudaEvent_t prof_sink = nullptr;                // target of profiling nodes past kMaxProfPairs
   cudaEvent_t ev_ring[8] = {};                    // asgd_run_tickets: completion of the last steps
+  StepArgs sa{};                                  // current step's arguments (K-0 / K-1 parameter)
   Launch lc() { return Launch{s, &launches, sms}; }
   Launch lc2() { return Launch{s2, &launches, sms}; }
   Launch lc3() { return Launch{s3, &launches, sms}; }
@@ -463,13 +469,13 @@ int enqueue_step(asgd_ctx* c, int n) {
   auto fork_k0 = [&]() -> int {
     CU(cudaEventRecord(c->ev_fork, c->s));
     CU(cudaStreamWaitEvent(c->s2, c->ev_fork, 0));
-    PCU_ON(c->s2, ASGD_K_TOUCHED, launch_touched(c->lc2(), P.rowsc, n, x.row_ptr, x.col, x.val, m.F, P, c->L, m.b_max));
+    PCU_ON(c->s2, ASGD_K_TOUCHED, launch_touched(c->lc2(), c->sa, x, m.F, P, c->L, m.b_max));
     CU(cudaEventRecord(c->ev_join, c->s2));
     return ASGD_OK;
   };
   if (!k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   // K-1
-  PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, P.rowsc, n, x.row_ptr, x.col, x.val, W1, b1, H, P, c->L, bf));
+  PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, c->sa, x, W1, b1, H, P, c->L, bf));
   if (k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   if (!bf) {
     // fp32 path: one stream, G2 reads W2 before G3 updates it in place
@@ -602,6 +608,26 @@ int step_graph(asgd_ctx* c, int n) {
     }
     G.graph = graph;
     CU(cudaGraphInstantiate(&G.exec, graph, 0));
+    {  // K-0 / K-1 nodes: their StepArgs parameter is rebound per replay
+      size_t nn = 0;
+      CU(cudaGraphGetNodes(graph, nullptr, &nn));
+      std::vector<cudaGraphNode_t> nodes(nn);
+      CU(cudaGraphGetNodes(graph, nodes.data(), &nn));
+      const void* f1 = spmm_fwd_func((int)c->d.H);
+      const void* f0 = touched_func();
+      for (cudaGraphNode_t nd : nodes) {
+        cudaGraphNodeType t;
+        if (cudaGraphNodeGetType(nd, &t) != cudaSuccess || t != cudaGraphNodeTypeKernel) continue;
+        cudaKernelNodeParams kp;
+        CU(cudaGraphKernelNodeGetParams(nd, &kp));
+        if (kp.func != f1 && kp.func != f0) continue;
+        const int na = kp.func == f1 ? spmm_fwd_nargs() : touched_nargs();
+        StepGraph::ArgNode an{nd, kp, std::vector<void*>(kp.kernelParams, kp.kernelParams + na)};
+        an.args[0] = &G.sa;
+        G.arg_nodes.push_back(std::move(an));
+      }
+      if (G.arg_nodes.size() != 2) return fail(ASGD_E_STATE, "step graph: %zu K-0/K-1 nodes", G.arg_nodes.size());
+    }
     if (!c->cap_ph.empty()) {
       size_t nn = 0;
       CU(cudaGraphGetNodes(graph, nullptr, &nn));
@@ -623,6 +649,13 @@ int step_graph(asgd_ctx* c, int n) {
     c->cap_ph.clear();
   }
   if (!G.prof.empty()) bind_prof_events(c, G);
+  G.sa = c->sa;
+  for (auto& an : G.arg_nodes) {
+    cudaKernelNodeParams kp = an.p;
+    kp.kernelParams = an.args.data();
+    kp.extra = nullptr;
+    CU(cudaGraphExecKernelNodeSetParams(G.exec, an.node, &kp));
+  }
   CU(cudaGraphLaunch(G.exec, c->s));
   c->launches += G.kernels;
   return ASGD_OK;
@@ -641,9 +674,8 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
   const asgd_csr& x = c->data;
   float* g = c->dbg;
   if (g) CU(cudaMemsetAsync(g, 0, c->Pn * sizeof(float), c->s));
-  // K-0 (a): batch view + the step's row ids, lr and loss pointer, launched eagerly;
-  // the rest of the step replays a cached CUDA graph when possible
-  CU(launch_batch_scan(lc, rows, n, x.row_ptr, x.lab_ptr, x.n_rows, P, c->L.nz_cap, c->L.nl_cap, lr, loss_dev));
+  // the step's only per-call arguments; K-0 and K-1 build the batch view from them
+  c->sa = StepArgs{rows, loss_dev, lr, n};
   const int rc = (graphs_enabled() && !g) ? step_graph(c, n) : enqueue_step(c, n);
   if (rc != ASGD_OK) return rc;
   if (m.precision == ASGD_PREC_BF16) c->w2b_cur ^= 1;
@@ -724,9 +756,7 @@ int asgd_eval_topk(asgd_ctx* c, const asgd_csr* t, const int32_t* rows, int32_t 
   float* b2 = c->params + c->o_b2;
   for (int32_t r0 = 0; r0 < n; r0 += m.b_max) {
     const int nb = std::min<int32_t>(m.b_max, n - r0);
-    CU(launch_batch_scan(lc, rows + r0, nb, t->row_ptr, t->lab_ptr, t->n_rows, P, c->L.nz_cap,
-                         c->L.nl_cap));
-    CU(launch_spmm_fwd(lc, rows + r0, nb, t->row_ptr, t->col, t->val, W1, b1, H, P, c->L, bf));
+    CU(launch_spmm_fwd(lc, StepArgs{rows + r0, nullptr, 0.f, nb}, *t, W1, b1, H, P, c->L, bf));
     if (!bf) {
       GemmArgs a{};
       a.M = nb; a.N = (int)m.L; a.K = H;

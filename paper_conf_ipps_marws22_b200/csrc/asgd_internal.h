@@ -92,17 +92,30 @@ cudaError_t launch_k(const Launch& lc, void (*kernel)(KArgs...), dim3 grid, dim3
 }
 
 // ---------------------------------------------------------------- K-0
-// Also copies rows to P.rowsc and stores lr / loss_dev in meta (M_LR, M_LOSS).
-cudaError_t launch_batch_scan(const Launch&, const int32_t* rows, int n, const int64_t* row_ptr,
-                              const int64_t* lab_ptr, int64_t n_data_rows, const Ptrs&,
-                              int64_t nz_cap, int64_t nl_cap, float lr = 0.f, float* loss_dev = nullptr);
-cudaError_t launch_touched(const Launch&, const int32_t* rows, int n, const int64_t* row_ptr,
-                           const int32_t* col, const float* val, int64_t F, const Ptrs&,
+// The step's per-call arguments: the only kernel arguments that change from
+// step to step (the first parameter of K-0 and K-1; CUDA-graph replays update
+// just these two nodes).
+struct StepArgs {
+  const int32_t* rows;   // dataset row ids of the batch (device)
+  float* loss;           // nullable device scalar for the mean loss
+  float lr;
+  int n;
+};
+// Global batch view published by CTA 0 of K-1 for the rest of the step.
+struct ViewOut {
+  int32_t* boff; int32_t* loff; int64_t* rbase; int32_t* rowsc; int32_t* meta;
+};
+// K-0 (b-e): touched-feature set; builds its own batch view.
+cudaError_t launch_touched(const Launch&, const StepArgs&, const asgd_csr&, int64_t F, const Ptrs&,
                            const WsLayout&, int b_max);
 // ---------------------------------------------------------------- K-1
-cudaError_t launch_spmm_fwd(const Launch&, const int32_t* rows, int n, const int64_t* row_ptr,
-                            const int32_t* col, const float* val, const float* W1, const float* b1,
+// Builds the batch view (K-0 (a)) and publishes it, meta and the row ids for the step.
+cudaError_t launch_spmm_fwd(const Launch&, const StepArgs&, const asgd_csr&, const float* W1, const float* b1,
                             int H, const Ptrs&, const WsLayout&, bool want_bf16);
+const void* spmm_fwd_func(int H);
+const void* touched_func();
+int spmm_fwd_nargs();   // parameter counts (all K-1 instantiations share the signature)
+int touched_nargs();
 // ---------------------------------------------------------------- K-5
 // dA1b: bf16 copy of dA1 (bf16 path) or null (fp32 path stages fp32 dA1).
 // The learning rate of every SGD update is the step's meta[M_LR].

@@ -113,81 +113,6 @@ struct RowIO {
   }
 };
 
-// -------------------------------------------------------------------------
-// K-0 (a): per-row entry / label offsets of the batch (one CTA, exclusive scan)
-// -------------------------------------------------------------------------
-__global__ void __launch_bounds__(1024) k_batch_scan(const int32_t* __restrict__ rows, int n,
-                                                     const int64_t* __restrict__ row_ptr,
-                                                     const int64_t* __restrict__ lab_ptr,
-                                                     int64_t n_data_rows, int32_t* boff,
-                                                     int32_t* loff, int32_t* meta, int64_t nz_cap,
-                                                     int64_t nl_cap, int64_t* rbase, int32_t* rowsc,
-                                                     float lr, float* loss_dev) {
-  pdl_trigger();
-  pdl_wait();
-  if (threadIdx.x == 0) {
-    meta[M_LR] = __float_as_int(lr);
-    *reinterpret_cast<float**>(meta + M_LOSS) = loss_dev;
-  }
-  __shared__ long long wf[32], wl[32];
-  const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
-  const int per = (n + blockDim.x - 1) / blockDim.x;
-  const int r0 = min(n, t * per), r1 = min(n, r0 + per);
-  long long sf = 0, sl = 0;
-  int bad = 0;
-  for (int r = r0; r < r1; ++r) {
-    int64_t id = rows[r];
-    if (id < 0 || id >= n_data_rows) { bad = 1; continue; }
-    sf += row_ptr[id + 1] - row_ptr[id];
-    sl += lab_ptr[id + 1] - lab_ptr[id];
-  }
-  // inclusive warp scan
-  long long xf = sf, xl = sl;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    long long yf = __shfl_up_sync(kFull, xf, o), yl = __shfl_up_sync(kFull, xl, o);
-    if (lane >= o) { xf += yf; xl += yl; }
-  }
-  if (lane == 31) { wf[wid] = xf; wl[wid] = xl; }
-  __syncthreads();
-  if (wid == 0) {
-    long long a = lane < (int)(blockDim.x >> 5) ? wf[lane] : 0;
-    long long b = lane < (int)(blockDim.x >> 5) ? wl[lane] : 0;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      long long ya = __shfl_up_sync(kFull, a, o), yb = __shfl_up_sync(kFull, b, o);
-      if (lane >= o) { a += ya; b += yb; }
-    }
-    wf[lane] = a; wl[lane] = b;
-  }
-  __syncthreads();
-  long long pf = xf - sf + (wid ? wf[wid - 1] : 0);
-  long long pl = xl - sl + (wid ? wl[wid - 1] : 0);
-  for (int r = r0; r < r1; ++r) {
-    boff[r] = (int32_t)min(pf, (long long)nz_cap);
-    loff[r] = (int32_t)min(pl, (long long)nl_cap);
-    int64_t id = rows[r];
-    rowsc[r] = (int32_t)id;
-    rbase[r] = (id < 0 || id >= n_data_rows) ? 0 : row_ptr[id];
-    if (id < 0 || id >= n_data_rows) continue;
-    pf += row_ptr[id + 1] - row_ptr[id];
-    pl += lab_ptr[id + 1] - lab_ptr[id];
-  }
-  if (bad) atomicOr(&meta[M_ERR], ERR_ROW_ID);
-  if (t == blockDim.x - 1) {
-    long long tf = wf[(blockDim.x >> 5) - 1], tl = wl[(blockDim.x >> 5) - 1];
-    int err = 0;
-    if (tf > nz_cap) { err |= ERR_NNZ_CAP; tf = nz_cap; }
-    if (tl > nl_cap) { err |= ERR_LAB_CAP; tl = nl_cap; }
-    boff[n] = (int32_t)tf;
-    loff[n] = (int32_t)tl;
-    meta[M_NNZ] = (int32_t)tf;
-    meta[M_NLAB] = (int32_t)tl;
-    meta[M_NROWS] = n;
-    if (err) atomicOr(&meta[M_ERR], err);
-  }
-}
-
 // Batch view in shared memory: sboff[n + 1] entry offsets, then srbase[n] (8-byte
 // aligned) = row_ptr[rows[r]], both written by K-0 (a).
 __host__ __device__ __forceinline__ size_t view_smem(int n) {
@@ -204,11 +129,98 @@ __device__ __forceinline__ int64_t entry_index(const int32_t* sboff, int n, int 
   return view_rbase(sboff, n)[rr] + (e - sboff[rr]);
 }
 
-__device__ __forceinline__ void load_view(int32_t* sboff, const int32_t* boff, const int64_t* rbase, int n) {
+// -------------------------------------------------------------------------
+// K-0 (a): the batch view, built in shared memory by every CTA of K-0 and K-1
+// (no separate launch on the step's critical path): sboff[r] = flat offset of
+// row r's entries (clamped to nz_cap), srb[r] = row_ptr[rows[r]].  With
+// `publish` (CTA 0 of K-1) it also writes the global view for the later
+// kernels: row ids (rowsc), label offsets, meta (nnz, labels, rows, lr, loss
+// pointer) and the error bits.  Returns the batch nnz (clamped).
+// -------------------------------------------------------------------------
+constexpr int kViewPer = 8;   // rows per thread: n <= kViewPer * blockDim (b_max <= 2048, >= 256 threads)
+
+__device__ int build_view(const StepArgs& sa, const int64_t* __restrict__ row_ptr,
+                          const int64_t* __restrict__ lab_ptr, int64_t n_data_rows, int64_t nz_cap,
+                          int64_t nl_cap, int32_t* sboff, bool publish, const ViewOut& out) {
+  __shared__ long long wf[32], wl[32];
+  const int n = sa.n;
   int64_t* srb = const_cast<int64_t*>(view_rbase(sboff, n));
-  for (int i = threadIdx.x; i <= n; i += blockDim.x) sboff[i] = boff[i];
-  for (int i = threadIdx.x; i < n; i += blockDim.x) srb[i] = rbase[i];
+  const int t = threadIdx.x, lane = t & 31, wid = t >> 5, nw = blockDim.x >> 5;
+  const int r0 = t * kViewPer;
+  int64_t len[kViewPer], llen[kViewPer];
+  long long sf = 0, sl = 0;
+  int bad = 0;
+#pragma unroll
+  for (int i = 0; i < kViewPer; ++i) {
+    len[i] = 0; llen[i] = 0;
+    const int r = r0 + i;
+    if (r < n) {
+      const int64_t id = sa.rows[r];
+      if (id < 0 || id >= n_data_rows) { bad = 1; srb[r] = 0; continue; }
+      const int64_t a = row_ptr[id];
+      len[i] = row_ptr[id + 1] - a;
+      srb[r] = a;
+      if (publish) {
+        llen[i] = lab_ptr[id + 1] - lab_ptr[id];
+        out.rowsc[r] = (int32_t)id;
+        out.rbase[r] = a;
+      }
+      sf += len[i];
+      sl += llen[i];
+    }
+  }
+  long long xf = sf, xl = sl;   // inclusive warp scan
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const long long yf = __shfl_up_sync(kFull, xf, o), yl = __shfl_up_sync(kFull, xl, o);
+    if (lane >= o) { xf += yf; xl += yl; }
+  }
+  if (lane == 31) { wf[wid] = xf; wl[wid] = xl; }
   __syncthreads();
+  if (wid == 0) {
+    long long a = lane < nw ? wf[lane] : 0, c = lane < nw ? wl[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const long long ya = __shfl_up_sync(kFull, a, o), yc = __shfl_up_sync(kFull, c, o);
+      if (lane >= o) { a += ya; c += yc; }
+    }
+    wf[lane] = a; wl[lane] = c;
+  }
+  __syncthreads();
+  long long pf = xf - sf + (wid ? wf[wid - 1] : 0), pl = xl - sl + (wid ? wl[wid - 1] : 0);
+#pragma unroll
+  for (int i = 0; i < kViewPer; ++i) {
+    const int r = r0 + i;
+    if (r < n) {
+      sboff[r] = (int32_t)min(pf, (long long)nz_cap);
+      if (publish) {
+        out.boff[r] = (int32_t)min(pf, (long long)nz_cap);
+        out.loff[r] = (int32_t)min(pl, (long long)nl_cap);
+      }
+      pf += len[i];
+      pl += llen[i];
+    }
+  }
+  long long tf = wf[nw - 1], tl = wl[nw - 1];
+  if (t == 0) sboff[n] = (int32_t)min(tf, (long long)nz_cap);
+  if (publish) {
+    if (bad) atomicOr(&out.meta[M_ERR], ERR_ROW_ID);
+    if (t == 0) {
+      int err = 0;
+      if (tf > nz_cap) { err |= ERR_NNZ_CAP; tf = nz_cap; }
+      if (tl > nl_cap) { err |= ERR_LAB_CAP; tl = nl_cap; }
+      out.boff[n] = (int32_t)tf;
+      out.loff[n] = (int32_t)tl;
+      out.meta[M_NNZ] = (int32_t)tf;
+      out.meta[M_NLAB] = (int32_t)tl;
+      out.meta[M_NROWS] = n;
+      out.meta[M_LR] = __float_as_int(sa.lr);
+      *reinterpret_cast<float**>(out.meta + M_LOSS) = sa.loss;
+      if (err) atomicOr(&out.meta[M_ERR], err);
+    }
+  }
+  __syncthreads();
+  return (int)min(tf, (long long)nz_cap);
 }
 
 // -------------------------------------------------------------------------
@@ -243,10 +255,10 @@ __device__ __forceinline__ void grid_barrier(unsigned long long* ctr) {
   __syncthreads();
 }
 
-__global__ void __launch_bounds__(512) k_touched(int n, const int64_t* __restrict__ rbase,
+__global__ void __launch_bounds__(512) k_touched(StepArgs sa, const int64_t* __restrict__ row_ptr,
+                                                 int64_t n_data_rows, int64_t nz_cap,
                                                  const int32_t* __restrict__ col,
-                                                 const float* __restrict__ val,
-                                                 const int32_t* __restrict__ boff, int32_t* meta,
+                                                 const float* __restrict__ val, int32_t* meta,
                                                  int32_t* cnt, int32_t* tsum, int64_t F, int ntiles,
                                                  int32_t* fseg, int32_t* fuid, int32_t* uniq,
                                                  int32_t* useg, uint32_t* bits, int W, int32_t* e_n,
@@ -260,10 +272,10 @@ __global__ void __launch_bounds__(512) k_touched(int n, const int64_t* __restric
   const int par = meta[M_K0PAR] & 1;
   int32_t* ts = tsum + (size_t)par * 2 * ntiles;          // this step's tile (count, touched) sums
   int32_t* ts_next = tsum + (size_t)(par ^ 1) * 2 * ntiles;
+  const int n = sa.n;
   int32_t* hist = sboff + ((view_smem(n) + 3) / 4);       // [ntiles][2] after the batch view
   for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x) hist[i] = 0;
-  load_view(sboff, boff, rbase, n);
-  const int nnz = meta[M_NNZ];
+  const int nnz = build_view(sa, row_ptr, nullptr, n_data_rows, nz_cap, 0, sboff, false, ViewOut{});
   const int gt = blockIdx.x * blockDim.x + threadIdx.x, gs = gridDim.x * blockDim.x;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
   // ---- A
@@ -358,13 +370,13 @@ __global__ void __launch_bounds__(512) k_touched(int n, const int64_t* __restric
 // -------------------------------------------------------------------------
 template <int VPL>
 // (256, 2): two CTAs per SM, all kU gathers of a group in flight (<= 128 regs)
-__global__ void __launch_bounds__(256, 2) k_spmm_fwd(int n, const int64_t* __restrict__ rbase,
+__global__ void __launch_bounds__(256, 2) k_spmm_fwd(StepArgs sa, const int64_t* __restrict__ row_ptr,
+                                                  const int64_t* __restrict__ lab_ptr, int64_t n_data_rows,
+                                                  int64_t nz_cap, int64_t nl_cap, ViewOut vo,
                                                   const int32_t* __restrict__ col,
                                                   const float* __restrict__ val,
                                                   const float* __restrict__ W1,
-                                                  const float* __restrict__ b1,
-                                                  const int32_t* __restrict__ boff,
-                                                  const int32_t* __restrict__ meta, float* H1,
+                                                  const float* __restrict__ b1, float* H1,
                                                   bf16* H1b, float* part, int32_t* rowcnt) {
   pdl_trigger();
   pdl_wait();
@@ -372,10 +384,10 @@ __global__ void __launch_bounds__(256, 2) k_spmm_fwd(int n, const int64_t* __res
   constexpr int H = 32 * VPL;
   constexpr int kU = VPL >= 16 ? 4 : 8;   // W1 rows in flight per warp
   extern __shared__ int32_t sboff[];
-  load_view(sboff, boff, rbase, n);
+  const int n = sa.n;
+  const int nnz = build_view(sa, row_ptr, lab_ptr, n_data_rows, nz_cap, nl_cap, sboff, blockIdx.x == 0, vo);
   const int64_t* srb = view_rbase(sboff, n);
   const int lane = threadIdx.x & 31;
-  const int nnz = meta[M_NNZ];
   const int npieces = (nnz + kPiece - 1) / kPiece;
   const int nwarps = gridDim.x * (blockDim.x >> 5);
   float bias[VPL];
@@ -803,14 +815,14 @@ int wave_grid(const Launch& lc, K kernel, size_t smem, int64_t pieces, int& occ)
 }
 
 template <int VPL>
-cudaError_t spmm_fwd_t(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
-                       const int32_t* col, const float* val, const float* W1, const float* b1,
+cudaError_t spmm_fwd_t(const Launch& lc, const StepArgs& sa, const asgd_csr& x, const float* W1, const float* b1,
                        const Ptrs& P, const WsLayout& L, bool want_bf16) {
-  const size_t smem = view_smem(n);
+  const size_t smem = view_smem(sa.n);
   static int occ = 0;
   const int grid = wave_grid(lc, k_spmm_fwd<VPL>, view_smem(2048), L.n_pieces, occ);
-  launch_k(lc, k_spmm_fwd<VPL>, dim3(grid), dim3(256), smem, n, P.rbase, col, val, W1, b1, P.boff, P.meta,
-                                             P.h1, want_bf16 ? P.h1b : nullptr, P.part1, P.rowcnt);
+  const ViewOut vo{P.boff, P.loff, P.rbase, P.rowsc, P.meta};
+  launch_k(lc, k_spmm_fwd<VPL>, dim3(grid), dim3(256), smem, sa, x.row_ptr, x.lab_ptr, x.n_rows, L.nz_cap, L.nl_cap,
+           vo, x.col, x.val, W1, b1, P.h1, want_bf16 ? P.h1b : nullptr, P.part1, P.rowcnt);
   return cudaGetLastError();
 }
 
@@ -827,17 +839,9 @@ cudaError_t scatter_t(const Launch& lc, float* W1, const Ptrs& P, const WsLayout
 
 }  // namespace
 
-cudaError_t launch_batch_scan(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
-                              const int64_t* lab_ptr, int64_t n_data_rows, const Ptrs& P,
-                              int64_t nz_cap, int64_t nl_cap, float lr, float* loss_dev) {
-  launch_k(lc, k_batch_scan, dim3(1), dim3(1024), 0, rows, n, row_ptr, lab_ptr, n_data_rows, P.boff, P.loff, P.meta,
-                                     nz_cap, nl_cap, P.rbase, P.rowsc, lr, loss_dev);
-  return cudaGetLastError();
-}
-
-cudaError_t launch_touched(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
-                           const int32_t* col, const float* val, int64_t F, const Ptrs& P,
+cudaError_t launch_touched(const Launch& lc, const StepArgs& sa, const asgd_csr& x, int64_t F, const Ptrs& P,
                            const WsLayout& L, int b_max) {
+  const int n = sa.n;
   const size_t smem = view_smem(n);
   const int nt = (int)L.n_tiles_f;
   const int W = (b_max + 31) / 32;
@@ -851,22 +855,37 @@ cudaError_t launch_touched(const Launch& lc, const int32_t* rows, int n, const i
     if (e != cudaSuccess) return e;
     attr = smem_all;
   }
-  return launch_k(lc, k_touched, dim3(ctas), dim3(512), smem_all, n, P.rbase, col, val,
-                  P.boff, P.meta, P.cnt, P.tsum, F, nt, P.fseg, P.fuid, P.uniq, P.useg, P.bits, W, P.e_n,
+  return launch_k(lc, k_touched, dim3(ctas), dim3(512), smem_all, sa, x.row_ptr, x.n_rows, L.nz_cap, x.col, x.val,
+                  P.meta, P.cnt, P.tsum, F, nt, P.fseg, P.fuid, P.uniq, P.useg, P.bits, W, P.e_n,
                   P.e_v, P.e_u, P.e_f);
 }
 
-cudaError_t launch_spmm_fwd(const Launch& lc, const int32_t* rows, int n, const int64_t* row_ptr,
-                            const int32_t* col, const float* val, const float* W1, const float* b1,
-                            int H, const Ptrs& P, const WsLayout& L, bool want_bf16) {
+cudaError_t launch_spmm_fwd(const Launch& lc, const StepArgs& sa, const asgd_csr& x, const float* W1,
+                            const float* b1, int H, const Ptrs& P, const WsLayout& L, bool want_bf16) {
   switch (H) {
-    case 64: return spmm_fwd_t<2>(lc, rows, n, row_ptr, col, val, W1, b1, P, L, want_bf16);
-    case 128: return spmm_fwd_t<4>(lc, rows, n, row_ptr, col, val, W1, b1, P, L, want_bf16);
-    case 256: return spmm_fwd_t<8>(lc, rows, n, row_ptr, col, val, W1, b1, P, L, want_bf16);
-    case 512: return spmm_fwd_t<16>(lc, rows, n, row_ptr, col, val, W1, b1, P, L, want_bf16);
+    case 64: return spmm_fwd_t<2>(lc, sa, x, W1, b1, P, L, want_bf16);
+    case 128: return spmm_fwd_t<4>(lc, sa, x, W1, b1, P, L, want_bf16);
+    case 256: return spmm_fwd_t<8>(lc, sa, x, W1, b1, P, L, want_bf16);
+    case 512: return spmm_fwd_t<16>(lc, sa, x, W1, b1, P, L, want_bf16);
     default: return cudaErrorInvalidValue;
   }
 }
+
+const void* spmm_fwd_func(int H) {
+  switch (H) {
+    case 64: return reinterpret_cast<const void*>(k_spmm_fwd<2>);
+    case 128: return reinterpret_cast<const void*>(k_spmm_fwd<4>);
+    case 256: return reinterpret_cast<const void*>(k_spmm_fwd<8>);
+    default: return reinterpret_cast<const void*>(k_spmm_fwd<16>);
+  }
+}
+
+const void* touched_func() { return reinterpret_cast<const void*>(k_touched); }
+
+template <typename... A>
+constexpr int nargs_of(void (*)(A...)) { return (int)sizeof...(A); }
+int spmm_fwd_nargs() { return nargs_of(k_spmm_fwd<8>); }
+int touched_nargs() { return nargs_of(k_touched); }
 
 template <typename T, int CPL>
 cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float* W1,
