@@ -184,6 +184,27 @@ int asgd_merge_finish(asgd_ctx* ctx, float gamma);
 int asgd_replicas_weighted_sum(asgd_ctx* ctx, const float* const* replicas_dev,
                                const double* alpha_dev, int32_t n, float* out_dev);
 
+/* Fused peer-memory merge (Alg. 2 lines 8-9 over NVLink
+ * in one kernel instead of prescale + all-reduce + epilogue).  One process per
+ * GPU, N <= 8 ranks on one node.
+ *   asgd_peer_export: writes this replica's CUDA IPC handle (replica and
+ *     workspace allocations) into out[ASGD_PEER_HANDLE_BYTES] (host).
+ *   asgd_peer_open: maps the N ranks' handles (host array of
+ *     N * ASGD_PEER_HANDLE_BYTES, in rank order; entry `rank` is ignored).
+ *     Synchronous; call once after asgd_replica_init on every rank.
+ *   asgd_merge_fused: rank r computes, for its shard of the parameters,
+ *     S = sum_j alpha[j] w_j (fp64, j = 0..N-1) reading every replica over
+ *     P2P, w' = S + gamma d, d <- w' - w, w <- w' on that shard, and stores w'
+ *     into every replica; the stream then waits until all N ranks delivered
+ *     their shards (system-scope counters).  alpha: host fp64[N] (Alg. 2 lines
+ *     1-7, identical on all ranks).  The caller must ensure every rank
+ *     finished its local steps first (the statistics all-gather does).  w and d
+ *     are kept up to date on this rank's shard only.  u <- 0.  Asynchronous. */
+#define ASGD_PEER_HANDLE_BYTES 160
+int asgd_peer_export(asgd_ctx* ctx, void* out_host);
+int asgd_peer_open(asgd_ctx* ctx, int32_t rank, int32_t world, const void* handles_host);
+int asgd_merge_fused(asgd_ctx* ctx, const double* alpha_host, float gamma);
+
 /* ---------------------------------------------------------------- scaling */
 
 /* Alg. 1, host, pure, exact integers: increments

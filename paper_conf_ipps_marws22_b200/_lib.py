@@ -16,6 +16,7 @@ HEADER = os.path.join(_HERE, "..", "include", "asgd.h")
 
 OK, E_ARG, E_SHAPE, E_CUDA, E_STATE, E_UNSUPPORTED = 0, 1, 2, 3, 4, 5
 PREC_FP32, PREC_BF16 = 0, 1
+PEER_HANDLE_BYTES = 160   # ASGD_PEER_HANDLE_BYTES
 PROF_NAMES = ["touched", "spmm", "g1", "softmax", "g2", "dh_b1", "b2", "g3", "scatter", "merge"]
 
 
@@ -55,6 +56,9 @@ _SIGS = {
                                      C.POINTER(_i32), C.POINTER(_i32)]),
     "asgd_merge_prescale": (C.c_int, [_P, _f64]),
     "asgd_merge_finish": (C.c_int, [_P, _f32]),
+    "asgd_peer_export": (C.c_int, [_P, _P]),
+    "asgd_peer_open": (C.c_int, [_P, _i32, _i32, _P]),
+    "asgd_merge_fused": (C.c_int, [_P, _P, _f32]),
     "asgd_replicas_weighted_sum": (C.c_int, [_P, _P, _P, _i32, _P]),
     "asgd_scale_batches": (C.c_int, [_i32, _P, _P, _P, _i64, _i64, _i64, _f64]),
     "asgd_sched_open": (C.c_int, [C.c_char_p, _i32, _i64, _i32, C.POINTER(_P)]),

@@ -162,6 +162,21 @@ class Replica:
     def finish(self, gamma: float):
         call("asgd_merge_finish", self.ctx, float(gamma))
 
+    # -- fused peer-memory merge (asgd_peer_* / asgd_merge_fused)
+    def peer_export(self) -> bytes:
+        buf = (C.c_char * _lib.PEER_HANDLE_BYTES)()
+        call("asgd_peer_export", self.ctx, buf)
+        return bytes(buf)
+
+    def peer_open(self, rank: int, handles: Sequence[bytes]):
+        blob = b"".join(bytes(h).ljust(_lib.PEER_HANDLE_BYTES, b"\0") for h in handles)
+        buf = (C.c_char * len(blob)).from_buffer_copy(blob)
+        call("asgd_peer_open", self.ctx, int(rank), len(handles), buf)
+
+    def merge_fused(self, alpha: Sequence[float], gamma: float):
+        al = (C.c_double * len(alpha))(*[float(a) for a in alpha])
+        call("asgd_merge_fused", self.ctx, al, float(gamma))
+
     def params_changed(self):
         call("asgd_params_changed", self.ctx)
 

@@ -21,6 +21,8 @@
 #include <string>
 #include <vector>
 
+#include <cuda.h>
+
 #include "asgd_internal.h"
 
 using namespace asgd;
@@ -209,6 +211,12 @@ struct asgd_ctx {
   cudaEvent_t prof_sink = nullptr;                // target of profiling nodes past kMaxProfPairs
   cudaEvent_t ev_ring[8] = {};                    // asgd_run_tickets: completion of the last steps
   StepArgs sa{};                                  // current step's arguments (K-0 / K-1 parameter)
+  // fused peer-memory merge (asgd_peer_open / asgd_merge_fused)
+  int peer_rank = -1, peer_world = 0;
+  float* peer_params[kMaxPeers] = {};
+  unsigned long long* peer_sync[kMaxPeers] = {};
+  std::vector<void*> peer_mapped;                 // IPC mappings to close
+  unsigned long long merge_epoch = 0;
   Launch lc() { return Launch{s, &launches, sms}; }
   Launch lc2() { return Launch{s2, &launches, sms}; }
   Launch lc3() { return Launch{s3, &launches, sms}; }
@@ -374,6 +382,7 @@ int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device, v
 int asgd_replica_destroy(asgd_ctx* c) {
   if (c) {
     clear_graphs(c);
+    for (void* pm : c->peer_mapped) cudaIpcCloseMemHandle(pm);
     if (c->prof_sink) cudaEventDestroy(c->prof_sink);
     for (cudaEvent_t ev : c->ev_ring)
       if (ev) cudaEventDestroy(ev);
@@ -723,6 +732,119 @@ int asgd_merge_prescale(asgd_ctx* c, double alpha) {
 int asgd_merge_finish(asgd_ctx* c, float gamma) {
   if (!c) return fail(ASGD_E_ARG, "null ctx");
   PCU(ASGD_K_MERGE, launch_finish(c->lc(), c->params, c->w, c->dd, c->Pn, gamma));
+  if (c->d.precision == ASGD_PREC_BF16)
+    CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->w2b_buf[c->w2b_cur], c->d.L * c->d.H));
+  c->u = 0;
+  return ASGD_OK;
+}
+
+namespace {
+struct PeerHandle {                 // ASGD_PEER_HANDLE_BYTES, opaque to the caller
+  cudaIpcMemHandle_t params;        // allocation holding the replica
+  int64_t params_off;               // replica offset inside it
+  cudaIpcMemHandle_t ws;            // allocation holding the workspace (arrival counter)
+  int64_t ws_off;
+  int32_t device, pad;
+};
+static_assert(sizeof(PeerHandle) <= ASGD_PEER_HANDLE_BYTES, "peer handle size");
+
+using PFN_getRange = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
+
+int alloc_base(const void* p, char** base) {
+  static PFN_getRange fn = [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return (PFN_getRange) nullptr;
+    return reinterpret_cast<PFN_getRange>(f);
+  }();
+  if (!fn) return fail(ASGD_E_CUDA, "cuMemGetAddressRange unavailable");
+  CUdeviceptr b = 0;
+  size_t sz = 0;
+  if (fn(&b, &sz, (CUdeviceptr)p) != CUDA_SUCCESS) return fail(ASGD_E_ARG, "not a device allocation");
+  *base = reinterpret_cast<char*>(b);
+  return ASGD_OK;
+}
+}  // namespace
+
+int asgd_peer_export(asgd_ctx* c, void* out) {
+  if (!c || !out) return fail(ASGD_E_ARG, "null argument");
+  PeerHandle h{};
+  char* bp = nullptr;
+  char* bw = nullptr;
+  int rc = alloc_base(c->params, &bp);
+  if (rc) return rc;
+  rc = alloc_base(c->ws, &bw);
+  if (rc) return rc;
+  CU(cudaIpcGetMemHandle(&h.params, bp));
+  CU(cudaIpcGetMemHandle(&h.ws, bw));
+  h.params_off = reinterpret_cast<char*>(c->params) - bp;
+  h.ws_off = c->ws - bw;
+  h.device = c->device;
+  memset(out, 0, ASGD_PEER_HANDLE_BYTES);
+  memcpy(out, &h, sizeof(h));
+  return ASGD_OK;
+}
+
+int asgd_peer_open(asgd_ctx* c, int32_t rank, int32_t world, const void* handles) {
+  if (!c || !handles) return fail(ASGD_E_ARG, "null argument");
+  if (world < 1 || world > kMaxPeers || rank < 0 || rank >= world)
+    return fail(ASGD_E_ARG, "rank %d / world %d (world <= %d)", rank, world, kMaxPeers);
+  CU(cudaSetDevice(c->device));
+  for (void* pm : c->peer_mapped) cudaIpcCloseMemHandle(pm);
+  c->peer_mapped.clear();
+  std::vector<std::pair<cudaIpcMemHandle_t, char*>> opened;   // one mapping per distinct allocation
+  auto open = [&](const cudaIpcMemHandle_t& hd, char** base) -> int {
+    for (auto& o : opened)
+      if (memcmp(&o.first, &hd, sizeof(hd)) == 0) { *base = o.second; return ASGD_OK; }
+    void* p = nullptr;
+    CU(cudaIpcOpenMemHandle(&p, hd, cudaIpcMemLazyEnablePeerAccess));
+    c->peer_mapped.push_back(p);
+    opened.push_back({hd, static_cast<char*>(p)});
+    *base = static_cast<char*>(p);
+    return ASGD_OK;
+  };
+  for (int j = 0; j < world; ++j) {
+    if (j == rank) {
+      c->peer_params[j] = c->params;
+      c->peer_sync[j] = reinterpret_cast<unsigned long long*>(c->P.meta + M_MSYNC);
+      continue;
+    }
+    PeerHandle h;
+    memcpy(&h, static_cast<const char*>(handles) + (size_t)j * ASGD_PEER_HANDLE_BYTES, sizeof(h));
+    char* bp = nullptr;
+    char* bw = nullptr;
+    int rc = open(h.params, &bp);
+    if (rc) return rc;
+    rc = open(h.ws, &bw);
+    if (rc) return rc;
+    c->peer_params[j] = reinterpret_cast<float*>(bp + h.params_off);
+    c->peer_sync[j] = reinterpret_cast<unsigned long long*>(bw + h.ws_off + (size_t)c->L.meta + M_MSYNC * 4);
+  }
+  c->peer_rank = rank;
+  c->peer_world = world;
+  CU(cudaStreamSynchronize(c->s));
+  c->merge_epoch = 0;
+  CU(cudaMemsetAsync(c->P.meta + M_MSYNC, 0, 12, c->s));   // arrival counter + CTA counter
+  CU(cudaStreamSynchronize(c->s));
+  return ASGD_OK;
+}
+
+int asgd_merge_fused(asgd_ctx* c, const double* alpha, float gamma) {
+  if (!c || !alpha) return fail(ASGD_E_ARG, "null argument");
+  if (c->peer_world < 1) return fail(ASGD_E_STATE, "asgd_peer_open first");
+  const int N = c->peer_world, r = c->peer_rank;
+  PeerSet ps{};
+  ps.n = N;
+  for (int j = 0; j < N; ++j) { ps.p[j] = c->peer_params[j]; ps.sync[j] = c->peer_sync[j]; ps.alpha[j] = alpha[j]; }
+  const int64_t P4 = c->Pn / 4, per = (P4 + N - 1) / N;
+  const int64_t lo = std::min(P4, (int64_t)r * per) * 4;
+  const int64_t hi = (r == N - 1) ? c->Pn : std::min(P4, (int64_t)(r + 1) * per) * 4;
+  const unsigned long long goal = (++c->merge_epoch) * (unsigned long long)N;
+  PCU(ASGD_K_MERGE, launch_merge_fused(c->lc(), ps, c->w, c->dd, lo, hi, gamma,
+                                       reinterpret_cast<unsigned int*>(c->P.meta + M_MDONE),
+                                       reinterpret_cast<unsigned long long*>(c->P.meta + M_MSYNC), goal));
   if (c->d.precision == ASGD_PREC_BF16)
     CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->w2b_buf[c->w2b_cur], c->d.L * c->d.H));
   c->u = 0;

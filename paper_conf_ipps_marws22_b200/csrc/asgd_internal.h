@@ -20,8 +20,9 @@ constexpr int kScanTile = 1024;
 // rest of the step (and its CUDA graph) takes no per-step scalar arguments;
 // M_BAR: 64-bit grid-barrier counter (slots 32-33).
 // M_K0PAR: parity of K-0's double-buffered tile sums.
+// M_MSYNC: fused merge arrival counter (64-bit, slots 40-41), M_MDONE: its CTA counter.
 enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_LR = 6, M_K0PAR = 7, M_COUNT = 8,
-       M_LOSS = 10, M_BAR = 32 };
+       M_LOSS = 10, M_BAR = 32, M_MSYNC = 40, M_MDONE = 42 };
 // error bits in meta[M_ERR]
 enum { ERR_NNZ_CAP = 1, ERR_LAB_CAP = 2, ERR_ROW_ID = 4 };
 
@@ -174,6 +175,18 @@ cudaError_t launch_scale(const Launch&, float* x, int64_t P, double alpha);
 cudaError_t launch_finish(const Launch&, float* params, float* w, float* d, int64_t P, float gamma);
 cudaError_t launch_wsum(const Launch&, const float* const* reps, const double* alpha, int n,
                         int64_t P, float* out);
+// Fused peer-memory merge (NEXT-1): replica pointers, arrival counters and
+// weights of the N ranks (N <= 8), by value.
+constexpr int kMaxPeers = 8;
+struct PeerSet {
+  float* p[kMaxPeers];
+  unsigned long long* sync[kMaxPeers];
+  double alpha[kMaxPeers];
+  int n;
+};
+cudaError_t launch_merge_fused(const Launch&, const PeerSet&, float* w, float* d, int64_t lo, int64_t hi,
+                               float gamma, unsigned int* cta_done, const unsigned long long* arrived,
+                               unsigned long long goal);
 cudaError_t launch_topk(const Launch&, int n, int64_t L, int64_t ldz, int k, const float* z,
                         int32_t* out);
 cudaError_t launch_validate_csr(const Launch&, const asgd_csr* c, int64_t F, int64_t L, int32_t* err);

@@ -116,6 +116,72 @@ __global__ void __launch_bounds__(256) k_wsum(const float* const* __restrict__ r
   }
 }
 
+// ------------------------------------------------ fused peer-memory merge (NEXT-1)
+// Alg. 2 lines 8-9 over NVLink peer memory in one kernel (SURVEY §8(f) NEXT-1,
+// the B200 analogue of the paper's multi-stream ring all-reduce):
+// rank r owns the parameter shard [lo, hi).  For each element it reads every
+// replica j's value over P2P (fixed order j = 0..N-1, fp64), forms
+// S = sum_j alpha_j w_j, applies the momentum epilogue on its own shard of
+// (w, d), and stores w' into every replica (P2P stores).  Every element is
+// computed by exactly one rank and broadcast, so the replicas end bitwise
+// identical; no prescale pass, no NCCL staging.  The last CTA signals every
+// peer's arrival counter (system-scope atomics); k_merge_wait blocks the stream
+// until all N ranks have delivered their shards.
+__device__ __forceinline__ void merge1(const PeerSet& ps, int64_t i, float& w, float& d, float gamma) {
+  double s = 0.0;
+  for (int j = 0; j < ps.n; ++j) s += ps.alpha[j] * (double)ps.p[j][i];
+  const float wn = fmaf(gamma, d, (float)s);
+  d = wn - w;
+  w = wn;
+  for (int j = 0; j < ps.n; ++j) ps.p[j][i] = wn;
+}
+
+__global__ void __launch_bounds__(256) k_merge_fused(PeerSet ps, float* w, float* d, int64_t lo, int64_t hi,
+                                                     float gamma, unsigned int* cta_done) {
+  pdl_trigger();
+  pdl_wait();
+  const int64_t lo4 = lo / 4, hi4 = hi / 4;   // lo is a multiple of 4; the tail (hi % 4) is scalar
+  for (int64_t i4 = lo4 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i4 < hi4;
+       i4 += (int64_t)gridDim.x * blockDim.x) {
+    double s[4] = {0.0, 0.0, 0.0, 0.0};
+    for (int j = 0; j < ps.n; ++j) {
+      const float4 v = reinterpret_cast<const float4*>(ps.p[j])[i4];
+      const double a = ps.alpha[j];
+      s[0] += a * (double)v.x; s[1] += a * (double)v.y; s[2] += a * (double)v.z; s[3] += a * (double)v.w;
+    }
+    float4 ww = reinterpret_cast<float4*>(w)[i4], dd = reinterpret_cast<float4*>(d)[i4];
+    float4 o;
+    o.x = fmaf(gamma, dd.x, (float)s[0]); o.y = fmaf(gamma, dd.y, (float)s[1]);
+    o.z = fmaf(gamma, dd.z, (float)s[2]); o.w = fmaf(gamma, dd.w, (float)s[3]);
+    dd.x = o.x - ww.x; dd.y = o.y - ww.y; dd.z = o.z - ww.z; dd.w = o.w - ww.w;
+    reinterpret_cast<float4*>(w)[i4] = o;
+    reinterpret_cast<float4*>(d)[i4] = dd;
+    for (int j = 0; j < ps.n; ++j) reinterpret_cast<float4*>(ps.p[j])[i4] = o;
+  }
+  if (blockIdx.x == 0)
+    for (int64_t i = hi4 * 4 + threadIdx.x; i < hi; i += blockDim.x) merge1(ps, i, w[i], d[i], gamma);
+  // completion: the last CTA tells every rank that this shard has arrived
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const unsigned int old = atomicAdd(cta_done, 1u);
+    if (old == gridDim.x - 1) {
+      *cta_done = 0u;
+      __threadfence_system();
+      for (int j = 0; j < ps.n; ++j) atomicAdd_system(ps.sync[j], 1ull);
+    }
+  }
+}
+
+__global__ void k_merge_wait(const unsigned long long* arrived, unsigned long long goal) {
+  unsigned long long v;
+  do {
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(arrived) : "memory");
+    if (v < goal) __nanosleep(256);
+  } while (v < goal);
+  __threadfence_system();
+}
+
 // ------------------------------------------------------------------- top-k
 struct Cand { float v; int id; };
 __device__ __forceinline__ bool better(const Cand& a, const Cand& b) {
@@ -220,6 +286,15 @@ cudaError_t launch_finish(const Launch& lc, float* params, float* w, float* d, i
 cudaError_t launch_wsum(const Launch& lc, const float* const* reps, const double* alpha, int n,
                         int64_t P, float* out) {
   launch_k(lc, k_wsum, dim3(grid_for(lc, P)), dim3(256), 0, reps, alpha, n, P, out);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_merge_fused(const Launch& lc, const PeerSet& ps, float* w, float* d, int64_t lo, int64_t hi,
+                               float gamma, unsigned int* cta_done, const unsigned long long* arrived,
+                               unsigned long long goal) {
+  launch_k(lc, k_merge_fused, dim3(grid_for(lc, std::max<int64_t>((hi - lo) / 4, 1))), dim3(256), 0, ps, w, d, lo, hi,
+           gamma, cta_done);
+  launch_k(lc, k_merge_wait, dim3(1), dim3(32), 0, arrived, goal);
   return cudaGetLastError();
 }
 

@@ -109,11 +109,25 @@ class DistributedAdaptiveSGD:
     """Rank `rank` of `world` (one GPU each)."""
 
     def __init__(self, replica: api.Replica, hyper: Hyper, rank: int, world: int,
-                 sched: api.Scheduler, group=None, inflight: int = 2, native: bool = True):
+                 sched: api.Scheduler, group=None, inflight: int = 2, native: bool = True,
+                 merge: str = "nccl"):
         """native: run the ticket loop in libasgd (asgd_run_tickets); False keeps
-        the Python loop of run_tickets (same routing semantics)."""
+        the Python loop of run_tickets (same routing semantics).
+        merge: "nccl" = prescale + all_reduce(SUM) + epilogue (K-6, NCCL, K-7);
+        "fused" = asgd_merge_fused over CUDA-IPC peer memory (NEXT-1)."""
         self.rep, self.h, self.rank, self.world = replica, hyper, rank, world
         self.native = native
+        if merge not in ("nccl", "fused"):
+            raise ValueError(f"merge={merge!r}")
+        self.merge = merge
+        if merge == "fused":
+            handles = [None] * world
+            mine = replica.peer_export()
+            if world > 1:
+                dist.all_gather_object(handles, mine, group=group)
+            else:
+                handles = [mine]
+            replica.peer_open(rank, handles)
         self.sched, self.group, self.inflight = sched, group, inflight
         self.b = [hyper.b_max] * world            # P:1565-1566: initial b = b_max
         self.lr = [hyper.lr_max] * world
@@ -146,10 +160,13 @@ class DistributedAdaptiveSGD:
         if r == 0:
             self.sched.reset(self.mb + 1)        # every rank is past its tickets
         alpha, rr, ss, pert = api.merge_weights(us, bs, nu, h.pert_thr, h.delta, h.pert_renorm)
-        rep.prescale(alpha[r])
-        if self.world > 1:
-            dist.all_reduce(rep.params, op=dist.ReduceOp.SUM, group=self.group)
-        rep.finish(h.gamma)
+        if self.merge == "fused":
+            rep.merge_fused(alpha, h.gamma)
+        else:
+            rep.prescale(alpha[r])
+            if self.world > 1:
+                dist.all_reduce(rep.params, op=dist.ReduceOp.SUM, group=self.group)
+            rep.finish(h.gamma)
         # ---- Alg. 1 ----------------------------------------------------------
         lr_used = list(self.lr)
         self.b, self.lr = api.scale_batches(us, bs, h.b_min, h.b_max, h.beta, h.lr_max)

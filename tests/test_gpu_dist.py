@@ -1,7 +1,9 @@
 """The real multi-process driver (DistributedAdaptiveSGD) on one GPU: two ranks
 share cuda:0, take tickets from the shm scheduler, merge through
-torch.distributed (gloo here; NCCL on multi-GPU boxes), and must end with
-bitwise-identical global models equal to the oracle replaying their ticket log."""
+torch.distributed (gloo all-reduce here; NCCL on multi-GPU boxes) or through
+the fused peer-memory merge kernel (CUDA IPC between the two processes), and
+must end with bitwise-identical global models equal to the oracle replaying
+their ticket log."""
 import os
 import socket
 import uuid
@@ -22,7 +24,7 @@ def _port():
     return p
 
 
-def _rank(rank, world, port, shm, out, precision, n_mb):
+def _rank(rank, world, port, shm, out, precision, n_mb, merge):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     import torch.distributed as dist
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -41,7 +43,7 @@ def _rank(rank, world, port, shm, out, precision, n_mb):
     dist.barrier()
     if rank != 0:
         sched = api.Scheduler(shm, world, h.M, create=False)
-    drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=1)
+    drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=1, merge=merge)
     logs, stats = [], []
     for mb in range(n_mb):
         ids = sample_stream(cfg, mb * h.M, h.M)
@@ -49,18 +51,19 @@ def _rank(rank, world, port, shm, out, precision, n_mb):
         logs.append([r for _, r, _, _ in st.routes])
         stats.append((st.u, st.b, st.lr, st.alpha, st.perturbed))
     torch.cuda.synchronize()
-    np.save(os.path.join(out, f"w{rank}.npy"), rep.w.cpu().numpy())
+    np.save(os.path.join(out, f"w{rank}.npy"), rep.params.cpu().numpy())   # = w' after every merge
     np.save(os.path.join(out, f"s{rank}.npy"), np.array([logs, stats], dtype=object), allow_pickle=True)
     dist.barrier()
     sched.close()
     dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("merge", ["nccl", "fused"])
 @pytest.mark.parametrize("precision,tol", [("fp32", 1e-4), ("bf16", 2e-2)])
-def test_two_ranks_one_gpu(tmp_path, precision, tol):
+def test_two_ranks_one_gpu(tmp_path, precision, tol, merge):
     world, n_mb = 2, 4
     shm = "/asgd_d_" + uuid.uuid4().hex[:8]
-    mp.spawn(_rank, args=(world, _port(), shm, str(tmp_path), precision, n_mb), nprocs=world, join=True)
+    mp.spawn(_rank, args=(world, _port(), shm, str(tmp_path), precision, n_mb, merge), nprocs=world, join=True)
     w0, w1 = (np.load(tmp_path / f"w{r}.npy") for r in range(world))
     np.testing.assert_array_equal(w0, w1)          # replicas end bitwise identical (Q20)
     logs, stats = np.load(tmp_path / "s0.npy", allow_pickle=True)
