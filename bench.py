@@ -44,6 +44,8 @@ def _args():
     p.add_argument("--precision", default="auto", choices=["auto", "fp32", "bf16"])
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--inflight", type=int, default=2)
+    p.add_argument("--method", default="adaptive", choices=["adaptive", "elastic"],
+                   help="adaptive: dynamic tickets + Alg. 1/2; elastic: Elastic SGD A/B (static batches, alpha = 1/N)")
     p.add_argument("--merge", default="fused", choices=["fused", "nccl"],
                    help="fused: peer-memory merge kernel over CUDA IPC (NEXT-1); nccl: prescale + all_reduce + epilogue")
     p.add_argument("--e2e-steps", type=int, default=None)
@@ -228,12 +230,14 @@ def main():
         sched = api.Scheduler(shm, world, M, create=False)
     merge_used = a.merge
     try:
-        drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=a.inflight, merge=a.merge)
+        drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=a.inflight, merge=a.merge,
+                                           method=a.method)
     except Exception as e:   # e.g. no CUDA IPC between the ranks' GPUs: NCCL all-reduce merge instead
         if a.merge != "fused":
             raise
         merge_used = f"nccl (fused unavailable: {type(e).__name__}: {str(e)[:120]})"
-        drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=a.inflight, merge="nccl")
+        drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=a.inflight, merge="nccl",
+                                           method=a.method)
     K, W = a.steps, a.warmup
     Ke = a.e2e_steps if a.e2e_steps is not None else min(K, 10)
     ids = [sample_stream(cfg, mb * M, M) for mb in range(W + K + Ke)]
@@ -340,7 +344,7 @@ def main():
                        "mega_batch_samples": M, "step": "1 mega-batch = local steps + merge",
                        "precision": prec, "l2": "flushed (256 MiB write) between timed steps",
                        "inflight": a.inflight, "parallelism": f"dp{world} (model averaging)",
-                       "merge": merge_used,
+                       "merge": merge_used, "method": a.method,
                        "mean_batch_nnz": round(wl["nnz"], 1), "mean_touched_rows": round(wl["U"], 1)},
             "roofline": roof,
             "kernels_warmup_profile": per,

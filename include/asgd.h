@@ -255,6 +255,17 @@ int asgd_run_tickets(asgd_ctx* ctx, asgd_sched* s, int32_t rank, int64_t b_i,
                      const int32_t* stream_rows_dev, float lr, float* losses_dev,
                      int64_t losses_cap, int32_t inflight, int64_t* n_steps);
 
+/* Elastic SGD's static schedule (elastic model averaging; SURVEY
+ * NEXT-2): the mega-batch of M samples is cut into batches of b samples and
+ * batch k goes to rank k mod world, so every rank processes the same number
+ * of batches (+-1 when world does not divide the batch count, reading R10).
+ * Enqueues this rank's steps exactly like asgd_run_tickets (same inflight,
+ * losses and n_steps semantics), without the shared counter. */
+int asgd_run_static(asgd_ctx* ctx, int32_t rank, int32_t world, int64_t b,
+                    const int32_t* stream_rows_dev, int64_t M, float lr,
+                    float* losses_dev, int64_t losses_cap, int32_t inflight,
+                    int64_t* n_steps);
+
 /* Replay (parity): ranks in ticket order -> routes (rank, start, len) with the
  * batch sizes b[rank], stopping at M.  out: int64[3*cap]. */
 int asgd_route_replay(int32_t n_tickets, const int32_t* order, const int64_t* b,

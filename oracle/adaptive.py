@@ -89,3 +89,33 @@ def run(F: int, H: int, L: int, data, w0: np.ndarray, stream_rows_of: Callable[[
         b, lr = _scaling.scale_batches(u, b, b_min, b_max, beta, lr_max)
         out.append(rec)
     return out
+
+
+def run_elastic(F: int, H: int, L: int, data, w0: np.ndarray, stream_rows_of: Callable[[int], np.ndarray],
+                n_rep: int, n_mb: int, M: int, b: int, lr: float,
+                gamma: float = 0.9) -> List[MegaBatchRecord]:
+    """Elastic SGD (model averaging): static equal
+    batches (routing.static), every replica starts from the global model, the
+    merge averages the replicas with alpha_i = 1/N and applies the same
+    momentum update rule as Adaptive SGD (both run in the same
+    framework with the same model update).  No batch-size scaling, no
+    perturbation."""
+    w = np.asarray(w0, dtype=np.float64).copy()
+    d = np.zeros_like(w)
+    out: List[MegaBatchRecord] = []
+    alpha = [1.0 / n_rep] * n_rep
+    for mb in range(n_mb):
+        rows = stream_rows_of(mb)
+        routes = _routing.static(n_rep, b, M)
+        replicas = [w.copy() for _ in range(n_rep)]
+        losses = []
+        for (r, start, n) in routes:
+            batch = data.row_slice(rows[start:start + n])
+            replicas[r], loss, _ = _model.sgd_step(replicas[r], batch, lr, F, H, L)
+            losses.append(loss)
+        u = _routing.updates(routes, n_rep)
+        nu = [_merge.norm_per_param(x) for x in replicas]
+        w, d = _merge.merge_models(replicas, alpha, w, d, gamma)
+        out.append(MegaBatchRecord(routes, losses, u, [b] * n_rep, [lr] * n_rep, nu, list(alpha), False, -1, -1,
+                                   w.copy(), d.copy()))
+    return out

@@ -56,6 +56,19 @@ def simulate(b: Sequence[int], M: int,
     return out
 
 
+def static(N: int, b: int, M: int) -> List[Route]:
+    """Elastic model averaging's static schedule (§II; P:597-599:
+    "every GPU has to process the same number of batches"): the mega-batch is
+    cut into batches of b samples; batch k goes to rank k mod N (reading R10:
+    when N does not divide the batch count the first ranks get one more)."""
+    out: List[Route] = []
+    k = 0
+    for c in range(0, M, b):
+        out.append((k % N, c, min(b, M - c)))
+        k += 1
+    return out
+
+
 def updates(routes: Sequence[Route], N: int) -> List[int]:
     """u_i = number of batches (model updates) rank i received."""
     u = [0] * N

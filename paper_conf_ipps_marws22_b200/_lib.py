@@ -64,6 +64,7 @@ _SIGS = {
     "asgd_sched_open": (C.c_int, [C.c_char_p, _i32, _i64, _i32, C.POINTER(_P)]),
     "asgd_sched_next": (C.c_int, [_P, _i32, _i64, C.POINTER(_i64), C.POINTER(_i64)]),
     "asgd_run_tickets": (C.c_int, [_P, _P, _i32, _i64, _P, _f32, _P, _i64, _i32, C.POINTER(_i64)]),
+    "asgd_run_static": (C.c_int, [_P, _i32, _i32, _i64, _P, _i64, _f32, _P, _i64, _i32, C.POINTER(_i64)]),
     "asgd_sched_log": (C.c_int, [_P, _P, _i64, C.POINTER(_i64)]),
     "asgd_sched_reset": (C.c_int, [_P, _i64]),
     "asgd_sched_wait": (C.c_int, [_P, _i64, _i64]),

@@ -137,6 +137,16 @@ class Replica:
              int(inflight), C.byref(n))
         return n.value
 
+    def run_static(self, rank: int, world: int, b: int, stream_rows: torch.Tensor, lr: float,
+                   losses: Optional[torch.Tensor] = None, inflight: int = 2) -> int:
+        """Elastic SGD's static share of the mega-batch (asgd_run_static)."""
+        assert stream_rows.dtype == torch.int32 and stream_rows.is_cuda and stream_rows.is_contiguous()
+        n = C.c_int64()
+        call("asgd_run_static", self.ctx, int(rank), int(world), int(b), _ptr(stream_rows), int(stream_rows.numel()),
+             float(lr), _ptr(losses) if losses is not None else None,
+             int(losses.numel()) if losses is not None else 0, int(inflight), C.byref(n))
+        return n.value
+
     def updates(self) -> int:
         u = C.c_int64()
         call("asgd_updates", self.ctx, C.byref(u))

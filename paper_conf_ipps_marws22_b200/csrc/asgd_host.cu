@@ -1115,9 +1115,14 @@ int asgd_sched_next(asgd_sched* s, int32_t rank, int64_t b, int64_t* start, int6
   return 1;
 }
 
-int asgd_run_tickets(asgd_ctx* c, asgd_sched* s, int32_t rank, int64_t b_i, const int32_t* stream_rows,
-                     float lr, float* losses, int64_t losses_cap, int32_t inflight, int64_t* n_steps) {
-  if (!c || !s || !stream_rows || !n_steps || b_i < 1) return fail(ASGD_E_ARG, "bad argument");
+}  // extern "C"
+
+namespace {
+// The rank's step loop shared by the dynamic and the static schedule: next(&start, &len)
+// returns 1 for a batch, 0 when the rank's share is done, < 0 on error.
+template <typename Next>
+int run_steps(asgd_ctx* c, Next next, const int32_t* stream_rows, float lr, float* losses, int64_t losses_cap,
+              int32_t inflight, int64_t* n_steps) {
   if (inflight < 1 || inflight > kMaxInflight) return fail(ASGD_E_ARG, "inflight=%d not in [1, %d]", inflight, kMaxInflight);
   for (auto& ev : c->ev_ring)
     if (!ev) CU(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
@@ -1125,8 +1130,8 @@ int asgd_run_tickets(asgd_ctx* c, asgd_sched* s, int32_t rank, int64_t b_i, cons
   for (;;) {
     if (k >= inflight) CU(cudaEventSynchronize(c->ev_ring[(k - inflight) % kMaxInflight]));
     int64_t start = 0, len = 0;
-    const int r = asgd_sched_next(s, rank, b_i, &start, &len);
-    if (r < 0) return fail(-r, "asgd_sched_next failed");
+    const int r = next(&start, &len);
+    if (r < 0) return fail(-r, "scheduler failed");
     if (r == 0) break;
     const int rc = asgd_local_step(c, stream_rows + start, (int32_t)len, lr,
                                    (losses && k < losses_cap) ? losses + k : nullptr);
@@ -1136,6 +1141,31 @@ int asgd_run_tickets(asgd_ctx* c, asgd_sched* s, int32_t rank, int64_t b_i, cons
   }
   *n_steps = k;
   return ASGD_OK;
+}
+}  // namespace
+
+extern "C" {
+
+int asgd_run_tickets(asgd_ctx* c, asgd_sched* s, int32_t rank, int64_t b_i, const int32_t* stream_rows,
+                     float lr, float* losses, int64_t losses_cap, int32_t inflight, int64_t* n_steps) {
+  if (!c || !s || !stream_rows || !n_steps || b_i < 1) return fail(ASGD_E_ARG, "bad argument");
+  return run_steps(c, [&](int64_t* st, int64_t* ln) { return asgd_sched_next(s, rank, b_i, st, ln); }, stream_rows,
+                   lr, losses, losses_cap, inflight, n_steps);
+}
+
+int asgd_run_static(asgd_ctx* c, int32_t rank, int32_t world, int64_t b, const int32_t* stream_rows, int64_t M,
+                    float lr, float* losses, int64_t losses_cap, int32_t inflight, int64_t* n_steps) {
+  if (!c || !stream_rows || !n_steps || b < 1 || M < 0 || world < 1 || rank < 0 || rank >= world)
+    return fail(ASGD_E_ARG, "bad argument");
+  int64_t cur = (int64_t)rank * b;
+  return run_steps(c, [&](int64_t* st, int64_t* ln) {
+                     if (cur >= M) return 0;
+                     *st = cur;
+                     *ln = std::min<int64_t>(b, M - cur);
+                     cur += (int64_t)world * b;
+                     return 1;
+                   },
+                   stream_rows, lr, losses, losses_cap, inflight, n_steps);
 }
 
 int asgd_sched_log(asgd_sched* s, int64_t* out, int64_t cap, int64_t* n_out) {

@@ -110,13 +110,18 @@ class DistributedAdaptiveSGD:
 
     def __init__(self, replica: api.Replica, hyper: Hyper, rank: int, world: int,
                  sched: api.Scheduler, group=None, inflight: int = 2, native: bool = True,
-                 merge: str = "nccl"):
+                 merge: str = "nccl", method: str = "adaptive"):
         """native: run the ticket loop in libasgd (asgd_run_tickets); False keeps
         the Python loop of run_tickets (same routing semantics).
         merge: "nccl" = prescale + all_reduce(SUM) + epilogue (K-6, NCCL, K-7);
-        "fused" = asgd_merge_fused over CUDA-IPC peer memory (NEXT-1)."""
+        "fused" = asgd_merge_fused over CUDA-IPC peer memory (NEXT-1).
+        method: "adaptive" (dynamic tickets, Alg. 1 + Alg. 2) or "elastic"
+        (Elastic SGD: static equal batches, alpha = 1/N, same update rule)."""
         self.rep, self.h, self.rank, self.world = replica, hyper, rank, world
         self.native = native
+        if method not in ("adaptive", "elastic"):
+            raise ValueError(f"method={method!r}")
+        self.method = method
         if merge not in ("nccl", "fused"):
             raise ValueError(f"merge={merge!r}")
         self.merge = merge
@@ -141,6 +146,8 @@ class DistributedAdaptiveSGD:
     def megabatch(self, stream_rows: torch.Tensor, keep_log: bool = False) -> MegaBatchStats:
         """One mega-batch over the M sample ids stream_rows (device int32)."""
         rep, h, r = self.rep, self.h, self.rank
+        if self.method == "elastic":
+            return self._megabatch_elastic(stream_rows, keep_log)
         self.sched.wait(self.mb)
         b_i, lr_i = self.b[r], self.lr[r]
 
@@ -160,17 +167,38 @@ class DistributedAdaptiveSGD:
         if r == 0:
             self.sched.reset(self.mb + 1)        # every rank is past its tickets
         alpha, rr, ss, pert = api.merge_weights(us, bs, nu, h.pert_thr, h.delta, h.pert_renorm)
-        if self.merge == "fused":
-            rep.merge_fused(alpha, h.gamma)
-        else:
-            rep.prescale(alpha[r])
-            if self.world > 1:
-                dist.all_reduce(rep.params, op=dist.ReduceOp.SUM, group=self.group)
-            rep.finish(h.gamma)
+        self._merge(alpha)
         # ---- Alg. 1 ----------------------------------------------------------
         lr_used = list(self.lr)
         self.b, self.lr = api.scale_batches(us, bs, h.b_min, h.b_max, h.beta, h.lr_max)
         st = MegaBatchStats(self.mb, us, bs, lr_used, nu, alpha, rr, ss, pert, routes, n_steps)
+        self.mb += 1
+        return st
+
+    def _merge(self, alpha):
+        rep, h = self.rep, self.h
+        if self.merge == "fused":
+            rep.merge_fused(alpha, h.gamma)
+        else:
+            rep.prescale(alpha[self.rank])
+            if self.world > 1:
+                dist.all_reduce(rep.params, op=dist.ReduceOp.SUM, group=self.group)
+            rep.finish(h.gamma)
+
+    def _megabatch_elastic(self, stream_rows: torch.Tensor, keep_log: bool) -> MegaBatchStats:
+        """Elastic SGD: static equal batches of
+        b_max, alpha_i = 1/N, the same momentum update; no Alg. 1."""
+        rep, h, r, N = self.rep, self.h, self.rank, self.world
+        M = int(stream_rows.numel())
+        n_steps = rep.run_static(r, N, h.b_max, stream_rows, h.lr_max, self.losses, self.inflight)
+        rep.sqnorm(self.sq)
+        us, bs, nu = exchange_stats(n_steps, h.b_max, self.sq, rep.P, N, self.group)   # also the barrier
+        alpha = [1.0 / N] * N
+        self._merge(alpha)
+        routes = []
+        if keep_log and r == 0:
+            routes = [(k, k % N, c, min(h.b_max, M - c)) for k, c in enumerate(range(0, M, h.b_max))]
+        st = MegaBatchStats(self.mb, us, bs, [h.lr_max] * N, nu, alpha, -1, -1, False, routes, n_steps)
         self.mb += 1
         return st
 

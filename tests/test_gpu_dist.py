@@ -24,7 +24,7 @@ def _port():
     return p
 
 
-def _rank(rank, world, port, shm, out, precision, n_mb, merge):
+def _rank(rank, world, port, shm, out, precision, n_mb, merge, method="adaptive"):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     import torch.distributed as dist
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -43,7 +43,7 @@ def _rank(rank, world, port, shm, out, precision, n_mb, merge):
     dist.barrier()
     if rank != 0:
         sched = api.Scheduler(shm, world, h.M, create=False)
-    drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=1, merge=merge)
+    drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=1, merge=merge, method=method)
     logs, stats = [], []
     for mb in range(n_mb):
         ids = sample_stream(cfg, mb * h.M, h.M)
@@ -80,5 +80,29 @@ def test_two_ranks_one_gpu(tmp_path, precision, tol, merge):
     for (u, b, lr, alpha, pert), rec in zip(stats, recs):
         assert list(u) == rec.u and list(b) == rec.b and list(lr) == rec.lr and pert == rec.perturbed
         np.testing.assert_allclose(alpha, rec.alpha, rtol=1e-12)
+    ref = recs[-1].w
+    assert np.linalg.norm(w0 - ref) / np.linalg.norm(ref) <= tol
+
+
+@pytest.mark.parametrize("precision,tol", [("fp32", 1e-4), ("bf16", 2e-2)])
+def test_two_ranks_elastic(tmp_path, precision, tol):
+    """Elastic SGD mode (NEXT-2): static equal batches, alpha = 1/N, fused merge."""
+    world, n_mb = 2, 3
+    shm = "/asgd_e_" + uuid.uuid4().hex[:8]
+    mp.spawn(_rank, args=(world, _port(), shm, str(tmp_path), precision, n_mb, "fused", "elastic"), nprocs=world,
+             join=True)
+    w0, w1 = (np.load(tmp_path / f"w{r}.npy") for r in range(world))
+    np.testing.assert_array_equal(w0, w1)
+    logs, stats = np.load(tmp_path / "s0.npy", allow_pickle=True)
+    from oracle import adaptive
+    from synth import config, generate, init_params, sample_stream
+    cfg = config("tiny")
+    data = generate(cfg)
+    M = cfg.mega_batch
+    recs = adaptive.run_elastic(cfg.F, cfg.H, cfg.L, data, init_params(cfg), lambda mb: sample_stream(cfg, mb * M, M),
+                                n_rep=world, n_mb=n_mb, M=M, b=cfg.b_max, lr=cfg.lr_max)
+    for log, (u, b, lr, alpha, pert), rec in zip(logs, stats, recs):
+        assert log == [r for r, _, _ in rec.routes]
+        assert list(u) == rec.u and list(alpha) == rec.alpha and not pert
     ref = recs[-1].w
     assert np.linalg.norm(w0 - ref) / np.linalg.norm(ref) <= tol
