@@ -166,6 +166,8 @@ def kernel_work(cls: str, cfg, bf16: bool, st):
     if cls == "scatter":
         return ("bytes", 8.0 * nnz + 4.0 * B * H + 8.0 * U * H)
     if cls == "softmax":
+        if bf16 and cfg.b_max * L * 4 > (64 << 20):   # fused path: k_lse + G1b (Z recomputed on tensor cores)
+            return ("flops", 2.0 * B * H * L)
         return ("bytes", (6.0 if bf16 else 8.0) * B * L + 8.0 * st["nlab"])
     if cls == "touched":
         return ("bytes", 4.0 * nnz + 12.0 * nnz + 8.0 * F + 12.0 * B)
@@ -314,7 +316,7 @@ def main():
         avg_s = ms[dom] / max(cnt[dom], 1) / 1e3
         if kind == "flops":
             achieved = work / avg_s / 1e12
-            if bf16:
+            if bf16 or dname == "softmax":
                 bound, peak, unit = "tensor", peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"]), "TFLOP/s"
             else:
                 bound, unit = "alu", "TFLOP/s"

@@ -94,6 +94,11 @@ CONFIGS: Dict[str, XmlConfig] = {
         XmlConfig("amazon670k", 4, F=135909, L=670091, H=256, n_train=490449,
                   n_test=153025, s_bar=76.0, s_sigma=0.8, y_bar=5.0,
                   b_max=1024),
+        # the second Table I dataset; W1 is
+        # 800 MB, 75 labels per row
+        XmlConfig("delicious200k", 5, F=782585, L=205443, H=256, n_train=196606,
+                  n_test=100095, s_bar=302.0, s_sigma=0.8, y_bar=75.0,
+                  b_max=1024),
     ]
 }
 

@@ -64,3 +64,8 @@ def test_amazon670k_bench_launch():
 
 def test_wiki10_full_split_bench_launch():
     _check_big("wiki10_31k", None, "bf16", chunk=256)
+
+
+def test_delicious200k_bench_launch():
+    """NEXT-3: F = 782,585 (800 MB of W1), L = 205,443, 75 labels per row."""
+    _check_big("delicious200k", 8192, "bf16", chunk=128)
