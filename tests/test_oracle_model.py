@@ -40,19 +40,20 @@ def _batch_and_params(cfg, B=4, rng_seed=0):
     return data, batch, w
 
 
-def test_finite_differences():
+@pytest.mark.parametrize("loss_kind", ["softmax", "sigmoid"])
+def test_finite_differences(loss_kind):
     cfg = _small()
     F, H, L = cfg.F, cfg.H, cfg.L
     _, batch, w = _batch_and_params(cfg)
     A1, _, _ = model.forward(w, batch, F, H, L)
     h = 1e-6
     assert np.abs(A1).min() > 100 * h, "a ReLU kink is within FD reach; pick another seed"
-    loss, g = model.loss_and_grad(w, batch, F, H, L)
+    loss, g = model.loss_and_grad(w, batch, F, H, L, loss_kind)
     fd = np.zeros_like(w)
     for i in range(len(w)):
         wp = w.copy(); wp[i] += h
         wm = w.copy(); wm[i] -= h
-        fd[i] = (model.loss_only(wp, batch, F, H, L) - model.loss_only(wm, batch, F, H, L)) / (2 * h)
+        fd[i] = (model.loss_only(wp, batch, F, H, L, loss_kind) - model.loss_only(wm, batch, F, H, L, loss_kind)) / (2 * h)
     from synth import param_layout
     lay = param_layout(F, H, L)
     for name in ("W1", "b1", "W2", "b2"):
@@ -65,7 +66,7 @@ def test_finite_differences():
     assert np.isfinite(loss) and loss > 0
 
 
-def _torch_loss(w, batch, F, H, L):
+def _torch_loss(w, batch, F, H, L, loss_kind="softmax"):
     from synth import param_layout
     lay = param_layout(F, H, L)
     wt = torch.tensor(w, dtype=torch.float64, requires_grad=True)
@@ -81,20 +82,24 @@ def _torch_loss(w, batch, F, H, L):
         X[n, torch.as_tensor(cols, dtype=torch.long)] = torch.as_tensor(
             batch.val[batch.row_ptr[n]:batch.row_ptr[n + 1]], dtype=torch.float64)
         labs = batch.lab[batch.lab_ptr[n]:batch.lab_ptr[n + 1]]
-        T[n, torch.as_tensor(labs, dtype=torch.long)] = 1.0 / len(labs)
+        T[n, torch.as_tensor(labs, dtype=torch.long)] = 1.0 / len(labs) if loss_kind == "softmax" else 1.0
     Z = torch.relu(X @ W1 + b1) @ W2.T + b2
-    loss = torch.nn.functional.cross_entropy(Z, T)   # soft targets, batch mean
+    if loss_kind == "softmax":
+        loss = torch.nn.functional.cross_entropy(Z, T)   # soft targets, batch mean
+    else:   # per-label BCE summed over labels, batch mean (R11)
+        loss = torch.nn.functional.binary_cross_entropy_with_logits(Z, T, reduction="sum") / B
     loss.backward()
     return float(loss), wt.grad.numpy()
 
 
+@pytest.mark.parametrize("loss_kind", ["softmax", "sigmoid"])
 @pytest.mark.parametrize("seed_index,B", [(7, 4), (11, 16)])
-def test_against_torch_autograd(seed_index, B):
+def test_against_torch_autograd(seed_index, B, loss_kind):
     cfg = _small(seed_index, n_train=64)
     F, H, L = cfg.F, cfg.H, cfg.L
     _, batch, w = _batch_and_params(cfg, B=B)
-    loss, g = model.loss_and_grad(w, batch, F, H, L)
-    tl, tg = _torch_loss(w, batch, F, H, L)
+    loss, g = model.loss_and_grad(w, batch, F, H, L, loss_kind)
+    tl, tg = _torch_loss(w, batch, F, H, L, loss_kind)
     assert abs(loss - tl) <= 1e-12 * abs(tl)
     assert np.linalg.norm(g - tg) <= 1e-12 * np.linalg.norm(tg)
 
