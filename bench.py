@@ -48,6 +48,8 @@ def _args():
                    help="adaptive: dynamic tickets + Alg. 1/2; elastic: Elastic SGD A/B (static batches, alpha = 1/N)")
     p.add_argument("--merge", default="fused", choices=["fused", "nccl"],
                    help="fused: peer-memory merge kernel over CUDA IPC (NEXT-1); nccl: prescale + all_reduce + epilogue")
+    p.add_argument("--loss", default="softmax", choices=["softmax", "sigmoid"],
+                   help="output head: softmax-CE (the paper's) or per-label sigmoid BCE (R11)")
     p.add_argument("--e2e-steps", type=int, default=None)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -121,7 +123,7 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ CPU oracle
-def cpu_baseline(cfg, data, budget_s: float):
+def cpu_baseline(cfg, data, budget_s: float, loss: str = "softmax"):
     """The oracle as it stands (fp64 numpy/scipy) on the host cores: consecutive
     b_max-row local steps of the same workload plus the per-mega-batch merge,
     amortised over the mega-batch's 100 steps."""
@@ -138,7 +140,7 @@ def cpu_baseline(cfg, data, budget_s: float):
     t0 = time.perf_counter()
     while True:
         rows = sample_stream(cfg, steps * b, b)
-        w, _, _ = omodel.sgd_step(w, data.row_slice(rows), cfg.lr_max, cfg.F, cfg.H, cfg.L)
+        w, _, _ = omodel.sgd_step(w, data.row_slice(rows), cfg.lr_max, cfg.F, cfg.H, cfg.L, loss)
         steps += 1
         samples += b
         if time.perf_counter() - t0 > budget_s:
@@ -155,7 +157,7 @@ def cpu_baseline(cfg, data, budget_s: float):
 
 
 # ------------------------------------------------------------------ roofline
-def kernel_work(cls: str, cfg, bf16: bool, st):
+def kernel_work(cls: str, cfg, bf16: bool, st, loss: str = "softmax"):
     """Algorithmic bytes or flops of one launch of a kernel class."""
     B, H, L, F, P = st["B"], cfg.H, cfg.L, cfg.F, cfg.n_params
     nnz, U = st["nnz"], st["U"]
@@ -166,6 +168,10 @@ def kernel_work(cls: str, cfg, bf16: bool, st):
     if cls == "scatter":
         return ("bytes", 8.0 * nnz + 4.0 * B * H + 8.0 * U * H)
     if cls == "softmax":
+        if loss == "sigmoid":   # fp32: k_sigmoid_ce over stored Z; bf16: k_tile_loss (the BCE is in G1)
+            if bf16:
+                return ("bytes", 8.0 * B * 2 * ((L + 255) // 256) + 4.0 * B)
+            return ("bytes", 8.0 * B * L + 8.0 * st["nlab"])
         if bf16 and cfg.b_max * L * 4 > (64 << 20):   # fused path: k_lse + G1b (Z recomputed on tensor cores)
             return ("flops", 2.0 * B * H * L)
         return ("bytes", (6.0 if bf16 else 8.0) * B * L + 8.0 * st["nlab"])
@@ -218,7 +224,7 @@ def main():
         cfg = config(a.config, n_train=data.n_rows)
     w0 = init_params(cfg)
     nz, nl = api.max_step_sizes([data], cfg.b_max)
-    rep = api.Replica(cfg.F, cfg.L, cfg.H, cfg.b_max, nz, nl, prec, device=local, w0=w0)
+    rep = api.Replica(cfg.F, cfg.L, cfg.H, cfg.b_max, nz, nl, prec, device=local, w0=w0, loss=a.loss)
     dd = api.DeviceCsr(data, device=dev)
     rep.register(dd)
     h = train.Hyper.from_config(cfg)
@@ -312,7 +318,7 @@ def main():
                           "launches": int(wcnt[i])}
                for i in range(len(names))}
         dname = names[dom]
-        kind, work = kernel_work(dname, cfg, bf16, wl)
+        kind, work = kernel_work(dname, cfg, bf16, wl, a.loss)
         avg_s = ms[dom] / max(cnt[dom], 1) / 1e3
         if kind == "flops":
             achieved = work / avg_s / 1e12
@@ -346,7 +352,7 @@ def main():
                        "mega_batch_samples": M, "step": "1 mega-batch = local steps + merge",
                        "precision": prec, "l2": "flushed (256 MiB write) between timed steps",
                        "inflight": a.inflight, "parallelism": f"dp{world} (model averaging)",
-                       "merge": merge_used, "method": a.method,
+                       "merge": merge_used, "method": a.method, "loss": a.loss,
                        "mean_batch_nnz": round(wl["nnz"], 1), "mean_touched_rows": round(wl["U"], 1)},
             "roofline": roof,
             "kernels_warmup_profile": per,
@@ -356,9 +362,9 @@ def main():
             "cpu_baseline": None,
         }
         if world == 1 and a.ttp_megabatches > 0:
-            out["time_to_p1"] = time_to_p1(cfg, prec, a.ttp_megabatches, dev, lr_max=a.lr_max)
+            out["time_to_p1"] = time_to_p1(cfg, prec, a.ttp_megabatches, dev, lr_max=a.lr_max, loss=a.loss)
         if world == 1 and not a.no_cpu_baseline:
-            out["cpu_baseline"], _ = cpu_baseline(cfg, data, a.cpu_seconds)
+            out["cpu_baseline"], _ = cpu_baseline(cfg, data, a.cpu_seconds, a.loss)
         print(json.dumps(out), flush=True)
     if world > 1:
         dist.barrier()
@@ -424,7 +430,7 @@ def run_e2e(rep, drv, data, ids_list, dev, flush, world, M):
             "h2d_bytes_per_step": int(h2d * world / Ke), "d2h_bytes_per_step": int(d2h * world / Ke)}
 
 
-def time_to_p1(cfg, prec, n_mb, dev, pert_renorm=False, lr_max=None, eval_rows=10000):
+def time_to_p1(cfg, prec, n_mb, dev, pert_renorm=False, lr_max=None, eval_rows=10000, loss="softmax"):
     """Time-to-P@1 on one GPU: cumulative CUDA-event time of the
     mega-batches (local steps + merge) until test P@1 first reaches
     floor + 0.9 (best - floor); floor = the majority-label P@1 of the test
@@ -436,7 +442,8 @@ def time_to_p1(cfg, prec, n_mb, dev, pert_renorm=False, lr_max=None, eval_rows=1
     data = generate(cfg, "train")
     test = generate(cfg, "test", eval_rows)
     nz, nl = api.max_step_sizes([data, test], cfg.b_max)
-    rep = api.Replica(cfg.F, cfg.L, cfg.H, cfg.b_max, nz, nl, prec, device=dev.index or 0, w0=init_params(cfg))
+    rep = api.Replica(cfg.F, cfg.L, cfg.H, cfg.b_max, nz, nl, prec, device=dev.index or 0, w0=init_params(cfg),
+                      loss=loss)
     rep.register(api.DeviceCsr(data, device=dev))
     td = api.DeviceCsr(test, device=dev)
     h = train.Hyper.from_config(cfg, pert_renorm=pert_renorm, **({"lr_max": lr_max} if lr_max else {}))
@@ -478,7 +485,7 @@ def reference_arm(a, rank, world):
     vals = []
     base = None
     for k in range(a.warmup + a.steps):
-        cb, _ = cpu_baseline(cfg, data, per_step)
+        cb, _ = cpu_baseline(cfg, data, per_step, a.loss)
         if k >= a.warmup:
             vals.append(cb["value"])
             base = cb
@@ -488,7 +495,7 @@ def reference_arm(a, rank, world):
            "warmup": a.warmup, "ms_per_step": None, "higher_is_better": True, "scaling": "strong",
            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
            "config": {"workload": cfg.name, "F": cfg.F, "L": cfg.L, "H": cfg.H, "b_max": cfg.b_max,
-                      "mega_batch_samples": cfg.mega_batch},
+                      "mega_batch_samples": cfg.mega_batch, "loss": a.loss},
            "cpu_baseline": base,
            "e2e": {"value": round(v, 2), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)

@@ -26,7 +26,10 @@
  *
  * Model (§V-A; D3): a 3-layer MLP  X (B x F, CSR) -> ReLU hidden
  * (H) -> softmax over L labels, cross-entropy loss with the uniform target
- * T_nj = 1/|Y_n| on the true labels (Q3), batch-mean reduction (Q4).  The
+ * T_nj = 1/|Y_n| on the true labels (Q3), batch-mean reduction (Q4); or, with
+ * loss = ASGD_LOSS_SIGMOID, per-label sigmoid binary cross-entropy with 0/1
+ * targets summed over the L labels, batch mean (north_star "softmax/sigmoid
+ * cross-entropy"; reading R11).  The
  * parameters are ONE flat fp32 vector of P = F*H + H + L*H + L entries, in
  * order W1 (F x H row-major, feature-major), b1 (H), W2 (L x H row-major,
  * label-major), b2 (L), so that one all-reduce covers the whole replica.
@@ -55,6 +58,14 @@ extern "C" {
 #define ASGD_PREC_FP32 0
 #define ASGD_PREC_BF16 1
 
+/* Output-layer loss (a5).
+ * ASGD_LOSS_SOFTMAX: loss_n = lse(Z_n) - sum_j T_nj Z_nj, T_nj = 1/|Y_n| on Y_n;
+ *                    dZ = (softmax(Z) - T) / B                      (Q3, Q4).
+ * ASGD_LOSS_SIGMOID: loss_n = sum_j [softplus(Z_nj) - Y_nj Z_nj], Y_nj in {0,1};
+ *                    dZ = (sigmoid(Z) - Y) / B                       (R11). */
+#define ASGD_LOSS_SOFTMAX 0
+#define ASGD_LOSS_SIGMOID 1
+
 typedef struct asgd_ctx asgd_ctx;
 typedef struct asgd_sched asgd_sched;
 
@@ -66,6 +77,8 @@ typedef struct {
   int32_t b_max;          /* max rows of one local step (<= 2048)           */
   int64_t max_step_nnz;   /* max feature nnz of one step's rows             */
   int64_t max_step_labels;/* max label entries of one step's rows           */
+  int32_t loss;           /* ASGD_LOSS_* (0 = softmax-CE, the paper's)      */
+  int32_t reserved;       /* must be 0                                      */
 } asgd_model_desc;
 
 /* A CSR split: features (row_ptr, col, val) and labels (lab_ptr, lab).
@@ -129,7 +142,9 @@ int asgd_data_upload(asgd_ctx* ctx, const asgd_csr* host_src, const asgd_csr* de
  * replica's learning rate lr_i.  Computes, all on the device:
  *   K-0 batch CSR view + touched-feature set (sorted unique cols, segments);
  *   K-1 A1 = X W1 + b1, H1 = ReLU(A1);   G1 Z = H1 W2^T + b2;
- *   softmax-CE: per-row lse, loss, dZ = (softmax(Z) - T)/B;
+ *   softmax-CE: per-row lse, loss, dZ = (softmax(Z) - T)/B  (or, for
+ *   ASGD_LOSS_SIGMOID, dZ = (sigmoid(Z) - Y)/B and the BCE row loss, fused
+ *   into G1's epilogue on the bf16 path);
  *   G2 dH1 = dZ W2 (pre-step W2), dA1 = dH1 * [A1 > 0], b1 -= lr 1^T dA1;
  *   G3 W2 -= lr dZ^T H1, b2 -= lr 1^T dZ;
  *   K-5 W1[f,:] -= lr sum_{n: X_nf != 0} X_nf dA1[n,:] on touched f only.

@@ -16,13 +16,15 @@ HEADER = os.path.join(_HERE, "..", "include", "asgd.h")
 
 OK, E_ARG, E_SHAPE, E_CUDA, E_STATE, E_UNSUPPORTED = 0, 1, 2, 3, 4, 5
 PREC_FP32, PREC_BF16 = 0, 1
+LOSS_SOFTMAX, LOSS_SIGMOID = 0, 1
 PEER_HANDLE_BYTES = 160   # ASGD_PEER_HANDLE_BYTES
 PROF_NAMES = ["touched", "spmm", "g1", "softmax", "g2", "dh_b1", "b2", "g3", "scatter", "merge"]
 
 
 class ModelDesc(C.Structure):
     _fields_ = [("F", C.c_int64), ("L", C.c_int64), ("H", C.c_int64), ("precision", C.c_int32),
-                ("b_max", C.c_int32), ("max_step_nnz", C.c_int64), ("max_step_labels", C.c_int64)]
+                ("b_max", C.c_int32), ("max_step_nnz", C.c_int64), ("max_step_labels", C.c_int64),
+                ("loss", C.c_int32), ("reserved", C.c_int32)]
 
 
 class Csr(C.Structure):

@@ -16,6 +16,7 @@ from . import _lib
 from ._lib import Csr, ModelDesc, call, lib
 
 PRECISIONS = {"fp32": _lib.PREC_FP32, "bf16": _lib.PREC_BF16}
+LOSSES = {"softmax": _lib.LOSS_SOFTMAX, "sigmoid": _lib.LOSS_SIGMOID}
 
 
 def _ptr(t) -> int:
@@ -80,13 +81,14 @@ class Replica:
 
     def __init__(self, F: int, L: int, H: int, b_max: int, max_step_nnz: int, max_step_labels: int,
                  precision: str = "fp32", device: int = 0, w0=None, stream=None,
-                 share_global: Optional["Replica"] = None):
+                 share_global: Optional["Replica"] = None, loss: str = "softmax"):
         self.F, self.L, self.H, self.b_max = F, L, H, b_max
         self.P = F * H + H + L * H + L
         self.device = torch.device("cuda", device)
         self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
-        self.desc = ModelDesc(F, L, H, PRECISIONS[precision], b_max, max_step_nnz, max_step_labels)
-        self.precision = precision
+        self.desc = ModelDesc(F, L, H, PRECISIONS[precision], b_max, max_step_nnz, max_step_labels,
+                              LOSSES[loss], 0)
+        self.precision, self.loss = precision, loss
         ws_bytes = lib().asgd_workspace_bytes(C.byref(self.desc))
         if ws_bytes == 0:
             raise _lib.AsgdError("asgd_workspace_bytes", _lib.E_SHAPE, "bad model desc")

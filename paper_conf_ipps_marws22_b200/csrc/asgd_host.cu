@@ -119,7 +119,7 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.da1b = take(bf ? (size_t)B * H * 2 : 0);
   L.stats_ld = B;
   L.lse = take(B * 4);
-  L.zstat = take(bf ? (size_t)((Lb + 31) / 32 + 2) * B * 8 : 0);   // G1 softmax partials (2 per N tile)
+  L.zstat = take(bf ? (size_t)((Lb + 31) / 32 + 8) * B * 8 : 0);   // G1 partials (2 or 4 per N tile)
   L.rowloss = take(B * 4);
   L.dhpart = take((size_t)L.splitk * B * H * 4);
   L.da1 = take(B * H * 4);
@@ -331,6 +331,8 @@ int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device, v
                 (long long)m.L, m.b_max, (long long)m.max_step_nnz);
   if (m.precision != ASGD_PREC_FP32 && m.precision != ASGD_PREC_BF16)
     return fail(ASGD_E_ARG, "precision %d", m.precision);
+  if ((m.loss != ASGD_LOSS_SOFTMAX && m.loss != ASGD_LOSS_SIGMOID) || m.reserved != 0)
+    return fail(ASGD_E_ARG, "loss %d / reserved %d", m.loss, m.reserved);
   const size_t need = ws_layout(m).total;
   if (ws_bytes < need) return fail(ASGD_E_SHAPE, "workspace %zu < %zu bytes", ws_bytes, need);
   CU(cudaSetDevice(device));
@@ -495,7 +497,10 @@ int enqueue_step(asgd_ctx* c, int n) {
     a.B = W2; a.bs0 = 1; a.bs1 = H;
     a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = Lp; a.bias = b2; a.splitk = 1;
     PCU(ASGD_K_G1, launch_gemm_f32(lc, a));
-    PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, false));
+    if (m.loss == ASGD_LOSS_SIGMOID)
+      PCU(ASGD_K_SOFTMAX, launch_sigmoid_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, false));
+    else
+      PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, false));
     // G2: dH1 partials = dZ W2 (pre-step W2)
     a = GemmArgs{};
     a.M = n; a.N = H; a.K = (int)Lb;
@@ -535,7 +540,13 @@ int enqueue_step(asgd_ctx* c, int n) {
     if (2 * g2c <= c->sms) lc3.sms = c->sms - g2c;
     float2* zstat = reinterpret_cast<float2*>(c->ws + c->L.zstat);
     int ntiles = 0;
-    if ((int64_t)m.b_max * Lb * 4 <= kFusedCeBytes) {
+    if (m.loss == ASGD_LOSS_SIGMOID) {
+      // sigmoid-BCE needs no row normaliser: G1's epilogue writes dZ (bf16) and per-tile
+      // row-loss partials directly, Z never stored, at every L (R11)
+      PCU(ASGD_K_G1, launch_gemm_tc(lc, 6, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles, P.rowsc,
+                                    x.lab_ptr, x.lab));
+      PCU(ASGD_K_SOFTMAX, launch_tile_loss(lc, n, ntiles, c->L.stats_ld, zstat, P));
+    } else if ((int64_t)m.b_max * Lb * 4 <= kFusedCeBytes) {
       // logits fit in L2: G1 stores Z (+ per-tile softmax partials), one pass of softmax-CE
       PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
       PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, true, zstat, ntiles,

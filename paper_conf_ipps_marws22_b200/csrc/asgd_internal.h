@@ -144,6 +144,11 @@ cudaError_t launch_softmax_ce(const Launch&, int n, int64_t L, int64_t ldz, cons
                               const int64_t* lab_ptr, const int32_t* lab, const Ptrs&,
                               bool bf16_out, const float2* stats = nullptr, int ntiles = 0,
                               int64_t stats_ld = 0);
+// Sigmoid-BCE (R11) over the stored Z (fp32 path): row loss, dZ = (sigmoid(Z) - Y)/B.
+cudaError_t launch_sigmoid_ce(const Launch&, int n, int64_t L, int64_t ldz, const int32_t* rows,
+                              const int64_t* lab_ptr, const int32_t* lab, const Ptrs&, bool bf16_out);
+// Row loss of the fused sigmoid path from G1's per-(tile half, row) BCE partials.
+cudaError_t launch_tile_loss(const Launch&, int n, int ntiles, int64_t stats_ld, const float2* stats, const Ptrs&);
 cudaError_t launch_dh_reduce(const Launch&, int n, int H, int splitk, const Ptrs&, const WsLayout&,
                              bool want_bf16);
 cudaError_t launch_b1_update(const Launch&, int n, int H, float* b1, const Ptrs&,
@@ -165,6 +170,8 @@ cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int 
 int gemm_tc_g2_ctas(int n, int H, const WsLayout&, int sms);
 // which = 4 (G1b): dZ = (softmax - T)/B from a recomputed Z tile; needs P.lse from k_lse.
 // which = 5: G1 without storing Z (only the softmax partials), for the fused path.
+// which = 6: G1 with the sigmoid-BCE epilogue (R11): dZ = (sigmoid(Z) - Y)/B stored bf16,
+//            per-(tile half, row) loss partials in stats; Z never stored.
 cudaError_t launch_lse(const Launch&, int n, int H, int ntiles, int64_t stats_ld, const float2* stats,
                        const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab, const bf16* h1b,
                        const bf16* w2b, const float* b2, const Ptrs&);

@@ -204,6 +204,97 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
   }
 }
 
+// ------------------------------------------------------- sigmoid + BCE (R11)
+// One CTA per batch row n (fp32 path, Z stored): per-label binary cross-entropy
+// with 0/1 targets, loss_n = sum_j softplus(Z_nj) - sum_{y in Y_n} Z_ny;
+// dZ_nj = (sigmoid(Z_nj) - Y_nj) / B, written in place (or as bf16).
+__device__ __forceinline__ float softplus_f(float z) { return fmaxf(z, 0.f) + log1pf(expf(-fabsf(z))); }
+__device__ __forceinline__ float sigmoid_f(float z) {
+  const float e = expf(-fabsf(z));
+  return z >= 0.f ? 1.f / (1.f + e) : e / (1.f + e);
+}
+
+__global__ void __launch_bounds__(512) k_sigmoid_ce(int B, int64_t L, int64_t ldz,
+                                                    const int32_t* __restrict__ rows,
+                                                    const int64_t* __restrict__ lab_ptr,
+                                                    const int32_t* __restrict__ lab, float* Z,
+                                                    bf16* dZb, float* rowloss) {
+  pdl_trigger();
+  pdl_wait();
+  __shared__ int s_lab[kMaxRowLabels];
+  __shared__ float s_lz[kMaxRowLabels];
+  __shared__ float s_sp[16];
+  const int n = blockIdx.x;
+  const int64_t id = rows[n];
+  const int64_t l0 = lab_ptr[id];
+  const int64_t nl64 = lab_ptr[id + 1] - l0;
+  const int nl = (int)(nl64 < kMaxRowLabels ? nl64 : kMaxRowLabels);
+  float* z = Z + (int64_t)n * ldz;
+  for (int i = threadIdx.x; i < nl; i += blockDim.x) {
+    const int y = lab[l0 + i];
+    s_lab[i] = y;
+    s_lz[i] = z[y];
+  }
+  __syncthreads();   // label logits are read before dZ overwrites Z
+  const float invB = 1.f / (float)B;
+  constexpr int kSU = 8;
+  float sp = 0.f;
+  bf16* d = dZb ? dZb + (int64_t)n * ldz : nullptr;
+  for (int64_t j0 = threadIdx.x; j0 < L; j0 += (int64_t)kSU * blockDim.x) {
+    float v[kSU];
+#pragma unroll
+    for (int k = 0; k < kSU; ++k) {
+      const int64_t j = j0 + (int64_t)k * blockDim.x;
+      v[k] = j < L ? z[j] : 0.f;
+    }
+#pragma unroll
+    for (int k = 0; k < kSU; ++k) {
+      const int64_t j = j0 + (int64_t)k * blockDim.x;
+      if (j < L) {
+        sp += softplus_f(v[k]);
+        const float g = sigmoid_f(v[k]) * invB;
+        if (d) d[j] = __float2bfloat16_rn(g); else z[j] = g;
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) sp += __shfl_xor_sync(kFull, sp, o);
+  const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) s_sp[wid] = sp;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float S = 0.f, ls = 0.f;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) S += s_sp[w];
+    for (int i = 0; i < nl; ++i) ls += s_lz[i];
+    rowloss[n] = S - ls;
+  }
+  for (int i = threadIdx.x; i < nl; i += blockDim.x) {
+    const float g = (sigmoid_f(s_lz[i]) - 1.f) * invB;
+    if (d) d[s_lab[i]] = __float2bfloat16_rn(g); else z[s_lab[i]] = g;
+  }
+}
+
+// Row loss of the fused sigmoid path: rowloss[n] = sum over G1's column tiles t
+// of the per-(tile half, row) BCE partials stats[t][n].x, in tile order.
+__global__ void __launch_bounds__(256) k_tile_loss(int ntiles, int64_t stats_ld, const float2* __restrict__ stats,
+                                                   float* rowloss) {
+  pdl_trigger();
+  pdl_wait();
+  __shared__ float s_w[8];
+  const int n = blockIdx.x;
+  float a = 0.f;
+  for (int t = threadIdx.x; t < ntiles; t += blockDim.x) a += stats[(int64_t)t * stats_ld + n].x;
+#pragma unroll
+  for (int o = 16; o; o >>= 1) a += __shfl_xor_sync(kFull, a, o);
+  if ((threadIdx.x & 31) == 0) s_w[threadIdx.x >> 5] = a;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float S = 0.f;
+    for (int w = 0; w < 8; ++w) S += s_w[w];
+    rowloss[n] = S;
+  }
+}
+
 // ------------------------------------------------------------ fused CE: lse
 // lse_n from G1's per-tile (max, sum exp) partials; the label logits
 // Z_ny = H1_n . W2_y + b2_y (bf16 operands, fp32 sum, as on the tensor cores);
@@ -386,6 +477,17 @@ cudaError_t launch_softmax_ce(const Launch& lc, int n, int64_t L, int64_t ldz, c
   launch_k(lc, k_softmax_ce, dim3(n), dim3(512), 0, n, L, ldz, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
                                     P.rowloss, stats, ntiles, stats_ld);
   return cudaGetLastError();
+}
+
+cudaError_t launch_sigmoid_ce(const Launch& lc, int n, int64_t L, int64_t ldz, const int32_t* rows,
+                              const int64_t* lab_ptr, const int32_t* lab, const Ptrs& P, bool bf16_out) {
+  launch_k(lc, k_sigmoid_ce, dim3(n), dim3(512), 0, n, L, ldz, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
+           P.rowloss);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tile_loss(const Launch& lc, int n, int ntiles, int64_t stats_ld, const float2* stats, const Ptrs& P) {
+  return launch_k(lc, k_tile_loss, dim3(n), dim3(256), 0, ntiles, stats_ld, stats, P.rowloss);
 }
 
 cudaError_t launch_lse(const Launch& lc, int n, int H, int ntiles, int64_t stats_ld, const float2* stats,

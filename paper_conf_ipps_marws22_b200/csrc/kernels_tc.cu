@@ -22,7 +22,9 @@ namespace {
 
 constexpr int BM = 128, BK = 64;
 
-enum { TC_EPI_Z = 0, TC_EPI_PART = 1, TC_EPI_SGD = 2, TC_EPI_DZ = 3 };
+// Z: fp32 Z store (+ softmax partials); PART: split-K partial store; SGD: W2 update;
+// DZ: softmax dZ (bf16); SIG: sigmoid dZ (bf16) + BCE partials; STATS: softmax partials only
+enum { TC_EPI_Z = 0, TC_EPI_PART = 1, TC_EPI_SGD = 2, TC_EPI_DZ = 3, TC_EPI_SIG = 4, TC_EPI_STATS = 5 };
 
 struct TcArgs {
   int M, N, K;
@@ -36,7 +38,8 @@ struct TcArgs {
   int splits;                         // split-K factor (tiles = M tiles x N tiles x splits)
   int n_fast;                         // tile order: N tiles vary fastest (else M tiles)
   int write_z;                        // G1: store Z (eval) or only the softmax partials (step)
-  // G1b (TC_EPI_DZ): dZ = (exp(Z - lse) - T) / B recomputed from the MMA, stored bf16
+  // G1b (TC_EPI_DZ): dZ = (exp(Z - lse) - T) / B recomputed from the MMA, stored bf16;
+  // G1 sigmoid (TC_EPI_SIG): dZ = (sigmoid(Z) - Y) / B, BCE row partials in stats
   const float* lse; const int32_t* rows; const int64_t* lab_ptr; const int32_t* lab; float invB;
 };
 
@@ -139,6 +142,26 @@ __device__ __forceinline__ float ex2_approx(float x) {   // 2^x on the MUFU (ex2
   return y;
 }
 
+__device__ __forceinline__ float rcp_approx(float x) {
+  float y;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+
+// log1p(x) for x in [0, 1] on the FMA pipe: degree-8 Chebyshev fit, |error| < 2e-7
+// (keeps the sigmoid epilogue at 2 MUFU ops per element: ex2 and rcp).
+__device__ __forceinline__ float log1p_01(float x) {
+  float p = -0.0060747526586055756f;
+  p = fmaf(p, x, 0.03441791236400604f);
+  p = fmaf(p, x, -0.09231230616569519f);
+  p = fmaf(p, x, 0.16478188335895538f);
+  p = fmaf(p, x, -0.2391897290945053f);
+  p = fmaf(p, x, 0.3313336670398712f);
+  p = fmaf(p, x, -0.4998010993003845f);
+  p = fmaf(p, x, 0.9999914765357971f);
+  return fmaf(p, x, 9.099033349002639e-08f);
+}
+
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -149,22 +172,33 @@ constexpr uint32_t pow2ceil(uint32_t x) {
   return p;
 }
 
-// Persistent tcgen05 GEMM.  CTA = 12 warps: warp 0 TMA producer, warp 1 MMA
-// issuer, warp 2 TMEM allocator, warps 4-11 epilogue (warp w drains TMEM lanes
-// 32 (w % 4) .. + 31, column half (w - 4) / 4).  Tiles (M fastest, or N fastest
+// Persistent tcgen05 GEMM.  CTA = 4 + E warps: warp 0 TMA producer, warp 1 MMA
+// issuer, warp 2 TMEM allocator, warps 4..3+E epilogue (warp w drains TMEM lanes
+// 32 (w % 4) .. + 31, column group (w - 4) / 4 of E / 4).  E = 16 for the
+// MUFU-heavy softmax / sigmoid epilogues on wide tiles (4 warps per scheduler
+// hide the exp latency), else 8.  Tiles (M fastest, or N fastest
 // when g.n_fast) are strided over the grid; the smem ring (full/empty mbarriers)
 // and the TMEM accumulators (tfull/tempty, double-buffered when 2 fit in 512
 // columns) carry across tiles, so a tile's epilogue overlaps the next tile's
 // loads and MMAs.
+template <int BN, int EPI>
+constexpr int epi_warps() {
+  return (BN >= 128 && (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG || EPI == TC_EPI_STATS)) ? 16 : 8;
+}
 template <int EPI>
-constexpr int stages_of() { return EPI == 2 ? 3 : ((EPI == 0 || EPI == 3) ? 2 : 3); }
+constexpr int stages_of() { return EPI == TC_EPI_STATS ? 4 : (EPI == TC_EPI_Z ? 2 : 3); }
 template <int EPI>
-constexpr uint32_t staging_bytes() {   // per epilogue warp: 2 x 4 KB fp32 boxes (+ 2 x 2 KB bf16 for G3)
-  return EPI == 2 ? 8u * 12288u : 8u * 2u * 4096u;
+constexpr uint32_t box_bytes() {   // one 32 x 32 store box: fp32 (Z, PART) or bf16 (DZ, SIG)
+  return (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG) ? 2048u : 4096u;
+}
+template <int BN, int EPI>
+constexpr uint32_t staging_bytes() {   // per epilogue warp: 2 store boxes (G3: 2 x (4 KB fp32 + 2 KB bf16) + pad)
+  return EPI == TC_EPI_SGD ? 8u * 12288u
+                           : (EPI == TC_EPI_STATS ? 1024u : (uint32_t)epi_warps<BN, EPI>() * 2u * box_bytes<EPI>());
 }
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
-__global__ void __launch_bounds__(384, 1)
+__global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
     k_gemm_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
               const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmD, TcArgs g) {
   constexpr int STAGES = stages_of<EPI>();
@@ -174,14 +208,18 @@ __global__ void __launch_bounds__(384, 1)
   constexpr int NACC = (2 * ACC_COLS <= 512) ? 2 : 1;
   constexpr uint32_t TMEM_COLS = pow2ceil(NACC * ACC_COLS);
   constexpr uint32_t ONES_BYTES = ONES ? 16 * 128 : 0; // K-major 16 x 64 bf16 tile, row 0 = 1
-  constexpr int EPI_WARPS = 8;
+  constexpr int EPI_WARPS = epi_warps<BN, EPI>();
+  constexpr int NQ = EPI_WARPS / 4;      // column groups
+  constexpr int CW = BN / NQ;            // columns per epilogue warp
+  static_assert(CW % 32 == 0, "epilogue chunks are 32 columns");
+  constexpr uint32_t BOX = box_bytes<EPI>();
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + STAGES * A_BYTES;
   uint8_t* sOnes = smem + STAGES * STAGE;
   uint8_t* sStg = smem + STAGES * STAGE + ONES_BYTES;   // TMA-store staging (1024-aligned)
-  uint64_t* full = reinterpret_cast<uint64_t*>(sStg + staging_bytes<EPI>());
+  uint64_t* full = reinterpret_cast<uint64_t*>(sStg + staging_bytes<BN, EPI>());
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
   uint64_t* tempty = tfull + 2;
@@ -315,20 +353,20 @@ __global__ void __launch_bounds__(384, 1)
       float st_m = -INFINITY, st_s = 0.f;   // G1 softmax partials of row m over this column half
       float lse_m = 0.f, tinv = 0.f;        // G1b: row m's lse and 1 / (|Y_m| B)
       int64_t lab_cur = 0, lab_end = 0;
-      if constexpr (EPI == TC_EPI_DZ) {
+      if constexpr (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG) {
         if (m < g.M) {
-          lse_m = g.lse[m];
+          if constexpr (EPI == TC_EPI_DZ) lse_m = g.lse[m];
           const int64_t id = g.rows[m];
           lab_cur = g.lab_ptr[id];
           lab_end = g.lab_ptr[id + 1];
           tinv = g.invB / (float)(lab_end - lab_cur);
           // skip labels left of this warp's first column
-          const int cfirst = n0 + wh * (BN / 2);
+          const int cfirst = n0 + wh * CW;
           while (lab_cur < lab_end && g.lab[lab_cur] < cfirst) ++lab_cur;
         }
       }
 #pragma unroll 1
-      for (int c = wh * (BN / 2); c < (wh + 1) * (BN / 2); c += 32) {
+      for (int c = wh * CW; c < (wh + 1) * CW; c += 32) {
         float v[32];
         if (nk > 0) {
           tmem_ld32(d + (uint32_t)c, v);
@@ -338,34 +376,66 @@ __global__ void __launch_bounds__(384, 1)
         }
         const int n = n0 + c;
         if (n >= g.N) continue;   // warp-uniform
-        if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_DZ) {
-          const float bl = n + lane < g.N ? __ldg(g.bias + n + lane) : 0.f;
+        if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_DZ || EPI == TC_EPI_SIG || EPI == TC_EPI_STATS) {
+          // + b2 (the same 32 values for every lane: broadcast vector loads); columns >= N -> -inf
+          if (n + 32 <= g.N) {
+            const float4* b4 = reinterpret_cast<const float4*>(g.bias + n);
 #pragma unroll
-          for (int j = 0; j < 32; ++j) {
-            v[j] += __shfl_sync(0xffffffffu, bl, j);
-            if (n + j >= g.N) v[j] = -INFINITY;
+            for (int q = 0; q < 8; ++q) {
+              const float4 t = __ldg(b4 + q);
+              v[4 * q] += t.x; v[4 * q + 1] += t.y; v[4 * q + 2] += t.z; v[4 * q + 3] += t.w;
+            }
+          } else {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) v[j] = n + j < g.N ? v[j] + __ldg(g.bias + n + j) : -INFINITY;
           }
         }
-        if constexpr (EPI == TC_EPI_DZ) {
-          // softmax - uniform target over the row's labels (Q3), / B (Q4); labels are sorted,
-          // lab_cur walks forward as this warp's columns increase
+        if constexpr (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG) {
           constexpr float kL2E = 1.4426950408889634f;
-          const float ls = lse_m * kL2E;
+          if constexpr (EPI == TC_EPI_DZ) {
+            // softmax - uniform target over the row's labels (Q3), / B (Q4); labels are sorted,
+            // lab_cur walks forward as this warp's columns increase
+            const float ls = lse_m * kL2E;
 #pragma unroll
-          for (int j = 0; j < 32; ++j) v[j] = ex2_approx(fmaf(v[j], kL2E, -ls)) * g.invB;
-          while (lab_cur < lab_end) {
-            const int y = g.lab[lab_cur];
-            if (y >= n + 32) break;
-            if (y >= n) {
-              const int jy = y - n;
+            for (int j = 0; j < 32; ++j) v[j] = ex2_approx(fmaf(v[j], kL2E, -ls)) * g.invB;
+            while (lab_cur < lab_end) {
+              const int y = g.lab[lab_cur];
+              if (y >= n + 32) break;
+              if (y >= n) {
+                const int jy = y - n;
 #pragma unroll
-              for (int j = 0; j < 32; ++j)
-                if (j == jy) v[j] -= tinv;
+                for (int j = 0; j < 32; ++j)
+                  if (j == jy) v[j] -= tinv;
+              }
+              ++lab_cur;
             }
-            ++lab_cur;
+          } else {
+            // sigmoid BCE (R11): dZ = (sigmoid(z) - y) / B; row partial += softplus(z) - y z.
+            // e = exp(-|z|) in (0, 1]; sigmoid(|z|) = 1 / (1 + e); softplus(z) = max(z, 0) + log1p(e).
+            // Padding columns carry z = -inf: e = 0, sigmoid = 0, softplus = 0.
+            uint32_t ym = 0;   // label columns of this 32-column chunk (labels sorted)
+            while (lab_cur < lab_end) {
+              const int y = g.lab[lab_cur];
+              if (y >= n + 32) break;
+              if (y >= n) ym |= 1u << (y - n);
+              ++lab_cur;
+            }
+            float a0 = 0.f, a1 = 0.f;
+#pragma unroll
+            for (int j = 0; j < 32; ++j) {
+              const float z = v[j];
+              const float e = ex2_approx(-fabsf(z) * kL2E);
+              const float r = rcp_approx(1.f + e);
+              const float sg = z >= 0.f ? r : e * r;
+              const float sp = fmaxf(z, 0.f) + log1p_01(e);
+              const bool y = (ym >> j) & 1u;
+              if (j & 1) a1 += y ? sp - z : sp; else a0 += y ? sp - z : sp;
+              v[j] = (y ? sg - 1.f : sg) * g.invB;
+            }
+            st_s += a0 + a1;
           }
           // stage a 32 x 32 bf16 box (64B swizzle) and TMA-store it into dZ
-          uint8_t* buf = sStg + ((warp - 4) * 2 + sbuf) * 4096;
+          uint8_t* buf = sStg + ((warp - 4) * 2 + sbuf) * BOX;
           if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
           __syncwarp();
 #pragma unroll
@@ -388,7 +458,7 @@ __global__ void __launch_bounds__(384, 1)
           sbuf ^= 1;
           continue;
         }
-        if constexpr (EPI == TC_EPI_Z) {
+        if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_STATS) {
           if (g.stats) {   // online (max, sum exp) of row m over the columns seen so far
             float cm = v[0];
 #pragma unroll
@@ -407,13 +477,11 @@ __global__ void __launch_bounds__(384, 1)
             st_s += (a0 + a1) + (a2 + a3);
           }
         }
-        if constexpr (EPI == TC_EPI_Z) {
-          if (!g.write_z) continue;   // step: only the softmax partials are needed
-        }
+        if constexpr (EPI == TC_EPI_STATS) continue;   // step: only the softmax partials are needed
         if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_PART) {
           // stage the warp's 32 x 32 fp32 box (128B swizzle: conflict-free) and TMA-store it;
           // rows >= M / columns >= N are clipped by the tensor map
-          uint8_t* buf = sStg + ((warp - 4) * 2 + sbuf) * 4096;
+          uint8_t* buf = sStg + ((warp - 4) * 2 + sbuf) * BOX;
           if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
           __syncwarp();
 #pragma unroll
@@ -479,8 +547,11 @@ __global__ void __launch_bounds__(384, 1)
           }
         }
       }
-      if constexpr (EPI == TC_EPI_Z) {
-        if (g.stats && m < g.M) g.stats[(int64_t)(nt * 2 + wh) * g.stats_ld + m] = make_float2(st_m, st_s);
+      if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_STATS) {
+        if (g.stats && m < g.M) g.stats[(int64_t)(nt * NQ + wh) * g.stats_ld + m] = make_float2(st_m, st_s);
+      }
+      if constexpr (EPI == TC_EPI_SIG) {
+        if (m < g.M) g.stats[(int64_t)(nt * NQ + wh) * g.stats_ld + m] = make_float2(st_s, 0.f);
       }
       if constexpr (ONES) {
         if (nt == 0 && wh == 0) {   // db2[m] = sum_n dZ[n, m]; b2 -= lr db2
@@ -567,7 +638,7 @@ template <int BN, bool A_MN, bool B_MN, int EPI>
 cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c,
                const CUtensorMap& d, TcArgs g, int splits) {
   const size_t smem = (size_t)stages_of<EPI>() * (BM * BK * 2 + BN * BK * 2) + (EPI == TC_EPI_SGD ? 2048 : 0) +
-                      staging_bytes<EPI>() + 1024 + 512;
+                      staging_bytes<BN, EPI>() + 1024 + 512;
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(k_gemm_tc<BN, A_MN, B_MN, EPI>,
@@ -578,7 +649,8 @@ cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, co
   g.splits = splits;
   const int64_t tiles = (int64_t)((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN) * splits;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, lc.sms));
-  return launch_k(lc, k_gemm_tc<BN, A_MN, B_MN, EPI>, dim3(grid), dim3(384), smem, a, b, c, d, g);
+  return launch_k(lc, k_gemm_tc<BN, A_MN, B_MN, EPI>, dim3(grid), dim3(128 + 32 * epi_warps<BN, EPI>()), smem, a, b,
+                  c, d, g);
 }
 
 // Widest N tile that still gives >= one CTA per SM (and does not overhang N by 2x).
@@ -618,21 +690,37 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
     const int bn = pick_bn((n + BM - 1) / BM, L, lc.sms);
     g.stats = stats; g.stats_ld = W.stats_ld;
     g.write_z = which == 1;
-    if (stats_ntiles) *stats_ntiles = (int)(2 * ((L + bn - 1) / bn));   // two column halves per tile
+    // per tile, one partial per epilogue column group
+    const int nq = which == 1 ? 2 : (bn >= 128 ? 4 : 2);
+    if (stats_ntiles) *stats_ntiles = (int)(nq * ((L + bn - 1) / bn));
     if ((e = make_map(&ta, P.h1b, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
     if ((e = make_map(&tb, P.w2b, H, L, (uint64_t)H * 2, 64, bn)) != cudaSuccess) return e;
     if ((e = make_store_map(&tc, P.z, L, n, (uint64_t)Lp * 4, 1, 0, 2)) != cudaSuccess) return e;
+    if (which == 5) {
+      if (bn == 256) return run<256, false, false, TC_EPI_STATS>(lc, ta, tb, tc, tc, g, 1);
+      if (bn == 128) return run<128, false, false, TC_EPI_STATS>(lc, ta, tb, tc, tc, g, 1);
+      return run<64, false, false, TC_EPI_STATS>(lc, ta, tb, tc, tc, g, 1);
+    }
     if (bn == 256) return run<256, false, false, TC_EPI_Z>(lc, ta, tb, tc, tc, g, 1);
     if (bn == 128) return run<128, false, false, TC_EPI_Z>(lc, ta, tb, tc, tc, g, 1);
     return run<64, false, false, TC_EPI_Z>(lc, ta, tb, tc, tc, g, 1);
   }
-  if (which == 4) {  // G1b: dZ (bf16) = (softmax(H1 W2^T + b2) - T) / B, recomputed tile by tile
+  if (which == 4 || which == 6) {
+    // 4 (G1b): dZ (bf16) = (softmax(H1 W2^T + b2) - T) / B, recomputed tile by tile;
+    // 6 (G1 sigmoid): dZ (bf16) = (sigmoid(H1 W2^T + b2) - Y) / B + BCE row partials
     g.M = n; g.N = (int)L; g.K = H;
     g.bias = b2; g.lse = P.lse; g.rows = dz_rows; g.lab_ptr = dz_lab_ptr; g.lab = dz_lab; g.invB = 1.f / (float)n;
     const int bn = pick_bn((n + BM - 1) / BM, L, lc.sms);
     if ((e = make_map(&ta, P.h1b, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
     if ((e = make_map(&tb, P.w2b, H, L, (uint64_t)H * 2, 64, bn)) != cudaSuccess) return e;
     if ((e = make_bf16_store_map(&tc, P.dzb, L, n, (uint64_t)Lp * 2)) != cudaSuccess) return e;
+    if (which == 6) {
+      g.stats = stats; g.stats_ld = W.stats_ld;
+      if (stats_ntiles) *stats_ntiles = (int)((bn >= 128 ? 4 : 2) * ((L + bn - 1) / bn));
+      if (bn == 256) return run<256, false, false, TC_EPI_SIG>(lc, ta, tb, tc, tc, g, 1);
+      if (bn == 128) return run<128, false, false, TC_EPI_SIG>(lc, ta, tb, tc, tc, g, 1);
+      return run<64, false, false, TC_EPI_SIG>(lc, ta, tb, tc, tc, g, 1);
+    }
     if (bn == 256) return run<256, false, false, TC_EPI_DZ>(lc, ta, tb, tc, tc, g, 1);
     if (bn == 128) return run<128, false, false, TC_EPI_DZ>(lc, ta, tb, tc, tc, g, 1);
     return run<64, false, false, TC_EPI_DZ>(lc, ta, tb, tc, tc, g, 1);

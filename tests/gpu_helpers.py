@@ -29,13 +29,13 @@ def split_grad(g, F, H, L):
     return out
 
 
-def make_replica(cfg, data, precision="fp32", w0=None, b_max=None, extra=()):
+def make_replica(cfg, data, precision="fp32", w0=None, b_max=None, extra=(), loss="softmax"):
     from paper_conf_ipps_marws22_b200 import api
     b_max = b_max or cfg.b_max
     nz, nl = api.max_step_sizes([data, *extra], b_max)
     if w0 is None:
         w0 = init_params(cfg)
-    rep = api.Replica(cfg.F, cfg.L, cfg.H, b_max, nz, nl, precision, w0=w0)
+    rep = api.Replica(cfg.F, cfg.L, cfg.H, b_max, nz, nl, precision, w0=w0, loss=loss)
     dd = api.DeviceCsr(data)
     rep.register(dd)
     rep._keep_data = dd

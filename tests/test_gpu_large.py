@@ -16,25 +16,25 @@ pytestmark = pytest.mark.gpu
 TOL = {"fp32": 1e-4, "bf16": 2e-2}
 
 
-def _chunked_oracle(w, batch, F, H, L, chunk):
+def _chunked_oracle(w, batch, F, H, L, chunk, loss_kind="softmax"):
     B = batch.n_rows
     loss, g = 0.0, None
     for r0 in range(0, B, chunk):
         sub = batch.row_slice(np.arange(r0, min(B, r0 + chunk)))
-        lo, go = omodel.loss_and_grad(w, sub, F, H, L)
+        lo, go = omodel.loss_and_grad(w, sub, F, H, L, loss_kind)
         f = sub.n_rows / B
         loss += f * lo
         g = f * go if g is None else g + f * go
     return loss, g
 
 
-def _check_big(name, n_rows, precision, chunk, seed_pos=0):
+def _check_big(name, n_rows, precision, chunk, seed_pos=0, loss_kind="softmax"):
     cfg = config(name)
     data = dataset(name, n_rows)
     cfg_sub = config(name, n_train=data.n_rows)
     rows = sample_stream(cfg_sub, seed_pos, cfg.b_max)
     w0 = init_params(cfg)
-    rep = make_replica(cfg, data, precision, w0=w0)
+    rep = make_replica(cfg, data, precision, w0=w0, loss=loss_kind)
     g = torch.zeros(rep.P, dtype=torch.float32, device="cuda")
     loss = torch.zeros(1, dtype=torch.float32, device="cuda")
     rep.set_debug_grads(g)
@@ -42,7 +42,7 @@ def _check_big(name, n_rows, precision, chunk, seed_pos=0):
     rep.sync()
     touched = rep.last_touched().cpu().numpy()
     batch = data.row_slice(rows)
-    lo, go = _chunked_oracle(w0.astype(np.float64), batch, cfg.F, cfg.H, cfg.L, chunk)
+    lo, go = _chunked_oracle(w0.astype(np.float64), batch, cfg.F, cfg.H, cfg.L, chunk, loss_kind)
     tol = TOL[precision]
     assert abs(loss.item() - lo) <= tol * abs(lo)
     np.testing.assert_array_equal(touched, omodel.touched_features(batch))
@@ -69,3 +69,8 @@ def test_wiki10_full_split_bench_launch():
 def test_delicious200k_bench_launch():
     """NEXT-3: F = 782,585 (800 MB of W1), L = 205,443, 75 labels per row."""
     _check_big("delicious200k", 8192, "bf16", chunk=128)
+
+
+def test_amazon670k_sigmoid_bench_launch():
+    """Sigmoid-BCE head (R11) at L = 670,091: one G1 pass writes dZ, no lse pass."""
+    _check_big("amazon670k", 16384, "bf16", chunk=128, loss_kind="sigmoid")

@@ -16,8 +16,8 @@ pytestmark = pytest.mark.gpu
 TOL = {"fp32": 1e-4, "bf16": 2e-2}
 
 
-def _one_step(cfg, data, rows, precision, lr=0.5, w0=None, b_max=None):
-    rep = make_replica(cfg, data, precision, w0=w0, b_max=b_max)
+def _one_step(cfg, data, rows, precision, lr=0.5, w0=None, b_max=None, loss_kind="softmax"):
+    rep = make_replica(cfg, data, precision, w0=w0, b_max=b_max, loss=loss_kind)
     w0 = init_params(cfg) if w0 is None else w0
     g = torch.zeros(rep.P, dtype=torch.float32, device="cuda")
     loss = torch.zeros(1, dtype=torch.float32, device="cuda")
@@ -27,7 +27,7 @@ def _one_step(cfg, data, rows, precision, lr=0.5, w0=None, b_max=None):
     rep.sync()
     touched = rep.last_touched().cpu().numpy()
     batch = data.row_slice(rows)
-    lo, go = omodel.loss_and_grad(np.asarray(w0, dtype=np.float64), batch, cfg.F, cfg.H, cfg.L)
+    lo, go = omodel.loss_and_grad(np.asarray(w0, dtype=np.float64), batch, cfg.F, cfg.H, cfg.L, loss_kind)
     return rep, g.cpu().numpy(), float(loss.item()), touched, lo, go, batch
 
 
@@ -114,3 +114,31 @@ def test_teacher_forced_steps_tiny():
         assert normwise(g.cpu().numpy(), go) <= 1e-4
         w_after = rep.params.cpu().numpy().astype(np.float64)
         assert normwise(w_after, w_before - 0.7 * go) <= 1e-6
+
+
+# ---------------------------------------------------------------- sigmoid-BCE head (R11)
+@pytest.mark.parametrize("precision", ["fp32", "bf16"])
+@pytest.mark.parametrize("name", ["tiny", "eurlex4k"])
+def test_step_sigmoid_bce(name, precision):
+    """loss = ASGD_LOSS_SIGMOID: per-label BCE (R11); bf16 fuses it into G1's epilogue."""
+    cfg = config(name)
+    data = dataset(name)
+    rows = sample_stream(cfg, 0, cfg.b_max)
+    _check(cfg, *_one_step(cfg, data, rows, precision, loss_kind="sigmoid"), precision)
+
+
+@pytest.mark.parametrize("precision", ["fp32", "bf16"])
+def test_step_sigmoid_ragged_trained(precision):
+    """Ragged batch (37 rows, an empty and a repeated row) from a model whose logits are
+    far from 0 (W2 and b2 scaled up), so both sigmoid branches and the saturated softplus
+    tail are exercised."""
+    cfg = config("eurlex4k")
+    data = with_empty_row(dataset("eurlex4k"), 5)
+    rows = np.array([5, 0, 17, 5, 1000] + list(range(2000, 2032)), dtype=np.int32)
+    w0 = init_params(cfg).astype(np.float64)
+    F, H, L = cfg.F, cfg.H, cfg.L
+    o2 = F * H + H
+    w0[o2:o2 + L * H] *= 40.0
+    w0[o2 + L * H:] = np.linspace(-12.0, 6.0, L)
+    w0 = w0.astype(np.float32)
+    _check(cfg, *_one_step(cfg, data, rows, precision, w0=w0, loss_kind="sigmoid"), precision)
