@@ -129,6 +129,8 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.red = take((L.n_red + 8) * 8);
   L.eval_top = take(B * 8 * 4);
   L.rowsc = take(B * 4);
+  L.cen = take(bf ? (size_t)2 * H * 4 : 0);
+  L.cenpart = take(bf ? (size_t)2 * kCenterParts * H * 4 : 0);
   L.total = o;
   return L;
 }
@@ -151,6 +153,8 @@ Ptrs ws_ptrs(char* b, const WsLayout& L) {
   p.da1b = (bf16*)(b + L.da1b);
   p.lse = (float*)(b + L.lse);
   p.rowsc = (int32_t*)(b + L.rowsc);
+  p.cen = (float*)(b + L.cen);
+  p.cenpart = (float*)(b + L.cenpart);
   return p;
 }
 
@@ -545,7 +549,12 @@ int enqueue_step(asgd_ctx* c, int n) {
       // row-loss partials directly, Z never stored, at every L (R11)
       PCU(ASGD_K_G1, launch_gemm_tc(lc, 6, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles, P.rowsc,
                                     x.lab_ptr, x.lab));
-      PCU(ASGD_K_SOFTMAX, launch_tile_loss(lc, n, ntiles, c->L.stats_ld, zstat, P));
+      PCU(ASGD_K_SOFTMAX, ([&]() -> cudaError_t {
+            cudaError_t e = launch_tile_loss(lc, n, ntiles, c->L.stats_ld, zstat, P);
+            return e != cudaSuccess ? e
+                                    : launch_sig_center(lc, Pr.w2b, Lb, H, P.h1, n, P.cenpart,
+                                                        reinterpret_cast<unsigned int*>(P.meta + M_CEN), P.cen);
+          })());
     } else if ((int64_t)m.b_max * Lb * 4 <= kFusedCeBytes) {
       // logits fit in L2: G1 stores Z (+ per-tile softmax partials), one pass of softmax-CE
       PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
@@ -565,10 +574,12 @@ int enqueue_step(asgd_ctx* c, int n) {
     }
     CU(cudaEventRecord(c->ev_sm, c->s));
     CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
+    const bool centred = m.loss == ASGD_LOSS_SIGMOID;   // G1 stored dZ - 1/(2B) (R11)
     PCU_ON(c->s3, ASGD_K_G3, launch_gemm_tc(lc3, 3, n, Lb, H, Pw, c->L, W2, b2, g ? g + c->o_w2 : nullptr,
-                                            g ? g + c->o_b2 : nullptr));
+                                            g ? g + c->o_b2 : nullptr, nullptr, nullptr, nullptr, nullptr, nullptr,
+                                            centred ? P.cen + H : nullptr));
     PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr));
-    PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, true));
+    PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, true, centred ? P.cen : nullptr));
     CU(cudaEventRecord(c->ev_dh, c->s));
     CU(cudaStreamWaitEvent(c->s3, c->ev_dh, 0));
     PCU_ON(c->s3, ASGD_K_DH, launch_b1_update(lc3, n, H, b1, P, c->L, g ? g + c->o_b1 : nullptr));

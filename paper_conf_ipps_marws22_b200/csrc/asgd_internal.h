@@ -22,7 +22,7 @@ constexpr int kScanTile = 1024;
 // M_K0PAR: parity of K-0's double-buffered tile sums.
 // M_MSYNC: fused merge arrival counter (64-bit, slots 40-41), M_MDONE: its CTA counter.
 enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_LR = 6, M_K0PAR = 7, M_COUNT = 8,
-       M_LOSS = 10, M_BAR = 32, M_MSYNC = 40, M_MDONE = 42 };
+       M_LOSS = 10, M_BAR = 32, M_MSYNC = 40, M_MDONE = 42, M_CEN = 44 };
 // error bits in meta[M_ERR]
 enum { ERR_NNZ_CAP = 1, ERR_LAB_CAP = 2, ERR_ROW_ID = 4 };
 
@@ -33,7 +33,7 @@ struct WsLayout {
   size_t meta, boff, loff, cnt, fseg, fuid, uniq, useg, tsum, tpre;
   size_t e_n, e_v, e_u, e_f, part1, rowcnt, part5, ucnt, bits;
   size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, b2part, rbase, da1b, zstat, lse;
-  size_t rowsc;
+  size_t rowsc, cen, cenpart;
   size_t total;
   int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride, stats_ld;
 };
@@ -50,6 +50,8 @@ struct Ptrs {  // typed views of the workspace
   bf16* da1b;       // bf16 copy of dA1 (bf16 path; staged by K-5)
   float* lse;       // per-row log-sum-exp of Z (bf16 path)
   int32_t* rowsc;   // copy of the step's dataset row ids (written by K-0 (a))
+  float* cen;       // centred sigmoid offsets [2 H] (bf16 path, R11)
+  float* cenpart;   // their per-CTA partials [kCenterParts H]
 };
 __device__ __forceinline__ float step_lr(const int32_t* meta) { return __int_as_float(meta[M_LR]); }
 __device__ __forceinline__ float* step_loss(const int32_t* meta) {
@@ -150,7 +152,12 @@ cudaError_t launch_sigmoid_ce(const Launch&, int n, int64_t L, int64_t ldz, cons
 // Row loss of the fused sigmoid path from G1's per-(tile half, row) BCE partials.
 cudaError_t launch_tile_loss(const Launch&, int n, int ntiles, int64_t stats_ld, const float2* stats, const Ptrs&);
 cudaError_t launch_dh_reduce(const Launch&, int n, int H, int splitk, const Ptrs&, const WsLayout&,
-                             bool want_bf16);
+                             bool want_bf16, const float* dh_off = nullptr);
+// Centred sigmoid dZ (R11): cen[0:H] = (1/(2B)) sum_j W2_j (bf16 shadow, the dH1 offset),
+// cen[H:2H] = (1/(2B)) sum_n H1_n (the dW2 offset).  part: fp32[2 parts H]; counter: zeroed.
+cudaError_t launch_sig_center(const Launch&, const bf16* w2b, int64_t L, int H, const float* h1, int n, float* part,
+                              unsigned int* counter, float* cen);
+constexpr int kCenterParts = 148;
 cudaError_t launch_b1_update(const Launch&, int n, int H, float* b1, const Ptrs&,
                              const WsLayout&, float* grad_b1);
 cudaError_t launch_b2_update(const Launch&, int n, int64_t L, int64_t ldz, float* b2,
@@ -165,7 +172,7 @@ cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int 
                            const Ptrs&, const WsLayout&, float* W2, float* b2, float* grad_w2,
                            float* grad_b2, float2* stats = nullptr, int* stats_ntiles = nullptr,
                            const int32_t* dz_rows = nullptr, const int64_t* dz_lab_ptr = nullptr,
-                           const int32_t* dz_lab = nullptr);
+                           const int32_t* dz_lab = nullptr, const float* hoff = nullptr);
 // CTAs G2 runs with (the concurrent G3 leaves those SMs to it).
 int gemm_tc_g2_ctas(int n, int H, const WsLayout&, int sms);
 // which = 4 (G1b): dZ = (softmax - T)/B from a recomputed Z tile; needs P.lse from k_lse.

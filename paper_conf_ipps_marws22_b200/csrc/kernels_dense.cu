@@ -295,6 +295,89 @@ __global__ void __launch_bounds__(256) k_tile_loss(int ntiles, int64_t stats_ld,
   }
 }
 
+// ------------------------------------------ centred sigmoid dZ offsets (R11)
+// G1 stores dZc = dZ - 1/(2B) (bf16 keeps the z-dependent part near sigmoid = 1/2);
+// the constant comes back exactly through
+//   dH1 = dZc W2 + (1/(2B)) 1 (1^T W2)     -> cen[0:H]  = (1/(2B)) sum_j W2_j
+//   dW2 = dZc^T H1 + (1/(2B)) 1 (1^T H1)   -> cen[H:2H] = (1/(2B)) sum_n H1_n
+// (db2's + 1/2 is G3's).  W2 is the bf16 shadow G2 multiplies with.  Phase 1: each
+// CTA sums a contiguous label range (8 columns per thread, 16-B loads, 4 in
+// flight); phase 2: the last CTA adds the partials in CTA order (deterministic).
+__global__ void __launch_bounds__(256) k_sig_center(const bf16* __restrict__ w2b, int64_t L, int H,
+                                                    const float* __restrict__ h1, int n, float* part,
+                                                    unsigned int* counter, float* cen) {
+  pdl_trigger();
+  pdl_wait();
+  __shared__ float s_acc[8][512];
+  __shared__ bool s_last;
+  const int tpr = H / 8;                   // threads per W2 row (H <= 512 -> <= 64)
+  const int rows_per_it = 256 / tpr;
+  const int c8 = (threadIdx.x % tpr) * 8, r0 = threadIdx.x / tpr;
+  const int64_t j0 = (int64_t)blockIdx.x * L / gridDim.x, j1 = (int64_t)(blockIdx.x + 1) * L / gridDim.x;
+  float a[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+  int64_t j = j0 + r0;
+  for (; j + 3 * rows_per_it < j1; j += 4 * rows_per_it) {
+    uint4 u[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) u[q] = __ldcs(reinterpret_cast<const uint4*>(w2b + (j + q * rows_per_it) * H + c8));
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const __nv_bfloat162* b = reinterpret_cast<const __nv_bfloat162*>(&u[q]);
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const float2 f = __bfloat1622float2(b[i]);
+        a[2 * i] += f.x; a[2 * i + 1] += f.y;
+      }
+    }
+  }
+  for (; j < j1; j += rows_per_it) {
+    const uint4 u = __ldcs(reinterpret_cast<const uint4*>(w2b + j * H + c8));
+    const __nv_bfloat162* b = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float2 f = __bfloat1622float2(b[i]);
+      a[2 * i] += f.x; a[2 * i + 1] += f.y;
+    }
+  }
+  // combine the rows_per_it row groups of this CTA in fixed order
+  const int grp = r0 & 7, sub = r0 >> 3;   // <= 8 groups per pass
+  for (int pass = 0; pass * 8 < rows_per_it; ++pass) {
+    if (sub == pass)
+      for (int i = 0; i < 8; ++i) s_acc[grp][c8 + i] = (pass == 0 ? 0.f : s_acc[grp][c8 + i]) + a[i];
+    __syncthreads();
+  }
+  // this CTA's slice of the batch rows of H1 (fp32), rows in order
+  const int n0 = (int)((int64_t)blockIdx.x * n / gridDim.x), n1 = (int)((int64_t)(blockIdx.x + 1) * n / gridDim.x);
+  float* part2 = part + (int64_t)gridDim.x * H;
+  for (int c = threadIdx.x; c < H; c += blockDim.x) {
+    float t = 0.f;
+    for (int g = 0; g < min(8, rows_per_it); ++g) t += s_acc[g][c];
+    part[(int64_t)blockIdx.x * H + c] = t;
+    float hs = 0.f;
+    for (int r = n0; r < n1; ++r) hs += h1[(int64_t)r * H + c];
+    part2[(int64_t)blockIdx.x * H + c] = hs;
+  }
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) s_last = atomicAdd(counter, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  const float o = 0.5f / (float)n;
+  for (int c = threadIdx.x; c < 2 * H; c += blockDim.x) {   // both sums, partials in CTA order
+    const float* pp = (c < H ? part : part2) + (c % H);
+    float t[4] = {0.f, 0.f, 0.f, 0.f};
+    int b = 0;
+    for (; b + 4 <= (int)gridDim.x; b += 4) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) t[q] += __ldcg(pp + (int64_t)(b + q) * H);
+    }
+    for (; b < (int)gridDim.x; ++b) t[0] += __ldcg(pp + (int64_t)b * H);
+    cen[c] = o * ((t[0] + t[1]) + (t[2] + t[3]));
+  }
+  if (threadIdx.x == 0) *counter = 0u;
+}
+
 // ------------------------------------------------------------ fused CE: lse
 // lse_n from G1's per-tile (max, sum exp) partials; the label logits
 // Z_ny = H1_n . W2_y + b2_y (bf16 operands, fp32 sum, as on the tensor cores);
@@ -358,7 +441,7 @@ __global__ void __launch_bounds__(256) k_lse(int H, int ntiles, int64_t stats_ld
 // split-K loads all in flight; fixed summation order (deterministic).
 __global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
                             const float* __restrict__ part, const float* __restrict__ H1, float* dA1,
-                            bf16* dA1b) {
+                            bf16* dA1b, const float* __restrict__ dh_off) {
   pdl_trigger();
   pdl_wait();
   const int r = blockIdx.x, c = threadIdx.x;
@@ -371,7 +454,8 @@ __global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
     for (int q = 0; q < 8; ++q)
       if (z + q < splitk) a[q] += __ldcs(part + (int64_t)(z + q) * part_stride + o);
   }
-  const float s = ((a[0] + a[1]) + (a[2] + a[3])) + ((a[4] + a[5]) + (a[6] + a[7]));
+  float s = ((a[0] + a[1]) + (a[2] + a[3])) + ((a[4] + a[5]) + (a[6] + a[7]));
+  if (dh_off) s += dh_off[c];   // centred sigmoid dZ: + (1/(2B)) sum_j W2_j
   const float v = H1[o] > 0.f ? s : 0.f;
   dA1[o] = v;
   if (dA1b) dA1b[o] = __float2bfloat16_rn(v);
@@ -490,6 +574,11 @@ cudaError_t launch_tile_loss(const Launch& lc, int n, int ntiles, int64_t stats_
   return launch_k(lc, k_tile_loss, dim3(n), dim3(256), 0, ntiles, stats_ld, stats, P.rowloss);
 }
 
+cudaError_t launch_sig_center(const Launch& lc, const bf16* w2b, int64_t L, int H, const float* h1, int n, float* part,
+                              unsigned int* counter, float* cen) {
+  return launch_k(lc, k_sig_center, dim3(kCenterParts), dim3(256), 0, w2b, L, H, h1, n, part, counter, cen);
+}
+
 cudaError_t launch_lse(const Launch& lc, int n, int H, int ntiles, int64_t stats_ld, const float2* stats,
                        const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab, const bf16* h1b,
                        const bf16* w2b, const float* b2, const Ptrs& P) {
@@ -498,10 +587,10 @@ cudaError_t launch_lse(const Launch& lc, int n, int H, int ntiles, int64_t stats
 }
 
 cudaError_t launch_dh_reduce(const Launch& lc, int n, int H, int splitk, const Ptrs& P,
-                             const WsLayout& L, bool want_bf16) {
+                             const WsLayout& L, bool want_bf16, const float* dh_off) {
   // split-K partial z of dH1 lives at dhpart + z * (b_max * H)
   launch_k(lc, k_dh_reduce, dim3(n), dim3(H), 0, n, H, splitk, L.part_stride, P.dhpart, P.h1, P.da1,
-                  want_bf16 ? P.da1b : nullptr);
+                  want_bf16 ? P.da1b : nullptr, dh_off);
   return cudaGetLastError();
 }
 

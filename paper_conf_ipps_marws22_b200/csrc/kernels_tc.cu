@@ -37,7 +37,13 @@ struct TcArgs {
   float2* stats; int64_t stats_ld;    // G1: per (N-tile half, row) softmax partials (max, sum exp)
   int splits;                         // split-K factor (tiles = M tiles x N tiles x splits)
   int n_fast;                         // tile order: N tiles vary fastest (else M tiles)
+  int chunked;                        // CTA c runs the contiguous tiles [c T / G, (c + 1) T / G) in
+                                      // M-major order (N fastest): its rows change at most once or
+                                      // twice, and the G CTAs sweep the N tiles in lockstep per M
+                                      // tile, so every W2 tile is read from HBM about once
   int write_z;                        // G1: store Z (eval) or only the softmax partials (step)
+  // G3, centred sigmoid dZ (R11): dW2 += hoff (per H column: (1/(2B)) sum_n H1_n), db2 += db2_off
+  const float* hoff; float db2_off;
   // G1b (TC_EPI_DZ): dZ = (exp(Z - lse) - T) / B recomputed from the MMA, stored bf16;
   // G1 sigmoid (TC_EPI_SIG): dZ = (sigmoid(Z) - Y) / B, BCE row partials in stats
   const float* lse; const int32_t* rows; const int64_t* lab_ptr; const int32_t* lab; float invB;
@@ -191,6 +197,14 @@ template <int EPI>
 constexpr uint32_t box_bytes() {   // one 32 x 32 store box: fp32 (Z, PART) or bf16 (DZ, SIG)
   return (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG) ? 2048u : 4096u;
 }
+template <int EPI>
+constexpr bool has_bias() {
+  return EPI == TC_EPI_Z || EPI == TC_EPI_DZ || EPI == TC_EPI_SIG || EPI == TC_EPI_STATS;
+}
+template <int BN, int EPI>
+constexpr uint32_t bias_bytes() {   // per epilogue warp: its tile columns' b2 (smem broadcast copy)
+  return has_bias<EPI>() ? (uint32_t)epi_warps<BN, EPI>() * (uint32_t)(BN / (epi_warps<BN, EPI>() / 4)) * 4u : 0u;
+}
 template <int BN, int EPI>
 constexpr uint32_t staging_bytes() {   // per epilogue warp: 2 store boxes (G3: 2 x (4 KB fp32 + 2 KB bf16) + pad)
   return EPI == TC_EPI_SGD ? 8u * 12288u
@@ -219,7 +233,8 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
   uint8_t* sB = smem + STAGES * A_BYTES;
   uint8_t* sOnes = smem + STAGES * STAGE;
   uint8_t* sStg = smem + STAGES * STAGE + ONES_BYTES;   // TMA-store staging (1024-aligned)
-  uint64_t* full = reinterpret_cast<uint64_t*>(sStg + staging_bytes<BN, EPI>());
+  float* sBias = reinterpret_cast<float*>(sStg + staging_bytes<BN, EPI>());
+  uint64_t* full = reinterpret_cast<uint64_t*>(sStg + staging_bytes<BN, EPI>() + bias_bytes<BN, EPI>());
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
   uint64_t* tempty = tfull + 2;
@@ -232,8 +247,12 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
   const int T = MT * NT * Z;
   const int nkb = (g.K + BK - 1) / BK;
   const int per = (nkb + Z - 1) / Z;
+  // this CTA's tiles: t = t_first, t_first + t_step, ... < t_end
+  const int t_first = g.chunked ? (int)((int64_t)blockIdx.x * T / gridDim.x) : (int)blockIdx.x;
+  const int t_end = g.chunked ? (int)((int64_t)(blockIdx.x + 1) * T / gridDim.x) : T;
+  const int t_step = g.chunked ? 1 : (int)gridDim.x;
   auto decode = [&](int t, int& mt, int& nt, int& z, int& kb0, int& nk) {
-    if (g.n_fast) { nt = t % NT; mt = (t / NT) % MT; } else { mt = t % MT; nt = (t / MT) % NT; }
+    if (g.n_fast || g.chunked) { nt = t % NT; mt = (t / NT) % MT; } else { mt = t % MT; nt = (t / MT) % NT; }
     z = t / (MT * NT);
     kb0 = z * per;
     nk = max(0, min(nkb, kb0 + per) - kb0);
@@ -271,7 +290,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
     if (lane == 0) {
       // ------------------------------------------------ TMA producer
       int it = 0;
-      for (int t = blockIdx.x; t < T; t += gridDim.x) {
+      for (int t = t_first; t < t_end; t += t_step) {
         int mt, nt, z, kb0, nk;
         decode(t, mt, nt, z, kb0, nk);
         const int m0 = mt * BM, n0 = nt * BN;
@@ -305,7 +324,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
       constexpr uint32_t idesc1 = make_idesc(16, A_MN, false);
       const uint32_t ones_base = smem_u32(sOnes);
       int it = 0, tl = 0;
-      for (int t = blockIdx.x; t < T; t += gridDim.x, ++tl) {
+      for (int t = t_first; t < t_end; t += t_step, ++tl) {
         int mt, nt, z, kb0, nk;
         decode(t, mt, nt, z, kb0, nk);
         const int acc = tl % NACC;
@@ -336,35 +355,55 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
       }
     }
   } else if (warp >= 4) {
-    // ------------------------------------------------ epilogue (8 warps)
+    // ------------------------------------------------ epilogue (EPI_WARPS warps)
     const int wq = (warp - 4) & 3, wh = (warp - 4) >> 2;
     const float lr = EPI == TC_EPI_SGD ? step_lr(g.meta) : 0.f;
     int tl = 0, sbuf = 0, kc = 0;
-    for (int t = blockIdx.x; t < T; t += gridDim.x, ++tl) {
+    // G1b / sigmoid: row m's lse, 1 / (|Y_m| B) and label cursor, kept while the tile's M
+    // block does not change (chunked order: N increases, so the cursor only moves forward)
+    int row_mt = -1;
+    float lse_m = 0.f, tinv = 0.f;
+    int64_t lab_cur = 0, lab_end = 0;
+    float* bias_w = sBias + (has_bias<EPI>() ? (warp - 4) * CW : 0);
+    for (int t = t_first; t < t_end; t += t_step, ++tl) {
       int mt, nt, z, kb0, nk;
       decode(t, mt, nt, z, kb0, nk);
       const int m0 = mt * BM, n0 = nt * BN;
       const int acc = tl % NACC;
       const uint32_t aph = (tl / NACC) & 1;
+      const int m = m0 + wq * 32 + lane;
+      // before waiting for the accumulator: this warp's b2 columns into smem (coalesced
+      // loads, read back below as broadcast float4) and the row state of a new M block
+      if constexpr (has_bias<EPI>()) {
+        __syncwarp();
+#pragma unroll
+        for (int c = 0; c < CW; c += 32) {
+          const int col = n0 + wh * CW + c + lane;
+          bias_w[c + lane] = col < g.N ? __ldg(g.bias + col) : 0.f;
+        }
+        __syncwarp();
+      }
+      if constexpr (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG) {
+        if (mt != row_mt) {
+          row_mt = mt;
+          lab_cur = lab_end = 0;
+          if (m < g.M) {
+            if constexpr (EPI == TC_EPI_DZ) lse_m = g.lse[m];
+            const int64_t id = g.rows[m];
+            lab_cur = g.lab_ptr[id];
+            lab_end = g.lab_ptr[id + 1];
+            tinv = g.invB / (float)(lab_end - lab_cur);
+          }
+        }
+        // skip labels left of this warp's first column (cursor is monotone within an M block
+        // in the chunked order; a restart at a lower column would need the full walk)
+        const int cfirst = n0 + wh * CW;
+        while (lab_cur < lab_end && g.lab[lab_cur] < cfirst) ++lab_cur;
+      }
       mbar_wait(&tfull[acc], aph);
       tc_fence_after();
       const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS) + ((uint32_t)(wq * 32) << 16);
-      const int m = m0 + wq * 32 + lane;
-      float st_m = -INFINITY, st_s = 0.f;   // G1 softmax partials of row m over this column half
-      float lse_m = 0.f, tinv = 0.f;        // G1b: row m's lse and 1 / (|Y_m| B)
-      int64_t lab_cur = 0, lab_end = 0;
-      if constexpr (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG) {
-        if (m < g.M) {
-          if constexpr (EPI == TC_EPI_DZ) lse_m = g.lse[m];
-          const int64_t id = g.rows[m];
-          lab_cur = g.lab_ptr[id];
-          lab_end = g.lab_ptr[id + 1];
-          tinv = g.invB / (float)(lab_end - lab_cur);
-          // skip labels left of this warp's first column
-          const int cfirst = n0 + wh * CW;
-          while (lab_cur < lab_end && g.lab[lab_cur] < cfirst) ++lab_cur;
-        }
-      }
+      float st_m = -INFINITY, st_s = 0.f;   // G1 softmax partials of row m over this column group
 #pragma unroll 1
       for (int c = wh * CW; c < (wh + 1) * CW; c += 32) {
         float v[32];
@@ -377,17 +416,17 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
         const int n = n0 + c;
         if (n >= g.N) continue;   // warp-uniform
         if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_DZ || EPI == TC_EPI_SIG || EPI == TC_EPI_STATS) {
-          // + b2 (the same 32 values for every lane: broadcast vector loads); columns >= N -> -inf
-          if (n + 32 <= g.N) {
-            const float4* b4 = reinterpret_cast<const float4*>(g.bias + n);
+          // + b2 (the same 32 values for every lane: broadcast smem reads); columns >= N -> -inf
+          const float4* b4 = reinterpret_cast<const float4*>(bias_w + (c - wh * CW));
 #pragma unroll
-            for (int q = 0; q < 8; ++q) {
-              const float4 t = __ldg(b4 + q);
-              v[4 * q] += t.x; v[4 * q + 1] += t.y; v[4 * q + 2] += t.z; v[4 * q + 3] += t.w;
-            }
-          } else {
+          for (int q = 0; q < 8; ++q) {
+            const float4 t = b4[q];
+            v[4 * q] += t.x; v[4 * q + 1] += t.y; v[4 * q + 2] += t.z; v[4 * q + 3] += t.w;
+          }
+          if (n + 32 > g.N) {
 #pragma unroll
-            for (int j = 0; j < 32; ++j) v[j] = n + j < g.N ? v[j] + __ldg(g.bias + n + j) : -INFINITY;
+            for (int j = 0; j < 32; ++j)
+              if (n + j >= g.N) v[j] = -INFINITY;
           }
         }
         if constexpr (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG) {
@@ -410,9 +449,13 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
               ++lab_cur;
             }
           } else {
-            // sigmoid BCE (R11): dZ = (sigmoid(z) - y) / B; row partial += softplus(z) - y z.
-            // e = exp(-|z|) in (0, 1]; sigmoid(|z|) = 1 / (1 + e); softplus(z) = max(z, 0) + log1p(e).
-            // Padding columns carry z = -inf: e = 0, sigmoid = 0, softplus = 0.
+            // sigmoid BCE (R11): row partial += softplus(z) - y z; dZ is stored CENTRED,
+            // dZc = (sigmoid(z) - 1/2 - y) / B: near initialisation sigmoid(z) = 1/2 + z/4 with
+            // |z| ~ 1e-3, and bf16(sigmoid / B) would round the z-dependent part away.  The
+            // constant 1/(2B) is added back exactly by k_sig_center (dH1, dW2) and G3 (db2).
+            // e = exp(-|z|) in (0, 1]; sigmoid(|z|) - 1/2 = (1 - e) / (2 (1 + e));
+            // softplus(z) = max(z, 0) + log1p(e).  Padding columns carry z = -inf: e = 0,
+            // softplus = 0 (their dZ is clipped by the store).
             uint32_t ym = 0;   // label columns of this 32-column chunk (labels sorted)
             while (lab_cur < lab_end) {
               const int y = g.lab[lab_cur];
@@ -426,11 +469,12 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
               const float z = v[j];
               const float e = ex2_approx(-fabsf(z) * kL2E);
               const float r = rcp_approx(1.f + e);
-              const float sg = z >= 0.f ? r : e * r;
+              const float ch = 0.5f * (1.f - e) * r;              // sigmoid(|z|) - 1/2
+              const float cz = z >= 0.f ? ch : -ch;               // sigmoid(z) - 1/2
               const float sp = fmaxf(z, 0.f) + log1p_01(e);
               const bool y = (ym >> j) & 1u;
               if (j & 1) a1 += y ? sp - z : sp; else a0 += y ? sp - z : sp;
-              v[j] = (y ? sg - 1.f : sg) * g.invB;
+              v[j] = (y ? cz - 1.f : cz) * g.invB;
             }
             st_s += a0 + a1;
           }
@@ -518,6 +562,14 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
             tma_load_2d(wb, &tmC, wl, n, row0);   // rows >= L are zero-filled
           }
           mbar_wait(wl, ph);
+          if (g.hoff) {   // centred sigmoid dZ: dW2[m][h] += (1/(2B)) sum_n H1[n][h]
+            const float4* h4 = reinterpret_cast<const float4*>(g.hoff + n);
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+              const float4 t = __ldg(h4 + q);
+              v[4 * q] += t.x; v[4 * q + 1] += t.y; v[4 * q + 2] += t.z; v[4 * q + 3] += t.w;
+            }
+          }
 #pragma unroll
           for (int q = 0; q < 8; ++q) {
             float4* p = reinterpret_cast<float4*>(wb + lane * 128 + ((q ^ (lane & 7)) * 16));
@@ -562,8 +614,9 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
             v[0] = 0.f;
           }
           if (m < g.M) {
-            g.b2[m] -= lr * v[0];
-            if (g.grad_b2) g.grad_b2[m] = v[0];
+            const float db = v[0] + g.db2_off;
+            g.b2[m] -= lr * db;
+            if (g.grad_b2) g.grad_b2[m] = db;
           }
         }
       }
@@ -638,7 +691,7 @@ template <int BN, bool A_MN, bool B_MN, int EPI>
 cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c,
                const CUtensorMap& d, TcArgs g, int splits) {
   const size_t smem = (size_t)stages_of<EPI>() * (BM * BK * 2 + BN * BK * 2) + (EPI == TC_EPI_SGD ? 2048 : 0) +
-                      staging_bytes<BN, EPI>() + 1024 + 512;
+                      staging_bytes<BN, EPI>() + bias_bytes<BN, EPI>() + 1024 + 512;
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(k_gemm_tc<BN, A_MN, B_MN, EPI>,
@@ -678,7 +731,7 @@ int64_t padded_ld(int64_t L) { return (L + 7) / 8 * 8; }
 cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H, const Ptrs& P,
                            const WsLayout& W, float* W2, float* b2, float* grad_w2, float* grad_b2,
                            float2* stats, int* stats_ntiles, const int32_t* dz_rows,
-                           const int64_t* dz_lab_ptr, const int32_t* dz_lab) {
+                           const int64_t* dz_lab_ptr, const int32_t* dz_lab, const float* hoff) {
   if (!tc_available()) return cudaErrorNotSupported;
   const int64_t Lp = padded_ld(L);
   CUtensorMap ta, tb, tc;
@@ -690,6 +743,7 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
     const int bn = pick_bn((n + BM - 1) / BM, L, lc.sms);
     g.stats = stats; g.stats_ld = W.stats_ld;
     g.write_z = which == 1;
+    g.chunked = 1;
     // per tile, one partial per epilogue column group
     const int nq = which == 1 ? 2 : (bn >= 128 ? 4 : 2);
     if (stats_ntiles) *stats_ntiles = (int)(nq * ((L + bn - 1) / bn));
@@ -710,6 +764,7 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
     // 6 (G1 sigmoid): dZ (bf16) = (sigmoid(H1 W2^T + b2) - Y) / B + BCE row partials
     g.M = n; g.N = (int)L; g.K = H;
     g.bias = b2; g.lse = P.lse; g.rows = dz_rows; g.lab_ptr = dz_lab_ptr; g.lab = dz_lab; g.invB = 1.f / (float)n;
+    g.chunked = 1;
     const int bn = pick_bn((n + BM - 1) / BM, L, lc.sms);
     if ((e = make_map(&ta, P.h1b, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
     if ((e = make_map(&tb, P.w2b, H, L, (uint64_t)H * 2, 64, bn)) != cudaSuccess) return e;
@@ -745,6 +800,7 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
   g.M = (int)L; g.N = H; g.K = n;
   g.out = W2; g.ldo = H; g.meta = P.meta; g.shadow = P.w2b; g.grad = grad_w2;
   g.b2 = b2; g.grad_b2 = grad_b2;
+  g.hoff = hoff; g.db2_off = hoff ? 0.5f : 0.f;   // centred sigmoid dZ: sum_n 1/(2B) = 1/2
   if ((e = make_map(&ta, P.dzb, L, n, (uint64_t)Lp * 2, 64, 64)) != cudaSuccess) return e;
   if ((e = make_map(&tb, P.h1b, H, n, (uint64_t)H * 2, 64, 64)) != cudaSuccess) return e;
   // N tiles of one M tile run back to back (n_fast), so the dZ^T tile is read
