@@ -192,7 +192,9 @@ constexpr int epi_warps() {
   return (BN >= 128 && (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG || EPI == TC_EPI_STATS)) ? 16 : 8;
 }
 template <int EPI>
-constexpr int stages_of() { return EPI == TC_EPI_STATS ? 4 : (EPI == TC_EPI_Z ? 2 : 3); }
+constexpr int stages_of() {   // G3 streams dZ^T from HBM: the deepest ring (its epilogue needs no smem)
+  return EPI == TC_EPI_SGD ? 5 : (EPI == TC_EPI_STATS ? 4 : (EPI == TC_EPI_Z ? 2 : 3));
+}
 template <int EPI>
 constexpr uint32_t box_bytes() {   // one 32 x 32 store box: fp32 (Z, PART) or bf16 (DZ, SIG)
   return (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG) ? 2048u : 4096u;
@@ -207,8 +209,9 @@ constexpr uint32_t bias_bytes() {   // per epilogue warp: its tile columns' b2 (
 }
 template <int BN, int EPI>
 constexpr uint32_t staging_bytes() {   // per epilogue warp: 2 store boxes (G3: 2 x (4 KB fp32 + 2 KB bf16) + pad)
-  return EPI == TC_EPI_SGD ? 8u * 12288u
-                           : (EPI == TC_EPI_STATS ? 1024u : (uint32_t)epi_warps<BN, EPI>() * 2u * box_bytes<EPI>());
+  return EPI == TC_EPI_STATS ? 0u
+                             : (EPI == TC_EPI_SGD ? 8u * 4096u   // per warp: one 32 x 32 fp32 transpose tile
+                                                  : (uint32_t)epi_warps<BN, EPI>() * 2u * box_bytes<EPI>());
 }
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
@@ -238,8 +241,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
   uint64_t* tempty = tfull + 2;
-  uint64_t* wbar = tempty + 2;   // G3: per epilogue warp, 2 W2-box load barriers
-  uint32_t* tbase = reinterpret_cast<uint32_t*>(wbar + 16);
+  uint32_t* tbase = reinterpret_cast<uint32_t*>(tempty + 2);
 
   pdl_trigger();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -263,8 +265,6 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
     for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
     for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], EPI_WARPS); }
-    if constexpr (EPI == TC_EPI_SGD)
-      for (int a = 0; a < 16; ++a) mbar_init(&wbar[a], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
@@ -358,7 +358,8 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
     // ------------------------------------------------ epilogue (EPI_WARPS warps)
     const int wq = (warp - 4) & 3, wh = (warp - 4) >> 2;
     const float lr = EPI == TC_EPI_SGD ? step_lr(g.meta) : 0.f;
-    int tl = 0, sbuf = 0, kc = 0;
+    int tl = 0, sbuf = 0;
+    static_assert(EPI != TC_EPI_SGD || CW <= 64, "G3: at most 2 W2 row segments per warp per tile");
     // G1b / sigmoid: row m's lse, 1 / (|Y_m| B) and label cursor, kept while the tile's M
     // block does not change (chunked order: N increases, so the cursor only moves forward)
     int row_mt = -1;
@@ -400,6 +401,65 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
         const int cfirst = n0 + wh * CW;
         while (lab_cur < lab_end && g.lab[lab_cur] < cfirst) ++lab_cur;
       }
+      if constexpr (EPI == TC_EPI_SGD) {
+        // G3: W2 -= lr (dZ^T H1 [+ centred-sigmoid offset]), b2 -= lr db2, bf16 shadow refresh.
+        // Per 32 x 32 chunk: the accumulator (lane = W2 row) goes through a swizzled smem
+        // tile so that W2 is read and written coalesced (8 lanes x 16 B per row, 4 rows
+        // per instruction); the W2 chunks are loaded into registers before the
+        // accumulator wait, so their HBM latency hides under this tile's MMAs.
+        constexpr int NCH = CW / 32;
+        const int cb = n0 + wh * CW;
+        const int m0w = m0 + wq * 32;
+        const int lr8 = lane >> 3, lc4 = (lane & 7) * 4;   // coalesced layout: row 4 i + lr8, cols lc4..+3
+        uint8_t* tt = sStg + (warp - 4) * 4096;
+        float4 wr[NCH][8];
+#pragma unroll
+        for (int ch = 0; ch < NCH; ++ch)
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const int r = m0w + 4 * i + lr8;
+            wr[ch][i] = r < g.M ? *reinterpret_cast<const float4*>(g.out + (int64_t)r * g.ldo + cb + 32 * ch + lc4)
+                                : make_float4(0.f, 0.f, 0.f, 0.f);
+          }
+        mbar_wait(&tfull[acc], aph);
+        tc_fence_after();
+        const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS) + ((uint32_t)(wq * 32) << 16);
+#pragma unroll
+        for (int ch = 0; ch < NCH; ++ch) {
+          float v[32];
+          if (nk > 0) {
+            tmem_ld32(d + (uint32_t)(wh * CW + 32 * ch), v);
+          } else {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = 0.f;
+          }
+          __syncwarp();   // the previous chunk's reads of tt are done
+#pragma unroll
+          for (int q = 0; q < 8; ++q)
+            *reinterpret_cast<float4*>(tt + lane * 128 + ((q ^ (lane & 7)) * 16)) =
+                make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+          __syncwarp();
+          float4 ho = make_float4(0.f, 0.f, 0.f, 0.f);
+          if (g.hoff) ho = __ldg(reinterpret_cast<const float4*>(g.hoff + cb + 32 * ch + lc4));   // centred sigmoid
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const int rl = 4 * i + lr8, r = m0w + rl;
+            float4 a = *reinterpret_cast<const float4*>(tt + rl * 128 + (((lane & 7) ^ (rl & 7)) * 16));
+            a.x += ho.x; a.y += ho.y; a.z += ho.z; a.w += ho.w;
+            if (r < g.M) {
+              float4 x = wr[ch][i];
+              x.x -= lr * a.x; x.y -= lr * a.y; x.z -= lr * a.z; x.w -= lr * a.w;
+              const int64_t o = (int64_t)r * g.ldo + cb + 32 * ch + lc4;
+              __stcs(reinterpret_cast<float4*>(g.out + o), x);
+              __nv_bfloat162 p0 = __floats2bfloat162_rn(x.x, x.y), p1 = __floats2bfloat162_rn(x.z, x.w);
+              uint2 pk;
+              pk.x = *reinterpret_cast<uint32_t*>(&p0); pk.y = *reinterpret_cast<uint32_t*>(&p1);
+              __stcs(reinterpret_cast<uint2*>(g.shadow + o), pk);
+              if (g.grad) *reinterpret_cast<float4*>(g.grad + o) = a;
+            }
+          }
+        }
+      } else {
       mbar_wait(&tfull[acc], aph);
       tc_fence_after();
       const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS) + ((uint32_t)(wq * 32) << 16);
@@ -548,55 +608,6 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
             asm volatile("cp.async.bulk.commit_group;" ::: "memory");
           }
           sbuf ^= 1;
-        } else {  // TC_EPI_SGD: W2 box += -lr dW2 through smem; TMA load, TMA stores (W2 fp32, bf16 shadow)
-          const int b = kc & 1;
-          const uint32_t ph = (kc >> 1) & 1;
-          ++kc;
-          uint8_t* wb = sStg + (warp - 4) * 12288 + b * 4096;          // 32 x 32 fp32, 128B swizzle
-          uint8_t* hb = sStg + (warp - 4) * 12288 + 8192 + b * 2048;   // 32 x 32 bf16, 64B swizzle
-          uint64_t* wl = &wbar[(warp - 4) * 2 + b];
-          const int row0 = m0 + wq * 32;
-          if (lane == 0) {
-            asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");   // buffer b read out
-            mbar_expect_tx(wl, 4096);
-            tma_load_2d(wb, &tmC, wl, n, row0);   // rows >= L are zero-filled
-          }
-          mbar_wait(wl, ph);
-          if (g.hoff) {   // centred sigmoid dZ: dW2[m][h] += (1/(2B)) sum_n H1[n][h]
-            const float4* h4 = reinterpret_cast<const float4*>(g.hoff + n);
-#pragma unroll
-            for (int q = 0; q < 8; ++q) {
-              const float4 t = __ldg(h4 + q);
-              v[4 * q] += t.x; v[4 * q + 1] += t.y; v[4 * q + 2] += t.z; v[4 * q + 3] += t.w;
-            }
-          }
-#pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            float4* p = reinterpret_cast<float4*>(wb + lane * 128 + ((q ^ (lane & 7)) * 16));
-            float4 x = *p;
-            x.x -= lr * v[4 * q]; x.y -= lr * v[4 * q + 1]; x.z -= lr * v[4 * q + 2]; x.w -= lr * v[4 * q + 3];
-            *p = x;
-            __nv_bfloat162 p0 = __floats2bfloat162_rn(x.x, x.y), p1 = __floats2bfloat162_rn(x.z, x.w);
-            uint2 pk;
-            pk.x = *reinterpret_cast<uint32_t*>(&p0);
-            pk.y = *reinterpret_cast<uint32_t*>(&p1);
-            *reinterpret_cast<uint2*>(hb + lane * 64 + ((((q >> 1) ^ ((lane >> 1) & 3))) * 16) + (q & 1) * 8) = pk;
-          }
-          if (g.grad && m < g.M) {
-            float* gr = g.grad + (int64_t)m * g.ldo + n;
-#pragma unroll
-            for (int j = 0; j < 32; j += 4)
-              reinterpret_cast<float4*>(gr)[j / 4] = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-          }
-          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-          __syncwarp();
-          if (lane == 0) {   // rows >= L are clipped (never touch b2)
-            asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
-                             reinterpret_cast<uint64_t>(&tmC)), "r"(smem_u32(wb)), "r"(n), "r"(row0) : "memory");
-            asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
-                             reinterpret_cast<uint64_t>(&tmD)), "r"(smem_u32(hb)), "r"(n), "r"(row0) : "memory");
-            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-          }
         }
       }
       if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_STATS) {
@@ -605,11 +616,12 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
       if constexpr (EPI == TC_EPI_SIG) {
         if (m < g.M) g.stats[(int64_t)(nt * NQ + wh) * g.stats_ld + m] = make_float2(st_s, 0.f);
       }
+      }   // EPI != SGD
       if constexpr (ONES) {
         if (nt == 0 && wh == 0) {   // db2[m] = sum_n dZ[n, m]; b2 -= lr db2
           float v[32];
           if (nk > 0) {
-            tmem_ld32(d + (uint32_t)BN, v);
+            tmem_ld32(tmem + (uint32_t)(acc * ACC_COLS + BN) + ((uint32_t)(wq * 32) << 16), v);
           } else {
             v[0] = 0.f;
           }
@@ -812,7 +824,6 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
   CUtensorMap td;   // W2 fp32 boxes (load + store) and the bf16 shadow boxes (store)
   if ((e = make_store_map(&tc, W2, H, L, (uint64_t)H * 4, 1, 0, 2)) != cudaSuccess) return e;
   if ((e = make_bf16_store_map(&td, P.w2b, H, L)) != cudaSuccess) return e;
-  if (bn == 256) return run<256, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
   if (bn == 128) return run<128, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
   return run<64, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
 }
