@@ -72,7 +72,8 @@ typedef struct asgd_sched asgd_sched;
 typedef struct {
   int64_t F;              /* input features                                 */
   int64_t L;              /* labels (output units)                          */
-  int64_t H;              /* hidden units; one of 64, 128, 256, 512         */
+  int64_t H;              /* hidden units; one of 64, 128, 256, 512 (bf16:
+                             <= 256, ASGD_E_UNSUPPORTED otherwise)          */
   int32_t precision;      /* ASGD_PREC_*                                    */
   int32_t b_max;          /* max rows of one local step (<= 2048)           */
   int64_t max_step_nnz;   /* max feature nnz of one step's rows             */

@@ -345,6 +345,8 @@ int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device, v
   if (prop.major != 10 || prop.minor != 0)
     return fail(ASGD_E_UNSUPPORTED, "device %d is sm_%d%d; libasgd is built for sm_100a only", device,
                 prop.major, prop.minor);
+  if (m.precision == ASGD_PREC_BF16 && m.H > 256)   // G1's resident H1 block holds K = H <= 256
+    return fail(ASGD_E_UNSUPPORTED, "bf16 path: H=%lld > 256", (long long)m.H);
   if (m.precision == ASGD_PREC_BF16 && !tc_available())
     return fail(ASGD_E_UNSUPPORTED, "bf16 tcgen05 path not built");
   asgd_ctx* c = new (std::nothrow) asgd_ctx();

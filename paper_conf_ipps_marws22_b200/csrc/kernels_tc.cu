@@ -68,10 +68,10 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   while (!ok) {
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
         "selp.u32 %0, 1, 0, p;\n\t}"
         : "=r"(ok)
-        : "r"(a), "r"(parity)
+        : "r"(a), "r"(parity), "r"(1000000u)   // suspend up to 1 ms instead of spinning on issue slots
         : "memory");
   }
 }
@@ -142,6 +142,31 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float (&v)[32]) {
   for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
 }
 
+// Asynchronous variant: the 32 registers are written when tcgen05.wait::ld retires;
+// tmem_wait_regs() waits and then ties the registers to that point (empty asm with
+// "+r"), so no use can be scheduled before the wait.
+__device__ __forceinline__ void tmem_ld32_async(uint32_t taddr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, "
+      "%16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+        "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]),
+        "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]),
+        "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_wait_regs(uint32_t (&r)[32]) {
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+  asm volatile(""
+               : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]), "+r"(r[6]),
+                 "+r"(r[7]), "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]), "+r"(r[12]), "+r"(r[13]),
+                 "+r"(r[14]), "+r"(r[15]), "+r"(r[16]), "+r"(r[17]), "+r"(r[18]), "+r"(r[19]), "+r"(r[20]),
+                 "+r"(r[21]), "+r"(r[22]), "+r"(r[23]), "+r"(r[24]), "+r"(r[25]), "+r"(r[26]), "+r"(r[27]),
+                 "+r"(r[28]), "+r"(r[29]), "+r"(r[30]), "+r"(r[31]));
+}
+
 __device__ __forceinline__ float ex2_approx(float x) {   // 2^x on the MUFU (ex2.approx, -inf -> 0)
   float y;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
@@ -207,11 +232,21 @@ template <int BN, int EPI>
 constexpr uint32_t bias_bytes() {   // per epilogue warp: its tile columns' b2 (smem broadcast copy)
   return has_bias<EPI>() ? (uint32_t)epi_warps<BN, EPI>() * (uint32_t)(BN / (epi_warps<BN, EPI>() / 4)) * 4u : 0u;
 }
-template <int BN, int EPI>
-constexpr uint32_t staging_bytes() {   // per epilogue warp: 2 store boxes (G3: 2 x (4 KB fp32 + 2 KB bf16) + pad)
+// G1 variants with the A operand (the H1 row block, K = H <= 256) resident in smem: a CTA
+// keeps its M block for many consecutive tiles (chunked order), so only W2 tiles stream.
+template <int EPI, bool A_MN>
+constexpr bool a_resident() {
+  return !A_MN && (EPI == TC_EPI_STATS || EPI == TC_EPI_DZ || EPI == TC_EPI_SIG);
+}
+constexpr int kAresK = 256;   // largest K (= H) of the resident A block
+template <int EPI, bool A_MN>
+constexpr int store_bufs() { return a_resident<EPI, A_MN>() ? 1 : 2; }   // TMA-store boxes per warp
+template <int BN, int EPI, bool A_MN>
+constexpr uint32_t staging_bytes() {   // per epilogue warp: store boxes / G3 transpose tile
   return EPI == TC_EPI_STATS ? 0u
                              : (EPI == TC_EPI_SGD ? 8u * 4096u   // per warp: one 32 x 32 fp32 transpose tile
-                                                  : (uint32_t)epi_warps<BN, EPI>() * 2u * box_bytes<EPI>());
+                                                  : (uint32_t)epi_warps<BN, EPI>() * store_bufs<EPI, A_MN>() *
+                                                        box_bytes<EPI>());
 }
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
@@ -219,7 +254,11 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
     k_gemm_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
               const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmD, TcArgs g) {
   constexpr int STAGES = stages_of<EPI>();
-  constexpr uint32_t A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE = A_BYTES + B_BYTES;
+  constexpr bool ARES = a_resident<EPI, A_MN>();
+  constexpr uint32_t A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2;
+  constexpr uint32_t STAGE = (ARES ? 0u : A_BYTES) + B_BYTES;
+  constexpr uint32_t ARES_BYTES = ARES ? (uint32_t)(kAresK / BK) * A_BYTES : 0u;
+  constexpr int NSTG = store_bufs<EPI, A_MN>();
   constexpr bool ONES = (EPI == TC_EPI_SGD);           // db2 column block after the accumulator
   constexpr int ACC_COLS = BN + (ONES ? 32 : 0);
   constexpr int NACC = (2 * ACC_COLS <= 512) ? 2 : 1;
@@ -231,17 +270,20 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
   static_assert(CW % 32 == 0, "epilogue chunks are 32 columns");
   constexpr uint32_t BOX = box_bytes<EPI>();
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t* sA = smem;
-  uint8_t* sB = smem + STAGES * A_BYTES;
-  uint8_t* sOnes = smem + STAGES * STAGE;
-  uint8_t* sStg = smem + STAGES * STAGE + ONES_BYTES;   // TMA-store staging (1024-aligned)
-  float* sBias = reinterpret_cast<float*>(sStg + staging_bytes<BN, EPI>());
-  uint64_t* full = reinterpret_cast<uint64_t*>(sStg + staging_bytes<BN, EPI>() + bias_bytes<BN, EPI>());
+  // 1024-aligned base, derived from smem_raw by an offset so the compiler keeps the shared
+  // address space (LDS/STS instead of generic LD/ST in the epilogues)
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint8_t* sA = smem;                                          // ring A stages, or the resident A block
+  uint8_t* sB = smem + (ARES ? ARES_BYTES : STAGES * A_BYTES);
+  uint8_t* sOnes = smem + ARES_BYTES + STAGES * STAGE;
+  uint8_t* sStg = sOnes + ONES_BYTES;   // TMA-store staging (1024-aligned)
+  float* sBias = reinterpret_cast<float*>(sStg + staging_bytes<BN, EPI, A_MN>());
+  uint64_t* full = reinterpret_cast<uint64_t*>(sStg + staging_bytes<BN, EPI, A_MN>() + bias_bytes<BN, EPI>());
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;
   uint64_t* tempty = tfull + 2;
-  uint32_t* tbase = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* afull = tempty + 2;   // resident A block loaded
+  uint32_t* tbase = reinterpret_cast<uint32_t*>(afull + 1);
 
   pdl_trigger();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -265,6 +307,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
     for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
     for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], EPI_WARPS); }
+    mbar_init(afull, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
@@ -289,11 +332,19 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
   if (warp == 0) {
     if (lane == 0) {
       // ------------------------------------------------ TMA producer
-      int it = 0;
+      int it = 0, amt = -1;
       for (int t = t_first; t < t_end; t += t_step) {
         int mt, nt, z, kb0, nk;
         decode(t, mt, nt, z, kb0, nk);
         const int m0 = mt * BM, n0 = nt * BN;
+        if constexpr (ARES) {
+          if (mt != amt) {   // new M block: reload the resident A once every MMA reading it retired
+            if (it > 0) mbar_wait(&empty[(it - 1) % STAGES], ((it - 1) / STAGES) & 1);
+            mbar_expect_tx(afull, (uint32_t)nk * A_BYTES);
+            for (int i = 0; i < nk; ++i) tma_load_2d(sA + i * A_BYTES, &tmA, afull, (kb0 + i) * BK, m0);
+            amt = mt;
+          }
+        }
         for (int i = 0; i < nk; ++i, ++it) {
           const int s = it % STAGES;
           const uint32_t ph = (it / STAGES) & 1;
@@ -302,7 +353,8 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
           const int kc = (kb0 + i) * BK;
           uint8_t* a = sA + s * A_BYTES;
           uint8_t* b = sB + s * B_BYTES;
-          if constexpr (!A_MN) {
+          if constexpr (ARES) {
+          } else if constexpr (!A_MN) {
             tma_load_2d(a, &tmA, &full[s], kc, m0);
           } else {
             tma_load_2d(a, &tmA, &full[s], m0, kc);
@@ -323,13 +375,16 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
       constexpr uint32_t idesc = make_idesc(BN, A_MN, B_MN);
       constexpr uint32_t idesc1 = make_idesc(16, A_MN, false);
       const uint32_t ones_base = smem_u32(sOnes);
-      int it = 0, tl = 0;
+      int it = 0, tl = 0, amt = -1, aloads = 0;
       for (int t = t_first; t < t_end; t += t_step, ++tl) {
         int mt, nt, z, kb0, nk;
         decode(t, mt, nt, z, kb0, nk);
         const int acc = tl % NACC;
         const uint32_t aph = (tl / NACC) & 1;
         mbar_wait(&tempty[acc], aph ^ 1);     // epilogue drained this accumulator
+        if constexpr (ARES) {
+          if (mt != amt) { mbar_wait(afull, (uint32_t)aloads & 1u); ++aloads; amt = mt; }
+        }
         tc_fence_after();
         const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS);
         const bool ones = ONES && nt == 0;
@@ -338,7 +393,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
           const uint32_t ph = (it / STAGES) & 1;
           mbar_wait(&full[s], ph);
           tc_fence_after();
-          const uint32_t a_base = smem_u32(sA + s * A_BYTES), b_base = smem_u32(sB + s * B_BYTES);
+          const uint32_t a_base = smem_u32(sA + (ARES ? i : s) * A_BYTES), b_base = smem_u32(sB + s * B_BYTES);
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k) {
             // K-major: advance 16 elements (32 B) inside the 128B swizzle atom.
@@ -363,8 +418,9 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
     // G1b / sigmoid: row m's lse, 1 / (|Y_m| B) and label cursor, kept while the tile's M
     // block does not change (chunked order: N increases, so the cursor only moves forward)
     int row_mt = -1;
-    float lse_m = 0.f, tinv = 0.f;
+    float lse_m = 0.f, tinv = 0.f, crow = 0.f;   // crow (DZ): -lse log2(e) - log2(B)
     int64_t lab_cur = 0, lab_end = 0;
+    int nxt = 0x7fffffff;                        // next label column of row m (labels sorted)
     float* bias_w = sBias + (has_bias<EPI>() ? (warp - 4) * CW : 0);
     for (int t = t_first; t < t_end; t += t_step, ++tl) {
       int mt, nt, z, kb0, nk;
@@ -376,11 +432,12 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
       // before waiting for the accumulator: this warp's b2 columns into smem (coalesced
       // loads, read back below as broadcast float4) and the row state of a new M block
       if constexpr (has_bias<EPI>()) {
+        constexpr float bscale = EPI == TC_EPI_DZ ? 1.4426950408889634f : 1.f;   // DZ: log2 domain
         __syncwarp();
 #pragma unroll
         for (int c = 0; c < CW; c += 32) {
           const int col = n0 + wh * CW + c + lane;
-          bias_w[c + lane] = col < g.N ? __ldg(g.bias + col) : 0.f;
+          bias_w[c + lane] = col < g.N ? __ldg(g.bias + col) * bscale : 0.f;
         }
         __syncwarp();
       }
@@ -389,17 +446,24 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
           row_mt = mt;
           lab_cur = lab_end = 0;
           if (m < g.M) {
-            if constexpr (EPI == TC_EPI_DZ) lse_m = g.lse[m];
+            if constexpr (EPI == TC_EPI_DZ) {
+              lse_m = g.lse[m];
+              crow = -lse_m * 1.4426950408889634f - __log2f(1.f / g.invB);
+            }
             const int64_t id = g.rows[m];
             lab_cur = g.lab_ptr[id];
             lab_end = g.lab_ptr[id + 1];
             tinv = g.invB / (float)(lab_end - lab_cur);
           }
+          nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
         }
         // skip labels left of this warp's first column (cursor is monotone within an M block
         // in the chunked order; a restart at a lower column would need the full walk)
         const int cfirst = n0 + wh * CW;
-        while (lab_cur < lab_end && g.lab[lab_cur] < cfirst) ++lab_cur;
+        while (nxt < cfirst) {
+          ++lab_cur;
+          nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
+        }
       }
       if constexpr (EPI == TC_EPI_SGD) {
         // G3: W2 -= lr (dZ^T H1 [+ centred-sigmoid offset]), b2 -= lr db2, bf16 shadow refresh.
@@ -464,18 +528,27 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
       tc_fence_after();
       const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS) + ((uint32_t)(wq * 32) << 16);
       float st_m = -INFINITY, st_s = 0.f;   // G1 softmax partials of row m over this column group
-#pragma unroll 1
-      for (int c = wh * CW; c < (wh + 1) * CW; c += 32) {
+      // chunks of 32 columns; the next chunk's TMEM load is in flight while this one is processed
+      constexpr int NCHK = CW / 32;
+      const bool have = EPI != TC_EPI_PART || nk > 0;   // only split-K slices can be empty
+      uint32_t rr[2][32];
+      if (have) tmem_ld32_async(d + (uint32_t)(wh * CW), rr[0]);
+#pragma unroll
+      for (int k = 0; k < NCHK; ++k) {
+        const int c = wh * CW + 32 * k;
         float v[32];
-        if (nk > 0) {
-          tmem_ld32(d + (uint32_t)c, v);
+        if (have) {
+          tmem_wait_regs(rr[k & 1]);
+          if (k + 1 < NCHK) tmem_ld32_async(d + (uint32_t)(c + 32), rr[(k + 1) & 1]);
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(rr[k & 1][i]);
         } else {
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = 0.f;
         }
         const int n = n0 + c;
         if (n >= g.N) continue;   // warp-uniform
-        if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_DZ || EPI == TC_EPI_SIG || EPI == TC_EPI_STATS) {
+        if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_SIG || EPI == TC_EPI_STATS) {
           // + b2 (the same 32 values for every lane: broadcast smem reads); columns >= N -> -inf
           const float4* b4 = reinterpret_cast<const float4*>(bias_w + (c - wh * CW));
 #pragma unroll
@@ -492,21 +565,30 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
         if constexpr (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG) {
           constexpr float kL2E = 1.4426950408889634f;
           if constexpr (EPI == TC_EPI_DZ) {
-            // softmax - uniform target over the row's labels (Q3), / B (Q4); labels are sorted,
-            // lab_cur walks forward as this warp's columns increase
-            const float ls = lse_m * kL2E;
+            // softmax - uniform target over the row's labels (Q3), / B (Q4):
+            // exp(acc + b2 - lse) / B = 2^(acc log2(e) + b2 log2(e) - lse log2(e) - log2(B)),
+            // b2 log2(e) staged per column; labels are sorted, nxt walks forward with the columns
+            const float4* b4 = reinterpret_cast<const float4*>(bias_w + (c - wh * CW));
 #pragma unroll
-            for (int j = 0; j < 32; ++j) v[j] = ex2_approx(fmaf(v[j], kL2E, -ls)) * g.invB;
-            while (lab_cur < lab_end) {
-              const int y = g.lab[lab_cur];
-              if (y >= n + 32) break;
-              if (y >= n) {
-                const int jy = y - n;
+            for (int q = 0; q < 8; ++q) {
+              const float4 t = b4[q];
+              v[4 * q] = ex2_approx(fmaf(v[4 * q], kL2E, t.x + crow));
+              v[4 * q + 1] = ex2_approx(fmaf(v[4 * q + 1], kL2E, t.y + crow));
+              v[4 * q + 2] = ex2_approx(fmaf(v[4 * q + 2], kL2E, t.z + crow));
+              v[4 * q + 3] = ex2_approx(fmaf(v[4 * q + 3], kL2E, t.w + crow));
+            }
+            if (n + 32 > g.N) {   // columns >= N (stores are clipped; keep them finite)
 #pragma unroll
-                for (int j = 0; j < 32; ++j)
-                  if (j == jy) v[j] -= tinv;
-              }
+              for (int j = 0; j < 32; ++j)
+                if (n + j >= g.N) v[j] = 0.f;
+            }
+            while (nxt < n + 32) {   // rare: a label of row m in this chunk
+              const int jy = nxt - n;
+#pragma unroll
+              for (int j = 0; j < 32; ++j)
+                if (j == jy) v[j] -= tinv;
               ++lab_cur;
+              nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
             }
           } else {
             // sigmoid BCE (R11): row partial += softplus(z) - y z; dZ is stored CENTRED,
@@ -517,11 +599,10 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
             // softplus(z) = max(z, 0) + log1p(e).  Padding columns carry z = -inf: e = 0,
             // softplus = 0 (their dZ is clipped by the store).
             uint32_t ym = 0;   // label columns of this 32-column chunk (labels sorted)
-            while (lab_cur < lab_end) {
-              const int y = g.lab[lab_cur];
-              if (y >= n + 32) break;
-              if (y >= n) ym |= 1u << (y - n);
+            while (nxt < n + 32) {
+              ym |= 1u << (nxt - n);
               ++lab_cur;
+              nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
             }
             float a0 = 0.f, a1 = 0.f;
 #pragma unroll
@@ -539,17 +620,26 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
             st_s += a0 + a1;
           }
           // stage a 32 x 32 bf16 box (64B swizzle) and TMA-store it into dZ
-          uint8_t* buf = sStg + ((warp - 4) * 2 + sbuf) * BOX;
-          if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+          uint8_t* buf = sStg + ((warp - 4) * NSTG + (NSTG > 1 ? sbuf : 0)) * BOX;
+          if (lane == 0) {
+            if constexpr (NSTG > 1) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+            else asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+          }
           __syncwarp();
+          {
+            uint8_t* rowp = buf + lane * 64;
+            const int sw = (lane >> 1) & 3;   // 64B swizzle of this row's four 16-byte chunks
 #pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            __nv_bfloat162 p0 = __floats2bfloat162_rn(v[4 * q], v[4 * q + 1]);
-            __nv_bfloat162 p1 = __floats2bfloat162_rn(v[4 * q + 2], v[4 * q + 3]);
-            uint2 pk;
-            pk.x = *reinterpret_cast<uint32_t*>(&p0);
-            pk.y = *reinterpret_cast<uint32_t*>(&p1);
-            *reinterpret_cast<uint2*>(buf + lane * 64 + ((((q >> 1) ^ ((lane >> 1) & 3))) * 16) + (q & 1) * 8) = pk;
+            for (int h = 0; h < 4; ++h) {
+              __nv_bfloat162 p0 = __floats2bfloat162_rn(v[8 * h], v[8 * h + 1]);
+              __nv_bfloat162 p1 = __floats2bfloat162_rn(v[8 * h + 2], v[8 * h + 3]);
+              __nv_bfloat162 p2 = __floats2bfloat162_rn(v[8 * h + 4], v[8 * h + 5]);
+              __nv_bfloat162 p3 = __floats2bfloat162_rn(v[8 * h + 6], v[8 * h + 7]);
+              uint4 pk;
+              pk.x = *reinterpret_cast<uint32_t*>(&p0); pk.y = *reinterpret_cast<uint32_t*>(&p1);
+              pk.z = *reinterpret_cast<uint32_t*>(&p2); pk.w = *reinterpret_cast<uint32_t*>(&p3);
+              *reinterpret_cast<uint4*>(rowp + ((h ^ sw) * 16)) = pk;
+            }
           }
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           __syncwarp();
@@ -702,8 +792,11 @@ cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t 
 template <int BN, bool A_MN, bool B_MN, int EPI>
 cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c,
                const CUtensorMap& d, TcArgs g, int splits) {
-  const size_t smem = (size_t)stages_of<EPI>() * (BM * BK * 2 + BN * BK * 2) + (EPI == TC_EPI_SGD ? 2048 : 0) +
-                      staging_bytes<BN, EPI>() + bias_bytes<BN, EPI>() + 1024 + 512;
+  constexpr bool ARES = a_resident<EPI, A_MN>();
+  const size_t smem = (ARES ? (size_t)(kAresK / BK) * BM * BK * 2 : 0) +
+                      (size_t)stages_of<EPI>() * ((ARES ? 0 : BM * BK * 2) + BN * BK * 2) +
+                      (EPI == TC_EPI_SGD ? 2048 : 0) + staging_bytes<BN, EPI, A_MN>() + bias_bytes<BN, EPI>() + 1024 + 512;
+  if (ARES && g.K > kAresK) return cudaErrorNotSupported;   // resident A block holds K <= 256
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(k_gemm_tc<BN, A_MN, B_MN, EPI>,

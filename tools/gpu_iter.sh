@@ -1,0 +1,11 @@
+# usage: bash tools/gpu_iter.sh TAG  -- full GPU suite, Amazon-670K + EURLex bench lines, ncu of the 4 GEMMs
+T=$1
+mkdir -p gpurun_out
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/${T}_pytest.log 2>&1; echo pytest $?
+tail -5 gpurun_out/${T}_pytest.log | grep -E "passed|failed|Error|error|assert" | head
+timeout 900 python bench.py --config amazon670k --steps 5 --no-cpu-baseline --ttp-megabatches 0 --e2e-steps 0 > gpurun_out/${T}_a670k.json 2>&1; echo bench2 $?
+timeout 600 python bench.py --no-cpu-baseline --ttp-megabatches 0 --e2e-steps 0 > gpurun_out/${T}_eurlex.json 2>&1; echo bench1 $?
+for f in gpurun_out/${T}_a670k.json gpurun_out/${T}_eurlex.json; do python -c "
+import json,sys; d=json.loads(open('$f').read().strip().splitlines()[-1]); print('$f', d['value'], d['ms_per_step'], d['roofline']['kernel'], d['roofline']['frac'], {k:v['us_per_launch'] for k,v in d['kernels_warmup_profile'].items()})"; done
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:"k_gemm_tc" -s 12 -c 4 \
+  -o gpurun_out/${T}_a670k python tools/prof_step.py amazon670k bf16 softmax 3 1 65536 > gpurun_out/${T}_1.log 2>&1; echo ncu $?
