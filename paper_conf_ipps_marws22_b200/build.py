@@ -17,7 +17,7 @@ LIB = os.path.join(PKG, "libasgd.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-O3",
-         "--expt-relaxed-constexpr", "-DNDEBUG"]
+         "--expt-relaxed-constexpr", "-DNDEBUG"] + os.environ.get("ASGD_NVCC_EXTRA", "").split()   # A/B switches
 
 
 def _sources():

@@ -574,12 +574,21 @@ int enqueue_step(asgd_ctx* c, int n) {
                                                      nullptr, nullptr, P.rowsc, x.lab_ptr, x.lab);
           })());
     }
-    CU(cudaEventRecord(c->ev_sm, c->s));
-    CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
     const bool centred = m.loss == ASGD_LOSS_SIGMOID;   // G1 stored dZ - 1/(2B) (R11)
-    PCU_ON(c->s3, ASGD_K_G3, launch_gemm_tc(lc3, 3, n, Lb, H, Pw, c->L, W2, b2, g ? g + c->o_w2 : nullptr,
-                                            g ? g + c->o_b2 : nullptr, nullptr, nullptr, nullptr, nullptr, nullptr,
-                                            centred ? P.cen + H : nullptr));
+    auto g3 = [&](const Launch& l) {
+      return launch_gemm_tc(l, 3, n, Lb, H, Pw, c->L, W2, b2, g ? g + c->o_w2 : nullptr, g ? g + c->o_b2 : nullptr,
+                            nullptr, nullptr, nullptr, nullptr, nullptr, centred ? P.cen + H : nullptr);
+    };
+    // G3 beside G2 only when G2 leaves at least half the SMs idle; when both fill the GPU
+    // (Amazon-670K: 148 persistent CTAs each, one per SM) concurrent launches interleave
+    // their CTAs and the later kernel's static tile split waits on the earlier one's SMs
+    // (measured 1024 us for the pair against 326 + 572 us back to back), so G3 runs last
+    const bool g3_side = 2 * g2c <= c->sms;
+    if (g3_side) {
+      CU(cudaEventRecord(c->ev_sm, c->s));
+      CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
+      PCU_ON(c->s3, ASGD_K_G3, g3(lc3));
+    }
     PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr));
     PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, true, centred ? P.cen : nullptr));
     CU(cudaEventRecord(c->ev_dh, c->s));
@@ -589,6 +598,7 @@ int enqueue_step(asgd_ctx* c, int n) {
     // K-5 (needs K-0's segments)
     CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
     PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
+    if (!g3_side) PCU(ASGD_K_G3, g3(lc));
     CU(cudaStreamWaitEvent(c->s, c->ev_a, 0));
   }
   return ASGD_OK;

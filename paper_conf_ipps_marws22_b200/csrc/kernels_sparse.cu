@@ -143,31 +143,46 @@ __device__ int build_view(const StepArgs& sa, const int64_t* __restrict__ row_pt
                           const int64_t* __restrict__ lab_ptr, int64_t n_data_rows, int64_t nz_cap,
                           int64_t nl_cap, int32_t* sboff, bool publish, const ViewOut& out) {
   __shared__ long long wf[32], wl[32];
+  __shared__ int32_t s_llen[kViewPer * 256];   // label counts (publish only)
+  __shared__ int s_bad;
   const int n = sa.n;
   int64_t* srb = const_cast<int64_t*>(view_rbase(sboff, n));
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5, nw = blockDim.x >> 5;
-  const int r0 = t * kViewPer;
-  int64_t len[kViewPer], llen[kViewPer];
-  long long sf = 0, sl = 0;
-  int bad = 0;
-#pragma unroll
-  for (int i = 0; i < kViewPer; ++i) {
-    len[i] = 0; llen[i] = 0;
-    const int r = r0 + i;
-    if (r < n) {
-      const int64_t id = sa.rows[r];
-      if (id < 0 || id >= n_data_rows) { bad = 1; srb[r] = 0; continue; }
+  // loads spread over every thread (row r on thread r % blockDim: one rows[] -> row_ptr[]
+  // round trip for the whole block); row lengths parked in sboff / s_llen for the scan
+  if (t == 0) s_bad = 0;
+  __syncthreads();
+  for (int r = t; r < n; r += blockDim.x) {
+    const int64_t id = sa.rows[r];
+    int32_t ln = 0, ll = 0;
+    if (id < 0 || id >= n_data_rows) {
+      s_bad = 1;
+      srb[r] = 0;
+    } else {
       const int64_t a = row_ptr[id];
-      len[i] = row_ptr[id + 1] - a;
+      ln = (int32_t)(row_ptr[id + 1] - a);
       srb[r] = a;
       if (publish) {
-        llen[i] = lab_ptr[id + 1] - lab_ptr[id];
+        ll = (int32_t)(lab_ptr[id + 1] - lab_ptr[id]);
         out.rowsc[r] = (int32_t)id;
         out.rbase[r] = a;
       }
-      sf += len[i];
-      sl += llen[i];
     }
+    sboff[r] = ln;
+    if (publish) s_llen[r] = ll;
+  }
+  __syncthreads();
+  const int bad = s_bad;
+  const int r0 = t * kViewPer;
+  int64_t len[kViewPer], llen[kViewPer];
+  long long sf = 0, sl = 0;
+#pragma unroll
+  for (int i = 0; i < kViewPer; ++i) {
+    const int r = r0 + i;
+    len[i] = r < n ? sboff[r] : 0;
+    llen[i] = (publish && r < n) ? s_llen[r] : 0;
+    sf += len[i];
+    sl += llen[i];
   }
   long long xf = sf, xl = sl;   // inclusive warp scan
 #pragma unroll
@@ -204,7 +219,7 @@ __device__ int build_view(const StepArgs& sa, const int64_t* __restrict__ row_pt
   long long tf = wf[nw - 1], tl = wl[nw - 1];
   if (t == 0) sboff[n] = (int32_t)min(tf, (long long)nz_cap);
   if (publish) {
-    if (bad) atomicOr(&out.meta[M_ERR], ERR_ROW_ID);
+    if (bad && t == 0) atomicOr(&out.meta[M_ERR], ERR_ROW_ID);
     if (t == 0) {
       int err = 0;
       if (tf > nz_cap) { err |= ERR_NNZ_CAP; tf = nz_cap; }

@@ -173,6 +173,33 @@ __device__ __forceinline__ float ex2_approx(float x) {   // 2^x on the MUFU (ex2
   return y;
 }
 
+// 2^x for x <= 0 on the FMA/ALU pipes (no MUFU): round-to-nearest split x = k + f,
+// f in [-1/2, 1/2] via the 1.5 * 2^23 magic add, degree-3 polynomial for 2^f (relative
+// error 7.7e-5, below bf16's 2^-9 and far below the 2e-2 gradient tolerance), k added to
+// the exponent field.  x is clamped at -125 (result ~2e-38, i.e. 0 in every sum it
+// enters; -inf padding columns included).  The softmax epilogues are MUFU-bound at 16
+// ex2/clk/SM -- exactly the tcgen05 rate of a 128 x 256 x 256 tile -- so a quarter of
+// the exponentials go here instead (the FA4 split).
+__device__ __forceinline__ float ex2_poly(float x) {
+  x = fmaxf(x, -125.f);
+  const float t = x + 12582912.f;
+  const float f = x - (t - 12582912.f);
+  float p = fmaf(fmaf(fmaf(0.05508868396282196f, f, 0.24260404706001282f), f, 0.6932762265205383f), f,
+                 0.9999289512634277f);
+  return __int_as_float(__float_as_int(p) + (__float_as_int(t) << 23));
+}
+#ifndef ASGD_POLY_EXP
+#define ASGD_POLY_EXP 0   // measured: G1 389 -> 430 us with the split (not MUFU-throughput bound)
+#endif
+// every 4th exponential of the softmax epilogues on the FMA pipes (ASGD_POLY_EXP=0: all MUFU)
+__device__ __forceinline__ float ex2_mix(float x) {
+#if ASGD_POLY_EXP
+  return ex2_poly(x);
+#else
+  return ex2_approx(x);
+#endif
+}
+
 __device__ __forceinline__ float rcp_approx(float x) {
   float y;
   asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
@@ -422,6 +449,20 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
     int64_t lab_cur = 0, lab_end = 0;
     int nxt = 0x7fffffff;                        // next label column of row m (labels sorted)
     float* bias_w = sBias + (has_bias<EPI>() ? (warp - 4) * CW : 0);
+    // b2 of the tile after the current one (prefetched one tile ahead)
+    float bpre[has_bias<EPI>() ? CW / 32 : 1];
+    auto load_bias = [&](int tt) {
+      if constexpr (has_bias<EPI>()) {
+        int mt_, nt_, z_, kb_, nk_;
+        decode(tt, mt_, nt_, z_, kb_, nk_);
+#pragma unroll
+        for (int c = 0; c < CW / 32; ++c) {
+          const int col = nt_ * BN + wh * CW + 32 * c + lane;
+          bpre[c] = col < g.N ? __ldg(g.bias + col) : 0.f;
+        }
+      }
+    };
+    if (t_first < t_end) load_bias(t_first);
     for (int t = t_first; t < t_end; t += t_step, ++tl) {
       int mt, nt, z, kb0, nk;
       decode(t, mt, nt, z, kb0, nk);
@@ -429,17 +470,17 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
       const int acc = tl % NACC;
       const uint32_t aph = (tl / NACC) & 1;
       const int m = m0 + wq * 32 + lane;
-      // before waiting for the accumulator: this warp's b2 columns into smem (coalesced
-      // loads, read back below as broadcast float4) and the row state of a new M block
+      // before waiting for the accumulator: this warp's b2 columns into smem (read back
+      // below as broadcast float4), then the next tile's b2 loads are issued into
+      // registers -- their latency hides under this tile's epilogue instead of stalling
+      // the warp at the top of every tile -- and the row state of a new M block
       if constexpr (has_bias<EPI>()) {
-        constexpr float bscale = EPI == TC_EPI_DZ ? 1.4426950408889634f : 1.f;   // DZ: log2 domain
         __syncwarp();
 #pragma unroll
-        for (int c = 0; c < CW; c += 32) {
-          const int col = n0 + wh * CW + c + lane;
-          bias_w[c + lane] = col < g.N ? __ldg(g.bias + col) * bscale : 0.f;
-        }
+        for (int c = 0; c < CW / 32; ++c)   // DZ: log2 domain
+          bias_w[32 * c + lane] = EPI == TC_EPI_DZ ? bpre[c] * 1.4426950408889634f : bpre[c];
         __syncwarp();
+        if (t + t_step < t_end) load_bias(t + t_step);
       }
       if constexpr (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG) {
         if (mt != row_mt) {
@@ -575,7 +616,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
               v[4 * q] = ex2_approx(fmaf(v[4 * q], kL2E, t.x + crow));
               v[4 * q + 1] = ex2_approx(fmaf(v[4 * q + 1], kL2E, t.y + crow));
               v[4 * q + 2] = ex2_approx(fmaf(v[4 * q + 2], kL2E, t.z + crow));
-              v[4 * q + 3] = ex2_approx(fmaf(v[4 * q + 3], kL2E, t.w + crow));
+              v[4 * q + 3] = ex2_mix(fmaf(v[4 * q + 3], kL2E, t.w + crow));
             }
             if (n + 32 > g.N) {   // columns >= N (stores are clipped; keep them finite)
 #pragma unroll
@@ -654,9 +695,14 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
         }
         if constexpr (EPI == TC_EPI_Z || EPI == TC_EPI_STATS) {
           if (g.stats) {   // online (max, sum exp) of row m over the columns seen so far
-            float cm = v[0];
+            float mx[16];   // max as a depth-5 tree (a 31-long FMNMX chain is 124 cycles of latency)
 #pragma unroll
-            for (int j = 1; j < 32; ++j) cm = fmaxf(cm, v[j]);
+            for (int j = 0; j < 16; ++j) mx[j] = fmaxf(v[j], v[j + 16]);
+#pragma unroll
+            for (int w = 8; w; w >>= 1)
+#pragma unroll
+              for (int j = 0; j < w; ++j) mx[j] = fmaxf(mx[j], mx[j + w]);
+            const float cm = mx[0];
             constexpr float kL2E = 1.4426950408889634f;
             if (cm > st_m) { st_s = (st_m == -INFINITY) ? 0.f : st_s * ex2_approx((st_m - cm) * kL2E); st_m = cm; }
             const float ms = st_m * kL2E;
@@ -666,7 +712,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
               a0 += ex2_approx(fmaf(v[j], kL2E, -ms));
               a1 += ex2_approx(fmaf(v[j + 1], kL2E, -ms));
               a2 += ex2_approx(fmaf(v[j + 2], kL2E, -ms));
-              a3 += ex2_approx(fmaf(v[j + 3], kL2E, -ms));
+              a3 += ex2_mix(fmaf(v[j + 3], kL2E, -ms));
             }
             st_s += (a0 + a1) + (a2 + a3);
           }
