@@ -702,27 +702,46 @@ __global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restr
   T* sd = reinterpret_cast<T*>(sm_raw);      // [n][CS]
   const int nsl = gridDim.y, slice = blockIdx.y, c0 = slice * CS;
   const int n = meta[M_NROWS];
-  {  // stage dA1[:, c0 : c0 + CS] (16-byte chunks, 8 loads in flight per thread)
-    constexpr int CH = CS * (int)sizeof(T) / 16;
-    const uint4* src = reinterpret_cast<const uint4*>(dA1);
-    uint4* dst = reinterpret_cast<uint4*>(sd);
-    const int rowchunks = H * (int)sizeof(T) / 16;
-    const int total = n * CH;
-    for (int i0 = threadIdx.x; i0 < total; i0 += 8 * blockDim.x) {
-      uint4 v[8];
-#pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        const int i = i0 + k * blockDim.x;
-        if (i < total) v[k] = __ldg(src + (int64_t)(i / CH) * rowchunks + slice * CH + (i % CH));
-      }
-#pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        const int i = i0 + k * blockDim.x;
-        if (i < total) dst[i] = v[k];
-      }
-    }
+  // stage dA1[:, c0 : c0 + CS] with bulk async copies (one for the whole block when the
+  // slice is the full row, else one per row issued by warp 0); the warps load their
+  // piece entries while the copy is in flight and wait on the mbarrier only before the
+  // first shared-memory gather
+  __shared__ __align__(8) uint64_t sbar;
+  const uint32_t bar = static_cast<uint32_t>(__cvta_generic_to_shared(&sbar));
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
+  if (threadIdx.x < 32) {
+    const uint32_t row_bytes = CS * (uint32_t)sizeof(T);
+    const uint32_t dst0 = static_cast<uint32_t>(__cvta_generic_to_shared(sd));
+    if (threadIdx.x == 0)
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"((uint32_t)n * row_bytes)
+                   : "memory");
+    __syncwarp();
+    if (nsl == 1) {
+      if (threadIdx.x == 0 && n > 0)
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst0),
+                     "l"(dA1), "r"((uint32_t)n * row_bytes), "r"(bar)
+                     : "memory");
+    } else {
+      for (int r = threadIdx.x; r < n; r += 32)
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                         dst0 + (uint32_t)r * row_bytes),
+                     "l"(dA1 + (int64_t)r * H + c0), "r"(row_bytes), "r"(bar)
+                     : "memory");
+    }
+  }
+  bool staged = false;
+  auto wait_staged = [&]() {
+    if (staged) return;
+    uint32_t ok = 0;
+    while (!ok)
+      asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                   : "=r"(ok) : "r"(bar) : "memory");
+    staged = true;
+  };
   const int lane = threadIdx.x & 31;
   const int nnz = meta[M_NNZ];
   const int npieces = (nnz + kPiece - 1) / kPiece;
@@ -740,6 +759,7 @@ __global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restr
     const int fprev = __shfl_sync(kFull, nb, 0), fnext = __shfl_sync(kFull, nb, 1);
     const int fup = __shfl_up_sync(kFull, myf, 1);
     uint32_t smask = __ballot_sync(kFull, lane < cnt && (lane == 0 || myf != fup));
+    wait_staged();
     while (smask) {
       const int j0 = __ffs(smask) - 1;
       smask &= smask - 1;
@@ -817,6 +837,7 @@ __global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restr
       }
     }
   }
+  wait_staged();   // no CTA exits with its bulk copy still writing shared memory
 }
 
 // One resident wave of 256-thread CTAs (occupancy from the compiled kernel), no

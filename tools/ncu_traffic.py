@@ -20,11 +20,13 @@ SECTIONS = {"dh_b1": 2, "merge": 3}
 def kclass(name: str):
     if name.startswith("k_gemm_tc"):
         epi = int(re.findall(r"\d+", name.split("<")[1])[-1])
-        return {0: "g1", 1: "g2", 2: "g3", 3: "softmax"}[epi]
+        return {0: "g1", 1: "g2", 2: "g3", 3: "softmax", 4: "g1", 5: "g1"}[epi]   # 4: sigmoid G1, 5: stats G1
     for pre, cls in (("k_touched", "touched"), ("k_spmm_fwd", "spmm"), ("k_softmax_ce", "softmax"),
                      ("k_lse", "softmax"), ("k_dh_reduce", "dh_b1"), ("k_b1_update", "dh_b1"),
                      ("k_scatter_sgd", "scatter"), ("k_sqnorm", "merge"), ("k_scale", "merge"),
-                     ("k_finish", "merge"), ("k_gemm_f32", None), ("k_b2_", "b2")):
+                     ("k_finish", "merge"), ("k_merge_fused", "merge"), ("k_merge_wait", "merge"),
+                     ("k_tile_loss", "softmax"), ("k_sig_center", "softmax"), ("k_sigmoid_ce", "softmax"),
+                     ("k_gemm_f32", None), ("k_b2_", "b2")):
         if name.startswith(pre):
             return cls
     return None
