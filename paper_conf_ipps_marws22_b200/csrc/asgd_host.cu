@@ -60,6 +60,14 @@ constexpr int kMaxInflight = 8;
 // Above this many bytes of fp32 logits per step the bf16 path fuses softmax-CE
 // into the GEMMs (Z never written); below, Z stays L2-resident and is stored.
 constexpr int64_t kFusedCeBytes = 64ll << 20;
+// threshold override in MB (A/B experiments only)
+int64_t fused_ce_bytes() {
+  static const int64_t v = [] {
+    const char* e = getenv("ASGD_FUSED_CE_MB");
+    return e ? (int64_t)atoll(e) << 20 : kFusedCeBytes;
+  }();
+  return v;
+}
 
 int splitk_for(const asgd_model_desc& d) {
   // G2 (dH1 = dZ W2, M = b_max, N = H, K = L): split K so ~2 waves of CTAs run.
@@ -557,7 +565,7 @@ int enqueue_step(asgd_ctx* c, int n) {
                                     : launch_sig_center(lc, Pr.w2b, Lb, H, P.h1, n, P.cenpart,
                                                         reinterpret_cast<unsigned int*>(P.meta + M_CEN), P.cen);
           })());
-    } else if ((int64_t)m.b_max * Lb * 4 <= kFusedCeBytes) {
+    } else if ((int64_t)m.b_max * Lb * 4 <= fused_ce_bytes()) {
       // logits fit in L2: G1 stores Z (+ per-tile softmax partials), one pass of softmax-CE
       PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
       PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, true, zstat, ntiles,

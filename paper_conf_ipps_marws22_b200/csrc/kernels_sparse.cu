@@ -698,35 +698,37 @@ __global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restr
   const float lr = step_lr(meta);
   constexpr int CS = 32 * CPL;               // columns of this CTA's slice
   constexpr int kU = 8;
+#ifndef ASGD_SEG_AHEAD
+#define ASGD_SEG_AHEAD 1
+#endif
+  constexpr int kSegAhead = ASGD_SEG_AHEAD;   // segments whose W1 rows are in flight together
   extern __shared__ __align__(16) uint8_t sm_raw[];
   T* sd = reinterpret_cast<T*>(sm_raw);      // [n][CS]
   const int nsl = gridDim.y, slice = blockIdx.y, c0 = slice * CS;
   const int n = meta[M_NROWS];
   // stage dA1[:, c0 : c0 + CS] with bulk async copies (one for the whole block when the
-  // slice is the full row, else one per row issued by warp 0); the warps load their
+  // slice is the full row, else one per row, issued by every thread); the warps load their
   // piece entries while the copy is in flight and wait on the mbarrier only before the
   // first shared-memory gather
   __shared__ __align__(8) uint64_t sbar;
   const uint32_t bar = static_cast<uint32_t>(__cvta_generic_to_shared(&sbar));
+  const uint32_t row_bytes = CS * (uint32_t)sizeof(T);
   if (threadIdx.x == 0) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar) : "memory");
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"((uint32_t)n * row_bytes)
+                 : "memory");
   }
   __syncthreads();
-  if (threadIdx.x < 32) {
-    const uint32_t row_bytes = CS * (uint32_t)sizeof(T);
+  {
     const uint32_t dst0 = static_cast<uint32_t>(__cvta_generic_to_shared(sd));
-    if (threadIdx.x == 0)
-      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"((uint32_t)n * row_bytes)
-                   : "memory");
-    __syncwarp();
-    if (nsl == 1) {
+    if (nsl == 1) {   // the slice is the whole row: one copy
       if (threadIdx.x == 0 && n > 0)
         asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst0),
                      "l"(dA1), "r"((uint32_t)n * row_bytes), "r"(bar)
                      : "memory");
-    } else {
-      for (int r = threadIdx.x; r < n; r += 32)
+    } else {          // one copy per row, issued by every thread of the block
+      for (int r = threadIdx.x; r < n; r += blockDim.x)
         asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                          dst0 + (uint32_t)r * row_bytes),
                      "l"(dA1 + (int64_t)r * H + c0), "r"(row_bytes), "r"(bar)
@@ -761,14 +763,35 @@ __global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restr
     uint32_t smask = __ballot_sync(kFull, lane < cnt && (lane == 0 || myf != fup));
     wait_staged();
     while (smask) {
-      const int j0 = __ffs(smask) - 1;
-      smask &= smask - 1;
-      const int j1 = smask ? __ffs(smask) - 1 : cnt;
+      // kSegAhead segments at a time: their W1 row slices are all requested before the
+      // first one is summed (1 = one segment at a time; A/B switch ASGD_SEG_AHEAD)
+      int sj0[kSegAhead], sj1[kSegAhead];
+      float wp[kSegAhead][CPL];
+#pragma unroll
+      for (int d = 0; d < kSegAhead; ++d) {
+        sj0[d] = -1;
+        sj1[d] = 0;
+        if (smask) {   // warp-uniform
+          const int a = __ffs(smask) - 1;
+          smask &= smask - 1;
+          const int b = smask ? __ffs(smask) - 1 : cnt;
+          sj0[d] = a;
+          sj1[d] = b;
+          const int fa = __shfl_sync(kFull, myf, a);
+          if (!((a == 0 && fprev == fa) || (b == cnt && fnext == fa)))   // in flight during the gathers
+            ld_cols<CPL>(W1 + (int64_t)fa * H + c0 + lane * CPL, wp[d], false);
+        }
+      }
+#pragma unroll
+      for (int d = 0; d < kSegAhead; ++d) {
+      if (sj0[d] < 0) break;   // warp-uniform
+      const int j0 = sj0[d], j1 = sj1[d];
       const int f = __shfl_sync(kFull, myf, j0), u = __shfl_sync(kFull, myu, j0);
       const bool before = (j0 == 0 && fprev == f), after = (j1 == cnt && fnext == f);
       float* wrow = W1 + (int64_t)f * H + c0 + lane * CPL;
       float w[CPL];
-      if (!before && !after) ld_cols<CPL>(wrow, w, false);     // in flight during the gathers
+#pragma unroll
+      for (int i = 0; i < CPL; ++i) w[i] = wp[d][i];   // boundary segments reload it below
       float acc[CPL];
 #pragma unroll
       for (int i = 0; i < CPL; ++i) acc[i] = 0.f;
@@ -834,6 +857,7 @@ __global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restr
         st_cols<CPL>(wrow, w, false);
         if (grad_w1) st_cols<CPL>(grad_w1 + (int64_t)f * H + c0 + lane * CPL, acc, false);
         if (slice == 0) reset_feature(fcnt, bits, W, f, lane);
+      }
       }
     }
   }
