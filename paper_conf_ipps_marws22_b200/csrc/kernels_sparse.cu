@@ -682,8 +682,14 @@ __device__ __forceinline__ void st_cols(float* p, const float (&v)[CPL], bool cg
   }
 }
 
+// Threads per K-5 CTA: the bf16 64-column slices (AmazonCat, Amazon-670K: ~10 short
+// segments per piece, each waiting on one W1 row slice from HBM) fit 64 registers, so
+// they run 32 warps per SM instead of 16 for twice the row loads in flight.
 template <typename T, int CPL>
-__global__ void __launch_bounds__(512, 1) k_scatter_sgd_s(const int32_t* __restrict__ e_n,
+constexpr int scatter_threads() { return (sizeof(T) == 2 && CPL == 2) ? 1024 : 512; }
+
+template <typename T, int CPL>
+__global__ void __launch_bounds__(scatter_threads<T, CPL>(), 1) k_scatter_sgd_s(const int32_t* __restrict__ e_n,
                                                           const float* __restrict__ e_v,
                                                           const int32_t* __restrict__ e_u,
                                                           const int32_t* __restrict__ e_f,
@@ -961,7 +967,7 @@ cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float*
     attr = true;
   }
   const int gx = std::max(1, lc.sms / nsl);
-  return launch_k(lc, k_scatter_sgd_s<T, CPL>, dim3(gx, nsl), dim3(512), smem, P.e_n, P.e_v, P.e_u,
+  return launch_k(lc, k_scatter_sgd_s<T, CPL>, dim3(gx, nsl), dim3(scatter_threads<T, CPL>()), smem, P.e_n, P.e_v, P.e_u,
                   P.e_f, P.useg, P.meta, dA1, H, W1, P.part5, P.ucnt, grad_w1, P.cnt, P.bits,
                   (b_max + 31) / 32);
 }
