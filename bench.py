@@ -168,7 +168,7 @@ def kernel_work(cls: str, cfg, bf16: bool, st, loss: str = "softmax"):
     B, H, L, F, P = st["B"], cfg.H, cfg.L, cfg.F, cfg.n_params
     nnz, U = st["nnz"], st["U"]
     e = 2.0 if bf16 else 4.0                      # bytes per GEMM operand element
-    fused = bf16 and loss == "softmax" and cfg.b_max * L * 4 > (64 << 20)
+    fused = bf16 and loss == "softmax" and cfg.b_max * L * 4 > (32 << 20)
     gemm = 2.0 * B * H * L
     if cls == "g1":     # H1 . W2^T + b2: W2 (shadow) + H1 in; Z (fp32, unfused) or 2 fp32 stats per row and tile
         out = (8.0 * B * 2 * ((L + 255) // 256)) if (fused or (bf16 and loss == "sigmoid")) else 4.0 * B * L

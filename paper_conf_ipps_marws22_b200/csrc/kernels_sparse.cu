@@ -383,9 +383,14 @@ __global__ void __launch_bounds__(512) k_touched(StepArgs sa, const int64_t* __r
 // -------------------------------------------------------------------------
 // K-1: A1 = X W1 + b1, H1 = ReLU(A1)
 // -------------------------------------------------------------------------
+#ifndef ASGD_K1_GROUP
+#define ASGD_K1_GROUP 16   // measured (8 / 16 / per-piece partials): EURLex 3.64 / 4.02 / 4.02 M, Wiki10 1.30 / 1.35 / 1.27 M samples/s
+#endif
+template <int VPL>   // pieces per group = warps per K-1 CTA (H = 512: 8, the partials fill 32 KB)
+constexpr int k1_group() { return VPL >= 16 ? 8 : ASGD_K1_GROUP; }
 template <int VPL>
 // (256, 2): two CTAs per SM, all kU gathers of a group in flight (<= 128 regs)
-__global__ void __launch_bounds__(256, 2) k_spmm_fwd(StepArgs sa, const int64_t* __restrict__ row_ptr,
+__global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_spmm_fwd(StepArgs sa, const int64_t* __restrict__ row_ptr,
                                                   const int64_t* __restrict__ lab_ptr, int64_t n_data_rows,
                                                   int64_t nz_cap, int64_t nl_cap, ViewOut vo,
                                                   const int32_t* __restrict__ col,
@@ -405,97 +410,145 @@ __global__ void __launch_bounds__(256, 2) k_spmm_fwd(StepArgs sa, const int64_t*
   const int lane = threadIdx.x & 31;
   const int npieces = (nnz + kPiece - 1) / kPiece;
   const int nwarps = gridDim.x * (blockDim.x >> 5);
-  float bias[VPL];
-  IO::load_ldg(b1, lane, bias);
 
-  // Row segment [.., ..) of row r ends inside this piece: finish it (ReLU(acc + b1))
-  // when the piece holds the whole row, else publish a partial; the last of the
-  // row's pieces to arrive sums the partials in piece order and finishes.
-  auto flush = [&](int p, int e0, int e1, int r, float (&acc)[VPL]) {
-    const int rs = sboff[r], re = sboff[r + 1];
-    const bool before = rs < e0, after = re > e1;
-    if (before || after) {
-      IO::store_cg(part + (int64_t)(before ? 2 * p : 2 * p + 1) * H, lane, acc);
-      __threadfence();
-      int old = 0;
-      if (lane == 0) old = atomicAdd(&rowcnt[r], 1);
-      old = __shfl_sync(kFull, old, 0);
-      const int q0 = rs / kPiece, q1 = (re - 1) / kPiece;
-      if (old != q1 - q0) return;
-      __threadfence();
-#pragma unroll
-      for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
-      for (int q = q0; q <= q1; q += 4) {   // 4 partials in flight, summed in piece order
-        float t[4][VPL];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          if (q + u <= q1) IO::load_cg(part + (int64_t)(q + u == q0 ? 2 * q0 + 1 : 2 * (q + u)) * H, lane, t[u]);
-          else {
-#pragma unroll
-            for (int i = 0; i < VPL; ++i) t[u][i] = 0.f;
-          }
-        }
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          if (q + u <= q1) {
-#pragma unroll
-            for (int i = 0; i < VPL; ++i) acc[i] += t[u][i];
-          }
-        }
-      }
-      if (lane == 0) rowcnt[r] = 0;
-    }
+  // Pieces are taken in groups of 8 consecutive pieces, one per warp of the CTA, so a
+  // row that crosses pieces is first combined inside the CTA through shared memory;
+  // only rows that cross a group boundary go through global partials, one per group.
+  constexpr int kGroup = k1_group<VPL>();        // pieces per group = warps per CTA
+  __shared__ __align__(16) float spart[kGroup][2][H];   // per warp: [0] its first segment, [1] its last
+  const int warp = threadIdx.x >> 5;
+  const int ngroups = (npieces + kGroup - 1) / kGroup;
+  auto finish = [&](int r, float (&acc)[VPL]) {
+    float bias[VPL];   // b1 re-read (L1) instead of held in registers across the gathers
+    IO::load_ldg(b1, lane, bias);
 #pragma unroll
     for (int i = 0; i < VPL; ++i) acc[i] = fmaxf(acc[i] + bias[i], 0.f);
     IO::store(H1 + (int64_t)r * H, lane, acc);
     if (H1b) IO::store_bf16(H1b + (int64_t)r * H, lane, acc);
   };
-
-  for (int p = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); p < npieces; p += nwarps) {
-    const int e0 = p * kPiece, e1 = min(e0 + kPiece, nnz), cnt = e1 - e0;
-    // lane j holds entry e0 + j: its row, column and value (one round trip)
-    int myr = 0, mycol = 0;
-    float myval = 0.f;
-    if (lane < cnt) {
-      myr = entry_row(sboff, n, e0 + lane);
-      const int64_t k = srb[myr] + (e0 + lane - sboff[myr]);
-      mycol = __ldg(col + k);
-      myval = __ldg(val + k);
-    }
-    int rcur = __shfl_sync(kFull, myr, 0);
-    float acc[VPL];
+  // group g's partial of row r (global): slot 2 g + 1 if r starts in g, else 2 g; the
+  // last group to arrive sums the row's group partials in group order and finishes
+  auto publish = [&](int g, int r, float (&acc)[VPL]) {
+    constexpr int GE = kGroup * kPiece;          // entries per group
+    const int rs = sboff[r], re = sboff[r + 1];
+    const int g0 = rs / GE, g1 = (re - 1) / GE;
+    IO::store_cg(part + (int64_t)(g == g0 ? 2 * g + 1 : 2 * g) * H, lane, acc);
+    __threadfence();
+    int old = 0;
+    if (lane == 0) old = atomicAdd(&rowcnt[r], 1);
+    old = __shfl_sync(kFull, old, 0);
+    if (old != g1 - g0) return;
+    __threadfence();
 #pragma unroll
     for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
-    // groups of kU W1 rows in flight, row changes handled between FMAs
-    for (int j0 = 0; j0 < cnt; j0 += kU) {
-      float w[kU][VPL];
+    for (int q = g0; q <= g1; q += 4) {   // 4 partials in flight, summed in group order
+      float t[4][VPL];
 #pragma unroll
-      for (int q = 0; q < kU; ++q) {
-        const int c = __shfl_sync(kFull, mycol, j0 + q);
-        if (j0 + q < cnt) IO::load_ldg(W1 + (int64_t)c * H, lane, w[q]);
+      for (int u = 0; u < 4; ++u) {
+        if (q + u <= g1) IO::load_cg(part + (int64_t)(q + u == g0 ? 2 * g0 + 1 : 2 * (q + u)) * H, lane, t[u]);
         else {
 #pragma unroll
-          for (int i = 0; i < VPL; ++i) w[q][i] = 0.f;
+          for (int i = 0; i < VPL; ++i) t[u][i] = 0.f;
         }
       }
 #pragma unroll
-      for (int q = 0; q < kU; ++q) {
-        const int j = j0 + q;
-        const int rq = __shfl_sync(kFull, myr, j);
-        const float v = __shfl_sync(kFull, myval, j);
-        if (j < cnt) {
-          if (rq != rcur) {
-            flush(p, e0, e1, rcur, acc);
+      for (int u = 0; u < 4; ++u) {
+        if (q + u <= g1) {
 #pragma unroll
-            for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
-            rcur = rq;
-          }
-#pragma unroll
-          for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, w[q][i], acc[i]);
+          for (int i = 0; i < VPL; ++i) acc[i] += t[u][i];
         }
       }
     }
-    if (cnt > 0) flush(p, e0, e1, rcur, acc);
+    if (lane == 0) rowcnt[r] = 0;
+    finish(r, acc);
+  };
+
+  for (int g = blockIdx.x; g < ngroups; g += gridDim.x) {
+    const int p = g * kGroup + warp;
+    const int G0 = g * kGroup * kPiece, G1 = min(G0 + kGroup * kPiece, nnz);
+    const int e0 = p * kPiece, e1 = min(e0 + kPiece, nnz), cnt = max(0, e1 - e0);
+    // Row segment of row r ends inside this piece: finish it (ReLU(acc + b1)) when the
+    // piece holds the whole row, else park it in shared memory for the group combine
+    auto flush = [&](int r, float (&acc)[VPL]) {
+      const int rs = sboff[r], re = sboff[r + 1];
+      const bool before = rs < e0, after = re > e1;
+      if (!before && !after) { finish(r, acc); return; }
+      IO::store(&spart[warp][before ? 0 : 1][0], lane, acc);
+    };
+    int rfirst = -1, rlast = -1;   // rows of this piece's first / last entry
+    if (cnt > 0) {
+      // lane j holds entry e0 + j: its row, column and value (one round trip)
+      int myr = 0, mycol = 0;
+      float myval = 0.f;
+      if (lane < cnt) {
+        myr = entry_row(sboff, n, e0 + lane);
+        const int64_t k = srb[myr] + (e0 + lane - sboff[myr]);
+        mycol = __ldg(col + k);
+        myval = __ldg(val + k);
+      }
+      int rcur = __shfl_sync(kFull, myr, 0);
+      rfirst = rcur;
+      rlast = __shfl_sync(kFull, myr, cnt - 1);
+      float acc[VPL];
+#pragma unroll
+      for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+      // groups of kU W1 rows in flight, row changes handled between FMAs
+      for (int j0 = 0; j0 < cnt; j0 += kU) {
+        float w[kU][VPL];
+#pragma unroll
+        for (int q = 0; q < kU; ++q) {
+          const int c = __shfl_sync(kFull, mycol, j0 + q);
+          if (j0 + q < cnt) IO::load_ldg(W1 + (int64_t)c * H, lane, w[q]);
+          else {
+#pragma unroll
+            for (int i = 0; i < VPL; ++i) w[q][i] = 0.f;
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < kU; ++q) {
+          const int j = j0 + q;
+          const int rq = __shfl_sync(kFull, myr, j);
+          const float v = __shfl_sync(kFull, myval, j);
+          if (j < cnt) {
+            if (rq != rcur) {
+              flush(rcur, acc);
+#pragma unroll
+              for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+              rcur = rq;
+            }
+#pragma unroll
+            for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, w[q][i], acc[i]);
+          }
+        }
+      }
+      flush(rcur, acc);
+    }
+    __syncthreads();
+    // group combine: warp w takes the rows whose first segment inside the group is in
+    // its piece and that continue past it (or reach back before the group, warp 0),
+    // sums the parked segments of the following warps in warp order, then finishes
+    // the row or publishes the group's partial
+    if (cnt > 0) {
+      for (int k = 0; k < 2; ++k) {
+        if (k == 1 && rlast == rfirst) break;
+        const int r = k == 0 ? rfirst : rlast;
+        const int rs = sboff[r], re = sboff[r + 1];
+        const bool before = rs < e0, after = re > e1;
+        if (!before && !after) continue;        // finished in flush
+        if (max(rs, G0) < e0) continue;          // an earlier warp of the group holds its first segment
+        float acc[VPL];
+        IO::load(&spart[warp][before ? 0 : 1][0], lane, acc);
+        for (int w2 = warp + 1; w2 < kGroup && (g * kGroup + w2) * kPiece < min(re, G1); ++w2) {
+          float t[VPL];
+          IO::load(&spart[w2][0][0], lane, t);   // row r is w2's first segment
+#pragma unroll
+          for (int i = 0; i < VPL; ++i) acc[i] += t[i];
+        }
+        if (rs >= G0 && re <= G1) finish(r, acc);
+        else publish(g, r, acc);
+      }
+    }
+    __syncthreads();   // spart is reused by the next group
   }
   // rows without entries: H1 = ReLU(b1)
   const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
@@ -503,9 +556,8 @@ __global__ void __launch_bounds__(256, 2) k_spmm_fwd(StepArgs sa, const int64_t*
     if (sboff[r + 1] == sboff[r]) {
       float acc[VPL];
 #pragma unroll
-      for (int i = 0; i < VPL; ++i) acc[i] = fmaxf(bias[i], 0.f);
-      IO::store(H1 + (int64_t)r * H, lane, acc);
-      if (H1b) IO::store_bf16(H1b + (int64_t)r * H, lane, acc);
+      for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+      finish(r, acc);
     }
   }
 }
@@ -873,10 +925,10 @@ __global__ void __launch_bounds__(scatter_threads<T, CPL>(), 1) k_scatter_sgd_s(
 // One resident wave of 256-thread CTAs (occupancy from the compiled kernel), no
 // more CTAs than there are 8-piece groups for the largest step.
 template <typename K>
-int wave_grid(const Launch& lc, K kernel, size_t smem, int64_t pieces, int& occ) {
-  if (!occ && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, 256, smem) != cudaSuccess || occ < 1))
+int wave_grid(const Launch& lc, K kernel, size_t smem, int64_t pieces, int& occ, int warps = 8) {
+  if (!occ && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, 32 * warps, smem) != cudaSuccess || occ < 1))
     occ = 1;
-  const int64_t need = (pieces + 7) / 8;
+  const int64_t need = (pieces + warps - 1) / warps;
   return (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)lc.sms * occ));
 }
 
@@ -884,10 +936,17 @@ template <int VPL>
 cudaError_t spmm_fwd_t(const Launch& lc, const StepArgs& sa, const asgd_csr& x, const float* W1, const float* b1,
                        const Ptrs& P, const WsLayout& L, bool want_bf16) {
   const size_t smem = view_smem(sa.n);
+  static bool attr = false;
+  if (!attr) {   // the batch view (dynamic) + the group partials (static) exceed 48 KB at b_max = 2048
+    cudaError_t e = cudaFuncSetAttribute(k_spmm_fwd<VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)view_smem(2048));
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
   static int occ = 0;
-  const int grid = wave_grid(lc, k_spmm_fwd<VPL>, view_smem(2048), L.n_pieces, occ);
+  const int grid = wave_grid(lc, k_spmm_fwd<VPL>, view_smem(2048), L.n_pieces, occ, k1_group<VPL>());
   const ViewOut vo{P.boff, P.loff, P.rbase, P.rowsc, P.meta};
-  launch_k(lc, k_spmm_fwd<VPL>, dim3(grid), dim3(256), smem, sa, x.row_ptr, x.lab_ptr, x.n_rows, L.nz_cap, L.nl_cap,
+  launch_k(lc, k_spmm_fwd<VPL>, dim3(grid), dim3(32 * k1_group<VPL>()), smem, sa, x.row_ptr, x.lab_ptr, x.n_rows, L.nz_cap, L.nl_cap,
            vo, x.col, x.val, W1, b1, P.h1, want_bf16 ? P.h1b : nullptr, P.part1, P.rowcnt);
   return cudaGetLastError();
 }
