@@ -65,6 +65,7 @@ struct Launch {       // launch bookkeeping of one ctx
   cudaStream_t s;
   int64_t* counter;
   int sms;
+  bool pdl;           // programmatic dependent launch (see pdl_mode)
 };
 
 // Programmatic dependent launch: every kernel of the step lets its successor be
@@ -75,7 +76,10 @@ struct Launch {       // launch bookkeeping of one ctx
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 
-bool pdl_enabled();   // ASGD_PDL=0 disables programmatic dependent launch (default on)
+// ASGD_PDL: unset = on for the bf16 path, off for fp32; 0 off; 1 every kernel; 2 the
+// tcgen05 GEMMs only
+int pdl_mode();
+bool pdl_for(bool bf16);   // launch_k: this ctx's kernels use PDL
 
 template <typename... KArgs, typename... Args>
 cudaError_t launch_k(const Launch& lc, void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
@@ -89,7 +93,24 @@ cudaError_t launch_k(const Launch& lc, void (*kernel)(KArgs...), dim3 grid, dim3
   at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
-  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  cfg.numAttrs = lc.pdl ? 1 : 0;
+  ++*lc.counter;
+  return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
+
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k_pdl(const Launch& lc, bool pdl, void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                     Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = lc.s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl ? 1 : 0;
   ++*lc.counter;
   return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
 }

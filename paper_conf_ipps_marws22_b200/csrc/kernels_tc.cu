@@ -853,8 +853,8 @@ cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, co
   g.splits = splits;
   const int64_t tiles = (int64_t)((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN) * splits;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, lc.sms));
-  return launch_k(lc, k_gemm_tc<BN, A_MN, B_MN, EPI>, dim3(grid), dim3(128 + 32 * epi_warps<BN, EPI>()), smem, a, b,
-                  c, d, g);
+  return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_gemm_tc<BN, A_MN, B_MN, EPI>, dim3(grid),
+                      dim3(128 + 32 * epi_warps<BN, EPI>()), smem, a, b, c, d, g);
 }
 
 // Widest N tile that still gives >= one CTA per SM (and does not overhang N by 2x).
