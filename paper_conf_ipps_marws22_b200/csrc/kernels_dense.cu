@@ -106,18 +106,11 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
   __shared__ float s_m[16], s_s[16];
   __shared__ float s_lse, s_lsum;
   const int n = blockIdx.x;
-  const int64_t id = rows[n];
-  const int64_t l0 = lab_ptr[id];
-  const int64_t nl64 = lab_ptr[id + 1] - l0;
-  const int nl = (int)(nl64 < kMaxRowLabels ? nl64 : kMaxRowLabels);
-  float* z = Z + (int64_t)n * ldz;
-  for (int i = threadIdx.x; i < nl; i += blockDim.x) {
-    int y = lab[l0 + i];
-    s_lab[i] = y;
-    s_lz[i] = z[y];
-  }
+  const int64_t id = rows[n];   // in flight with the partials below
   // pass 1: online max / sum-exp, kSU loads in flight per thread -- or, when G1
-  // left per-tile partials, combine those instead of re-reading the row.
+  // left per-tile partials, combine those instead of re-reading the row.  The
+  // partials need only n, so they are combined before the label chain
+  // (rows -> lab_ptr -> lab -> Z) starts instead of after it.
   constexpr int kSU = 8;
   float m = -INFINITY, s = 0.f;
   if (stats) {
@@ -127,6 +120,15 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
       if (p.x > m) { s = (m == -INFINITY ? 0.f : s * __expf(m - p.x)) + p.y; m = p.x; }
       else s += p.y * __expf(p.x - m);
     }
+  }
+  const int64_t l0 = lab_ptr[id];
+  const int64_t nl64 = lab_ptr[id + 1] - l0;
+  const int nl = (int)(nl64 < kMaxRowLabels ? nl64 : kMaxRowLabels);
+  float* z = Z + (int64_t)n * ldz;
+  for (int i = threadIdx.x; i < nl; i += blockDim.x) {
+    int y = lab[l0 + i];
+    s_lab[i] = y;
+    s_lz[i] = z[y];
   }
   for (int64_t j0 = stats ? L : threadIdx.x; j0 < L; j0 += (int64_t)kSU * blockDim.x) {
     float v[kSU];
