@@ -1,0 +1,8 @@
+# G1b / sigmoid G1 epilogues: next label prefetched one ahead
+mkdir -p gpurun_out
+show() { python -c "
+import json,sys; d=json.loads(open('$1').read().strip().splitlines()[-1]); print('$1', d['value'], d['ms_per_step'], {k:v['us_per_launch'] for k,v in d['kernels_warmup_profile'].items()})"; }
+timeout 900 python -m pytest tests/test_gpu_step.py tests/test_gpu_large.py -m gpu -x -q 2>&1 | tail -1
+for i in 1 2; do timeout 900 python bench.py --config amazon670k --steps 3 --no-cpu-baseline --ttp-megabatches 0 --e2e-steps 0 > gpurun_out/r5d_a670k_$i.json 2>&1; show gpurun_out/r5d_a670k_$i.json; done
+timeout 900 python bench.py --config delicious200k --steps 3 --no-cpu-baseline --ttp-megabatches 0 --e2e-steps 0 > gpurun_out/r5d_del.json 2>&1; show gpurun_out/r5d_del.json
+timeout 900 python bench.py --config amazon670k --loss sigmoid --steps 3 --no-cpu-baseline --ttp-megabatches 0 --e2e-steps 0 > gpurun_out/r5d_a670k_sig.json 2>&1; show gpurun_out/r5d_a670k_sig.json
