@@ -219,6 +219,31 @@ def roofline_of(cls, cfg, bf16, st, loss, avg_s, peaks):
     return {"bound": "hbm", "achieved": by / avg_s / 1e9, "peak": hbm, "unit": "GB/s", "work_per_launch": by}
 
 
+def l2_view(cls, cfg, bf16, st, avg_s):
+    """Secondary roofline for the sparse kernels, whose operands are L2-resident at
+    EURLex size: the bytes they actually move through L2 per launch (K-1: fp32 W1 row
+    gathers 4 nnz H + entries 8 nnz + H1 fp32/bf16 6 B H; K-5: W1 rows read and
+    written 8 U H + entries 16 nnz + each CTA's staged dA1 slice) over the launch time,
+    against the L2-resident copy bandwidth measured by tools/l2_peak.py."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "l2_peak.json")) as f:
+            peak = float(json.load(f)["l2_gbs"])
+    except Exception:
+        return None
+    B, H, nnz, U = st["B"], cfg.H, st["nnz"], st["U"]
+    if cls == "spmm":
+        by = 4.0 * nnz * H + 8.0 * nnz + 6.0 * B * H
+    elif cls == "scatter":
+        elem = 2 if bf16 else 4
+        cs = next((c for c in (256, 128, 64) if c <= H and H % c == 0 and cfg.b_max * c * elem <= 160 * 1024), H)
+        by = 8.0 * U * H + 16.0 * nnz + 148.0 * B * cs * elem   # 148 CTAs each stage a B x cs slice
+    else:
+        return None
+    ach = by / avg_s / 1e9
+    return {"bytes_per_launch": by, "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(ach / peak, 4), "peak_source": "profiles/l2_peak.json (torch copy, L2-resident)"}
+
+
 def step_ideal_s(cfg, B, nnz, U, nlab, hbm_gbs, tc_tflops):
     """SURVEY.md §8(d) ideal time of one local step: max(algorithmic HBM bytes /
     HBM peak, algorithmic flops / tensor peak).  Bytes: 8 nnz + 12 B + 4 labels
@@ -374,6 +399,9 @@ def main():
                 "step_share": round(float(ms[dom] / max(t_prof_ms, 1e-9)), 4),
                 "timed_in": f"second pass of {K} mega-batches with CUDA events around each launch "
                             f"({t_prof_ms / K:.4f} ms per mega-batch there vs {t_ms / K:.4f} ms unprofiled)"}
+        lv = l2_view(dname, cfg, bf16, wl, avg_s)
+        if lv:
+            roof["l2_view"] = lv
         side = {}
         for i in range(len(names)):
             if names[i] == "touched" and wcnt[i]:
