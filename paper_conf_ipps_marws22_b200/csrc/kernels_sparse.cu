@@ -548,7 +548,7 @@ __global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_
         else publish(g, r, acc);
       }
     }
-    __syncthreads();   // spart is reused by the next group
+    if (g + (int)gridDim.x < ngroups) __syncthreads();   // spart is reused by this CTA's next group
   }
   // rows without entries: H1 = ReLU(b1)
   const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
