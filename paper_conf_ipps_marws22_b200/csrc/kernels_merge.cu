@@ -174,6 +174,7 @@ __global__ void __launch_bounds__(256) k_merge_fused(PeerSet ps, float* w, float
 }
 
 __global__ void k_merge_wait(const unsigned long long* arrived, unsigned long long goal) {
+  pdl_wait();   // launched with programmatic dependent launch: start polling after k_merge_fused completed
   unsigned long long v;
   do {
     asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(arrived) : "memory");
