@@ -50,6 +50,10 @@ def _args():
                    help="fused: peer-memory merge kernel over CUDA IPC (NEXT-1); nccl: prescale + all_reduce + epilogue")
     p.add_argument("--loss", default="softmax", choices=["softmax", "sigmoid"],
                    help="output head: softmax-CE (the paper's) or per-label sigmoid BCE (R11)")
+    p.add_argument("--norm", default="u", choices=["u", "ub"],
+                   help="Alg. 2 line 3: u_i-normalised (the paper's default) or u_i b_i (R12, P:1088-1090)")
+    p.add_argument("--scale-every", type=int, default=1,
+                   help="run Alg. 1 after every k-th mega-batch (R13, P:922-925; 1 = the paper's default)")
     p.add_argument("--e2e-steps", type=int, default=None)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -285,7 +289,7 @@ def main():
     rep = api.Replica(cfg.F, cfg.L, cfg.H, cfg.b_max, nz, nl, prec, device=local, w0=w0, loss=a.loss)
     dd = api.DeviceCsr(data, device=dev)
     rep.register(dd)
-    h = train.Hyper.from_config(cfg)
+    h = train.Hyper.from_config(cfg, norm=a.norm, scale_every=a.scale_every)
     M = h.M
     shm = f"/asgd_bench_{os.environ.get('MASTER_PORT', os.getpid())}"
     if rank == 0:
@@ -428,6 +432,7 @@ def main():
                        "precision": prec, "l2": "flushed (256 MiB write) between timed steps",
                        "inflight": a.inflight, "parallelism": f"dp{world} (model averaging)",
                        "merge": merge_used, "method": a.method, "loss": a.loss,
+                       "norm": a.norm, "scale_every": a.scale_every,
                        "mean_batch_nnz": round(wl["nnz"], 1), "mean_touched_rows": round(wl["U"], 1)},
             "roofline": roof,
             "side_stream": side,
@@ -438,7 +443,8 @@ def main():
             "cpu_baseline": None,
         }
         if world == 1 and a.ttp_megabatches > 0:
-            out["time_to_p1"] = time_to_p1(cfg, prec, a.ttp_megabatches, dev, lr_max=a.lr_max, loss=a.loss)
+            out["time_to_p1"] = time_to_p1(cfg, prec, a.ttp_megabatches, dev, lr_max=a.lr_max, loss=a.loss,
+                                           norm=a.norm, scale_every=a.scale_every)
         if world == 1 and not a.no_cpu_baseline:
             out["cpu_baseline"], _ = cpu_baseline(cfg, data, a.cpu_seconds, a.loss)
         print(json.dumps(out), flush=True)
@@ -506,7 +512,8 @@ def run_e2e(rep, drv, data, ids_list, dev, flush, world, M):
             "h2d_bytes_per_step": int(h2d * world / Ke), "d2h_bytes_per_step": int(d2h * world / Ke)}
 
 
-def time_to_p1(cfg, prec, n_mb, dev, pert_renorm=False, lr_max=None, eval_rows=10000, loss="softmax"):
+def time_to_p1(cfg, prec, n_mb, dev, pert_renorm=False, lr_max=None, eval_rows=10000, loss="softmax",
+               norm="u", scale_every=1):
     """Time-to-P@1 on one GPU: cumulative CUDA-event time of the
     mega-batches (local steps + merge) until test P@1 first reaches
     floor + 0.9 (best - floor); floor = the majority-label P@1 of the test
@@ -522,7 +529,8 @@ def time_to_p1(cfg, prec, n_mb, dev, pert_renorm=False, lr_max=None, eval_rows=1
                       loss=loss)
     rep.register(api.DeviceCsr(data, device=dev))
     td = api.DeviceCsr(test, device=dev)
-    h = train.Hyper.from_config(cfg, pert_renorm=pert_renorm, **({"lr_max": lr_max} if lr_max else {}))
+    h = train.Hyper.from_config(cfg, pert_renorm=pert_renorm, norm=norm, scale_every=scale_every,
+                                **({"lr_max": lr_max} if lr_max else {}))
     sched = api.Scheduler(f"/asgd_ttp_{os.getpid()}", 1, h.M, create=True)
     drv = train.DistributedAdaptiveSGD(rep, h, 0, 1, sched)
     rows = np.arange(test.n_rows, dtype=np.int32)

@@ -176,11 +176,16 @@ int asgd_replica_sqnorm(asgd_ctx* ctx, double* out_dev);
 /* Alg. 2 lines 1-7, host, pure.  u, b: int64[n]; nu: fp64[n]
  * norms per parameter ||w_i||_2 / P.  Ties: key (u_i, b_i), lowest index,
  * perturbation skipped when key(r) == key(s) (Q17); no renormalisation unless
- * pert_renorm != 0 (Q18, Q34).  alpha_out: fp64[n]; r_out, s_out,
- * perturbed_out: nullable. */
+ * flags has ASGD_MERGE_RENORM (Q18, Q34).  With ASGD_MERGE_NORM_UB line 3
+ * becomes alpha_i = u_i b_i / sum_j u_j b_j ("normalize based on
+ * the product between the number of updates and the batch size", reading
+ * R12); line 2 is unchanged.  Other bits: ASGD_E_ARG.  alpha_out: fp64[n];
+ * r_out, s_out, perturbed_out: nullable. */
+#define ASGD_MERGE_RENORM 1   /* divide alpha by sum(alpha) after line 6    */
+#define ASGD_MERGE_NORM_UB 2  /* line 3 normalises u_i * b_i (R12)          */
 int asgd_merge_weights(int32_t n, const int64_t* u, const int64_t* b,
                        const double* nu, double pert_thr, double delta,
-                       int32_t pert_renorm, double* alpha_out, int32_t* r_out,
+                       int32_t flags, double* alpha_out, int32_t* r_out,
                        int32_t* s_out, int32_t* perturbed_out);
 
 /* params <- alpha * params (Alg. 2 line 8's alpha_i w_i, K-6).  Asynchronous.

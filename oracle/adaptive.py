@@ -58,10 +58,16 @@ def run(F: int, H: int, L: int, data, w0: np.ndarray, stream_rows_of: Callable[[
         n_rep: int, n_mb: int, M: int, b_max: int, b_min: int, beta: int, lr_max: float,
         gamma: float = 0.9, delta: float = 0.1, pert_thr: float = 0.1,
         pert_renorm: bool = False, cost_factors: Optional[Sequence[float]] = None,
-        route_logs: Optional[List[List[int]]] = None) -> List[MegaBatchRecord]:
+        route_logs: Optional[List[List[int]]] = None, norm: str = "u",
+        scale_every: int = 1) -> List[MegaBatchRecord]:
     """Run n_mb mega-batches.  stream_rows_of(mb) gives the M sample ids of
     mega-batch mb.  Routing is simulated with cost_factors, or replayed from
-    route_logs[mb] (ranks in ticket order)."""
+    route_logs[mb] (ranks in ticket order).  norm: Alg. 2 line 3 ("u") or the
+    u_i b_i variant ("ub", R12).  scale_every: Alg. 1 runs after mega-batches
+    mb with (mb + 1) % scale_every == 0 (R13; 1 = every mega-batch,
+    the paper's default)."""
+    if scale_every < 1:
+        raise ValueError(scale_every)
     w = np.asarray(w0, dtype=np.float64).copy()
     d = np.zeros_like(w)                                   # Q19: w_p = w_0
     b = [int(b_max)] * n_rep                               # P:1565-1566
@@ -82,11 +88,12 @@ def run(F: int, H: int, L: int, data, w0: np.ndarray, stream_rows_of: Callable[[
             losses.append(loss)
         u = _routing.updates(routes, n_rep)
         nu = [_merge.norm_per_param(x) for x in replicas]
-        alpha, r, s, pert = _merge.merge_weights(u, b, nu, pert_thr, delta, pert_renorm)
+        alpha, r, s, pert = _merge.merge_weights(u, b, nu, pert_thr, delta, pert_renorm, norm)
         w, d = _merge.merge_models(replicas, alpha, w, d, gamma)
         rec = MegaBatchRecord(routes, losses, u, list(b), list(lr), nu, alpha, pert, r, s,
                               w.copy(), d.copy())
-        b, lr = _scaling.scale_batches(u, b, b_min, b_max, beta, lr_max)
+        if (mb + 1) % scale_every == 0:                    # R13
+            b, lr = _scaling.scale_batches(u, b, b_min, b_max, beta, lr_max)
         out.append(rec)
     return out
 

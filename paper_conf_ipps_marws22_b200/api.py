@@ -229,13 +229,19 @@ class Replica:
 
 
 # ----------------------------------------------------------------- host-pure
-def merge_weights(u, b, nu, pert_thr=0.1, delta=0.1, pert_renorm=False):
+MERGE_RENORM, MERGE_NORM_UB = 1, 2       # asgd.h flags of asgd_merge_weights
+
+
+def merge_weights(u, b, nu, pert_thr=0.1, delta=0.1, pert_renorm=False, norm="u"):
+    if norm not in ("u", "ub"):
+        raise ValueError(f"norm must be 'u' or 'ub', got {norm!r}")
+    flags = (MERGE_RENORM if pert_renorm else 0) | (MERGE_NORM_UB if norm == "ub" else 0)
     n = len(u)
     u_, b_, nu_ = _np(u, np.int64), _np(b, np.int64), _np(nu, np.float64)
     alpha = np.zeros(n, dtype=np.float64)
     r, s, p = C.c_int32(), C.c_int32(), C.c_int32()
     call("asgd_merge_weights", n, _ptr(u_), _ptr(b_), _ptr(nu_), float(pert_thr), float(delta),
-         int(bool(pert_renorm)), _ptr(alpha), C.byref(r), C.byref(s), C.byref(p))
+         flags, _ptr(alpha), C.byref(r), C.byref(s), C.byref(p))
     return alpha.tolist(), r.value, s.value, bool(p.value)
 
 

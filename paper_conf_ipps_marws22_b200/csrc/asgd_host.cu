@@ -997,9 +997,10 @@ int asgd_copy_to_host(asgd_ctx* c, void* dst, const void* src, size_t bytes) {
 // =================================================================== host-pure
 
 int asgd_merge_weights(int32_t n, const int64_t* u, const int64_t* b, const double* nu,
-                       double pert_thr, double delta, int32_t pert_renorm, double* alpha,
+                       double pert_thr, double delta, int32_t flags, double* alpha,
                        int32_t* r_out, int32_t* s_out, int32_t* perturbed_out) {
   if (n < 1 || !u || !b || !nu || !alpha) return fail(ASGD_E_ARG, "bad argument");
+  if (flags & ~(ASGD_MERGE_RENORM | ASGD_MERGE_NORM_UB)) return fail(ASGD_E_ARG, "unknown merge flag");
   bool equal = true;                                   // Alg. 2 line 2
   for (int i = 1; i < n; ++i) equal = equal && (u[i] == u[0]);
   if (equal) {
@@ -1007,11 +1008,16 @@ int asgd_merge_weights(int32_t n, const int64_t* u, const int64_t* b, const doub
     for (int i = 0; i < n; ++i) sb += b[i];
     const double d = (double)sb;
     for (int i = 0; i < n; ++i) alpha[i] = (double)b[i] / d;
-  } else {                                             // line 3
+  } else if (!(flags & ASGD_MERGE_NORM_UB)) {          // line 3
     int64_t su = 0;
     for (int i = 0; i < n; ++i) su += u[i];
     const double d = (double)su;
     for (int i = 0; i < n; ++i) alpha[i] = (double)u[i] / d;
+  } else {                                             // R12: u_i b_i
+    int64_t sub = 0;
+    for (int i = 0; i < n; ++i) sub += u[i] * b[i];
+    const double d = (double)sub;
+    for (int i = 0; i < n; ++i) alpha[i] = (double)(u[i] * b[i]) / d;
   }
   bool gate = true;                                    // line 4 (Q16: strict <)
   for (int i = 0; i < n; ++i) gate = gate && (nu[i] < pert_thr);
@@ -1027,7 +1033,7 @@ int asgd_merge_weights(int32_t n, const int64_t* u, const int64_t* b, const doub
       pert = 1;
     }
   }
-  if (pert_renorm) {                                   // Q34 option
+  if (flags & ASGD_MERGE_RENORM) {                     // Q34 option
     double tot = 0.0;
     for (int i = 0; i < n; ++i) tot += alpha[i];
     for (int i = 0; i < n; ++i) alpha[i] = alpha[i] / tot;

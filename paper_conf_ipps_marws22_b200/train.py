@@ -37,6 +37,14 @@ class Hyper:
     delta: float = 0.1
     pert_thr: float = 0.1
     pert_renorm: bool = False   # Q34 option (literal Alg. 2 by default)
+    norm: str = "u"             # Alg. 2 line 3: "u", or "ub" = u_i b_i (R12)
+    scale_every: int = 1        # Alg. 1 after every scale_every-th mega-batch (R13)
+
+    def __post_init__(self):
+        if self.norm not in ("u", "ub"):
+            raise ValueError(f"norm must be 'u' or 'ub', got {self.norm!r}")
+        if self.scale_every < 1:
+            raise ValueError(f"scale_every must be >= 1, got {self.scale_every}")
 
     @classmethod
     def from_config(cls, cfg, **kw):
@@ -166,11 +174,12 @@ class DistributedAdaptiveSGD:
         routes = self.sched.log() if keep_log and r == 0 else []
         if r == 0:
             self.sched.reset(self.mb + 1)        # every rank is past its tickets
-        alpha, rr, ss, pert = api.merge_weights(us, bs, nu, h.pert_thr, h.delta, h.pert_renorm)
+        alpha, rr, ss, pert = api.merge_weights(us, bs, nu, h.pert_thr, h.delta, h.pert_renorm, h.norm)
         self._merge(alpha)
         # ---- Alg. 1 ----------------------------------------------------------
         lr_used = list(self.lr)
-        self.b, self.lr = api.scale_batches(us, bs, h.b_min, h.b_max, h.beta, h.lr_max)
+        if (self.mb + 1) % h.scale_every == 0:    # R13
+            self.b, self.lr = api.scale_batches(us, bs, h.b_min, h.b_max, h.beta, h.lr_max)
         st = MegaBatchStats(self.mb, us, bs, lr_used, nu, alpha, rr, ss, pert, routes, n_steps)
         self.mb += 1
         return st
@@ -237,7 +246,7 @@ class SimulatedAdaptiveSGD:
             rep.sqnorm(self.sq[i:i + 1])
         P = self.reps[0].P
         nu = [math.sqrt(float(x)) / P for x in self.sq.cpu().numpy()]
-        alpha, rr, ss, pert = api.merge_weights(u, self.b, nu, h.pert_thr, h.delta, h.pert_renorm)
+        alpha, rr, ss, pert = api.merge_weights(u, self.b, nu, h.pert_thr, h.delta, h.pert_renorm, h.norm)
         r0 = self.reps[0]
         r0.weighted_sum(self.reps, alpha, r0.params)
         r0.finish(h.gamma)
@@ -245,7 +254,8 @@ class SimulatedAdaptiveSGD:
             rep.params.copy_(r0.params)
             rep.params_changed()
         lr_used, b_used = list(self.lr), list(self.b)
-        self.b, self.lr = api.scale_batches(u, self.b, h.b_min, h.b_max, h.beta, h.lr_max)
+        if (self.mb + 1) % h.scale_every == 0:    # R13
+            self.b, self.lr = api.scale_batches(u, self.b, h.b_min, h.b_max, h.beta, h.lr_max)
         st = MegaBatchStats(self.mb, u, b_used, lr_used, nu, alpha, rr, ss, pert, routes, len(routes))
         self.mb += 1
         return st

@@ -75,8 +75,9 @@ def test_merge_weights_random_bitexact():
         b = [rng.choice([32, 64, 100, 128]) for _ in range(n)]
         nu = [rng.choice([0.01, 0.05, 0.2]) for _ in range(n)]
         renorm = rng.random() < 0.3
-        got = api.merge_weights(u, b, nu, 0.1, 0.1, renorm)
-        want = merge.merge_weights(u, b, nu, 0.1, 0.1, renorm)
+        norm = rng.choice(["u", "ub"])
+        got = api.merge_weights(u, b, nu, 0.1, 0.1, renorm, norm)
+        want = merge.merge_weights(u, b, nu, 0.1, 0.1, renorm, norm)
         assert got[0] == want[0] and got[3] == want[3], (u, b, nu)
         if want[3]:
             assert got[1:3] == want[1:3]
@@ -153,3 +154,16 @@ def test_scheduler_single_process():
         assert s.next(0, 1) is None
     finally:
         s.close()
+
+
+def test_merge_weights_unknown_flag_rejected():
+    import ctypes as C
+    import numpy as np
+    from paper_conf_ipps_marws22_b200 import _lib
+    u = np.array([1, 2], dtype=np.int64)
+    b = np.array([32, 32], dtype=np.int64)
+    nu = np.array([1.0, 1.0])
+    a = np.zeros(2)
+    rc = _lib.lib().asgd_merge_weights(2, u.ctypes.data, b.ctypes.data, nu.ctypes.data, 0.1, 0.1, 4,
+                                       a.ctypes.data, None, None, None)
+    assert rc == 1      # ASGD_E_ARG

@@ -36,14 +36,16 @@ def test_sqnorm_prescale_finish():
     assert rep.updates() == 0
 
 
-@pytest.mark.parametrize("precision,tol", [("fp32", 1e-4), ("bf16", 2e-2)])
-def test_simulated_two_replicas_tiny_trajectory(precision, tol):
+@pytest.mark.parametrize("precision,tol,norm,scale_every", [
+    ("fp32", 1e-4, "u", 1), ("bf16", 2e-2, "u", 1),
+    ("fp32", 1e-4, "ub", 2)])        # R12 u_i b_i weights, R13 Alg. 1 every 2nd mega-batch
+def test_simulated_two_replicas_tiny_trajectory(precision, tol, norm, scale_every):
     """BASELINE.json configs[0]: 2 simulated replicas, ~50 steps, free-running."""
     from paper_conf_ipps_marws22_b200 import api, train
     cfg = config("tiny")
     data = dataset("tiny")
     w0 = init_params(cfg)
-    h = train.Hyper.from_config(cfg)
+    h = train.Hyper.from_config(cfg, norm=norm, scale_every=scale_every)
     r0 = make_replica(cfg, data, precision, w0=w0)
     r1 = api.Replica(cfg.F, cfg.L, cfg.H, cfg.b_max, r0.desc.max_step_nnz, r0.desc.max_step_labels,
                      precision, w0=w0, share_global=r0)
@@ -58,7 +60,7 @@ def test_simulated_two_replicas_tiny_trajectory(precision, tol):
         stats.append(sim.megabatch(torch.as_tensor(ids, device="cuda"), ids))
     recs = adaptive.run(cfg.F, cfg.H, cfg.L, data, w0, lambda mb: sample_stream(cfg, mb * h.M, h.M),
                         n_rep=2, n_mb=n_mb, M=h.M, b_max=h.b_max, b_min=h.b_min, beta=h.beta,
-                        lr_max=h.lr_max, cost_factors=cf)
+                        lr_max=h.lr_max, cost_factors=cf, norm=norm, scale_every=scale_every)
     for st, rec in zip(stats, recs):
         assert [tuple(x) for x in st.routes] == [tuple(x) for x in rec.routes]   # bit-exact
         assert st.u == rec.u and st.b == rec.b and st.lr == rec.lr

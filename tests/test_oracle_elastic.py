@@ -4,6 +4,7 @@ Elastic and Adaptive coincide on one GPU) -- not gpu."""
 import random
 
 import numpy as np
+import pytest
 
 from oracle import adaptive, merge, model, routing
 from synth import config, generate, init_params, sample_stream
@@ -64,3 +65,35 @@ def test_elastic_two_replicas_is_the_average_of_two_sgd_runs():
     want = 0.5 * (reps[0] + reps[1])              # d = 0 at the first merge (Q19)
     np.testing.assert_allclose(rec.w, want, rtol=0, atol=1e-12)
     assert rec.u == [4, 4] and rec.alpha == [0.5, 0.5]
+
+
+def test_adaptive_scale_every_and_ub_norm():
+    """R13: with scale_every = k, Alg. 1 runs only after mega-batches
+    k-1, 2k-1, ...; b is frozen at b_max in between, and those mega-batches
+    route exactly like the first one under the same costs.  R12: with the
+    b-normalised line 2 untouched, the first mega-batch (all b_i = b_max) gives
+    identical alphas in both norms."""
+    cfg, data = _tiny()
+    M = cfg.mega_batch
+    stream = lambda mb: sample_stream(cfg, mb * M, M)
+    kw = dict(n_rep=2, n_mb=3, M=M, b_max=cfg.b_max, b_min=cfg.b_min, beta=cfg.beta,
+              lr_max=cfg.lr_max, cost_factors=[1.0, 1.6])
+    every = adaptive.run(cfg.F, cfg.H, cfg.L, data, init_params(cfg), stream, **kw)
+    frozen = adaptive.run(cfg.F, cfg.H, cfg.L, data, init_params(cfg), stream, scale_every=4, **kw)
+    assert every[1].b != [cfg.b_max] * 2          # the 1.6x slower rank was rescaled
+    for rec in frozen:
+        assert rec.b == [cfg.b_max] * 2 and rec.lr == [cfg.lr_max] * 2
+    np.testing.assert_array_equal(every[0].w, frozen[0].w)
+    ub = adaptive.run(cfg.F, cfg.H, cfg.L, data, init_params(cfg), stream, norm="ub", **kw)
+    assert ub[0].alpha == every[0].alpha
+    assert ub[1].b == every[1].b                  # Alg. 1 does not read alpha
+    u, b = ub[1].u, ub[1].b
+    assert u[0] != u[1]
+    tot = u[0] * b[0] + u[1] * b[1]
+    want = [u[0] * b[0] / tot, u[1] * b[1] / tot]
+    if ub[1].perturbed:                           # Alg. 2 lines 5-6, delta = 0.1
+        want[ub[1].r] *= 1.1
+        want[ub[1].s] *= 0.9
+    assert ub[1].alpha == want
+    with pytest.raises(ValueError):
+        adaptive.run(cfg.F, cfg.H, cfg.L, data, init_params(cfg), stream, scale_every=0, **kw)

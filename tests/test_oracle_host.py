@@ -186,3 +186,32 @@ def test_precision_at_k_bruteforce():
     Zh = np.array([[1.0, 3.0, 3.0, 0.0]])
     assert metrics.topk(Zh, 2).tolist() == [[1, 2]]
     assert metrics.precision_at_k(metrics.topk(Zh, 1), np.array([0, 1]), np.array([2]), 1) == 0.0
+
+
+def test_alg2_ub_variant_pins():
+    """R12: alpha_i = u_i b_i / sum_j u_j b_j in place of line 3."""
+    # hand-worked: u = (3, 1), b = (100, 300): u b = (300, 300) -> (1/2, 1/2),
+    # where line 3 alone gives (3/4, 1/4)
+    a, *_ = merge.merge_weights([3, 1], [100, 300], [1.0, 1.0], norm="ub")
+    assert a == [0.5, 0.5]
+    a, *_ = merge.merge_weights([3, 1], [100, 300], [1.0, 1.0])
+    assert a == [0.75, 0.25]
+    # u = (2, 1, 1), b = (64, 64, 128): u b = (128, 64, 128) -> (0.4, 0.2, 0.4)
+    a, *_ = merge.merge_weights([2, 1, 1], [64, 64, 128], [1.0] * 3, norm="ub")
+    assert a == [0.4, 0.2, 0.4]
+    rng = random.Random(7)
+    for _ in range(1000):
+        N = rng.randint(1, 8)
+        u = [rng.randint(1, 30) for _ in range(N)]
+        b = [rng.randint(1, 1024) for _ in range(N)]
+        a, *_ = merge.merge_weights(u, b, [1.0] * N, norm="ub")
+        assert abs(sum(a) - 1.0) < 1e-14
+        # equal batch sizes: the product is proportional to u -> line 3's weights
+        a_eq, *_ = merge.merge_weights(u, [64] * N, [1.0] * N, norm="ub")
+        a_u, *_ = merge.merge_weights(u, [64] * N, [1.0] * N)
+        assert all(abs(x - y) < 1e-15 for x, y in zip(a_eq, a_u))
+        # all u equal: line 2 still applies (b-normalised)
+        a_b, *_ = merge.merge_weights([5] * N, b, [1.0] * N, norm="ub")
+        assert all(abs(x - bi / sum(b)) < 1e-15 for x, bi in zip(a_b, b))
+    with pytest.raises(ValueError):
+        merge.merge_weights([1], [1], [1.0], norm="bu")
