@@ -53,7 +53,8 @@ def _worker(rank, world, port, shm, M, out_dir):
         log = sched.log() if rank == 0 else None
         if rank == 0:
             sched.reset(mb + 1)
-        alpha, r, s, p = api.merge_weights(us, bs, nu, 0.1, 0.1)
+        norm = "ub" if mb == 2 else "u"          # R12 on the last mega-batch
+        alpha, r, s, p = api.merge_weights(us, bs, nu, 0.1, 0.1, False, norm)
         # prescale + all-reduce SUM == sum_i alpha_i w_i
         t = torch.from_numpy(replica.astype(np.float64) * alpha[rank])
         dist.all_reduce(t)
@@ -62,7 +63,7 @@ def _worker(rank, world, port, shm, M, out_dir):
         S_ref, _ = omerge.merge_models([x.numpy() for x in allrep], alpha, w_global, np.zeros_like(w_global), 0.0)
         allsteps = [None] * world
         dist.all_gather_object(allsteps, got)
-        results[mb] = dict(us=us, bs=bs, nu=nu, alpha=alpha, pert=p, log=log, steps=allsteps,
+        results[mb] = dict(us=us, bs=bs, nu=nu, alpha=alpha, pert=p, norm=norm, log=log, steps=allsteps,
                            merge_err=float(np.abs(t.numpy() - S_ref).max()))
     np.save(os.path.join(out_dir, f"r{rank}.npy"), np.array([results], dtype=object), allow_pickle=True)
     dist.barrier()
@@ -95,6 +96,6 @@ def test_two_ranks_gloo(tmp_path):
         assert [(r, s, n) for _, r, s, n in log] == orouting.replay(order, a["bs"], M)
         # Alg. 2 on the exchanged statistics equals the oracle
         assert a["nu"] == b["nu"]
-        ow = omerge.merge_weights(a["us"], a["bs"], a["nu"], 0.1, 0.1)
+        ow = omerge.merge_weights(a["us"], a["bs"], a["nu"], 0.1, 0.1, False, a["norm"])
         assert a["alpha"] == ow[0] and a["pert"] == ow[3]
         assert a["merge_err"] < 1e-12
