@@ -1,5 +1,5 @@
 """Cross-check of one heterogeneity point of profiles/r01_telemetry.md on the CPU
-oracle (test infrastructure; run by hand): EURLex-4K-shaped, 4 replicas, cost
+oracle (test infrastructure, kept under tests/ with the other oracle users; run by hand): EURLex-4K-shaped, 4 replicas, cost
 factors 1..1+h, n_mb mega-batches, paper defaults (or --norm ub --scale-every 2).
 Prints per-mega-batch b_i of the routed replicas and the final P@1 of the fp64
 model, to compare with the CUDA path's trajectory (same routing, bf16 vs fp64)."""
