@@ -167,3 +167,15 @@ def test_merge_weights_unknown_flag_rejected():
     rc = _lib.lib().asgd_merge_weights(2, u.ctypes.data, b.ctypes.data, nu.ctypes.data, 0.1, 0.1, 4,
                                        a.ctypes.data, None, None, None)
     assert rc == 1      # ASGD_E_ARG
+
+
+def test_hyper_rejects_unknown_method_switches():
+    from paper_conf_ipps_marws22_b200 import train
+    base = dict(b_max=256, b_min=32, beta=4, lr_max=1.0, M=25600)
+    assert train.Hyper(**base, norm="ub", scale_every=3).scale_every == 3
+    with pytest.raises(ValueError):
+        train.Hyper(**base, norm="b")
+    with pytest.raises(ValueError):
+        train.Hyper(**base, scale_every=0)
+    with pytest.raises(ValueError):
+        api.merge_weights([1, 2], [32, 32], [1.0, 1.0], norm="uu")
