@@ -298,16 +298,10 @@ def main():
         dist.barrier()
     if rank != 0:
         sched = api.Scheduler(shm, world, M, create=False)
-    merge_used = a.merge
-    try:
-        drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=a.inflight, merge=a.merge,
-                                           method=a.method)
-    except Exception as e:   # e.g. no CUDA IPC between the ranks' GPUs: NCCL all-reduce merge instead
-        if a.merge != "fused":
-            raise
-        merge_used = f"nccl (fused unavailable: {type(e).__name__}: {str(e)[:120]})"
-        drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=a.inflight, merge="nccl",
-                                           method=a.method)
+    # the fused merge falls back to NCCL on EVERY rank when any rank cannot map its peers
+    drv = train.DistributedAdaptiveSGD(rep, h, rank, world, sched, inflight=a.inflight, merge=a.merge,
+                                       method=a.method)
+    merge_used = drv.merge if not drv.merge_note else f"{drv.merge} (fused unavailable: {drv.merge_note})"
     K, W = a.steps, a.warmup
     Ke = a.e2e_steps if a.e2e_steps is not None else min(K, 10)
     ids = [sample_stream(cfg, mb * M, M) for mb in range(W + K + Ke)]

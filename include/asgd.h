@@ -188,6 +188,16 @@ int asgd_merge_weights(int32_t n, const int64_t* u, const int64_t* b,
                        int32_t flags, double* alpha_out, int32_t* r_out,
                        int32_t* s_out, int32_t* perturbed_out);
 
+/* Alg. 2 line 4's norm per parameter (reading Q16):
+ * nu_i = sqrt(sqnorm_i) / P, fp64, from the squared norms asgd_replica_sqnorm
+ * produced (all-gathered across ranks).  Host, pure.  sqnorm: fp64[n];
+ * nu_out: fp64[n].  ASGD_E_ARG if n < 1, P < 1 or a sqnorm is negative/NaN. */
+int asgd_norm_per_param(int32_t n, const double* sqnorm, int64_t P, double* nu_out);
+
+/* Elastic SGD's merge weights (elastic model averaging; reading
+ * R10): alpha_i = 1/N for the N = n replicas.  Host, pure.  alpha_out: fp64[n]. */
+int asgd_elastic_weights(int32_t n, double* alpha_out);
+
 /* params <- alpha * params (Alg. 2 line 8's alpha_i w_i, K-6).  Asynchronous.
  * After it the caller sums the prescaled replicas (one NCCL all-reduce SUM
  * over NVLink, or asgd_replicas_weighted_sum on one device). */
@@ -224,6 +234,11 @@ int asgd_replicas_weighted_sum(asgd_ctx* ctx, const float* const* replicas_dev,
 #define ASGD_PEER_HANDLE_BYTES 160
 int asgd_peer_export(asgd_ctx* ctx, void* out_host);
 int asgd_peer_open(asgd_ctx* ctx, int32_t rank, int32_t world, const void* handles_host);
+/* Close the peer mappings asgd_peer_open made (synchronises the ctx stream);
+ * asgd_merge_fused then fails with ASGD_E_STATE until the next asgd_peer_open.
+ * A rank that opened its peers but must fall back to the NCCL merge because
+ * another rank could not calls this. */
+int asgd_peer_close(asgd_ctx* ctx);
 int asgd_merge_fused(asgd_ctx* ctx, const double* alpha_host, float gamma);
 
 /* ---------------------------------------------------------------- scaling */
@@ -288,9 +303,11 @@ int asgd_run_static(asgd_ctx* ctx, int32_t rank, int32_t world, int64_t b,
                     int64_t* n_steps);
 
 /* Replay (parity): ranks in ticket order -> routes (rank, start, len) with the
- * batch sizes b[rank], stopping at M.  out: int64[3*cap]. */
-int asgd_route_replay(int32_t n_tickets, const int32_t* order, const int64_t* b,
-                      int64_t M, int64_t* out, int64_t cap, int64_t* n_out);
+ * batch sizes b[rank] (host int64[n_ranks]), stopping at M.  out: int64[3*cap].
+ * ASGD_E_ARG if an order entry is outside [0, n_ranks). */
+int asgd_route_replay(int32_t n_ranks, int32_t n_tickets, const int32_t* order,
+                      const int64_t* b, int64_t M, int64_t* out, int64_t cap,
+                      int64_t* n_out);
 /* Simulated clock (Q10): every rank free at t = 0; the rank free first (ties:
  * lowest id) takes the next batch; it stays busy
  * cost_factor[r] * (nnz(batch) + per_row * len).  row_nnz: int64[M] nnz of the

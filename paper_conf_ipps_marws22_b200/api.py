@@ -185,6 +185,9 @@ class Replica:
         buf = (C.c_char * len(blob)).from_buffer_copy(blob)
         call("asgd_peer_open", self.ctx, int(rank), len(handles), buf)
 
+    def peer_close(self):
+        call("asgd_peer_close", self.ctx)
+
     def merge_fused(self, alpha: Sequence[float], gamma: float):
         al = (C.c_double * len(alpha))(*[float(a) for a in alpha])
         call("asgd_merge_fused", self.ctx, al, float(gamma))
@@ -253,12 +256,28 @@ def scale_batches(u, b, b_min, b_max, beta, lr_max):
     return b_.tolist(), lr.tolist()
 
 
+def norm_per_param(sqnorm, P: int) -> List[float]:
+    """Alg. 2 line 4's ||w_i||_2 / |w| from the all-gathered squared norms (Q16)."""
+    sq = _np(sqnorm, np.float64)
+    nu = np.zeros(len(sq), dtype=np.float64)
+    call("asgd_norm_per_param", len(sq), _ptr(sq), int(P), _ptr(nu))
+    return nu.tolist()
+
+
+def elastic_weights(n: int) -> List[float]:
+    """Elastic SGD's alpha_i = 1/N (R10)."""
+    al = np.zeros(int(n), dtype=np.float64)
+    call("asgd_elastic_weights", int(n), _ptr(al))
+    return al.tolist()
+
+
 def route_replay(order, b, M) -> List[Tuple[int, int, int]]:
     o = _np(order, np.int32)
     b_ = _np(b, np.int64)
     out = np.zeros(3 * (len(o) + 1), dtype=np.int64)
     n = C.c_int64()
-    call("asgd_route_replay", len(o), _ptr(o) if len(o) else None, _ptr(b_), int(M), _ptr(out), len(o) + 1, C.byref(n))
+    call("asgd_route_replay", len(b_), len(o), _ptr(o) if len(o) else None, _ptr(b_), int(M), _ptr(out),
+         len(o) + 1, C.byref(n))
     return [tuple(int(x) for x in out[3 * i:3 * i + 3]) for i in range(n.value)]
 
 

@@ -17,6 +17,8 @@
 #include <cstdlib>
 #include <cstring>
 #include <list>
+#include <map>
+#include <mutex>
 #include <new>
 #include <string>
 #include <vector>
@@ -878,6 +880,18 @@ int asgd_peer_open(asgd_ctx* c, int32_t rank, int32_t world, const void* handles
   return ASGD_OK;
 }
 
+int asgd_peer_close(asgd_ctx* c) {
+  if (!c) return fail(ASGD_E_ARG, "null ctx");
+  CU(cudaSetDevice(c->device));
+  CU(cudaStreamSynchronize(c->s));
+  for (void* pm : c->peer_mapped) cudaIpcCloseMemHandle(pm);
+  c->peer_mapped.clear();
+  for (int j = 0; j < kMaxPeers; ++j) { c->peer_params[j] = nullptr; c->peer_sync[j] = nullptr; }
+  c->peer_rank = -1;
+  c->peer_world = 0;
+  return ASGD_OK;
+}
+
 int asgd_merge_fused(asgd_ctx* c, const double* alpha, float gamma) {
   if (!c || !alpha) return fail(ASGD_E_ARG, "null argument");
   if (c->peer_world < 1) return fail(ASGD_E_STATE, "asgd_peer_open first");
@@ -1044,6 +1058,21 @@ int asgd_merge_weights(int32_t n, const int64_t* u, const int64_t* b, const doub
   return ASGD_OK;
 }
 
+int asgd_norm_per_param(int32_t n, const double* sqnorm, int64_t P, double* nu) {
+  if (n < 1 || !sqnorm || !nu || P < 1) return fail(ASGD_E_ARG, "bad argument");
+  for (int i = 0; i < n; ++i) {
+    if (!(sqnorm[i] >= 0.0)) return fail(ASGD_E_ARG, "sqnorm[%d] = %g is negative or NaN", i, sqnorm[i]);
+    nu[i] = std::sqrt(sqnorm[i]) / (double)P;        // Q16: ||w_i||_2 / |w|
+  }
+  return ASGD_OK;
+}
+
+int asgd_elastic_weights(int32_t n, double* alpha) {
+  if (n < 1 || !alpha) return fail(ASGD_E_ARG, "bad argument");
+  for (int i = 0; i < n; ++i) alpha[i] = 1.0 / (double)n;   // R10: alpha_i = 1/N
+  return ASGD_OK;
+}
+
 int asgd_scale_batches(int32_t n, const int64_t* u, int64_t* b, double* lr_out, int64_t b_min,
                        int64_t b_max, int64_t beta, double lr_max) {
   if (n < 1 || !u || !b || b_min < 1 || b_max < b_min) return fail(ASGD_E_ARG, "bad argument");
@@ -1060,12 +1089,13 @@ int asgd_scale_batches(int32_t n, const int64_t* u, int64_t* b, double* lr_out, 
   return ASGD_OK;
 }
 
-int asgd_route_replay(int32_t nt, const int32_t* order, const int64_t* b, int64_t M, int64_t* out,
-                      int64_t cap, int64_t* n_out) {
-  if (nt < 0 || (nt && !order) || !b || !out || !n_out) return fail(ASGD_E_ARG, "bad argument");
+int asgd_route_replay(int32_t n_ranks, int32_t nt, const int32_t* order, const int64_t* b, int64_t M,
+                      int64_t* out, int64_t cap, int64_t* n_out) {
+  if (n_ranks < 1 || nt < 0 || (nt && !order) || !b || !out || !n_out) return fail(ASGD_E_ARG, "bad argument");
   int64_t c = 0, k = 0;
   for (int32_t t = 0; t < nt && c < M; ++t) {
     const int32_t r = order[t];
+    if (r < 0 || r >= n_ranks) return fail(ASGD_E_ARG, "order[%d] = %d not in [0, %d)", t, r, n_ranks);
     const int64_t len = std::min<int64_t>(b[r], M - c);
     if (k >= cap) return fail(ASGD_E_SHAPE, "route cap %lld too small", (long long)cap);
     out[3 * k] = r; out[3 * k + 1] = c; out[3 * k + 2] = len;
@@ -1160,8 +1190,10 @@ int asgd_sched_next(asgd_sched* s, int32_t rank, int64_t b, int64_t* start, int6
   const int64_t ticket = (int64_t)(v >> 40), c = (int64_t)(v & kCurMask);
   if (c >= h->M) return 0;
   const int64_t l = std::min<int64_t>(b, h->M - c);
-  if (ticket < h->cap) {
-    h->log[ticket][0] = ticket; h->log[ticket][1] = rank; h->log[ticket][2] = c; h->log[ticket][3] = l;
+  if (ticket < h->cap) {   // entry [0] = mega-batch generation << 40 | ticket, stored last (release)
+    const int64_t gen = __atomic_load_n(&h->mb, __ATOMIC_ACQUIRE);
+    h->log[ticket][1] = rank; h->log[ticket][2] = c; h->log[ticket][3] = l;
+    __atomic_store_n(&h->log[ticket][0], (gen << 40) | ticket, __ATOMIC_RELEASE);
   }
   *start = c;
   *len = l;
@@ -1225,11 +1257,16 @@ int asgd_sched_log(asgd_sched* s, int64_t* out, int64_t cap, int64_t* n_out) {
   if (!s || !out || !n_out) return fail(ASGD_E_ARG, "null argument");
   ShmSched* h = s->h;
   const int64_t T = (int64_t)(h->packed.load(std::memory_order_acquire) >> 40);
+  const int64_t gen = __atomic_load_n(&h->mb, __ATOMIC_ACQUIRE);
   int64_t c = 0, k = 0;
   while (k < T && k < h->cap && c < h->M) {
-    if (h->log[k][2] != c) return fail(ASGD_E_STATE, "log entry %lld not yet written", (long long)k);
+    // an entry of an earlier mega-batch (same ticket slot) carries an older generation
+    const int64_t tag = __atomic_load_n(&h->log[k][0], __ATOMIC_ACQUIRE);
+    if (tag != ((gen << 40) | k) || h->log[k][2] != c)
+      return fail(ASGD_E_STATE, "log entry %lld of mega-batch %lld not yet written", (long long)k, (long long)gen);
     if (k >= cap) return fail(ASGD_E_SHAPE, "cap too small");
-    for (int j = 0; j < 4; ++j) out[4 * k + j] = h->log[k][j];
+    out[4 * k] = k;
+    for (int j = 1; j < 4; ++j) out[4 * k + j] = h->log[k][j];
     c += h->log[k][3];
     ++k;
   }
@@ -1265,6 +1302,20 @@ int asgd_sched_close(asgd_sched* s, int32_t unlink_shm) {
 }  // extern "C"
 
 namespace asgd {
+cudaError_t smem_attr_raw(const void* kernel, size_t bytes) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, size_t> done;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> g(mu);
+  size_t& have = done[{kernel, dev}];
+  if (have >= bytes) return cudaSuccess;
+  e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  if (e == cudaSuccess) have = bytes;
+  return e;
+}
+
 // Programmatic dependent launch: each kernel's prologue overlaps its predecessor's tail.
 // Measured (samples/s, PDL off -> on): bf16 EURLex 4.01 -> 4.22 M, AmazonCat 5.35 -> 5.46 M,
 // Wiki10 1.356 -> 1.383 M, Amazon-670K / Delicious-200K even; fp32 EURLex 1.52 -> 1.34 M.

@@ -81,6 +81,14 @@ __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;"
 int pdl_mode();
 bool pdl_for(bool bf16);   // launch_k: this ctx's kernels use PDL
 
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) is a per-device setting: it is
+// applied once per (kernel, current device) and raised when a larger size is needed.
+cudaError_t smem_attr_raw(const void* kernel, size_t bytes);   // thread-safe
+template <typename... KArgs>
+cudaError_t ensure_smem(void (*kernel)(KArgs...), size_t bytes) {
+  return smem_attr_raw(reinterpret_cast<const void*>(kernel), bytes);
+}
+
 template <typename... KArgs, typename... Args>
 cudaError_t launch_k(const Launch& lc, void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
                      Args&&... args) {

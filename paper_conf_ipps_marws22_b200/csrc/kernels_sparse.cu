@@ -936,13 +936,9 @@ template <int VPL>
 cudaError_t spmm_fwd_t(const Launch& lc, const StepArgs& sa, const asgd_csr& x, const float* W1, const float* b1,
                        const Ptrs& P, const WsLayout& L, bool want_bf16) {
   const size_t smem = view_smem(sa.n);
-  static bool attr = false;
-  if (!attr) {   // the batch view (dynamic) + the group partials (static) exceed 48 KB at b_max = 2048
-    cudaError_t e = cudaFuncSetAttribute(k_spmm_fwd<VPL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)view_smem(2048));
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
+  // the batch view (dynamic) + the group partials (static) exceed 48 KB at b_max = 2048
+  cudaError_t e = ensure_smem(k_spmm_fwd<VPL>, view_smem(2048));
+  if (e != cudaSuccess) return e;
   static int occ = 0;
   const int grid = wave_grid(lc, k_spmm_fwd<VPL>, view_smem(2048), L.n_pieces, occ, k1_group<VPL>());
   const ViewOut vo{P.boff, P.loff, P.rbase, P.rowsc, P.meta};
@@ -974,11 +970,9 @@ cudaError_t launch_touched(const Launch& lc, const StepArgs& sa, const asgd_csr&
   static const int max_ctas = [] { const char* e = getenv("ASGD_K0_CTAS"); return e ? atoi(e) : 0; }();
   int64_t cap = max_ctas > 0 ? max_ctas : kTouchCtas;
   const int ctas = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)lc.sms, cap, (L.nz_cap + 1023) / 1024}));
-  static size_t attr = 48 * 1024;
-  if (smem_all > attr) {
-    cudaError_t e = cudaFuncSetAttribute(k_touched, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_all);
+  if (smem_all > 48 * 1024) {
+    cudaError_t e = ensure_smem(k_touched, smem_all);
     if (e != cudaSuccess) return e;
-    attr = smem_all;
   }
   return launch_k(lc, k_touched, dim3(ctas), dim3(512), smem_all, sa, x.row_ptr, x.n_rows, L.nz_cap, x.col, x.val,
                   P.meta, P.cnt, P.tsum, F, nt, P.fseg, P.fuid, P.uniq, P.useg, P.bits, W, P.e_n,
@@ -1018,13 +1012,8 @@ cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float*
   constexpr int CS = 32 * CPL;
   const int nsl = H / CS;
   const size_t smem = (size_t)b_max * CS * sizeof(T);
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(k_scatter_sgd_s<T, CPL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         200 * 1024);
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
+  cudaError_t e = ensure_smem(k_scatter_sgd_s<T, CPL>, 200 * 1024);
+  if (e != cudaSuccess) return e;
   const int gx = std::max(1, lc.sms / nsl);
   return launch_k(lc, k_scatter_sgd_s<T, CPL>, dim3(gx, nsl), dim3(scatter_threads<T, CPL>()), smem, P.e_n, P.e_v, P.e_u,
                   P.e_f, P.useg, P.meta, dA1, H, W1, P.part5, P.ucnt, grad_w1, P.cnt, P.bits,

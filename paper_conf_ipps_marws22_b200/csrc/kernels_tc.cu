@@ -843,12 +843,9 @@ cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, co
                       (size_t)stages_of<EPI>() * ((ARES ? 0 : BM * BK * 2) + BN * BK * 2) +
                       (EPI == TC_EPI_SGD ? 2048 : 0) + staging_bytes<BN, EPI, A_MN>() + bias_bytes<BN, EPI>() + 1024 + 512;
   if (ARES && g.K > kAresK) return cudaErrorNotSupported;   // resident A block holds K <= 256
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(k_gemm_tc<BN, A_MN, B_MN, EPI>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  {
+    cudaError_t e = ensure_smem(k_gemm_tc<BN, A_MN, B_MN, EPI>, smem);
     if (e != cudaSuccess) return e;
-    attr = true;
   }
   g.splits = splits;
   const int64_t tiles = (int64_t)((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN) * splits;

@@ -108,7 +108,7 @@ def exchange_stats(u: int, b: int, sqnorm: torch.Tensor, P: int, world: int,
         allv = mine.reshape(1, 3).cpu().numpy()
     us = [int(round(x)) for x in allv[:, 0]]
     bs = [int(round(x)) for x in allv[:, 1]]
-    nu = [math.sqrt(float(x)) / P for x in allv[:, 2]]
+    nu = api.norm_per_param(allv[:, 2], P)
     return us, bs, nu
 
 
@@ -133,14 +133,9 @@ class DistributedAdaptiveSGD:
         if merge not in ("nccl", "fused"):
             raise ValueError(f"merge={merge!r}")
         self.merge = merge
+        self.merge_note = ""
         if merge == "fused":
-            handles = [None] * world
-            mine = replica.peer_export()
-            if world > 1:
-                dist.all_gather_object(handles, mine, group=group)
-            else:
-                handles = [mine]
-            replica.peer_open(rank, handles)
+            self.merge, self.merge_note = self._open_peers(replica, rank, world, group)
         self.sched, self.group, self.inflight = sched, group, inflight
         self.b = [hyper.b_max] * world            # initial b = b_max
         self.lr = [hyper.lr_max] * world
@@ -184,6 +179,47 @@ class DistributedAdaptiveSGD:
         self.mb += 1
         return st
 
+    @staticmethod
+    def _open_peers(replica: api.Replica, rank: int, world: int, group):
+        """Map every rank's replica for the fused merge, or agree on the NCCL merge.
+
+        Each rank tries export / all-gather / open locally, then the ranks take the
+        MIN of a success flag, so either every rank runs asgd_merge_fused or every
+        rank runs prescale + all_reduce + finish: a rank on the other path would
+        spin in k_merge_wait or block in the all-reduce forever.  A rank whose
+        peers opened but that falls back closes its mappings."""
+        ok, why = 1, ""
+        mine = b""
+        try:
+            mine = replica.peer_export()
+        except Exception as e:          # e.g. IPC unsupported on this device
+            ok, why = 0, f"peer_export: {type(e).__name__}: {str(e)[:100]}"
+        if world > 1:
+            handles = [None] * world
+            dist.all_gather_object(handles, mine, group=group)
+        else:
+            handles = [mine]
+        if ok and all(handles):
+            try:
+                replica.peer_open(rank, handles)
+            except Exception as e:      # e.g. no P2P/IPC between these GPUs
+                ok, why = 0, f"peer_open: {type(e).__name__}: {str(e)[:100]}"
+        elif ok:
+            ok, why = 0, "another rank could not export its replica"
+        if world > 1:
+            flag = torch.tensor([ok], dtype=torch.int32)
+            if dist.get_backend(group) != "gloo":
+                flag = flag.to(replica.device)
+            dist.all_reduce(flag, op=dist.ReduceOp.MIN, group=group)
+            ok_all = int(flag.item())
+        else:
+            ok_all = ok
+        if ok_all:
+            return "fused", ""
+        if ok:
+            replica.peer_close()
+        return "nccl", why or "another rank could not open its peers"
+
     def _merge(self, alpha):
         rep, h = self.rep, self.h
         if self.merge == "fused":
@@ -202,7 +238,7 @@ class DistributedAdaptiveSGD:
         n_steps = rep.run_static(r, N, h.b_max, stream_rows, h.lr_max, self.losses, self.inflight)
         rep.sqnorm(self.sq)
         us, bs, nu = exchange_stats(n_steps, h.b_max, self.sq, rep.P, N, self.group)   # also the barrier
-        alpha = [1.0 / N] * N
+        alpha = api.elastic_weights(N)
         self._merge(alpha)
         routes = []
         if keep_log and r == 0:
@@ -245,7 +281,7 @@ class SimulatedAdaptiveSGD:
         for i, rep in enumerate(self.reps):
             rep.sqnorm(self.sq[i:i + 1])
         P = self.reps[0].P
-        nu = [math.sqrt(float(x)) / P for x in self.sq.cpu().numpy()]
+        nu = api.norm_per_param(self.sq.cpu().numpy(), P)
         alpha, rr, ss, pert = api.merge_weights(u, self.b, nu, h.pert_thr, h.delta, h.pert_renorm, h.norm)
         r0 = self.reps[0]
         r0.weighted_sum(self.reps, alpha, r0.params)

@@ -7,7 +7,8 @@ PAPER.md P:1408-1413), the per-pass sample permutations, the initial model
 parameters, and the per-config hyperparameters.  See DESIGN.md "Inputs".
 """
 from .xmlgen import (CONFIGS, XmlConfig, Dataset, generate, init_params,
-                     pass_permutation, sample_stream, config, param_layout)
+                     pass_permutation, sample_stream, config, param_layout,
+                     planted_params)
 
 __all__ = ["CONFIGS", "XmlConfig", "Dataset", "generate", "init_params",
-           "pass_permutation", "sample_stream", "config", "param_layout"]
+           "pass_permutation", "sample_stream", "config", "param_layout", "planted_params"]

@@ -7,7 +7,8 @@ Recipe:
   chunking, thread count and machine.  Uniforms take the top 53 bits.
   Streams: 0 nnz counts, 1 feature ids, 2 values, 3 label counts, 4 label ids,
   5 label signatures, 6 per-pass permutations, 7 init weights, 8 block nnz
-  multipliers, 9 label-rank scramble, 10 feature-rank scramble.
+  multipliers, 9 label-rank scramble, 10 feature-rank scramble, 11 planted
+  biases (planted_params).
 * nnz per row: lognormal with mean s_bar (sigma per config), rounded
   half-to-even, clipped to [1, F].  Wiki10-shaped rows come in blocks of 64
   sharing a lognormal(sigma_b = 1, mean 1) multiplier ("heavy nnz skew across
@@ -379,4 +380,36 @@ def init_params(cfg: XmlConfig) -> np.ndarray:
     for c0 in range(0, n2, 1 << 24):
         i = np.arange(c0, min(n2, c0 + (1 << 24)), dtype=np.int64)
         w[o + c0:o + c0 + len(i)] = (_normal(cfg.seed, 7, 2, i) / math.sqrt(cfg.L)).astype(np.float32)
+    return w
+
+
+def planted_params(cfg: XmlConfig, kappa: float = 100.0) -> np.ndarray:
+    """A trained-like parameter state for teacher-forced parity steps (fp32,
+    same layout as init_params).  Not a trained model: a seeded surrogate
+    whose softmax is peaked the way a trained one is.
+
+    W1 is the init W1 (stream 7); W2 row j is kappa times the unit vector of
+    the sum of the W1 rows of label j's 16 signature features (stream 5), so
+    rows carrying j's signature score high on j; b1 ~ 0.01 N(0, 1) and
+    b2 ~ 0.5 N(0, 1) (stream 11).  At kappa = 100 the EURLex-shaped softmax
+    has a median top probability ~0.4 and a median logit range ~33 (a flat
+    ~1/L at init).  This is input generation: a linear combination of the
+    generator's own tables, no step of the method."""
+    F, H, L = cfg.F, cfg.H, cfg.L
+    lay = param_layout(F, H, L)
+    w = init_params(cfg)
+    W1 = w[:F * H].reshape(F, H)
+    sig = _tables(cfg)[4]
+    o2 = lay["W2"][0]
+    W2 = w[o2:o2 + L * H].reshape(L, H)
+    for j0 in range(0, L, 32768):
+        j1 = min(L, j0 + 32768)
+        S = np.zeros((j1 - j0, H), dtype=np.float64)
+        for k in range(sig.shape[1]):
+            S += W1[sig[j0:j1, k]]
+        S /= np.maximum(np.linalg.norm(S, axis=1, keepdims=True), 1e-30)
+        W2[j0:j1] = (kappa * S).astype(np.float32)
+    ob1, ob2 = lay["b1"][0], lay["b2"][0]
+    w[ob1:ob1 + H] = (0.01 * _normal(cfg.seed, 11, 0, np.arange(H, dtype=np.int64))).astype(np.float32)
+    w[ob2:ob2 + L] = (0.5 * _normal(cfg.seed, 11, 1, np.arange(L, dtype=np.int64))).astype(np.float32)
     return w

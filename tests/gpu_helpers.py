@@ -1,5 +1,7 @@
 """Shared helpers of the GPU parity tests (CUDA path vs the CPU oracle)."""
 import functools
+import json
+import os
 
 import numpy as np
 import torch
@@ -18,6 +20,56 @@ def normwise(a, b):
     b = np.asarray(b, dtype=np.float64)
     nb = np.linalg.norm(b)
     return np.linalg.norm(a - b) / (nb if nb > 0 else 1.0)
+
+
+def _row_errors(a, b):
+    """Per-row error ||a_r - b_r|| / max(||b_r||, rms row norm of b): relative to
+    the row's own norm, with rows far below the typical norm measured against
+    the typical norm (a row wrong by 100 % of a typical row fails)."""
+    a = np.asarray(a, dtype=np.float64)
+    b = np.asarray(b, dtype=np.float64)
+    if a.shape[0] == 0:
+        return np.zeros(0)
+    nb = np.linalg.norm(b, axis=1)
+    floor = np.sqrt(np.mean(nb * nb))
+    return np.linalg.norm(a - b, axis=1) / np.maximum(nb, floor if floor > 0 else 1.0)
+
+
+def check_grads(gg, og, tol, F, H, touched, tag=""):
+    """Normwise, per-row and elementwise parity of the four gradient tensors.
+
+    * normwise ||g - o|| / ||o|| <= tol per tensor (north_star tolerance);
+    * per row (W1 touched rows, W2 rows): _row_errors <= tol;
+    * elementwise: |g - o| <= tol |o| + tol rms(o) (numpy assert_allclose with
+      rtol = tol, atol = tol rms), W1 restricted to the touched rows.
+    The achieved errors are returned and appended to $ASGD_PARITY_LOG (JSON
+    lines) when that is set, so the margin under each bar is on record."""
+    L = len(og["b2"])
+    rec = {"tag": tag, "tol": tol}
+    for k in ("W1", "b1", "W2", "b2"):
+        rec[f"norm_{k}"] = float(normwise(gg[k], og[k]))
+    W1g = np.asarray(gg["W1"]).reshape(F, H)[touched]
+    W1o = np.asarray(og["W1"]).reshape(F, H)[touched]
+    W2g = np.asarray(gg["W2"]).reshape(L, H)
+    W2o = np.asarray(og["W2"]).reshape(L, H)
+    rec["row_W1_max"] = float(_row_errors(W1g, W1o).max(initial=0.0))
+    rec["row_W2_max"] = float(_row_errors(W2g, W2o).max(initial=0.0))
+    pairs = {"W1": (W1g, W1o), "b1": (gg["b1"], og["b1"]), "W2": (W2g, W2o), "b2": (gg["b2"], og["b2"])}
+    for k, (a, b) in pairs.items():
+        a = np.asarray(a, dtype=np.float64)
+        b = np.asarray(b, dtype=np.float64)
+        rms = float(np.sqrt(np.mean(b * b))) if b.size else 0.0
+        rec[f"elem_{k}"] = float((np.abs(a - b) / (tol * np.abs(b) + tol * rms + 1e-300)).max(initial=0.0))
+    log = os.environ.get("ASGD_PARITY_LOG")
+    if log:
+        with open(log, "a") as f:
+            f.write(json.dumps(rec) + "\n")
+    for k in ("W1", "b1", "W2", "b2"):
+        assert rec[f"norm_{k}"] <= tol, (tag, k, rec)
+        assert rec[f"elem_{k}"] <= 1.0, (tag, "elementwise", k, rec)
+    assert rec["row_W1_max"] <= tol, (tag, "W1 row", rec)
+    assert rec["row_W2_max"] <= tol, (tag, "W2 row", rec)
+    return rec
 
 
 def split_grad(g, F, H, L):

@@ -179,3 +179,29 @@ def test_hyper_rejects_unknown_method_switches():
         train.Hyper(**base, scale_every=0)
     with pytest.raises(ValueError):
         api.merge_weights([1, 2], [32, 32], [1.0, 1.0], norm="uu")
+
+
+def test_route_replay_rejects_out_of_range_ranks():
+    from paper_conf_ipps_marws22_b200 import _lib
+    for bad in ([0, 2, 1], [0, -1]):
+        with pytest.raises(_lib.AsgdError):
+            api.route_replay(bad, [8, 8], 40)
+
+
+def test_norm_per_param_and_elastic_weights():
+    """Alg. 2 line 4's nu (Q16) from squared norms equals the oracle's
+    ||w||_2 / |w|; Elastic's alpha_i = 1/N (R10)."""
+    from oracle import merge as omerge
+    rng = np.random.default_rng(3)
+    for _ in range(50):
+        n = int(rng.integers(1, 9))
+        reps = [rng.normal(0, rng.uniform(0.01, 3.0), int(rng.integers(1, 5000))) for _ in range(n)]
+        P = len(reps[0])
+        reps = [r[:P] if len(r) >= P else np.resize(r, P) for r in reps]
+        sq = [float(np.dot(r, r)) for r in reps]
+        assert api.norm_per_param(sq, P) == [omerge.norm_per_param(r) for r in reps]
+    from paper_conf_ipps_marws22_b200 import _lib
+    with pytest.raises(_lib.AsgdError):
+        api.norm_per_param([-1.0], 10)
+    for n in range(1, 9):
+        assert api.elastic_weights(n) == [1.0 / n] * n

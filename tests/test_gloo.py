@@ -99,3 +99,59 @@ def test_two_ranks_gloo(tmp_path):
         ow = omerge.merge_weights(a["us"], a["bs"], a["nu"], 0.1, 0.1, False, a["norm"])
         assert a["alpha"] == ow[0] and a["pert"] == ow[3]
         assert a["merge_err"] < 1e-12
+
+
+class _FakeReplica:
+    """Stands in for api.Replica in the fused-merge consensus: rank `bad` cannot
+    export (or open) its peers."""
+    def __init__(self, rank, fail_export, fail_open):
+        self.rank, self.fail_export, self.fail_open = rank, fail_export, fail_open
+        self.device = torch.device("cpu")
+        self.opened = self.closed = False
+
+    def peer_export(self):
+        if self.fail_export:
+            raise RuntimeError("no IPC")
+        return b"h%d" % self.rank
+
+    def peer_open(self, rank, handles):
+        if self.fail_open:
+            raise RuntimeError("no P2P")
+        self.opened = True
+
+    def peer_close(self):
+        self.closed = True
+
+
+def _consensus_worker(rank, world, port, case, out_dir):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_marws22_b200 import train
+    fe = case == "export" and rank == 1
+    fo = case == "open" and rank == 1
+    rep = _FakeReplica(rank, fe, fo)
+    merge, note = train.DistributedAdaptiveSGD._open_peers(rep, rank, world, None)
+    np.save(os.path.join(out_dir, f"c{rank}.npy"),
+            np.array([dict(merge=merge, note=note, opened=rep.opened, closed=rep.closed)], dtype=object),
+            allow_pickle=True)
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("case", ["ok", "export", "open"])
+def test_fused_merge_consensus(tmp_path, case):
+    """every rank takes the same merge path.  If one rank cannot map
+    its peers all ranks fall back to NCCL, and a rank that had opened its
+    mappings closes them."""
+    world = 2
+    mp.spawn(_consensus_worker, args=(world, _free_port(), case, str(tmp_path)), nprocs=world, join=True)
+    res = [np.load(tmp_path / f"c{r}.npy", allow_pickle=True)[0] for r in range(world)]
+    merges = {r["merge"] for r in res}
+    assert len(merges) == 1
+    if case == "ok":
+        assert merges == {"fused"} and all(r["opened"] and not r["closed"] for r in res)
+    else:
+        assert merges == {"nccl"} and all(r["note"] for r in res)
+        # rank 0 opened (case "open": rank 1 failed after the all-gather) and must close
+        assert res[0]["closed"] == res[0]["opened"]
+        assert not res[1]["opened"]

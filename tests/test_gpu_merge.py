@@ -95,3 +95,75 @@ def _lab(sub, mask):
     idx = np.nonzero(mask)[0]
     s2 = sub.row_slice(idx)
     return s2.lab_ptr, s2.lab
+
+
+def _bf16(x):
+    """Round-to-nearest-even to bf16 of fp32(x) (the kernels' __float2bfloat16_rn),
+    returned as fp64, and per element the bf16 ulp where fp32(x) lies within 64
+    fp32 ulps of a rounding midpoint (0 elsewhere): there the GPU's fp32 H1
+    (~1e-6 relative, i.e. ~8 fp32 ulps, off the fp64 one) may round the other
+    way, by one bf16 ulp."""
+    f = np.asarray(x, dtype=np.float32).copy()
+    u = f.view(np.uint32)
+    low = (u & 0xFFFF).astype(np.int64)
+    near = np.abs(low - 0x8000) < 64
+    u += 0x7FFF + ((u >> 16) & 1)
+    u &= 0xFFFF0000
+    q = f.astype(np.float64)
+    ulp = np.abs(q) * 2.0 ** -7
+    return q, np.where(near, ulp, 0.0)
+
+
+@pytest.mark.parametrize("precision", ["bf16", "fp32"])
+@pytest.mark.parametrize("name", ["eurlex4k", "amazoncat13k"])
+def test_eval_topk_planted_state(name, precision):
+    """asgd_eval_topk on the bf16 path (H1 and the W2 shadow rounded to bf16, fp32
+    accumulation) -- the path bench.py's time_to_p1 evaluates with -- and on the
+    fp32 path, from the trained-like planted state (peaked, structured logits).
+
+    The top-k is an integer decided by floating point, so both sides decide it in
+    the kernel's precision: for bf16 the reference logits are formed from the same
+    bf16-rounded operands (exact products, fp64 sums), which leaves the fp32
+    accumulation order: |Z^ - Zq| <= 300 * 2^-24 * sum_h |Hq_nh| |Wq_jh| + 2^-23 |b2_j|
+    (fp32 path: 600 * 2^-24 to cover the fp32 SpMM's H1 as well).  Rows whose
+    consecutive top-(k+1) gaps all exceed twice the row's largest bound (bf16:
+    plus one bf16 ulp of every H1 element near a rounding midpoint, times |Wq_j|)
+    must match the oracle's top-k exactly (ids and order); every row must return
+    a valid top-k: each returned id's reference logit is within that bound of the
+    reference logit of the same rank."""
+    from paper_conf_ipps_marws22_b200 import api
+    from synth import planted_params
+    cfg = config(name)
+    data = dataset(name, 4096)
+    test = dataset(name, 2048, "test")
+    w0 = planted_params(cfg)
+    rep = make_replica(cfg, data, precision, w0=w0, extra=(test,))
+    td = api.DeviceCsr(test)
+    k = 5
+    rows = np.arange(min(1024, test.n_rows), dtype=np.int32)
+    top = rep.eval_topk(td, torch.as_tensor(rows, device="cuda"), k).cpu().numpy()
+    sub = test.row_slice(rows)
+    w = w0.astype(np.float64)
+    A1, H1, _ = omodel.forward(w, sub, cfg.F, cfg.H, cfg.L)
+    W1, b1, W2, b2 = omodel.split_params(w, cfg.F, cfg.H, cfg.L)
+    if precision == "bf16":
+        Hq, flip = _bf16(H1)
+        Wq, _ = _bf16(W2)
+        e = 300 * 2.0 ** -24
+    else:
+        Hq, Wq, e = H1, W2, 600 * 2.0 ** -24
+        flip = np.zeros_like(H1)
+    Z = Hq @ Wq.T + b2[None, :]
+    E = e * (np.abs(Hq) @ np.abs(Wq).T) + 2.0 ** -23 * np.abs(b2)[None, :] + flip @ np.abs(Wq).T
+    bound = 2.0 * E.max(axis=1)
+    ref = metrics.topk(Z, k)
+    srt = -np.sort(-Z, axis=1)[:, :k + 1]
+    clear = (srt[:, :k] - srt[:, 1:k + 1]).min(axis=1) > bound
+    assert clear.mean() >= 0.8, clear.mean()
+    np.testing.assert_array_equal(top[clear], ref[clear])
+    got = np.take_along_axis(Z, top.astype(np.int64), axis=1)
+    assert np.all(np.abs(got - srt[:, :k]) <= bound[:, None])
+    assert len(set(map(tuple, top.tolist()))) > 1
+    # P@k over all rows: the library's count equals the brute-force count of the same ids
+    assert api.precision_at_k_hits(top, sub.lab_ptr, sub.lab, k) == \
+        round(metrics.precision_at_k(top, sub.lab_ptr, sub.lab, k) * k * len(rows))

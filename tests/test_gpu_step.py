@@ -8,8 +8,8 @@ import pytest
 import torch
 
 from oracle import model as omodel
-from synth import config, init_params, sample_stream
-from tests.gpu_helpers import dataset, make_replica, normwise, split_grad, with_empty_row
+from synth import config, init_params, planted_params, sample_stream
+from tests.gpu_helpers import check_grads, dataset, make_replica, normwise, split_grad, with_empty_row
 
 pytestmark = pytest.mark.gpu
 
@@ -31,14 +31,12 @@ def _one_step(cfg, data, rows, precision, lr=0.5, w0=None, b_max=None, loss_kind
     return rep, g.cpu().numpy(), float(loss.item()), touched, lo, go, batch
 
 
-def _check(cfg, rep, g, loss, touched, lo, go, batch, precision):
+def _check(cfg, rep, g, loss, touched, lo, go, batch, precision, tag=""):
     tol = TOL[precision]
     assert abs(loss - lo) <= tol * abs(lo), (loss, lo)
     np.testing.assert_array_equal(touched, omodel.touched_features(batch))
     gg, og = split_grad(g, cfg.F, cfg.H, cfg.L), split_grad(go, cfg.F, cfg.H, cfg.L)
-    for k in ("W1", "b1", "W2", "b2"):
-        e = normwise(gg[k], og[k])
-        assert e <= tol, (k, e)
+    check_grads(gg, og, tol, cfg.F, cfg.H, touched, tag=f"{cfg.name}/{precision}/{tag}")
     # W1 gradient is exactly zero off the touched rows
     W1g = gg["W1"].reshape(cfg.F, cfg.H)
     off = np.ones(cfg.F, dtype=bool)
@@ -51,7 +49,7 @@ def test_step_tiny(precision):
     cfg = config("tiny")
     data = dataset("tiny")
     rows = sample_stream(cfg, 0, cfg.b_max)
-    _check(cfg, *_one_step(cfg, data, rows, precision), precision)
+    _check(cfg, *_one_step(cfg, data, rows, precision), precision, "init")
 
 
 @pytest.mark.parametrize("precision", ["fp32", "bf16"])
@@ -59,7 +57,19 @@ def test_step_eurlex_full_batch(precision):
     cfg = config("eurlex4k")
     data = dataset("eurlex4k")
     rows = sample_stream(cfg, 0, cfg.b_max)
-    _check(cfg, *_one_step(cfg, data, rows, precision), precision)
+    _check(cfg, *_one_step(cfg, data, rows, precision), precision, "init")
+
+
+@pytest.mark.parametrize("precision", ["fp32", "bf16"])
+@pytest.mark.parametrize("name", ["tiny", "eurlex4k"])
+def test_step_planted_peaked_softmax(name, precision):
+    """Teacher-forced step from the trained-like planted state (synth.planted_params:
+    peaked softmax, logit range ~30, large W2), full batch, rows from pass 3."""
+    cfg = config(name)
+    data = dataset(name)
+    rows = sample_stream(cfg, 3 * cfg.n_train + 7, cfg.b_max)
+    w0 = planted_params(cfg)
+    _check(cfg, *_one_step(cfg, data, rows, precision, w0=w0), precision, "planted")
 
 
 @pytest.mark.parametrize("precision", ["fp32", "bf16"])
@@ -98,22 +108,33 @@ def test_step_is_deterministic(precision):
     np.testing.assert_array_equal(outs[0], outs[1])
 
 
-def test_teacher_forced_steps_tiny():
-    """Every step starts both sides from the same (GPU) state."""
+@pytest.mark.parametrize("precision", ["fp32", "bf16"])
+def test_teacher_forced_steps_tiny(precision):
+    """Every step starts both sides from the same state: the ORACLE's free-running
+    trajectory (fp64 SGD from w0) is rounded to fp32 and loaded into the replica
+    before each GPU step (no oracle input ever comes from the GPU)."""
     cfg = config("tiny")
     data = dataset("tiny")
-    rep = make_replica(cfg, data, "fp32")
+    rep = make_replica(cfg, data, precision)
     g = torch.zeros(rep.P, dtype=torch.float32, device="cuda")
     rep.set_debug_grads(g)
+    w = init_params(cfg).astype(np.float64)
+    tol = TOL[precision]
     for k in range(10):
         rows = sample_stream(cfg, k * 32, 32)
-        w_before = rep.params.cpu().numpy().astype(np.float64)
+        w32 = w.astype(np.float32)
+        rep.params.copy_(torch.from_numpy(w32))
+        rep.params_changed()
         rep.step(torch.as_tensor(rows, device="cuda"), 0.7)
         rep.sync()
-        _, go = omodel.loss_and_grad(w_before, data.row_slice(rows), cfg.F, cfg.H, cfg.L)
-        assert normwise(g.cpu().numpy(), go) <= 1e-4
-        w_after = rep.params.cpu().numpy().astype(np.float64)
-        assert normwise(w_after, w_before - 0.7 * go) <= 1e-6
+        batch = data.row_slice(rows)
+        _, go = omodel.loss_and_grad(w32.astype(np.float64), batch, cfg.F, cfg.H, cfg.L)
+        gg, og = split_grad(g.cpu().numpy(), cfg.F, cfg.H, cfg.L), split_grad(go, cfg.F, cfg.H, cfg.L)
+        check_grads(gg, og, tol, cfg.F, cfg.H, omodel.touched_features(batch), tag=f"tiny/{precision}/tf{k}")
+        if precision == "fp32":
+            w_after = rep.params.cpu().numpy().astype(np.float64)
+            assert normwise(w_after, w32 - 0.7 * go) <= 1e-6
+        w, _, _ = omodel.sgd_step(w, batch, 0.7, cfg.F, cfg.H, cfg.L)
 
 
 # ---------------------------------------------------------------- sigmoid-BCE head (R11)
