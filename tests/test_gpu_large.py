@@ -9,6 +9,7 @@ import torch
 
 from oracle import model as omodel
 from synth import config, init_params, planted_params, sample_stream
+from tests.bf16_emul import grads_bf16
 from tests.gpu_helpers import check_grads, dataset, make_replica, split_grad
 
 pytestmark = pytest.mark.gpu
@@ -16,16 +17,22 @@ pytestmark = pytest.mark.gpu
 TOL = {"fp32": 1e-4, "bf16": 2e-2}
 
 
-def _chunked_oracle(w, batch, F, H, L, chunk, loss_kind="softmax"):
+def _chunked_oracle(w, batch, F, H, L, chunk, loss_kind="softmax", emulate=False):
+    """Oracle loss and gradient of the batch in row chunks; with emulate, also the
+    bf16-rounding reference (tests/bf16_emul.py), whose chunks sum directly (the
+    1/B of the full batch is applied before its dZ rounding)."""
     B = batch.n_rows
-    loss, g = 0.0, None
+    loss, g, e = 0.0, None, None
     for r0 in range(0, B, chunk):
         sub = batch.row_slice(np.arange(r0, min(B, r0 + chunk)))
         lo, go = omodel.loss_and_grad(w, sub, F, H, L, loss_kind)
         f = sub.n_rows / B
         loss += f * lo
         g = f * go if g is None else g + f * go
-    return loss, g
+        if emulate:
+            ge = grads_bf16(w, sub, F, H, L, loss_kind, B_full=B)
+            e = ge if e is None else e + ge
+    return loss, g, e
 
 
 def _check_big(name, n_rows, precision, chunk, seed_pos=0, loss_kind="softmax", planted=False):
@@ -42,13 +49,15 @@ def _check_big(name, n_rows, precision, chunk, seed_pos=0, loss_kind="softmax", 
     rep.sync()
     touched = rep.last_touched().cpu().numpy()
     batch = data.row_slice(rows)
-    lo, go = _chunked_oracle(w0.astype(np.float64), batch, cfg.F, cfg.H, cfg.L, chunk, loss_kind)
+    lo, go, em = _chunked_oracle(w0.astype(np.float64), batch, cfg.F, cfg.H, cfg.L, chunk, loss_kind,
+                                 emulate=precision == "bf16")
     tol = TOL[precision]
     assert abs(loss.item() - lo) <= tol * abs(lo)
     np.testing.assert_array_equal(touched, omodel.touched_features(batch))
     gg, og = split_grad(g.cpu().numpy(), cfg.F, cfg.H, cfg.L), split_grad(go, cfg.F, cfg.H, cfg.L)
+    eg = split_grad(em, cfg.F, cfg.H, cfg.L) if em is not None else None
     check_grads(gg, og, tol, cfg.F, cfg.H, touched,
-                tag=f"{name}/{precision}/{loss_kind}/{'planted' if planted else 'init'}")
+                tag=f"{name}/{precision}/{loss_kind}/{'planted' if planted else 'init'}", emul=eg)
 
 
 @pytest.mark.parametrize("precision", ["bf16", "fp32"])
