@@ -165,42 +165,35 @@ def cpu_baseline(cfg, data, budget_s: float, loss: str = "softmax"):
 
 # ------------------------------------------------------------------ roofline
 def kernel_work(cls: str, cfg, bf16: bool, st, loss: str = "softmax"):
-    """Algorithmic (bytes, flops) of one launch of a kernel class:
-    operands read once, outputs written once, no credit for cache reuse across
-    kernels.  The kernel's bound is whichever of bytes / HBM peak and flops /
-    compute peak is larger (`roofline_of`)."""
+    """Algorithmic (bytes, flops) of one launch of a kernel class (DESIGN.md §5,
+    SURVEY.md §8(d)): operands read once, outputs written once, no credit for
+    cache reuse across kernels.  Logits traffic (Z, dZ), the W2 operand shadow's
+    refresh and the fused softmax's Z recompute are IMPLEMENTATION bytes / flops
+    (§8(d)) and are not counted: they show up as ncu traffic above the
+    algorithmic bytes.  GEMM operands count in the precision the path feeds the
+    tensor cores (bf16: 2 B; fp32 path: bf16x3 hi + lo, 4 B).  The kernel's bound
+    is whichever of bytes / HBM peak and flops / compute peak is larger
+    (`roofline_of`)."""
     B, H, L, F, P = st["B"], cfg.H, cfg.L, cfg.F, cfg.n_params
     nnz, U = st["nnz"], st["U"]
     e = 2.0 if bf16 else 4.0                      # bytes per GEMM operand element
-    fused = bf16 and loss == "softmax" and cfg.b_max * L * 4 > (32 << 20)
     gemm = 2.0 * B * H * L
-    if cls == "g1":     # H1 . W2^T + b2: W2 (shadow) + H1 in; Z (fp32, unfused) or 2 fp32 stats per row and tile
-        out = (8.0 * B * 2 * ((L + 255) // 256)) if (fused or (bf16 and loss == "sigmoid")) else 4.0 * B * L
-        if bf16 and loss == "sigmoid":
-            out += 2.0 * B * L                    # dZ written by G1's sigmoid epilogue
-        return (e * H * L + e * B * H + 4.0 * L + out, gemm)
-    if cls == "g2":     # dZ . W2: dZ + W2 (shadow) in, dH1 out (split-K partials are implementation bytes)
-        return (e * B * L + e * H * L + 4.0 * B * H, gemm)
-    if cls == "g3":     # W2 -= lr dZ^T H1: dZ + H1 in, W2 read + written (fp32), bf16 shadow written, b2
-        return (e * B * L + e * B * H + 8.0 * H * L + (2.0 * H * L if bf16 else 0.0) + 8.0 * L, gemm)
+    if cls == "g1":     # Z = H1 . W2^T + b2: W2 and H1 operands, b2
+        return (e * H * L + e * B * H + 4.0 * L, gemm)
+    if cls == "g2":     # dH1 = dZ . W2: the W2 operand in, dH1 out (dZ is logits traffic)
+        return (e * H * L + 4.0 * B * H, gemm)
+    if cls == "g3":     # W2 -= lr dZ^T H1, b2 -= lr 1^T dZ: W2 and b2 read + written (fp32), the H1 operand
+        return (8.0 * H * L + 8.0 * L + e * B * H, gemm)
     if cls == "spmm":
         return (8.0 * nnz + 12.0 * B + 4.0 * U * H + 4.0 * B * H, 2.0 * nnz * H)
     if cls == "scatter":
         return (8.0 * nnz + 4.0 * B * H + 8.0 * U * H, 2.0 * nnz * H)
-    if cls == "softmax":
-        if loss == "sigmoid":   # fp32: k_sigmoid_ce over stored Z; bf16: k_tile_loss (the BCE is in G1)
-            if bf16:
-                return (8.0 * B * 2 * ((L + 255) // 256) + 4.0 * B, 0.0)
-            return (8.0 * B * L + 8.0 * st["nlab"], 0.0)
-        if fused:   # k_lse + G1b: Z recomputed on tensor cores, bf16 dZ stored
-            return (2.0 * H * L + 2.0 * B * H + 2.0 * B * L + 8.0 * st["nlab"], gemm)
-        return ((6.0 if bf16 else 8.0) * B * L + 8.0 * st["nlab"], 0.0)
+    if cls == "softmax":   # the row loss from the labels; Z in / dZ out are logits traffic
+        return (8.0 * st["nlab"] + 4.0 * B, 0.0)
     if cls == "touched":
         return (4.0 * nnz + 12.0 * nnz + 8.0 * F + 12.0 * B, 0.0)
     if cls == "dh_b1":
         return (4.0 * st.get("splitk", 1) * B * H + 8.0 * B * H, 0.0)
-    if cls == "b2":
-        return ((2.0 if bf16 else 4.0) * B * L + 8.0 * L, 0.0)
     if cls == "merge":
         return (12.0 * P, 0.0)   # 36 P per mega-batch over its 3 launches
     return (0.0, 0.0)
@@ -208,13 +201,15 @@ def kernel_work(cls: str, cfg, bf16: bool, st, loss: str = "softmax"):
 
 def roofline_of(cls, cfg, bf16, st, loss, avg_s, peaks):
     """Bound, achieved, peak and unit of one kernel class from its algorithmic
-    (bytes, flops) per launch and its measured average launch time."""
+    (bytes, flops) per launch and its measured average launch time.  Tensor peak:
+    the measured bf16 one (sustained: the kernels run inside a long step); the
+    fp32 path issues three bf16 MMAs per product (bf16x3, R14), so its
+    contraction ceiling is a third of it."""
     by, fl = kernel_work(cls, cfg, bf16, st, loss)
     hbm = peaks["hbm_gbs"]
-    if bf16:
-        cpk, cb = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"]), "tensor"
-    else:   # fp32 SIMT path: FFMA peak, 148 SMs x 128 lanes x 2 x max clock
-        cpk, cb = 148 * 128 * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12, "alu"
+    cpk, cb = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"]), "tensor"
+    if not bf16:
+        cpk = cpk / 3.0
     if cls in ("spmm", "scatter"):   # CUDA-core FMAs
         cpk, cb = 148 * 128 * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12, "alu"
     if fl / (cpk * 1e12) > by / (hbm * 1e9):
@@ -410,8 +405,7 @@ def main():
                                    "note": "side stream s2, overlapped with K-1..G2 (warm-up profile)"}
         # whole-job roofline: sum of per-step ideal times with
         # each step's measured B, nnz, U, + merge 36 P bytes / HBM peak, over the timed time
-        tc_peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"]) if bf16 else \
-            148 * 128 * 2 * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+        tc_peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"]) / (1.0 if bf16 else 3.0)
         t_ideal = sum(step_ideal_s(cfg, b_, z_, u_, l_, peaks["hbm_gbs"], tc_peak)
                       for b_, z_, u_, l_ in zip(B_list, nnz_l, U_l, lab_l))
         t_ideal += K * 36.0 * cfg.n_params / (peaks["hbm_gbs"] * 1e9)

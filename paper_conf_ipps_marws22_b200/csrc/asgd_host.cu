@@ -77,8 +77,9 @@ int splitk_for(const asgd_model_desc& d) {
   // G2 (dH1 = dZ W2, M = b_max, N = H, K = L): split K so ~2 waves of CTAs run (ASGD_G2_WAVES;
   // one wave measured: Amazon-670K G2 372 -> 602 us, Delicious-200K 125 -> 192 us, AmazonCat even)
   int64_t tiles;
+  // N tile: 256 (bf16) or 128 (bf16x3 fp32 path, R14: hi + lo stages)
   if (d.precision == ASGD_PREC_BF16) tiles = ((d.b_max + 127) / 128) * ((d.H + 255) / 256);
-  else tiles = ((d.b_max + 63) / 64) * ((d.H + 63) / 64);
+  else tiles = ((d.b_max + 127) / 128) * ((d.H + 127) / 128);
   static const int64_t waves = [] { const char* e = getenv("ASGD_G2_WAVES"); return e ? atoll(e) : 2ll; }();
   int64_t s = (waves * 148 + tiles - 1) / tiles;
   s = std::min<int64_t>(s, std::max<int64_t>(1, d.L / 256));
@@ -103,7 +104,10 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   const int64_t Lp = padded_ld(Lb);
   L.n_red = kSqnormParts;
   L.part_stride = B * H;
-  const bool bf = d.precision == ASGD_PREC_BF16;
+  // both paths run the output layer on the tensor cores: bf16 operands, or (fp32 path,
+  // R14) bf16x3 hi + lo operands -- every bf16 operand buffer exists on both paths
+  const bool bf = true;
+  L.x3 = d.precision != ASGD_PREC_BF16;
   size_t o = 0;
   auto take = [&](size_t bytes) { size_t r = o; o = up256(o + std::max<size_t>(bytes, 1)); return r; };
   L.meta = take(64 * 4);
@@ -129,7 +133,6 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.h1b = take(bf ? B * H * 2 : 0);
   L.z = take((size_t)B * Lp * 4);
   L.dzb = take(bf ? (size_t)B * Lp * 2 : 0);
-  L.b2part = take((size_t)b2_chunks() * Lb * 4);
   L.rbase = take((size_t)(B + 1) * 8);
   L.da1b = take(bf ? (size_t)B * H * 2 : 0);
   L.stats_ld = B;
@@ -146,6 +149,10 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.rowsc = take(B * 4);
   L.cen = take(bf ? (size_t)2 * H * 4 : 0);
   L.cenpart = take(bf ? (size_t)2 * kCenterParts * H * 4 : 0);
+  L.h1l = take(L.x3 ? B * H * 2 : 0);
+  L.dzl = take(L.x3 ? (size_t)B * Lp * 2 : 0);
+  L.w2l = take(L.x3 ? (size_t)Lb * H * 2 : 0);
+  L.w2l2 = take(L.x3 ? (size_t)Lb * H * 2 : 0);
   L.total = o;
   return L;
 }
@@ -163,13 +170,15 @@ Ptrs ws_ptrs(char* b, const WsLayout& L) {
   p.rowloss = (float*)(b + L.rowloss); p.dhpart = (float*)(b + L.dhpart); p.da1 = (float*)(b + L.da1);
   p.db1part = (float*)(b + L.db1part); p.w2b = (bf16*)(b + L.w2b); p.red = (double*)(b + L.red);
   p.eval_top = (int32_t*)(b + L.eval_top);
-  p.b2part = (float*)(b + L.b2part);
   p.rbase = (int64_t*)(b + L.rbase);
   p.da1b = (bf16*)(b + L.da1b);
   p.lse = (float*)(b + L.lse);
   p.rowsc = (int32_t*)(b + L.rowsc);
   p.cen = (float*)(b + L.cen);
   p.cenpart = (float*)(b + L.cenpart);
+  p.h1l = L.x3 ? (bf16*)(b + L.h1l) : nullptr;
+  p.dzl = L.x3 ? (bf16*)(b + L.dzl) : nullptr;
+  p.w2l = L.x3 ? (bf16*)(b + L.w2l) : nullptr;
   return p;
 }
 
@@ -220,7 +229,8 @@ struct asgd_ctx {
   cudaStream_t s3 = nullptr;                     // side stream: G3 + b1 (bf16 path)
   cudaStream_t sc = nullptr;                     // private stream the step graphs are captured on
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_sm = nullptr, ev_dh = nullptr, ev_a = nullptr;
-  bf16* w2b_buf[2] = {nullptr, nullptr};         // double-buffered bf16 W2 shadow
+  bf16* w2b_buf[2] = {nullptr, nullptr};         // double-buffered bf16 W2 shadow (hi half on fp32)
+  bf16* w2l_buf[2] = {nullptr, nullptr};         // fp32 path: its bf16x3 lo half (R14)
   int w2b_cur = 0;
   std::list<StepGraph> graphs;                   // CUDA-graph cache of the step, LRU (stable addresses:
                                                  // the graphs point at their own StepArgs)
@@ -243,6 +253,12 @@ struct asgd_ctx {
 
 namespace {
 constexpr size_t kMaxProfPairs = 8192;
+
+// The GEMM operand copy of W2 (bf16 shadow; fp32 path: its hi and lo halves) from params.
+cudaError_t refresh_shadow(asgd_ctx* c) {
+  return launch_to_bf16(c->lc(), c->params + c->o_w2, c->w2b_buf[c->w2b_cur], c->d.L * c->d.H,
+                        c->w2l_buf[c->w2b_cur]);
+}
 
 // Record an event on stream st at the start / end of a kernel-class section.
 void prof_mark(asgd_ctx* c, int cls, bool begin, cudaStream_t st) {
@@ -329,7 +345,7 @@ extern "C" {
 
 const char* asgd_last_error(void) { return g_err.c_str(); }
 
-const char* asgd_version(void) { return "libasgd sm_100a (tcgen05/TMA bf16 + fp32 SIMT) r1 bf16-ready"; }
+const char* asgd_version(void) { return "libasgd sm_100a (tcgen05/TMA: bf16, fp32 as bf16x3) r2 bf16-ready"; }
 
 size_t asgd_workspace_bytes(const asgd_model_desc* d) {
   if (!d || d->F <= 0 || d->L <= 0 || d->b_max <= 0 || d->max_step_nnz <= 0) return 0;
@@ -362,8 +378,8 @@ int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device, v
                 prop.major, prop.minor);
   if (m.precision == ASGD_PREC_BF16 && m.H > 256)   // G1's resident H1 block holds K = H <= 256
     return fail(ASGD_E_UNSUPPORTED, "bf16 path: H=%lld > 256", (long long)m.H);
-  if (m.precision == ASGD_PREC_BF16 && !tc_available())
-    return fail(ASGD_E_UNSUPPORTED, "bf16 tcgen05 path not built");
+  if (!tc_available())   // both precisions run the output layer on tcgen05
+    return fail(ASGD_E_UNSUPPORTED, "tcgen05 path unavailable (cuTensorMapEncodeTiled)");
   asgd_ctx* c = new (std::nothrow) asgd_ctx();
   if (!c) return fail(ASGD_E_ARG, "out of host memory");
   c->d = m;
@@ -389,13 +405,16 @@ int asgd_replica_init(asgd_ctx** out, const asgd_model_desc* desc, int device, v
   c->Pn = c->o_b2 + m.L;
   c->w2b_buf[0] = c->P.w2b;
   c->w2b_buf[1] = reinterpret_cast<bf16*>(c->ws + c->L.w2b2);
+  if (c->L.x3) {
+    c->w2l_buf[0] = c->P.w2l;
+    c->w2l_buf[1] = reinterpret_cast<bf16*>(c->ws + c->L.w2l2);
+  }
   cudaError_t e = cudaStreamCreateWithFlags(&c->s2, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->s3, cudaStreamNonBlocking);
   for (cudaEvent_t* ev : {&c->ev_fork, &c->ev_join, &c->ev_sm, &c->ev_dh, &c->ev_a})
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(ev, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->ws, 0, c->L.total, c->s);
-  if (e == cudaSuccess && m.precision == ASGD_PREC_BF16)
-    e = launch_to_bf16(c->lc(), c->params + c->o_w2, c->w2b_buf[c->w2b_cur], m.L * m.H);
+  if (e == cudaSuccess) e = refresh_shadow(c);
   if (e == cudaSuccess) e = cudaStreamSynchronize(c->s);
   if (e != cudaSuccess) { asgd_replica_destroy(c); return cuda_fail(e, "replica_init"); }
   *out = c;
@@ -429,8 +448,7 @@ int asgd_set_stream(asgd_ctx* c, void* stream) {
 
 int asgd_params_changed(asgd_ctx* c) {
   if (!c) return fail(ASGD_E_ARG, "null ctx");
-  if (c->d.precision == ASGD_PREC_BF16)
-    CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->w2b_buf[c->w2b_cur], c->d.L * c->d.H));
+  CU(refresh_shadow(c));
   return ASGD_OK;
 }
 
@@ -507,53 +525,20 @@ int enqueue_step(asgd_ctx* c, int n) {
   };
   if (!k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   // K-1
-  PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, c->sa, x, W1, b1, H, P, c->L, bf));
+  PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, c->sa, x, W1, b1, H, P, c->L, true));   // H1 fp32 + bf16 (+ lo)
   if (k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
-  if (!bf) {
-    // fp32 path: one stream, G2 reads W2 before G3 updates it in place
-    GemmArgs a{};
-    // G1: Z[n x L] = H1 W2^T + b2
-    a.M = n; a.N = (int)Lb; a.K = H;
-    a.A = P.h1; a.as0 = H; a.as1 = 1;
-    a.B = W2; a.bs0 = 1; a.bs1 = H;
-    a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = Lp; a.bias = b2; a.splitk = 1;
-    PCU(ASGD_K_G1, launch_gemm_f32(lc, a));
-    if (m.loss == ASGD_LOSS_SIGMOID)
-      PCU(ASGD_K_SOFTMAX, launch_sigmoid_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, false));
-    else
-      PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, false));
-    // G2: dH1 partials = dZ W2 (pre-step W2)
-    a = GemmArgs{};
-    a.M = n; a.N = H; a.K = (int)Lb;
-    a.A = P.z; a.as0 = Lp; a.as1 = 1;
-    a.B = W2; a.bs0 = H; a.bs1 = 1;
-    a.epi = EPI_SPLITK; a.C = P.dhpart; a.ldc = H; a.splitk = (int)c->L.splitk;
-    a.part_stride = c->L.part_stride;
-    PCU(ASGD_K_G2, launch_gemm_f32(lc, a));
-    PCU(ASGD_K_DH, ([&]() -> cudaError_t {
-          cudaError_t e = launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, false);
-          return e != cudaSuccess ? e : launch_b1_update(lc, n, H, b1, P, c->L, g ? g + c->o_b1 : nullptr);
-        })());
-    PCU(ASGD_K_B2, launch_b2_update(lc, n, Lb, Lp, b2, P, false, g ? g + c->o_b2 : nullptr));
-    // G3: W2 -= lr dZ^T H1
-    a = GemmArgs{};
-    a.M = (int)Lb; a.N = H; a.K = n;
-    a.A = P.z; a.as0 = 1; a.as1 = Lp;
-    a.B = P.h1; a.bs0 = H; a.bs1 = 1;
-    a.epi = EPI_SGD; a.C = W2; a.ldc = H; a.meta = P.meta; a.grad = g ? g + c->o_w2 : nullptr;
-    a.splitk = 1;
-    PCU(ASGD_K_G3, launch_gemm_f32(lc, a));
-    // K-5 (needs K-0's segments)
-    CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
-    PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
-  } else {
-    // bf16 path, a DAG over three streams:
+  {
+    // A DAG over three streams (both precisions; the fp32 path's GEMMs take bf16x3
+    // hi + lo operands, R14, and always store Z):
     //   s : G1 -> softmax -> G2 -> dH reduce -> [K-0 joined] K-5
     //   s3: [after softmax] G3 (W2, b2 and the next step's bf16 W2 shadow) -> [after dH] b1
     // G1/G2 read the bf16 shadow w2b[cur]; G3 writes w2b[cur ^ 1], so G2 and G3 never race.
+    const bool x3 = c->L.x3;
     Ptrs Pr = P, Pw = P;
     Pr.w2b = c->w2b_buf[c->w2b_cur];
     Pw.w2b = c->w2b_buf[c->w2b_cur ^ 1];
+    Pr.w2l = c->w2l_buf[c->w2b_cur];
+    Pw.w2l = c->w2l_buf[c->w2b_cur ^ 1];
     // G3 (s3) runs beside G2 (s): both need ~200 KB of smem per CTA, so G3's
     // persistent grid leaves G2's CTAs their own SMs when G2 is small
     Launch lc3 = c->lc3();
@@ -561,7 +546,21 @@ int enqueue_step(asgd_ctx* c, int n) {
     if (2 * g2c <= c->sms) lc3.sms = c->sms - g2c;
     float2* zstat = reinterpret_cast<float2*>(c->ws + c->L.zstat);
     int ntiles = 0;
-    if (m.loss == ASGD_LOSS_SIGMOID) {
+    if (x3) {
+      // fp32 path: G1 stores Z (+ per-tile softmax partials), then the loss kernel writes dZ
+      // as bf16x3 hi + lo (sigmoid: centred, R11 / R14)
+      PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
+      if (m.loss == ASGD_LOSS_SIGMOID)
+        PCU(ASGD_K_SOFTMAX, ([&]() -> cudaError_t {
+              cudaError_t e = launch_sigmoid_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, true);
+              return e != cudaSuccess ? e
+                                      : launch_sig_center(lc, nullptr, W2, Lb, H, P.h1, n, P.cenpart,
+                                                          reinterpret_cast<unsigned int*>(P.meta + M_CEN), P.cen);
+            })());
+      else
+        PCU(ASGD_K_SOFTMAX, launch_softmax_ce(lc, n, Lb, Lp, P.rowsc, x.lab_ptr, x.lab, P, true, zstat, ntiles,
+                                              c->L.stats_ld));
+    } else if (m.loss == ASGD_LOSS_SIGMOID) {
       // sigmoid-BCE needs no row normaliser: G1's epilogue writes dZ (bf16) and per-tile
       // row-loss partials directly, Z never stored, at every L (R11)
       PCU(ASGD_K_G1, launch_gemm_tc(lc, 6, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles, P.rowsc,
@@ -569,7 +568,7 @@ int enqueue_step(asgd_ctx* c, int n) {
       PCU(ASGD_K_SOFTMAX, ([&]() -> cudaError_t {
             cudaError_t e = launch_tile_loss(lc, n, ntiles, c->L.stats_ld, zstat, P);
             return e != cudaSuccess ? e
-                                    : launch_sig_center(lc, Pr.w2b, Lb, H, P.h1, n, P.cenpart,
+                                    : launch_sig_center(lc, Pr.w2b, nullptr, Lb, H, P.h1, n, P.cenpart,
                                                         reinterpret_cast<unsigned int*>(P.meta + M_CEN), P.cen);
           })());
     } else if ((int64_t)m.b_max * Lb * 4 <= fused_ce_bytes()) {
@@ -605,7 +604,7 @@ int enqueue_step(asgd_ctx* c, int n) {
       PCU_ON(c->s3, ASGD_K_G3, g3(lc3));
     }
     PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr));
-    PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, true, centred ? P.cen : nullptr));
+    PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, bf, centred ? P.cen : nullptr));
     CU(cudaEventRecord(c->ev_dh, c->s));
     CU(cudaStreamWaitEvent(c->s3, c->ev_dh, 0));
     PCU_ON(c->s3, ASGD_K_DH, launch_b1_update(lc3, n, H, b1, P, c->L, g ? g + c->o_b1 : nullptr));
@@ -736,7 +735,7 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
   c->sa = StepArgs{rows, loss_dev, lr, n};
   const int rc = (graphs_enabled() && !g) ? step_graph(c, n) : enqueue_step(c, n);
   if (rc != ASGD_OK) return rc;
-  if (m.precision == ASGD_PREC_BF16) c->w2b_cur ^= 1;
+  c->w2b_cur ^= 1;   // G3 wrote the other shadow buffer
   ++c->u;
   return ASGD_OK;
 }
@@ -781,8 +780,7 @@ int asgd_merge_prescale(asgd_ctx* c, double alpha) {
 int asgd_merge_finish(asgd_ctx* c, float gamma) {
   if (!c) return fail(ASGD_E_ARG, "null ctx");
   PCU(ASGD_K_MERGE, launch_finish(c->lc(), c->params, c->w, c->dd, c->Pn, gamma));
-  if (c->d.precision == ASGD_PREC_BF16)
-    CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->w2b_buf[c->w2b_cur], c->d.L * c->d.H));
+  CU(refresh_shadow(c));
   c->u = 0;
   return ASGD_OK;
 }
@@ -906,8 +904,7 @@ int asgd_merge_fused(asgd_ctx* c, const double* alpha, float gamma) {
   PCU(ASGD_K_MERGE, launch_merge_fused(c->lc(), ps, c->w, c->dd, lo, hi, gamma,
                                        reinterpret_cast<unsigned int*>(c->P.meta + M_MDONE),
                                        reinterpret_cast<unsigned long long*>(c->P.meta + M_MSYNC), goal));
-  if (c->d.precision == ASGD_PREC_BF16)
-    CU(launch_to_bf16(c->lc(), c->params + c->o_w2, c->w2b_buf[c->w2b_cur], c->d.L * c->d.H));
+  CU(refresh_shadow(c));
   c->u = 0;
   return ASGD_OK;
 }
@@ -939,19 +936,11 @@ int asgd_eval_topk(asgd_ctx* c, const asgd_csr* t, const int32_t* rows, int32_t 
   float* b2 = c->params + c->o_b2;
   for (int32_t r0 = 0; r0 < n; r0 += m.b_max) {
     const int nb = std::min<int32_t>(m.b_max, n - r0);
-    CU(launch_spmm_fwd(lc, StepArgs{rows + r0, nullptr, 0.f, nb}, *t, W1, b1, H, P, c->L, bf));
-    if (!bf) {
-      GemmArgs a{};
-      a.M = nb; a.N = (int)m.L; a.K = H;
-      a.A = P.h1; a.as0 = H; a.as1 = 1;
-      a.B = W2; a.bs0 = 1; a.bs1 = H;
-      a.epi = EPI_STORE_BIAS; a.C = P.z; a.ldc = padded_ld(m.L); a.bias = b2; a.splitk = 1;
-      CU(launch_gemm_f32(lc, a));
-    } else {
-      Ptrs Pr = P;
-      Pr.w2b = c->w2b_buf[c->w2b_cur];
-      CU(launch_gemm_tc(lc, 1, nb, m.L, H, Pr, c->L, W2, b2, nullptr, nullptr));
-    }
+    CU(launch_spmm_fwd(lc, StepArgs{rows + r0, nullptr, 0.f, nb}, *t, W1, b1, H, P, c->L, true));
+    Ptrs Pr = P;   // Z = H1 W2^T + b2 on the tensor cores (bf16, or bf16x3 on the fp32 path)
+    Pr.w2b = c->w2b_buf[c->w2b_cur];
+    Pr.w2l = c->w2l_buf[c->w2b_cur];
+    CU(launch_gemm_tc(lc, 1, nb, m.L, H, Pr, c->L, W2, b2, nullptr, nullptr));
     CU(launch_topk(lc, nb, m.L, padded_ld(m.L), k, P.z, topk + (int64_t)r0 * k));
   }
   return ASGD_OK;
@@ -1318,8 +1307,9 @@ cudaError_t smem_attr_raw(const void* kernel, size_t bytes) {
 
 // Programmatic dependent launch: each kernel's prologue overlaps its predecessor's tail.
 // Measured (samples/s, PDL off -> on): bf16 EURLex 4.01 -> 4.22 M, AmazonCat 5.35 -> 5.46 M,
-// Wiki10 1.356 -> 1.383 M, Amazon-670K / Delicious-200K even; fp32 EURLex 1.52 -> 1.34 M.
-// ASGD_PDL: unset = on for bf16, off for fp32; 0 = off; 1 = every kernel; 2 = GEMMs only.
+// Wiki10 1.356 -> 1.383 M, Amazon-670K / Delicious-200K even.  (Round 1's fp32 path, SIMT
+// GEMMs, measured 1.52 -> 1.34 M with it; the fp32 path now runs the same tcgen05 DAG.)
+// ASGD_PDL: unset = on; 0 = off; 1 = every kernel; 2 = GEMMs only.
 int pdl_mode() {
   static const int m = [] {
     const char* v = getenv("ASGD_PDL");
@@ -1327,5 +1317,5 @@ int pdl_mode() {
   }();
   return m;
 }
-bool pdl_for(bool bf16) { return pdl_mode() < 0 ? bf16 : pdl_mode() == 1; }
+bool pdl_for(bool) { return pdl_mode() < 0 ? true : pdl_mode() == 1; }
 }  // namespace asgd

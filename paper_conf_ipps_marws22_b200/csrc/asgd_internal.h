@@ -32,8 +32,10 @@ typedef __nv_bfloat16 bf16;
 struct WsLayout {
   size_t meta, boff, loff, cnt, fseg, fuid, uniq, useg, tsum, tpre;
   size_t e_n, e_v, e_u, e_f, part1, rowcnt, part5, ucnt, bits;
-  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, b2part, rbase, da1b, zstat, lse;
+  size_t h1, h1b, z, dzb, rowloss, dhpart, da1, db1part, w2b, w2b2, red, eval_top, rbase, da1b, zstat, lse;
   size_t rowsc, cen, cenpart;
+  size_t h1l, dzl, w2l, w2l2;   // bf16x3 lo halves (fp32 path, R14)
+  bool x3;                      // fp32 path: GEMM operands split hi + lo (R14)
   size_t total;
   int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride, stats_ld;
 };
@@ -45,20 +47,22 @@ struct Ptrs {  // typed views of the workspace
   int32_t* uniq; int32_t* useg; int32_t* tsum; int32_t* tpre;
   int32_t* e_n; float* e_v; int32_t* e_u; int32_t* e_f; uint32_t* bits; float* part1; int32_t* rowcnt; float* part5;
   int32_t* ucnt; float* h1; bf16* h1b; float* z; bf16* dzb; float* rowloss; float* dhpart;
-  float* da1; float* db1part; bf16* w2b; double* red; int32_t* eval_top; float* b2part;
+  float* da1; float* db1part; bf16* w2b; double* red; int32_t* eval_top;
   int64_t* rbase;   // row_ptr[rows[r]] of the current batch (written by K-0 (a))
   bf16* da1b;       // bf16 copy of dA1 (bf16 path; staged by K-5)
   float* lse;       // per-row log-sum-exp of Z (bf16 path)
   int32_t* rowsc;   // copy of the step's dataset row ids (written by K-0 (a))
   float* cen;       // centred sigmoid offsets [2 H] (bf16 path, R11)
   float* cenpart;   // their per-CTA partials [kCenterParts H]
+  // fp32 path (R14): the bf16x3 lo halves of H1, dZ and the W2 shadow (h1b / dzb / w2b are
+  // the hi halves); null on the bf16 path
+  bf16* h1l; bf16* dzl; bf16* w2l;
 };
 __device__ __forceinline__ float step_lr(const int32_t* meta) { return __int_as_float(meta[M_LR]); }
 __device__ __forceinline__ float* step_loss(const int32_t* meta) {
   return *reinterpret_cast<float* const*>(meta + M_LOSS);
 }
 int row_block();   // rows per db1 partial (kernels_dense.cu)
-int b2_chunks();   // row chunks of the db2 partial sums
 Ptrs ws_ptrs(char* base, const WsLayout& L);
 
 struct Launch {       // launch bookkeeping of one ctx
@@ -80,6 +84,13 @@ __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;"
 // tcgen05 GEMMs only
 int pdl_mode();
 bool pdl_for(bool bf16);   // launch_k: this ctx's kernels use PDL
+
+// fp32 path on the tensor cores ("bf16x3", R14): x = hi + lo with hi = bf16(x)
+// and lo = bf16(x - hi) (x - hi is exact in fp32); a product x y is taken as
+// hi_x hi_y + hi_x lo_y + lo_x hi_y in three bf16 MMAs with fp32 accumulation.
+__device__ __forceinline__ float bf16_lo_of(float x) {
+  return x - __bfloat162float(__float2bfloat16_rn(x));
+}
 
 // cudaFuncSetAttribute(MaxDynamicSharedMemorySize) is a per-device setting: it is
 // applied once per (kernel, current device) and raised when a larger size is needed.
@@ -153,21 +164,7 @@ int touched_nargs();
 // The learning rate of every SGD update is the step's meta[M_LR].
 cudaError_t launch_scatter_sgd(const Launch&, float* W1, int H, const Ptrs&,
                                const WsLayout&, float* grad_w1, const bf16* dA1b, int b_max);
-// ---------------------------------------------------------------- dense (fp32 SIMT)
-// C(m,n) = sum_k A(m,k) B(k,n), A(m,k) = A[m*as0 + k*as1], B(k,n) = B[k*bs0 + n*bs1]
-enum GemmEpi { EPI_STORE_BIAS = 0, EPI_SPLITK = 1, EPI_SGD = 2 };
-struct GemmArgs {
-  int M, N, K;
-  const float* A; int64_t as0, as1;
-  const float* B; int64_t bs0, bs1;
-  int epi;
-  float* C; int64_t ldc;          // STORE_BIAS: C[m*ldc+n] = acc + bias[n]
-  const float* bias;
-  int splitk; int64_t part_stride; // SPLITK: C[z*part_stride + m*ldc + n]
-  const int32_t* meta; float* grad; // SGD: C[m*ldc+n] -= lr*acc (lr = meta[M_LR]); grad[m*ldc+n] = acc
-  bf16* shadow;                    // SGD: shadow[m*ldc+n] = bf16(new C)
-};
-cudaError_t launch_gemm_f32(const Launch&, const GemmArgs&);
+// ---------------------------------------------------------------- dense (CUDA cores)
 // Leading dimension of the B x L logit buffers (16-byte rows for TMA).
 int64_t padded_ld(int64_t L);
 // stats (nullable): G1's per (N tile, row) (max, sum exp) partials -> one pass over Z.
@@ -184,14 +181,14 @@ cudaError_t launch_dh_reduce(const Launch&, int n, int H, int splitk, const Ptrs
                              bool want_bf16, const float* dh_off = nullptr);
 // Centred sigmoid dZ (R11): cen[0:H] = (1/(2B)) sum_j W2_j (bf16 shadow, the dH1 offset),
 // cen[H:2H] = (1/(2B)) sum_n H1_n (the dW2 offset).  part: fp32[2 parts H]; counter: zeroed.
-cudaError_t launch_sig_center(const Launch&, const bf16* w2b, int64_t L, int H, const float* h1, int n, float* part,
-                              unsigned int* counter, float* cen);
+// w2f (nullable): sum the fp32 W2 instead (bf16x3 fp32 path, R14).
+cudaError_t launch_sig_center(const Launch&, const bf16* w2b, const float* w2f, int64_t L, int H, const float* h1,
+                              int n, float* part, unsigned int* counter, float* cen);
 constexpr int kCenterParts = 148;
 cudaError_t launch_b1_update(const Launch&, int n, int H, float* b1, const Ptrs&,
                              const WsLayout&, float* grad_b1);
-cudaError_t launch_b2_update(const Launch&, int n, int64_t L, int64_t ldz, float* b2,
-                             const Ptrs&, bool from_bf16, float* grad_b2);
-cudaError_t launch_to_bf16(const Launch&, const float* src, bf16* dst, int64_t count);
+// dst_lo (nullable): also the bf16x3 lo half bf16(x - bf16(x)) (R14)
+cudaError_t launch_to_bf16(const Launch&, const float* src, bf16* dst, int64_t count, bf16* dst_lo = nullptr);
 // ---------------------------------------------------------------- tcgen05 (bf16)
 bool tc_available();
 // which: 1 = G1 (Z = H1 W2^T + b2), 2 = G2 (dH1 split-K partials), 3 = G3 (W2 -= lr dZ^T H1 and

@@ -1,13 +1,11 @@
-// Dense kernels of the local step (sm_100a), fp32 path and shared epilogues:
-//   G1  Z = H1 W2^T + b2                     (row a4)
-//   softmax-CE: lse, loss, dZ = (softmax(Z) - T)/B   (row a5)
-//   G2  dH1 = dZ W2 (split-K partials), dA1 = dH1 * [A1 > 0], b1 update (rows a6, a7)
-//   G3  W2 -= lr dZ^T H1 (SGD fused into the GEMM epilogue), b2 -= lr 1^T dZ (row a6)
+// Dense element-wise / reduction kernels of the local step (sm_100a) around the
+// tcgen05 GEMMs G1-G3 of kernels_tc.cu:
+//   softmax-CE: lse, loss, dZ = (softmax(Z) - T)/B   (row a5; sigmoid-BCE, R11)
+//   dA1 = dH1 * [A1 > 0] from G2's split-K partials, b1 update (rows a6, a7)
+//   merge-side helpers: the bf16 W2 shadow (and its bf16x3 lo half, R14)
 // Model: PAPER.md P:1525-1531 (§V-A); SGD: P:437-455 (§II); fused element-wise
-// work follows the paper's kernel fusion (§IV).
-// The fp32 contractions here run on CUDA cores (FFMA) so that the fp32 path
-// keeps fp32 products (tolerance 1e-4 vs the fp64 oracle); the bf16 path runs
-// G1-G3 on tcgen05 tensor cores (kernels_tc.cu).
+// work follows the paper's kernel fusion (§IV).  Both precisions run
+// the contractions on the tensor cores; the fp32 path as bf16x3 (R14).
 #include <algorithm>
 
 #include "asgd_internal.h"
@@ -17,78 +15,6 @@ namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
 
-// ----------------------------------------------------------------- SIMT GEMM
-constexpr int BM = 64, BN = 64, BK = 16;
-
-__global__ void __launch_bounds__(256) k_gemm_f32(GemmArgs g) {
-  pdl_trigger();
-  pdl_wait();
-  __shared__ float As[BK][BM + 4];
-  __shared__ float Bs[BK][BN + 4];
-  const int t = threadIdx.x, tx = t & 15, ty = t >> 4;
-  const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
-  // split-K range
-  int kc = (g.K + g.splitk - 1) / g.splitk;
-  kc = (kc + BK - 1) / BK * BK;
-  const int kb = blockIdx.z * kc, ke = min(g.K, kb + kc);
-  float acc[4][4];
-#pragma unroll
-  for (int i = 0; i < 4; ++i)
-#pragma unroll
-    for (int j = 0; j < 4; ++j) acc[i][j] = 0.f;
-  const bool a_kcontig = (g.as1 == 1);
-  const bool b_ncontig = (g.bs1 == 1);
-  for (int k0 = kb; k0 < ke; k0 += BK) {
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int i = t + 256 * q;
-      int m, k;
-      if (a_kcontig) { k = i & 15; m = i >> 4; } else { m = i & 63; k = i >> 6; }
-      const int gm = m0 + m, gk = k0 + k;
-      As[k][m] = (gm < g.M && gk < ke) ? g.A[(int64_t)gm * g.as0 + (int64_t)gk * g.as1] : 0.f;
-      int n, kk;
-      if (b_ncontig) { n = i & 63; kk = i >> 6; } else { kk = i & 15; n = i >> 4; }
-      const int gn = n0 + n, gk2 = k0 + kk;
-      Bs[kk][n] = (gn < g.N && gk2 < ke) ? g.B[(int64_t)gk2 * g.bs0 + (int64_t)gn * g.bs1] : 0.f;
-    }
-    __syncthreads();
-#pragma unroll
-    for (int k = 0; k < BK; ++k) {
-      float a[4], b[4];
-#pragma unroll
-      for (int i = 0; i < 4; ++i) a[i] = As[k][ty + 16 * i];
-#pragma unroll
-      for (int j = 0; j < 4; ++j) b[j] = Bs[k][tx + 16 * j];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
-    }
-    __syncthreads();
-  }
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const int m = m0 + ty + 16 * i;
-    if (m >= g.M) continue;
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int n = n0 + tx + 16 * j;
-      if (n >= g.N) continue;
-      const int64_t o = (int64_t)m * g.ldc + n;
-      if (g.epi == EPI_STORE_BIAS) {
-        g.C[o] = acc[i][j] + (g.bias ? g.bias[n] : 0.f);
-      } else if (g.epi == EPI_SPLITK) {
-        g.C[(int64_t)blockIdx.z * g.part_stride + o] = acc[i][j];
-      } else {  // EPI_SGD
-        const float nw = g.C[o] - step_lr(g.meta) * acc[i][j];
-        g.C[o] = nw;
-        if (g.grad) g.grad[o] = acc[i][j];
-        if (g.shadow) g.shadow[o] = __float2bfloat16_rn(nw);
-      }
-    }
-  }
-}
-
 // ------------------------------------------------------------ softmax + CE
 // One CTA per batch row n: lse = log sum_j exp(Z_nj); loss_n = lse - mean_{y in Y_n} Z_ny;
 // dZ_nj = (exp(Z_nj - lse) - T_nj) / B with T_nj = 1/|Y_n| on Y_n (Q3, Q4).
@@ -96,7 +22,7 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
                                                     const int32_t* __restrict__ rows,
                                                     const int64_t* __restrict__ lab_ptr,
                                                     const int32_t* __restrict__ lab, float* Z,
-                                                    bf16* dZb, float* rowloss,
+                                                    bf16* dZb, bf16* dZl, float* rowloss,
                                                     const float2* __restrict__ stats, int ntiles,
                                                     int64_t stats_ld) {
   pdl_trigger();
@@ -168,8 +94,9 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
   }
   __syncthreads();
   const float lse = s_lse, invB = 1.f / (float)B;
-  if (dZb) {
+  if (dZb) {   // bf16 dZ, with dZl its bf16x3 lo half (fp32 path, R14)
     bf16* d = dZb + (int64_t)n * ldz;
+    bf16* dl = dZl ? dZl + (int64_t)n * ldz : nullptr;
     for (int64_t j0 = threadIdx.x; j0 < L; j0 += (int64_t)kSU * blockDim.x) {
       float v[kSU];
 #pragma unroll
@@ -180,12 +107,19 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
 #pragma unroll
       for (int k = 0; k < kSU; ++k) {
         const int64_t j = j0 + (int64_t)k * blockDim.x;
-        if (j < L) d[j] = __float2bfloat16_rn(__expf(v[k] - lse) * invB);
+        if (j < L) {
+          const float g = __expf(v[k] - lse) * invB;
+          d[j] = __float2bfloat16_rn(g);
+          if (dl) dl[j] = __float2bfloat16_rn(bf16_lo_of(g));
+        }
       }
     }
     __syncthreads();
-    for (int i = threadIdx.x; i < nl; i += blockDim.x)
-      d[s_lab[i]] = __float2bfloat16_rn((__expf(s_lz[i] - lse) - 1.f / (float)nl) * invB);
+    for (int i = threadIdx.x; i < nl; i += blockDim.x) {
+      const float g = (__expf(s_lz[i] - lse) - 1.f / (float)nl) * invB;
+      d[s_lab[i]] = __float2bfloat16_rn(g);
+      if (dl) dl[s_lab[i]] = __float2bfloat16_rn(bf16_lo_of(g));
+    }
   } else {
     for (int64_t j0 = threadIdx.x; j0 < L; j0 += (int64_t)kSU * blockDim.x) {
       float v[kSU];
@@ -215,17 +149,27 @@ __device__ __forceinline__ float sigmoid_f(float z) {
   const float e = expf(-fabsf(z));
   return z >= 0.f ? 1.f / (1.f + e) : e / (1.f + e);
 }
+// sigmoid(z) - 1/2 without cancellation: (1 - e) / (2 (1 + e)), e = exp(-|z|), sign of z
+__device__ __forceinline__ float sigmoid_c(float z) {
+  const float e = expf(-fabsf(z));
+  const float c = 0.5f * (1.f - e) / (1.f + e);
+  return z >= 0.f ? c : -c;
+}
 
 __global__ void __launch_bounds__(512) k_sigmoid_ce(int B, int64_t L, int64_t ldz,
                                                     const int32_t* __restrict__ rows,
                                                     const int64_t* __restrict__ lab_ptr,
                                                     const int32_t* __restrict__ lab, float* Z,
-                                                    bf16* dZb, float* rowloss) {
+                                                    bf16* dZb, bf16* dZl, float* rowloss) {
   pdl_trigger();
   pdl_wait();
   __shared__ int s_lab[kMaxRowLabels];
   __shared__ float s_lz[kMaxRowLabels];
   __shared__ float s_sp[16];
+  // dZl (bf16x3 fp32 path, R14): dZ is stored CENTRED as hi + lo of (sigmoid(Z) - 1/2 - Y) / B,
+  // as on the bf16 path (R11): the z-dependent part of sigmoid near 1/2 would otherwise sit
+  // below the split's 2^-17 relative precision; the offsets come back through k_sig_center
+  const bool centred = dZl != nullptr;
   const int n = blockIdx.x;
   const int64_t id = rows[n];
   const int64_t l0 = lab_ptr[id];
@@ -254,8 +198,14 @@ __global__ void __launch_bounds__(512) k_sigmoid_ce(int B, int64_t L, int64_t ld
       const int64_t j = j0 + (int64_t)k * blockDim.x;
       if (j < L) {
         sp += softplus_f(v[k]);
-        const float g = sigmoid_f(v[k]) * invB;
-        if (d) d[j] = __float2bfloat16_rn(g); else z[j] = g;
+        if (centred) {
+          const float g = sigmoid_c(v[k]) * invB;
+          d[j] = __float2bfloat16_rn(g);
+          dZl[(int64_t)n * ldz + j] = __float2bfloat16_rn(bf16_lo_of(g));
+        } else {
+          const float g = sigmoid_f(v[k]) * invB;
+          if (d) d[j] = __float2bfloat16_rn(g); else z[j] = g;
+        }
       }
     }
   }
@@ -270,9 +220,16 @@ __global__ void __launch_bounds__(512) k_sigmoid_ce(int B, int64_t L, int64_t ld
     for (int i = 0; i < nl; ++i) ls += s_lz[i];
     rowloss[n] = S - ls;
   }
+  __syncthreads();   // the label columns' non-label values are written before they are replaced
   for (int i = threadIdx.x; i < nl; i += blockDim.x) {
-    const float g = (sigmoid_f(s_lz[i]) - 1.f) * invB;
-    if (d) d[s_lab[i]] = __float2bfloat16_rn(g); else z[s_lab[i]] = g;
+    if (centred) {
+      const float g = (sigmoid_c(s_lz[i]) - 1.f) * invB;
+      d[s_lab[i]] = __float2bfloat16_rn(g);
+      dZl[(int64_t)n * ldz + s_lab[i]] = __float2bfloat16_rn(bf16_lo_of(g));
+    } else {
+      const float g = (sigmoid_f(s_lz[i]) - 1.f) * invB;
+      if (d) d[s_lab[i]] = __float2bfloat16_rn(g); else z[s_lab[i]] = g;
+    }
   }
 }
 
@@ -305,9 +262,9 @@ __global__ void __launch_bounds__(256) k_tile_loss(int ntiles, int64_t stats_ld,
 // (db2's + 1/2 is G3's).  W2 is the bf16 shadow G2 multiplies with.  Phase 1: each
 // CTA sums a contiguous label range (8 columns per thread, 16-B loads, 4 in
 // flight); phase 2: the last CTA adds the partials in CTA order (deterministic).
-__global__ void __launch_bounds__(256) k_sig_center(const bf16* __restrict__ w2b, int64_t L, int H,
-                                                    const float* __restrict__ h1, int n, float* part,
-                                                    unsigned int* counter, float* cen) {
+__global__ void __launch_bounds__(256) k_sig_center(const bf16* __restrict__ w2b, const float* __restrict__ w2f,
+                                                    int64_t L, int H, const float* __restrict__ h1, int n,
+                                                    float* part, unsigned int* counter, float* cen) {
   pdl_trigger();
   pdl_wait();
   __shared__ float s_acc[8][512];
@@ -318,6 +275,14 @@ __global__ void __launch_bounds__(256) k_sig_center(const bf16* __restrict__ w2b
   const int64_t j0 = (int64_t)blockIdx.x * L / gridDim.x, j1 = (int64_t)(blockIdx.x + 1) * L / gridDim.x;
   float a[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
   int64_t j = j0 + r0;
+  if (w2f) {   // bf16x3 fp32 path (R14): the offset from the fp32 W2
+    for (; j < j1; j += rows_per_it) {
+      const float4 u0 = __ldcs(reinterpret_cast<const float4*>(w2f + j * H + c8));
+      const float4 u1 = __ldcs(reinterpret_cast<const float4*>(w2f + j * H + c8 + 4));
+      a[0] += u0.x; a[1] += u0.y; a[2] += u0.z; a[3] += u0.w;
+      a[4] += u1.x; a[5] += u1.y; a[6] += u1.z; a[7] += u1.w;
+    }
+  }
   for (; j + 3 * rows_per_it < j1; j += 4 * rows_per_it) {
     uint4 u[4];
 #pragma unroll
@@ -498,77 +463,31 @@ __global__ void __launch_bounds__(256) k_b1_update(int n, int H, const float* __
   }
 }
 
-// db2 partials: b2part[y][j] = sum over row chunk y of dZ[r][j]
-constexpr int kB2Chunks = 16;
-__global__ void __launch_bounds__(256) k_b2_part(int n, int64_t L, int64_t ldz, const float* __restrict__ dz,
-                                                 const bf16* __restrict__ dzb, float* b2part) {
-  pdl_trigger();
-  pdl_wait();
-  const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (j >= L) return;
-  const int per = (n + gridDim.y - 1) / gridDim.y;
-  const int r0 = blockIdx.y * per, r1 = min(n, r0 + per);
-  float s0 = 0.f, s1 = 0.f;
-  int r = r0;
-  if (dzb) {
-    for (; r + 2 <= r1; r += 2) {
-      s0 += __bfloat162float(dzb[(int64_t)r * ldz + j]);
-      s1 += __bfloat162float(dzb[(int64_t)(r + 1) * ldz + j]);
-    }
-    for (; r < r1; ++r) s0 += __bfloat162float(dzb[(int64_t)r * ldz + j]);
-  } else {
-    for (; r + 2 <= r1; r += 2) {
-      s0 += dz[(int64_t)r * ldz + j];
-      s1 += dz[(int64_t)(r + 1) * ldz + j];
-    }
-    for (; r < r1; ++r) s0 += dz[(int64_t)r * ldz + j];
-  }
-  b2part[(int64_t)blockIdx.y * L + j] = s0 + s1;
-}
-
-// b2 -= lr * sum_y b2part[y]
-__global__ void __launch_bounds__(256) k_b2_apply(int64_t L, int chunks, const float* __restrict__ b2part,
-                                                  float* b2, const int32_t* __restrict__ meta, float* grad_b2) {
-  pdl_trigger();
-  pdl_wait();
-  const float lr = step_lr(meta);
-  const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (j >= L) return;
-  float s = 0.f;
-  for (int y = 0; y < chunks; ++y) s += b2part[(int64_t)y * L + j];
-  b2[j] -= lr * s;
-  if (grad_b2) grad_b2[j] = s;
-}
-
-__global__ void k_to_bf16(const float* __restrict__ src, bf16* dst, int64_t count) {
+__global__ void k_to_bf16(const float* __restrict__ src, bf16* dst, bf16* dst_lo, int64_t count) {
   pdl_trigger();
   pdl_wait();
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count;
-       i += (int64_t)gridDim.x * blockDim.x)
-    dst[i] = __float2bfloat16_rn(src[i]);
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const float x = src[i];
+    dst[i] = __float2bfloat16_rn(x);
+    if (dst_lo) dst_lo[i] = __float2bfloat16_rn(bf16_lo_of(x));
+  }
 }
 
 }  // namespace
-
-cudaError_t launch_gemm_f32(const Launch& lc, const GemmArgs& g) {
-  if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaSuccess;
-  dim3 grid((g.N + BN - 1) / BN, (g.M + BM - 1) / BM, g.splitk);
-  launch_k(lc, k_gemm_f32, dim3(grid), dim3(256), 0, g);
-  return cudaGetLastError();
-}
 
 cudaError_t launch_softmax_ce(const Launch& lc, int n, int64_t L, int64_t ldz, const int32_t* rows,
                               const int64_t* lab_ptr, const int32_t* lab, const Ptrs& P,
                               bool bf16_out, const float2* stats, int ntiles, int64_t stats_ld) {
   launch_k(lc, k_softmax_ce, dim3(n), dim3(512), 0, n, L, ldz, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
-                                    P.rowloss, stats, ntiles, stats_ld);
+           bf16_out ? P.dzl : nullptr, P.rowloss, stats, ntiles, stats_ld);
   return cudaGetLastError();
 }
 
 cudaError_t launch_sigmoid_ce(const Launch& lc, int n, int64_t L, int64_t ldz, const int32_t* rows,
                               const int64_t* lab_ptr, const int32_t* lab, const Ptrs& P, bool bf16_out) {
   launch_k(lc, k_sigmoid_ce, dim3(n), dim3(512), 0, n, L, ldz, rows, lab_ptr, lab, P.z, bf16_out ? P.dzb : nullptr,
-           P.rowloss);
+           bf16_out ? P.dzl : nullptr, P.rowloss);
   return cudaGetLastError();
 }
 
@@ -576,9 +495,9 @@ cudaError_t launch_tile_loss(const Launch& lc, int n, int ntiles, int64_t stats_
   return launch_k(lc, k_tile_loss, dim3(n), dim3(256), 0, ntiles, stats_ld, stats, P.rowloss);
 }
 
-cudaError_t launch_sig_center(const Launch& lc, const bf16* w2b, int64_t L, int H, const float* h1, int n, float* part,
-                              unsigned int* counter, float* cen) {
-  return launch_k(lc, k_sig_center, dim3(kCenterParts), dim3(256), 0, w2b, L, H, h1, n, part, counter, cen);
+cudaError_t launch_sig_center(const Launch& lc, const bf16* w2b, const float* w2f, int64_t L, int H, const float* h1,
+                              int n, float* part, unsigned int* counter, float* cen) {
+  return launch_k(lc, k_sig_center, dim3(kCenterParts), dim3(256), 0, w2b, w2f, L, H, h1, n, part, counter, cen);
 }
 
 cudaError_t launch_lse(const Launch& lc, int n, int H, int ntiles, int64_t stats_ld, const float2* stats,
@@ -602,22 +521,12 @@ cudaError_t launch_b1_update(const Launch& lc, int n, int H, float* b1, const Pt
   return cudaGetLastError();
 }
 
-cudaError_t launch_b2_update(const Launch& lc, int n, int64_t L, int64_t ldz, float* b2,
-                             const Ptrs& P, bool from_bf16, float* grad_b2) {
-  const int chunks = std::max(1, std::min(kB2Chunks, n / 16));
-  dim3 grid((unsigned)((L + 255) / 256), (unsigned)chunks);
-  launch_k(lc, k_b2_part, dim3(grid), dim3(256), 0, n, L, ldz, P.z, from_bf16 ? P.dzb : nullptr, P.b2part);
-  launch_k(lc, k_b2_apply, dim3((unsigned)((L + 255) / 256)), dim3(256), 0, L, chunks, P.b2part, b2, P.meta, grad_b2);
-  return cudaGetLastError();
-}
-
-cudaError_t launch_to_bf16(const Launch& lc, const float* src, bf16* dst, int64_t count) {
+cudaError_t launch_to_bf16(const Launch& lc, const float* src, bf16* dst, int64_t count, bf16* dst_lo) {
   const int64_t blocks = std::min<int64_t>((count + 255) / 256, (int64_t)lc.sms * 16);
-  launch_k(lc, k_to_bf16, dim3((int)std::max<int64_t>(blocks, 1)), dim3(256), 0, src, dst, count);
+  launch_k(lc, k_to_bf16, dim3((int)std::max<int64_t>(blocks, 1)), dim3(256), 0, src, dst, dst_lo, count);
   return cudaGetLastError();
 }
 
 int row_block() { return 1; }
-int b2_chunks() { return kB2Chunks; }
 
 }  // namespace asgd

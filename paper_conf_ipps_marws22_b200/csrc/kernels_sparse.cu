@@ -96,6 +96,13 @@ struct RowIO {
                make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]));
     }
   }
+  // the lo half of the bf16x3 split (R14): bf16(v - bf16(v))
+  __device__ __forceinline__ static void store_bf16_lo(bf16* row, int lane, const float (&v)[VPL]) {
+    float r[VPL];
+#pragma unroll
+    for (int i = 0; i < VPL; ++i) r[i] = bf16_lo_of(v[i]);
+    store_bf16(row, lane, r);
+  }
   __device__ __forceinline__ static void store_bf16(bf16* row, int lane, const float (&v)[VPL]) {
     if constexpr (VPL == 2) {
       reinterpret_cast<__nv_bfloat162*>(row)[lane] = __floats2bfloat162_rn(v[0], v[1]);
@@ -397,7 +404,7 @@ __global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_
                                                   const float* __restrict__ val,
                                                   const float* __restrict__ W1,
                                                   const float* __restrict__ b1, float* H1,
-                                                  bf16* H1b, float* part, int32_t* rowcnt) {
+                                                  bf16* H1b, bf16* H1l, float* part, int32_t* rowcnt) {
   pdl_trigger();
   pdl_wait();
   using IO = RowIO<VPL>;
@@ -425,6 +432,7 @@ __global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_
     for (int i = 0; i < VPL; ++i) acc[i] = fmaxf(acc[i] + bias[i], 0.f);
     IO::store(H1 + (int64_t)r * H, lane, acc);
     if (H1b) IO::store_bf16(H1b + (int64_t)r * H, lane, acc);
+    if (H1l) IO::store_bf16_lo(H1l + (int64_t)r * H, lane, acc);
   };
   // group g's partial of row r (global): slot 2 g + 1 if r starts in g, else 2 g; the
   // last group to arrive sums the row's group partials in group order and finishes
@@ -943,7 +951,8 @@ cudaError_t spmm_fwd_t(const Launch& lc, const StepArgs& sa, const asgd_csr& x, 
   const int grid = wave_grid(lc, k_spmm_fwd<VPL>, view_smem(2048), L.n_pieces, occ, k1_group<VPL>());
   const ViewOut vo{P.boff, P.loff, P.rbase, P.rowsc, P.meta};
   launch_k(lc, k_spmm_fwd<VPL>, dim3(grid), dim3(32 * k1_group<VPL>()), smem, sa, x.row_ptr, x.lab_ptr, x.n_rows, L.nz_cap, L.nl_cap,
-           vo, x.col, x.val, W1, b1, P.h1, want_bf16 ? P.h1b : nullptr, P.part1, P.rowcnt);
+           vo, x.col, x.val, W1, b1, P.h1, want_bf16 ? P.h1b : nullptr, want_bf16 ? P.h1l : nullptr, P.part1,
+           P.rowcnt);
   return cudaGetLastError();
 }
 
@@ -974,6 +983,16 @@ cudaError_t launch_touched(const Launch& lc, const StepArgs& sa, const asgd_csr&
     cudaError_t e = ensure_smem(k_touched, smem_all);
     if (e != cudaSuccess) return e;
   }
+  // K-0's two software grid barriers need every CTA resident at once: at most one CTA per
+  // SM, and the kernel alone must fit ctas CTAs (asserted here instead of a cooperative
+  // launch, which graphs with programmatic dependent launch do not capture; the kernels
+  // beside it on other streams never wait for K-0, so its CTAs always get their SMs)
+  int occ = 0;
+  {
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_touched, 512, smem_all);
+    if (e != cudaSuccess) return e;
+  }
+  if ((int64_t)occ * lc.sms < ctas) return cudaErrorCooperativeLaunchTooLarge;
   return launch_k(lc, k_touched, dim3(ctas), dim3(512), smem_all, sa, x.row_ptr, x.n_rows, L.nz_cap, x.col, x.val,
                   P.meta, P.cnt, P.tsum, F, nt, P.fseg, P.fuid, P.uniq, P.useg, P.bits, W, P.e_n,
                   P.e_v, P.e_u, P.e_f);

@@ -33,6 +33,7 @@ struct TcArgs {
   int64_t part_stride;                // split-K partial z offset
   const float* bias;                  // G1
   const int32_t* meta; bf16* shadow; float* grad;// G3 (lr = meta[M_LR])
+  bf16* shadow_lo;                    // G3, bf16x3 (R14): the lo half of the new W2 shadow
   float* b2; float* grad_b2;          // G3: db2 = dZ^T 1 via an extra N = 16 MMA on N-tile 0
   float2* stats; int64_t stats_ld;    // G1: per (N-tile half, row) softmax partials (max, sum exp)
   int splits;                         // split-K factor (tiles = M tiles x N tiles x splits)
@@ -243,9 +244,10 @@ template <int BN, int EPI>
 constexpr int epi_warps() {
   return (BN >= 128 && (EPI == TC_EPI_DZ || EPI == TC_EPI_SIG || EPI == TC_EPI_STATS)) ? 16 : 8;
 }
-template <int EPI>
+template <int EPI, bool X3 = false>
 constexpr int stages_of() {   // G3 streams dZ^T from HBM: the deepest ring (its epilogue needs no smem)
-  return EPI == TC_EPI_SGD ? 5 : (EPI == TC_EPI_STATS ? 4 : (EPI == TC_EPI_Z ? 2 : 3));
+  // bf16x3 (R14): every stage holds hi and lo tiles of both operands, 2 stages fit
+  return X3 ? 2 : (EPI == TC_EPI_SGD ? 5 : (EPI == TC_EPI_STATS ? 4 : (EPI == TC_EPI_Z ? 2 : 3)));
 }
 template <int EPI>
 constexpr uint32_t box_bytes() {   // one 32 x 32 store box: fp32 (Z, PART) or bf16 (DZ, SIG)
@@ -276,14 +278,21 @@ constexpr uint32_t staging_bytes() {   // per epilogue warp: store boxes / G3 tr
                                                         box_bytes<EPI>());
 }
 
-template <int BN, bool A_MN, bool B_MN, int EPI>
+// X3 (fp32 path, R14): both operands come as bf16 hi + lo halves (tmA2 / tmB2 map the lo
+// halves, loaded into the same stage right after the hi tiles) and every K step issues
+// three MMAs, hi.hi + hi.lo + lo.hi, into the same fp32 accumulator.
+template <int BN, bool A_MN, bool B_MN, int EPI, bool X3>
 __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
     k_gemm_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-              const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmD, TcArgs g) {
-  constexpr int STAGES = stages_of<EPI>();
+              const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmD,
+              const __grid_constant__ CUtensorMap tmA2, const __grid_constant__ CUtensorMap tmB2, TcArgs g) {
+  constexpr int STAGES = stages_of<EPI, X3>();
   constexpr bool ARES = a_resident<EPI, A_MN>();
-  constexpr uint32_t A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2;
-  constexpr uint32_t STAGE = (ARES ? 0u : A_BYTES) + B_BYTES;
+  static_assert(!(X3 && ARES), "bf16x3 GEMMs stream A");
+  constexpr uint32_t XF = X3 ? 2u : 1u;
+  constexpr uint32_t A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2;   // one half (hi or lo)
+  constexpr uint32_t A_SLOT = A_BYTES * XF, B_SLOT = B_BYTES * XF;
+  constexpr uint32_t STAGE = (ARES ? 0u : A_SLOT) + B_SLOT;
   constexpr uint32_t ARES_BYTES = ARES ? (uint32_t)(kAresK / BK) * A_BYTES : 0u;
   constexpr int NSTG = store_bufs<EPI, A_MN>();
   constexpr bool ONES = (EPI == TC_EPI_SGD);           // db2 column block after the accumulator
@@ -301,7 +310,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
   // address space (LDS/STS instead of generic LD/ST in the epilogues)
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sA = smem;                                          // ring A stages, or the resident A block
-  uint8_t* sB = smem + (ARES ? ARES_BYTES : STAGES * A_BYTES);
+  uint8_t* sB = smem + (ARES ? ARES_BYTES : STAGES * A_SLOT);
   uint8_t* sOnes = smem + ARES_BYTES + STAGES * STAGE;
   uint8_t* sStg = sOnes + ONES_BYTES;   // TMA-store staging (1024-aligned)
   float* sBias = reinterpret_cast<float*>(sStg + staging_bytes<BN, EPI, A_MN>());
@@ -332,6 +341,10 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
+    if constexpr (X3) {
+      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA2)) : "memory");
+      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmB2)) : "memory");
+    }
     for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
     for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], EPI_WARPS); }
     mbar_init(afull, 1);
@@ -378,20 +391,27 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
           mbar_wait(&empty[s], ph ^ 1);
           mbar_expect_tx(&full[s], STAGE);
           const int kc = (kb0 + i) * BK;
-          uint8_t* a = sA + s * A_BYTES;
-          uint8_t* b = sB + s * B_BYTES;
-          if constexpr (ARES) {
-          } else if constexpr (!A_MN) {
-            tma_load_2d(a, &tmA, &full[s], kc, m0);
-          } else {
-            tma_load_2d(a, &tmA, &full[s], m0, kc);
-            tma_load_2d(a + 8192, &tmA, &full[s], m0 + 64, kc);
-          }
-          if constexpr (!B_MN) {
-            tma_load_2d(b, &tmB, &full[s], kc, n0);
-          } else {
+          uint8_t* a = sA + s * A_SLOT;
+          uint8_t* b = sB + s * B_SLOT;
 #pragma unroll
-            for (int j = 0; j < BN / 64; ++j) tma_load_2d(b + j * 8192, &tmB, &full[s], n0 + 64 * j, kc);
+          for (int h = 0; h < (int)XF; ++h) {   // h = 1: the lo halves (bf16x3)
+            const CUtensorMap* ma = h ? &tmA2 : &tmA;
+            const CUtensorMap* mb = h ? &tmB2 : &tmB;
+            uint8_t* ah = a + h * A_BYTES;
+            uint8_t* bh = b + h * B_BYTES;
+            if constexpr (ARES) {
+            } else if constexpr (!A_MN) {
+              tma_load_2d(ah, ma, &full[s], kc, m0);
+            } else {
+              tma_load_2d(ah, ma, &full[s], m0, kc);
+              tma_load_2d(ah + 8192, ma, &full[s], m0 + 64, kc);
+            }
+            if constexpr (!B_MN) {
+              tma_load_2d(bh, mb, &full[s], kc, n0);
+            } else {
+#pragma unroll
+              for (int j = 0; j < BN / 64; ++j) tma_load_2d(bh + j * 8192, mb, &full[s], n0 + 64 * j, kc);
+            }
           }
         }
       }
@@ -420,16 +440,30 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
           const uint32_t ph = (it / STAGES) & 1;
           mbar_wait(&full[s], ph);
           tc_fence_after();
-          const uint32_t a_base = smem_u32(sA + (ARES ? i : s) * A_BYTES), b_base = smem_u32(sB + s * B_BYTES);
+          const uint32_t a_base = smem_u32(sA + (ARES ? i * A_BYTES : s * A_SLOT)), b_base = smem_u32(sB + s * B_SLOT);
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k) {
             // K-major: advance 16 elements (32 B) inside the 128B swizzle atom.
             // MN-major: advance 16 K-rows (2 atoms of 8 rows x 128 B = 2048 B).
             const uint64_t ad = A_MN ? desc_sw128(a_base + k * 2048, 8192, 1024) : desc_sw128(a_base + k * 32, 16, 1024);
             const uint64_t bd = B_MN ? desc_sw128(b_base + k * 2048, 8192, 1024) : desc_sw128(b_base + k * 32, 16, 1024);
-            mma_bf16(d, ad, bd, idesc, (i > 0 || k > 0) ? 1u : 0u);
-            if (ONES && ones)   // TMEM column BN += dZ^T tile . e_0  (db2)
-              mma_bf16(d + BN, ad, desc_sw128(ones_base + k * 32, 16, 1024), idesc1, (i > 0 || k > 0) ? 1u : 0u);
+            const uint32_t first = (i > 0 || k > 0) ? 1u : 0u;
+            mma_bf16(d, ad, bd, idesc, first);
+            if constexpr (X3) {   // + hi.lo + lo.hi (the lo tiles sit one half further in the stage)
+              const uint64_t bdl = B_MN ? desc_sw128(b_base + B_BYTES + k * 2048, 8192, 1024)
+                                        : desc_sw128(b_base + B_BYTES + k * 32, 16, 1024);
+              const uint64_t adl = A_MN ? desc_sw128(a_base + A_BYTES + k * 2048, 8192, 1024)
+                                        : desc_sw128(a_base + A_BYTES + k * 32, 16, 1024);
+              mma_bf16(d, ad, bdl, idesc, 1u);
+              mma_bf16(d, adl, bd, idesc, 1u);
+              if (ONES && ones) {
+                mma_bf16(d + BN, ad, desc_sw128(ones_base + k * 32, 16, 1024), idesc1, first);
+                mma_bf16(d + BN, adl, desc_sw128(ones_base + k * 32, 16, 1024), idesc1, 1u);
+              }
+            } else {
+              if (ONES && ones)   // TMEM column BN += dZ^T tile . e_0  (db2)
+                mma_bf16(d + BN, ad, desc_sw128(ones_base + k * 32, 16, 1024), idesc1, first);
+            }
           }
           mma_commit(&empty[s]);   // frees the smem stage once these MMAs retire
         }
@@ -560,6 +594,13 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
               uint2 pk;
               pk.x = *reinterpret_cast<uint32_t*>(&p0); pk.y = *reinterpret_cast<uint32_t*>(&p1);
               __stcs(reinterpret_cast<uint2*>(g.shadow + o), pk);
+              if constexpr (X3) {   // lo half of the new shadow (R14)
+                __nv_bfloat162 q0 = __floats2bfloat162_rn(x.x - __low2float(p0), x.y - __high2float(p0));
+                __nv_bfloat162 q1 = __floats2bfloat162_rn(x.z - __low2float(p1), x.w - __high2float(p1));
+                uint2 pl;
+                pl.x = *reinterpret_cast<uint32_t*>(&q0); pl.y = *reinterpret_cast<uint32_t*>(&q1);
+                __stcs(reinterpret_cast<uint2*>(g.shadow_lo + o), pl);
+              }
               if (g.grad) *reinterpret_cast<float4*>(g.grad + o) = a;
             }
           }
@@ -835,23 +876,26 @@ cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t 
   return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }
 
-template <int BN, bool A_MN, bool B_MN, int EPI>
+template <int BN, bool A_MN, bool B_MN, int EPI, bool X3 = false>
 cudaError_t run(const Launch& lc, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c,
-               const CUtensorMap& d, TcArgs g, int splits) {
+               const CUtensorMap& d, TcArgs g, int splits, const CUtensorMap* a2 = nullptr,
+               const CUtensorMap* b2 = nullptr) {
   constexpr bool ARES = a_resident<EPI, A_MN>();
+  constexpr size_t XF = X3 ? 2 : 1;
   const size_t smem = (ARES ? (size_t)(kAresK / BK) * BM * BK * 2 : 0) +
-                      (size_t)stages_of<EPI>() * ((ARES ? 0 : BM * BK * 2) + BN * BK * 2) +
+                      (size_t)stages_of<EPI, X3>() * XF * ((ARES ? 0 : BM * BK * 2) + BN * BK * 2) +
                       (EPI == TC_EPI_SGD ? 2048 : 0) + staging_bytes<BN, EPI, A_MN>() + bias_bytes<BN, EPI>() + 1024 + 512;
   if (ARES && g.K > kAresK) return cudaErrorNotSupported;   // resident A block holds K <= 256
+  if (X3 && (!a2 || !b2)) return cudaErrorInvalidValue;
   {
-    cudaError_t e = ensure_smem(k_gemm_tc<BN, A_MN, B_MN, EPI>, smem);
+    cudaError_t e = ensure_smem(k_gemm_tc<BN, A_MN, B_MN, EPI, X3>, smem);
     if (e != cudaSuccess) return e;
   }
   g.splits = splits;
   const int64_t tiles = (int64_t)((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN) * splits;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, lc.sms));
-  return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_gemm_tc<BN, A_MN, B_MN, EPI>, dim3(grid),
-                      dim3(128 + 32 * epi_warps<BN, EPI>()), smem, a, b, c, d, g);
+  return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_gemm_tc<BN, A_MN, B_MN, EPI, X3>, dim3(grid),
+                      dim3(128 + 32 * epi_warps<BN, EPI>()), smem, a, b, c, d, X3 ? *a2 : a, X3 ? *b2 : b, g);
 }
 
 // Widest N tile that still gives >= one CTA per SM (and does not overhang N by 2x).
@@ -864,7 +908,7 @@ int pick_bn(int64_t tiles_m, int64_t N, int sms) {
 }  // namespace
 
 int gemm_tc_g2_ctas(int n, int H, const WsLayout& W, int sms) {
-  const int bn = H >= 256 ? 256 : H;
+  const int bn = W.x3 ? std::min(H, 128) : (H >= 256 ? 256 : H);
   const int64_t tiles = (int64_t)((n + BM - 1) / BM) * ((H + bn - 1) / bn) * W.splitk;
   return (int)std::min<int64_t>(tiles, sms);
 }
@@ -882,13 +926,15 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
                            const int64_t* dz_lab_ptr, const int32_t* dz_lab, const float* hoff) {
   if (!tc_available()) return cudaErrorNotSupported;
   const int64_t Lp = padded_ld(L);
-  CUtensorMap ta, tb, tc;
+  CUtensorMap ta, tb, tc, ta2, tb2;
   TcArgs g{};
   cudaError_t e;
+  const bool x3 = P.w2l != nullptr;   // fp32 path: bf16x3 operands (R14)
+  if (x3 && which != 1 && which != 2 && which != 3) return cudaErrorNotSupported;   // Z is stored on that path
   if (which == 1 || which == 5) {  // Z = H1 W2^T + b2 (5: only the per-tile softmax partials)
     g.M = n; g.N = (int)L; g.K = H;
     g.out = P.z; g.ldo = Lp; g.bias = b2;
-    const int bn = pick_bn((n + BM - 1) / BM, L, lc.sms);
+    const int bn = std::min(pick_bn((n + BM - 1) / BM, L, lc.sms), x3 ? 128 : 256);
     g.stats = stats; g.stats_ld = W.stats_ld;
     g.write_z = which == 1;
     g.chunked = 1;
@@ -898,6 +944,12 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
     if ((e = make_map(&ta, P.h1b, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
     if ((e = make_map(&tb, P.w2b, H, L, (uint64_t)H * 2, 64, bn)) != cudaSuccess) return e;
     if ((e = make_store_map(&tc, P.z, L, n, (uint64_t)Lp * 4, 1, 0, 2)) != cudaSuccess) return e;
+    if (x3) {
+      if ((e = make_map(&ta2, P.h1l, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
+      if ((e = make_map(&tb2, P.w2l, H, L, (uint64_t)H * 2, 64, bn)) != cudaSuccess) return e;
+      if (bn == 128) return run<128, false, false, TC_EPI_Z, true>(lc, ta, tb, tc, tc, g, 1, &ta2, &tb2);
+      return run<64, false, false, TC_EPI_Z, true>(lc, ta, tb, tc, tc, g, 1, &ta2, &tb2);
+    }
     if (which == 5) {
       if (bn == 256) return run<256, false, false, TC_EPI_STATS>(lc, ta, tb, tc, tc, g, 1);
       if (bn == 128) return run<128, false, false, TC_EPI_STATS>(lc, ta, tb, tc, tc, g, 1);
@@ -940,6 +992,12 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
     const int64_t bmax = W.part_stride / H;
     if ((e = make_store_map(&tc, P.dhpart, H, bmax, (uint64_t)H * 4, splits,
                             (uint64_t)W.part_stride * 4, 3)) != cudaSuccess) return e;
+    if (x3) {
+      if ((e = make_map(&ta2, P.dzl, L, n, (uint64_t)Lp * 2, 64, BM)) != cudaSuccess) return e;
+      if ((e = make_map(&tb2, P.w2l, H, L, (uint64_t)H * 2, 64, 64)) != cudaSuccess) return e;
+      if (H >= 128) return run<128, false, true, TC_EPI_PART, true>(lc, ta, tb, tc, tc, g, splits, &ta2, &tb2);
+      return run<64, false, true, TC_EPI_PART, true>(lc, ta, tb, tc, tc, g, splits, &ta2, &tb2);
+    }
     if (H >= 256) return run<256, false, true, TC_EPI_PART>(lc, ta, tb, tc, tc, g, splits);
     if (H == 128) return run<128, false, true, TC_EPI_PART>(lc, ta, tb, tc, tc, g, splits);
     return run<64, false, true, TC_EPI_PART>(lc, ta, tb, tc, tc, g, splits);
@@ -960,6 +1018,13 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
   CUtensorMap td;   // W2 fp32 boxes (load + store) and the bf16 shadow boxes (store)
   if ((e = make_store_map(&tc, W2, H, L, (uint64_t)H * 4, 1, 0, 2)) != cudaSuccess) return e;
   if ((e = make_bf16_store_map(&td, P.w2b, H, L)) != cudaSuccess) return e;
+  if (x3) {
+    g.shadow_lo = P.w2l;
+    if ((e = make_map(&ta2, P.dzl, L, n, (uint64_t)Lp * 2, 64, 64)) != cudaSuccess) return e;
+    if ((e = make_map(&tb2, P.h1l, H, n, (uint64_t)H * 2, 64, 64)) != cudaSuccess) return e;
+    if (bn == 128) return run<128, true, true, TC_EPI_SGD, true>(lc, ta, tb, tc, td, g, 1, &ta2, &tb2);
+    return run<64, true, true, TC_EPI_SGD, true>(lc, ta, tb, tc, td, g, 1, &ta2, &tb2);
+  }
   if (bn == 128) return run<128, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
   return run<64, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
 }

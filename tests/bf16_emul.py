@@ -19,8 +19,13 @@ product and sum in fp64:
   sigmoid (R11):     dZc = bf((sigmoid(Z) - 1/2 - Y) / B)   (centred)
                      dW2 = dZc^T Hq + (1/(2B)) 1 (sum_n H1_n)^T;  db2 = 1^T dZc + 1/2
                      dH1 = dZc Wq + (1/(2B)) sum_j Wq_j
-What is left between it and the kernels is fp32 accumulation order, ex2.approx
-and the rare element whose fp32 value sits at a bf16 rounding midpoint."""
+What is left between it and the kernels is fp32 accumulation order, ex2.approx,
+the rare element whose fp32 value sits at a bf16 rounding midpoint, and the
+ReLU mask where the GPU's fp32 A1 and the fp64 one straddle zero.  For the last
+one `slack` bounds what a flipped mask element can move: every (n, h) with
+|A1_nh| within the fp32 SpMM error bound (s_n 2^-24 sum_f |x_nf| |W1_fh| +
+2^-24 |b1_h|, s_n = the row's nnz) may go either way, moving dW1[f, h] by at
+most |x_nf| |dH1_nh| (1 + 2^-7) and db1[h] by |dH1_nh|."""
 import numpy as np
 import scipy.sparse as sp
 
@@ -34,10 +39,11 @@ def bf16(x):
     return f.astype(np.float64)
 
 
-def grads_bf16(w, batch, F, H, L, loss="softmax", B_full=None):
+def grads_bf16(w, batch, F, H, L, loss="softmax", B_full=None, with_slack=False):
     """Flat gradient (layout W1, b1, W2, b2) of the rows of `batch` as the bf16
     path computes it; B_full = the step's row count when `batch` is a chunk of
-    it (the 1/B scale is applied before the dZ rounding, as in the kernels)."""
+    it (the 1/B scale is applied before the dZ rounding, as in the kernels).
+    with_slack: also the flat per-element slack of ReLU-kink elements (above)."""
     w = np.asarray(w, dtype=np.float64)
     o = 0
     W1 = w[o:o + F * H].reshape(F, H); o += F * H
@@ -74,4 +80,14 @@ def grads_bf16(w, batch, F, H, L, loss="softmax", B_full=None):
     dA1 = dH1 * (A1 > 0.0)
     db1 = dA1.sum(axis=0)
     dW1 = np.asarray(X.T @ bf16(dA1))
-    return np.concatenate([dW1.ravel(), db1, dW2.ravel(), db2])
+    g = np.concatenate([dW1.ravel(), db1, dW2.ravel(), db2])
+    if not with_slack:
+        return g
+    Xa = abs(X)
+    nnz_row = np.diff(batch.row_ptr).astype(np.float64)[:, None]
+    bound = nnz_row * 2.0 ** -24 * np.asarray(Xa @ np.abs(W1)) + 2.0 ** -24 * np.abs(b1)[None, :]
+    kink = (np.abs(A1) <= bound) * np.abs(dH1) * (1 + 2.0 ** -7)
+    sl = np.zeros_like(g)
+    sl[:F * H] = np.asarray(Xa.T @ kink).ravel()
+    sl[F * H:F * H + H] = kink.sum(axis=0)
+    return g, sl

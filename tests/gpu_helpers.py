@@ -35,9 +35,9 @@ def _row_errors(a, b):
     return np.linalg.norm(a - b, axis=1) / np.maximum(nb, floor if floor > 0 else 1.0)
 
 
-def _elem_err(a, b, tol, per_row):
-    """max |a - b| / (tol |b| + tol s): s = the RMS of b's row (per_row) or of
-    the whole tensor; <= 1 passes."""
+def _elem_err(a, b, tol, per_row, slack=None):
+    """max (|a - b| - slack) / (tol |b| + tol s): s = the RMS of b's row (per_row)
+    or of the whole tensor; <= 1 passes."""
     a = np.asarray(a, dtype=np.float64)
     b = np.asarray(b, dtype=np.float64)
     if b.size == 0:
@@ -46,10 +46,13 @@ def _elem_err(a, b, tol, per_row):
         s = np.sqrt(np.mean(b * b, axis=1, keepdims=True))
     else:
         s = np.sqrt(np.mean(b * b))
-    return float((np.abs(a - b) / (tol * np.abs(b) + tol * s + 1e-300)).max(initial=0.0))
+    d = np.abs(a - b)
+    if slack is not None:
+        d = np.maximum(d - np.asarray(slack, dtype=np.float64).reshape(d.shape), 0.0)
+    return float((d / (tol * np.abs(b) + tol * s + 1e-300)).max(initial=0.0))
 
 
-def check_grads(gg, og, tol, F, H, touched, tag="", emul=None):
+def check_grads(gg, og, tol, F, H, touched, tag="", emul=None, slack=None):
     """Normwise, per-row and elementwise parity of the four gradient tensors.
 
     * normwise ||g - o|| / ||o|| <= tol per tensor against the fp64 oracle
@@ -60,7 +63,8 @@ def check_grads(gg, og, tol, F, H, touched, tag="", emul=None):
     fp32 path: the per-row and elementwise references r are the fp64 oracle, the
     RMS is the tensor's.  bf16 path (emul = the split gradient of
     tests/bf16_emul.py, the same mathematics with the kernels' bf16 rounding
-    points): r is that reference and the RMS is the row's -- bf16 operand
+    points; slack = its per-element allowance for ReLU-kink elements, whose fp32
+    and fp64 A1 may straddle zero): r is that reference and the RMS is the row's -- bf16 operand
     rounding alone moves single W2 rows of the exact gradient by a few percent
     (see bf16_emul.py), so a localized bug is looked for against the rounded
     arithmetic, while the exact-gradient bar stays the normwise one.
@@ -80,8 +84,12 @@ def check_grads(gg, og, tol, F, H, touched, tag="", emul=None):
     if emul is not None:   # for the record: per-row distance of the bf16 path to the exact gradient
         rec["row_W2_max_vs_oracle"] = float(_row_errors(W2g, np.asarray(og["W2"]).reshape(L, H)).max(initial=0.0))
     pairs = {"W1": (W1g, W1r), "b1": (gg["b1"], ref["b1"]), "W2": (W2g, W2r), "b2": (gg["b2"], ref["b2"])}
+    sl = {}
+    if slack is not None:
+        sl = {"W1": np.asarray(slack["W1"]).reshape(F, H)[touched], "b1": slack["b1"]}
+        rec["kink_elems"] = int((sl["W1"] > 0).sum())
     for k, (a, b) in pairs.items():
-        rec[f"elem_{k}"] = _elem_err(a, b, tol, per_row=emul is not None)
+        rec[f"elem_{k}"] = _elem_err(a, b, tol, per_row=emul is not None, slack=sl.get(k))
     log = os.environ.get("ASGD_PARITY_LOG")
     if log:
         with open(log, "a") as f:
