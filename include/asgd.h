@@ -308,6 +308,10 @@ int asgd_run_static(asgd_ctx* ctx, int32_t rank, int32_t world, int64_t b,
 int asgd_route_replay(int32_t n_ranks, int32_t n_tickets, const int32_t* order,
                       const int64_t* b, int64_t M, int64_t* out, int64_t cap,
                       int64_t* n_out);
+/* Elastic SGD's static routes (R10): the M samples cut into
+ * batches of b, batch k -> rank k mod n; out: int64[3*cap] (rank, start, len). */
+int asgd_route_static(int32_t n, int64_t b, int64_t M, int64_t* out, int64_t cap, int64_t* n_out);
+
 /* Simulated clock (Q10): every rank free at t = 0; the rank free first (ties:
  * lowest id) takes the next batch; it stays busy
  * cost_factor[r] * (nnz(batch) + per_row * len).  row_nnz: int64[M] nnz of the

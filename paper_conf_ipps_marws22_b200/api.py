@@ -281,6 +281,15 @@ def route_replay(order, b, M) -> List[Tuple[int, int, int]]:
     return [tuple(int(x) for x in out[3 * i:3 * i + 3]) for i in range(n.value)]
 
 
+def route_static(n, b, M) -> List[Tuple[int, int, int]]:
+    """Elastic SGD's static routes (R10): batch k of b samples -> rank k mod n."""
+    cap = int(M) // max(1, int(b)) + 2
+    out = np.zeros(3 * cap, dtype=np.int64)
+    k = C.c_int64()
+    call("asgd_route_static", int(n), int(b), int(M), _ptr(out), cap, C.byref(k))
+    return [tuple(int(x) for x in out[3 * i:3 * i + 3]) for i in range(k.value)]
+
+
 def route_simulate(b, M, cost_factor, per_row, row_nnz) -> List[Tuple[int, int, int]]:
     b_ = _np(b, np.int64)
     cf = _np(cost_factor, np.float64)

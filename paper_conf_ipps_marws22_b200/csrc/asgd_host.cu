@@ -73,6 +73,13 @@ int64_t fused_ce_bytes() {
   return v;
 }
 
+// G2 with the dH1 reduce + b1 update fused into its tail (default); ASGD_G2_FUSE=0: the
+// separate k_dh_reduce / k_b1_update launches (A/B).
+bool g2_fuse() {
+  static const bool v = [] { const char* e = getenv("ASGD_G2_FUSE"); return !(e && e[0] == '0'); }();
+  return v;
+}
+
 int splitk_for(const asgd_model_desc& d) {
   // G2 (dH1 = dZ W2, M = b_max, N = H, K = L): split K so ~2 waves of CTAs run (ASGD_G2_WAVES;
   // one wave measured: Amazon-670K G2 372 -> 602 us, Delicious-200K 125 -> 192 us, AmazonCat even)
@@ -141,7 +148,7 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.rowloss = take(B * 4);
   L.dhpart = take((size_t)L.splitk * B * H * 4);
   L.da1 = take(B * H * 4);
-  L.db1part = take(L.n_rowblk * H * 4);
+  L.db1part = take(std::max<int64_t>(L.n_rowblk, 160) * H * 4);   // + G2's fused column partials
   L.w2b = take(bf ? (size_t)Lb * H * 2 : 0);
   L.w2b2 = take(bf ? (size_t)Lb * H * 2 : 0);
   L.red = take((L.n_red + 8) * 8);
@@ -603,12 +610,20 @@ int enqueue_step(asgd_ctx* c, int n) {
       CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
       PCU_ON(c->s3, ASGD_K_G3, g3(lc3));
     }
-    PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr));
-    PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, bf, centred ? P.cen : nullptr));
-    CU(cudaEventRecord(c->ev_dh, c->s));
-    CU(cudaStreamWaitEvent(c->s3, c->ev_dh, 0));
-    PCU_ON(c->s3, ASGD_K_DH, launch_b1_update(lc3, n, H, b1, P, c->L, g ? g + c->o_b1 : nullptr));
-    CU(cudaEventRecord(c->ev_a, c->s3));
+    if (g2_fuse()) {
+      // G2 + the dH1 reduce + ReLU' + b1 update + mean loss in one launch (grid barrier)
+      const DhFuse fz{b1, g ? g + c->o_b1 : nullptr, centred ? P.cen : nullptr, bf};
+      PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, nullptr, nullptr,
+                                    nullptr, nullptr, nullptr, nullptr, &fz));
+      CU(cudaEventRecord(c->ev_a, c->s3));
+    } else {
+      PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr));
+      PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, bf, centred ? P.cen : nullptr));
+      CU(cudaEventRecord(c->ev_dh, c->s));
+      CU(cudaStreamWaitEvent(c->s3, c->ev_dh, 0));
+      PCU_ON(c->s3, ASGD_K_DH, launch_b1_update(lc3, n, H, b1, P, c->L, g ? g + c->o_b1 : nullptr));
+      CU(cudaEventRecord(c->ev_a, c->s3));
+    }
     // K-5 (needs K-0's segments)
     CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
     PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
@@ -1090,6 +1105,17 @@ int asgd_route_replay(int32_t n_ranks, int32_t nt, const int32_t* order, const i
     out[3 * k] = r; out[3 * k + 1] = c; out[3 * k + 2] = len;
     ++k;
     c += len;
+  }
+  *n_out = k;
+  return ASGD_OK;
+}
+
+int asgd_route_static(int32_t n, int64_t b, int64_t M, int64_t* out, int64_t cap, int64_t* n_out) {
+  if (n < 1 || b < 1 || M < 0 || !out || !n_out) return fail(ASGD_E_ARG, "bad argument");
+  int64_t k = 0;
+  for (int64_t c = 0; c < M; c += b, ++k) {   // R10: batch k -> rank k mod n
+    if (k >= cap) return fail(ASGD_E_SHAPE, "route cap %lld too small", (long long)cap);
+    out[3 * k] = k % n; out[3 * k + 1] = c; out[3 * k + 2] = std::min<int64_t>(b, M - c);
   }
   *n_out = k;
   return ASGD_OK;

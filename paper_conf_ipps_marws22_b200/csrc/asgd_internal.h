@@ -22,7 +22,7 @@ constexpr int kScanTile = 1024;
 // M_K0PAR: parity of K-0's double-buffered tile sums.
 // M_MSYNC: fused merge arrival counter (64-bit, slots 40-41), M_MDONE: its CTA counter.
 enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_LR = 6, M_K0PAR = 7, M_COUNT = 8,
-       M_LOSS = 10, M_BAR = 32, M_MSYNC = 40, M_MDONE = 42, M_CEN = 44 };
+       M_LOSS = 10, M_BAR = 32, M_MSYNC = 40, M_MDONE = 42, M_CEN = 44, M_G2BAR = 46 /* 46-48 */ };
 // error bits in meta[M_ERR]
 enum { ERR_NNZ_CAP = 1, ERR_LAB_CAP = 2, ERR_ROW_ID = 4 };
 
@@ -194,11 +194,16 @@ bool tc_available();
 // which: 1 = G1 (Z = H1 W2^T + b2), 2 = G2 (dH1 split-K partials), 3 = G3 (W2 -= lr dZ^T H1 and
 // b2 -= lr 1^T dZ, both fused in the epilogue)
 // stats (G1 only, nullable): per (N tile, row) softmax partials; *stats_ntiles = N tiles.
+// G2 with the dH1 reduce, ReLU' and the b1 update fused into its tail (which = 2).
+struct DhFuse {
+  float* b1; float* grad_b1; const float* dh_off; bool want_bf16;
+};
 cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int H,
                            const Ptrs&, const WsLayout&, float* W2, float* b2, float* grad_w2,
                            float* grad_b2, float2* stats = nullptr, int* stats_ntiles = nullptr,
                            const int32_t* dz_rows = nullptr, const int64_t* dz_lab_ptr = nullptr,
-                           const int32_t* dz_lab = nullptr, const float* hoff = nullptr);
+                           const int32_t* dz_lab = nullptr, const float* hoff = nullptr,
+                           const DhFuse* fuse = nullptr);
 // CTAs G2 runs with (the concurrent G3 leaves those SMs to it).
 int gemm_tc_g2_ctas(int n, int H, const WsLayout&, int sms);
 // which = 4 (G1b): dZ = (softmax - T)/B from a recomputed Z tile; needs P.lse from k_lse.

@@ -424,7 +424,11 @@ __global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_
   constexpr int kGroup = k1_group<VPL>();        // pieces per group = warps per CTA
   __shared__ __align__(16) float spart[kGroup][2][H];   // per warp: [0] its first segment, [1] its last
   const int warp = threadIdx.x >> 5;
-  const int ngroups = (npieces + kGroup - 1) / kGroup;
+  // pieces per group: up to one per warp, fewer when the batch has fewer than kGroup
+  // pieces per CTA, so every CTA of the grid gets a group (EURLex: 1,875 pieces -> 13 per
+  // group on 145 CTAs instead of 16 on 117); the idle warps only join the barriers
+  const int gs = max(1, min(kGroup, (npieces + (int)gridDim.x - 1) / (int)gridDim.x));
+  const int ngroups = (npieces + gs - 1) / gs;
   auto finish = [&](int r, float (&acc)[VPL]) {
     float bias[VPL];   // b1 re-read (L1) instead of held in registers across the gathers
     IO::load_ldg(b1, lane, bias);
@@ -437,7 +441,7 @@ __global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_
   // group g's partial of row r (global): slot 2 g + 1 if r starts in g, else 2 g; the
   // last group to arrive sums the row's group partials in group order and finishes
   auto publish = [&](int g, int r, float (&acc)[VPL]) {
-    constexpr int GE = kGroup * kPiece;          // entries per group
+    const int GE = gs * kPiece;                  // entries per group
     const int rs = sboff[r], re = sboff[r + 1];
     const int g0 = rs / GE, g1 = (re - 1) / GE;
     IO::store_cg(part + (int64_t)(g == g0 ? 2 * g + 1 : 2 * g) * H, lane, acc);
@@ -472,9 +476,10 @@ __global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_
   };
 
   for (int g = blockIdx.x; g < ngroups; g += gridDim.x) {
-    const int p = g * kGroup + warp;
-    const int G0 = g * kGroup * kPiece, G1 = min(G0 + kGroup * kPiece, nnz);
-    const int e0 = p * kPiece, e1 = min(e0 + kPiece, nnz), cnt = max(0, e1 - e0);
+    const int p = g * gs + warp;
+    const int G0 = g * gs * kPiece, G1 = min(G0 + gs * kPiece, nnz);
+    const int e0 = warp < gs ? p * kPiece : nnz;   // idle warps (warp >= gs): an empty piece
+    const int e1 = min(e0 + kPiece, nnz), cnt = max(0, e1 - e0);
     // Row segment of row r ends inside this piece: finish it (ReLU(acc + b1)) when the
     // piece holds the whole row, else park it in shared memory for the group combine
     auto flush = [&](int r, float (&acc)[VPL]) {
@@ -546,7 +551,7 @@ __global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_
         if (max(rs, G0) < e0) continue;          // an earlier warp of the group holds its first segment
         float acc[VPL];
         IO::load(&spart[warp][before ? 0 : 1][0], lane, acc);
-        for (int w2 = warp + 1; w2 < kGroup && (g * kGroup + w2) * kPiece < min(re, G1); ++w2) {
+        for (int w2 = warp + 1; w2 < gs && (g * gs + w2) * kPiece < min(re, G1); ++w2) {
           float t[VPL];
           IO::load(&spart[w2][0][0], lane, t);   // row r is w2's first segment
 #pragma unroll

@@ -48,6 +48,12 @@ struct TcArgs {
   // G1b (TC_EPI_DZ): dZ = (exp(Z - lse) - T) / B recomputed from the MMA, stored bf16;
   // G1 sigmoid (TC_EPI_SIG): dZ = (sigmoid(Z) - Y) / B, BCE row partials in stats
   const float* lse; const int32_t* rows; const int64_t* lab_ptr; const int32_t* lab; float invB;
+  // G2 fused with the dH1 reduce (DH_FUSE): after a grid barrier, CTA k sums the split-K
+  // partials of its (row block, column block), applies ReLU' (dA1 = dH1 [H1 > 0]), writes
+  // dA1 (fp32, + bf16) and its column sums; the last CTA applies b1 -= lr db1 and the mean loss
+  int dh_fuse;
+  const float* h1; float* da1; bf16* da1b; const float* dh_off;
+  float* b1; float* grad_b1; float* colpart; const float* rowloss; int32_t* bar;
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -229,6 +235,106 @@ constexpr uint32_t pow2ceil(uint32_t x) {
   uint32_t p = 32;
   while (p < x) p <<= 1;
   return p;
+}
+
+// G2's fused tail (TC_EPI_PART with g.dh_fuse, rows a6/a7 of DESIGN.md): replaces the
+// k_dh_reduce and k_b1_update launches.  Every CTA of the persistent grid is resident
+// (one per SM, grid <= SMs; the kernels beside it on other streams never wait for G2),
+// so a software grid barrier is safe.  CTA k then owns rows [r0, r1) x columns [c0, c1)
+// of dH1 (GC column blocks of >= 32 columns, GR = grid / GC row blocks):
+//   dA1 = [H1 > 0] * (sum_z part[z] (+ the centred-sigmoid offset))  -> dA1 (fp32, bf16)
+//   colpart[row block][c] = sum_{r in block} dA1[r][c]   (fixed order)
+// and the last CTA to finish sums colpart over the row blocks in order: b1 -= lr db1,
+// grad_b1 = db1, and the mean loss from the per-row losses (deterministic).
+__device__ void dh_reduce_phase(const TcArgs& g, float* sred) {
+  const int G = gridDim.x, k = blockIdx.x, H = g.N, n = g.M, S = g.splits;
+  __shared__ int s_last;
+  // (1) every CTA's partial stores are complete (each epilogue lane waited on its bulk
+  // groups before the kernel's final barrier): make them visible, then the grid barrier
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    volatile int32_t* cnt = g.bar;
+    volatile int32_t* gen = g.bar + 1;
+    const int32_t g0 = *gen;
+    __threadfence();
+    if (atomicAdd(g.bar, 1) == G - 1) {
+      *cnt = 0;
+      __threadfence();
+      atomicAdd(g.bar + 1, 1);
+    } else {
+      while (*gen == g0) __nanosleep(64);
+    }
+    __threadfence();
+  }
+  __syncthreads();
+  // (2) this CTA's block
+  int GC = H / 32;
+  if (GC > G) GC = G;
+  const int GR = G / GC;
+  if (k >= GR * GC) {   // no block (G not a multiple of GC): still arrive at the last-CTA count
+    __syncthreads();
+  } else {
+    const int cb = k % GC, rb = k / GC;
+    const int c0 = cb * H / GC, c1 = (cb + 1) * H / GC, nc = c1 - c0;
+    const int r0 = rb * n / GR, r1 = (rb + 1) * n / GR;
+    const float lr = step_lr(g.meta);
+    (void)lr;
+    for (int e = threadIdx.x; e < (r1 - r0) * nc; e += blockDim.x) {
+      const int r = r0 + e / nc, c = c0 + e % nc;
+      const int64_t o = (int64_t)r * H + c;
+      float a[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) a[q] = 0.f;
+      for (int z = 0; z < S; z += 8) {
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+          if (z + q < S) a[q] += __ldcg(g.out + (int64_t)(z + q) * g.part_stride + o);
+      }
+      float sum = ((a[0] + a[1]) + (a[2] + a[3])) + ((a[4] + a[5]) + (a[6] + a[7]));
+      if (g.dh_off) sum += g.dh_off[c];   // centred sigmoid dZ: + (1/(2B)) sum_j W2_j
+      const float v = g.h1[o] > 0.f ? sum : 0.f;
+      g.da1[o] = v;
+      if (g.da1b) g.da1b[o] = __float2bfloat16_rn(v);
+      sred[(e / nc) * nc + (e % nc)] = v;
+    }
+    __syncthreads();
+    // column sums of the block, rows in order (one thread per column, 4 partial chains)
+    for (int c = threadIdx.x; c < nc; c += blockDim.x) {
+      float t[4] = {0.f, 0.f, 0.f, 0.f};
+      const int nr = r1 - r0;
+      int r = 0;
+      for (; r + 4 <= nr; r += 4) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) t[q] += sred[(r + q) * nc + c];
+      }
+      for (; r < nr; ++r) t[0] += sred[r * nc + c];
+      g.colpart[(int64_t)rb * H + c0 + c] = (t[0] + t[1]) + (t[2] + t[3]);
+    }
+  }
+  // (3) the last CTA: db1 = sum over row blocks in order; b1 -= lr db1; mean loss
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) s_last = atomicAdd(g.bar + 2, 1) == G - 1;
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  const float lr = step_lr(g.meta);
+  for (int c = threadIdx.x; c < H; c += blockDim.x) {
+    float t = 0.f;
+    for (int rb = 0; rb < GR; ++rb) t += __ldcg(g.colpart + (int64_t)rb * H + c);
+    g.b1[c] -= lr * t;
+    if (g.grad_b1) g.grad_b1[c] = t;
+  }
+  float* loss_dev = step_loss(g.meta);
+  if (threadIdx.x < 32 && loss_dev) {
+    float t = 0.f;
+    for (int r = threadIdx.x; r < n; r += 32) t += __ldcg(g.rowloss + r);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+    if (threadIdx.x == 0) *loss_dev = t / (float)n;
+  }
+  if (threadIdx.x == 0) g.bar[2] = 0;
 }
 
 // Persistent tcgen05 GEMM.  CTA = 4 + E warps: warp 0 TMA producer, warp 1 MMA
@@ -821,6 +927,9 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS) : "memory");
   }
+  if constexpr (EPI == TC_EPI_PART) {
+    if (g.dh_fuse) dh_reduce_phase(g, reinterpret_cast<float*>(smem));
+  }
 }
 
 // ------------------------------------------------------------------ host side
@@ -923,7 +1032,8 @@ int64_t padded_ld(int64_t L) { return (L + 7) / 8 * 8; }
 cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H, const Ptrs& P,
                            const WsLayout& W, float* W2, float* b2, float* grad_w2, float* grad_b2,
                            float2* stats, int* stats_ntiles, const int32_t* dz_rows,
-                           const int64_t* dz_lab_ptr, const int32_t* dz_lab, const float* hoff) {
+                           const int64_t* dz_lab_ptr, const int32_t* dz_lab, const float* hoff,
+                           const DhFuse* fuse) {
   if (!tc_available()) return cudaErrorNotSupported;
   const int64_t Lp = padded_ld(L);
   CUtensorMap ta, tb, tc, ta2, tb2;
@@ -980,9 +1090,15 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
     if (bn == 128) return run<128, false, false, TC_EPI_DZ>(lc, ta, tb, tc, tc, g, 1);
     return run<64, false, false, TC_EPI_DZ>(lc, ta, tb, tc, tc, g, 1);
   }
-  if (which == 2) {  // dH1 partials = dZ W2
+  if (which == 2) {  // dH1 partials = dZ W2 (fuse: + the dH1 reduce, ReLU', b1 update)
     g.M = n; g.N = H; g.K = (int)L;
     g.out = P.dhpart; g.ldo = H; g.part_stride = W.part_stride;
+    if (fuse) {
+      g.dh_fuse = 1; g.meta = P.meta;
+      g.h1 = P.h1; g.da1 = P.da1; g.da1b = fuse->want_bf16 ? P.da1b : nullptr; g.dh_off = fuse->dh_off;
+      g.b1 = fuse->b1; g.grad_b1 = fuse->grad_b1; g.colpart = P.db1part; g.rowloss = P.rowloss;
+      g.bar = P.meta + M_G2BAR;
+    }
     const int nkb = (int)((L + BK - 1) / BK);
     const int splits = std::max(1, std::min<int>((int)W.splitk, nkb));
     if ((e = make_map(&ta, P.dzb, L, n, (uint64_t)Lp * 2, 64, BM)) != cudaSuccess) return e;

@@ -66,6 +66,7 @@ class MegaBatchStats:
     perturbed: bool
     routes: list
     n_steps: int
+    merge_events: Optional[tuple] = None   # (start, end) CUDA events of the merge phase (time_merge)
 
 
 # --------------------------------------------------------------- host logic
@@ -145,6 +146,7 @@ class DistributedAdaptiveSGD:
         self.sq = torch.zeros(1, dtype=torch.float64, device=dev)
         self.events = [torch.cuda.Event() for _ in range(cap)]
         self.mb = 0
+        self.time_merge = False   # record CUDA events around the merge phase of each mega-batch
 
     def megabatch(self, stream_rows: torch.Tensor, keep_log: bool = False) -> MegaBatchStats:
         """One mega-batch over the M sample ids stream_rows (device int32)."""
@@ -164,6 +166,10 @@ class DistributedAdaptiveSGD:
             n_steps = run_tickets(self.sched, r, b_i, step, self.inflight,
                                   wait=lambda k: self.events[k].synchronize())
         # ---- merge (Alg. 2) -------------------------------------------------
+        ev = None
+        if self.time_merge:   # from the end of this rank's local steps to the merged model
+            ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+            ev[0].record(rep.stream)
         rep.sqnorm(self.sq)
         us, bs, nu = exchange_stats(n_steps, b_i, self.sq, rep.P, self.world, self.group)
         routes = self.sched.log() if keep_log and r == 0 else []
@@ -171,11 +177,13 @@ class DistributedAdaptiveSGD:
             self.sched.reset(self.mb + 1)        # every rank is past its tickets
         alpha, rr, ss, pert = api.merge_weights(us, bs, nu, h.pert_thr, h.delta, h.pert_renorm, h.norm)
         self._merge(alpha)
+        if ev is not None:
+            ev[1].record(rep.stream)
         # ---- Alg. 1 ----------------------------------------------------------
         lr_used = list(self.lr)
         if (self.mb + 1) % h.scale_every == 0:    # R13
             self.b, self.lr = api.scale_batches(us, bs, h.b_min, h.b_max, h.beta, h.lr_max)
-        st = MegaBatchStats(self.mb, us, bs, lr_used, nu, alpha, rr, ss, pert, routes, n_steps)
+        st = MegaBatchStats(self.mb, us, bs, lr_used, nu, alpha, rr, ss, pert, routes, n_steps, ev)
         self.mb += 1
         return st
 
@@ -236,14 +244,20 @@ class DistributedAdaptiveSGD:
         rep, h, r, N = self.rep, self.h, self.rank, self.world
         M = int(stream_rows.numel())
         n_steps = rep.run_static(r, N, h.b_max, stream_rows, h.lr_max, self.losses, self.inflight)
+        ev = None
+        if self.time_merge:
+            ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+            ev[0].record(rep.stream)
         rep.sqnorm(self.sq)
         us, bs, nu = exchange_stats(n_steps, h.b_max, self.sq, rep.P, N, self.group)   # also the barrier
         alpha = api.elastic_weights(N)
         self._merge(alpha)
+        if ev is not None:
+            ev[1].record(rep.stream)
         routes = []
         if keep_log and r == 0:
             routes = [(k, k % N, c, min(h.b_max, M - c)) for k, c in enumerate(range(0, M, h.b_max))]
-        st = MegaBatchStats(self.mb, us, bs, [h.lr_max] * N, nu, alpha, -1, -1, False, routes, n_steps)
+        st = MegaBatchStats(self.mb, us, bs, [h.lr_max] * N, nu, alpha, -1, -1, False, routes, n_steps, ev)
         self.mb += 1
         return st
 
@@ -252,7 +266,12 @@ class SimulatedAdaptiveSGD:
     """N replicas on one GPU; routing by the simulated clock (Q10) or replay."""
 
     def __init__(self, replicas: Sequence[api.Replica], hyper: Hyper, row_nnz: np.ndarray,
-                 cost_factors: Sequence[float], per_row: float = 5.0):
+                 cost_factors: Sequence[float], per_row: float = 5.0, method: str = "adaptive"):
+        """method "elastic": Elastic SGD's static routes of b_max (R10), alpha_i = 1/N,
+        no Alg. 1 -- the NEXT-2 A/B arm under the same simulated clock."""
+        if method not in ("adaptive", "elastic"):
+            raise ValueError(f"method={method!r}")
+        self.method = method
         self.reps, self.h = list(replicas), hyper
         self.n = len(self.reps)
         self.row_nnz = np.asarray(row_nnz, dtype=np.int64)
@@ -269,7 +288,9 @@ class SimulatedAdaptiveSGD:
     def megabatch(self, stream_rows: torch.Tensor, stream_ids: np.ndarray,
                   route_order: Optional[Sequence[int]] = None) -> MegaBatchStats:
         h = self.h
-        if route_order is not None:
+        if self.method == "elastic":
+            routes = api.route_static(self.n, h.b_max, h.M)
+        elif route_order is not None:
             routes = api.route_replay(route_order, self.b, h.M)
         else:
             routes = api.route_simulate(self.b, h.M, self.cf, self.per_row, self.row_nnz[stream_ids])
@@ -282,7 +303,10 @@ class SimulatedAdaptiveSGD:
             rep.sqnorm(self.sq[i:i + 1])
         P = self.reps[0].P
         nu = api.norm_per_param(self.sq.cpu().numpy(), P)
-        alpha, rr, ss, pert = api.merge_weights(u, self.b, nu, h.pert_thr, h.delta, h.pert_renorm, h.norm)
+        if self.method == "elastic":
+            alpha, rr, ss, pert = api.elastic_weights(self.n), -1, -1, False
+        else:
+            alpha, rr, ss, pert = api.merge_weights(u, self.b, nu, h.pert_thr, h.delta, h.pert_renorm, h.norm)
         r0 = self.reps[0]
         r0.weighted_sum(self.reps, alpha, r0.params)
         r0.finish(h.gamma)
@@ -290,7 +314,7 @@ class SimulatedAdaptiveSGD:
             rep.params.copy_(r0.params)
             rep.params_changed()
         lr_used, b_used = list(self.lr), list(self.b)
-        if (self.mb + 1) % h.scale_every == 0:    # R13
+        if self.method == "adaptive" and (self.mb + 1) % h.scale_every == 0:    # R13
             self.b, self.lr = api.scale_batches(u, self.b, h.b_min, h.b_max, h.beta, h.lr_max)
         st = MegaBatchStats(self.mb, u, b_used, lr_used, nu, alpha, rr, ss, pert, routes, len(routes))
         self.mb += 1

@@ -39,11 +39,14 @@ def bf16(x):
     return f.astype(np.float64)
 
 
-def grads_bf16(w, batch, F, H, L, loss="softmax", B_full=None, with_slack=False):
+def grads_bf16(w, batch, F, H, L, loss="softmax", B_full=None, with_slack=False, rounding=True):
     """Flat gradient (layout W1, b1, W2, b2) of the rows of `batch` as the bf16
     path computes it; B_full = the step's row count when `batch` is a chunk of
     it (the 1/B scale is applied before the dZ rounding, as in the kernels).
-    with_slack: also the flat per-element slack of ReLU-kink elements (above)."""
+    with_slack: also the flat per-element slack of ReLU-kink elements (above).
+    rounding=False: the same code with every rounding point the identity (the exact
+    gradient; its slack serves the fp32 path's elementwise check)."""
+    bf = bf16 if rounding else (lambda x: np.asarray(x, dtype=np.float64))
     w = np.asarray(w, dtype=np.float64)
     o = 0
     W1 = w[o:o + F * H].reshape(F, H); o += F * H
@@ -56,7 +59,7 @@ def grads_bf16(w, batch, F, H, L, loss="softmax", B_full=None, with_slack=False)
     cnt = np.diff(batch.lab_ptr)
     A1 = np.asarray(X @ W1) + b1
     H1 = np.maximum(A1, 0.0)
-    Hq, Wq = bf16(H1), bf16(W2)
+    Hq, Wq = bf(H1), bf(W2)
     Z = Hq @ Wq.T + b2
     if loss == "softmax":
         tv = np.repeat(1.0 / np.maximum(cnt, 1), cnt)
@@ -64,14 +67,14 @@ def grads_bf16(w, batch, F, H, L, loss="softmax", B_full=None, with_slack=False)
         m = Z.max(axis=1, keepdims=True)
         P = np.exp(Z - m)
         P /= P.sum(axis=1, keepdims=True)
-        dZ = bf16((P - T) / B)
+        dZ = bf((P - T) / B)
         dW2 = dZ.T @ Hq
         db2 = dZ.sum(axis=0)
         dH1 = dZ @ Wq
     elif loss == "sigmoid":
         Y = sp.csr_matrix((np.ones(int(cnt.sum())), batch.lab, batch.lab_ptr), shape=(n, L)).toarray()
         S = 1.0 / (1.0 + np.exp(-Z))
-        dZ = bf16((S - 0.5 - Y) / B)
+        dZ = bf((S - 0.5 - Y) / B)
         dW2 = dZ.T @ Hq + (1.0 / (2 * B)) * H1.sum(axis=0)[None, :]
         db2 = dZ.sum(axis=0) + 0.5 * n / B
         dH1 = dZ @ Wq + (1.0 / (2 * B)) * Wq.sum(axis=0)[None, :]
@@ -79,7 +82,7 @@ def grads_bf16(w, batch, F, H, L, loss="softmax", B_full=None, with_slack=False)
         raise ValueError(loss)
     dA1 = dH1 * (A1 > 0.0)
     db1 = dA1.sum(axis=0)
-    dW1 = np.asarray(X.T @ bf16(dA1))
+    dW1 = np.asarray(X.T @ bf(dA1))
     g = np.concatenate([dW1.ravel(), db1, dW2.ravel(), db2])
     if not with_slack:
         return g

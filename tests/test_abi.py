@@ -205,3 +205,10 @@ def test_norm_per_param_and_elastic_weights():
         api.norm_per_param([-1.0], 10)
     for n in range(1, 9):
         assert api.elastic_weights(n) == [1.0 / n] * n
+
+
+def test_route_static_matches_oracle():
+    rng = random.Random(11)
+    for _ in range(300):
+        n, b, M = rng.randint(1, 8), rng.randint(1, 40), rng.randint(0, 500)
+        assert api.route_static(n, b, M) == [tuple(r) for r in routing.static(n, b, M)]

@@ -52,23 +52,21 @@ def _rank(rank, world, port, shm, out, precision, n_mb, merge, method="adaptive"
         stats.append((st.u, st.b, st.lr, st.alpha, st.perturbed))
     torch.cuda.synchronize()
     np.save(os.path.join(out, f"w{rank}.npy"), rep.params.cpu().numpy())   # = w' after every merge
-    np.save(os.path.join(out, f"s{rank}.npy"), np.array([logs, stats], dtype=object), allow_pickle=True)
+    np.save(os.path.join(out, f"s{rank}.npy"), np.array([logs, stats, drv.merge], dtype=object), allow_pickle=True)
     dist.barrier()
     sched.close()
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("merge", ["nccl", "fused"])
-@pytest.mark.parametrize("precision,tol", [("fp32", 1e-4), ("bf16", 2e-2)])
-def test_two_ranks_one_gpu(tmp_path, precision, tol, merge):
-    world, n_mb = 2, 4
-    shm = "/asgd_d_" + uuid.uuid4().hex[:8]
-    mp.spawn(_rank, args=(world, _port(), shm, str(tmp_path), precision, n_mb, merge), nprocs=world, join=True)
-    w0, w1 = (np.load(tmp_path / f"w{r}.npy") for r in range(world))
-    np.testing.assert_array_equal(w0, w1)          # replicas end bitwise identical (Q20)
-    logs, stats = np.load(tmp_path / "s0.npy", allow_pickle=True)
-    _, stats1 = np.load(tmp_path / "s1.npy", allow_pickle=True)
-    assert [s[:4] for s in stats] == [s[:4] for s in stats1]
+def _check_world(tmp_path, world, n_mb, precision, tol, merge):
+    ws = [np.load(tmp_path / f"w{r}.npy") for r in range(world)]
+    for w in ws[1:]:
+        np.testing.assert_array_equal(ws[0], w)    # replicas end bitwise identical (Q20)
+    logs, stats, used = np.load(tmp_path / "s0.npy", allow_pickle=True)
+    assert used == merge                          # no silent fallback from the fused merge
+    for r in range(1, world):
+        _, stats_r, _ = np.load(tmp_path / f"s{r}.npy", allow_pickle=True)
+        assert [s[:4] for s in stats] == [s[:4] for s in stats_r]
     from oracle import adaptive
     from synth import config, generate, init_params, sample_stream
     cfg = config("tiny")
@@ -81,7 +79,27 @@ def test_two_ranks_one_gpu(tmp_path, precision, tol, merge):
         assert list(u) == rec.u and list(b) == rec.b and list(lr) == rec.lr and pert == rec.perturbed
         np.testing.assert_allclose(alpha, rec.alpha, rtol=1e-12)
     ref = recs[-1].w
-    assert np.linalg.norm(w0 - ref) / np.linalg.norm(ref) <= tol
+    assert np.linalg.norm(ws[0] - ref) / np.linalg.norm(ref) <= tol
+
+
+@pytest.mark.parametrize("merge", ["nccl", "fused"])
+@pytest.mark.parametrize("precision,tol", [("fp32", 1e-4), ("bf16", 2e-2)])
+def test_two_ranks_one_gpu(tmp_path, precision, tol, merge):
+    world, n_mb = 2, 4
+    shm = "/asgd_d_" + uuid.uuid4().hex[:8]
+    mp.spawn(_rank, args=(world, _port(), shm, str(tmp_path), precision, n_mb, merge), nprocs=world, join=True)
+    _check_world(tmp_path, world, n_mb, precision, tol, merge)
+
+
+@pytest.mark.parametrize("world", [3, 4])
+def test_fused_merge_three_and_four_ranks(tmp_path, world):
+    """N > 2 ranks on one GPU through the fused peer-memory merge: the parameter
+    vector (P = 134,564) splits into uneven shards; every rank reduces its shard
+    over CUDA IPC and stores w' into every replica."""
+    n_mb = 3
+    shm = "/asgd_w_" + uuid.uuid4().hex[:8]
+    mp.spawn(_rank, args=(world, _port(), shm, str(tmp_path), "fp32", n_mb, "fused"), nprocs=world, join=True)
+    _check_world(tmp_path, world, n_mb, "fp32", 1e-4, "fused")
 
 
 @pytest.mark.parametrize("precision,tol", [("fp32", 1e-4), ("bf16", 2e-2)])
@@ -93,7 +111,7 @@ def test_two_ranks_elastic(tmp_path, precision, tol):
              join=True)
     w0, w1 = (np.load(tmp_path / f"w{r}.npy") for r in range(world))
     np.testing.assert_array_equal(w0, w1)
-    logs, stats = np.load(tmp_path / "s0.npy", allow_pickle=True)
+    logs, stats, _ = np.load(tmp_path / "s0.npy", allow_pickle=True)
     from oracle import adaptive
     from synth import config, generate, init_params, sample_stream
     cfg = config("tiny")

@@ -29,9 +29,8 @@ def _chunked_oracle(w, batch, F, H, L, chunk, loss_kind="softmax", emulate=False
         f = sub.n_rows / B
         loss += f * lo
         g = f * go if g is None else g + f * go
-        if emulate:
-            ge = grads_bf16(w, sub, F, H, L, loss_kind, B_full=B, with_slack=True)
-            e = ge if e is None else (e[0] + ge[0], e[1] + ge[1])
+        ge = grads_bf16(w, sub, F, H, L, loss_kind, B_full=B, with_slack=True, rounding=emulate)
+        e = ge if e is None else (e[0] + ge[0], e[1] + ge[1])
     return loss, g, e
 
 
@@ -55,8 +54,8 @@ def _check_big(name, n_rows, precision, chunk, seed_pos=0, loss_kind="softmax", 
     assert abs(loss.item() - lo) <= tol * abs(lo)
     np.testing.assert_array_equal(touched, omodel.touched_features(batch))
     gg, og = split_grad(g.cpu().numpy(), cfg.F, cfg.H, cfg.L), split_grad(go, cfg.F, cfg.H, cfg.L)
-    eg = split_grad(em[0], cfg.F, cfg.H, cfg.L) if em is not None else None
-    es = split_grad(em[1], cfg.F, cfg.H, cfg.L) if em is not None else None
+    eg = split_grad(em[0], cfg.F, cfg.H, cfg.L) if precision == "bf16" else None
+    es = split_grad(em[1], cfg.F, cfg.H, cfg.L)
     check_grads(gg, og, tol, cfg.F, cfg.H, touched,
                 tag=f"{name}/{precision}/{loss_kind}/{'planted' if planted else 'init'}", emul=eg, slack=es)
 
