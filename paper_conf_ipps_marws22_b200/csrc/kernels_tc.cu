@@ -280,23 +280,39 @@ __device__ void dh_reduce_phase(const TcArgs& g, float* sred) {
     const int r0 = rb * n / GR, r1 = (rb + 1) * n / GR;
     const float lr = step_lr(g.meta);
     (void)lr;
-    for (int e = threadIdx.x; e < (r1 - r0) * nc; e += blockDim.x) {
-      const int r = r0 + e / nc, c = c0 + e % nc;
+    // float4 groups of 4 columns (column blocks are multiples of 32), all of a group's
+    // split-K partial loads in flight (16 per round), summed in split order
+    const int nc4 = nc / 4;
+    for (int e = threadIdx.x; e < (r1 - r0) * nc4; e += blockDim.x) {
+      const int rl = e / nc4, cl = 4 * (e % nc4);
+      const int r = r0 + rl, c = c0 + cl;
       const int64_t o = (int64_t)r * H + c;
-      float a[8];
+      float4 sum = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int z = 0; z < S; z += 16) {
+        float4 t[16];
 #pragma unroll
-      for (int q = 0; q < 8; ++q) a[q] = 0.f;
-      for (int z = 0; z < S; z += 8) {
+        for (int q = 0; q < 16; ++q)
+          t[q] = (z + q < S) ? __ldcg(reinterpret_cast<const float4*>(g.out + (int64_t)(z + q) * g.part_stride + o))
+                             : make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
-        for (int q = 0; q < 8; ++q)
-          if (z + q < S) a[q] += __ldcg(g.out + (int64_t)(z + q) * g.part_stride + o);
+        for (int q = 0; q < 16; ++q) {
+          sum.x += t[q].x; sum.y += t[q].y; sum.z += t[q].z; sum.w += t[q].w;
+        }
       }
-      float sum = ((a[0] + a[1]) + (a[2] + a[3])) + ((a[4] + a[5]) + (a[6] + a[7]));
-      if (g.dh_off) sum += g.dh_off[c];   // centred sigmoid dZ: + (1/(2B)) sum_j W2_j
-      const float v = g.h1[o] > 0.f ? sum : 0.f;
-      g.da1[o] = v;
-      if (g.da1b) g.da1b[o] = __float2bfloat16_rn(v);
-      sred[(e / nc) * nc + (e % nc)] = v;
+      if (g.dh_off) {   // centred sigmoid dZ: + (1/(2B)) sum_j W2_j
+        sum.x += g.dh_off[c]; sum.y += g.dh_off[c + 1]; sum.z += g.dh_off[c + 2]; sum.w += g.dh_off[c + 3];
+      }
+      const float4 hv = *reinterpret_cast<const float4*>(g.h1 + o);
+      const float4 v = make_float4(hv.x > 0.f ? sum.x : 0.f, hv.y > 0.f ? sum.y : 0.f,
+                                   hv.z > 0.f ? sum.z : 0.f, hv.w > 0.f ? sum.w : 0.f);
+      *reinterpret_cast<float4*>(g.da1 + o) = v;
+      if (g.da1b) {
+        __nv_bfloat162 p0 = __floats2bfloat162_rn(v.x, v.y), p1 = __floats2bfloat162_rn(v.z, v.w);
+        uint2 pk;
+        pk.x = *reinterpret_cast<uint32_t*>(&p0); pk.y = *reinterpret_cast<uint32_t*>(&p1);
+        *reinterpret_cast<uint2*>(g.da1b + o) = pk;
+      }
+      *reinterpret_cast<float4*>(sred + rl * nc + cl) = v;
     }
     __syncthreads();
     // column sums of the block, rows in order (one thread per column, 4 partial chains)

@@ -65,17 +65,16 @@ def check_grads(gg, og, tol, F, H, touched, tag="", emul=None, slack=None):
       The row RMS, not the tensor's: the tensor-core paths round operands, so an
       element's error scales with its row's summands (a head feature's W1 row is
       ~100x the typical one), not with the tensor's typical element.
-    fp32 path: the per-row and elementwise references r are the fp64 oracle.
-    bf16 path (emul = the split gradient of
-    tests/bf16_emul.py, the same mathematics with the kernels' bf16 rounding
-    points): r is that reference -- bf16 operand
+    With emul (the gradient of tests/bf16_emul.py: the same mathematics with the
+    kernels' rounding points -- bf16 operands, or the fp32 path's bf16x3 products),
+    r is that reference; without, the fp64 oracle.  bf16 operand
     rounding alone moves single W2 rows of the exact gradient by a few percent
     (see bf16_emul.py), so a localized bug is looked for against the rounded
     arithmetic, while the exact-gradient bar stays the normwise one.
     The achieved errors are returned and appended to $ASGD_PARITY_LOG (JSON
     lines) when that is set, so the margin under each bar is on record."""
     L = len(og["b2"])
-    rec = {"tag": tag, "tol": tol, "ref": "bf16-emulation" if emul is not None else "oracle"}
+    rec = {"tag": tag, "tol": tol, "ref": "rounding-emulation" if emul is not None else "oracle"}
     for k in ("W1", "b1", "W2", "b2"):
         rec[f"norm_{k}"] = float(normwise(gg[k], og[k]))
     ref = emul if emul is not None else og
@@ -94,7 +93,15 @@ def check_grads(gg, og, tol, F, H, touched, tag="", emul=None, slack=None):
         rec["kink_elems"] = int((sl["W1"] > 0).sum())
     for k, (a, b) in pairs.items():
         rec[f"elem_{k}"] = _elem_err(a, b, tol, per_row=True, slack=sl.get(k))
-    # where the worst W1 element sits (diagnostics for the log)
+    # where the worst W1 / W2 elements sit (diagnostics for the log)
+    if W2r.size:
+        d = np.abs(W2g - W2r)
+        rr = np.sqrt(np.mean(W2r * W2r, axis=1, keepdims=True))
+        q = d / (tol * np.abs(W2r) + tol * rr + 1e-300)
+        i, j = np.unravel_index(int(np.argmax(q)), q.shape)
+        rec["worst_W2"] = {"label": int(i), "col": int(j), "got": float(W2g[i, j]), "ref": float(W2r[i, j]),
+                           "row_rms": float(rr[i, 0]), "row_norm_got": float(np.linalg.norm(W2g[i])),
+                           "oracle": float(np.asarray(og["W2"]).reshape(L, H)[i, j])}
     if W1r.size:
         d = np.abs(W1g - W1r)
         if "W1" in sl:

@@ -63,3 +63,18 @@ def test_kink_slack_is_zero_away_from_the_kink():
     w2[o1 + 3] = -A1[3]                       # b1[3] cancels row 0's A1[:, 3]
     _, sl2 = bf16_emul.grads_bf16(w2, batch, cfg.F, cfg.H, cfg.L, with_slack=True)
     assert sl2[o1 + 3] > 0 and sl2[X.col[0] * cfg.H + 3] > 0
+
+
+def test_x3_mode_is_close_to_exact():
+    """bf16x3 products lose ~2^-16 relative: the x3 reference sits within 1e-4 of the
+    exact gradient (the fp32 path's bar) but is not the exact gradient."""
+    cfg = config("tiny")
+    data = generate(cfg, "train", 256)
+    batch = data.row_slice(np.arange(32))
+    w = planted_params(cfg).astype(np.float64)
+    _, go = model.loss_and_grad(w, batch, cfg.F, cfg.H, cfg.L)
+    for loss in ("softmax", "sigmoid"):
+        _, go = model.loss_and_grad(w, batch, cfg.F, cfg.H, cfg.L, loss)
+        g3 = bf16_emul.grads_bf16(w, batch, cfg.F, cfg.H, cfg.L, loss, rounding="x3")
+        e = np.linalg.norm(g3 - go) / np.linalg.norm(go)
+        assert 1e-9 < e < 2e-5, (loss, e)

@@ -49,12 +49,12 @@ def _check_big(name, n_rows, precision, chunk, seed_pos=0, loss_kind="softmax", 
     touched = rep.last_touched().cpu().numpy()
     batch = data.row_slice(rows)
     lo, go, em = _chunked_oracle(w0.astype(np.float64), batch, cfg.F, cfg.H, cfg.L, chunk, loss_kind,
-                                 emulate=precision == "bf16")
+                                 emulate="bf16" if precision == "bf16" else "x3")
     tol = TOL[precision]
     assert abs(loss.item() - lo) <= tol * abs(lo)
     np.testing.assert_array_equal(touched, omodel.touched_features(batch))
     gg, og = split_grad(g.cpu().numpy(), cfg.F, cfg.H, cfg.L), split_grad(go, cfg.F, cfg.H, cfg.L)
-    eg = split_grad(em[0], cfg.F, cfg.H, cfg.L) if precision == "bf16" else None
+    eg = split_grad(em[0], cfg.F, cfg.H, cfg.L)
     es = split_grad(em[1], cfg.F, cfg.H, cfg.L)
     check_grads(gg, og, tol, cfg.F, cfg.H, touched,
                 tag=f"{name}/{precision}/{loss_kind}/{'planted' if planted else 'init'}", emul=eg, slack=es)

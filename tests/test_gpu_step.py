@@ -29,7 +29,7 @@ def _one_step(cfg, data, rows, precision, lr=0.5, w0=None, b_max=None, loss_kind
     touched = rep.last_touched().cpu().numpy()
     batch = data.row_slice(rows)
     lo, go = omodel.loss_and_grad(np.asarray(w0, dtype=np.float64), batch, cfg.F, cfg.H, cfg.L, loss_kind)
-    em = grads_bf16(w0, batch, cfg.F, cfg.H, cfg.L, loss_kind, with_slack=True, rounding=precision == "bf16")
+    em = grads_bf16(w0, batch, cfg.F, cfg.H, cfg.L, loss_kind, with_slack=True, rounding="bf16" if precision == "bf16" else "x3")
     return rep, g.cpu().numpy(), float(loss.item()), touched, lo, (go, em), batch
 
 
@@ -39,7 +39,7 @@ def _check(cfg, rep, g, loss, touched, lo, go_em, batch, precision, tag=""):
     assert abs(loss - lo) <= tol * abs(lo), (loss, lo)
     np.testing.assert_array_equal(touched, omodel.touched_features(batch))
     gg, og = split_grad(g, cfg.F, cfg.H, cfg.L), split_grad(go, cfg.F, cfg.H, cfg.L)
-    eg = split_grad(em[0], cfg.F, cfg.H, cfg.L) if precision == "bf16" else None
+    eg = split_grad(em[0], cfg.F, cfg.H, cfg.L)
     es = split_grad(em[1], cfg.F, cfg.H, cfg.L)
     check_grads(gg, og, tol, cfg.F, cfg.H, touched, tag=f"{cfg.name}/{precision}/{tag}", emul=eg, slack=es)
     # W1 gradient is exactly zero off the touched rows
@@ -135,8 +135,8 @@ def test_teacher_forced_steps_tiny(precision):
         batch = data.row_slice(rows)
         _, go = omodel.loss_and_grad(w32.astype(np.float64), batch, cfg.F, cfg.H, cfg.L)
         gg, og = split_grad(g.cpu().numpy(), cfg.F, cfg.H, cfg.L), split_grad(go, cfg.F, cfg.H, cfg.L)
-        e_, s_ = grads_bf16(w32, batch, cfg.F, cfg.H, cfg.L, with_slack=True, rounding=precision == "bf16")
-        eg = split_grad(e_, cfg.F, cfg.H, cfg.L) if precision == "bf16" else None
+        e_, s_ = grads_bf16(w32, batch, cfg.F, cfg.H, cfg.L, with_slack=True, rounding="bf16" if precision == "bf16" else "x3")
+        eg = split_grad(e_, cfg.F, cfg.H, cfg.L)
         es = split_grad(s_, cfg.F, cfg.H, cfg.L)
         check_grads(gg, og, tol, cfg.F, cfg.H, omodel.touched_features(batch), tag=f"tiny/{precision}/tf{k}",
                     emul=eg, slack=es)
