@@ -75,6 +75,13 @@ int64_t fused_ce_bytes() {
 
 // G2 with the dH1 reduce + b1 update fused into its tail (default); ASGD_G2_FUSE=0: the
 // separate k_dh_reduce / k_b1_update launches (A/B).
+// K-3's dH1 half (k_bwd_dh) in the fused softmax-CE regime (default); ASGD_BWD_FUSE=0 keeps
+// G1b + G2 (A/B).
+bool bwd_fuse() {
+  static const bool v = [] { const char* e = getenv("ASGD_BWD_FUSE"); return !(e && e[0] == '0'); }();
+  return v;
+}
+
 bool g2_fuse() {
   static const bool v = [] { const char* e = getenv("ASGD_G2_FUSE"); return !(e && e[0] == '0'); }();
   return v;
@@ -553,6 +560,9 @@ int enqueue_step(asgd_ctx* c, int n) {
     if (2 * g2c <= c->sms) lc3.sms = c->sms - g2c;
     float2* zstat = reinterpret_cast<float2*>(c->ws + c->L.zstat);
     int ntiles = 0;
+    // K-3 (dH1 half): the fused softmax-CE regime on the bf16 path with H = 256
+    const bool k3 = bf && m.loss == ASGD_LOSS_SOFTMAX && (int64_t)m.b_max * Lb * 4 > fused_ce_bytes() && H == 256 &&
+                    bwd_fuse();
     if (x3) {
       // fp32 path: G1 stores Z (+ per-tile softmax partials), then the loss kernel writes dZ
       // as bf16x3 hi + lo (sigmoid: centred, R11 / R14)
@@ -587,13 +597,17 @@ int enqueue_step(asgd_ctx* c, int n) {
       // fused softmax-CE: G1 keeps only per-tile (max, sum exp); k_lse -> lse, row loss;
       // G1b recomputes Z tile by tile and writes dZ = (softmax - T)/B (bf16) -- Z never hits HBM
       PCU(ASGD_K_G1, launch_gemm_tc(lc, 5, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
-      PCU(ASGD_K_SOFTMAX, ([&]() -> cudaError_t {
-            cudaError_t e = launch_lse(lc, n, H, ntiles, c->L.stats_ld, zstat, P.rowsc, x.lab_ptr, x.lab, P.h1b,
-                                       Pr.w2b, b2, P);
-            return e != cudaSuccess ? e
-                                    : launch_gemm_tc(lc, 4, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr,
-                                                     nullptr, nullptr, P.rowsc, x.lab_ptr, x.lab);
-          })());
+      if (k3)   // lse only; dZ is formed inside k_bwd_dh (K-3)
+        PCU(ASGD_K_SOFTMAX, launch_lse(lc, n, H, ntiles, c->L.stats_ld, zstat, P.rowsc, x.lab_ptr, x.lab, P.h1b,
+                                       Pr.w2b, b2, P));
+      else
+        PCU(ASGD_K_SOFTMAX, ([&]() -> cudaError_t {
+              cudaError_t e = launch_lse(lc, n, H, ntiles, c->L.stats_ld, zstat, P.rowsc, x.lab_ptr, x.lab, P.h1b,
+                                         Pr.w2b, b2, P);
+              return e != cudaSuccess ? e
+                                      : launch_gemm_tc(lc, 4, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr,
+                                                       nullptr, nullptr, P.rowsc, x.lab_ptr, x.lab);
+            })());
     }
     const bool centred = m.loss == ASGD_LOSS_SIGMOID;   // G1 stored dZ - 1/(2B) (R11)
     auto g3 = [&](const Launch& l) {
@@ -610,7 +624,12 @@ int enqueue_step(asgd_ctx* c, int n) {
       CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
       PCU_ON(c->s3, ASGD_K_G3, g3(lc3));
     }
-    if (g2_fuse()) {
+    if (k3) {
+      // K-3: Z recomputed, dZ on chip into dH1 (+ TMA-stored for G3), dH1 reduce + b1 in the tail
+      const DhFuse fz{b1, g ? g + c->o_b1 : nullptr, nullptr, bf};
+      PCU(ASGD_K_G2, launch_bwd_dh(lc, n, Lb, H, Pr, c->L, b2, P.rowsc, x.lab_ptr, x.lab, fz, true));
+      CU(cudaEventRecord(c->ev_a, c->s3));
+    } else if (g2_fuse()) {
       // G2 + the dH1 reduce + ReLU' + b1 update + mean loss in one launch (grid barrier)
       const DhFuse fz{b1, g ? g + c->o_b1 : nullptr, centred ? P.cen : nullptr, bf};
       PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, nullptr, nullptr,

@@ -204,6 +204,12 @@ cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int 
                            const int32_t* dz_rows = nullptr, const int64_t* dz_lab_ptr = nullptr,
                            const int32_t* dz_lab = nullptr, const float* hoff = nullptr,
                            const DhFuse* fuse = nullptr);
+// K-3 (dH1 half): G1b + G2 + the dH1 reduce in one persistent kernel for the fused
+// softmax-CE regime (bf16, H = 256): Z tiles recomputed from the resident H1 block, dZ
+// formed on chip and fed straight into dH1 += dZ W2; write_dz also TMA-stores dZ for G3.
+cudaError_t launch_bwd_dh(const Launch&, int n, int64_t L, int H, const Ptrs&, const WsLayout&, float* b2,
+                          const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab, const DhFuse& fz,
+                          bool write_dz);
 // CTAs G2 runs with (the concurrent G3 leaves those SMs to it).
 int gemm_tc_g2_ctas(int n, int H, const WsLayout&, int sms);
 // which = 4 (G1b): dZ = (softmax - T)/B from a recomputed Z tile; needs P.lse from k_lse.

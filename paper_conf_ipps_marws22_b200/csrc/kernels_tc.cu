@@ -948,6 +948,242 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
   }
 }
 
+// ------------------------------------------------------------------ K-3 (dH1 half)
+// Fused output-layer backward for the fused softmax-CE regime (PAPER.md
+// P:1286-1309 fuses the element-wise work into the GEMMs): G1b + G2 + the dH1 reduce in
+// one persistent kernel, so the logits of a label tile never leave the SM on their way
+// into dH1.  CTA (label range lr, row block mb) keeps H1[mb] (128 x 256 bf16) resident and
+// sweeps its label tiles j (64 labels each, in increasing order):
+//   MMA 1   S     = H1_mb . W2_j^T                 (TMEM, 128 x 64, double-buffered)
+//   epi     dZ    = exp(S + b2 - lse) / B - T      (bf16, written K-major into smem)
+//   MMA 2   dH1  += dZ . W2_j                      (TMEM, 128 x 256; the SAME W2_j tile,
+//                                                  read MN-major)
+//   [dZ tile TMA-stored to global for G3 when g.write_z]
+// then its dH1 partial (over its label range) goes to dhpart[lr] and, after a grid
+// barrier, dh_reduce_phase sums the LR partials, applies ReLU' and updates b1.
+constexpr int kBwdBN = 64, kBwdEpi = 8, kBwdStages = 3;
+constexpr uint32_t kBwdH1Bytes = 4u * 16384u, kBwdW2Bytes = 4u * 8192u, kBwdDzBytes = 16384u;
+
+__global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
+    k_bwd_dh(const __grid_constant__ CUtensorMap tmH1, const __grid_constant__ CUtensorMap tmW2,
+             const __grid_constant__ CUtensorMap tmDZ, TcArgs g, int LR) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint8_t* sH1 = smem;
+  uint8_t* sW2 = sH1 + kBwdH1Bytes;
+  uint8_t* sDZ = sW2 + kBwdStages * kBwdW2Bytes;
+  float* sBias = reinterpret_cast<float*>(sDZ + 2 * kBwdDzBytes);          // [kBwdEpi][32]
+  uint64_t* w2full = reinterpret_cast<uint64_t*>(sBias + kBwdEpi * 32);
+  uint64_t* w2empty = w2full + kBwdStages;
+  uint64_t* sfull = w2empty + kBwdStages;
+  uint64_t* sempty = sfull + 2;
+  uint64_t* dzfull = sempty + 2;
+  uint64_t* dzempty = dzfull + 2;
+  uint64_t* hfull = dzempty + 2;
+  uint64_t* dhfull = hfull + 1;
+  uint32_t* tbase = reinterpret_cast<uint32_t*>(dhfull + 1);
+
+  pdl_trigger();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int MT = (g.M + BM - 1) / BM, T = (g.N + kBwdBN - 1) / kBwdBN;
+  const int mb = blockIdx.x % MT, lr = blockIdx.x / MT;
+  const int t0 = (int)((int64_t)lr * T / LR), t1 = (int)((int64_t)(lr + 1) * T / LR), nt = t1 - t0;
+  const int m0 = mb * BM;
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmH1)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW2)) : "memory");
+    for (int s = 0; s < kBwdStages; ++s) { mbar_init(&w2full[s], 1); mbar_init(&w2empty[s], 1); }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(&sfull[a], 1); mbar_init(&sempty[a], kBwdEpi);
+      mbar_init(&dzfull[a], kBwdEpi); mbar_init(&dzempty[a], 1);
+    }
+    mbar_init(hfull, 1);
+    mbar_init(dhfull, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 2) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tbase)), "r"(512)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tbase;
+  pdl_wait();
+
+  if (warp == 0) {
+    if (lane == 0 && nt > 0) {   // ------------------------------------ TMA producer
+      mbar_expect_tx(hfull, kBwdH1Bytes);
+      for (int kb = 0; kb < 4; ++kb) tma_load_2d(sH1 + kb * 16384, &tmH1, hfull, kb * 64, m0);
+      for (int i = 0; i < nt; ++i) {
+        const int st = i % kBwdStages;
+        mbar_wait(&w2empty[st], ((i / kBwdStages) & 1) ^ 1);
+        mbar_expect_tx(&w2full[st], kBwdW2Bytes);
+        for (int kb = 0; kb < 4; ++kb)
+          tma_load_2d(sW2 + st * kBwdW2Bytes + kb * 8192, &tmW2, &w2full[st], kb * 64, (t0 + i) * kBwdBN);
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && nt > 0) {   // ------------------------------------ MMA issuer
+      constexpr uint32_t idesc1 = make_idesc(kBwdBN, false, false);   // S = H1 W2_j^T
+      constexpr uint32_t idesc2 = make_idesc(256, false, true);       // dH1 += dZ W2_j
+      mbar_wait(hfull, 0);
+      for (int i = 0; i <= nt; ++i) {
+        if (i < nt) {
+          const int st = i % kBwdStages, acc = i & 1;
+          mbar_wait(&w2full[st], (i / kBwdStages) & 1);
+          mbar_wait(&sempty[acc], ((i >> 1) & 1) ^ 1);
+          tc_fence_after();
+          const uint32_t d = tmem + (uint32_t)(acc * kBwdBN);
+          const uint32_t wb = smem_u32(sW2 + st * kBwdW2Bytes);
+#pragma unroll
+          for (int kb = 0; kb < 4; ++kb)
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+              mma_bf16(d, desc_sw128(smem_u32(sH1 + kb * 16384) + k * 32, 16, 1024),
+                       desc_sw128(wb + kb * 8192 + k * 32, 16, 1024), idesc1, (kb | k) ? 1u : 0u);
+          mma_commit(&sfull[acc]);
+        }
+        if (i > 0) {
+          const int j = i - 1, st = j % kBwdStages, buf = j & 1;
+          mbar_wait(&dzfull[buf], (j >> 1) & 1);
+          tc_fence_after();
+          const uint32_t wb = smem_u32(sW2 + st * kBwdW2Bytes);
+          const uint32_t zb = smem_u32(sDZ + buf * kBwdDzBytes);
+#pragma unroll
+          for (int k = 0; k < kBwdBN / 16; ++k)
+            mma_bf16(tmem + 256, desc_sw128(zb + k * 32, 16, 1024), desc_sw128(wb + k * 2048, 8192, 1024), idesc2,
+                     (j > 0 || k > 0) ? 1u : 0u);
+          mma_commit(&dzempty[buf]);
+          mma_commit(&w2empty[st]);
+        }
+      }
+      mma_commit(dhfull);
+    }
+  } else if (warp >= 4) {   // -------------------------------------------- epilogue
+    const int q = (warp - 4) & 3, wh = (warp - 4) >> 2;
+    const int m = m0 + q * 32 + lane;
+    constexpr float kL2E = 1.4426950408889634f;
+    float crow = 0.f, tinv = 0.f;
+    int64_t lab_cur = 0, lab_end = 0;
+    if (m < g.M) {
+      crow = -g.lse[m] * kL2E - __log2f(1.f / g.invB);
+      const int64_t id = g.rows[m];
+      lab_cur = g.lab_ptr[id];
+      lab_end = g.lab_ptr[id + 1];
+      tinv = g.invB / (float)(lab_end - lab_cur);
+    }
+    int nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
+    float* bias_w = sBias + (warp - 4) * 32;
+    for (int i = 0; i < nt; ++i) {
+      const int acc = i & 1, buf = i & 1;
+      const int c = (t0 + i) * kBwdBN + wh * 32;        // this warp's first label column
+      __syncwarp();
+      bias_w[lane] = (c + lane < g.N) ? __ldg(g.bias + c + lane) * kL2E : 0.f;
+      __syncwarp();
+      while (nxt < c) {
+        ++lab_cur;
+        nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
+      }
+      mbar_wait(&sfull[acc], (i >> 1) & 1);
+      tc_fence_after();
+      float v[32];
+      tmem_ld32(tmem + (uint32_t)(acc * kBwdBN + wh * 32) + ((uint32_t)(q * 32) << 16), v);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sempty[acc]);
+      const float4* b4 = reinterpret_cast<const float4*>(bias_w);
+#pragma unroll
+      for (int qq = 0; qq < 8; ++qq) {
+        const float4 t = b4[qq];
+        v[4 * qq] = ex2_approx(fmaf(v[4 * qq], kL2E, t.x + crow));
+        v[4 * qq + 1] = ex2_approx(fmaf(v[4 * qq + 1], kL2E, t.y + crow));
+        v[4 * qq + 2] = ex2_approx(fmaf(v[4 * qq + 2], kL2E, t.z + crow));
+        v[4 * qq + 3] = ex2_approx(fmaf(v[4 * qq + 3], kL2E, t.w + crow));
+      }
+      if (c + 32 > g.N || m >= g.M) {   // padding columns / rows: dZ = 0
+#pragma unroll
+        for (int jj = 0; jj < 32; ++jj)
+          if (c + jj >= g.N || m >= g.M) v[jj] = 0.f;
+      }
+      while (nxt < c + 32) {            // the row's labels in this chunk: - 1/(|Y| B)
+        const int jy = nxt - c;
+#pragma unroll
+        for (int jj = 0; jj < 32; ++jj)
+          if (jj == jy) v[jj] -= tinv;
+        ++lab_cur;
+        nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
+      }
+      // the dZ buffer: MMA 2 of tile i - 2 done, and (write_z) its TMA store done reading
+      mbar_wait(&dzempty[buf], ((i >> 1) & 1) ^ 1);
+      if (g.write_z) {
+        if (warp == 4 && lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+        asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
+      }
+      uint8_t* rowp = sDZ + buf * kBwdDzBytes + (q * 32 + lane) * 128;
+      const int sw = (q * 32 + lane) & 7;
+#pragma unroll
+      for (int h = 0; h < 4; ++h) {     // 16-byte chunk wh * 4 + h of the row, 128B-swizzled
+        __nv_bfloat162 p0 = __floats2bfloat162_rn(v[8 * h], v[8 * h + 1]);
+        __nv_bfloat162 p1 = __floats2bfloat162_rn(v[8 * h + 2], v[8 * h + 3]);
+        __nv_bfloat162 p2 = __floats2bfloat162_rn(v[8 * h + 4], v[8 * h + 5]);
+        __nv_bfloat162 p3 = __floats2bfloat162_rn(v[8 * h + 6], v[8 * h + 7]);
+        uint4 pk;
+        pk.x = *reinterpret_cast<uint32_t*>(&p0); pk.y = *reinterpret_cast<uint32_t*>(&p1);
+        pk.z = *reinterpret_cast<uint32_t*>(&p2); pk.w = *reinterpret_cast<uint32_t*>(&p3);
+        *reinterpret_cast<uint4*>(rowp + (((wh * 4 + h) ^ sw) * 16)) = pk;
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      if (g.write_z) {
+        asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
+        if (warp == 4 && lane == 0) {
+          asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                           reinterpret_cast<uint64_t>(&tmDZ)), "r"(smem_u32(sDZ + buf * kBwdDzBytes)),
+                       "r"((t0 + i) * kBwdBN), "r"(m0)
+                       : "memory");
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&dzfull[buf]);
+    }
+    // this CTA's dH1 partial (rows m, columns wh * 128 .. + 127) -> dhpart[lr]
+    float* dst = g.out + (int64_t)lr * g.part_stride + (int64_t)m * g.ldo + wh * 128;
+    if (nt > 0) {
+      mbar_wait(dhfull, 0);
+      tc_fence_after();
+    }
+#pragma unroll 1
+    for (int ch = 0; ch < 4; ++ch) {
+      float v[32];
+      if (nt > 0) {
+        tmem_ld32(tmem + 256 + (uint32_t)(wh * 128 + ch * 32) + ((uint32_t)(q * 32) << 16), v);
+      } else {
+#pragma unroll
+        for (int jj = 0; jj < 32; ++jj) v[jj] = 0.f;
+      }
+      if (m < g.M) {
+#pragma unroll
+        for (int qq = 0; qq < 8; ++qq)
+          *reinterpret_cast<float4*>(dst + ch * 32 + 4 * qq) =
+              make_float4(v[4 * qq], v[4 * qq + 1], v[4 * qq + 2], v[4 * qq + 3]);
+      }
+    }
+    if (warp == 4 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512) : "memory");
+  }
+  __threadfence();
+  TcArgs gt = g;    // the tail reduces H columns: N = H there
+  gt.N = g.K;
+  dh_reduce_phase(gt, reinterpret_cast<float*>(smem));
+}
+
 // ------------------------------------------------------------------ host side
 PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 std::once_flag g_once;
@@ -1159,6 +1395,35 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
   }
   if (bn == 128) return run<128, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
   return run<64, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
+}
+
+cudaError_t launch_bwd_dh(const Launch& lc, int n, int64_t L, int H, const Ptrs& P, const WsLayout& W, float* b2,
+                          const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab, const DhFuse& fz,
+                          bool write_dz) {
+  if (!tc_available()) return cudaErrorNotSupported;
+  if (H != 256 || P.w2l) return cudaErrorNotSupported;   // bf16 path, H = 256 (one N = 256 MMA)
+  const int64_t Lp = padded_ld(L);
+  const int MT = (n + BM - 1) / BM;
+  const int64_t T = (L + kBwdBN - 1) / kBwdBN;
+  const int LR = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)(lc.sms / MT), T, (int64_t)W.splitk}));
+  CUtensorMap th, tw, tz;
+  cudaError_t e;
+  if ((e = make_map(&th, P.h1b, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
+  if ((e = make_map(&tw, P.w2b, H, L, (uint64_t)H * 2, 64, kBwdBN)) != cudaSuccess) return e;
+  if ((e = make_map(&tz, P.dzb, L, n, (uint64_t)Lp * 2, kBwdBN, BM)) != cudaSuccess) return e;
+  TcArgs g{};
+  g.M = n; g.N = (int)L; g.K = H;
+  g.out = P.dhpart; g.ldo = H; g.part_stride = W.part_stride; g.splits = LR;
+  g.bias = b2; g.lse = P.lse; g.rows = rows; g.lab_ptr = lab_ptr; g.lab = lab; g.invB = 1.f / (float)n;
+  g.write_z = write_dz ? 1 : 0;
+  g.dh_fuse = 1; g.meta = P.meta;
+  g.h1 = P.h1; g.da1 = P.da1; g.da1b = fz.want_bf16 ? P.da1b : nullptr; g.dh_off = fz.dh_off;
+  g.b1 = fz.b1; g.grad_b1 = fz.grad_b1; g.colpart = P.db1part; g.rowloss = P.rowloss;
+  g.bar = P.meta + M_G2BAR;
+  const size_t smem = kBwdH1Bytes + kBwdStages * kBwdW2Bytes + 2 * kBwdDzBytes + kBwdEpi * 32 * 4 + 1024 + 256;
+  if ((e = ensure_smem(k_bwd_dh, smem)) != cudaSuccess) return e;
+  return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_bwd_dh, dim3(MT * LR), dim3(128 + 32 * kBwdEpi), smem, th,
+                      tw, tz, g, LR);
 }
 
 }  // namespace asgd

@@ -25,18 +25,29 @@ product and sum in fp64:
                      centred fp32 value) is split the same way; db2 = 1^T (hi + lo)
                      of dZ; dW1 = X^T dA1 with fp32 dA1; the centred-sigmoid offsets
                      use the fp32 W2 and H1.
-What is left between it and the kernels is fp32 accumulation order, ex2.approx,
-the rare element whose fp32 value sits at a bf16 rounding midpoint, the ReLU
-mask where the GPU's fp32 A1 and the fp64 one straddle zero, and the fp32
-accumulation of dH1 over the L labels.  `slack` bounds the last two, per element
-of dW1 and db1:
-  * kink: every (n, h) with |A1_nh| within the fp32 SpMM error bound
-    (s_n 2^-24 sum_f |x_nf| |W1_fh| + 2^-24 |b1_h|, s_n = the row's nnz) may go
-    either way, moving dW1[f, h] by at most |x_nf| |dH1_nh| (1 + 2^-7) and db1[h]
-    by |dH1_nh|;
-  * accumulation: |fl(dH1_nh) - dH1_nh| <= 4 sqrt(L) 2^-24 sum_j |dZ_nj| |W2_jh|
-    (a 4-sigma bound of the fp32 rounding walk over L terms; it matters only where
-    the sum cancels), carried to dW1 and db1 through the mask and |x_nf|."""
+What is left between the reference and the kernels are decisions the two sides
+may take differently: the GPU's fp32 A1 (K-1) straddling the ReLU kink or a bf16
+rounding midpoint where the fp64 one does not, its fp32 Z / lse / exp moving p
+by a few ulps (and through that a dZ rounding), and fp32 accumulation orders.
+With `with_slack` the function also returns a first-order componentwise bound of
+what those can move, per element of dW1, db1, dW2 and db2 (slack below), so the
+elementwise check can stay at the tolerance everywhere else.  R(.) is the
+rounding the path applies to a GEMM operand (bf16; the bf16x3 hi + lo; or none),
+flip(q, d) = max over q' in [q - d, q + d] of |R(q') - R(q)| (exact, elementwise),
+u = 2^-24:
+  dH  = flip(H1, eA1),  eA1 = s_n u sum_f |x_nf||W1_fh| + u |b1_h|   (K-1's fp32 sum)
+  dZl = dH |Wq|^T + 256 u |Hq||Wq|^T                     (logits; fp32 accumulation, K = H)
+  dp  = p (dZl + max_j dZl + 4e-6)                        (softmax: the lse error follows
+                                                          the max logit error; 4e-6: fp32 exp/log)
+        sigmoid: dZl / 4
+  ddZ = flip(dZ, dp / B + u |dZ|)
+  dW2 : ddZ^T |Hq| + |dZq|^T dH + B u |dZq|^T |Hq|
+  db2 : sum_n ddZ + B u sum_n |dZq|
+  dH1 : ddZ |Wq| + 4 sqrt(L) u |dZq| |Wq|               (a 4-sigma bound of the fp32
+                                                          rounding walk over L labels)
+  dA1 : [A1 > 0] dH1-error + [|A1| <= eA1] (|dH1| + its error)   (the kink)
+  dW1 : |X|^T flip(dA1, dA1-error) + B u |X|^T |dA1|;   db1: sum_n dA1-error + B u sum_n |dA1|
+"""
 import numpy as np
 import scipy.sparse as sp
 
@@ -125,12 +136,48 @@ def grads_bf16(w, batch, F, H, L, loss="softmax", B_full=None, with_slack=False,
     g = np.concatenate([dW1.ravel(), db1, dW2.ravel(), db2])
     if not with_slack:
         return g
+    return g, _slack(mode, X, W1, b1, A1, H1, Hq, Wq, W2, Z, dZ, dH1, dA1, B, L, F, H, loss,
+                     P if loss == "softmax" else S)
+
+
+def _rnd(mode):
+    if mode == "bf16":
+        return bf16
+    if mode == "x3":
+        return lambda x: sum(split3(x))
+    return lambda x: np.asarray(x, dtype=np.float64)
+
+
+def _flip(mode, q, d):
+    """max |R(q') - R(q)| over q' in [q - d, q + d] (R monotone: the two ends)."""
+    if mode == "exact":
+        return np.asarray(d, dtype=np.float64)
+    R = _rnd(mode)
+    r0 = R(q)
+    return np.maximum(np.abs(R(q + d) - r0), np.abs(R(q - d) - r0))
+
+
+def _slack(mode, X, W1, b1, A1, H1, Hq, Wq, W2, Z, dZ, dH1, dA1, B, L, F, H, loss, P):
+    u = 2.0 ** -24
     Xa = abs(X)
-    nnz_row = np.diff(batch.row_ptr).astype(np.float64)[:, None]
-    bound = nnz_row * 2.0 ** -24 * np.asarray(Xa @ np.abs(W1)) + 2.0 ** -24 * np.abs(b1)[None, :]
-    kink = (np.abs(A1) <= bound) * np.abs(dH1) * (1 + 2.0 ** -7)
-    acc = 4.0 * np.sqrt(L) * 2.0 ** -24 * (np.abs(dZ) @ np.abs(Wq)) * (A1 > 0.0) * (1 + 2.0 ** -7)
-    sl = np.zeros_like(g)
-    sl[:F * H] = np.asarray(Xa.T @ (kink + acc)).ravel()
-    sl[F * H:F * H + H] = (kink + acc).sum(axis=0)
-    return g, sl
+    n = X.shape[0]
+    nnz_row = np.diff(X.indptr).astype(np.float64)[:, None]
+    eA1 = nnz_row * u * np.asarray(Xa @ np.abs(W1)) + u * np.abs(b1)[None, :]
+    dH = _flip(mode, H1, eA1) * (A1 > -eA1)
+    aH, aW = np.abs(Hq), np.abs(Wq)
+    dZl = dH @ aW.T + 256 * u * (aH @ aW.T)
+    if loss == "softmax":
+        dp = P * (dZl + dZl.max(axis=1, keepdims=True) + 4e-6)
+    else:
+        dp = dZl / 4.0
+    ddZ = _flip(mode, dZ, dp / B + u * np.abs(dZ))
+    aZ = np.abs(dZ)
+    s_W2 = ddZ.T @ aH + aZ.T @ dH + B * u * (aZ.T @ aH)
+    s_b2 = ddZ.sum(axis=0) + B * u * aZ.sum(axis=0)
+    e_dH1 = ddZ @ aW + 4.0 * np.sqrt(L) * u * (aZ @ aW)
+    kink = np.abs(A1) <= eA1
+    e_dA1 = (A1 > 0.0) * e_dH1 + kink * (np.abs(dH1) + e_dH1)
+    k5 = _flip("bf16" if mode == "bf16" else "exact", dA1, e_dA1) if mode == "bf16" else e_dA1 + u * np.abs(dA1)
+    s_W1 = np.asarray(Xa.T @ k5) + B * u * np.asarray(Xa.T @ np.abs(dA1))
+    s_b1 = e_dA1.sum(axis=0) + B * u * np.abs(dA1).sum(axis=0)
+    return np.concatenate([s_W1.ravel(), s_b1, s_W2.ravel(), s_b2])

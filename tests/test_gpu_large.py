@@ -34,11 +34,11 @@ def _chunked_oracle(w, batch, F, H, L, chunk, loss_kind="softmax", emulate=False
     return loss, g, e
 
 
-def _check_big(name, n_rows, precision, chunk, seed_pos=0, loss_kind="softmax", planted=False):
+def _check_big(name, n_rows, precision, chunk, seed_pos=0, loss_kind="softmax", planted=False, batch=None):
     cfg = config(name)
     data = dataset(name, n_rows)
     cfg_sub = config(name, n_train=data.n_rows)
-    rows = sample_stream(cfg_sub, seed_pos, cfg.b_max)
+    rows = sample_stream(cfg_sub, seed_pos, batch or cfg.b_max)
     w0 = planted_params(cfg) if planted else init_params(cfg)
     rep = make_replica(cfg, data, precision, w0=w0, loss=loss_kind)
     g = torch.zeros(rep.P, dtype=torch.float32, device="cuda")
@@ -105,3 +105,10 @@ def test_delicious200k_planted_state():
 
 def test_wiki10_planted_state():
     _check_big("wiki10_31k", None, "bf16", chunk=256, seed_pos=20 * 14146 + 5, planted=True)
+
+
+def test_amazoncat_ragged_batch_k3():
+    """A 300-row batch at the AmazonCat shape (fused softmax-CE regime, K-3's k_bwd_dh):
+    the last 128-row block is partial (44 rows) and L = 13,330 ends in a partial 64-label
+    tile; planted (peaked) state."""
+    _check_big("amazoncat13k", 32768, "bf16", chunk=300, seed_pos=7 * 32768 + 11, planted=True, batch=300)
