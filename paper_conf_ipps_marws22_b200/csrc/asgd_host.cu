@@ -628,26 +628,27 @@ int enqueue_step(asgd_ctx* c, int n) {
       // K-3: Z recomputed, dZ on chip into dH1 (+ TMA-stored for G3), dH1 reduce + b1 in the tail
       const DhFuse fz{b1, g ? g + c->o_b1 : nullptr, nullptr, bf};
       PCU(ASGD_K_G2, launch_bwd_dh(lc, n, Lb, H, Pr, c->L, b2, P.rowsc, x.lab_ptr, x.lab, fz, true));
-      CU(cudaEventRecord(c->ev_a, c->s3));
     } else if (g2_fuse()) {
       // G2 + the dH1 reduce + ReLU' + b1 update + mean loss in one launch (grid barrier)
       const DhFuse fz{b1, g ? g + c->o_b1 : nullptr, centred ? P.cen : nullptr, bf};
       PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, nullptr, nullptr,
                                     nullptr, nullptr, nullptr, nullptr, &fz));
-      CU(cudaEventRecord(c->ev_a, c->s3));
     } else {
       PCU(ASGD_K_G2, launch_gemm_tc(lc, 2, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr));
       PCU(ASGD_K_DH, launch_dh_reduce(lc, n, H, (int)c->L.splitk, P, c->L, bf, centred ? P.cen : nullptr));
       CU(cudaEventRecord(c->ev_dh, c->s));
       CU(cudaStreamWaitEvent(c->s3, c->ev_dh, 0));
       PCU_ON(c->s3, ASGD_K_DH, launch_b1_update(lc3, n, H, b1, P, c->L, g ? g + c->o_b1 : nullptr));
-      CU(cudaEventRecord(c->ev_a, c->s3));
     }
+    // join s3 back into s only when work went there (an event recorded on a stream outside
+    // the capture cannot be waited on inside it)
+    const bool s3_used = g3_side || !(k3 || g2_fuse());
+    if (s3_used) CU(cudaEventRecord(c->ev_a, c->s3));
     // K-5 (needs K-0's segments)
     CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
     PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
     if (!g3_side) PCU(ASGD_K_G3, g3(lc));
-    CU(cudaStreamWaitEvent(c->s, c->ev_a, 0));
+    if (s3_used) CU(cudaStreamWaitEvent(c->s, c->ev_a, 0));
   }
   return ASGD_OK;
 }

@@ -21,6 +21,8 @@ def kclass(name: str):
     if name.startswith("k_gemm_tc"):
         epi = int(re.findall(r"\d+", name.split("<")[1])[-1])
         return {0: "g1", 1: "g2", 2: "g3", 3: "softmax", 4: "g1", 5: "g1"}[epi]   # 4: sigmoid G1, 5: stats G1
+    if name.startswith("k_bwd_dh"):
+        return "g2"   # K-3's dH1 half (G1b + G2 + dH reduce): profiled as G2
     for pre, cls in (("k_touched", "touched"), ("k_spmm_fwd", "spmm"), ("k_softmax_ce", "softmax"),
                      ("k_lse", "softmax"), ("k_dh_reduce", "dh_b1"), ("k_b1_update", "dh_b1"),
                      ("k_scatter_sgd", "scatter"), ("k_sqnorm", "merge"), ("k_scale", "merge"),
