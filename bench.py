@@ -136,11 +136,7 @@ def cpu_baseline(cfg, data, budget_s: float, loss: str = "softmax"):
     amortised over the mega-batch's 100 steps."""
     from oracle import merge as omerge, model as omodel
     from synth import init_params, sample_stream
-    try:
-        from threadpoolctl import threadpool_info
-        cores = max([i.get("num_threads", 1) for i in threadpool_info()] + [1])
-    except Exception:
-        cores = os.cpu_count()
+    cores, cpu_model, blas_threads = host_cores()
     w = init_params(cfg).astype(np.float64)
     b = cfg.b_max
     steps, samples = 0, 0
@@ -159,8 +155,28 @@ def cpu_baseline(cfg, data, budget_s: float, loss: str = "softmax"):
     steps_per_mb = cfg.mega_batch // b
     t_total = t_steps + t_merge * steps / steps_per_mb
     return {"value": samples / t_total, "unit": UNIT, "cores": int(cores), "kind": "oracle",
+            "cpu_model": cpu_model, "blas_threads": blas_threads,
             "sample": f"{steps} local steps x {b} rows of {cfg.name} (fp64 numpy/scipy oracle) + "
                       f"merge amortised over {steps_per_mb} steps/mega-batch"}, t_total
+
+
+def host_cores():
+    """the cores the oracle may use = len(os.sched_getaffinity(0)), the
+    CPU model from lscpu, and the BLAS thread pool size actually in use."""
+    cores = len(os.sched_getaffinity(0))
+    model = None
+    try:
+        import subprocess
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        model = next((ln.split(":", 1)[1].strip() for ln in out.splitlines() if ln.startswith("Model name")), None)
+    except Exception:
+        pass
+    try:
+        from threadpoolctl import threadpool_info
+        blas = max([i.get("num_threads", 1) for i in threadpool_info()] + [1])
+    except Exception:
+        blas = None
+    return cores, model, blas
 
 
 # ------------------------------------------------------------------ roofline
@@ -625,17 +641,20 @@ def reference_arm(a, rank, world):
     cfg = config(a.config)
     data = generate(cfg, "train")
     per_step = max(1.0, min(a.cpu_seconds, 20.0) / max(1, a.steps))
-    vals = []
+    vals, secs = [], []
     base = None
     for k in range(a.warmup + a.steps):
-        cb, _ = cpu_baseline(cfg, data, per_step, a.loss)
+        cb, t_s = cpu_baseline(cfg, data, per_step, a.loss)
         if k >= a.warmup:
             vals.append(cb["value"])
+            secs.append(t_s)
             base = cb
     v = float(np.mean(vals))
     base["value"] = round(v, 2)
+    # a timed step is one bounded sample of the workload (cpu_baseline's budget), its wall time
     out = {"metric": METRIC, "value": round(v, 2), "unit": UNIT, "n_gpus": world, "steps": a.steps,
-           "warmup": a.warmup, "ms_per_step": None, "higher_is_better": True, "scaling": "strong",
+           "warmup": a.warmup, "ms_per_step": round(1e3 * float(np.mean(secs)), 3), "higher_is_better": True,
+           "scaling": "strong",
            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
            "config": {"workload": cfg.name, "F": cfg.F, "L": cfg.L, "H": cfg.H, "b_max": cfg.b_max,
                       "mega_batch_samples": cfg.mega_batch, "loss": a.loss},

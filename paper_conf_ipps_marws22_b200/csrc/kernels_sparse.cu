@@ -391,7 +391,10 @@ __global__ void __launch_bounds__(512) k_touched(StepArgs sa, const int64_t* __r
 // K-1: A1 = X W1 + b1, H1 = ReLU(A1)
 // -------------------------------------------------------------------------
 #ifndef ASGD_K1_GROUP
-#define ASGD_K1_GROUP 16   // measured (8 / 16 / per-piece partials): EURLex 3.64 / 4.02 / 4.02 M, Wiki10 1.30 / 1.35 / 1.27 M samples/s
+// warps per K-1 CTA = the largest group.  Round 1 (fixed 16-piece groups, 117 of 148 CTAs busy
+// at EURLex): 8 / 16 -> 3.64 / 4.02 M samples/s.  Round 2, groups sized to the batch (gs):
+// 8 / 16 -> 4.14 / 4.05 M (8-warp CTAs, two per SM, 235 groups of 8 pieces)
+#define ASGD_K1_GROUP 8
 #endif
 template <int VPL>   // pieces per group = warps per K-1 CTA (H = 512: 8, the partials fill 32 KB)
 constexpr int k1_group() { return VPL >= 16 ? 8 : ASGD_K1_GROUP; }
@@ -935,6 +938,111 @@ __global__ void __launch_bounds__(scatter_threads<T, CPL>(), 1) k_scatter_sgd_s(
   wait_staged();   // no CTA exits with its bulk copy still writing shared memory
 }
 
+// K-5, segment-per-warp variant: warp w owns whole feature segments u = w, w + W, ...
+// (K-0's entries of feature uniq[u], sorted by row), so no segment is split across warps:
+// no partials, no atomics, no fences.  The W1 row slice is requested when the segment
+// starts and its latency hides under the segment's gathers from the staged dA1 slice;
+// the sum runs in the segment's (row) order, so it is deterministic.  A segment has at
+// most B entries (one per batch row), which bounds the per-warp imbalance.
+template <typename T, int CPL>
+__global__ void __launch_bounds__(scatter_threads<T, CPL>(), 1)
+    k_scatter_seg(const int32_t* __restrict__ e_n, const float* __restrict__ e_v,
+                  const int32_t* __restrict__ useg, const int32_t* __restrict__ uniq,
+                  const int32_t* __restrict__ meta, const T* __restrict__ dA1, int H, float* W1,
+                  float* grad_w1, int32_t* fcnt, uint32_t* bits, int W) {
+  pdl_trigger();
+  pdl_wait();
+  const float lr = step_lr(meta);
+  constexpr int CS = 32 * CPL;
+  extern __shared__ __align__(16) uint8_t sm_raw[];
+  T* sd = reinterpret_cast<T*>(sm_raw);      // [n][CS]
+  const int nsl = gridDim.y, slice = blockIdx.y, c0 = slice * CS;
+  const int n = meta[M_NROWS];
+  __shared__ __align__(8) uint64_t sbar;
+  const uint32_t bar = static_cast<uint32_t>(__cvta_generic_to_shared(&sbar));
+  const uint32_t row_bytes = CS * (uint32_t)sizeof(T);
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"((uint32_t)n * row_bytes)
+                 : "memory");
+  }
+  __syncthreads();
+  {
+    const uint32_t dst0 = static_cast<uint32_t>(__cvta_generic_to_shared(sd));
+    if (nsl == 1) {
+      if (threadIdx.x == 0 && n > 0)
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst0),
+                     "l"(dA1), "r"((uint32_t)n * row_bytes), "r"(bar)
+                     : "memory");
+    } else {
+      for (int r = threadIdx.x; r < n; r += blockDim.x)
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                         dst0 + (uint32_t)r * row_bytes),
+                     "l"(dA1 + (int64_t)r * H + c0), "r"(row_bytes), "r"(bar)
+                     : "memory");
+    }
+  }
+  const int lane = threadIdx.x & 31;
+  const int U = meta[M_U];
+  const int nwarps = gridDim.x * (blockDim.x >> 5);
+  using IO = SliceIO<T, CPL>;
+  bool staged = false;
+  for (int u = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); u < U; u += nwarps) {
+    const int j0 = useg[u], j1 = useg[u + 1];
+    const int f = uniq[u];
+    float* wrow = W1 + (int64_t)f * H + c0 + lane * CPL;
+    float w[CPL];
+    ld_cols<CPL>(wrow, w, false);                 // in flight during the gathers
+    if (!staged) {
+      uint32_t ok = 0;
+      while (!ok)
+        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                     : "=r"(ok) : "r"(bar) : "memory");
+      staged = true;
+    }
+    float acc[CPL];
+#pragma unroll
+    for (int i = 0; i < CPL; ++i) acc[i] = 0.f;
+    for (int jb = j0; jb < j1; jb += 32) {
+      const int cnt = min(32, j1 - jb);
+      int myn = 0;
+      float myv = 0.f;
+      if (lane < cnt) { myn = e_n[jb + lane]; myv = e_v[jb + lane]; }
+      int j = 0;
+      for (; j + 8 <= cnt; j += 8) {
+        float g[8][CPL];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) IO::load(sd + (int64_t)__shfl_sync(kFull, myn, j + q) * CS, lane, g[q]);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          const float v = __shfl_sync(kFull, myv, j + q);
+#pragma unroll
+          for (int i = 0; i < CPL; ++i) acc[i] = fmaf(v, g[q][i], acc[i]);
+        }
+      }
+      for (; j < cnt; ++j) {
+        float g[CPL];
+        IO::load(sd + (int64_t)__shfl_sync(kFull, myn, j) * CS, lane, g);
+        const float v = __shfl_sync(kFull, myv, j);
+#pragma unroll
+        for (int i = 0; i < CPL; ++i) acc[i] = fmaf(v, g[i], acc[i]);
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < CPL; ++i) w[i] = w[i] - lr * acc[i];
+    st_cols<CPL>(wrow, w, false);
+    if (grad_w1) st_cols<CPL>(grad_w1 + (int64_t)f * H + c0 + lane * CPL, acc, false);
+    if (slice == 0) reset_feature(fcnt, bits, W, f, lane);
+  }
+  if (!staged) {   // no CTA exits with its bulk copy still writing shared memory
+    uint32_t ok = 0;
+    while (!ok)
+      asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                   : "=r"(ok) : "r"(bar) : "memory");
+  }
+}
+
 // One resident wave of 256-thread CTAs (occupancy from the compiled kernel), no
 // more CTAs than there are 8-piece groups for the largest step.
 template <typename K>
@@ -1030,15 +1138,27 @@ constexpr int nargs_of(void (*)(A...)) { return (int)sizeof...(A); }
 int spmm_fwd_nargs() { return nargs_of(k_spmm_fwd<8>); }
 int touched_nargs() { return nargs_of(k_touched); }
 
+// K-5 layout: ASGD_K5_SEG=1 -> one warp per feature segment (k_scatter_seg), else nnz pieces
+bool k5_seg() {
+  static const bool v = [] { const char* e = getenv("ASGD_K5_SEG"); return e && e[0] == '1'; }();
+  return v;
+}
+
 template <typename T, int CPL>
 cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float* W1,
                         const Ptrs& P, float* grad_w1) {
   constexpr int CS = 32 * CPL;
   const int nsl = H / CS;
   const size_t smem = (size_t)b_max * CS * sizeof(T);
+  const int gx = std::max(1, lc.sms / nsl);
+  if (k5_seg()) {
+    cudaError_t e = ensure_smem(k_scatter_seg<T, CPL>, 200 * 1024);
+    if (e != cudaSuccess) return e;
+    return launch_k(lc, k_scatter_seg<T, CPL>, dim3(gx, nsl), dim3(scatter_threads<T, CPL>()), smem, P.e_n, P.e_v,
+                    P.useg, P.uniq, P.meta, dA1, H, W1, grad_w1, P.cnt, P.bits, (b_max + 31) / 32);
+  }
   cudaError_t e = ensure_smem(k_scatter_sgd_s<T, CPL>, 200 * 1024);
   if (e != cudaSuccess) return e;
-  const int gx = std::max(1, lc.sms / nsl);
   return launch_k(lc, k_scatter_sgd_s<T, CPL>, dim3(gx, nsl), dim3(scatter_threads<T, CPL>()), smem, P.e_n, P.e_v, P.e_u,
                   P.e_f, P.useg, P.meta, dA1, H, W1, P.part5, P.ucnt, grad_w1, P.cnt, P.bits,
                   (b_max + 31) / 32);
