@@ -79,6 +79,11 @@ bool bwd_fuse() {
   static const bool v = [] { const char* e = getenv("ASGD_BWD_FUSE"); return !(e && e[0] == '0'); }();
   return v;
 }
+// K-3's dW2 half (k_bwd_dw, replaces G3 there and dZ never reaches HBM) -- ASGD_BWD_DW=0: G3
+bool bwd_dw() {
+  static const bool v = [] { const char* e = getenv("ASGD_BWD_DW"); return !(e && e[0] == '0'); }();
+  return v;
+}
 
 // G2 with the dH1 reduce + b1 update fused into its tail (ASGD_G2_FUSE=1).  Off by default:
 // measured on EURLex-4K (bf16) 6.99 ms vs 6.30 ms per mega-batch -- the tail's grid barrier
@@ -565,6 +570,7 @@ int enqueue_step(asgd_ctx* c, int n) {
     // K-3 (dH1 half): the fused softmax-CE regime on the bf16 path with H = 256
     const bool k3 = bf && m.loss == ASGD_LOSS_SOFTMAX && (int64_t)m.b_max * Lb * 4 > fused_ce_bytes() && H == 256 &&
                     bwd_fuse();
+    const bool k3dw = k3 && bwd_dw() && n <= 1024;
     if (x3) {
       // fp32 path: G1 stores Z (+ per-tile softmax partials), then the loss kernel writes dZ
       // as bf16x3 hi + lo (sigmoid: centred, R11 / R14)
@@ -613,6 +619,9 @@ int enqueue_step(asgd_ctx* c, int n) {
     }
     const bool centred = m.loss == ASGD_LOSS_SIGMOID;   // G1 stored dZ - 1/(2B) (R11)
     auto g3 = [&](const Launch& l) {
+      if (k3dw)   // K-3's dW2 half: Z^T recomputed, dZ^T on chip, W2 / b2 SGD
+        return launch_bwd_dw(l, n, Lb, H, Pr, Pw, W2, b2, P.rowsc, x.lab_ptr, x.lab, g ? g + c->o_w2 : nullptr,
+                             g ? g + c->o_b2 : nullptr);
       return launch_gemm_tc(l, 3, n, Lb, H, Pw, c->L, W2, b2, g ? g + c->o_w2 : nullptr, g ? g + c->o_b2 : nullptr,
                             nullptr, nullptr, nullptr, nullptr, nullptr, centred ? P.cen + H : nullptr);
     };
@@ -629,7 +638,7 @@ int enqueue_step(asgd_ctx* c, int n) {
     if (k3) {
       // K-3: Z recomputed, dZ on chip into dH1 (+ TMA-stored for G3), dH1 reduce + b1 in the tail
       const DhFuse fz{b1, g ? g + c->o_b1 : nullptr, nullptr, bf};
-      PCU(ASGD_K_G2, launch_bwd_dh(lc, n, Lb, H, Pr, c->L, b2, P.rowsc, x.lab_ptr, x.lab, fz, true));
+      PCU(ASGD_K_G2, launch_bwd_dh(lc, n, Lb, H, Pr, c->L, b2, P.rowsc, x.lab_ptr, x.lab, fz, !k3dw));
     } else if (g2_fuse()) {
       // G2 + the dH1 reduce + ReLU' + b1 update + mean loss in one launch (grid barrier)
       const DhFuse fz{b1, g ? g + c->o_b1 : nullptr, centred ? P.cen : nullptr, bf};

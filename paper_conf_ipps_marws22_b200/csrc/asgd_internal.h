@@ -210,6 +210,11 @@ cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int 
 cudaError_t launch_bwd_dh(const Launch&, int n, int64_t L, int H, const Ptrs&, const WsLayout&, float* b2,
                           const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab, const DhFuse& fz,
                           bool write_dz);
+// K-3 (dW2 half): G1b + G3 in one persistent kernel: per W2 row tile, Z^T recomputed per row
+// chunk, dZ^T on chip into dW2, then W2 / b2 SGD and the next bf16 shadow (Pw.w2b).
+cudaError_t launch_bwd_dw(const Launch&, int n, int64_t L, int H, const Ptrs& Pr, const Ptrs& Pw, float* W2,
+                          float* b2, const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab,
+                          float* grad_w2, float* grad_b2);
 // CTAs G2 runs with (the concurrent G3 leaves those SMs to it).
 int gemm_tc_g2_ctas(int n, int H, const WsLayout&, int sms);
 // which = 4 (G1b): dZ = (softmax - T)/B from a recomputed Z tile; needs P.lse from k_lse.

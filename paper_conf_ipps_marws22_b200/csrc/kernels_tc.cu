@@ -1076,12 +1076,20 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
     }
     int nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
     float* bias_w = sBias + (warp - 4) * 32;
+    // b2 of the next tile's columns, loaded one tile ahead (its latency hides under this
+    // tile's epilogue instead of heading it: the top stall site in ncu before)
+    auto b2_of = [&](int i) {
+      const int cc = (t0 + i) * kBwdBN + wh * 32 + lane;
+      return (i < nt && cc < g.N) ? __ldg(g.bias + cc) * kL2E : 0.f;
+    };
+    float bnext = b2_of(0);
     for (int i = 0; i < nt; ++i) {
       const int acc = i & 1, buf = i & 1;
       const int c = (t0 + i) * kBwdBN + wh * 32;        // this warp's first label column
       __syncwarp();
-      bias_w[lane] = (c + lane < g.N) ? __ldg(g.bias + c + lane) * kL2E : 0.f;
+      bias_w[lane] = bnext;
       __syncwarp();
+      bnext = b2_of(i + 1);
       while (nxt < c) {
         ++lab_cur;
         nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
@@ -1182,6 +1190,304 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
   TcArgs gt = g;    // the tail reduces H columns: N = H there
   gt.N = g.K;
   dh_reduce_phase(gt, reinterpret_cast<float*>(smem));
+}
+
+// ------------------------------------------------------------------ K-3 (dW2 half)
+// G1b + G3 in one persistent kernel for the fused softmax-CE regime: the dZ^T tiles a W2
+// row tile needs are recomputed on chip instead of read back from HBM (K-3's second half,
+// SURVEY §7; with it the logits never reach HBM).  CTA c owns a contiguous range of label
+// tiles (128 labels = the MMA M) and, per tile j, sweeps the batch in row chunks of 64:
+//   MMA 1   S^T   = W2_j . H1_m^T          (TMEM 128 x 64, double-buffered)
+//   epi     dZ^T  = exp(S^T + b2 - lse) / B - T   (bf16, K-major smem tile; db2 in registers)
+//   MMA 2   dW2_j += dZ^T . H1_m          (TMEM 128 x 256; the SAME H1 chunk, MN-major)
+// then the SGD epilogue W2_j -= lr dW2_j (fp32, coalesced through a smem transpose), the next
+// bf16 shadow, b2_j -= lr db2_j.  A helper warp turns the rows' sorted label lists into a
+// per-(label, row) bitmap of the chunk (cursors in smem, advanced as the tiles increase).
+constexpr int kDwBM = 128, kDwRB = 64;
+constexpr uint32_t kDwW2Bytes = 4u * 16384u, kDwH1Bytes = 4u * 8192u, kDwDzBytes = 16384u;
+constexpr int kDwMaxRows = 1024;
+
+__global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
+    k_bwd_dw(const __grid_constant__ CUtensorMap tmW2, const __grid_constant__ CUtensorMap tmH1, TcArgs g) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint8_t* sW2 = smem;                                   // 4 boxes [128 labels x 64 H]
+  uint8_t* sH1 = sW2 + kDwW2Bytes;                       // 2 stages x 4 boxes [64 rows x 64 H]
+  uint8_t* sDZ = sH1 + 2 * kDwH1Bytes;                   // 2 x [128 labels x 64 rows]
+  uint8_t* sStg = sDZ + 2 * kDwDzBytes;                  // SGD transpose: 8 warps x 4 KB
+  float* sCrow = reinterpret_cast<float*>(sStg + kBwdEpi * 4096);   // [2][64]
+  float* sTinv = sCrow + 2 * kDwRB;                                  // [2][64]
+  uint32_t* sBits = reinterpret_cast<uint32_t*>(sTinv + 2 * kDwRB);  // [2][128][2]
+  float* sDb = reinterpret_cast<float*>(sBits + 2 * kDwBM * 2);      // [2][128]
+  int32_t* sCur = reinterpret_cast<int32_t*>(sDb + 2 * kDwBM);       // [rows] label cursor
+  int32_t* sNxt = sCur + kDwMaxRows;                                 // [rows] next label
+  uint64_t* w2full = reinterpret_cast<uint64_t*>(sNxt + kDwMaxRows);
+  uint64_t* w2empty = w2full + 1;
+  uint64_t* h1full = w2empty + 1;    // [2]
+  uint64_t* h1empty = h1full + 2;    // [2]
+  uint64_t* sfull = h1empty + 2;     // [2]
+  uint64_t* sempty = sfull + 2;      // [2]
+  uint64_t* dzfull = sempty + 2;     // [2]
+  uint64_t* dzempty = dzfull + 2;    // [2]
+  uint64_t* auxfull = dzempty + 2;   // [2]
+  uint64_t* auxempty = auxfull + 2;  // [2]
+  uint64_t* tfull = auxempty + 2;
+  uint64_t* tempty = tfull + 1;
+  uint32_t* tbase = reinterpret_cast<uint32_t*>(tempty + 1);
+
+  pdl_trigger();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int n = g.K;                                     // batch rows
+  const int T = (g.M + kDwBM - 1) / kDwBM, NM = (n + kDwRB - 1) / kDwRB;
+  const int j0 = (int)((int64_t)blockIdx.x * T / gridDim.x), j1 = (int)((int64_t)(blockIdx.x + 1) * T / gridDim.x);
+  const int nt = j1 - j0;
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW2)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmH1)) : "memory");
+    mbar_init(w2full, 1); mbar_init(w2empty, 1);
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(&h1full[a], 1); mbar_init(&h1empty[a], 1);
+      mbar_init(&sfull[a], 1); mbar_init(&sempty[a], kBwdEpi);
+      mbar_init(&dzfull[a], kBwdEpi); mbar_init(&dzempty[a], 1);
+      mbar_init(&auxfull[a], 1); mbar_init(&auxempty[a], kBwdEpi);
+    }
+    mbar_init(tfull, 1); mbar_init(tempty, kBwdEpi);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 2) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tbase)), "r"(512)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tbase;
+  pdl_wait();
+  // label cursors: the first label of each row >= this CTA's first label (binary search,
+  // all threads, rows strided), kept in smem and advanced as the tiles increase
+  if (nt > 0) {
+    const int l0 = j0 * kDwBM;
+    for (int r = threadIdx.x; r < n; r += blockDim.x) {
+      const int64_t id = g.rows[r];
+      int64_t lo = g.lab_ptr[id], hi = g.lab_ptr[id + 1];
+      const int64_t end = hi;
+      while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (g.lab[mid] < l0) lo = mid + 1; else hi = mid;
+      }
+      sCur[r] = (int32_t)(lo - g.lab_ptr[id]);
+      sNxt[r] = lo < end ? g.lab[lo] : 0x7fffffff;
+    }
+  }
+  __syncthreads();
+
+  if (warp == 0) {
+    if (lane == 0 && nt > 0) {   // ------------------------------------ TMA producer
+      int k = 0;
+      for (int t = 0; t < nt; ++t) {
+        mbar_wait(w2empty, (t & 1) ^ 1);
+        mbar_expect_tx(w2full, kDwW2Bytes);
+        for (int kb = 0; kb < 4; ++kb) tma_load_2d(sW2 + kb * 16384, &tmW2, w2full, kb * 64, (j0 + t) * kDwBM);
+        for (int m = 0; m < NM; ++m, ++k) {
+          const int st = k & 1;
+          mbar_wait(&h1empty[st], ((k >> 1) & 1) ^ 1);
+          mbar_expect_tx(&h1full[st], kDwH1Bytes);
+          for (int kb = 0; kb < 4; ++kb)
+            tma_load_2d(sH1 + st * kDwH1Bytes + kb * 8192, &tmH1, &h1full[st], kb * 64, m * kDwRB);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && nt > 0) {   // ------------------------------------ MMA issuer
+      constexpr uint32_t idesc1 = make_idesc(kDwRB, false, false);   // S^T = W2_j H1_m^T
+      constexpr uint32_t idesc2 = make_idesc(256, false, true);      // dW2 += dZ^T H1_m
+      const int K = nt * NM;
+      for (int k = 0; k <= K; ++k) {
+        if (k < K) {
+          const int t = k / NM, m = k % NM, st = k & 1, acc = k & 1;
+          if (m == 0) mbar_wait(w2full, t & 1);
+          mbar_wait(&h1full[st], (k >> 1) & 1);
+          mbar_wait(&sempty[acc], ((k >> 1) & 1) ^ 1);
+          tc_fence_after();
+          const uint32_t d = tmem + (uint32_t)(acc * kDwRB);
+          const uint32_t hb = smem_u32(sH1 + st * kDwH1Bytes);
+#pragma unroll
+          for (int kb = 0; kb < 4; ++kb)
+#pragma unroll
+            for (int kk = 0; kk < 4; ++kk)
+              mma_bf16(d, desc_sw128(smem_u32(sW2 + kb * 16384) + kk * 32, 16, 1024),
+                       desc_sw128(hb + kb * 8192 + kk * 32, 16, 1024), idesc1, (kb | kk) ? 1u : 0u);
+          mma_commit(&sfull[acc]);
+          if (m == NM - 1) mma_commit(w2empty);   // W2_j read by every MMA 1 of the tile
+        }
+        if (k > 0) {
+          const int kp = k - 1, t = kp / NM, m = kp % NM, st = kp & 1, buf = kp & 1;
+          if (m == 0) mbar_wait(tempty, (t & 1) ^ 1);   // the SGD epilogue drained dW2
+          mbar_wait(&dzfull[buf], (kp >> 1) & 1);
+          tc_fence_after();
+          const uint32_t zb = smem_u32(sDZ + buf * kDwDzBytes), hb = smem_u32(sH1 + st * kDwH1Bytes);
+#pragma unroll
+          for (int kk = 0; kk < kDwRB / 16; ++kk)
+            mma_bf16(tmem + 128, desc_sw128(zb + kk * 32, 16, 1024), desc_sw128(hb + kk * 2048, 8192, 1024), idesc2,
+                     (m > 0 || kk > 0) ? 1u : 0u);
+          mma_commit(&dzempty[buf]);
+          mma_commit(&h1empty[st]);
+          if (m == NM - 1) mma_commit(tfull);
+        }
+      }
+    }
+  } else if (warp == 3) {
+    if (nt > 0) {               // ------------------------------------ label bitmap helper
+      int k = 0;
+      for (int t = 0; t < nt; ++t) {
+        const int l0 = (j0 + t) * kDwBM;
+        for (int m = 0; m < NM; ++m, ++k) {
+          const int a = k & 1;
+          mbar_wait(&auxempty[a], ((k >> 1) & 1) ^ 1);
+          uint32_t* bits = sBits + a * kDwBM * 2;
+          for (int i = lane; i < kDwBM * 2; i += 32) bits[i] = 0u;
+          __syncwarp();
+          for (int rr = lane; rr < kDwRB; rr += 32) {
+            const int r = m * kDwRB + rr;
+            float cr = 0.f, ti = 0.f;
+            if (r < n) {
+              const int64_t id = g.rows[r];
+              const int64_t lb = g.lab_ptr[id], le = g.lab_ptr[id + 1];
+              cr = -g.lse[r] * 1.4426950408889634f - __log2f(1.f / g.invB);
+              ti = g.invB / (float)(le - lb);
+              int cur = sCur[r], nx = sNxt[r];
+              while (nx < l0 + kDwBM) {   // this tile's labels of row r (sorted)
+                atomicOr(&bits[(nx - l0) * 2 + (rr >> 5)], 1u << (rr & 31));
+                ++cur;
+                nx = lb + cur < le ? g.lab[lb + cur] : 0x7fffffff;
+              }
+              sCur[r] = cur;
+              sNxt[r] = nx;
+            }
+            sCrow[a * kDwRB + rr] = cr;
+            sTinv[a * kDwRB + rr] = ti;
+          }
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&auxfull[a]);
+        }
+      }
+    }
+  } else if (warp >= 4) {       // -------------------------------------------- epilogue
+    const int q = (warp - 4) & 3, wh = (warp - 4) >> 2;
+    const int ll = q * 32 + lane;                  // this thread's label within the tile
+    constexpr float kL2E = 1.4426950408889634f;
+    const float lr = step_lr(g.meta);
+    int k = 0;
+    for (int t = 0; t < nt; ++t) {
+      const int l = (j0 + t) * kDwBM + ll;
+      const float b2l = l < g.M ? __ldg(g.bias + l) * kL2E : 0.f;
+      float db = 0.f;
+      for (int m = 0; m < NM; ++m, ++k) {
+        const int acc = k & 1, buf = k & 1, a = k & 1;
+        mbar_wait(&auxfull[a], (k >> 1) & 1);
+        mbar_wait(&sfull[acc], (k >> 1) & 1);
+        tc_fence_after();
+        float v[32];
+        tmem_ld32(tmem + (uint32_t)(acc * kDwRB + wh * 32) + ((uint32_t)(q * 32) << 16), v);
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sempty[acc]);
+        const uint32_t bw = sBits[a * kDwBM * 2 + ll * 2 + wh];
+        const float* cr = sCrow + a * kDwRB + wh * 32;
+        const float* ti = sTinv + a * kDwRB + wh * 32;
+        const int rbase = m * kDwRB + wh * 32;
+#pragma unroll
+        for (int i = 0; i < 32; ++i) {
+          float z = ex2_approx(fmaf(v[i], kL2E, b2l + cr[i]));
+          if ((bw >> i) & 1u) z -= ti[i];
+          if (l >= g.M || rbase + i >= n) z = 0.f;
+          v[i] = z;
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&auxempty[a]);
+        mbar_wait(&dzempty[buf], ((k >> 1) & 1) ^ 1);
+        uint8_t* rowp = sDZ + buf * kDwDzBytes + ll * 128;
+        const int sw = ll & 7;
+#pragma unroll
+        for (int h = 0; h < 4; ++h) {
+          __nv_bfloat162 p0 = __floats2bfloat162_rn(v[8 * h], v[8 * h + 1]);
+          __nv_bfloat162 p1 = __floats2bfloat162_rn(v[8 * h + 2], v[8 * h + 3]);
+          __nv_bfloat162 p2 = __floats2bfloat162_rn(v[8 * h + 4], v[8 * h + 5]);
+          __nv_bfloat162 p3 = __floats2bfloat162_rn(v[8 * h + 6], v[8 * h + 7]);
+          db += ((__low2float(p0) + __high2float(p0)) + (__low2float(p1) + __high2float(p1))) +
+                ((__low2float(p2) + __high2float(p2)) + (__low2float(p3) + __high2float(p3)));
+          uint4 pk;
+          pk.x = *reinterpret_cast<uint32_t*>(&p0); pk.y = *reinterpret_cast<uint32_t*>(&p1);
+          pk.z = *reinterpret_cast<uint32_t*>(&p2); pk.w = *reinterpret_cast<uint32_t*>(&p3);
+          *reinterpret_cast<uint4*>(rowp + (((wh * 4 + h) ^ sw) * 16)) = pk;
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&dzfull[buf]);
+      }
+      // ---- SGD: W2_j -= lr dW2_j (rows = labels, this warp's 32 labels x 128 columns),
+      //      coalesced through a swizzled 32 x 32 smem transpose; next bf16 shadow; b2
+      const int m0w = (j0 + t) * kDwBM + q * 32;
+      const int lr8 = lane >> 3, lc4 = (lane & 7) * 4;
+      uint8_t* tt = sStg + (warp - 4) * 4096;
+      mbar_wait(tfull, t & 1);
+      tc_fence_after();
+#pragma unroll 1
+      for (int ch = 0; ch < 4; ++ch) {
+        const int cb = wh * 128 + ch * 32;
+        float4 wr[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const int r = m0w + 4 * i + lr8;
+          wr[i] = r < g.M ? *reinterpret_cast<const float4*>(g.out + (int64_t)r * g.ldo + cb + lc4)
+                          : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+        float vv[32];
+        tmem_ld32(tmem + 128 + (uint32_t)cb + ((uint32_t)(q * 32) << 16), vv);
+        __syncwarp();
+#pragma unroll
+        for (int qq = 0; qq < 8; ++qq)
+          *reinterpret_cast<float4*>(tt + lane * 128 + ((qq ^ (lane & 7)) * 16)) =
+              make_float4(vv[4 * qq], vv[4 * qq + 1], vv[4 * qq + 2], vv[4 * qq + 3]);
+        __syncwarp();
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const int rl = 4 * i + lr8, r = m0w + rl;
+          const float4 gv = *reinterpret_cast<const float4*>(tt + rl * 128 + (((lane & 7) ^ (rl & 7)) * 16));
+          if (r < g.M) {
+            float4 x = wr[i];
+            x.x -= lr * gv.x; x.y -= lr * gv.y; x.z -= lr * gv.z; x.w -= lr * gv.w;
+            const int64_t o = (int64_t)r * g.ldo + cb + lc4;
+            __stcs(reinterpret_cast<float4*>(g.out + o), x);
+            __nv_bfloat162 p0 = __floats2bfloat162_rn(x.x, x.y), p1 = __floats2bfloat162_rn(x.z, x.w);
+            uint2 pk;
+            pk.x = *reinterpret_cast<uint32_t*>(&p0); pk.y = *reinterpret_cast<uint32_t*>(&p1);
+            __stcs(reinterpret_cast<uint2*>(g.shadow + o), pk);
+            if (g.grad) *reinterpret_cast<float4*>(g.grad + o) = gv;
+          }
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(tempty);
+      // db2: the two column halves' row sums, added in half order
+      sDb[wh * kDwBM + ll] = db;
+      asm volatile("bar.sync 2, %0;" ::"r"(32 * kBwdEpi) : "memory");
+      if (wh == 0 && l < g.M) {
+        const float dbt = sDb[ll] + sDb[kDwBM + ll];
+        g.b2[l] -= lr * dbt;
+        if (g.grad_b2) g.grad_b2[l] = dbt;
+      }
+      asm volatile("bar.sync 2, %0;" ::"r"(32 * kBwdEpi) : "memory");
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512) : "memory");
+  }
 }
 
 // ------------------------------------------------------------------ host side
@@ -1424,6 +1730,28 @@ cudaError_t launch_bwd_dh(const Launch& lc, int n, int64_t L, int H, const Ptrs&
   if ((e = ensure_smem(k_bwd_dh, smem)) != cudaSuccess) return e;
   return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_bwd_dh, dim3(MT * LR), dim3(128 + 32 * kBwdEpi), smem, th,
                       tw, tz, g, LR);
+}
+
+cudaError_t launch_bwd_dw(const Launch& lc, int n, int64_t L, int H, const Ptrs& Pr, const Ptrs& Pw, float* W2,
+                          float* b2, const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab,
+                          float* grad_w2, float* grad_b2) {
+  if (!tc_available()) return cudaErrorNotSupported;
+  if (H != 256 || Pr.w2l || n > kDwMaxRows) return cudaErrorNotSupported;
+  CUtensorMap tw, th;
+  cudaError_t e;
+  if ((e = make_map(&tw, Pr.w2b, H, L, (uint64_t)H * 2, 64, kDwBM)) != cudaSuccess) return e;
+  if ((e = make_map(&th, Pr.h1b, H, n, (uint64_t)H * 2, 64, kDwRB)) != cudaSuccess) return e;
+  TcArgs g{};
+  g.M = (int)L; g.N = H; g.K = n;
+  g.out = W2; g.ldo = H; g.meta = Pr.meta; g.shadow = Pw.w2b; g.grad = grad_w2;
+  g.b2 = b2; g.grad_b2 = grad_b2; g.bias = b2;
+  g.lse = Pr.lse; g.rows = rows; g.lab_ptr = lab_ptr; g.lab = lab; g.invB = 1.f / (float)n;
+  const size_t smem = kDwW2Bytes + 2 * kDwH1Bytes + 2 * kDwDzBytes + kBwdEpi * 4096 + 2 * kDwRB * 8 +
+                      2 * kDwBM * 2 * 4 + 2 * kDwBM * 4 + 2 * kDwMaxRows * 4 + 256 + 1024;
+  if ((e = ensure_smem(k_bwd_dw, smem)) != cudaSuccess) return e;
+  const int64_t T = (L + kDwBM - 1) / kDwBM;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(T, lc.sms));
+  return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_bwd_dw, dim3(grid), dim3(128 + 32 * kBwdEpi), smem, tw, th, g);
 }
 
 }  // namespace asgd
