@@ -162,6 +162,17 @@ int asgd_updates(const asgd_ctx* ctx, int64_t* u_out);
  * The fused kernels never materialise it otherwise.  NULL turns it off. */
 int asgd_set_debug_grads(asgd_ctx* ctx, float* grad_dev);
 
+/* Step trace (per-rank step log): with tracing on, every local step
+ * records a pair of CUDA timing events around its enqueue on the ctx stream.
+ *   asgd_trace_enable(ctx, 1): (re)starts the trace, its time origin is now.
+ *   asgd_trace_read: synchronous; out: int64[4*cap] rows of (stream start of the
+ *     step's batch -- the ticket's start in asgd_run_tickets / asgd_run_static, -1
+ *     for a direct asgd_local_step --, rows, t0_ns, t1_ns) since the origin, in
+ *     step order; *n_out = steps; clears the trace.  ASGD_E_SHAPE if cap is short.
+ * The events add ~2 us of host work per step: leave tracing off for timing. */
+int asgd_trace_enable(asgd_ctx* ctx, int32_t on);
+int asgd_trace_read(asgd_ctx* ctx, int64_t* out_host, int64_t cap, int64_t* n_out);
+
 /* Debug/parity: the sorted unique feature ids of the last local step
  * (touched W1 rows).  out_dev: int32[cap] device; *n_out_host = count.
  * Synchronous. ASGD_E_SHAPE if cap is too small. */

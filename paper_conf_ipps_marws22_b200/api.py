@@ -149,6 +149,16 @@ class Replica:
              int(losses.numel()) if losses is not None else 0, int(inflight), C.byref(n))
         return n.value
 
+    def trace_enable(self, on: bool = True):
+        call("asgd_trace_enable", self.ctx, int(bool(on)))
+
+    def trace_read(self, cap: int = 1 << 16) -> List[Tuple[int, int, int, int]]:
+        """(stream start, rows, t0_ns, t1_ns) of each traced step since trace_enable."""
+        out = np.zeros(4 * cap, dtype=np.int64)
+        n = C.c_int64()
+        call("asgd_trace_read", self.ctx, _ptr(out), int(cap), C.byref(n))
+        return [tuple(int(x) for x in out[4 * i:4 * i + 4]) for i in range(n.value)]
+
     def updates(self) -> int:
         u = C.c_int64()
         call("asgd_updates", self.ctx, C.byref(u))

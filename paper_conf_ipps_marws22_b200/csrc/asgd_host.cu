@@ -59,6 +59,7 @@ size_t up256(size_t x) { return (x + 255) & ~size_t(255); }
 
 constexpr int kSqnormParts = 1024;
 constexpr int kMaxInflight = 8;
+constexpr size_t kMaxTrace = 1 << 16;   // traced steps kept between two asgd_trace_read calls
 // Above this many bytes of fp32 logits per step the bf16 path fuses softmax-CE
 // into the GEMMs (Z never written); below, Z stays L2-resident and is stored.
 // Measured: AmazonCat-13K (54.6 MB) 4.99M -> 5.35M samples/s fused; Wiki10-31K
@@ -252,6 +253,13 @@ struct asgd_ctx {
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_sm = nullptr, ev_dh = nullptr, ev_a = nullptr;
   bf16* w2b_buf[2] = {nullptr, nullptr};         // double-buffered bf16 W2 shadow (hi half on fp32)
   bf16* w2l_buf[2] = {nullptr, nullptr};         // fp32 path: its bf16x3 lo half (R14)
+  // step trace (asgd_trace_enable / asgd_trace_read): timing events around each local step
+  bool trace = false;
+  cudaEvent_t trace_ref = nullptr;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> trace_ev;
+  std::vector<int64_t> trace_meta;   // (stream start, rows) per traced step
+  size_t trace_n = 0;
+  int64_t cur_start = -1;            // stream position of the step being enqueued (run_steps)
   int w2b_cur = 0;
   std::list<StepGraph> graphs;                   // CUDA-graph cache of the step, LRU (stable addresses:
                                                  // the graphs point at their own StepArgs)
@@ -447,6 +455,8 @@ int asgd_replica_destroy(asgd_ctx* c) {
     clear_graphs(c);
     for (void* pm : c->peer_mapped) cudaIpcCloseMemHandle(pm);
     if (c->prof_sink) cudaEventDestroy(c->prof_sink);
+    if (c->trace_ref) cudaEventDestroy(c->trace_ref);
+    for (auto& pr : c->trace_ev) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
     for (cudaEvent_t ev : c->ev_ring)
       if (ev) cudaEventDestroy(ev);
     for (auto& v : c->pev)
@@ -779,10 +789,58 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
   if (g) CU(cudaMemsetAsync(g, 0, c->Pn * sizeof(float), c->s));
   // the step's only per-call arguments; K-0 and K-1 build the batch view from them
   c->sa = StepArgs{rows, loss_dev, lr, n};
+  const bool tr = c->trace && c->trace_n < kMaxTrace;
+  if (tr) {
+    if (c->trace_ev.size() <= c->trace_n) {
+      cudaEvent_t a, b;
+      CU(cudaEventCreate(&a));
+      CU(cudaEventCreate(&b));
+      c->trace_ev.push_back({a, b});
+    }
+    CU(cudaEventRecord(c->trace_ev[c->trace_n].first, c->s));
+  }
   const int rc = (graphs_enabled() && !g) ? step_graph(c, n) : enqueue_step(c, n);
   if (rc != ASGD_OK) return rc;
+  if (tr) {
+    CU(cudaEventRecord(c->trace_ev[c->trace_n].second, c->s));
+    c->trace_meta.push_back(c->cur_start);
+    c->trace_meta.push_back(n);
+    ++c->trace_n;
+  }
   c->w2b_cur ^= 1;   // G3 wrote the other shadow buffer
   ++c->u;
+  return ASGD_OK;
+}
+
+int asgd_trace_enable(asgd_ctx* c, int32_t on) {
+  if (!c) return fail(ASGD_E_ARG, "null ctx");
+  if (on) {
+    if (!c->trace_ref) CU(cudaEventCreate(&c->trace_ref));
+    CU(cudaEventRecord(c->trace_ref, c->s));
+    c->trace_n = 0;
+    c->trace_meta.clear();
+  }
+  c->trace = on != 0;
+  return ASGD_OK;
+}
+
+int asgd_trace_read(asgd_ctx* c, int64_t* out, int64_t cap, int64_t* n_out) {
+  if (!c || !out || !n_out) return fail(ASGD_E_ARG, "null argument");
+  if (!c->trace_ref) return fail(ASGD_E_STATE, "asgd_trace_enable first");
+  if ((int64_t)c->trace_n > cap) return fail(ASGD_E_SHAPE, "cap %lld < %zu traced steps", (long long)cap, c->trace_n);
+  if (c->trace_n) CU(cudaEventSynchronize(c->trace_ev[c->trace_n - 1].second));
+  for (size_t i = 0; i < c->trace_n; ++i) {
+    float t0 = 0.f, t1 = 0.f;
+    CU(cudaEventElapsedTime(&t0, c->trace_ref, c->trace_ev[i].first));
+    CU(cudaEventElapsedTime(&t1, c->trace_ref, c->trace_ev[i].second));
+    out[4 * i] = c->trace_meta[2 * i];
+    out[4 * i + 1] = c->trace_meta[2 * i + 1];
+    out[4 * i + 2] = (int64_t)((double)t0 * 1e6);
+    out[4 * i + 3] = (int64_t)((double)t1 * 1e6);
+  }
+  *n_out = (int64_t)c->trace_n;
+  c->trace_n = 0;
+  c->trace_meta.clear();
   return ASGD_OK;
 }
 
@@ -1264,8 +1322,10 @@ int run_steps(asgd_ctx* c, Next next, const int32_t* stream_rows, float lr, floa
     const int r = next(&start, &len);
     if (r < 0) return fail(-r, "scheduler failed");
     if (r == 0) break;
+    c->cur_start = start;
     const int rc = asgd_local_step(c, stream_rows + start, (int32_t)len, lr,
                                    (losses && k < losses_cap) ? losses + k : nullptr);
+    c->cur_start = -1;
     if (rc != ASGD_OK) return rc;
     CU(cudaEventRecord(c->ev_ring[k % kMaxInflight], c->s));
     ++k;

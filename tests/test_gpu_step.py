@@ -172,3 +172,24 @@ def test_step_sigmoid_ragged_trained(precision):
     w0[o2 + L * H:] = np.linspace(-12.0, 6.0, L)
     w0 = w0.astype(np.float32)
     _check(cfg, *_one_step(cfg, data, rows, precision, w0=w0, loss_kind="sigmoid"), precision)
+
+
+def test_step_trace():
+    """asgd_trace_enable / asgd_trace_read: one (start, rows, t0, t1) per local step, in
+    order, times increasing; starts are the tickets' stream positions."""
+    from paper_conf_ipps_marws22_b200 import api, train
+    cfg = config("tiny")
+    data = dataset("tiny")
+    rep = make_replica(cfg, data, "bf16")
+    h = train.Hyper.from_config(cfg)
+    sched = api.Scheduler("/asgd_tr_" + str(np.random.randint(1 << 30)), 1, h.M, create=True)
+    drv = train.DistributedAdaptiveSGD(rep, h, 0, 1, sched)
+    ids = sample_stream(cfg, 0, h.M)
+    rep.trace_enable(True)
+    st = drv.megabatch(torch.as_tensor(ids, device="cuda"), keep_log=True)
+    tr = rep.trace_read()
+    sched.close()
+    assert len(tr) == st.n_steps == len(st.routes)
+    assert [(s, n) for s, n, _, _ in tr] == [(s, n) for _, _, s, n in st.routes]
+    assert all(t1 >= t0 for _, _, t0, t1 in tr)
+    assert all(tr[i + 1][2] >= tr[i][2] for i in range(len(tr) - 1))
