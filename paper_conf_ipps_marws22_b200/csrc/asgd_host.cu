@@ -80,9 +80,13 @@ bool bwd_fuse() {
   static const bool v = [] { const char* e = getenv("ASGD_BWD_FUSE"); return !(e && e[0] == '0'); }();
   return v;
 }
-// K-3's dW2 half (k_bwd_dw, replaces G3 there and dZ never reaches HBM) -- ASGD_BWD_DW=0: G3
+// K-3's dW2 half (k_bwd_dw, replaces G3 there and dZ never reaches HBM): ASGD_BWD_DW=1.
+// Off by default: measured at Amazon-670K 2.59 ms vs 2.16 ms per step -- k_bwd_dh without the
+// dZ store drops 885 -> 644 us, but k_bwd_dw takes 1,374 us against G3's 625 (its SGD
+// epilogue, 128 KB of fp32 W2 read-modify-write per tile, cannot overlap the next tile's
+// MMAs: the dW2 accumulator takes 256 of TMEM's 512 columns and cannot be double-buffered).
 bool bwd_dw() {
-  static const bool v = [] { const char* e = getenv("ASGD_BWD_DW"); return !(e && e[0] == '0'); }();
+  static const bool v = [] { const char* e = getenv("ASGD_BWD_DW"); return e && e[0] == '1'; }();
   return v;
 }
 

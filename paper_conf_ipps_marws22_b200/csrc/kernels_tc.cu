@@ -1342,6 +1342,14 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       int k = 0;
       for (int t = 0; t < nt; ++t) {
         const int l0 = (j0 + t) * kDwBM;
+        // the tile's fp32 W2 rows (128 x 1 KB) into L2 while the chunks run, so the SGD
+        // epilogue's read-modify-write finds them there instead of paying HBM latency
+        for (int i = lane; i < kDwBM * 8; i += 32) {
+          const int r = l0 + (i >> 3);
+          if (r < g.M)
+            asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(g.out + (int64_t)r * g.ldo + (i & 7) * 32)
+                         : "memory");
+        }
         for (int m = 0; m < NM; ++m, ++k) {
           const int a = k & 1;
           mbar_wait(&auxempty[a], ((k >> 1) & 1) ^ 1);
