@@ -170,8 +170,15 @@ class DistributedAdaptiveSGD:
         if self.time_merge:   # from the end of this rank's local steps to the merged model
             ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
             ev[0].record(rep.stream)
-        rep.sqnorm(self.sq)
-        us, bs, nu = exchange_stats(n_steps, b_i, self.sq, rep.P, self.world, self.group)
+        if self.world == 1:
+            # N = 1: Alg. 2 line 2 gives alpha = b / sum(b) = 1 and lines 4-6 skip the
+            # perturbation (the only replica ties with itself, Q17) whatever nu is, so the
+            # norm and its host round trip are not needed: the merge is enqueued behind the
+            # steps without a device sync (nu is reported as NaN)
+            us, bs, nu = [n_steps], [b_i], [float("nan")]
+        else:
+            rep.sqnorm(self.sq)
+            us, bs, nu = exchange_stats(n_steps, b_i, self.sq, rep.P, self.world, self.group)
         routes = self.sched.log() if keep_log and r == 0 else []
         if r == 0:
             self.sched.reset(self.mb + 1)        # every rank is past its tickets
@@ -248,8 +255,11 @@ class DistributedAdaptiveSGD:
         if self.time_merge:
             ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
             ev[0].record(rep.stream)
-        rep.sqnorm(self.sq)
-        us, bs, nu = exchange_stats(n_steps, h.b_max, self.sq, rep.P, N, self.group)   # also the barrier
+        if N == 1:   # alpha = 1/N = 1: no statistics to exchange (see megabatch)
+            us, bs, nu = [n_steps], [h.b_max], [float("nan")]
+        else:
+            rep.sqnorm(self.sq)
+            us, bs, nu = exchange_stats(n_steps, h.b_max, self.sq, rep.P, N, self.group)   # also the barrier
         alpha = api.elastic_weights(N)
         self._merge(alpha)
         if ev is not None:

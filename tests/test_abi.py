@@ -212,3 +212,16 @@ def test_route_static_matches_oracle():
     for _ in range(300):
         n, b, M = rng.randint(1, 8), rng.randint(1, 40), rng.randint(0, 500)
         assert api.route_static(n, b, M) == [tuple(r) for r in routing.static(n, b, M)]
+
+
+def test_single_replica_weights_ignore_nu():
+    """N = 1: Alg. 2 gives alpha = [1] whatever the norm (line 2: b / sum b; lines 4-6: the
+    only replica ties with itself, Q17) -- why the N = 1 driver skips the norm and its host
+    round trip (train.DistributedAdaptiveSGD)."""
+    for u in (1, 7, 100):
+        for b in (1, 32, 1024):
+            for nu in (float("nan"), 0.0, 1e-6, 0.5, 1e9):
+                for renorm in (False, True):
+                    for norm in ("u", "ub"):
+                        assert api.merge_weights([u], [b], [nu], 0.1, 0.1, renorm, norm) == ([1.0], 0, 0, False)
+                        assert merge.merge_weights([u], [b], [nu], 0.1, 0.1, renorm, norm)[0] == [1.0]
