@@ -65,6 +65,12 @@ def test_amazoncat_bench_launch(precision):
     _check_big("amazoncat13k", 32768, precision, chunk=1024)
 
 
+def test_amazon670k_fp32_bench_launch():
+    """The fp32 path (bf16x3 on tcgen05, R14) at L = 670,091: Z stored (2.7 GB), dZ as
+    bf16 hi + lo halves; 1e-4 against the fp64 oracle."""
+    _check_big("amazon670k", 16384, "fp32", chunk=128)
+
+
 def test_amazon670k_bench_launch():
     """L = 670,091: the fused softmax-CE path (Z never stored), G2 splits K."""
     _check_big("amazon670k", 16384, "bf16", chunk=128)

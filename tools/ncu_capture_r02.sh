@@ -9,3 +9,14 @@ for spec in "eurlex4k bf16 400" "eurlex4k fp32 400" "amazoncat13k bf16 260" "ama
     --no-cpu-baseline --ttp-megabatches 0 --e2e-steps 0 > gpurun_out/e1_full_$1_$2.log 2>&1
   echo "full $1 $2 $?"
 done
+# summaries on the box (the reports themselves exceed gpurun's 64 MiB pull limit)
+for f in gpurun_out/e1_full_*.ncu-rep; do
+  b=${f%.ncu-rep}
+  python tools/ncu_details.py $f > $b.details.md 2>&1
+  python tools/ncu_tensor.py $f > $b.tensor.md 2>&1
+  ncu -i $f --page source --csv --print-source sass -k regex:"k_(spmm|scatter|bwd_dh|softmax)" > $b.src.csv 2>/dev/null
+  k=$(basename $b | sed 's/e1_full_//; s/_\(bf16\|fp32\)$//'); p=$(basename $b | sed 's/.*_//')
+  python tools/ncu_traffic.py $k/$p gpurun_out/e1_traffic_$k_$p.json $f > /dev/null 2>&1
+  python tools/ncu_traffic.py $k/$p - $f > $b.traffic.json 2>&1
+  rm -f $f
+done
