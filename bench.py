@@ -53,7 +53,8 @@ def _args():
     p.add_argument("--norm", default="u", choices=["u", "ub"],
                    help="Alg. 2 line 3: u_i-normalised (the paper's default) or u_i b_i (R12, P:1088-1090)")
     p.add_argument("--scale-every", type=int, default=1,
-                   help="run Alg. 1 after every k-th mega-batch (R13, P:922-925; 1 = the paper's default)")
+                   help="run Alg. 1 after every k-th mega-batch (R13, P:922-925; 1 = the paper's default; "
+                        "0 = the adaptive frequency of R17)")
     p.add_argument("--e2e-steps", type=int, default=None)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)

@@ -262,6 +262,17 @@ int asgd_scale_batches(int32_t n, const int64_t* u, int64_t* b_inout,
                        double* lr_out, int64_t b_min, int64_t b_max,
                        int64_t beta, double lr_max);
 
+/* Adaptive Alg. 1 frequency ("if stability is achieved or the system enters an
+ * oscillatory state, the frequency at which scaling is performed can be [reduced]";
+ * reading R17): after an Alg. 1 invocation moved b_before -> b_after (int64[n]), with
+ * d_i = sign(b_after_i - b_before_i): when every d_i is 0 (stable) or some d_i is
+ * opposite to rank i's previous non-zero move (oscillating), the interval to the next
+ * invocation doubles up to max_interval, otherwise it returns to 1.  last_sign:
+ * int32[n] in/out (the last non-zero move per rank, start at 0).  Host, pure. */
+int asgd_scale_frequency(int32_t n, const int64_t* b_before, const int64_t* b_after,
+                         int32_t* last_sign, int32_t interval, int32_t max_interval,
+                         int32_t* interval_out);
+
 /* -------------------------------------------------------------- routing */
 
 /* Dynamic scheduler (S3): a ticket counter in POSIX

@@ -59,15 +59,17 @@ def run(F: int, H: int, L: int, data, w0: np.ndarray, stream_rows_of: Callable[[
         gamma: float = 0.9, delta: float = 0.1, pert_thr: float = 0.1,
         pert_renorm: bool = False, cost_factors: Optional[Sequence[float]] = None,
         route_logs: Optional[List[List[int]]] = None, norm: str = "u",
-        scale_every: int = 1) -> List[MegaBatchRecord]:
+        scale_every: int = 1, max_interval: int = 8) -> List[MegaBatchRecord]:
     """Run n_mb mega-batches.  stream_rows_of(mb) gives the M sample ids of
     mega-batch mb.  Routing is simulated with cost_factors, or replayed from
     route_logs[mb] (ranks in ticket order).  norm: Alg. 2 line 3 ("u") or the
     u_i b_i variant ("ub", R12).  scale_every: Alg. 1 runs after mega-batches
     mb with (mb + 1) % scale_every == 0 (R13; 1 = every mega-batch,
-    the paper's default)."""
-    if scale_every < 1:
+    the paper's default); scale_every = 0: the adaptive frequency of reading R17
+    (scaling.scale_frequency, intervals up to max_interval)."""
+    if scale_every < 0:
         raise ValueError(scale_every)
+    interval, countdown, signs = 1, 1, [0] * n_rep     # R17 state
     w = np.asarray(w0, dtype=np.float64).copy()
     d = np.zeros_like(w)                                   # Q19: w_p = w_0
     b = [int(b_max)] * n_rep                               # P:1565-1566
@@ -92,7 +94,13 @@ def run(F: int, H: int, L: int, data, w0: np.ndarray, stream_rows_of: Callable[[
         w, d = _merge.merge_models(replicas, alpha, w, d, gamma)
         rec = MegaBatchRecord(routes, losses, u, list(b), list(lr), nu, alpha, pert, r, s,
                               w.copy(), d.copy())
-        if (mb + 1) % scale_every == 0:                    # R13
+        if scale_every == 0:                               # R17: adaptive frequency
+            countdown -= 1
+            if countdown == 0:
+                b_new, lr = _scaling.scale_batches(u, b, b_min, b_max, beta, lr_max)
+                interval, signs = _scaling.scale_frequency(b, b_new, signs, interval, max_interval)
+                b, countdown = b_new, interval
+        elif (mb + 1) % scale_every == 0:                  # R13
             b, lr = _scaling.scale_batches(u, b, b_min, b_max, beta, lr_max)
         out.append(rec)
     return out

@@ -73,6 +73,7 @@ _SIGS = {
     "asgd_sched_close": (C.c_int, [_P, _i32]),
     "asgd_route_replay": (C.c_int, [_i32, _i32, _P, _P, _i64, _P, _i64, C.POINTER(_i64)]),
     "asgd_norm_per_param": (C.c_int, [_i32, _P, _i64, _P]),
+    "asgd_scale_frequency": (C.c_int, [_i32, _P, _P, _P, _i32, _i32, C.POINTER(_i32)]),
     "asgd_route_static": (C.c_int, [_i32, _i64, _i64, _P, _i64, C.POINTER(_i64)]),
     "asgd_elastic_weights": (C.c_int, [_i32, _P]),
     "asgd_peer_close": (C.c_int, [_P]),

@@ -291,6 +291,16 @@ def route_replay(order, b, M) -> List[Tuple[int, int, int]]:
     return [tuple(int(x) for x in out[3 * i:3 * i + 3]) for i in range(n.value)]
 
 
+def scale_frequency(b_before, b_after, last_sign, interval: int, max_interval: int = 8):
+    """R17: the next Alg. 1 interval and the updated last move signs."""
+    bb, ba = _np(b_before, np.int64), _np(b_after, np.int64)
+    sg = _np(last_sign, np.int32).copy()
+    out = C.c_int32()
+    call("asgd_scale_frequency", len(bb), _ptr(bb), _ptr(ba), _ptr(sg), int(interval), int(max_interval),
+         C.byref(out))
+    return out.value, sg.tolist()
+
+
 def route_static(n, b, M) -> List[Tuple[int, int, int]]:
     """Elastic SGD's static routes (R10): batch k of b samples -> rank k mod n."""
     cap = int(M) // max(1, int(b)) + 2

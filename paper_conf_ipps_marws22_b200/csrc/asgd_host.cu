@@ -1155,6 +1155,21 @@ int asgd_merge_weights(int32_t n, const int64_t* u, const int64_t* b, const doub
   return ASGD_OK;
 }
 
+int asgd_scale_frequency(int32_t n, const int64_t* b_before, const int64_t* b_after, int32_t* last_sign,
+                         int32_t interval, int32_t max_interval, int32_t* interval_out) {
+  if (n < 1 || !b_before || !b_after || !last_sign || !interval_out || interval < 1 || max_interval < 1)
+    return fail(ASGD_E_ARG, "bad argument");
+  bool stable = true, osc = false;
+  for (int i = 0; i < n; ++i) {   // R17: d_i = sign of rank i's move
+    const int d = (b_after[i] > b_before[i]) - (b_after[i] < b_before[i]);
+    if (d != 0) stable = false;
+    if (d != 0 && last_sign[i] != 0 && d == -last_sign[i]) osc = true;
+    if (d != 0) last_sign[i] = d;
+  }
+  *interval_out = (stable || osc) ? std::min(2 * interval, max_interval) : 1;
+  return ASGD_OK;
+}
+
 int asgd_norm_per_param(int32_t n, const double* sqnorm, int64_t P, double* nu) {
   if (n < 1 || !sqnorm || !nu || P < 1) return fail(ASGD_E_ARG, "bad argument");
   for (int i = 0; i < n; ++i) {

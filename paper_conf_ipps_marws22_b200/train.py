@@ -38,19 +38,44 @@ class Hyper:
     pert_thr: float = 0.1
     pert_renorm: bool = False   # Q34 option (literal Alg. 2 by default)
     norm: str = "u"             # Alg. 2 line 3: "u", or "ub" = u_i b_i (R12)
-    scale_every: int = 1        # Alg. 1 after every scale_every-th mega-batch (R13)
+    scale_every: int = 1        # Alg. 1 after every scale_every-th mega-batch (R13);
+                                # 0: the adaptive frequency of R17 (asgd_scale_frequency)
+    max_interval: int = 8       # R17's longest interval
 
     def __post_init__(self):
         if self.norm not in ("u", "ub"):
             raise ValueError(f"norm must be 'u' or 'ub', got {self.norm!r}")
-        if self.scale_every < 1:
-            raise ValueError(f"scale_every must be >= 1, got {self.scale_every}")
+        if self.scale_every < 0:
+            raise ValueError(f"scale_every must be >= 0, got {self.scale_every}")
 
     @classmethod
     def from_config(cls, cfg, **kw):
         h = dict(b_max=cfg.b_max, b_min=cfg.b_min, beta=cfg.beta, lr_max=cfg.lr_max, M=cfg.mega_batch)
         h.update(kw)
         return cls(**h)
+
+
+class ScaleClock:
+    """When Alg. 1 runs (R13: every k-th mega-batch; R17: the adaptive frequency)."""
+
+    def __init__(self, hyper: "Hyper", n: int):
+        self.h = hyper
+        self.interval, self.countdown, self.signs = 1, 1, [0] * n
+
+    def step(self, mb: int, u, b):
+        """Alg. 1 after mega-batch mb if due; returns (b, lr) or None."""
+        h = self.h
+        if h.scale_every > 0:
+            if (mb + 1) % h.scale_every:
+                return None
+            return api.scale_batches(u, b, h.b_min, h.b_max, h.beta, h.lr_max)
+        self.countdown -= 1
+        if self.countdown:
+            return None
+        b_new, lr = api.scale_batches(u, b, h.b_min, h.b_max, h.beta, h.lr_max)
+        self.interval, self.signs = api.scale_frequency(b, b_new, self.signs, self.interval, h.max_interval)
+        self.countdown = self.interval
+        return b_new, lr
 
 
 @dataclasses.dataclass
@@ -146,6 +171,7 @@ class DistributedAdaptiveSGD:
         self.sq = torch.zeros(1, dtype=torch.float64, device=dev)
         self.events = [torch.cuda.Event() for _ in range(cap)]
         self.mb = 0
+        self.clock = ScaleClock(hyper, world)
         self.time_merge = False   # record CUDA events around the merge phase of each mega-batch
 
     def megabatch(self, stream_rows: torch.Tensor, keep_log: bool = False) -> MegaBatchStats:
@@ -188,8 +214,9 @@ class DistributedAdaptiveSGD:
             ev[1].record(rep.stream)
         # ---- Alg. 1 ----------------------------------------------------------
         lr_used = list(self.lr)
-        if (self.mb + 1) % h.scale_every == 0:    # R13
-            self.b, self.lr = api.scale_batches(us, bs, h.b_min, h.b_max, h.beta, h.lr_max)
+        nb = self.clock.step(self.mb, us, bs)     # R13 / R17
+        if nb is not None:
+            self.b, self.lr = nb
         st = MegaBatchStats(self.mb, us, bs, lr_used, nu, alpha, rr, ss, pert, routes, n_steps, ev)
         self.mb += 1
         return st
@@ -294,6 +321,7 @@ class SimulatedAdaptiveSGD:
         cap = hyper.M // max(1, hyper.b_min) + 2
         self.losses = torch.zeros(cap, dtype=torch.float32, device=dev)
         self.mb = 0
+        self.clock = ScaleClock(hyper, self.n)
 
     def megabatch(self, stream_rows: torch.Tensor, stream_ids: np.ndarray,
                   route_order: Optional[Sequence[int]] = None) -> MegaBatchStats:
@@ -324,8 +352,10 @@ class SimulatedAdaptiveSGD:
             rep.params.copy_(r0.params)
             rep.params_changed()
         lr_used, b_used = list(self.lr), list(self.b)
-        if self.method == "adaptive" and (self.mb + 1) % h.scale_every == 0:    # R13
-            self.b, self.lr = api.scale_batches(u, self.b, h.b_min, h.b_max, h.beta, h.lr_max)
+        if self.method == "adaptive":
+            nb = self.clock.step(self.mb, u, self.b)   # R13 / R17
+            if nb is not None:
+                self.b, self.lr = nb
         st = MegaBatchStats(self.mb, u, b_used, lr_used, nu, alpha, rr, ss, pert, routes, len(routes))
         self.mb += 1
         return st

@@ -38,7 +38,8 @@ def test_sqnorm_prescale_finish():
 
 @pytest.mark.parametrize("precision,tol,norm,scale_every", [
     ("fp32", 1e-4, "u", 1), ("bf16", 2e-2, "u", 1),
-    ("fp32", 1e-4, "ub", 2)])        # R12 u_i b_i weights, R13 Alg. 1 every 2nd mega-batch
+    ("fp32", 1e-4, "ub", 2),         # R12 u_i b_i weights, R13 Alg. 1 every 2nd mega-batch
+    ("bf16", 2e-2, "u", 0)])         # R17 adaptive Alg. 1 frequency
 def test_simulated_two_replicas_tiny_trajectory(precision, tol, norm, scale_every):
     """BASELINE.json configs[0]: 2 simulated replicas, ~50 steps, free-running."""
     from paper_conf_ipps_marws22_b200 import api, train

@@ -96,4 +96,4 @@ def test_adaptive_scale_every_and_ub_norm():
         want[ub[1].s] *= 0.9
     assert ub[1].alpha == want
     with pytest.raises(ValueError):
-        adaptive.run(cfg.F, cfg.H, cfg.L, data, init_params(cfg), stream, scale_every=0, **kw)
+        adaptive.run(cfg.F, cfg.H, cfg.L, data, init_params(cfg), stream, scale_every=-1, **kw)

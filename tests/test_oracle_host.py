@@ -8,6 +8,7 @@ import numpy as np
 import pytest
 
 from oracle import merge, metrics, routing, scaling
+from paper_conf_ipps_marws22_b200 import api
 from tests.conftest import GOLDEN
 
 
@@ -215,3 +216,55 @@ def test_alg2_ub_variant_pins():
         assert all(abs(x - bi / sum(b)) < 1e-15 for x, bi in zip(a_b, b))
     with pytest.raises(ValueError):
         merge.merge_weights([1], [1], [1.0], norm="bu")
+
+
+def test_scale_frequency_r17():
+    """Reading R17: stable or oscillating b doubles the Alg. 1 interval (up to
+    the cap), a consistent move resets it to 1; the C function equals the oracle."""
+    from oracle.scaling import scale_frequency
+    # stable: 1 -> 2 -> 4 -> 8 -> 8
+    k, s = 1, [0, 0]
+    seq = []
+    for _ in range(4):
+        k, s = scale_frequency([32, 32], [32, 32], s, k, 8)
+        seq.append(k)
+    assert seq == [2, 4, 8, 8] and s == [0, 0]
+    # consistent moves reset to 1, an opposite move (oscillation) doubles
+    k, s = scale_frequency([32, 32], [32, 28], [0, 0], 4, 8)
+    assert (k, s) == (1, [0, -1])
+    k, s = scale_frequency([32, 28], [32, 26], s, k, 8)
+    assert (k, s) == (1, [0, -1])
+    k, s = scale_frequency([32, 26], [32, 29], s, k, 8)
+    assert (k, s) == (2, [0, 1])
+    rng = random.Random(17)
+    for _ in range(2000):
+        n = rng.randint(1, 8)
+        bb = [rng.choice([28, 30, 32]) for _ in range(n)]
+        ba = [x + rng.choice([-2, 0, 0, 2]) for x in bb]
+        sg = [rng.choice([-1, 0, 1]) for _ in range(n)]
+        k0, cap = rng.choice([1, 2, 4, 8]), rng.choice([4, 8, 16])
+        assert api.scale_frequency(bb, ba, sg, k0, cap) == scale_frequency(bb, ba, sg, k0, cap)
+
+
+def test_adaptive_frequency_in_the_run():
+    """adaptive.run with scale_every = 0 runs Alg. 1 after mega-batch 0, then after the
+    R17 intervals; b changes only at those mega-batches."""
+    from oracle import adaptive
+    from synth import config, generate, init_params, sample_stream
+    cfg = config("tiny", n_train=1024)
+    data = generate(cfg, "train", 1024)
+    M = cfg.mega_batch
+    recs = adaptive.run(cfg.F, cfg.H, cfg.L, data, init_params(cfg), lambda mb: sample_stream(cfg, mb * M, M),
+                        n_rep=2, n_mb=8, M=M, b_max=cfg.b_max, b_min=cfg.b_min, beta=cfg.beta, lr_max=cfg.lr_max,
+                        cost_factors=[1.0, 1.6], scale_every=0)
+    from oracle.scaling import scale_batches, scale_frequency
+    k, cd, sg = 1, 1, [0, 0]
+    b = [cfg.b_max] * 2
+    for mb, rec in enumerate(recs):
+        assert rec.b == b
+        cd -= 1
+        if cd == 0:
+            bn, _ = scale_batches(rec.u, b, cfg.b_min, cfg.b_max, cfg.beta, cfg.lr_max)
+            k, sg = scale_frequency(b, bn, sg, k, 8)
+            b, cd = bn, k
+    assert recs[1].b != recs[0].b           # the slower replica was rescaled after mega-batch 0

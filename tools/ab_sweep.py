@@ -9,7 +9,8 @@ replica is a (1 + h)x slower "GPU".  Arms:
   renorm    the same with alpha / sum(alpha) after the perturbation (Q34's
             pert_renorm = true);
   ub_se2    alpha_i = u_i b_i / sum u_j b_j (R12) and Alg. 1 every 2nd mega-batch (R13);
-  elastic   Elastic SGD: static b_max batches, rank k mod N, alpha = 1/N (R10).
+  elastic   Elastic SGD: static b_max batches, rank k mod N, alpha = 1/N (R10);
+  renorm_r17  renorm with Alg. 1's adaptive frequency (R17; not in the default --arms).
 Per merge it logs ||w||_2 of the global model, sum(alpha), the perturbation flag,
 b_i, test P@1, and the simulated makespan of the mega-batch (the time the
 slowest replica is busy, in cost units; the paper's wall clock on
@@ -34,6 +35,7 @@ ARMS = {
     "renorm": dict(method="adaptive", pert_renorm=True, norm="u", scale_every=1),
     "ub_se2": dict(method="adaptive", pert_renorm=False, norm="ub", scale_every=2),
     "elastic": dict(method="elastic", pert_renorm=False, norm="u", scale_every=1),
+    "renorm_r17": dict(method="adaptive", pert_renorm=True, norm="u", scale_every=0),
 }
 
 
@@ -43,7 +45,7 @@ def main():
     p.add_argument("--precision", default="bf16", choices=["fp32", "bf16"])
     p.add_argument("--replicas", type=int, default=4)
     p.add_argument("--hetero", default="0,0.5,1")
-    p.add_argument("--arms", default=",".join(ARMS))
+    p.add_argument("--arms", default="literal,renorm,ub_se2,elastic")
     p.add_argument("--megabatches", type=int, default=40)
     p.add_argument("--eval-rows", type=int, default=5000)
     p.add_argument("--out", default="gpurun_out/ab_sweep.json")
