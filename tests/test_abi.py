@@ -175,8 +175,9 @@ def test_hyper_rejects_unknown_method_switches():
     assert train.Hyper(**base, norm="ub", scale_every=3).scale_every == 3
     with pytest.raises(ValueError):
         train.Hyper(**base, norm="b")
+    assert train.Hyper(**base, scale_every=0).scale_every == 0      # R17 adaptive frequency
     with pytest.raises(ValueError):
-        train.Hyper(**base, scale_every=0)
+        train.Hyper(**base, scale_every=-1)
     with pytest.raises(ValueError):
         api.merge_weights([1, 2], [32, 32], [1.0, 1.0], norm="uu")
 
