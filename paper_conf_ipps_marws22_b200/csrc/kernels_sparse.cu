@@ -1043,6 +1043,111 @@ __global__ void __launch_bounds__(scatter_threads<T, CPL>(), 1)
   }
 }
 
+// K-5 for 64-column bf16 slices (b_max = 1024 shapes): a quarter-warp (8 lanes x 8 columns)
+// per feature segment, so each warp keeps four segments' W1 row slices and entry loads in
+// flight instead of one (the segment-per-warp form waits on two dependent round trips --
+// entries, then the W1 row -- per short segment: AmazonCat averages 3 entries).  Sums run
+// in the segment's row order: deterministic.
+__global__ void __launch_bounds__(1024, 1)
+    k_scatter_q(const int32_t* __restrict__ e_n, const float* __restrict__ e_v,
+                const int32_t* __restrict__ useg, const int32_t* __restrict__ uniq,
+                const int32_t* __restrict__ meta, const bf16* __restrict__ dA1, int H, float* W1,
+                float* grad_w1, int32_t* fcnt, uint32_t* bits, int W) {
+  pdl_trigger();
+  pdl_wait();
+  const float lr = step_lr(meta);
+  constexpr int CS = 64;
+  extern __shared__ __align__(16) uint8_t sm_raw[];
+  bf16* sd = reinterpret_cast<bf16*>(sm_raw);   // [n][CS]
+  const int slice = blockIdx.y, c0 = slice * CS;
+  const int n = meta[M_NROWS];
+  __shared__ __align__(8) uint64_t sbar;
+  const uint32_t bar = static_cast<uint32_t>(__cvta_generic_to_shared(&sbar));
+  const uint32_t row_bytes = CS * 2;
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"((uint32_t)n * row_bytes)
+                 : "memory");
+  }
+  __syncthreads();
+  {
+    const uint32_t dst0 = static_cast<uint32_t>(__cvta_generic_to_shared(sd));
+    for (int r = threadIdx.x; r < n; r += blockDim.x)
+      asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                       dst0 + (uint32_t)r * row_bytes),
+                   "l"(dA1 + (int64_t)r * H + c0), "r"(row_bytes), "r"(bar)
+                   : "memory");
+  }
+  const int lane = threadIdx.x & 31, grp = lane >> 3, gl = lane & 7;
+  const unsigned gmask = 0xFFu << (grp * 8);
+  const int U = meta[M_U];
+  const int nwarps = gridDim.x * (blockDim.x >> 5);
+  const int wid = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int ngroups = 4 * nwarps;
+  bool staged = false;
+  for (int u = 4 * wid + grp; u - grp < U; u += ngroups) {   // warp-uniform trip count
+    const bool active = u < U;
+    int j0 = 0, j1 = 0, f = 0;
+    float w[8];
+    if (active) {
+      j0 = useg[u]; j1 = useg[u + 1]; f = uniq[u];
+      const float4* wp = reinterpret_cast<const float4*>(W1 + (int64_t)f * H + c0 + gl * 8);
+      const float4 a = wp[0], b = wp[1];   // in flight during the gathers
+      w[0] = a.x; w[1] = a.y; w[2] = a.z; w[3] = a.w; w[4] = b.x; w[5] = b.y; w[6] = b.z; w[7] = b.w;
+    }
+    if (!staged) {
+      uint32_t ok = 0;
+      while (!ok)
+        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                     : "=r"(ok) : "r"(bar) : "memory");
+      staged = true;
+    }
+    if (!active) continue;
+    float acc[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] = 0.f;
+    for (int jb = j0; jb < j1; jb += 8) {
+      const int cnt = min(8, j1 - jb);
+      int myn = 0;
+      float myv = 0.f;
+      if (gl < cnt) { myn = e_n[jb + gl]; myv = e_v[jb + gl]; }
+      for (int q = 0; q < cnt; ++q) {
+        const int rr = __shfl_sync(gmask, myn, grp * 8 + q);
+        const float v = __shfl_sync(gmask, myv, grp * 8 + q);
+        const uint4 pk = reinterpret_cast<const uint4*>(sd + (int64_t)rr * CS)[gl];
+        const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&pk);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const float2 g = __bfloat1622float2(h[i]);
+          acc[2 * i] = fmaf(v, g.x, acc[2 * i]);
+          acc[2 * i + 1] = fmaf(v, g.y, acc[2 * i + 1]);
+        }
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) w[i] = w[i] - lr * acc[i];
+    float4* wp = reinterpret_cast<float4*>(W1 + (int64_t)f * H + c0 + gl * 8);
+    wp[0] = make_float4(w[0], w[1], w[2], w[3]);
+    wp[1] = make_float4(w[4], w[5], w[6], w[7]);
+    if (grad_w1) {
+      float4* gp = reinterpret_cast<float4*>(grad_w1 + (int64_t)f * H + c0 + gl * 8);
+      gp[0] = make_float4(acc[0], acc[1], acc[2], acc[3]);
+      gp[1] = make_float4(acc[4], acc[5], acc[6], acc[7]);
+    }
+    if (slice == 0) {   // K-0's per-feature count and row bitmap back to zero
+      if (gl == 0) fcnt[f] = 0;
+      for (int ww = gl; ww < W; ww += 8) bits[(int64_t)f * W + ww] = 0u;
+    }
+  }
+  if (!staged) {
+    uint32_t ok = 0;
+    while (!ok)
+      asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                   : "=r"(ok) : "r"(bar) : "memory");
+  }
+}
+
 // One resident wave of 256-thread CTAs (occupancy from the compiled kernel), no
 // more CTAs than there are 8-piece groups for the largest step.
 template <typename K>
@@ -1143,6 +1248,11 @@ bool k5_seg() {
   static const bool v = [] { const char* e = getenv("ASGD_K5_SEG"); return e && e[0] == '1'; }();
   return v;
 }
+// 64-column bf16 slices: ASGD_K5_Q=1 -> a quarter-warp per feature segment (k_scatter_q)
+bool k5_quarter() {
+  static const bool v = [] { const char* e = getenv("ASGD_K5_Q"); return e && e[0] == '1'; }();
+  return v;
+}
 
 template <typename T, int CPL>
 cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float* W1,
@@ -1151,6 +1261,14 @@ cudaError_t scatter_s_t(const Launch& lc, const T* dA1, int H, int b_max, float*
   const int nsl = H / CS;
   const size_t smem = (size_t)b_max * CS * sizeof(T);
   const int gx = std::max(1, lc.sms / nsl);
+  if constexpr (sizeof(T) == 2 && CS == 64) {
+    if (k5_quarter()) {   // 64-column bf16 slices: a quarter-warp per feature segment
+      cudaError_t e = ensure_smem(k_scatter_q, 200 * 1024);
+      if (e != cudaSuccess) return e;
+      return launch_k(lc, k_scatter_q, dim3(gx, nsl), dim3(1024), smem, P.e_n, P.e_v, P.useg, P.uniq, P.meta,
+                      reinterpret_cast<const bf16*>(dA1), H, W1, grad_w1, P.cnt, P.bits, (b_max + 31) / 32);
+    }
+  }
   if (k5_seg()) {
     cudaError_t e = ensure_smem(k_scatter_seg<T, CPL>, 200 * 1024);
     if (e != cudaSuccess) return e;

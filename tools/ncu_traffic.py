@@ -19,7 +19,9 @@ SECTIONS = {"dh_b1": 2, "merge": 3}
 
 def kclass(name: str):
     if name.startswith("k_gemm_tc"):
-        epi = int(re.findall(r"\d+", name.split("<")[1])[-1])
+        # k_gemm_tc<BN, A_MN, B_MN, EPI, X3>: the 4th template argument is the epilogue
+        args = re.findall(r"\w+", name.split("<")[1])
+        epi = int(args[3])
         return {0: "g1", 1: "g2", 2: "g3", 3: "softmax", 4: "g1", 5: "g1"}[epi]   # 4: sigmoid G1, 5: stats G1
     if name.startswith("k_bwd_dh"):
         return "g2"   # K-3's dH1 half (G1b + G2 + dH reduce): profiled as G2
