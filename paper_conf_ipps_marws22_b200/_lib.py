@@ -79,6 +79,7 @@ _SIGS = {
     "asgd_peer_close": (C.c_int, [_P]),
     "asgd_trace_enable": (C.c_int, [_P, _i32]),
     "asgd_trace_read": (C.c_int, [_P, _P, _i64, C.POINTER(_i64)]),
+    "asgd_timeline_set": (C.c_int, [_P]),
     "asgd_route_simulate": (C.c_int, [_i32, _P, _i64, _P, _f64, _P, _P, _i64, C.POINTER(_i64)]),
     "asgd_eval_topk": (C.c_int, [_P, C.POINTER(Csr), _P, _i32, _i32, _P]),
     "asgd_precision_at_k": (C.c_int, [_P, _P, _P, _i32, _i32, C.POINTER(_i64)]),

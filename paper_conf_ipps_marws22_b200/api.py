@@ -365,3 +365,11 @@ class Scheduler:
 
 def version() -> str:
     return lib().asgd_version().decode()
+
+
+TIMELINE_KERNELS = ["touched", "spmm", "g1", "softmax", "g2", "dh", "b1", "g3", "scatter", "g1b", "merge", "other"]
+
+
+def timeline_set(buf: Optional[torch.Tensor]):
+    """asgd_timeline_set: uint64[3 * len(TIMELINE_KERNELS)] device buffer (int64 tensor) or None."""
+    call("asgd_timeline_set", _ptr(buf) if buf is not None else None)

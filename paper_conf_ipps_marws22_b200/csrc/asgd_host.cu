@@ -848,6 +848,16 @@ int asgd_trace_read(asgd_ctx* c, int64_t* out, int64_t cap, int64_t* n_out) {
   return ASGD_OK;
 }
 
+int asgd_timeline_set(void* buf) {
+  unsigned long long* p = static_cast<unsigned long long*>(buf);
+  for (auto fn : {tl_set_sparse, tl_set_dense, tl_set_tc, tl_set_merge}) {
+    const cudaError_t e = fn(p);
+    if (e == cudaErrorNotSupported) return fail(ASGD_E_UNSUPPORTED, "libasgd built without -DASGD_TIMELINE");
+    if (e != cudaSuccess) return cuda_fail(e, "asgd_timeline_set");
+  }
+  return ASGD_OK;
+}
+
 int asgd_updates(const asgd_ctx* c, int64_t* u) {
   if (!c || !u) return fail(ASGD_E_ARG, "null argument");
   *u = c->u;

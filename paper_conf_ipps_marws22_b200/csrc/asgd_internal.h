@@ -80,6 +80,49 @@ struct Launch {       // launch bookkeeping of one ctx
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 
+// Kernel timeline (asgd_timeline_set, tools/timeline.py), compiled in only with
+// -DASGD_TIMELINE: per kernel class, [0] the earliest CTA arrival, [1] the earliest
+// return from griddepcontrol.wait (the predecessor's outputs are visible: on the
+// step's chain, the predecessor's end), [2] the latest CTA end (its last thread), in
+// %globaltimer ns.  Each translation unit holds its own copy of the buffer pointer.
+enum { TL_TOUCHED = 0, TL_SPMM, TL_G1, TL_SOFTMAX, TL_G2, TL_DH, TL_B1, TL_G3, TL_SCATTER, TL_G1B, TL_MERGE,
+       TL_OTHER, TL_N };
+#ifdef ASGD_TIMELINE
+static __device__ unsigned long long* g_tl;
+__device__ __forceinline__ unsigned long long tl_now() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+struct Tl {
+  int id;
+  unsigned long long t0;
+  __device__ explicit Tl(int i) : id(i), t0(tl_now()) {}
+  __device__ void ready() {
+    if (threadIdx.x == 0 && g_tl) {
+      atomicMin(&g_tl[3 * id], t0);
+      atomicMin(&g_tl[3 * id + 1], tl_now());
+    }
+  }
+  __device__ ~Tl() {
+    if (threadIdx.x == blockDim.x - 1 && g_tl) atomicMax(&g_tl[3 * id + 2], tl_now());
+  }
+};
+#define ASGD_TL_SETTER(fn) \
+  cudaError_t fn(unsigned long long* p) { return cudaMemcpyToSymbol(g_tl, &p, sizeof(p)); }
+#else
+struct Tl {
+  __device__ explicit Tl(int) {}
+  __device__ void ready() {}
+};
+#define ASGD_TL_SETTER(fn) \
+  cudaError_t fn(unsigned long long*) { return cudaErrorNotSupported; }
+#endif
+cudaError_t tl_set_sparse(unsigned long long*);
+cudaError_t tl_set_dense(unsigned long long*);
+cudaError_t tl_set_tc(unsigned long long*);
+cudaError_t tl_set_merge(unsigned long long*);
+
 // ASGD_PDL: unset = on for the bf16 path, off for fp32; 0 off; 1 every kernel; 2 the
 // tcgen05 GEMMs only
 int pdl_mode();

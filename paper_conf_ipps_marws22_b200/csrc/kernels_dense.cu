@@ -25,8 +25,10 @@ __global__ void __launch_bounds__(512) k_softmax_ce(int B, int64_t L, int64_t ld
                                                     bf16* dZb, bf16* dZl, float* rowloss,
                                                     const float2* __restrict__ stats, int ntiles,
                                                     int64_t stats_ld) {
+  Tl tl_(TL_SOFTMAX);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   __shared__ int s_lab[kMaxRowLabels];
   __shared__ float s_lz[kMaxRowLabels];
   __shared__ float s_m[16], s_s[16];
@@ -161,8 +163,10 @@ __global__ void __launch_bounds__(512) k_sigmoid_ce(int B, int64_t L, int64_t ld
                                                     const int64_t* __restrict__ lab_ptr,
                                                     const int32_t* __restrict__ lab, float* Z,
                                                     bf16* dZb, bf16* dZl, float* rowloss) {
+  Tl tl_(TL_SOFTMAX);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   __shared__ int s_lab[kMaxRowLabels];
   __shared__ float s_lz[kMaxRowLabels];
   __shared__ float s_sp[16];
@@ -237,8 +241,10 @@ __global__ void __launch_bounds__(512) k_sigmoid_ce(int B, int64_t L, int64_t ld
 // of the per-(tile half, row) BCE partials stats[t][n].x, in tile order.
 __global__ void __launch_bounds__(256) k_tile_loss(int ntiles, int64_t stats_ld, const float2* __restrict__ stats,
                                                    float* rowloss) {
+  Tl tl_(TL_SOFTMAX);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   __shared__ float s_w[8];
   const int n = blockIdx.x;
   float a = 0.f;
@@ -265,8 +271,10 @@ __global__ void __launch_bounds__(256) k_tile_loss(int ntiles, int64_t stats_ld,
 __global__ void __launch_bounds__(256) k_sig_center(const bf16* __restrict__ w2b, const float* __restrict__ w2f,
                                                     int64_t L, int H, const float* __restrict__ h1, int n,
                                                     float* part, unsigned int* counter, float* cen) {
+  Tl tl_(TL_OTHER);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   __shared__ float s_acc[8][512];
   __shared__ bool s_last;
   const int tpr = H / 8;                   // threads per W2 row (H <= 512 -> <= 64)
@@ -354,8 +362,10 @@ __global__ void __launch_bounds__(256) k_lse(int H, int ntiles, int64_t stats_ld
                                              const int32_t* __restrict__ lab, const bf16* __restrict__ h1b,
                                              const bf16* __restrict__ w2b, const float* __restrict__ b2,
                                              float* lse, float* rowloss) {
+  Tl tl_(TL_SOFTMAX);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   __shared__ float s_m[8], s_s[8], s_z[8];
   const int n = blockIdx.x, lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   float m = -INFINITY, s = 0.f;
@@ -409,8 +419,10 @@ __global__ void __launch_bounds__(256) k_lse(int H, int ntiles, int64_t stats_ld
 __global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
                             const float* __restrict__ part, const float* __restrict__ H1, float* dA1,
                             bf16* dA1b, const float* __restrict__ dh_off) {
+  Tl tl_(TL_DH);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   const int r = blockIdx.x, c = threadIdx.x;
   const int64_t o = (int64_t)r * H + c;
   float a[8];
@@ -433,8 +445,10 @@ __global__ void k_dh_reduce(int n, int H, int splitk, int64_t part_stride,
 __global__ void __launch_bounds__(256) k_b1_update(int n, int H, const float* __restrict__ dA1, float* b1,
                                                    const int32_t* __restrict__ meta, float* grad_b1,
                                                    const float* __restrict__ rowloss) {
+  Tl tl_(TL_B1);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   const float lr = step_lr(meta);
   float* loss_dev = step_loss(meta);
   const int lane = threadIdx.x & 31;
@@ -464,8 +478,10 @@ __global__ void __launch_bounds__(256) k_b1_update(int n, int H, const float* __
 }
 
 __global__ void k_to_bf16(const float* __restrict__ src, bf16* dst, bf16* dst_lo, int64_t count) {
+  Tl tl_(TL_OTHER);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count;
        i += (int64_t)gridDim.x * blockDim.x) {
     const float x = src[i];
@@ -529,4 +545,9 @@ cudaError_t launch_to_bf16(const Launch& lc, const float* src, bf16* dst, int64_
 
 int row_block() { return 1; }
 
+}  // namespace asgd
+
+
+namespace asgd {
+ASGD_TL_SETTER(tl_set_dense)
 }  // namespace asgd

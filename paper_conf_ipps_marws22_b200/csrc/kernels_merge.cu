@@ -18,8 +18,10 @@ constexpr unsigned kFull = 0xffffffffu;
 
 __global__ void __launch_bounds__(256) k_sqnorm_part(const float* __restrict__ x, int64_t P,
                                                      double* partials) {
+  Tl tl_(TL_MERGE);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   double s = 0.0;
   const int64_t P4 = P / 4;
   const float4* x4 = reinterpret_cast<const float4*>(x);
@@ -43,8 +45,10 @@ __global__ void __launch_bounds__(256) k_sqnorm_part(const float* __restrict__ x
 }
 
 __global__ void k_sqnorm_final(const double* __restrict__ partials, int n, double* out) {
+  Tl tl_(TL_MERGE);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   __shared__ double sh[32];
   double s = 0.0;
   // fixed assignment: thread t sums partials t, t+blockDim, ... in order
@@ -62,8 +66,10 @@ __global__ void k_sqnorm_final(const double* __restrict__ partials, int n, doubl
 }
 
 __global__ void __launch_bounds__(256) k_scale(float* x, int64_t P, double alpha) {
+  Tl tl_(TL_MERGE);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   const int64_t P4 = P / 4;
   float4* x4 = reinterpret_cast<float4*>(x);
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P4;
@@ -86,8 +92,10 @@ __device__ __forceinline__ void finish1(float& p, float& w, float& d, float gamm
 
 __global__ void __launch_bounds__(256) k_finish(float* params, float* w, float* d, int64_t P,
                                                 float gamma) {
+  Tl tl_(TL_MERGE);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   const int64_t P4 = P / 4;
   float4* p4 = reinterpret_cast<float4*>(params);
   float4* w4 = reinterpret_cast<float4*>(w);
@@ -106,8 +114,10 @@ __global__ void __launch_bounds__(256) k_finish(float* params, float* w, float* 
 __global__ void __launch_bounds__(256) k_wsum(const float* const* __restrict__ reps,
                                               const double* __restrict__ alpha, int n, int64_t P,
                                               float* out) {
+  Tl tl_(TL_MERGE);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P;
        i += (int64_t)gridDim.x * blockDim.x) {
     double s = 0.0;
@@ -138,8 +148,10 @@ __device__ __forceinline__ void merge1(const PeerSet& ps, int64_t i, float& w, f
 
 __global__ void __launch_bounds__(256) k_merge_fused(PeerSet ps, float* w, float* d, int64_t lo, int64_t hi,
                                                      float gamma, unsigned int* cta_done) {
+  Tl tl_(TL_MERGE);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   const int64_t lo4 = lo / 4, hi4 = hi / 4;   // lo is a multiple of 4; the tail (hi % 4) is scalar
   for (int64_t i4 = lo4 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i4 < hi4;
        i4 += (int64_t)gridDim.x * blockDim.x) {
@@ -192,8 +204,10 @@ __device__ __forceinline__ bool better(const Cand& a, const Cand& b) {
 template <int K>
 __global__ void __launch_bounds__(256) k_topk(int64_t L, int64_t ldz, int k, const float* __restrict__ z,
                                               int32_t* out) {
+  Tl tl_(TL_OTHER);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   const int n = blockIdx.x;
   const float* row = z + (int64_t)n * ldz;
   Cand top[K];
@@ -230,8 +244,10 @@ __global__ void __launch_bounds__(256) k_topk(int64_t L, int64_t ldz, int k, con
 
 // -------------------------------------------------------------- validation
 __global__ void k_validate(asgd_csr c, int64_t F, int64_t L, int32_t* err) {
+  Tl tl_(TL_OTHER);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < c.n_rows;
        r += (int64_t)gridDim.x * blockDim.x) {
     int e = 0;
@@ -312,4 +328,9 @@ cudaError_t launch_validate_csr(const Launch& lc, const asgd_csr* c, int64_t F, 
   return cudaGetLastError();
 }
 
+}  // namespace asgd
+
+
+namespace asgd {
+ASGD_TL_SETTER(tl_set_merge)
 }  // namespace asgd

@@ -285,8 +285,10 @@ __global__ void __launch_bounds__(512) k_touched(StepArgs sa, const int64_t* __r
                                                  int32_t* fseg, int32_t* fuid, int32_t* uniq,
                                                  int32_t* useg, uint32_t* bits, int W, int32_t* e_n,
                                                  float* e_v, int32_t* e_u, int32_t* e_f) {
+  Tl tl_(TL_TOUCHED);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   extern __shared__ int32_t sboff[];
   __shared__ int s_red[2][16];
   __shared__ int s_pre[2];
@@ -398,9 +400,24 @@ __global__ void __launch_bounds__(512) k_touched(StepArgs sa, const int64_t* __r
 #endif
 template <int VPL>   // pieces per group = warps per K-1 CTA (H = 512: 8, the partials fill 32 KB)
 constexpr int k1_group() { return VPL >= 16 ? 8 : ASGD_K1_GROUP; }
+// TMA-staged K-1 (k1_tma()): every W1 row of a warp's piece is requested at once as one
+// bulk async copy per entry into the warp's 32-row shared-memory slot array, completed on
+// the warp's mbarrier; the FMAs then read shared memory.  fp32 rows of H floats: 6 warps
+// x 32 KB at H = 256 (one CTA per SM), 8 warps below.
 template <int VPL>
+constexpr int k1_group_tma() { return VPL >= 8 ? 6 : 8; }
+template <int VPL, bool TMA>
+constexpr int k1_warps() { return TMA ? k1_group_tma<VPL>() : k1_group<VPL>(); }
+template <int VPL, bool TMA>
+constexpr int k1_min_ctas() { return TMA ? (VPL >= 8 ? 1 : 2) : 16 / k1_group<VPL>(); }
+// dynamic shared memory of K-1: the batch view of up to b_max = 2048 rows, then (TMA) the
+// row slots, 128-B aligned
+constexpr size_t k1_view_bytes() { return (view_smem(2048) + 127) & ~size_t(127); }
+template <int VPL, bool TMA>
+constexpr size_t k1_smem() { return k1_view_bytes() + (TMA ? (size_t)k1_warps<VPL, TMA>() * kPiece * VPL * 128 : 0); }
+template <int VPL, bool TMA>
 // (256, 2): two CTAs per SM, all kU gathers of a group in flight (<= 128 regs)
-__global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_spmm_fwd(StepArgs sa, const int64_t* __restrict__ row_ptr,
+__global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, TMA>())) k_spmm_fwd(StepArgs sa, const int64_t* __restrict__ row_ptr,
                                                   const int64_t* __restrict__ lab_ptr, int64_t n_data_rows,
                                                   int64_t nz_cap, int64_t nl_cap, ViewOut vo,
                                                   const int32_t* __restrict__ col,
@@ -408,8 +425,10 @@ __global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_
                                                   const float* __restrict__ W1,
                                                   const float* __restrict__ b1, float* H1,
                                                   bf16* H1b, bf16* H1l, float* part, int32_t* rowcnt) {
+  Tl tl_(TL_SPMM);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   using IO = RowIO<VPL>;
   constexpr int H = 32 * VPL;
   constexpr int kU = VPL >= 16 ? 4 : 8;   // W1 rows in flight per warp
@@ -424,9 +443,22 @@ __global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_
   // Pieces are taken in groups of 8 consecutive pieces, one per warp of the CTA, so a
   // row that crosses pieces is first combined inside the CTA through shared memory;
   // only rows that cross a group boundary go through global partials, one per group.
-  constexpr int kGroup = k1_group<VPL>();        // pieces per group = warps per CTA
+  constexpr int kGroup = k1_warps<VPL, TMA>();   // pieces per group = warps per CTA
   __shared__ __align__(16) float spart[kGroup][2][H];   // per warp: [0] its first segment, [1] its last
   const int warp = threadIdx.x >> 5;
+  // TMA: this warp's kPiece row slots and its mbarrier (one phase per piece)
+  float* slots = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(sboff) + k1_view_bytes()) +
+                 (size_t)warp * kPiece * H;
+  __shared__ __align__(8) uint64_t sbar[kGroup];
+  const uint32_t bar = static_cast<uint32_t>(__cvta_generic_to_shared(&sbar[warp]));
+  uint32_t phase = 0;
+  if constexpr (TMA) {
+    if (lane == 0) {
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar) : "memory");
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+  }
   // pieces per group: up to one per warp, fewer when the batch has fewer than kGroup
   // pieces per CTA, so every CTA of the grid gets a group (EURLex: 1,875 pieces -> 13 per
   // group on 145 CTAs instead of 16 on 117); the idle warps only join the barriers
@@ -508,32 +540,70 @@ __global__ void __launch_bounds__(32 * k1_group<VPL>(), 16 / k1_group<VPL>()) k_
       float acc[VPL];
 #pragma unroll
       for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
-      // groups of kU W1 rows in flight, row changes handled between FMAs
-      for (int j0 = 0; j0 < cnt; j0 += kU) {
-        float w[kU][VPL];
-#pragma unroll
-        for (int q = 0; q < kU; ++q) {
-          const int c = __shfl_sync(kFull, mycol, j0 + q);
-          if (j0 + q < cnt) IO::load_ldg(W1 + (int64_t)c * H, lane, w[q]);
-          else {
-#pragma unroll
-            for (int i = 0; i < VPL; ++i) w[q][i] = 0.f;
-          }
-        }
-#pragma unroll
-        for (int q = 0; q < kU; ++q) {
-          const int j = j0 + q;
+      if constexpr (TMA) {
+        // every row of the piece in flight at once: one bulk copy per entry into slot j
+        if (lane == 0)
+          asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
+                       "r"((uint32_t)(cnt * H * 4))
+                       : "memory");
+        __syncwarp();
+        if (lane < cnt)
+          asm volatile(
+              "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                  static_cast<uint32_t>(__cvta_generic_to_shared(slots + (size_t)lane * H))),
+              "l"(W1 + (int64_t)mycol * H), "r"((uint32_t)(H * 4)), "r"(bar)
+              : "memory");
+        uint32_t ok = 0;
+        while (!ok)
+          asm volatile(
+              "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+              : "=r"(ok)
+              : "r"(bar), "r"(phase)
+              : "memory");
+        phase ^= 1u;
+        for (int j = 0; j < cnt; ++j) {
+          float w[VPL];
+          IO::load(slots + (size_t)j * H, lane, w);
           const int rq = __shfl_sync(kFull, myr, j);
           const float v = __shfl_sync(kFull, myval, j);
-          if (j < cnt) {
-            if (rq != rcur) {
-              flush(rcur, acc);
+          if (rq != rcur) {
+            flush(rcur, acc);
 #pragma unroll
-              for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
-              rcur = rq;
+            for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+            rcur = rq;
+          }
+#pragma unroll
+          for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, w[i], acc[i]);
+        }
+        __syncwarp();   // every lane has read the slots before the next piece's copies land
+      } else {
+      // groups of kU W1 rows in flight, row changes handled between FMAs
+        for (int j0 = 0; j0 < cnt; j0 += kU) {
+          float w[kU][VPL];
+  #pragma unroll
+          for (int q = 0; q < kU; ++q) {
+            const int c = __shfl_sync(kFull, mycol, j0 + q);
+            if (j0 + q < cnt) IO::load_ldg(W1 + (int64_t)c * H, lane, w[q]);
+            else {
+  #pragma unroll
+              for (int i = 0; i < VPL; ++i) w[q][i] = 0.f;
             }
-#pragma unroll
-            for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, w[q][i], acc[i]);
+          }
+  #pragma unroll
+          for (int q = 0; q < kU; ++q) {
+            const int j = j0 + q;
+            const int rq = __shfl_sync(kFull, myr, j);
+            const float v = __shfl_sync(kFull, myval, j);
+            if (j < cnt) {
+              if (rq != rcur) {
+                flush(rcur, acc);
+  #pragma unroll
+                for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
+                rcur = rq;
+              }
+  #pragma unroll
+              for (int i = 0; i < VPL; ++i) acc[i] = fmaf(v, w[q][i], acc[i]);
+            }
           }
         }
       }
@@ -598,8 +668,10 @@ __global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__
                                                      const float* __restrict__ dA1, float* W1,
                                                      float* part, int32_t* ucnt,
                                                      float* grad_w1, int32_t* cnt, uint32_t* bits, int W) {
+  Tl tl_(TL_SCATTER);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   const float lr = step_lr(meta);
   using IO = RowIO<VPL>;
   constexpr int H = 32 * VPL;
@@ -767,8 +839,10 @@ __global__ void __launch_bounds__(scatter_threads<T, CPL>(), 1) k_scatter_sgd_s(
                                                           float* part, int32_t* ucnt,
                                                           float* grad_w1, int32_t* fcnt, uint32_t* bits,
                                                           int W) {
+  Tl tl_(TL_SCATTER);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   const float lr = step_lr(meta);
   constexpr int CS = 32 * CPL;               // columns of this CTA's slice
   constexpr int kU = 8;
@@ -950,8 +1024,10 @@ __global__ void __launch_bounds__(scatter_threads<T, CPL>(), 1)
                   const int32_t* __restrict__ useg, const int32_t* __restrict__ uniq,
                   const int32_t* __restrict__ meta, const T* __restrict__ dA1, int H, float* W1,
                   float* grad_w1, int32_t* fcnt, uint32_t* bits, int W) {
+  Tl tl_(TL_SCATTER);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   const float lr = step_lr(meta);
   constexpr int CS = 32 * CPL;
   extern __shared__ __align__(16) uint8_t sm_raw[];
@@ -1053,8 +1129,10 @@ __global__ void __launch_bounds__(1024, 1)
                 const int32_t* __restrict__ useg, const int32_t* __restrict__ uniq,
                 const int32_t* __restrict__ meta, const bf16* __restrict__ dA1, int H, float* W1,
                 float* grad_w1, int32_t* fcnt, uint32_t* bits, int W) {
+  Tl tl_(TL_SCATTER);
   pdl_trigger();
   pdl_wait();
+  tl_.ready();
   const float lr = step_lr(meta);
   constexpr int CS = 64;
   extern __shared__ __align__(16) uint8_t sm_raw[];
@@ -1158,19 +1236,20 @@ int wave_grid(const Launch& lc, K kernel, size_t smem, int64_t pieces, int& occ,
   return (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)lc.sms * occ));
 }
 
-template <int VPL>
+template <int VPL, bool TMA>
 cudaError_t spmm_fwd_t(const Launch& lc, const StepArgs& sa, const asgd_csr& x, const float* W1, const float* b1,
                        const Ptrs& P, const WsLayout& L, bool want_bf16) {
-  const size_t smem = view_smem(sa.n);
+  const size_t smem = TMA ? k1_smem<VPL, TMA>() : view_smem(sa.n);
   // the batch view (dynamic) + the group partials (static) exceed 48 KB at b_max = 2048
-  cudaError_t e = ensure_smem(k_spmm_fwd<VPL>, view_smem(2048));
+  cudaError_t e = ensure_smem(k_spmm_fwd<VPL, TMA>, TMA ? k1_smem<VPL, TMA>() : view_smem(2048));
   if (e != cudaSuccess) return e;
   static int occ = 0;
-  const int grid = wave_grid(lc, k_spmm_fwd<VPL>, view_smem(2048), L.n_pieces, occ, k1_group<VPL>());
+  const int grid = wave_grid(lc, k_spmm_fwd<VPL, TMA>, TMA ? k1_smem<VPL, TMA>() : view_smem(2048), L.n_pieces, occ,
+                             k1_warps<VPL, TMA>());
   const ViewOut vo{P.boff, P.loff, P.rbase, P.rowsc, P.meta};
-  launch_k(lc, k_spmm_fwd<VPL>, dim3(grid), dim3(32 * k1_group<VPL>()), smem, sa, x.row_ptr, x.lab_ptr, x.n_rows, L.nz_cap, L.nl_cap,
-           vo, x.col, x.val, W1, b1, P.h1, want_bf16 ? P.h1b : nullptr, want_bf16 ? P.h1l : nullptr, P.part1,
-           P.rowcnt);
+  launch_k(lc, k_spmm_fwd<VPL, TMA>, dim3(grid), dim3(32 * k1_warps<VPL, TMA>()), smem, sa, x.row_ptr, x.lab_ptr,
+           x.n_rows, L.nz_cap, L.nl_cap, vo, x.col, x.val, W1, b1, P.h1, want_bf16 ? P.h1b : nullptr,
+           want_bf16 ? P.h1l : nullptr, P.part1, P.rowcnt);
   return cudaGetLastError();
 }
 
@@ -1216,23 +1295,34 @@ cudaError_t launch_touched(const Launch& lc, const StepArgs& sa, const asgd_csr&
                   P.e_v, P.e_u, P.e_f);
 }
 
+// K-1 with TMA-staged W1 rows (H <= 256): ASGD_K1_TMA=0 keeps the register-gather kernel
+bool k1_tma() {
+  static const bool v = [] { const char* e = getenv("ASGD_K1_TMA"); return !(e && e[0] == '0'); }();
+  return v;
+}
+
 cudaError_t launch_spmm_fwd(const Launch& lc, const StepArgs& sa, const asgd_csr& x, const float* W1,
                             const float* b1, int H, const Ptrs& P, const WsLayout& L, bool want_bf16) {
+  const bool t = k1_tma();
   switch (H) {
-    case 64: return spmm_fwd_t<2>(lc, sa, x, W1, b1, P, L, want_bf16);
-    case 128: return spmm_fwd_t<4>(lc, sa, x, W1, b1, P, L, want_bf16);
-    case 256: return spmm_fwd_t<8>(lc, sa, x, W1, b1, P, L, want_bf16);
-    case 512: return spmm_fwd_t<16>(lc, sa, x, W1, b1, P, L, want_bf16);
+    case 64: return t ? spmm_fwd_t<2, true>(lc, sa, x, W1, b1, P, L, want_bf16)
+                      : spmm_fwd_t<2, false>(lc, sa, x, W1, b1, P, L, want_bf16);
+    case 128: return t ? spmm_fwd_t<4, true>(lc, sa, x, W1, b1, P, L, want_bf16)
+                       : spmm_fwd_t<4, false>(lc, sa, x, W1, b1, P, L, want_bf16);
+    case 256: return t ? spmm_fwd_t<8, true>(lc, sa, x, W1, b1, P, L, want_bf16)
+                       : spmm_fwd_t<8, false>(lc, sa, x, W1, b1, P, L, want_bf16);
+    case 512: return spmm_fwd_t<16, false>(lc, sa, x, W1, b1, P, L, want_bf16);
     default: return cudaErrorInvalidValue;
   }
 }
 
 const void* spmm_fwd_func(int H) {
+  const bool t = k1_tma();
   switch (H) {
-    case 64: return reinterpret_cast<const void*>(k_spmm_fwd<2>);
-    case 128: return reinterpret_cast<const void*>(k_spmm_fwd<4>);
-    case 256: return reinterpret_cast<const void*>(k_spmm_fwd<8>);
-    default: return reinterpret_cast<const void*>(k_spmm_fwd<16>);
+    case 64: return t ? reinterpret_cast<const void*>(k_spmm_fwd<2, true>) : reinterpret_cast<const void*>(k_spmm_fwd<2, false>);
+    case 128: return t ? reinterpret_cast<const void*>(k_spmm_fwd<4, true>) : reinterpret_cast<const void*>(k_spmm_fwd<4, false>);
+    case 256: return t ? reinterpret_cast<const void*>(k_spmm_fwd<8, true>) : reinterpret_cast<const void*>(k_spmm_fwd<8, false>);
+    default: return reinterpret_cast<const void*>(k_spmm_fwd<16, false>);
   }
 }
 
@@ -1240,7 +1330,7 @@ const void* touched_func() { return reinterpret_cast<const void*>(k_touched); }
 
 template <typename... A>
 constexpr int nargs_of(void (*)(A...)) { return (int)sizeof...(A); }
-int spmm_fwd_nargs() { return nargs_of(k_spmm_fwd<8>); }
+int spmm_fwd_nargs() { return nargs_of(k_spmm_fwd<8, false>); }
 int touched_nargs() { return nargs_of(k_touched); }
 
 // K-5 layout: ASGD_K5_SEG=1 -> one warp per feature segment (k_scatter_seg), else nnz pieces
@@ -1312,4 +1402,9 @@ cudaError_t launch_scatter_sgd(const Launch& lc, float* W1, int H, const Ptrs& P
   }
 }
 
+}  // namespace asgd
+
+
+namespace asgd {
+ASGD_TL_SETTER(tl_set_sparse)
 }  // namespace asgd

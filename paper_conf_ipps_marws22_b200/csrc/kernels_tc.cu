@@ -443,6 +443,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
   uint64_t* afull = tempty + 2;   // resident A block loaded
   uint32_t* tbase = reinterpret_cast<uint32_t*>(afull + 1);
 
+  Tl tl_((EPI == TC_EPI_PART ? TL_G2 : EPI == TC_EPI_SGD ? TL_G3 : EPI == TC_EPI_DZ ? TL_G1B : TL_G1));
   pdl_trigger();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int MT = (g.M + BM - 1) / BM, NT = (g.N + BN - 1) / BN, Z = g.splits;
@@ -490,6 +491,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
   tc_fence_after();
   const uint32_t tmem = *tbase;
   pdl_wait();   // operands / outputs of the previous kernel are visible from here on
+  tl_.ready();
 
   if (warp == 0) {
     if (lane == 0) {
@@ -983,6 +985,7 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
   uint64_t* dhfull = hfull + 1;
   uint32_t* tbase = reinterpret_cast<uint32_t*>(dhfull + 1);
 
+  Tl tl_(TL_G2);
   pdl_trigger();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int MT = (g.M + BM - 1) / BM, T = (g.N + kBwdBN - 1) / kBwdBN;
@@ -1011,6 +1014,7 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
   tc_fence_after();
   const uint32_t tmem = *tbase;
   pdl_wait();
+  tl_.ready();
 
   if (warp == 0) {
     if (lane == 0 && nt > 0) {   // ------------------------------------ TMA producer
@@ -1235,6 +1239,7 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
   uint64_t* tempty = tfull + 1;
   uint32_t* tbase = reinterpret_cast<uint32_t*>(tempty + 1);
 
+  Tl tl_(TL_G3);
   pdl_trigger();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n = g.K;                                     // batch rows
@@ -1264,6 +1269,7 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
   tc_fence_after();
   const uint32_t tmem = *tbase;
   pdl_wait();
+  tl_.ready();
   // label cursors: the first label of each row >= this CTA's first label (binary search,
   // all threads, rows strided), kept in smem and advanced as the tiles increase
   if (nt > 0) {
@@ -1762,4 +1768,9 @@ cudaError_t launch_bwd_dw(const Launch& lc, int n, int64_t L, int H, const Ptrs&
   return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_bwd_dw, dim3(grid), dim3(128 + 32 * kBwdEpi), smem, tw, th, g);
 }
 
+}  // namespace asgd
+
+
+namespace asgd {
+ASGD_TL_SETTER(tl_set_tc)
 }  // namespace asgd

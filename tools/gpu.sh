@@ -10,6 +10,8 @@
 #   full:CFG:REGEX   ncu --set full capture of the kernels matching REGEX (one step)
 #   sanitize         compute-sanitizer memcheck / racecheck / synccheck on tiny + EURLex steps
 #   sass             per-kernel SASS census of libasgd.so (UTC*MMA, UTMALDG, LDTM ...)
+#   timeline:CFG[:PREC]  live per-kernel timeline of one local step (-DASGD_TIMELINE build)
+#   ab:NAME:FLAGS    bench line with libasgd rebuilt with ASGD_NVCC_EXTRA=FLAGS     -> TAG_ab_NAME.json
 T=$1; shift
 mkdir -p gpurun_out
 export ASGD_PARITY_LOG=$PWD/gpurun_out/${T}_parity.jsonl
@@ -45,6 +47,17 @@ for J in "$@"; do
       timeout 1200 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_steps.py \
         > gpurun_out/${T}_san_${tool}.log 2>&1; echo "sanitize $tool $?"; tail -2 gpurun_out/${T}_san_${tool}.log
     done ;;
+  timeline)
+    ASGD_NVCC_EXTRA=-DASGD_TIMELINE python -m paper_conf_ipps_marws22_b200.build --force > /dev/null 2>&1
+    timeout 600 python tools/timeline.py --config $A --precision ${B:-bf16} --out gpurun_out/${T}_tl_${A}_${B:-bf16}.json \
+      > gpurun_out/${T}_tl_${A}_${B:-bf16}.txt 2>&1; echo "timeline $A $?"; cat gpurun_out/${T}_tl_${A}_${B:-bf16}.txt
+    python -m paper_conf_ipps_marws22_b200.build --force > /dev/null 2>&1 ;;
+  ab)
+    ASGD_NVCC_EXTRA="$B" python -m paper_conf_ipps_marws22_b200.build --force > /dev/null 2>&1 || echo "build $B failed"
+    O=gpurun_out/${T}_ab_${A}.json
+    timeout 900 python bench.py --no-cpu-baseline --ttp-megabatches 0 > $O 2> ${O%.json}.err
+    echo "ab $A [$B] $?"; python tools/bench_brief.py $O
+    python -m paper_conf_ipps_marws22_b200.build --force > /dev/null 2>&1 ;;
   sass)
     python tools/sass_census.py > gpurun_out/${T}_sass.md; echo "sass $?" ;;
   *)
