@@ -175,9 +175,10 @@ int asgd_trace_read(asgd_ctx* ctx, int64_t* out_host, int64_t cap, int64_t* n_ou
 
 /* Kernel timeline (diagnostic, process-wide, current device): with buf_dev non-null
  * every kernel of the library records, per kernel class k (TL_* order: touched, spmm,
- * g1, softmax, g2, dh, b1, g3, scatter, g1b, merge, other), buf_dev[3k] = min CTA
- * arrival, buf_dev[3k+1] = min return from its wait on the predecessor kernel,
- * buf_dev[3k+2] = max CTA end, as %globaltimer ns (uint64[36] device, caller-owned;
+ * g1, softmax, g2, dh, b1, g3, scatter, g1b, merge, other, then 8 in-kernel phase
+ * marks ph0..ph7), buf_dev[3k] = min CTA arrival, buf_dev[3k+1] = min return from its
+ * wait on the predecessor kernel, buf_dev[3k+2] = max CTA end (phase marks: only this
+ * slot), as %globaltimer ns (uint64[60] device, caller-owned;
  * the caller fills the min slots with ~0 and the max slots with 0 before a step).
  * NULL turns it off.  ASGD_E_UNSUPPORTED unless libasgd was built with
  * -DASGD_TIMELINE (the probes are compiled out of the default build). */

@@ -367,7 +367,8 @@ def version() -> str:
     return lib().asgd_version().decode()
 
 
-TIMELINE_KERNELS = ["touched", "spmm", "g1", "softmax", "g2", "dh", "b1", "g3", "scatter", "g1b", "merge", "other"]
+TIMELINE_KERNELS = ["touched", "spmm", "g1", "softmax", "g2", "dh", "b1", "g3", "scatter", "g1b", "merge", "other",
+                    "ph0", "ph1", "ph2", "ph3", "ph4", "ph5", "ph6", "ph7"]
 
 
 def timeline_set(buf: Optional[torch.Tensor]):

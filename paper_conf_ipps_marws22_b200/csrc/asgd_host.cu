@@ -94,6 +94,20 @@ bool bwd_dw() {
 // measured on EURLex-4K (bf16) 6.99 ms vs 6.30 ms per mega-batch -- the tail's grid barrier
 // and its 30-CTA reduce cost more than the separate 256-CTA k_dh_reduce launch (b1 runs
 // off the critical path on s3).  The same tail ends K-3's k_bwd_dh, where the grid is 144 CTAs.
+// K-3 one-pass for the stored-Z regime (bf16, softmax, H = 256: EURLex-4K): k_bwd_dh alone
+// replaces G1 + softmax-CE + G2 + the dH reduce on the critical path (ASGD_ONEPASS=1).
+// Measured slower at EURLex (34 vs ~25 us for the four kernels): with one label tile per
+// CTA the 63 dH1 partials (16 MB) and two grid barriers outweigh the launches it saves.
+bool one_pass_on() {
+  static const bool v = [] { const char* e = getenv("ASGD_ONEPASS"); return e && e[0] == '1'; }();
+  return v;
+}
+// K-3 softmax-only for the stored-Z regime (ASGD_K3DZ=1): k_bwd_dh with one label tile per
+// CTA stands for G1 + softmax-CE (statistics from its S tiles, a grid barrier, dZ stored)
+bool k3dz_on() {
+  static const bool v = [] { const char* e = getenv("ASGD_K3DZ"); return e && e[0] == '1'; }();
+  return v;
+}
 bool g2_fuse() {
   static const bool v = [] { const char* e = getenv("ASGD_G2_FUSE"); return e && e[0] == '1'; }();
   return v;
@@ -165,7 +179,12 @@ WsLayout ws_layout(const asgd_model_desc& d) {
   L.lse = take(B * 4);
   L.zstat = take(bf ? (size_t)((Lb + 31) / 32 + 8) * B * 8 : 0);   // G1 partials (2 or 4 per N tile)
   L.rowloss = take(B * 4);
-  L.dhpart = take((size_t)L.splitk * B * H * 4);
+  // K-3 one-pass regime (bf16 softmax, H = 256, logits below the fused-CE bound): room for
+  // one dH1 partial per label tile of 64 (at most 64), so every SM gets a K-3 CTA
+  L.dh_parts = L.splitk;
+  if (d.precision == ASGD_PREC_BF16 && d.loss == ASGD_LOSS_SOFTMAX && H == 256 && B * Lb * 4 <= fused_ce_bytes())
+    L.dh_parts = std::max<int64_t>(L.splitk, std::min<int64_t>((Lb + 63) / 64, 64));
+  L.dhpart = take((size_t)L.dh_parts * B * H * 4);
   L.da1 = take(B * H * 4);
   L.db1part = take(std::max<int64_t>(L.n_rowblk, 160) * H * 4);   // + G2's fused column partials
   L.w2b = take(bf ? (size_t)Lb * H * 2 : 0);
@@ -550,7 +569,8 @@ int enqueue_step(asgd_ctx* c, int n) {
   float* W2 = c->params + c->o_w2;
   float* b2 = c->params + c->o_b2;
   float* g = c->dbg;
-  static const bool k0_late = [] { const char* e = getenv("ASGD_K0_LATE"); return e && e[0] == '1'; }();
+  // K-0 after K-1 (ASGD_K0_LATE=1, or with K-0's phase A folded into K-1)
+  static const bool k0_late = [] { const char* e = getenv("ASGD_K0_LATE"); return (e && e[0] == '1') || k0_fold(); }();
   auto fork_k0 = [&]() -> int {
     CU(cudaEventRecord(c->ev_fork, c->s));
     CU(cudaStreamWaitEvent(c->s2, c->ev_fork, 0));
@@ -560,7 +580,7 @@ int enqueue_step(asgd_ctx* c, int n) {
   };
   if (!k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   // K-1
-  PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, c->sa, x, W1, b1, H, P, c->L, true));   // H1 fp32 + bf16 (+ lo)
+  PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, c->sa, x, W1, b1, H, P, c->L, true, k0_fold(), (int)m.b_max));   // H1 fp32 + bf16 (+ lo)
   if (k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   {
     // A DAG over three streams (both precisions; the fp32 path's GEMMs take bf16x3
@@ -585,7 +605,18 @@ int enqueue_step(asgd_ctx* c, int n) {
     const bool k3 = bf && m.loss == ASGD_LOSS_SOFTMAX && (int64_t)m.b_max * Lb * 4 > fused_ce_bytes() && H == 256 &&
                     bwd_fuse();
     const bool k3dw = k3 && bwd_dw() && n <= 1024;
-    if (x3) {
+    // K-3 one-pass: no G1 / softmax launch before it (the statistics come from its S tiles)
+    const bool k3one = bf && m.loss == ASGD_LOSS_SOFTMAX && H == 256 && !k3 && bwd_fuse() && one_pass_on() &&
+                       bwd_dh_one_pass_fits(n, Lb, c->L, c->sms);
+    const bool k3dz = !k3one && bf && m.loss == ASGD_LOSS_SOFTMAX && H == 256 && !k3 && k3dz_on() &&
+                      (int64_t)m.b_max * Lb * 4 <= fused_ce_bytes();
+    if (k3one) {
+      // nothing before K-3: G3 follows it (needs its dZ)
+    } else if (k3dz) {
+      // G1 + softmax-CE as one kernel: S tiles -> statistics -> grid barrier -> lse, row loss -> dZ
+      const DhFuse fz{nullptr, nullptr, nullptr, bf};
+      PCU(ASGD_K_G1, launch_bwd_dh(lc, n, Lb, H, Pr, c->L, b2, P.rowsc, x.lab_ptr, x.lab, fz, true, true, zstat, true));
+    } else if (x3) {
       // fp32 path: G1 stores Z (+ per-tile softmax partials), then the loss kernel writes dZ
       // as bf16x3 hi + lo (sigmoid: centred, R11 / R14)
       PCU(ASGD_K_G1, launch_gemm_tc(lc, 1, n, Lb, H, Pr, c->L, W2, b2, nullptr, nullptr, zstat, &ntiles));
@@ -643,13 +674,21 @@ int enqueue_step(asgd_ctx* c, int n) {
     // (Amazon-670K: 148 persistent CTAs each, one per SM) concurrent launches interleave
     // their CTAs and the later kernel's static tile split waits on the earlier one's SMs
     // (measured 1024 us for the pair against 326 + 572 us back to back), so G3 runs last
-    const bool g3_side = 2 * g2c <= c->sms;
+    const bool g3_side = 2 * g2c <= c->sms && !k3one;
     if (g3_side) {
       CU(cudaEventRecord(c->ev_sm, c->s));
       CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
       PCU_ON(c->s3, ASGD_K_G3, g3(lc3));
     }
-    if (k3) {
+    if (k3one) {
+      // K-3 one-pass: S tiles -> softmax partials -> grid barrier -> lse, row loss -> dZ (on
+      // chip into dH1, TMA-stored for G3) -> dH1 reduce + b1 in the tail; G3 beside K-5
+      const DhFuse fz{b1, g ? g + c->o_b1 : nullptr, nullptr, bf};
+      PCU(ASGD_K_G2, launch_bwd_dh(lc, n, Lb, H, Pr, c->L, b2, P.rowsc, x.lab_ptr, x.lab, fz, true, true, zstat));
+      CU(cudaEventRecord(c->ev_sm, c->s));
+      CU(cudaStreamWaitEvent(c->s3, c->ev_sm, 0));
+      PCU_ON(c->s3, ASGD_K_G3, g3(c->lc3()));
+    } else if (k3) {
       // K-3: Z recomputed, dZ on chip into dH1 (+ TMA-stored for G3), dH1 reduce + b1 in the tail
       const DhFuse fz{b1, g ? g + c->o_b1 : nullptr, nullptr, bf};
       PCU(ASGD_K_G2, launch_bwd_dh(lc, n, Lb, H, Pr, c->L, b2, P.rowsc, x.lab_ptr, x.lab, fz, !k3dw));
@@ -667,12 +706,12 @@ int enqueue_step(asgd_ctx* c, int n) {
     }
     // join s3 back into s only when work went there (an event recorded on a stream outside
     // the capture cannot be waited on inside it)
-    const bool s3_used = g3_side || !(k3 || g2_fuse());
+    const bool s3_used = g3_side || k3one || !(k3 || g2_fuse());
     if (s3_used) CU(cudaEventRecord(c->ev_a, c->s3));
     // K-5 (needs K-0's segments)
     CU(cudaStreamWaitEvent(c->s, c->ev_join, 0));
     PCU(ASGD_K_SCATTER, launch_scatter_sgd(lc, W1, H, P, c->L, g ? g + c->o_w1 : nullptr, bf ? P.da1b : nullptr, m.b_max));
-    if (!g3_side) PCU(ASGD_K_G3, g3(lc));
+    if (!g3_side && !k3one) PCU(ASGD_K_G3, g3(lc));
     if (s3_used) CU(cudaStreamWaitEvent(c->s, c->ev_a, 0));
   }
   return ASGD_OK;
@@ -731,7 +770,7 @@ int step_graph(asgd_ctx* c, int n) {
       std::vector<cudaGraphNode_t> nodes(nn);
       CU(cudaGraphGetNodes(graph, nodes.data(), &nn));
       const void* f1 = spmm_fwd_func((int)c->d.H);
-      const void* f0 = touched_func();
+      const void* f0 = touched_func((int)c->d.b_max);
       for (cudaGraphNode_t nd : nodes) {
         cudaGraphNodeType t;
         if (cudaGraphNodeGetType(nd, &t) != cudaSuccess || t != cudaGraphNodeTypeKernel) continue;

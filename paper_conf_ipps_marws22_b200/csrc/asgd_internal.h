@@ -22,7 +22,8 @@ constexpr int kScanTile = 1024;
 // M_K0PAR: parity of K-0's double-buffered tile sums.
 // M_MSYNC: fused merge arrival counter (64-bit, slots 40-41), M_MDONE: its CTA counter.
 enum { M_NNZ = 0, M_NLAB = 1, M_U = 2, M_ERR = 3, M_NROWS = 4, M_TILE = 5, M_LR = 6, M_K0PAR = 7, M_COUNT = 8,
-       M_LOSS = 10, M_BAR = 32, M_MSYNC = 40, M_MDONE = 42, M_CEN = 44, M_G2BAR = 46 /* 46-48 */ };
+       M_LOSS = 10, M_BAR = 32, M_MSYNC = 40, M_MDONE = 42, M_CEN = 44, M_G2BAR = 46 /* 46-48 */,
+       M_KBAR = 50 /* 50-51: K-3's packed grid barrier */ };
 // error bits in meta[M_ERR]
 enum { ERR_NNZ_CAP = 1, ERR_LAB_CAP = 2, ERR_ROW_ID = 4 };
 
@@ -38,6 +39,7 @@ struct WsLayout {
   bool x3;                      // fp32 path: GEMM operands split hi + lo (R14)
   size_t total;
   int64_t nz_cap, nl_cap, u_cap, n_tiles_f, n_pieces, splitk, n_rowblk, n_red, part_stride, stats_ld;
+  int64_t dh_parts;             // dH1 partial slices (>= splitk; K-3 one-pass: up to one per label tile)
 };
 
 WsLayout ws_layout(const asgd_model_desc& d);
@@ -85,8 +87,10 @@ __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;"
 // return from griddepcontrol.wait (the predecessor's outputs are visible: on the
 // step's chain, the predecessor's end), [2] the latest CTA end (its last thread), in
 // %globaltimer ns.  Each translation unit holds its own copy of the buffer pointer.
+// TL_MARK(k): phase marks inside a kernel (slots [3 k], [3 k + 1] = the earliest and [3 k + 2]
+// the latest time a CTA's calling thread passed mark k; TL_PH0.. are the K-3 phases).
 enum { TL_TOUCHED = 0, TL_SPMM, TL_G1, TL_SOFTMAX, TL_G2, TL_DH, TL_B1, TL_G3, TL_SCATTER, TL_G1B, TL_MERGE,
-       TL_OTHER, TL_N };
+       TL_OTHER, TL_PH0, TL_PH1, TL_PH2, TL_PH3, TL_PH4, TL_PH5, TL_PH6, TL_PH7, TL_N };
 #ifdef ASGD_TIMELINE
 static __device__ unsigned long long* g_tl;
 __device__ __forceinline__ unsigned long long tl_now() {
@@ -110,7 +114,17 @@ struct Tl {
 };
 #define ASGD_TL_SETTER(fn) \
   cudaError_t fn(unsigned long long* p) { return cudaMemcpyToSymbol(g_tl, &p, sizeof(p)); }
+#define TL_MARK(k)                                  \
+  do {                                              \
+    if (g_tl) {                                     \
+      const unsigned long long t_ = tl_now();       \
+      atomicMin(&g_tl[3 * (k)], t_);                \
+      atomicMin(&g_tl[3 * (k) + 1], t_);            \
+      atomicMax(&g_tl[3 * (k) + 2], t_);            \
+    }                                               \
+  } while (0)
 #else
+#define TL_MARK(k) do { } while (0)
 struct Tl {
   __device__ explicit Tl(int) {}
   __device__ void ready() {}
@@ -196,10 +210,12 @@ cudaError_t launch_touched(const Launch&, const StepArgs&, const asgd_csr&, int6
                            const WsLayout&, int b_max);
 // ---------------------------------------------------------------- K-1
 // Builds the batch view (K-0 (a)) and publishes it, meta and the row ids for the step.
+// fold: K-0's phase A inside K-1 (k0_fold(); the step's K-0 then starts at phase C)
 cudaError_t launch_spmm_fwd(const Launch&, const StepArgs&, const asgd_csr&, const float* W1, const float* b1,
-                            int H, const Ptrs&, const WsLayout&, bool want_bf16);
+                            int H, const Ptrs&, const WsLayout&, bool want_bf16, bool fold = false, int b_max = 0);
+bool k0_fold();
 const void* spmm_fwd_func(int H);
-const void* touched_func();
+const void* touched_func(int b_max);
 int spmm_fwd_nargs();   // parameter counts (all K-1 instantiations share the signature)
 int touched_nargs();
 // ---------------------------------------------------------------- K-5
@@ -250,9 +266,16 @@ cudaError_t launch_gemm_tc(const Launch&, int which, int n_rows, int64_t L, int 
 // K-3 (dH1 half): G1b + G2 + the dH1 reduce in one persistent kernel for the fused
 // softmax-CE regime (bf16, H = 256): Z tiles recomputed from the resident H1 block, dZ
 // formed on chip and fed straight into dH1 += dZ W2; write_dz also TMA-stores dZ for G3.
+// one_pass: no G1 / k_lse before it -- a first sweep of S tiles gives the softmax
+// statistics (partials in stats), a grid barrier, then lse, the row losses and the dZ /
+// dH1 sweep (S recomputed).
 cudaError_t launch_bwd_dh(const Launch&, int n, int64_t L, int H, const Ptrs&, const WsLayout&, float* b2,
                           const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab, const DhFuse& fz,
-                          bool write_dz);
+                          bool write_dz, bool one_pass = false, float2* stats = nullptr, bool dz_only = false);
+// dz_only: one label tile per CTA (LR = label tiles), no MMA 2 / reduce: the kernel replaces
+// G1 + softmax-CE (dZ to P.dzb, row losses), G2 and the dH reduce run after it.
+// the one-pass mode's partials fit the workspace (LR x MT CTAs of K-3 for n rows)
+bool bwd_dh_one_pass_fits(int n, int64_t L, const WsLayout&, int sms);
 // K-3 (dW2 half): G1b + G3 in one persistent kernel: per W2 row tile, Z^T recomputed per row
 // chunk, dZ^T on chip into dW2, then W2 / b2 SGD and the next bf16 shadow (Pw.w2b).
 cudaError_t launch_bwd_dw(const Launch&, int n, int64_t L, int H, const Ptrs& Pr, const Ptrs& Pw, float* W2,

@@ -277,14 +277,20 @@ __device__ __forceinline__ void grid_barrier(unsigned long long* ctr) {
   __syncthreads();
 }
 
-__global__ void __launch_bounds__(512) k_touched(StepArgs sa, const int64_t* __restrict__ row_ptr,
+// FOLD (k0_fold()): phase A ran inside K-1 (counts, row bitmaps and tile sums as K-1 reads
+// the entries); this kernel starts at phase C from the batch view K-1 published (gboff,
+// grbase) and runs after K-1 on the side stream.
+template <int NT, bool FOLD>   // threads per CTA: 128, 256 or 512 (the batch view needs 8 NT >= n)
+__global__ void __launch_bounds__(NT) k_touched(StepArgs sa, const int64_t* __restrict__ row_ptr,
                                                  int64_t n_data_rows, int64_t nz_cap,
                                                  const int32_t* __restrict__ col,
                                                  const float* __restrict__ val, int32_t* meta,
                                                  int32_t* cnt, int32_t* tsum, int64_t F, int ntiles,
                                                  int32_t* fseg, int32_t* fuid, int32_t* uniq,
                                                  int32_t* useg, uint32_t* bits, int W, int32_t* e_n,
-                                                 float* e_v, int32_t* e_u, int32_t* e_f) {
+                                                 float* e_v, int32_t* e_u, int32_t* e_f,
+                                                 const int32_t* __restrict__ gboff,
+                                                 const int64_t* __restrict__ grbase) {
   Tl tl_(TL_TOUCHED);
   pdl_trigger();
   pdl_wait();
@@ -298,26 +304,38 @@ __global__ void __launch_bounds__(512) k_touched(StepArgs sa, const int64_t* __r
   int32_t* ts_next = tsum + (size_t)(par ^ 1) * 2 * ntiles;
   const int n = sa.n;
   int32_t* hist = sboff + ((view_smem(n) + 3) / 4);       // [ntiles][2] after the batch view
-  for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x) hist[i] = 0;
-  const int nnz = build_view(sa, row_ptr, nullptr, n_data_rows, nz_cap, 0, sboff, false, ViewOut{});
   const int gt = blockIdx.x * blockDim.x + threadIdx.x, gs = gridDim.x * blockDim.x;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  // ---- A
-  for (int e = gt; e < nnz; e += gs) {
-    int r;
-    const int f = col[entry_index(sboff, n, e, &r)];
-    const int old = atomicAdd(&cnt[f], 1);
-    atomicOr(&bits[(int64_t)f * W + (r >> 5)], 1u << (r & 31));
-    const int t = f / kScanTile;
-    atomicAdd(&hist[2 * t], 1);
-    if (old == 0) atomicAdd(&hist[2 * t + 1], 1);
+  int nnz;
+  if constexpr (FOLD) {
+    // the view K-1 published: entry offsets and row bases
+    int64_t* srb = const_cast<int64_t*>(view_rbase(sboff, n));
+    for (int r = threadIdx.x; r <= n; r += blockDim.x) {
+      sboff[r] = gboff[r];
+      if (r < n) srb[r] = grbase[r];
+    }
+    __syncthreads();
+    nnz = sboff[n];
+  } else {
+    for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x) hist[i] = 0;
+    nnz = build_view(sa, row_ptr, nullptr, n_data_rows, nz_cap, 0, sboff, false, ViewOut{});
+    // ---- A
+    for (int e = gt; e < nnz; e += gs) {
+      int r;
+      const int f = col[entry_index(sboff, n, e, &r)];
+      const int old = atomicAdd(&cnt[f], 1);
+      atomicOr(&bits[(int64_t)f * W + (r >> 5)], 1u << (r & 31));
+      const int t = f / kScanTile;
+      atomicAdd(&hist[2 * t], 1);
+      if (old == 0) atomicAdd(&hist[2 * t + 1], 1);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x)
+      if (hist[i]) atomicAdd(&ts[i], hist[i]);
+    grid_barrier(bar);
   }
-  __syncthreads();
-  for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x)
-    if (hist[i]) atomicAdd(&ts[i], hist[i]);
-  grid_barrier(bar);
   // ---- C: prefix of the earlier tiles + in-tile scan
-  constexpr int PER = kScanTile / 512;
+  constexpr int PER = kScanTile / NT;
   for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
     int a = 0, b = 0;
     for (int j = threadIdx.x; j < t; j += blockDim.x) { a += ts[2 * j]; b += ts[2 * j + 1]; }
@@ -372,19 +390,41 @@ __global__ void __launch_bounds__(512) k_touched(StepArgs sa, const int64_t* __r
     __syncthreads();
   }
   grid_barrier(bar);
-  // ---- E: placement
-  for (int e = gt; e < nnz; e += gs) {
-    int r;
-    const int64_t k = entry_index(sboff, n, e, &r);
-    const int f = col[k];
-    const uint32_t* bw = bits + (int64_t)f * W;
-    int rank = __popc(bw[r >> 5] & ((1u << (r & 31)) - 1u));
-    for (int w = 0; w < (r >> 5); ++w) rank += __popc(bw[w]);
-    const int pos = fseg[f] + rank;
-    e_n[pos] = r;
-    e_v[pos] = val[k];
-    e_u[pos] = fuid[f];
-    e_f[pos] = f;
+  // ---- E: placement, kE entries per thread at a time (their dependent loads overlap)
+  constexpr int kE = 4;
+  for (int e0 = gt; e0 < nnz; e0 += kE * gs) {
+    int r[kE], f[kE], seg[kE], uid[kE], rank[kE];
+    int64_t k[kE];
+    float v[kE];
+#pragma unroll
+    for (int i = 0; i < kE; ++i) {
+      const int e = e0 + i * gs;
+      k[i] = e < nnz ? entry_index(sboff, n, e, &r[i]) : -1;
+      f[i] = k[i] >= 0 ? col[k[i]] : 0;
+      v[i] = k[i] >= 0 ? val[k[i]] : 0.f;
+    }
+#pragma unroll
+    for (int i = 0; i < kE; ++i) {
+      rank[i] = 0;
+      seg[i] = 0;
+      uid[i] = 0;
+      if (k[i] >= 0) {
+        const uint32_t* bw = bits + (int64_t)f[i] * W;
+        rank[i] = __popc(bw[r[i] >> 5] & ((1u << (r[i] & 31)) - 1u));
+        for (int w = 0; w < (r[i] >> 5); ++w) rank[i] += __popc(bw[w]);
+        seg[i] = fseg[f[i]];
+        uid[i] = fuid[f[i]];
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < kE; ++i) {
+      if (k[i] < 0) continue;
+      const int pos = seg[i] + rank[i];
+      e_n[pos] = r[i];
+      e_v[pos] = v[i];
+      e_u[pos] = uid[i];
+      e_f[pos] = f[i];
+    }
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) meta[M_K0PAR] = par ^ 1;   // every CTA read par before barrier 1
 }
@@ -402,10 +442,10 @@ template <int VPL>   // pieces per group = warps per K-1 CTA (H = 512: 8, the pa
 constexpr int k1_group() { return VPL >= 16 ? 8 : ASGD_K1_GROUP; }
 // TMA-staged K-1 (k1_tma()): every W1 row of a warp's piece is requested at once as one
 // bulk async copy per entry into the warp's 32-row shared-memory slot array, completed on
-// the warp's mbarrier; the FMAs then read shared memory.  fp32 rows of H floats: 6 warps
-// x 32 KB at H = 256 (one CTA per SM), 8 warps below.
+// the warp's mbarrier; the FMAs then read shared memory.  fp32 rows of H floats: 5 warps
+// x 32 KB at H = 256 (one CTA per SM; with the static view and partials ~207 KB), 8 warps below.
 template <int VPL>
-constexpr int k1_group_tma() { return VPL >= 8 ? 6 : 8; }
+constexpr int k1_group_tma() { return VPL >= 8 ? 5 : 8; }
 template <int VPL, bool TMA>
 constexpr int k1_warps() { return TMA ? k1_group_tma<VPL>() : k1_group<VPL>(); }
 template <int VPL, bool TMA>
@@ -415,6 +455,9 @@ constexpr int k1_min_ctas() { return TMA ? (VPL >= 8 ? 1 : 2) : 16 / k1_group<VP
 constexpr size_t k1_view_bytes() { return (view_smem(2048) + 127) & ~size_t(127); }
 template <int VPL, bool TMA>
 constexpr size_t k1_smem() { return k1_view_bytes() + (TMA ? (size_t)k1_warps<VPL, TMA>() * kPiece * VPL * 128 : 0); }
+// the folded K-0 phase A's tile histograms: after the view (and the TMA row slots)
+template <int VPL, bool TMA>
+__host__ __device__ constexpr size_t k1_hist_off(int n) { return TMA ? k1_smem<VPL, TMA>() : (view_smem(n) + 15) & ~size_t(15); }
 template <int VPL, bool TMA>
 // (256, 2): two CTAs per SM, all kU gathers of a group in flight (<= 128 regs)
 __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, TMA>())) k_spmm_fwd(StepArgs sa, const int64_t* __restrict__ row_ptr,
@@ -424,7 +467,9 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
                                                   const float* __restrict__ val,
                                                   const float* __restrict__ W1,
                                                   const float* __restrict__ b1, float* H1,
-                                                  bf16* H1b, bf16* H1l, float* part, int32_t* rowcnt) {
+                                                  bf16* H1b, bf16* H1l, float* part, int32_t* rowcnt,
+                                                  int32_t* kcnt, uint32_t* kbits, int W, int32_t* tsum,
+                                                  int ntiles) {
   Tl tl_(TL_SPMM);
   pdl_trigger();
   pdl_wait();
@@ -439,6 +484,11 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
   const int lane = threadIdx.x & 31;
   const int npieces = (nnz + kPiece - 1) / kPiece;
   const int nwarps = gridDim.x * (blockDim.x >> 5);
+  // K-0 phase A folded in (ntiles > 0, k0_fold()): per entry cnt[f] += 1 and the row
+  // bitmap bit, per CTA (count, first touch) histograms of the feature tiles in shared
+  // memory after the view / row slots, flushed to this step's tile sums at the end
+  int32_t* hist = reinterpret_cast<int32_t*>(reinterpret_cast<uint8_t*>(sboff) + k1_hist_off<VPL, TMA>(n));
+  for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x) hist[i] = 0;
 
   // Pieces are taken in groups of 8 consecutive pieces, one per warp of the CTA, so a
   // row that crosses pieces is first combined inside the CTA through shared memory;
@@ -534,6 +584,11 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
         mycol = __ldg(col + k);
         myval = __ldg(val + k);
       }
+      int k0old = 1;   // folded phase A: issued before the gathers, the counts read after them
+      if (ntiles && lane < cnt) {
+        k0old = atomicAdd(&kcnt[mycol], 1);
+        atomicOr(&kbits[(int64_t)mycol * W + (myr >> 5)], 1u << (myr & 31));
+      }
       int rcur = __shfl_sync(kFull, myr, 0);
       rfirst = rcur;
       rlast = __shfl_sync(kFull, myr, cnt - 1);
@@ -608,6 +663,13 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
         }
       }
       flush(rcur, acc);
+      if (ntiles) {   // tile histograms, aggregated per warp over equal tiles
+        const int t = lane < cnt ? mycol / kScanTile : -1;
+        const unsigned same = __match_any_sync(kFull, t);
+        const unsigned first = __match_any_sync(kFull, t * 2 + (k0old == 0));
+        if (t >= 0 && lane == __ffs(same) - 1) atomicAdd(&hist[2 * t], __popc(same));
+        if (t >= 0 && k0old == 0 && lane == __ffs(first) - 1) atomicAdd(&hist[2 * t + 1], __popc(first));
+      }
     }
     __syncthreads();
     // group combine: warp w takes the rows whose first segment inside the group is in
@@ -635,6 +697,12 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
       }
     }
     if (g + (int)gridDim.x < ngroups) __syncthreads();   // spart is reused by this CTA's next group
+  }
+  if (ntiles) {   // this CTA's tile histograms -> the step's tile sums (K-0 parity buffer)
+    __syncthreads();
+    int32_t* ts = tsum + (size_t)(vo.meta[M_K0PAR] & 1) * 2 * ntiles;
+    for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x)
+      if (hist[i]) atomicAdd(&ts[i], hist[i]);
   }
   // rows without entries: H1 = ReLU(b1)
   const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
@@ -1236,20 +1304,28 @@ int wave_grid(const Launch& lc, K kernel, size_t smem, int64_t pieces, int& occ,
   return (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)lc.sms * occ));
 }
 
+// K-1 grid cap (ASGD_K1_CTAS, A/B): the CTAs that stay resident beside K-0's
+int k1_cap() {
+  static const int v = [] { const char* e = getenv("ASGD_K1_CTAS"); return e ? atoi(e) : 0; }();
+  return v;
+}
+
 template <int VPL, bool TMA>
 cudaError_t spmm_fwd_t(const Launch& lc, const StepArgs& sa, const asgd_csr& x, const float* W1, const float* b1,
-                       const Ptrs& P, const WsLayout& L, bool want_bf16) {
-  const size_t smem = TMA ? k1_smem<VPL, TMA>() : view_smem(sa.n);
+                       const Ptrs& P, const WsLayout& L, bool want_bf16, bool fold, int b_max) {
+  const int ntiles = fold ? (int)L.n_tiles_f : 0;
+  const size_t smem = k1_hist_off<VPL, TMA>(sa.n) + (size_t)ntiles * 8;
   // the batch view (dynamic) + the group partials (static) exceed 48 KB at b_max = 2048
-  cudaError_t e = ensure_smem(k_spmm_fwd<VPL, TMA>, TMA ? k1_smem<VPL, TMA>() : view_smem(2048));
+  cudaError_t e = ensure_smem(k_spmm_fwd<VPL, TMA>, k1_hist_off<VPL, TMA>(2048) + (size_t)L.n_tiles_f * 8);
   if (e != cudaSuccess) return e;
   static int occ = 0;
-  const int grid = wave_grid(lc, k_spmm_fwd<VPL, TMA>, TMA ? k1_smem<VPL, TMA>() : view_smem(2048), L.n_pieces, occ,
-                             k1_warps<VPL, TMA>());
+  int grid = wave_grid(lc, k_spmm_fwd<VPL, TMA>, TMA ? k1_smem<VPL, TMA>() : view_smem(2048), L.n_pieces, occ,
+                       k1_warps<VPL, TMA>());
+  if (k1_cap() > 0) grid = std::min(grid, k1_cap());
   const ViewOut vo{P.boff, P.loff, P.rbase, P.rowsc, P.meta};
   launch_k(lc, k_spmm_fwd<VPL, TMA>, dim3(grid), dim3(32 * k1_warps<VPL, TMA>()), smem, sa, x.row_ptr, x.lab_ptr,
            x.n_rows, L.nz_cap, L.nl_cap, vo, x.col, x.val, W1, b1, P.h1, want_bf16 ? P.h1b : nullptr,
-           want_bf16 ? P.h1l : nullptr, P.part1, P.rowcnt);
+           want_bf16 ? P.h1l : nullptr, P.part1, P.rowcnt, P.cnt, P.bits, (b_max + 31) / 32, P.tsum, ntiles);
   return cudaGetLastError();
 }
 
@@ -1266,6 +1342,38 @@ cudaError_t scatter_t(const Launch& lc, float* W1, const Ptrs& P, const WsLayout
 
 }  // namespace
 
+// K-0 threads per CTA (ASGD_K0_THREADS = 128 / 256 / 512): fewer threads leave more of
+// each SM's register file to the kernels beside it (K-1 or the dense chain); at least
+// b_max / 8 (the batch view: 8 rows per thread)
+int touched_threads(int b_max) {
+  static const int v = [] { const char* e = getenv("ASGD_K0_THREADS"); return e ? atoi(e) : 512; }();
+  int t = v == 128 || v == 256 ? v : 512;
+  while (8 * t < b_max && t < 512) t *= 2;
+  return t;
+}
+
+template <int NT, bool FOLD>
+cudaError_t touched_t(const Launch& lc, const StepArgs& sa, const asgd_csr& x, int64_t F, const Ptrs& P,
+                      const WsLayout& L, int W, int ctas, size_t smem_all) {
+  if (smem_all > 48 * 1024) {
+    cudaError_t e = ensure_smem(k_touched<NT, FOLD>, smem_all);
+    if (e != cudaSuccess) return e;
+  }
+  // K-0's two software grid barriers need every CTA resident at once: at most one CTA per
+  // SM, and the kernel alone must fit ctas CTAs (asserted here instead of a cooperative
+  // launch, which graphs with programmatic dependent launch do not capture; the kernels
+  // beside it on other streams never wait for K-0, so its CTAs always get their SMs)
+  int occ = 0;
+  {
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_touched<NT, FOLD>, NT, smem_all);
+    if (e != cudaSuccess) return e;
+  }
+  if ((int64_t)occ * lc.sms < ctas) return cudaErrorCooperativeLaunchTooLarge;
+  return launch_k(lc, k_touched<NT, FOLD>, dim3(ctas), dim3(NT), smem_all, sa, x.row_ptr, x.n_rows, L.nz_cap, x.col,
+                  x.val, P.meta, P.cnt, P.tsum, F, (int)L.n_tiles_f, P.fseg, P.fuid, P.uniq, P.useg, P.bits, W, P.e_n,
+                  P.e_v, P.e_u, P.e_f, P.boff, P.rbase);
+}
+
 cudaError_t launch_touched(const Launch& lc, const StepArgs& sa, const asgd_csr& x, int64_t F, const Ptrs& P,
                            const WsLayout& L, int b_max) {
   const int n = sa.n;
@@ -1276,42 +1384,44 @@ cudaError_t launch_touched(const Launch& lc, const StepArgs& sa, const asgd_csr&
   static const int max_ctas = [] { const char* e = getenv("ASGD_K0_CTAS"); return e ? atoi(e) : 0; }();
   int64_t cap = max_ctas > 0 ? max_ctas : kTouchCtas;
   const int ctas = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)lc.sms, cap, (L.nz_cap + 1023) / 1024}));
-  if (smem_all > 48 * 1024) {
-    cudaError_t e = ensure_smem(k_touched, smem_all);
-    if (e != cudaSuccess) return e;
+  const bool fd = k0_fold();
+  switch (touched_threads(b_max)) {
+    case 128: return fd ? touched_t<128, true>(lc, sa, x, F, P, L, W, ctas, smem_all)
+                        : touched_t<128, false>(lc, sa, x, F, P, L, W, ctas, smem_all);
+    case 256: return fd ? touched_t<256, true>(lc, sa, x, F, P, L, W, ctas, smem_all)
+                        : touched_t<256, false>(lc, sa, x, F, P, L, W, ctas, smem_all);
+    default: return fd ? touched_t<512, true>(lc, sa, x, F, P, L, W, ctas, smem_all)
+                       : touched_t<512, false>(lc, sa, x, F, P, L, W, ctas, smem_all);
   }
-  // K-0's two software grid barriers need every CTA resident at once: at most one CTA per
-  // SM, and the kernel alone must fit ctas CTAs (asserted here instead of a cooperative
-  // launch, which graphs with programmatic dependent launch do not capture; the kernels
-  // beside it on other streams never wait for K-0, so its CTAs always get their SMs)
-  int occ = 0;
-  {
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_touched, 512, smem_all);
-    if (e != cudaSuccess) return e;
-  }
-  if ((int64_t)occ * lc.sms < ctas) return cudaErrorCooperativeLaunchTooLarge;
-  return launch_k(lc, k_touched, dim3(ctas), dim3(512), smem_all, sa, x.row_ptr, x.n_rows, L.nz_cap, x.col, x.val,
-                  P.meta, P.cnt, P.tsum, F, nt, P.fseg, P.fuid, P.uniq, P.useg, P.bits, W, P.e_n,
-                  P.e_v, P.e_u, P.e_f);
 }
 
-// K-1 with TMA-staged W1 rows (H <= 256): ASGD_K1_TMA=0 keeps the register-gather kernel
+// K-1 with TMA-staged W1 rows (H <= 256, ASGD_K1_TMA=1; measured slower at EURLex: 31 vs 21 us live)
 bool k1_tma() {
-  static const bool v = [] { const char* e = getenv("ASGD_K1_TMA"); return !(e && e[0] == '0'); }();
+  static const bool v = [] { const char* e = getenv("ASGD_K1_TMA"); return e && e[0] == '1'; }();
+  return v;
+}
+
+// K-0's phase A inside K-1 (default; ASGD_K0_FOLD=0 keeps the separate K-0 beside K-1): K-1
+// counts the batch's features as it reads the entries, and K-0 (phases C, E) runs after it
+// on the side stream.  Measured at EURLex (live kernel timeline): K-1 beside the full K-0
+// 21.4 us, alone 10.8, with the folded counts 15.1; step 66.8 -> 61.3 us back to back.
+bool k0_fold() {
+  static const bool v = [] { const char* e = getenv("ASGD_K0_FOLD"); return !(e && e[0] == '0'); }();
   return v;
 }
 
 cudaError_t launch_spmm_fwd(const Launch& lc, const StepArgs& sa, const asgd_csr& x, const float* W1,
-                            const float* b1, int H, const Ptrs& P, const WsLayout& L, bool want_bf16) {
+                            const float* b1, int H, const Ptrs& P, const WsLayout& L, bool want_bf16, bool fold,
+                            int b_max) {
   const bool t = k1_tma();
   switch (H) {
-    case 64: return t ? spmm_fwd_t<2, true>(lc, sa, x, W1, b1, P, L, want_bf16)
-                      : spmm_fwd_t<2, false>(lc, sa, x, W1, b1, P, L, want_bf16);
-    case 128: return t ? spmm_fwd_t<4, true>(lc, sa, x, W1, b1, P, L, want_bf16)
-                       : spmm_fwd_t<4, false>(lc, sa, x, W1, b1, P, L, want_bf16);
-    case 256: return t ? spmm_fwd_t<8, true>(lc, sa, x, W1, b1, P, L, want_bf16)
-                       : spmm_fwd_t<8, false>(lc, sa, x, W1, b1, P, L, want_bf16);
-    case 512: return spmm_fwd_t<16, false>(lc, sa, x, W1, b1, P, L, want_bf16);
+    case 64: return t ? spmm_fwd_t<2, true>(lc, sa, x, W1, b1, P, L, want_bf16, fold, b_max)
+                      : spmm_fwd_t<2, false>(lc, sa, x, W1, b1, P, L, want_bf16, fold, b_max);
+    case 128: return t ? spmm_fwd_t<4, true>(lc, sa, x, W1, b1, P, L, want_bf16, fold, b_max)
+                       : spmm_fwd_t<4, false>(lc, sa, x, W1, b1, P, L, want_bf16, fold, b_max);
+    case 256: return t ? spmm_fwd_t<8, true>(lc, sa, x, W1, b1, P, L, want_bf16, fold, b_max)
+                       : spmm_fwd_t<8, false>(lc, sa, x, W1, b1, P, L, want_bf16, fold, b_max);
+    case 512: return spmm_fwd_t<16, false>(lc, sa, x, W1, b1, P, L, want_bf16, fold, b_max);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -1326,12 +1436,19 @@ const void* spmm_fwd_func(int H) {
   }
 }
 
-const void* touched_func() { return reinterpret_cast<const void*>(k_touched); }
+const void* touched_func(int b_max) {
+  const bool fd = k0_fold();
+  switch (touched_threads(b_max)) {
+    case 128: return fd ? reinterpret_cast<const void*>(k_touched<128, true>) : reinterpret_cast<const void*>(k_touched<128, false>);
+    case 256: return fd ? reinterpret_cast<const void*>(k_touched<256, true>) : reinterpret_cast<const void*>(k_touched<256, false>);
+    default: return fd ? reinterpret_cast<const void*>(k_touched<512, true>) : reinterpret_cast<const void*>(k_touched<512, false>);
+  }
+}
 
 template <typename... A>
 constexpr int nargs_of(void (*)(A...)) { return (int)sizeof...(A); }
 int spmm_fwd_nargs() { return nargs_of(k_spmm_fwd<8, false>); }
-int touched_nargs() { return nargs_of(k_touched); }
+int touched_nargs() { return nargs_of(k_touched<512, false>); }
 
 // K-5 layout: ASGD_K5_SEG=1 -> one warp per feature segment (k_scatter_seg), else nnz pieces
 bool k5_seg() {

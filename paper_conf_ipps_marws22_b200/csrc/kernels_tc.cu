@@ -54,6 +54,14 @@ struct TcArgs {
   int dh_fuse;
   const float* h1; float* da1; bf16* da1b; const float* dh_off;
   float* b1; float* grad_b1; float* colpart; const float* rowloss; int32_t* bar;
+  // K-3 one-pass (k_bwd_dh): the softmax statistics come from a first sweep of S tiles
+  // (recomputed in the second): per (label range, row) partials (max2, sum
+  // 2^(t - max2)) in stats[lr][row], then the label-logit sums as floats [lr][row];
+  // after a grid barrier lse -> g.lse, row loss -> rowloss_w
+  int one_pass; float* rowloss_w;
+  // K-3 softmax-only (dz_only, implies one_pass): no MMA 2 / dH1 partials / reduce tail --
+  // the kernel stands for G1 + softmax-CE (dZ TMA-stored, row losses), G2 follows it
+  int dz_only; unsigned long long* gbar;   // packed grid barrier (generation << 32 | count)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -246,6 +254,38 @@ constexpr uint32_t pow2ceil(uint32_t x) {
 //   colpart[row block][c] = sum_{r in block} dA1[r][c]   (fixed order)
 // and the last CTA to finish sums colpart over the row blocks in order: b1 -= lr db1,
 // grad_b1 = db1, and the mean loss from the per-row losses (deterministic).
+// Software grid barrier over every CTA of the launch (all resident: one per SM), one
+// thread per CTA; bar[0] = arrivals, bar[1] = generation (reusable).
+__device__ __forceinline__ void grid_sync_thread(int32_t* bar, int G) {
+  volatile int32_t* cnt = bar;
+  volatile int32_t* gen = bar + 1;
+  const int32_t g0 = *gen;
+  __threadfence();
+  if (atomicAdd(bar, 1) == G - 1) {
+    *cnt = 0;
+    __threadfence();
+    atomicAdd(bar + 1, 1);
+  } else {
+    while (*gen == g0) __nanosleep(64);
+  }
+  __threadfence();
+}
+
+// The same with one 64-bit word, generation << 32 | count: the last arriver resets the count
+// and bumps the generation in one atomic (one round trip fewer than the two-word version).
+__device__ __forceinline__ void grid_sync_packed(unsigned long long* bar, int G) {
+  __threadfence();
+  const unsigned long long old = atomicAdd(bar, 1ull);
+  const unsigned int g0 = (unsigned int)(old >> 32);
+  if ((unsigned int)(old & 0xffffffffull) == (unsigned int)(G - 1)) {
+    atomicAdd(bar, (1ull << 32) - (unsigned long long)G);
+  } else {
+    volatile unsigned long long* vb = bar;
+    while ((unsigned int)(*vb >> 32) == g0) __nanosleep(32);
+  }
+  __threadfence();
+}
+
 __device__ void dh_reduce_phase(const TcArgs& g, float* sred) {
   const int G = gridDim.x, k = blockIdx.x, H = g.N, n = g.M, S = g.splits;
   __shared__ int s_last;
@@ -253,21 +293,9 @@ __device__ void dh_reduce_phase(const TcArgs& g, float* sred) {
   // groups before the kernel's final barrier): make them visible, then the grid barrier
   asm volatile("fence.proxy.async.global;" ::: "memory");
   __syncthreads();
-  if (threadIdx.x == 0) {
-    volatile int32_t* cnt = g.bar;
-    volatile int32_t* gen = g.bar + 1;
-    const int32_t g0 = *gen;
-    __threadfence();
-    if (atomicAdd(g.bar, 1) == G - 1) {
-      *cnt = 0;
-      __threadfence();
-      atomicAdd(g.bar + 1, 1);
-    } else {
-      while (*gen == g0) __nanosleep(64);
-    }
-    __threadfence();
-  }
+  if (threadIdx.x == 0) grid_sync_thread(g.bar, G);
   __syncthreads();
+  if (threadIdx.x == 0) TL_MARK(TL_PH7);
   // (2) this CTA's block
   int GC = H / 32;
   if (GC > G) GC = G;
@@ -974,8 +1002,8 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
   uint8_t* sH1 = smem;
   uint8_t* sW2 = sH1 + kBwdH1Bytes;
   uint8_t* sDZ = sW2 + kBwdStages * kBwdW2Bytes;
-  float* sBias = reinterpret_cast<float*>(sDZ + 2 * kBwdDzBytes);          // [kBwdEpi][32]
-  uint64_t* w2full = reinterpret_cast<uint64_t*>(sBias + kBwdEpi * 32);
+  float* sBias = reinterpret_cast<float*>(sDZ + 2 * kBwdDzBytes);          // [kBwdEpi][32], then [128][3]
+  uint64_t* w2full = reinterpret_cast<uint64_t*>(sBias + kBwdEpi * 32 + 128 * 3);
   uint64_t* w2empty = w2full + kBwdStages;
   uint64_t* sfull = w2empty + kBwdStages;
   uint64_t* sempty = sfull + 2;
@@ -985,7 +1013,7 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
   uint64_t* dhfull = hfull + 1;
   uint32_t* tbase = reinterpret_cast<uint32_t*>(dhfull + 1);
 
-  Tl tl_(TL_G2);
+  Tl tl_(g.dz_only ? TL_G1 : TL_G2);
   pdl_trigger();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int MT = (g.M + BM - 1) / BM, T = (g.N + kBwdBN - 1) / kBwdBN;
@@ -1020,9 +1048,13 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
     if (lane == 0 && nt > 0) {   // ------------------------------------ TMA producer
       mbar_expect_tx(hfull, kBwdH1Bytes);
       for (int kb = 0; kb < 4; ++kb) tma_load_2d(sH1 + kb * 16384, &tmH1, hfull, kb * 64, m0);
-      for (int i = 0; i < nt; ++i) {
-        const int st = i % kBwdStages;
-        mbar_wait(&w2empty[st], ((i / kBwdStages) & 1) ^ 1);
+      // one-pass: the range's W2 tiles twice (statistics sweep, then the dZ / dH1 sweep),
+      // once when the S tiles stay in TMEM (keep: nt <= 2)
+      const bool keep = g.one_pass && nt <= 2;
+      const int nu = (g.one_pass && !keep) ? 2 * nt : nt;
+      for (int u = 0; u < nu; ++u) {
+        const int st = u % kBwdStages, i = u % nt;
+        mbar_wait(&w2empty[st], ((u / kBwdStages) & 1) ^ 1);
         mbar_expect_tx(&w2full[st], kBwdW2Bytes);
         for (int kb = 0; kb < 4; ++kb)
           tma_load_2d(sW2 + st * kBwdW2Bytes + kb * 8192, &tmW2, &w2full[st], kb * 64, (t0 + i) * kBwdBN);
@@ -1033,11 +1065,31 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       constexpr uint32_t idesc1 = make_idesc(kBwdBN, false, false);   // S = H1 W2_j^T
       constexpr uint32_t idesc2 = make_idesc(256, false, true);       // dH1 += dZ W2_j
       mbar_wait(hfull, 0);
+      // one-pass statistics sweep: S tiles only (use u = i of the S buffers / W2 stages);
+      // keep (nt <= 2): they stay in their TMEM buffers and W2 stages for the second sweep
+      const bool keep = g.one_pass && nt <= 2;
+      const int base = (g.one_pass && !keep) ? nt : 0;
+      for (int u = 0; u < (g.one_pass ? nt : 0); ++u) {
+        const int st = u % kBwdStages, acc = u & 1;
+        mbar_wait(&w2full[st], (u / kBwdStages) & 1);
+        mbar_wait(&sempty[acc], ((u >> 1) & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t d = tmem + (uint32_t)(acc * kBwdBN);
+        const uint32_t wb = smem_u32(sW2 + st * kBwdW2Bytes);
+#pragma unroll
+        for (int kb = 0; kb < 4; ++kb)
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            mma_bf16(d, desc_sw128(smem_u32(sH1 + kb * 16384) + k * 32, 16, 1024),
+                     desc_sw128(wb + kb * 8192 + k * 32, 16, 1024), idesc1, (kb | k) ? 1u : 0u);
+        mma_commit(&sfull[acc]);
+        if (!keep) mma_commit(&w2empty[st]);
+      }
       for (int i = 0; i <= nt; ++i) {
-        if (i < nt) {
-          const int st = i % kBwdStages, acc = i & 1;
-          mbar_wait(&w2full[st], (i / kBwdStages) & 1);
-          mbar_wait(&sempty[acc], ((i >> 1) & 1) ^ 1);
+        if (i < nt && !keep) {
+          const int u = base + i, st = u % kBwdStages, acc = u & 1;
+          mbar_wait(&w2full[st], (u / kBwdStages) & 1);
+          mbar_wait(&sempty[acc], ((u >> 1) & 1) ^ 1);
           tc_fence_after();
           const uint32_t d = tmem + (uint32_t)(acc * kBwdBN);
           const uint32_t wb = smem_u32(sW2 + st * kBwdW2Bytes);
@@ -1050,15 +1102,17 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
           mma_commit(&sfull[acc]);
         }
         if (i > 0) {
-          const int j = i - 1, st = j % kBwdStages, buf = j & 1;
+          const int j = i - 1, st = (base + j) % kBwdStages, buf = j & 1;
           mbar_wait(&dzfull[buf], (j >> 1) & 1);
           tc_fence_after();
           const uint32_t wb = smem_u32(sW2 + st * kBwdW2Bytes);
           const uint32_t zb = smem_u32(sDZ + buf * kBwdDzBytes);
+          if (!g.dz_only) {
 #pragma unroll
-          for (int k = 0; k < kBwdBN / 16; ++k)
-            mma_bf16(tmem + 256, desc_sw128(zb + k * 32, 16, 1024), desc_sw128(wb + k * 2048, 8192, 1024), idesc2,
-                     (j > 0 || k > 0) ? 1u : 0u);
+            for (int k = 0; k < kBwdBN / 16; ++k)
+              mma_bf16(tmem + 256, desc_sw128(zb + k * 32, 16, 1024), desc_sw128(wb + k * 2048, 8192, 1024), idesc2,
+                       (j > 0 || k > 0) ? 1u : 0u);
+          }
           mma_commit(&dzempty[buf]);
           mma_commit(&w2empty[st]);
         }
@@ -1072,14 +1126,134 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
     float crow = 0.f, tinv = 0.f;
     int64_t lab_cur = 0, lab_end = 0;
     if (m < g.M) {
-      crow = -g.lse[m] * kL2E - __log2f(1.f / g.invB);
+      if (!g.one_pass) crow = -g.lse[m] * kL2E - __log2f(1.f / g.invB);
       const int64_t id = g.rows[m];
       lab_cur = g.lab_ptr[id];
       lab_end = g.lab_ptr[id + 1];
       tinv = g.invB / (float)(lab_end - lab_cur);
     }
     int nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
+    if (warp == 4 && lane == 0) TL_MARK(TL_PH0);
+    if (g.one_pass) {
+      // (A) this CTA's softmax partials of row m over its label range, from a first sweep
+      // of S tiles (the MMA warp's statistics sweep), in base 2: t = (S + b2) log2 e
+      float mx = -INFINITY, se = 0.f, zs = 0.f;
+      int64_t lc = lab_cur;
+      int ny = nxt;
+      for (int i = 0; i < nt; ++i) {
+        const int c = (t0 + i) * kBwdBN + wh * 32, acc = i & 1;
+        mbar_wait(&sfull[acc], (i >> 1) & 1);
+        tc_fence_after();
+        float v[32];
+        tmem_ld32(tmem + (uint32_t)(acc * kBwdBN + wh * 32) + ((uint32_t)(q * 32) << 16), v);
+        if (nt > 2) {   // recomputed in the second sweep: release the buffer
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&sempty[acc]);
+        }
+        float tm = -INFINITY;
+#pragma unroll
+        for (int jj = 0; jj < 32; ++jj) {
+          const bool ok = c + jj < g.N;
+          v[jj] = ok ? v[jj] + __ldg(g.bias + c + jj) : -INFINITY;   // Z (natural units)
+          tm = fmaxf(tm, v[jj]);
+        }
+        while (ny < c) {
+          ++lc;
+          ny = lc < lab_end ? g.lab[lc] : 0x7fffffff;
+        }
+        while (ny < c + 32) {   // the row's labels among these columns: sum of Z_y
+          const int jy = ny - c;
+#pragma unroll
+          for (int jj = 0; jj < 32; ++jj)
+            if (jj == jy) zs += v[jj];
+          ++lc;
+          ny = lc < lab_end ? g.lab[lc] : 0x7fffffff;
+        }
+        const float tm2 = tm * kL2E;
+        float ts = 0.f;
+#pragma unroll
+        for (int jj = 0; jj < 32; ++jj) ts += ex2_approx(fmaf(v[jj], kL2E, -tm2));
+        if (tm2 > mx) { se = (mx == -INFINITY ? 0.f : se * ex2_approx(mx - tm2)) + ts; mx = tm2; }
+        else if (tm2 != -INFINITY) se += ts * ex2_approx(tm2 - mx);
+      }
+      if (warp == 4 && lane == 0) TL_MARK(TL_PH1);
+      // the two column halves (wh) of a row: wh = 1 hands its partial to wh = 0 via smem
+      float* xch = sBias + kBwdEpi * 32;   // [128][3] after the bias rows
+      const int rl = q * 32 + lane;
+      if (wh == 1) { xch[3 * rl] = mx; xch[3 * rl + 1] = se; xch[3 * rl + 2] = zs; }
+      asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
+      if (wh == 0 && m < g.M) {
+        const float om = xch[3 * rl], os = xch[3 * rl + 1];
+        const float nm = fmaxf(mx, om);
+        se = (mx == -INFINITY ? 0.f : se * ex2_approx(mx - nm)) + (om == -INFINITY ? 0.f : os * ex2_approx(om - nm));
+        mx = nm;
+        zs += xch[3 * rl + 2];
+        // [range][row] layout: the reads in (C) are coalesced over a warp's 32 rows
+        g.stats[(int64_t)lr * g.stats_ld + m] = make_float2(mx, se);
+        reinterpret_cast<float*>(g.stats + (int64_t)g.stats_ld * LR)[(int64_t)lr * g.stats_ld + m] = zs;
+      }
+      // (B) grid barrier over the CTAs (all resident); the producer / MMA warps go on
+      asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
+      if (warp == 4 && lane == 0) grid_sync_packed(g.gbar, (int)gridDim.x);
+      if (warp == 4 && lane == 0) TL_MARK(TL_PH2);
+      asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
+      // (C) lse of row m from the LR partials: the row's two warps (wh) each combine half of
+      // the ranges, 16 loads in flight, then exchange through smem; range 0 writes the row loss
+      float M2 = -INFINITY, S2 = 0.f, Zs = 0.f;
+      const int hh = (LR + 1) / 2, ra = wh ? hh : 0, rb = wh ? LR : hh;
+      if (m < g.M) {
+        const float2* pp = g.stats + m;
+        for (int r0 = ra; r0 < rb; r0 += 16) {
+          float2 pm[16];
+#pragma unroll
+          for (int u = 0; u < 16; ++u)
+            pm[u] = r0 + u < rb ? __ldcg(pp + (int64_t)(r0 + u) * g.stats_ld) : make_float2(-INFINITY, 0.f);
+#pragma unroll
+          for (int u = 0; u < 16; ++u) {
+            if (pm[u].x == -INFINITY) continue;
+            if (pm[u].x > M2) { S2 = (M2 == -INFINITY ? 0.f : S2 * ex2_approx(M2 - pm[u].x)) + pm[u].y; M2 = pm[u].x; }
+            else S2 += pm[u].y * ex2_approx(pm[u].x - M2);
+          }
+        }
+        if (warp == 4 && lane == 0) TL_MARK(TL_PH5);
+        if (lr == 0) {   // the row's label-logit sum (range order), for the row loss
+          const float* zp = reinterpret_cast<const float*>(g.stats + (int64_t)g.stats_ld * LR) + m;
+          for (int r0 = ra; r0 < rb; r0 += 16) {
+            float z[16];
+#pragma unroll
+            for (int u = 0; u < 16; ++u) z[u] = r0 + u < rb ? __ldcg(zp + (int64_t)(r0 + u) * g.stats_ld) : 0.f;
+#pragma unroll
+            for (int u = 0; u < 16; ++u) Zs += z[u];
+          }
+        }
+      }
+      if (warp == 4 && lane == 0) TL_MARK(TL_PH6);
+      if (wh == 1) { xch[3 * rl] = M2; xch[3 * rl + 1] = S2; xch[3 * rl + 2] = Zs; }
+      asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
+      if (wh == 0) {
+        const float om = xch[3 * rl], os = xch[3 * rl + 1];
+        const float nm = fmaxf(M2, om);
+        S2 = (M2 == -INFINITY ? 0.f : S2 * ex2_approx(M2 - nm)) + (om == -INFINITY ? 0.f : os * ex2_approx(om - nm));
+        M2 = nm;
+        Zs += xch[3 * rl + 2];
+      }
+      asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
+      if (wh == 0) { xch[3 * rl] = M2; xch[3 * rl + 1] = S2; }
+      asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
+      if (wh == 1) { M2 = xch[3 * rl]; S2 = xch[3 * rl + 1]; }
+      if (m < g.M) {
+        const float lse2 = M2 + __log2f(S2);   // lse log2 e
+        crow = -lse2 - __log2f(1.f / g.invB);
+        if (lr == 0 && wh == 0) {
+          const float lse = lse2 * 0.6931471805599453f;
+          g.rowloss_w[m] = lse - Zs / (float)(lab_end - lab_cur);
+          const_cast<float*>(g.lse)[m] = lse;
+        }
+      }
+    }
     float* bias_w = sBias + (warp - 4) * 32;
+    if (warp == 4 && lane == 0 && g.one_pass) TL_MARK(TL_PH3);
     // b2 of the next tile's columns, loaded one tile ahead (its latency hides under this
     // tile's epilogue instead of heading it: the top stall site in ncu before)
     auto b2_of = [&](int i) {
@@ -1087,8 +1261,9 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       return (i < nt && cc < g.N) ? __ldg(g.bias + cc) * kL2E : 0.f;
     };
     float bnext = b2_of(0);
+    const int base = (g.one_pass && nt > 2) ? nt : 0;   // S-buffer uses of the statistics sweep
     for (int i = 0; i < nt; ++i) {
-      const int acc = i & 1, buf = i & 1;
+      const int acc = (base + i) & 1, buf = i & 1;
       const int c = (t0 + i) * kBwdBN + wh * 32;        // this warp's first label column
       __syncwarp();
       bias_w[lane] = bnext;
@@ -1098,7 +1273,7 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
         ++lab_cur;
         nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
       }
-      mbar_wait(&sfull[acc], (i >> 1) & 1);
+      mbar_wait(&sfull[acc], ((base + i) >> 1) & 1);
       tc_fence_after();
       float v[32];
       tmem_ld32(tmem + (uint32_t)(acc * kBwdBN + wh * 32) + ((uint32_t)(q * 32) << 16), v);
@@ -1160,14 +1335,16 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       __syncwarp();
       if (lane == 0) mbar_arrive(&dzfull[buf]);
     }
+    if (warp == 4 && lane == 0) TL_MARK(TL_PH4);
     // this CTA's dH1 partial (rows m, columns wh * 128 .. + 127) -> dhpart[lr]
     float* dst = g.out + (int64_t)lr * g.part_stride + (int64_t)m * g.ldo + wh * 128;
-    if (nt > 0) {
+    if (nt > 0 && !g.dz_only) {
       mbar_wait(dhfull, 0);
+      if (warp == 4 && lane == 0) TL_MARK(TL_PH5);
       tc_fence_after();
     }
 #pragma unroll 1
-    for (int ch = 0; ch < 4; ++ch) {
+    for (int ch = 0; ch < (g.dz_only ? 0 : 4); ++ch) {
       float v[32];
       if (nt > 0) {
         tmem_ld32(tmem + 256 + (uint32_t)(wh * 128 + ch * 32) + ((uint32_t)(q * 32) << 16), v);
@@ -1191,8 +1368,10 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512) : "memory");
   }
   __threadfence();
+  if (g.dz_only) return;   // G2 and the dH1 reduce follow as kernels of their own
   TcArgs gt = g;    // the tail reduces H columns: N = H there
   gt.N = g.K;
+  if (threadIdx.x == 0) TL_MARK(TL_PH6);
   dh_reduce_phase(gt, reinterpret_cast<float*>(smem));
 }
 
@@ -1717,15 +1896,27 @@ cudaError_t launch_gemm_tc(const Launch& lc, int which, int n, int64_t L, int H,
   return run<64, true, true, TC_EPI_SGD>(lc, ta, tb, tc, td, g, 1);
 }
 
+bool bwd_dh_one_pass_fits(int n, int64_t L, const WsLayout& W, int sms) {
+  const int MT = (n + BM - 1) / BM;
+  const int64_t T = (L + kBwdBN - 1) / kBwdBN;
+  const int64_t LR = std::max<int64_t>(1, std::min<int64_t>({(int64_t)(sms / MT), T, (int64_t)W.dh_parts}));
+  return 2 * LR <= (L + 31) / 32 + 8;   // the partials fit the G1 stats area
+}
+
 cudaError_t launch_bwd_dh(const Launch& lc, int n, int64_t L, int H, const Ptrs& P, const WsLayout& W, float* b2,
                           const int32_t* rows, const int64_t* lab_ptr, const int32_t* lab, const DhFuse& fz,
-                          bool write_dz) {
+                          bool write_dz, bool one_pass, float2* stats, bool dz_only) {
   if (!tc_available()) return cudaErrorNotSupported;
   if (H != 256 || P.w2l) return cudaErrorNotSupported;   // bf16 path, H = 256 (one N = 256 MMA)
   const int64_t Lp = padded_ld(L);
   const int MT = (n + BM - 1) / BM;
   const int64_t T = (L + kBwdBN - 1) / kBwdBN;
-  const int LR = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)(lc.sms / MT), T, (int64_t)W.splitk}));
+  // label ranges: one per SM pair of row blocks, at most the dH1 partial slices the
+  // workspace holds (the one-pass regime has room for one range per tile)
+  if (dz_only) one_pass = write_dz = true;
+  const int LR = (int)std::max<int64_t>(
+      1, std::min<int64_t>({(int64_t)(lc.sms / MT), T,
+                            (int64_t)(dz_only ? T : one_pass ? W.dh_parts : W.splitk)}));
   CUtensorMap th, tw, tz;
   cudaError_t e;
   if ((e = make_map(&th, P.h1b, H, n, (uint64_t)H * 2, 64, BM)) != cudaSuccess) return e;
@@ -1740,7 +1931,17 @@ cudaError_t launch_bwd_dh(const Launch& lc, int n, int64_t L, int H, const Ptrs&
   g.h1 = P.h1; g.da1 = P.da1; g.da1b = fz.want_bf16 ? P.da1b : nullptr; g.dh_off = fz.dh_off;
   g.b1 = fz.b1; g.grad_b1 = fz.grad_b1; g.colpart = P.db1part; g.rowloss = P.rowloss;
   g.bar = P.meta + M_G2BAR;
-  const size_t smem = kBwdH1Bytes + kBwdStages * kBwdW2Bytes + 2 * kBwdDzBytes + kBwdEpi * 32 * 4 + 1024 + 256;
+  if (one_pass) {
+    // (max, sum) partials [LR][B] float2 + label-logit sums [LR][B] float: the G1 stats area
+    if (2 * LR > (L + 31) / 32 + 8) return cudaErrorNotSupported;
+    g.one_pass = 1;
+    g.stats = stats; g.stats_ld = W.stats_ld;
+    g.rowloss_w = P.rowloss;
+    g.gbar = reinterpret_cast<unsigned long long*>(P.meta + M_KBAR);
+    g.dz_only = dz_only ? 1 : 0;
+  }
+  const size_t smem = kBwdH1Bytes + kBwdStages * kBwdW2Bytes + 2 * kBwdDzBytes + kBwdEpi * 32 * 4 + 128 * 3 * 4 +
+                      1024 + 256;
   if ((e = ensure_smem(k_bwd_dh, smem)) != cudaSuccess) return e;
   return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_bwd_dh, dim3(MT * LR), dim3(128 + 32 * kBwdEpi), smem, th,
                       tw, tz, g, LR);

@@ -22,17 +22,22 @@ def normwise(a, b):
     return np.linalg.norm(a - b) / (nb if nb > 0 else 1.0)
 
 
-def _row_errors(a, b):
+def _row_errors(a, b, slack=None):
     """Per-row error ||a_r - b_r|| / max(||b_r||, rms row norm of b): relative to
     the row's own norm, with rows far below the typical norm measured against
-    the typical norm (a row wrong by 100 % of a typical row fails)."""
+    the typical norm (a row wrong by 100 % of a typical row fails).  With slack,
+    each element's difference is first reduced by its allowance, max(|a - b| -
+    slack, 0), as in the elementwise check (R16)."""
     a = np.asarray(a, dtype=np.float64)
     b = np.asarray(b, dtype=np.float64)
     if a.shape[0] == 0:
         return np.zeros(0)
     nb = np.linalg.norm(b, axis=1)
     floor = np.sqrt(np.mean(nb * nb))
-    return np.linalg.norm(a - b, axis=1) / np.maximum(nb, floor if floor > 0 else 1.0)
+    d = np.abs(a - b)
+    if slack is not None:
+        d = np.maximum(d - np.asarray(slack, dtype=np.float64).reshape(d.shape), 0.0)
+    return np.linalg.norm(d, axis=1) / np.maximum(nb, floor if floor > 0 else 1.0)
 
 
 def _elem_err(a, b, tol, per_row, slack=None):
@@ -83,10 +88,6 @@ def check_grads(gg, og, tol, F, H, touched, tag="", emul=None, slack=None):
     W1r = np.asarray(ref["W1"]).reshape(F, H)[touched]
     W2g = np.asarray(gg["W2"]).reshape(L, H)
     W2r = np.asarray(ref["W2"]).reshape(L, H)
-    rec["row_W1_max"] = float(_row_errors(W1g, W1r).max(initial=0.0))
-    rec["row_W2_max"] = float(_row_errors(W2g, W2r).max(initial=0.0))
-    if emul is not None:   # for the record: per-row distance of the bf16 path to the exact gradient
-        rec["row_W2_max_vs_oracle"] = float(_row_errors(W2g, np.asarray(og["W2"]).reshape(L, H)).max(initial=0.0))
     pairs = {"W1": (W1g, W1r), "b1": (gg["b1"], ref["b1"]), "W2": (W2g, W2r), "b2": (gg["b2"], ref["b2"])}
     sl = {}
     if slack is not None:
@@ -94,6 +95,15 @@ def check_grads(gg, og, tol, F, H, touched, tag="", emul=None, slack=None):
               "W2": np.asarray(slack["W2"]).reshape(L, H), "b2": slack["b2"]}
         rec["slack_rel"] = {k: float(np.linalg.norm(v) / (np.linalg.norm(np.asarray(pairs[k][1])) + 1e-300))
                             for k, v in sl.items()}
+    # per row, with the same componentwise allowance as the elementwise check (R16); the
+    # unreduced row error is logged beside it
+    rec["row_W1_max"] = float(_row_errors(W1g, W1r, sl.get("W1")).max(initial=0.0))
+    rec["row_W2_max"] = float(_row_errors(W2g, W2r, sl.get("W2")).max(initial=0.0))
+    if sl:
+        rec["row_W1_max_raw"] = float(_row_errors(W1g, W1r).max(initial=0.0))
+        rec["row_W2_max_raw"] = float(_row_errors(W2g, W2r).max(initial=0.0))
+    if emul is not None:   # for the record: per-row distance of the bf16 path to the exact gradient
+        rec["row_W2_max_vs_oracle"] = float(_row_errors(W2g, np.asarray(og["W2"]).reshape(L, H)).max(initial=0.0))
     for k, (a, b) in pairs.items():
         rec[f"elem_{k}"] = _elem_err(a, b, tol, per_row=True, slack=sl.get(k))
     # where the worst W1 / W2 elements sit (diagnostics for the log)

@@ -66,9 +66,9 @@ def main():
     rel = np.array(rel)
     med = np.nanmedian(rel, axis=0)
     print(f"{'kernel':10s} {'arrive':>8s} {'ready':>8s} {'end':>8s} {'ready->end':>10s}  (us, median of {a.steps})")
-    order = np.argsort(med[:, 1])
+    order = np.argsort(np.where(np.isnan(med[:, 1]), med[:, 2], med[:, 1]))
     for i in order:
-        if np.isnan(med[i, 0]):
+        if np.isnan(med[i, 0]) and np.isnan(med[i, 2]):
             continue
         name = api.TIMELINE_KERNELS[i]
         out[name] = dict(arrive=med[i, 0], ready=med[i, 1], end=med[i, 2], span=med[i, 2] - med[i, 1])
