@@ -316,6 +316,27 @@ __global__ void __launch_bounds__(NT) k_touched(StepArgs sa, const int64_t* __re
     }
     __syncthreads();
     nnz = sboff[n];
+    // ---- C0: this step's tile sums (count, touched features) from the counts K-1 left
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      int a = 0, b = 0;
+      for (int64_t f = (int64_t)t * kScanTile + threadIdx.x; f < min((int64_t)(t + 1) * kScanTile, F); f += blockDim.x) {
+        const int c = cnt[f];
+        a += c;
+        b += c > 0;
+      }
+#pragma unroll
+      for (int o = 16; o; o >>= 1) { a += __shfl_xor_sync(kFull, a, o); b += __shfl_xor_sync(kFull, b, o); }
+      if (lane == 0) { s_red[0][wid] = a; s_red[1][wid] = b; }
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        int x = 0, y = 0;
+        for (int w = 0; w < nw; ++w) { x += s_red[0][w]; y += s_red[1][w]; }
+        ts[2 * t] = x;
+        ts[2 * t + 1] = y;
+      }
+      __syncthreads();
+    }
+    grid_barrier(bar);
   } else {
     for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x) hist[i] = 0;
     nnz = build_view(sa, row_ptr, nullptr, n_data_rows, nz_cap, 0, sboff, false, ViewOut{});
@@ -455,9 +476,7 @@ constexpr int k1_min_ctas() { return TMA ? (VPL >= 8 ? 1 : 2) : 16 / k1_group<VP
 constexpr size_t k1_view_bytes() { return (view_smem(2048) + 127) & ~size_t(127); }
 template <int VPL, bool TMA>
 constexpr size_t k1_smem() { return k1_view_bytes() + (TMA ? (size_t)k1_warps<VPL, TMA>() * kPiece * VPL * 128 : 0); }
-// the folded K-0 phase A's tile histograms: after the view (and the TMA row slots)
-template <int VPL, bool TMA>
-__host__ __device__ constexpr size_t k1_hist_off(int n) { return TMA ? k1_smem<VPL, TMA>() : (view_smem(n) + 15) & ~size_t(15); }
+
 template <int VPL, bool TMA>
 // (256, 2): two CTAs per SM, all kU gathers of a group in flight (<= 128 regs)
 __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, TMA>())) k_spmm_fwd(StepArgs sa, const int64_t* __restrict__ row_ptr,
@@ -484,11 +503,8 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
   const int lane = threadIdx.x & 31;
   const int npieces = (nnz + kPiece - 1) / kPiece;
   const int nwarps = gridDim.x * (blockDim.x >> 5);
-  // K-0 phase A folded in (ntiles > 0, k0_fold()): per entry cnt[f] += 1 and the row
-  // bitmap bit, per CTA (count, first touch) histograms of the feature tiles in shared
-  // memory after the view / row slots, flushed to this step's tile sums at the end
-  int32_t* hist = reinterpret_cast<int32_t*>(reinterpret_cast<uint8_t*>(sboff) + k1_hist_off<VPL, TMA>(n));
-  for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x) hist[i] = 0;
+  // K-0 phase A folded in (ntiles > 0, k0_fold()): per entry cnt[f] += 1 and the row bitmap
+  // bit, as reductions; K-0 derives the tile sums from the counts
 
   // Pieces are taken in groups of 8 consecutive pieces, one per warp of the CTA, so a
   // row that crosses pieces is first combined inside the CTA through shared memory;
@@ -584,9 +600,8 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
         mycol = __ldg(col + k);
         myval = __ldg(val + k);
       }
-      int k0old = 1;   // folded phase A: issued before the gathers, the counts read after them
-      if (ntiles && lane < cnt) {
-        k0old = atomicAdd(&kcnt[mycol], 1);
+      if (ntiles && lane < cnt) {   // folded phase A: fire-and-forget reductions
+        atomicAdd(&kcnt[mycol], 1);
         atomicOr(&kbits[(int64_t)mycol * W + (myr >> 5)], 1u << (myr & 31));
       }
       int rcur = __shfl_sync(kFull, myr, 0);
@@ -663,13 +678,6 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
         }
       }
       flush(rcur, acc);
-      if (ntiles) {   // tile histograms, aggregated per warp over equal tiles
-        const int t = lane < cnt ? mycol / kScanTile : -1;
-        const unsigned same = __match_any_sync(kFull, t);
-        const unsigned first = __match_any_sync(kFull, t * 2 + (k0old == 0));
-        if (t >= 0 && lane == __ffs(same) - 1) atomicAdd(&hist[2 * t], __popc(same));
-        if (t >= 0 && k0old == 0 && lane == __ffs(first) - 1) atomicAdd(&hist[2 * t + 1], __popc(first));
-      }
     }
     __syncthreads();
     // group combine: warp w takes the rows whose first segment inside the group is in
@@ -697,12 +705,6 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
       }
     }
     if (g + (int)gridDim.x < ngroups) __syncthreads();   // spart is reused by this CTA's next group
-  }
-  if (ntiles) {   // this CTA's tile histograms -> the step's tile sums (K-0 parity buffer)
-    __syncthreads();
-    int32_t* ts = tsum + (size_t)(vo.meta[M_K0PAR] & 1) * 2 * ntiles;
-    for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x)
-      if (hist[i]) atomicAdd(&ts[i], hist[i]);
   }
   // rows without entries: H1 = ReLU(b1)
   const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
@@ -1314,9 +1316,9 @@ template <int VPL, bool TMA>
 cudaError_t spmm_fwd_t(const Launch& lc, const StepArgs& sa, const asgd_csr& x, const float* W1, const float* b1,
                        const Ptrs& P, const WsLayout& L, bool want_bf16, bool fold, int b_max) {
   const int ntiles = fold ? (int)L.n_tiles_f : 0;
-  const size_t smem = k1_hist_off<VPL, TMA>(sa.n) + (size_t)ntiles * 8;
+  const size_t smem = TMA ? k1_smem<VPL, TMA>() : view_smem(sa.n);
   // the batch view (dynamic) + the group partials (static) exceed 48 KB at b_max = 2048
-  cudaError_t e = ensure_smem(k_spmm_fwd<VPL, TMA>, k1_hist_off<VPL, TMA>(2048) + (size_t)L.n_tiles_f * 8);
+  cudaError_t e = ensure_smem(k_spmm_fwd<VPL, TMA>, TMA ? k1_smem<VPL, TMA>() : view_smem(2048));
   if (e != cudaSuccess) return e;
   static int occ = 0;
   int grid = wave_grid(lc, k_spmm_fwd<VPL, TMA>, TMA ? k1_smem<VPL, TMA>() : view_smem(2048), L.n_pieces, occ,
