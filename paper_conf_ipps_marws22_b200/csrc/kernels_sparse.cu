@@ -21,6 +21,18 @@ namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
 
+// Message-passing fence of the last-arriver combines (partial stores -> counter atomic,
+// counter observed -> partial loads): acquire-release at GPU scope is all the pattern needs
+// (ASGD_FENCE_SC=1 compiles the sequentially consistent __threadfence instead; ncu showed
+// the SC fences as K-5's top stall, 21 % membar).
+__device__ __forceinline__ void fence_mp() {
+#ifdef ASGD_FENCE_SC
+  __threadfence();
+#else
+  asm volatile("fence.acq_rel.gpu;" ::: "memory");
+#endif
+}
+
 __device__ __forceinline__ int entry_row(const int32_t* sboff, int n, int e) {
   // largest r in [0, n) with sboff[r] <= e (rows may be empty)
   int lo = 0, hi = n;          // invariant: answer in [lo, hi)
@@ -546,12 +558,12 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
     const int rs = sboff[r], re = sboff[r + 1];
     const int g0 = rs / GE, g1 = (re - 1) / GE;
     IO::store_cg(part + (int64_t)(g == g0 ? 2 * g + 1 : 2 * g) * H, lane, acc);
-    __threadfence();
+    fence_mp();
     int old = 0;
     if (lane == 0) old = atomicAdd(&rowcnt[r], 1);
     old = __shfl_sync(kFull, old, 0);
     if (old != g1 - g0) return;
-    __threadfence();
+    fence_mp();
 #pragma unroll
     for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
     for (int q = g0; q <= g1; q += 4) {   // 4 partials in flight, summed in group order
@@ -792,13 +804,13 @@ __global__ void __launch_bounds__(256) k_scatter_sgd(const int32_t* __restrict__
       if (!finish) {
         const int slot = before ? 2 * p : 2 * p + 1;
         IO::store_cg(part + (int64_t)slot * H, lane, acc);
-        __threadfence();
+        fence_mp();
         int old = 0;
         if (lane == 0) old = atomicAdd(&ucnt[u], 1);
         old = __shfl_sync(kFull, old, 0);
         const int q0 = ss / kPiece, q1 = (se_ - 1) / kPiece;
         if (old == q1 - q0) {
-          __threadfence();
+          fence_mp();
 #pragma unroll
           for (int i = 0; i < VPL; ++i) acc[i] = 0.f;
           for (int q = q0; q <= q1; ++q) {
@@ -1036,13 +1048,13 @@ __global__ void __launch_bounds__(scatter_threads<T, CPL>(), 1) k_scatter_sgd_s(
       if (!finish) {
         const int slot = before ? 2 * p : 2 * p + 1;
         st_cols<CPL>(part + (int64_t)slot * H + c0 + lane * CPL, acc, true);
-        __threadfence();
+        fence_mp();
         int old = 0;
         if (lane == 0) old = atomicAdd(&ucnt[(int64_t)u * nsl + slice], 1);
         old = __shfl_sync(kFull, old, 0);
         const int q0 = useg[u] / kPiece, q1 = (useg[u + 1] - 1) / kPiece;
         if (old == q1 - q0) {
-          __threadfence();
+          fence_mp();
           ld_cols<CPL>(wrow, w, false);
 #pragma unroll
           for (int i = 0; i < CPL; ++i) acc[i] = 0.f;
