@@ -581,7 +581,12 @@ int enqueue_step(asgd_ctx* c, int n) {
   if (!k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   // K-1
   PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, c->sa, x, W1, b1, H, P, c->L, true, k0_fold(), (int)m.b_max));   // H1 fp32 + bf16 (+ lo)
-  if (k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
+  // ASGD_K0_AFTER=1 (with the fold): K-0 forks after the loss stage (G1 + softmax, or K-3's
+  // softmax-only kernel), beside G2 / the dH reduce instead of beside G1.  Measured: EURLex
+  // 58.5 -> 57.2 us per step, but AmazonCat 181.9 -> 204.9 and Wiki10 179.2 -> 193.6 (K-0
+  // then ends after the dH reduce and holds up K-5), so it is off by default
+  static const bool k0_after = [] { const char* e = getenv("ASGD_K0_AFTER"); return e && e[0] == '1'; }() && k0_fold();
+  if (k0_late && !k0_after) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   {
     // A DAG over three streams (both precisions; the fp32 path's GEMMs take bf16x3
     // hi + lo operands, R14, and always store Z):
@@ -662,6 +667,7 @@ int enqueue_step(asgd_ctx* c, int n) {
                                                        nullptr, nullptr, P.rowsc, x.lab_ptr, x.lab);
             })());
     }
+    if (k0_after) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
     const bool centred = m.loss == ASGD_LOSS_SIGMOID;   // G1 stored dZ - 1/(2B) (R11)
     auto g3 = [&](const Launch& l) {
       if (k3dw)   // K-3's dW2 half: Z^T recomputed, dZ^T on chip, W2 / b2 SGD

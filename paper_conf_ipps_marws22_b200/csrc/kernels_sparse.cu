@@ -275,6 +275,8 @@ __device__ int build_view(const StepArgs& sa, const int64_t* __restrict__ row_pt
 // 64 CTAs: enough entries in flight, while leaving the register file of most
 // SMs to K-1, which runs beside K-0 (measured: 148 CTAs slow K-1 by ~3 us).
 constexpr int kTouchCtas = 64;
+constexpr int kK0OneCta = 0;   // folded K-0: feature tiles up to which CTA 0 alone scans (measured slower
+                               // at EURLex's 5 tiles: 63.5 vs 58.5 us per step; kept at 0)
 
 __device__ __forceinline__ void grid_barrier(unsigned long long* ctr) {
   __syncthreads();
@@ -328,8 +330,11 @@ __global__ void __launch_bounds__(NT) k_touched(StepArgs sa, const int64_t* __re
     }
     __syncthreads();
     nnz = sboff[n];
-    // ---- C0: this step's tile sums (count, touched features) from the counts K-1 left
-    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    // ---- C0: this step's tile sums (count, touched features) from the counts K-1 left.
+    // Few tiles (F <= kK0OneCta tiles, EURLex-4K: 5): CTA 0 runs C0 and C alone, the other
+    // CTAs go straight to the barrier before E (one grid barrier instead of two)
+    const bool one = ntiles <= kK0OneCta;
+    for (int t = one ? (blockIdx.x == 0 ? 0 : ntiles) : blockIdx.x; t < ntiles; t += one ? 1 : gridDim.x) {
       int a = 0, b = 0;
       for (int64_t f = (int64_t)t * kScanTile + threadIdx.x; f < min((int64_t)(t + 1) * kScanTile, F); f += blockDim.x) {
         const int c = cnt[f];
@@ -348,7 +353,7 @@ __global__ void __launch_bounds__(NT) k_touched(StepArgs sa, const int64_t* __re
       }
       __syncthreads();
     }
-    grid_barrier(bar);
+    if (!one) grid_barrier(bar);
   } else {
     for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x) hist[i] = 0;
     nnz = build_view(sa, row_ptr, nullptr, n_data_rows, nz_cap, 0, sboff, false, ViewOut{});
@@ -369,7 +374,8 @@ __global__ void __launch_bounds__(NT) k_touched(StepArgs sa, const int64_t* __re
   }
   // ---- C: prefix of the earlier tiles + in-tile scan
   constexpr int PER = kScanTile / NT;
-  for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+  const bool one_cta = FOLD && ntiles <= kK0OneCta;   // CTA 0 scans every tile (after its own C0)
+  for (int t = one_cta ? (blockIdx.x == 0 ? 0 : ntiles) : blockIdx.x; t < ntiles; t += one_cta ? 1 : gridDim.x) {
     int a = 0, b = 0;
     for (int j = threadIdx.x; j < t; j += blockDim.x) { a += ts[2 * j]; b += ts[2 * j + 1]; }
 #pragma unroll
