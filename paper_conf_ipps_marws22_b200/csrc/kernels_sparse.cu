@@ -997,7 +997,6 @@ __global__ void __launch_bounds__(scatter_threads<T, CPL>(), 1) k_scatter_sgd_s(
     const int fprev = __shfl_sync(kFull, nb, 0), fnext = __shfl_sync(kFull, nb, 1);
     const int fup = __shfl_up_sync(kFull, myf, 1);
     uint32_t smask = __ballot_sync(kFull, lane < cnt && (lane == 0 || myf != fup));
-    wait_staged();
     while (smask) {
       // kSegAhead segments at a time: their W1 row slices are all requested before the
       // first one is summed (1 = one segment at a time; A/B switch ASGD_SEG_AHEAD)
@@ -1031,6 +1030,7 @@ __global__ void __launch_bounds__(scatter_threads<T, CPL>(), 1) k_scatter_sgd_s(
       float acc[CPL];
 #pragma unroll
       for (int i = 0; i < CPL; ++i) acc[i] = 0.f;
+      wait_staged();   // after the first W1 row slice was requested: its load overlaps the staging
       int j = j0;
       for (; j + kU <= j1; j += kU) {
         float g[kU][CPL];

@@ -51,6 +51,30 @@ def test_device_entry_points_fail_cleanly_without_gpu():
     assert rc == _lib.E_UNSUPPORTED
 
 
+def test_timeline_probes_compiled_out_by_default():
+    """asgd_timeline_set: the kernel-timeline probes exist only in a -DASGD_TIMELINE build
+    (tools/timeline.py); the default library reports ASGD_E_UNSUPPORTED without touching
+    the device, for a buffer and for NULL alike."""
+    lib = _lib.lib()
+    buf = (C.c_uint64 * 60)()
+    assert lib.asgd_timeline_set(C.addressof(buf)) == _lib.E_UNSUPPORTED
+    assert lib.asgd_timeline_set(None) == _lib.E_UNSUPPORTED
+    assert b"ASGD_TIMELINE" in lib.asgd_last_error()
+
+
+def test_workspace_holds_one_dh_partial_per_label_tile_in_the_stored_z_regime():
+    """The K-3 one-pass / softmax-only modes keep up to one dH1 partial per label tile
+    (<= 64) in the stored-Z regime (bf16 softmax, H = 256): the workspace of that regime
+    grows by those slices, the fp32 path and the fused-CE regime do not."""
+    lib = _lib.lib()
+    bf = _lib.ModelDesc(5000, 3993, 256, _lib.PREC_BF16, 256, 80000, 3000, _lib.LOSS_SOFTMAX, 0)
+    f32 = _lib.ModelDesc(5000, 3993, 256, _lib.PREC_FP32, 256, 80000, 3000, _lib.LOSS_SOFTMAX, 0)
+    wb, wf = lib.asgd_workspace_bytes(C.byref(bf)), lib.asgd_workspace_bytes(C.byref(f32))
+    assert wb > 0 and wf > 0
+    # 63 label tiles x 256 rows x 256 x 4 B of partials at least (G2's split-K is 15 slices)
+    assert wb >= 63 * 256 * 256 * 4
+
+
 def _load(name):
     with open(os.path.join(GOLDEN, name)) as f:
         return json.load(f)

@@ -1,5 +1,8 @@
-bash tools/gpu.sh h19 build
-timeout 900 python -m pytest tests/test_gpu_step.py tests/test_gpu_large.py tests/test_gpu_dist.py -k "tiny or eurlex or wiki10 or amazoncat" -m gpu -q -p no:cacheprovider -x > gpurun_out/h19_pytest.log 2>&1; echo "pytest $?"; tail -2 gpurun_out/h19_pytest.log
-ab() { tag=$1; shift; env "$@" timeout 300 python tools/ab_step.py --tag $tag "${EXTRA[@]}" 2>/dev/null | tee -a gpurun_out/h19_ab.jsonl | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(d['tag'], d['config'], round(d['us_per_step'],2), round(d['min'],2), round(d['max'],2))"; }
-EXTRA=(); ab after1cta X=1; ab after1cta_t256 ASGD_K0_THREADS=256; ab early ASGD_K0_AFTER=0
-for c in amazoncat13k wiki10_31k; do EXTRA=(--config $c); ab after X=1; ab early ASGD_K0_AFTER=0; done
+python -m paper_conf_ipps_marws22_b200.build --force > /dev/null 2>&1
+b() { tag=$1; shift; env "$@" timeout 600 python bench.py --no-cpu-baseline --ttp-megabatches 0 --e2e-steps 0 > gpurun_out/h20_$tag.json 2>/dev/null; python -c "import json; d=json.load(open('gpurun_out/h20_$tag.json')); print('$tag', d['value'], d['ms_per_step'])"; }
+b fold1 X=1
+b nofold ASGD_K0_FOLD=0
+b fold2 X=1
+b nofold2 ASGD_K0_FOLD=0
+timeout 300 python tools/ab_step.py --tag fold_k5w 2>/dev/null | cut -c1-100
+ASGD_K0_FOLD=0 timeout 300 python tools/ab_step.py --tag nofold_k5w 2>/dev/null | cut -c1-100
