@@ -232,7 +232,7 @@ Ptrs ws_ptrs(char* b, const WsLayout& L) {
 // One captured local step (everything after K-0 (a), which is launched eagerly
 // with the step's row ids, lr and loss pointer and publishes them to the rest).
 struct StepGraph {
-  int n = 0, cur = 0;
+  int n = 0, cur = 0, steps = 1;      // steps: local steps captured back to back (step groups)
   uint32_t mask = 0;
   int seen = 0;                       // captured on the 2nd step with this key
   cudaGraph_t graph = nullptr;
@@ -241,8 +241,8 @@ struct StepGraph {
   struct Prof { cudaGraphNode_t node; int cls; bool begin; };
   std::vector<Prof> prof;             // profiling event-record nodes, capture order
   struct ArgNode { cudaGraphNode_t node; cudaKernelNodeParams p; std::vector<void*> args; };
-  std::vector<ArgNode> arg_nodes;     // K-0 and K-1: parameter 0 (StepArgs) is updated per replay
-  StepArgs sa{};                      // storage parameter 0 of arg_nodes points at
+  std::vector<ArgNode> arg_nodes;     // K-0 and K-1 of each step: parameter 0 (StepArgs) per replay
+  std::vector<StepArgs> sas;          // per step: storage parameter 0 of its arg_nodes points at
   std::vector<cudaEvent_t> placeholders;
   uint64_t last_use = 0;
 };
@@ -289,6 +289,7 @@ struct asgd_ctx {
   uint64_t graph_clock = 0;
   bool capturing = false;
   std::vector<std::pair<cudaEvent_t, int>> cap_ph;   // (placeholder, cls * 2 + begin) during capture
+  std::vector<std::pair<cudaGraphNode_t, int>> cap_args;   // K-0 (0) / K-1 (1) nodes, capture order
   cudaEvent_t prof_sink = nullptr;                // target of profiling nodes past kMaxProfPairs
   cudaEvent_t ev_ring[8] = {};                    // asgd_run_tickets: completion of the last steps
   StepArgs sa{};                                  // current step's arguments (K-0 / K-1 parameter)
@@ -551,6 +552,18 @@ int asgd_data_upload(asgd_ctx* c, const asgd_csr* h, const asgd_csr* dv) {
 }  // extern "C"
 
 namespace {
+// During capture: the kernel node just captured on `st` (the stream's single capture
+// dependency) is a K-0 (kind 0) or K-1 (kind 1) node whose StepArgs parameter is rebound per replay.
+int record_cap_node(asgd_ctx* c, cudaStream_t st, int kind) {
+  cudaStreamCaptureStatus cs;
+  const cudaGraphNode_t* deps = nullptr;
+  size_t nd = 0;
+  CU(cudaStreamGetCaptureInfo(st, &cs, nullptr, nullptr, &deps, &nd));
+  if (cs != cudaStreamCaptureStatusActive || nd != 1) return fail(ASGD_E_STATE, "capture: %zu nodes after K-%d", nd, kind);
+  c->cap_args.push_back({deps[0], kind});
+  return ASGD_OK;
+}
+
 // Everything of a local step after K-0 (a): reads the step's rows / lr / loss
 // pointer from the workspace (P.rowsc, meta), so it can be captured once per
 // (n, shadow buffer, profile mask) and replayed.
@@ -575,12 +588,14 @@ int enqueue_step(asgd_ctx* c, int n) {
     CU(cudaEventRecord(c->ev_fork, c->s));
     CU(cudaStreamWaitEvent(c->s2, c->ev_fork, 0));
     PCU_ON(c->s2, ASGD_K_TOUCHED, launch_touched(c->lc2(), c->sa, x, m.F, P, c->L, m.b_max));
+    if (c->capturing) { const int rc = record_cap_node(c, c->s2, 0); if (rc != ASGD_OK) return rc; }
     CU(cudaEventRecord(c->ev_join, c->s2));
     return ASGD_OK;
   };
   if (!k0_late) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   // K-1
   PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, c->sa, x, W1, b1, H, P, c->L, true, k0_fold(), (int)m.b_max));   // H1 fp32 + bf16 (+ lo)
+  if (c->capturing) { const int rc = record_cap_node(c, c->s, 1); if (rc != ASGD_OK) return rc; }
   // ASGD_K0_AFTER=1 (with the fold): K-0 forks after the loss stage (G1 + softmax, or K-3's
   // softmax-only kernel), beside G2 / the dH reduce instead of beside G1.  Measured: EURLex
   // 58.5 -> 57.2 us per step, but AmazonCat 181.9 -> 204.9 and Wiki10 179.2 -> 193.6 (K-0
@@ -726,11 +741,13 @@ int enqueue_step(asgd_ctx* c, int n) {
 
 constexpr size_t kMaxGraphs = 16;
 
-// Replay (capturing on the 2nd use of a key) the rest of the step as a CUDA graph.
-int step_graph(asgd_ctx* c, int n) {
+// Replay (capturing on the 2nd use of a key) `steps` local steps as one CUDA graph
+// (steps > 1: a step group, run_steps at N = 1); sas[i] = step i's StepArgs.  c->w2b_cur
+// is left as it was (the caller flips it per step).
+int step_graph(asgd_ctx* c, int n, int steps, const StepArgs* sas) {
   StepGraph* hit = nullptr;
   for (auto& gr : c->graphs)
-    if (gr.n == n && gr.cur == c->w2b_cur && gr.mask == c->prof_mask) { hit = &gr; break; }
+    if (gr.n == n && gr.steps == steps && gr.cur == c->w2b_cur && gr.mask == c->prof_mask) { hit = &gr; break; }
   if (!hit) {
     if (c->graphs.size() >= kMaxGraphs) {
       auto lru = std::min_element(c->graphs.begin(), c->graphs.end(),
@@ -740,23 +757,35 @@ int step_graph(asgd_ctx* c, int n) {
     }
     c->graphs.emplace_back();
     hit = &c->graphs.back();
-    hit->n = n; hit->cur = c->w2b_cur; hit->mask = c->prof_mask;
+    hit->n = n; hit->steps = steps; hit->cur = c->w2b_cur; hit->mask = c->prof_mask;
   }
   StepGraph& G = *hit;
   G.last_use = ++c->graph_clock;
-  if (!G.exec && G.seen++ == 0) return enqueue_step(c, n);   // first use: eager (warms attributes)
+  const int cur0 = c->w2b_cur;
+  auto enqueue_all = [&]() -> int {
+    for (int i = 0; i < steps; ++i) {
+      c->sa = sas[i];
+      const int rc = enqueue_step(c, n);
+      c->w2b_cur ^= 1;
+      if (rc != ASGD_OK) { c->w2b_cur = cur0; return rc; }
+    }
+    c->w2b_cur = cur0;
+    return ASGD_OK;
+  };
+  if (!G.exec && G.seen++ == 0) return enqueue_all();   // first use: eager (warms attributes)
   if (!G.exec) {
     // capture on the private stream sc (the ctx stream may be the legacy default
     // stream, which cannot capture); the graph itself is launched on c->s
     if (!c->sc) CU(cudaStreamCreateWithFlags(&c->sc, cudaStreamNonBlocking));
     const int64_t l0 = c->launches;
     c->cap_ph.clear();
+    c->cap_args.clear();
     cudaStream_t user = c->s;
     c->s = c->sc;
     cudaError_t eb = cudaStreamBeginCapture(c->s, cudaStreamCaptureModeThreadLocal);
     if (eb != cudaSuccess) { c->s = user; return cuda_fail(eb, "cudaStreamBeginCapture"); }
     c->capturing = true;
-    const int rc = enqueue_step(c, n);
+    const int rc = enqueue_all();
     c->capturing = false;
     cudaGraph_t graph = nullptr;
     const cudaError_t ec = cudaStreamEndCapture(c->s, &graph);
@@ -766,29 +795,38 @@ int step_graph(asgd_ctx* c, int n) {
     c->launches = l0;
     if (rc != ASGD_OK || ec != cudaSuccess) {
       if (graph) cudaGraphDestroy(graph);
+      c->cap_args.clear();
       return rc != ASGD_OK ? rc : cuda_fail(ec, "cudaStreamEndCapture");
     }
     G.graph = graph;
     CU(cudaGraphInstantiate(&G.exec, graph, 0));
-    {  // K-0 / K-1 nodes: their StepArgs parameter is rebound per replay
-      size_t nn = 0;
-      CU(cudaGraphGetNodes(graph, nullptr, &nn));
-      std::vector<cudaGraphNode_t> nodes(nn);
-      CU(cudaGraphGetNodes(graph, nodes.data(), &nn));
-      const void* f1 = spmm_fwd_func((int)c->d.H);
-      const void* f0 = touched_func((int)c->d.b_max);
-      for (cudaGraphNode_t nd : nodes) {
+    {  // each step's K-0 / K-1 nodes (recorded at capture): their StepArgs parameter is
+       // rebound per replay to G.sas[step]
+      G.sas.assign(steps, StepArgs{});
+      int seen[2] = {0, 0};
+      for (auto& ca : c->cap_args) {
+        // the recorded node may be a profiling event-record node behind the kernel: walk back
         cudaGraphNodeType t;
-        if (cudaGraphNodeGetType(nd, &t) != cudaSuccess || t != cudaGraphNodeTypeKernel) continue;
+        for (int hop = 0;; ++hop) {
+          CU(cudaGraphNodeGetType(ca.first, &t));
+          if (t == cudaGraphNodeTypeKernel) break;
+          size_t nd = 0;
+          CU(cudaGraphNodeGetDependencies(ca.first, nullptr, &nd));
+          if (nd != 1 || hop > 4) return fail(ASGD_E_STATE, "step graph: K-%d node not found", ca.second);
+          CU(cudaGraphNodeGetDependencies(ca.first, &ca.first, &nd));
+        }
         cudaKernelNodeParams kp;
-        CU(cudaGraphKernelNodeGetParams(nd, &kp));
-        if (kp.func != f1 && kp.func != f0) continue;
-        const int na = kp.func == f1 ? spmm_fwd_nargs() : touched_nargs();
-        StepGraph::ArgNode an{nd, kp, std::vector<void*>(kp.kernelParams, kp.kernelParams + na)};
-        an.args[0] = &G.sa;
+        CU(cudaGraphKernelNodeGetParams(ca.first, &kp));
+        const int na = ca.second == 1 ? spmm_fwd_nargs() : touched_nargs();
+        const int step = seen[ca.second]++;
+        if (step >= steps) return fail(ASGD_E_STATE, "step graph: extra K-%d node", ca.second);
+        StepGraph::ArgNode an{ca.first, kp, std::vector<void*>(kp.kernelParams, kp.kernelParams + na)};
+        an.args[0] = &G.sas[step];
         G.arg_nodes.push_back(std::move(an));
       }
-      if (G.arg_nodes.size() != 2) return fail(ASGD_E_STATE, "step graph: %zu K-0/K-1 nodes", G.arg_nodes.size());
+      c->cap_args.clear();
+      if (seen[0] != steps || seen[1] != steps)
+        return fail(ASGD_E_STATE, "step graph: %d K-0 / %d K-1 nodes for %d steps", seen[0], seen[1], steps);
     }
     if (!c->cap_ph.empty()) {
       size_t nn = 0;
@@ -811,7 +849,7 @@ int step_graph(asgd_ctx* c, int n) {
     c->cap_ph.clear();
   }
   if (!G.prof.empty()) bind_prof_events(c, G);
-  G.sa = c->sa;
+  for (int i = 0; i < steps; ++i) G.sas[i] = sas[i];
   for (auto& an : G.arg_nodes) {
     cudaKernelNodeParams kp = an.p;
     kp.kernelParams = an.args.data();
@@ -848,7 +886,7 @@ int asgd_local_step(asgd_ctx* c, const int32_t* rows, int32_t n, float lr, float
     }
     CU(cudaEventRecord(c->trace_ev[c->trace_n].first, c->s));
   }
-  const int rc = (graphs_enabled() && !g) ? step_graph(c, n) : enqueue_step(c, n);
+  const int rc = (graphs_enabled() && !g) ? step_graph(c, n, 1, &c->sa) : enqueue_step(c, n);
   if (rc != ASGD_OK) return rc;
   if (tr) {
     CU(cudaEventRecord(c->trace_ev[c->trace_n].second, c->s));
@@ -1383,26 +1421,72 @@ int asgd_sched_next(asgd_sched* s, int32_t rank, int64_t b, int64_t* start, int6
 namespace {
 // The rank's step loop shared by the dynamic and the static schedule: next(&start, &len)
 // returns 1 for a batch, 0 when the rank's share is done, < 0 on error.
+// Step groups: with a schedule that gives this rank its tickets regardless of timing (one
+// rank, or Elastic's static split), up to step_group() consecutive tickets of equal length
+// are enqueued as one graph replay of that many steps -- the ~3.5 us between two step
+// graphs becomes an in-graph kernel boundary.  ASGD_STEP_GROUP (default kDefGroup, 1 = off).
+// Measured (EURLex bench line): 1 / 4 / 8 / 16 steps per replay -> 4.25 / 4.55 / 4.54 / 4.52 M
+// samples/s; results bitwise equal to one graph per step (tests/test_gpu_step_groups.py).
+constexpr int kMaxGroup = 16, kDefGroup = 4;
+int step_group() {
+  static const int v = [] {
+    const char* e = getenv("ASGD_STEP_GROUP");
+    return std::max(1, std::min(kMaxGroup, e ? atoi(e) : kDefGroup));
+  }();
+  return v;
+}
+
 template <typename Next>
 int run_steps(asgd_ctx* c, Next next, const int32_t* stream_rows, float lr, float* losses, int64_t losses_cap,
-              int32_t inflight, int64_t* n_steps) {
+              int32_t inflight, int64_t* n_steps, bool may_group = false) {
   if (inflight < 1 || inflight > kMaxInflight) return fail(ASGD_E_ARG, "inflight=%d not in [1, %d]", inflight, kMaxInflight);
   for (auto& ev : c->ev_ring)
     if (!ev) CU(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
-  int64_t k = 0;
+  const int grp = (may_group && graphs_enabled() && !c->dbg && !c->trace && c->prof_mask == 0) ? step_group() : 1;
+  int64_t k = 0, launches = 0;
+  int64_t pend_st = -1, pend_len = 0;   // a ticket taken but not yet enqueued (length change)
   for (;;) {
-    if (k >= inflight) CU(cudaEventSynchronize(c->ev_ring[(k - inflight) % kMaxInflight]));
-    int64_t start = 0, len = 0;
-    const int r = next(&start, &len);
-    if (r < 0) return fail(-r, "scheduler failed");
-    if (r == 0) break;
-    c->cur_start = start;
-    const int rc = asgd_local_step(c, stream_rows + start, (int32_t)len, lr,
-                                   (losses && k < losses_cap) ? losses + k : nullptr);
-    c->cur_start = -1;
-    if (rc != ASGD_OK) return rc;
-    CU(cudaEventRecord(c->ev_ring[k % kMaxInflight], c->s));
-    ++k;
+    if (launches >= inflight) CU(cudaEventSynchronize(c->ev_ring[(launches - inflight) % kMaxInflight]));
+    if (grp == 1) {
+      int64_t start = 0, len = 0;
+      const int r = next(&start, &len);
+      if (r < 0) return fail(-r, "scheduler failed");
+      if (r == 0) break;
+      c->cur_start = start;
+      const int rc = asgd_local_step(c, stream_rows + start, (int32_t)len, lr,
+                                     (losses && k < losses_cap) ? losses + k : nullptr);
+      c->cur_start = -1;
+      if (rc != ASGD_OK) return rc;
+      ++k;
+    } else {
+      int64_t st[kMaxGroup];
+      int64_t len = 0;
+      int g = 0;
+      if (pend_st >= 0) { st[g++] = pend_st; len = pend_len; pend_st = -1; }
+      while (g < grp) {
+        int64_t a = 0, l = 0;
+        const int r = next(&a, &l);
+        if (r < 0) return fail(-r, "scheduler failed");
+        if (r == 0) break;
+        if (g > 0 && l != len) { pend_st = a; pend_len = l; break; }
+        st[g++] = a;
+        len = l;
+      }
+      if (g == 0) break;
+      const asgd_model_desc& m = c->d;
+      if (len < 1 || len > m.b_max) return fail(ASGD_E_SHAPE, "n_rows=%lld not in [1, %d]", (long long)len, m.b_max);
+      if (!c->has_data) return fail(ASGD_E_STATE, "no data registered");
+      StepArgs sas[kMaxGroup];
+      for (int i = 0; i < g; ++i)
+        sas[i] = StepArgs{stream_rows + st[i], (losses && k + i < losses_cap) ? losses + k + i : nullptr, lr, (int)len};
+      const int rc = step_graph(c, (int)len, g, sas);
+      if (rc != ASGD_OK) return rc;
+      c->w2b_cur ^= (g & 1);
+      c->u += g;
+      k += g;
+    }
+    CU(cudaEventRecord(c->ev_ring[launches % kMaxInflight], c->s));
+    ++launches;
   }
   *n_steps = k;
   return ASGD_OK;
@@ -1414,8 +1498,9 @@ extern "C" {
 int asgd_run_tickets(asgd_ctx* c, asgd_sched* s, int32_t rank, int64_t b_i, const int32_t* stream_rows,
                      float lr, float* losses, int64_t losses_cap, int32_t inflight, int64_t* n_steps) {
   if (!c || !s || !stream_rows || !n_steps || b_i < 1) return fail(ASGD_E_ARG, "bad argument");
+  // one rank takes every ticket in order whatever the timing: its tickets may be grouped
   return run_steps(c, [&](int64_t* st, int64_t* ln) { return asgd_sched_next(s, rank, b_i, st, ln); }, stream_rows,
-                   lr, losses, losses_cap, inflight, n_steps);
+                   lr, losses, losses_cap, inflight, n_steps, s->h->n_ranks == 1);
 }
 
 int asgd_run_static(asgd_ctx* c, int32_t rank, int32_t world, int64_t b, const int32_t* stream_rows, int64_t M,
@@ -1430,7 +1515,7 @@ int asgd_run_static(asgd_ctx* c, int32_t rank, int32_t world, int64_t b, const i
                      cur += (int64_t)world * b;
                      return 1;
                    },
-                   stream_rows, lr, losses, losses_cap, inflight, n_steps);
+                   stream_rows, lr, losses, losses_cap, inflight, n_steps, true);   // static split: groupable
 }
 
 int asgd_sched_log(asgd_sched* s, int64_t* out, int64_t cap, int64_t* n_out) {
