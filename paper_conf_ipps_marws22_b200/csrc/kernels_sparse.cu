@@ -158,11 +158,14 @@ __device__ __forceinline__ int64_t entry_index(const int32_t* sboff, int n, int 
 // -------------------------------------------------------------------------
 constexpr int kViewPer = 8;   // rows per thread: n <= kViewPer * blockDim (b_max <= 2048, >= 256 threads)
 
+// build_view's label counts, then (defer) the label offsets; (defer) nnz, labels, error bits
+__shared__ int32_t s_llen[kViewPer * 256];
+__shared__ long long s_vtot[3];
+
 __device__ int build_view(const StepArgs& sa, const int64_t* __restrict__ row_ptr,
                           const int64_t* __restrict__ lab_ptr, int64_t n_data_rows, int64_t nz_cap,
-                          int64_t nl_cap, int32_t* sboff, bool publish, const ViewOut& out) {
+                          int64_t nl_cap, int32_t* sboff, bool publish, const ViewOut& out, bool defer = false) {
   __shared__ long long wf[32], wl[32];
-  __shared__ int32_t s_llen[kViewPer * 256];   // label counts (publish only)
   __shared__ int s_bad;
   const int n = sa.n;
   int64_t* srb = const_cast<int64_t*>(view_rbase(sboff, n));
@@ -183,8 +186,10 @@ __device__ int build_view(const StepArgs& sa, const int64_t* __restrict__ row_pt
       srb[r] = a;
       if (publish) {
         ll = (int32_t)(lab_ptr[id + 1] - lab_ptr[id]);
-        out.rowsc[r] = (int32_t)id;
-        out.rbase[r] = a;
+        if (!defer) {
+          out.rowsc[r] = (int32_t)id;
+          out.rbase[r] = a;
+        }
       }
     }
     sboff[r] = ln;
@@ -228,8 +233,12 @@ __device__ int build_view(const StepArgs& sa, const int64_t* __restrict__ row_pt
     if (r < n) {
       sboff[r] = (int32_t)min(pf, (long long)nz_cap);
       if (publish) {
-        out.boff[r] = (int32_t)min(pf, (long long)nz_cap);
-        out.loff[r] = (int32_t)min(pl, (long long)nl_cap);
+        if (defer) {
+          s_llen[r] = (int32_t)min(pl, (long long)nl_cap);   // this thread's own rows: read above
+        } else {
+          out.boff[r] = (int32_t)min(pf, (long long)nz_cap);
+          out.loff[r] = (int32_t)min(pl, (long long)nl_cap);
+        }
       }
       pf += len[i];
       pl += llen[i];
@@ -237,7 +246,16 @@ __device__ int build_view(const StepArgs& sa, const int64_t* __restrict__ row_pt
   }
   long long tf = wf[nw - 1], tl = wl[nw - 1];
   if (t == 0) sboff[n] = (int32_t)min(tf, (long long)nz_cap);
-  if (publish) {
+  if (publish && defer) {
+    if (t == 0) {
+      int err = bad ? ERR_ROW_ID : 0;
+      if (tf > nz_cap) err |= ERR_NNZ_CAP;
+      if (tl > nl_cap) err |= ERR_LAB_CAP;
+      s_vtot[0] = min(tf, (long long)nz_cap);
+      s_vtot[1] = min(tl, (long long)nl_cap);
+      s_vtot[2] = err;
+    }
+  } else if (publish) {
     if (bad && t == 0) atomicOr(&out.meta[M_ERR], ERR_ROW_ID);
     if (t == 0) {
       int err = 0;
@@ -255,6 +273,34 @@ __device__ int build_view(const StepArgs& sa, const int64_t* __restrict__ row_pt
   }
   __syncthreads();
   return (int)min(tf, (long long)nz_cap);
+}
+
+// The deferred publication of build_view(..., defer = true) (K-1's CTA 0, after its
+// griddepcontrol.wait: the previous step's kernels may still read the published view
+// while K-1 builds its own in shared memory).
+__device__ void publish_view(const StepArgs& sa, int64_t n_data_rows, const int32_t* sboff, const ViewOut& out) {
+  const int n = sa.n;
+  const int64_t* srb = view_rbase(sboff, n);
+  for (int r = threadIdx.x; r < n; r += blockDim.x) {
+    const int64_t id = sa.rows[r];
+    if (id >= 0 && id < n_data_rows) {
+      out.rowsc[r] = (int32_t)id;
+      out.rbase[r] = srb[r];
+    }
+    out.boff[r] = sboff[r];
+    out.loff[r] = s_llen[r];
+  }
+  if (threadIdx.x == 0) {
+    const int tf = (int)s_vtot[0], tl = (int)s_vtot[1], err = (int)s_vtot[2];
+    out.boff[n] = tf;
+    out.loff[n] = tl;
+    out.meta[M_NNZ] = tf;
+    out.meta[M_NLAB] = tl;
+    out.meta[M_NROWS] = n;
+    out.meta[M_LR] = __float_as_int(sa.lr);
+    *reinterpret_cast<float**>(out.meta + M_LOSS) = sa.loss;
+    if (err) atomicOr(&out.meta[M_ERR], err);
+  }
 }
 
 // -------------------------------------------------------------------------
@@ -509,14 +555,18 @@ __global__ void __launch_bounds__(32 * k1_warps<VPL, TMA>(), (k1_min_ctas<VPL, T
                                                   int ntiles) {
   Tl tl_(TL_SPMM);
   pdl_trigger();
-  pdl_wait();
-  tl_.ready();
   using IO = RowIO<VPL>;
   constexpr int H = 32 * VPL;
   constexpr int kU = VPL >= 16 ? 4 : 8;   // W1 rows in flight per warp
   extern __shared__ int32_t sboff[];
   const int n = sa.n;
-  const int nnz = build_view(sa, row_ptr, lab_ptr, n_data_rows, nz_cap, nl_cap, sboff, blockIdx.x == 0, vo);
+  // The batch view reads only the step's rows and the dataset, which no kernel writes: it is
+  // built before griddepcontrol.wait, so under programmatic dependent launch (a step group's
+  // graph) it overlaps the previous step's tail; CTA 0 publishes it after the wait.
+  const int nnz = build_view(sa, row_ptr, lab_ptr, n_data_rows, nz_cap, nl_cap, sboff, blockIdx.x == 0, vo, true);
+  pdl_wait();
+  tl_.ready();
+  if (blockIdx.x == 0) publish_view(sa, n_data_rows, sboff, vo);
   const int64_t* srb = view_rbase(sboff, n);
   const int lane = threadIdx.x & 31;
   const int npieces = (nnz + kPiece - 1) / kPiece;
