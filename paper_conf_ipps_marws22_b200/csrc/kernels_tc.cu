@@ -994,7 +994,10 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<BN, EPI>(), 1)
 constexpr int kBwdBN = 64, kBwdEpi = 8, kBwdStages = 3;
 constexpr uint32_t kBwdH1Bytes = 4u * 16384u, kBwdW2Bytes = 4u * 8192u, kBwdDzBytes = 16384u;
 
-__global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
+// EG epilogue groups of kBwdEpi warps: group g drains the label tiles i = g, g + EG, ... (its
+// own S buffer and dZ buffer when EG = 2), so two tiles' epilogues run at once.
+template <int EG>
+__global__ void __launch_bounds__(128 + 32 * kBwdEpi * EG, 1)
     k_bwd_dh(const __grid_constant__ CUtensorMap tmH1, const __grid_constant__ CUtensorMap tmW2,
              const __grid_constant__ CUtensorMap tmDZ, TcArgs g, int LR) {
   extern __shared__ uint8_t smem_raw[];
@@ -1002,8 +1005,8 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
   uint8_t* sH1 = smem;
   uint8_t* sW2 = sH1 + kBwdH1Bytes;
   uint8_t* sDZ = sW2 + kBwdStages * kBwdW2Bytes;
-  float* sBias = reinterpret_cast<float*>(sDZ + 2 * kBwdDzBytes);          // [kBwdEpi][32], then [128][3]
-  uint64_t* w2full = reinterpret_cast<uint64_t*>(sBias + kBwdEpi * 32 + 128 * 3);
+  float* sBias = reinterpret_cast<float*>(sDZ + 2 * kBwdDzBytes);          // [EG kBwdEpi][32], then [128][3]
+  uint64_t* w2full = reinterpret_cast<uint64_t*>(sBias + EG * kBwdEpi * 32 + 128 * 3);
   uint64_t* w2empty = w2full + kBwdStages;
   uint64_t* sfull = w2empty + kBwdStages;
   uint64_t* sempty = sfull + 2;
@@ -1120,7 +1123,9 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       mma_commit(dhfull);
     }
   } else if (warp >= 4) {   // -------------------------------------------- epilogue
-    const int q = (warp - 4) & 3, wh = (warp - 4) >> 2;
+    const int grp = (warp - 4) / kBwdEpi, ew = (warp - 4) % kBwdEpi;   // group, warp in group
+    const int q = ew & 3, wh = ew >> 2;
+    const bool lead = ew == 0 && lane == 0;   // the group's TMA-store thread
     const int m = m0 + q * 32 + lane;
     constexpr float kL2E = 1.4426950408889634f;
     float crow = 0.f, tinv = 0.f;
@@ -1179,7 +1184,7 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       }
       if (warp == 4 && lane == 0) TL_MARK(TL_PH1);
       // the two column halves (wh) of a row: wh = 1 hands its partial to wh = 0 via smem
-      float* xch = sBias + kBwdEpi * 32;   // [128][3] after the bias rows
+      float* xch = sBias + EG * kBwdEpi * 32;   // [128][3] after the bias rows (EG = 1 here)
       const int rl = q * 32 + lane;
       if (wh == 1) { xch[3 * rl] = mx; xch[3 * rl + 1] = se; xch[3 * rl + 2] = zs; }
       asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
@@ -1253,6 +1258,7 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       }
     }
     float* bias_w = sBias + (warp - 4) * 32;
+    const uint32_t gbar = 1 + grp;   // the group's named barrier
     if (warp == 4 && lane == 0 && g.one_pass) TL_MARK(TL_PH3);
     // b2 of the next tile's columns, loaded one tile ahead (its latency hides under this
     // tile's epilogue instead of heading it: the top stall site in ncu before)
@@ -1260,15 +1266,15 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       const int cc = (t0 + i) * kBwdBN + wh * 32 + lane;
       return (i < nt && cc < g.N) ? __ldg(g.bias + cc) * kL2E : 0.f;
     };
-    float bnext = b2_of(0);
+    float bnext = b2_of(grp);
     const int base = (g.one_pass && nt > 2) ? nt : 0;   // S-buffer uses of the statistics sweep
-    for (int i = 0; i < nt; ++i) {
+    for (int i = grp; i < nt; i += EG) {
       const int acc = (base + i) & 1, buf = i & 1;
       const int c = (t0 + i) * kBwdBN + wh * 32;        // this warp's first label column
       __syncwarp();
       bias_w[lane] = bnext;
       __syncwarp();
-      bnext = b2_of(i + 1);
+      bnext = b2_of(i + EG);
       while (nxt < c) {
         ++lab_cur;
         nxt = lab_cur < lab_end ? g.lab[lab_cur] : 0x7fffffff;
@@ -1305,8 +1311,8 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       // the dZ buffer: MMA 2 of tile i - 2 done, and (write_z) its TMA store done reading
       mbar_wait(&dzempty[buf], ((i >> 1) & 1) ^ 1);
       if (g.write_z) {
-        if (warp == 4 && lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
-        asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
+        if (lead) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+        asm volatile("bar.sync %0, %1;" ::"r"(gbar), "r"(32 * kBwdEpi) : "memory");
       }
       uint8_t* rowp = sDZ + buf * kBwdDzBytes + (q * 32 + lane) * 128;
       const int sw = (q * 32 + lane) & 7;
@@ -1323,8 +1329,8 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       if (g.write_z) {
-        asm volatile("bar.sync 1, %0;" ::"r"(32 * kBwdEpi) : "memory");
-        if (warp == 4 && lane == 0) {
+        asm volatile("bar.sync %0, %1;" ::"r"(gbar), "r"(32 * kBwdEpi) : "memory");
+        if (lead) {
           asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
                            reinterpret_cast<uint64_t>(&tmDZ)), "r"(smem_u32(sDZ + buf * kBwdDzBytes)),
                        "r"((t0 + i) * kBwdBN), "r"(m0)
@@ -1344,7 +1350,7 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
       tc_fence_after();
     }
 #pragma unroll 1
-    for (int ch = 0; ch < (g.dz_only ? 0 : 4); ++ch) {
+    for (int ch = grp * (4 / EG); ch < (g.dz_only ? 0 : (grp + 1) * (4 / EG)); ++ch) {
       float v[32];
       if (nt > 0) {
         tmem_ld32(tmem + 256 + (uint32_t)(wh * 128 + ch * 32) + ((uint32_t)(q * 32) << 16), v);
@@ -1359,7 +1365,7 @@ __global__ void __launch_bounds__(128 + 32 * kBwdEpi, 1)
               make_float4(v[4 * qq], v[4 * qq + 1], v[4 * qq + 2], v[4 * qq + 3]);
       }
     }
-    if (warp == 4 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    if (lead) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
   tc_fence_before();
   __syncthreads();
@@ -1940,10 +1946,20 @@ cudaError_t launch_bwd_dh(const Launch& lc, int n, int64_t L, int H, const Ptrs&
     g.gbar = reinterpret_cast<unsigned long long*>(P.meta + M_KBAR);
     g.dz_only = dz_only ? 1 : 0;
   }
-  const size_t smem = kBwdH1Bytes + kBwdStages * kBwdW2Bytes + 2 * kBwdDzBytes + kBwdEpi * 32 * 4 + 128 * 3 * 4 +
-                      1024 + 256;
-  if ((e = ensure_smem(k_bwd_dh, smem)) != cudaSuccess) return e;
-  return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_bwd_dh, dim3(MT * LR), dim3(128 + 32 * kBwdEpi), smem, th,
+  // two epilogue groups (two label tiles drained at once) unless a one-pass mode needs the
+  // single-group statistics exchange; ASGD_K3_EG=1 keeps one group.  Measured: Amazon-670K
+  // 0.467 -> 0.490 M samples/s, AmazonCat-13K even (5.48 / 5.46 M)
+  static const int eg_env = [] { const char* v = getenv("ASGD_K3_EG"); return v ? atoi(v) : 2; }();
+  const int eg = (one_pass || eg_env == 1) ? 1 : 2;
+  const size_t smem = kBwdH1Bytes + kBwdStages * kBwdW2Bytes + 2 * kBwdDzBytes + eg * kBwdEpi * 32 * 4 +
+                      128 * 3 * 4 + 1024 + 256;
+  if (eg == 2) {
+    if ((e = ensure_smem(k_bwd_dh<2>, smem)) != cudaSuccess) return e;
+    return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_bwd_dh<2>, dim3(MT * LR), dim3(128 + 32 * kBwdEpi * 2),
+                        smem, th, tw, tz, g, LR);
+  }
+  if ((e = ensure_smem(k_bwd_dh<1>, smem)) != cudaSuccess) return e;
+  return launch_k_pdl(lc, lc.pdl || pdl_mode() == 2, k_bwd_dh<1>, dim3(MT * LR), dim3(128 + 32 * kBwdEpi), smem, th,
                       tw, tz, g, LR);
 }
 
