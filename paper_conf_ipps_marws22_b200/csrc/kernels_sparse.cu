@@ -376,6 +376,7 @@ __global__ void __launch_bounds__(NT) k_touched(StepArgs sa, const int64_t* __re
     }
     __syncthreads();
     nnz = sboff[n];
+    if (threadIdx.x == 0) TL_MARK(TL_PH0);   // K-0 (fold): view copied
     // ---- C0: this step's tile sums (count, touched features) from the counts K-1 left.
     // Few tiles (F <= kK0OneCta tiles, EURLex-4K: 5): CTA 0 runs C0 and C alone, the other
     // CTAs go straight to the barrier before E (one grid barrier instead of two)
@@ -400,6 +401,7 @@ __global__ void __launch_bounds__(NT) k_touched(StepArgs sa, const int64_t* __re
       __syncthreads();
     }
     if (!one) grid_barrier(bar);
+    if (threadIdx.x == 0) TL_MARK(TL_PH1);   // K-0 (fold): C0 done, barrier 1 passed
   } else {
     for (int i = threadIdx.x; i < 2 * ntiles; i += blockDim.x) hist[i] = 0;
     nnz = build_view(sa, row_ptr, nullptr, n_data_rows, nz_cap, 0, sboff, false, ViewOut{});
@@ -474,7 +476,9 @@ __global__ void __launch_bounds__(NT) k_touched(StepArgs sa, const int64_t* __re
     }
     __syncthreads();
   }
+  if (threadIdx.x == 0) TL_MARK(TL_PH2);   // K-0: C done
   grid_barrier(bar);
+  if (threadIdx.x == 0) TL_MARK(TL_PH3);   // K-0: C done, barrier 2 passed
   // ---- E: placement, kE entries per thread at a time (their dependent loads overlap)
   constexpr int kE = 4;
   for (int e0 = gt; e0 < nnz; e0 += kE * gs) {
@@ -495,8 +499,17 @@ __global__ void __launch_bounds__(NT) k_touched(StepArgs sa, const int64_t* __re
       uid[i] = 0;
       if (k[i] >= 0) {
         const uint32_t* bw = bits + (int64_t)f[i] * W;
-        rank[i] = __popc(bw[r[i] >> 5] & ((1u << (r[i] & 31)) - 1u));
-        for (int w = 0; w < (r[i] >> 5); ++w) rank[i] += __popc(bw[w]);
+        const int wr = r[i] >> 5;
+        rank[i] = __popc(bw[wr] & ((1u << (r[i] & 31)) - 1u));
+        // the bitmap words below row r's word: loaded 8 at a time (independent loads in
+        // flight together, one round for b_max <= 256) instead of one after another
+        for (int w0 = 0; w0 < wr; w0 += 8) {
+          uint32_t wv[8];
+#pragma unroll
+          for (int w = 0; w < 8; ++w) wv[w] = w0 + w < wr ? bw[w0 + w] : 0u;
+#pragma unroll
+          for (int w = 0; w < 8; ++w) rank[i] += __popc(wv[w]);
+        }
         seg[i] = fseg[f[i]];
         uid[i] = fuid[f[i]];
       }
