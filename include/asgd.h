@@ -137,6 +137,19 @@ int asgd_data_register(asgd_ctx* ctx, const asgd_csr* dev_csr);
  * Asynchronous. */
 int asgd_data_upload(asgd_ctx* ctx, const asgd_csr* host_src, const asgd_csr* dev_dst);
 
+/* asgd_data_upload in two halves, so that the next split's H2D copies overlap the current
+ * split's local steps (the e2e path with two device staging buffers):
+ *   asgd_data_stage: the copies host_src -> dev_dst (same sizes as asgd_data_upload) on
+ *     `stream` (cudaStream_t, NULL = the ctx stream); nothing is registered.  The caller
+ *     must not stage into a buffer that enqueued steps may still read.
+ *   asgd_data_use: registers dev (its nnz / n_lab = the staged split's counts; no
+ *     re-validation) for the steps enqueued after it; the ctx stream first waits for the
+ *     copies last staged into that buffer.  Step graphs are cached per dataset (pointers
+ *     and row count), so alternating buffers are not re-captured.
+ * Both asynchronous; asgd_data_upload = stage on the ctx stream + use. */
+int asgd_data_stage(asgd_ctx* ctx, const asgd_csr* host_src, const asgd_csr* dev_dst, void* stream);
+int asgd_data_use(asgd_ctx* ctx, const asgd_csr* dev);
+
 /* One local minibatch SGD step on the replica (A1; rows a2-a8 of
  * DESIGN.md §Path): rows_dev: int32[n_rows] device, sample ids of the batch
  * (a slice of the pass permutation, Q31), 1 <= n_rows <= b_max; lr: this

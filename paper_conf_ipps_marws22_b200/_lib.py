@@ -49,6 +49,8 @@ _SIGS = {
     "asgd_params_changed": (C.c_int, [_P]),
     "asgd_data_register": (C.c_int, [_P, C.POINTER(Csr)]),
     "asgd_data_upload": (C.c_int, [_P, C.POINTER(Csr), C.POINTER(Csr)]),
+    "asgd_data_stage": (C.c_int, [_P, C.POINTER(Csr), C.POINTER(Csr), _P]),
+    "asgd_data_use": (C.c_int, [_P, C.POINTER(Csr)]),
     "asgd_local_step": (C.c_int, [_P, _P, _i32, _f32, _P]),
     "asgd_updates": (C.c_int, [_P, C.POINTER(_i64)]),
     "asgd_set_debug_grads": (C.c_int, [_P, _P]),

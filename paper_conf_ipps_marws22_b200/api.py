@@ -122,6 +122,18 @@ class Replica:
         self._hcsr, self._csr = host.csr(), dev.csr()
         call("asgd_data_upload", self.ctx, C.byref(self._hcsr), C.byref(self._csr))
 
+    def stage(self, host: DeviceCsr, dev: DeviceCsr, stream: Optional[torch.cuda.Stream] = None):
+        """asgd_data_stage: host -> dev copies on `stream` (None: the ctx stream), not registered."""
+        h, d = host.csr(), dev.csr()
+        call("asgd_data_stage", self.ctx, C.byref(h), C.byref(d), stream.cuda_stream if stream is not None else None)
+
+    def use(self, dev: DeviceCsr, nnz: int, n_lab: int):
+        """asgd_data_use: register a staged buffer (the staged split's nnz / n_lab) for the next steps."""
+        self._data = dev
+        self._csr = dev.csr()
+        self._csr.nnz, self._csr.n_lab = int(nnz), int(n_lab)
+        call("asgd_data_use", self.ctx, C.byref(self._csr))
+
     # -- local step
     def step(self, rows: torch.Tensor, lr: float, loss_out: Optional[torch.Tensor] = None):
         assert rows.dtype == torch.int32 and rows.is_cuda

@@ -233,6 +233,7 @@ Ptrs ws_ptrs(char* b, const WsLayout& L) {
 // with the step's row ids, lr and loss pointer and publishes them to the rest).
 struct StepGraph {
   int n = 0, cur = 0, steps = 1;      // steps: local steps captured back to back (step groups)
+  asgd_csr data{};                    // the dataset its kernels were captured with
   uint32_t mask = 0;
   int seen = 0;                       // captured on the 2nd step with this key
   cudaGraph_t graph = nullptr;
@@ -291,6 +292,7 @@ struct asgd_ctx {
   std::vector<std::pair<cudaEvent_t, int>> cap_ph;   // (placeholder, cls * 2 + begin) during capture
   std::vector<std::pair<cudaGraphNode_t, int>> cap_args;   // K-0 (0) / K-1 (1) nodes, capture order
   cudaEvent_t prof_sink = nullptr;                // target of profiling nodes past kMaxProfPairs
+  std::vector<std::pair<const int64_t*, cudaEvent_t>> staged;   // asgd_data_stage: per buffer, its copies
   cudaEvent_t ev_ring[8] = {};                    // asgd_run_tickets: completion of the last steps
   StepArgs sa{};                                  // current step's arguments (K-0 / K-1 parameter)
   // fused peer-memory merge (asgd_peer_open / asgd_merge_fused)
@@ -531,20 +533,46 @@ int asgd_data_register(asgd_ctx* c, const asgd_csr* x) {
 }
 
 int asgd_data_upload(asgd_ctx* c, const asgd_csr* h, const asgd_csr* dv) {
+  const int rc = asgd_data_stage(c, h, dv, nullptr);
+  if (rc != ASGD_OK) return rc;
+  asgd_csr d = *dv;
+  d.nnz = h->nnz;
+  d.n_lab = h->n_lab;
+  return asgd_data_use(c, &d);
+}
+
+int asgd_data_stage(asgd_ctx* c, const asgd_csr* h, const asgd_csr* dv, void* stream) {
   if (!c || !h || !dv) return fail(ASGD_E_ARG, "null argument");
   if (h->n_rows != dv->n_rows || h->nnz > dv->nnz || h->n_lab > dv->n_lab)
     return fail(ASGD_E_SHAPE, "destination too small");
-  CU(cudaMemcpyAsync((void*)dv->row_ptr, h->row_ptr, (h->n_rows + 1) * 8, cudaMemcpyHostToDevice, c->s));
-  CU(cudaMemcpyAsync((void*)dv->col, h->col, h->nnz * 4, cudaMemcpyHostToDevice, c->s));
-  CU(cudaMemcpyAsync((void*)dv->val, h->val, h->nnz * 4, cudaMemcpyHostToDevice, c->s));
-  CU(cudaMemcpyAsync((void*)dv->lab_ptr, h->lab_ptr, (h->n_rows + 1) * 8, cudaMemcpyHostToDevice, c->s));
-  CU(cudaMemcpyAsync((void*)dv->lab, h->lab, h->n_lab * 4, cudaMemcpyHostToDevice, c->s));
-  if (!c->has_data || c->data.row_ptr != dv->row_ptr || c->data.col != dv->col || c->data.val != dv->val ||
-      c->data.lab_ptr != dv->lab_ptr || c->data.lab != dv->lab || c->data.n_rows != dv->n_rows)
-    clear_graphs(c);   // graphs hold the dataset pointers and row count
+  cudaStream_t st = stream ? static_cast<cudaStream_t>(stream) : c->s;
+  CU(cudaMemcpyAsync((void*)dv->row_ptr, h->row_ptr, (h->n_rows + 1) * 8, cudaMemcpyHostToDevice, st));
+  CU(cudaMemcpyAsync((void*)dv->col, h->col, h->nnz * 4, cudaMemcpyHostToDevice, st));
+  CU(cudaMemcpyAsync((void*)dv->val, h->val, h->nnz * 4, cudaMemcpyHostToDevice, st));
+  CU(cudaMemcpyAsync((void*)dv->lab_ptr, h->lab_ptr, (h->n_rows + 1) * 8, cudaMemcpyHostToDevice, st));
+  CU(cudaMemcpyAsync((void*)dv->lab, h->lab, h->n_lab * 4, cudaMemcpyHostToDevice, st));
+  if (st != c->s) {   // asgd_data_use of this buffer makes the ctx stream wait for these copies
+    cudaEvent_t ev = nullptr;
+    for (auto& se : c->staged)
+      if (se.first == dv->row_ptr) ev = se.second;
+    if (!ev) {
+      CU(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+      c->staged.push_back({dv->row_ptr, ev});
+    }
+    CU(cudaEventRecord(ev, st));
+  }
+  return ASGD_OK;
+}
+
+int asgd_data_use(asgd_ctx* c, const asgd_csr* dv) {
+  if (!c || !dv || !dv->row_ptr || !dv->col || !dv->val || !dv->lab_ptr || !dv->lab)
+    return fail(ASGD_E_ARG, "null argument");
+  if (dv->n_rows <= 0 || dv->nnz < 0 || dv->n_lab <= 0) return fail(ASGD_E_SHAPE, "empty split");
+  for (auto& se : c->staged)
+    if (se.first == dv->row_ptr) CU(cudaStreamWaitEvent(c->s, se.second, 0));
+  // the step graphs are keyed by the dataset (pointers and row count): alternating staging
+  // buffers keep both sets of graphs
   c->data = *dv;
-  c->data.nnz = h->nnz;
-  c->data.n_lab = h->n_lab;
   c->has_data = true;
   return ASGD_OK;
 }
@@ -741,13 +769,22 @@ int enqueue_step(asgd_ctx* c, int n) {
 
 constexpr size_t kMaxGraphs = 16;
 
+// the dataset fields a captured step bakes into its kernel parameters
+bool same_data(const asgd_csr& a, const asgd_csr& b) {
+  return a.row_ptr == b.row_ptr && a.col == b.col && a.val == b.val && a.lab_ptr == b.lab_ptr && a.lab == b.lab &&
+         a.n_rows == b.n_rows;
+}
+
 // Replay (capturing on the 2nd use of a key) `steps` local steps as one CUDA graph
 // (steps > 1: a step group, run_steps at N = 1); sas[i] = step i's StepArgs.  c->w2b_cur
 // is left as it was (the caller flips it per step).
 int step_graph(asgd_ctx* c, int n, int steps, const StepArgs* sas) {
   StepGraph* hit = nullptr;
   for (auto& gr : c->graphs)
-    if (gr.n == n && gr.steps == steps && gr.cur == c->w2b_cur && gr.mask == c->prof_mask) { hit = &gr; break; }
+    if (gr.n == n && gr.steps == steps && gr.cur == c->w2b_cur && gr.mask == c->prof_mask && same_data(gr.data, c->data)) {
+      hit = &gr;
+      break;
+    }
   if (!hit) {
     if (c->graphs.size() >= kMaxGraphs) {
       auto lru = std::min_element(c->graphs.begin(), c->graphs.end(),
@@ -757,7 +794,7 @@ int step_graph(asgd_ctx* c, int n, int steps, const StepArgs* sas) {
     }
     c->graphs.emplace_back();
     hit = &c->graphs.back();
-    hit->n = n; hit->steps = steps; hit->cur = c->w2b_cur; hit->mask = c->prof_mask;
+    hit->n = n; hit->steps = steps; hit->cur = c->w2b_cur; hit->mask = c->prof_mask; hit->data = c->data;
   }
   StepGraph& G = *hit;
   G.last_use = ++c->graph_clock;
