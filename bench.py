@@ -332,7 +332,7 @@ def main():
     wcnt = np.zeros(NCLS, dtype=np.int64)
     call("asgd_profile_read", rep.ctx, wms.ctypes.data, wcnt.ctypes.data)
     # dominant kernel: the largest per-step time among the kernels on the step's critical
-    # path.  K-0 (`touched`) runs on side stream s2 beside K-1..G2 and is joined only
+    # path.  K-0 (`touched`) runs on side stream s2 after K-1 (its phase A folded into K-1), beside G1..G2, joined only
     # before K-5, so its duration does not bound the step; it is reported under
     # `side_stream` with its own roofline.
     crit = [i for i in range(NCLS) if _lib.PROF_NAMES[i] != "touched" and wcnt[i]]
@@ -430,7 +430,7 @@ def main():
                 rs = roofline_of("touched", cfg, bf16, wl, a.loss, s_avg, peaks)
                 side["touched"] = {"us_per_launch": round(s_avg * 1e6, 3), "bound": rs["bound"],
                                    "frac": round(rs["achieved"] / rs["peak"], 4),
-                                   "note": "side stream s2, overlapped with K-1..G2 (warm-up profile)"}
+                                   "note": "side stream s2 after K-1 (phase A folded into K-1), overlapped with G1..G2 (warm-up profile)"}
         # whole-job roofline: sum of per-step ideal times with
         # each step's measured B, nnz, U, + merge 36 P bytes / HBM peak, over the timed time
         tc_peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"]) / (1.0 if bf16 else 3.0)
