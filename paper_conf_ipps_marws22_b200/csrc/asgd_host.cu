@@ -489,6 +489,7 @@ int asgd_replica_destroy(asgd_ctx* c) {
       for (cudaEvent_t e : v) cudaEventDestroy(e);
     for (cudaEvent_t ev : {c->ev_fork, c->ev_join, c->ev_sm, c->ev_dh, c->ev_a})
       if (ev) cudaEventDestroy(ev);
+    for (auto& se : c->staged) cudaEventDestroy(se.second);
     if (c->s2) cudaStreamDestroy(c->s2);
     if (c->s3) cudaStreamDestroy(c->s3);
     if (c->sc) cudaStreamDestroy(c->sc);
