@@ -625,11 +625,15 @@ int enqueue_step(asgd_ctx* c, int n) {
   // K-1
   PCU(ASGD_K_SPMM, launch_spmm_fwd(lc, c->sa, x, W1, b1, H, P, c->L, true, k0_fold(), (int)m.b_max));   // H1 fp32 + bf16 (+ lo)
   if (c->capturing) { const int rc = record_cap_node(c, c->s, 1); if (rc != ASGD_OK) return rc; }
-  // ASGD_K0_AFTER=1 (with the fold): K-0 forks after the loss stage (G1 + softmax, or K-3's
-  // softmax-only kernel), beside G2 / the dH reduce instead of beside G1.  Measured: EURLex
-  // 58.5 -> 57.2 us per step, but AmazonCat 181.9 -> 204.9 and Wiki10 179.2 -> 193.6 (K-0
-  // then ends after the dH reduce and holds up K-5), so it is off by default
-  static const bool k0_after = [] { const char* e = getenv("ASGD_K0_AFTER"); return e && e[0] == '1'; }() && k0_fold();
+  // With the fold, K-0 forks after the loss stage (G1 + softmax, or K-3's softmax-only
+  // kernel), beside G2 / the dH reduce instead of beside G1, on the bf16 path when the
+  // feature space has at most 8 scan tiles (F <= 8192: K-0's scan is short and it ends
+  // inside the G2 / dH window).  Measured: EURLex bf16 4.54 -> 4.64 M samples/s; EURLex fp32
+  // 3.99 -> 3.68 M, AmazonCat 181.9 -> 204.9 and Wiki10 179.2 -> 193.6 us per step (K-0 then
+  // ends after the dH reduce and holds up K-5).  ASGD_K0_AFTER=0 / 1 forces it.
+  static const int k0_after_env = [] { const char* e = getenv("ASGD_K0_AFTER"); return e ? (e[0] == '1' ? 1 : 0) : -1; }();
+  const bool k0_after = k0_fold() && (k0_after_env >= 0 ? k0_after_env == 1
+                                                         : (bf && m.F <= 8 * (int64_t)kScanTile));
   if (k0_late && !k0_after) { const int rc = fork_k0(); if (rc != ASGD_OK) return rc; }
   {
     // A DAG over three streams (both precisions; the fp32 path's GEMMs take bf16x3
